@@ -1,0 +1,244 @@
+/*
+ * mucudnn.h -- C ABI of the B200-native micro-batched convolution library
+ * (the hot path of mu-cuDNN: Oyama, Ben-Nun, Hoefler, Matsuoka, IEEE CLUSTER
+ * 2018; text in /root/reference/PAPER.md, cited as P:Lnn = line nn).
+ *
+ * What the library does (north_star of BASELINE.json):
+ *   A convolution layer's mini-batch of N samples is split into micro-batches
+ *   (Sec. II/III, Fig. 3).  Each micro-batch is executed with
+ *   one of three equivalent sm_100a convolution algorithms that trade
+ *   workspace for speed: implicit GEMM (zero workspace), explicit
+ *   im2col + GEMM, Winograd F(2x2,3x3).  A benchmark pass times every
+ *   (algorithm, micro-batch size) pair (WR step 1); a dynamic program
+ *   picks the partition of N and per-part algorithm minimising the total time
+ *   within a per-layer workspace limit (WR policy, Sec. III-B); a
+ *   set-valued DP + Pareto pruning + exact multiple-choice-knapsack solve the
+ *   whole-network shared-workspace problem (WD policy, Sec. III-C,
+ *   ILP Eq. (1)-(4)).  Plans are executed on the caller's CUDA stream and
+ *   workspace.
+ *
+ * Conventions (all functions):
+ *   - Every function returns mucu_status_t; none throws, aborts or prints.
+ *     On error, mucu_last_error() returns a thread-local detail string.
+ *   - Tensors: activations NHWC (x: [N,H,W,C], y/dy: [N,P,Q,K], dx: [N,H,W,C]),
+ *     filters KRSC (w: [K,R,S,C]), all densely packed.  Element type by math
+ *     mode: MUCU_MATH_F32 / MUCU_MATH_TF32 -> float32; MUCU_MATH_BF16 ->
+ *     bfloat16.  The filter gradient dw is ALWAYS float32 [K,R,S,C].
+ *     P = (H + 2 pad - R)/stride + 1, Q likewise (reading G1/G3).
+ *   - Device memory (tensors, workspace, benchmark scratch) is owned by the
+ *     caller (PyTorch allocator).  Host objects (handle, network) are created
+ *     and destroyed by the library.  The handle additionally owns one small
+ *     device buffer (split-K ordering semaphores, 256 KiB) allocated in
+ *     mucu_create.
+ *   - GPU work is asynchronous on the caller's `cuda_stream` (a cudaStream_t
+ *     passed as void*; NULL = legacy default stream), except
+ *     mucu_benchmark / mucu_plan_layer / mucu_network_plan which synchronise
+ *     that stream before returning.
+ *   - Pure host functions (marked "host") never touch the GPU and are
+ *     reentrant.  A handle is not thread-safe; use one per host thread.
+ */
+#ifndef MUCUDNN_H_
+#define MUCUDNN_H_
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define MUCU_VERSION 100 /* 1.0.0 */
+
+typedef enum {
+    MUCU_OK = 0,
+    MUCU_ERR_INVALID_VALUE = 1,          /* bad dims, null pointer, plan parts not summing to N */
+    MUCU_ERR_UNSUPPORTED = 2,            /* algorithm ineligible for this layer/type (e.g. WG on 5x5) */
+    MUCU_ERR_INSUFFICIENT_WORKSPACE = 3, /* ws_bytes below what the plan needs / nothing fits the limit */
+    MUCU_ERR_INFEASIBLE = 4,             /* WD budget below the sum of minimal workspaces */
+    MUCU_ERR_CAPACITY = 5,               /* caller array too small; *count holds the needed size */
+    MUCU_ERR_MISALIGNED = 6,             /* device pointer not 16-byte aligned */
+    MUCU_ERR_CUDA = 7,                   /* CUDA runtime/driver error (message in mucu_last_error) */
+    MUCU_ERR_INTERNAL = 8
+} mucu_status_t;
+
+/* The three convolution operations of cuDNN. */
+typedef enum { MUCU_FWD = 0, MUCU_BWD_DATA = 1, MUCU_BWD_FILTER = 2 } mucu_conv_type_t;
+
+/* Algorithms; the enum order is the tie-break order (reading G11). */
+typedef enum {
+    MUCU_ALGO_IMPLICIT_GEMM = 0,     /* (a) zero workspace                                   */
+    MUCU_ALGO_IM2COL_GEMM = 1,       /* (b) explicit im2col (+col2im for DGRAD) + GEMM        */
+    MUCU_ALGO_WINOGRAD_2X2_3X3 = 2,  /* (c) Winograd F(2x2,3x3), Lavin & Gray (ref [23])      */
+    MUCU_NUM_ALGOS = 3
+} mucu_algo_t;
+
+/* Arithmetic: F32 = fp32 SIMT FFMA; TF32 = fp32 storage, tcgen05 kind::tf32;
+ * BF16 = bf16 storage, tcgen05 kind::f16 (bf16 x bf16 -> fp32 in TMEM). */
+typedef enum { MUCU_MATH_F32 = 0, MUCU_MATH_TF32 = 1, MUCU_MATH_BF16 = 2 } mucu_math_t;
+
+/* Batch-size policies of P:L149-155: which micro-batch sizes b are benchmarked.
+ * ALL: b = 1..N.  POW2: {2^k <= N} U {N} (reading G20).  UNDIVIDED: {N}. */
+typedef enum { MUCU_POLICY_ALL = 0, MUCU_POLICY_POW2 = 1, MUCU_POLICY_UNDIVIDED = 2 } mucu_policy_t;
+
+/* Layer descriptor (north_star: N,C,H,W,K,R,S,pad,stride; dilation 1, groups 1). */
+typedef struct {
+    int32_t n, c, h, w, k, r, s, pad, stride;
+    int32_t math; /* mucu_math_t */
+} mucu_conv_desc_t;
+
+/* Micro-configuration: an (algorithm, micro-batch size) pair.  A
+ * configuration / plan is an array of these; its micro_n sum to desc.n and it
+ * is executed in array order (reading G8: non-increasing micro_n). */
+typedef struct {
+    int32_t algo;
+    int32_t micro_n;
+} mucu_micro_config_t;
+
+typedef struct mucu_handle* mucu_handle_t;   /* library-owned, one per device */
+typedef struct mucu_network* mucu_network_t; /* library-owned WD kernel list */
+
+/* ---------------------------------------------------------------- misc ---- */
+const char* mucu_status_string(mucu_status_t status);   /* host; static string */
+const char* mucu_last_error(void);                      /* host; thread-local detail */
+int32_t mucu_version(void);                             /* host */
+
+/* Create a handle bound to CUDA device `device` (makes it current on the
+ * calling thread).  Reads env MUCU_BATCH_POLICY={all,pow2,undivided} (default
+ * pow2), MUCU_BENCH_WARMUP (default 2), MUCU_BENCH_REPS (default 5). */
+mucu_status_t mucu_create(mucu_handle_t* handle, int device);
+mucu_status_t mucu_destroy(mucu_handle_t handle);
+/* the batch-size policy "can be specified via an environment variable
+ * or through a special library function" -- this is the function. */
+mucu_status_t mucu_set_policy(mucu_handle_t handle, mucu_policy_t policy);
+mucu_status_t mucu_set_bench_params(mucu_handle_t handle, int32_t warmup, int32_t reps);
+
+/* ------------------------------------------------------ host: geometry ---- */
+/* P and Q of the output (host).  INVALID_VALUE if any dim <= 0 or P,Q <= 0. */
+mucu_status_t mucu_output_dims(const mucu_conv_desc_t* desc, int32_t* p, int32_t* q);
+
+/* Exact workspace bytes of one micro-configuration (host; "within the
+ * workspace constraint").  Closed forms (elt = 4 for F32/TF32, 2 for BF16,
+ * every segment rounded up to 256 B):
+ *   IG  (all types):  0
+ *   I2C FWD/WGRAD:    b*P*Q*ceil_e(R*S*C)*elt  (+ K*ceil_e(R*S*C)*elt when R*S*C*elt % 16 != 0)
+ *                     0 for 1x1, stride 1, pad 0 (the im2col matrix is x itself)
+ *   I2C DGRAD:        b*P*Q*ceil_4(R*S*C)*4 (fp32 dcol)  (+ filter copy as above); 0 for 1x1/s1/p0
+ *   WG  FWD:          16*K*C*elt + 16*b*T*C*elt + 16*b*T*K*4,   T = ceil(P/2)*ceil(Q/2)
+ *   WG  DGRAD:        16*C*K*elt + 16*b*T'*K*elt + 16*b*T'*C*4, T' = ceil(H/2)*ceil(W/2)
+ * ceil_e rounds up to a multiple of 16/elt elements.  UNSUPPORTED if the
+ * algorithm is ineligible (WG needs R=S=3, stride 1, pad <= 2, and is not
+ * implemented for BWD_FILTER). */
+mucu_status_t mucu_workspace_size(const mucu_conv_desc_t* desc, mucu_conv_type_t type,
+                                  mucu_algo_t algo, int32_t micro_n, uint64_t* bytes);
+
+/* ---------------------------------------------------- host: optimisers ---- */
+/* Timing tables (P:L88 step 1): time_ns and ws are row-major
+ * [MUCU_NUM_ALGOS][n+1]; entry [a][b] is the time (ns, int64) and workspace
+ * (bytes) of algorithm a at micro-batch b; time < 0 = not benchmarked /
+ * ineligible; column b = 0 is ignored. */
+
+/* WR dynamic program (Sec. III-B):
+ *   T(b) = min( T_mu(b), min_{1<=b'<b} T_mu(b') + T(b-b') ),  T(0) = 0,
+ * T_mu(b) = fastest present entry with ws <= ws_limit (ties: smaller ws, then
+ * smaller algo id; reading G11).  Canonical tie-break among optimal plans
+ * (reading G8): fewer micro-batches, then parts sorted non-increasing and
+ * compared lexicographically larger-first.  Output: *count micro-configs in
+ * out[0..cap) in non-increasing micro_n, *total_ns = T(n).
+ * Errors: INSUFFICIENT_WORKSPACE if no plan fits; CAPACITY if cap < count. */
+mucu_status_t mucu_plan_wr(int32_t n, const int64_t* time_ns, const uint64_t* ws, uint64_t ws_limit,
+                           mucu_micro_config_t* out, int32_t cap, int32_t* count, int64_t* total_ns);
+
+/* WD desirable set of one kernel (Sec. III-C1): the set-valued DP
+ *   C(b) = D( U_{1<=b'<=b} { [c] (+) C' : c in C_mu(b'), C' in C(b-b') } ),  C(0) = {[]}
+ * with T = sum of times, M = max of workspaces (reading G13) and D the Pareto
+ * filter "keep C iff no other configuration is at least as fast with no more
+ * workspace" (reading G15).  Only micro-configs with ws <= ws_cap take part.
+ * Output sorted by M ascending (T strictly decreasing): front_t[i], front_m[i],
+ * and one plan per point in plans[i*n .. i*n + plan_len[i]) (valid, not
+ * necessarily unique among equal-cost plans).  CAPACITY if cap < *front_len. */
+mucu_status_t mucu_pareto_front(int32_t n, const int64_t* time_ns, const uint64_t* ws, uint64_t ws_cap,
+                                int64_t* front_t, uint64_t* front_m, int32_t cap, int32_t* front_len,
+                                mucu_micro_config_t* plans, int32_t* plan_len);
+
+/* WD 0-1 ILP (Eq. (1)-(4)) as an exact multiple-choice knapsack:
+ *   min sum_k t_k(c_k)  s.t.  sum_k align256(m_k(c_k)) <= total_limit, one c per kernel.
+ * Options of kernel k are t[off_k .. off_k+front_len[k]), m[...] with off_k the
+ * prefix sum of front_len.  Ties: smaller sum of aligned m, then the
+ * lexicographically smallest choice vector (reading G17).  Output choice[k],
+ * offset[k] (byte offset of kernel k's segment = running sum of aligned m in
+ * kernel order, reading G18), *total_ns.  INFEASIBLE if even the smallest
+ * options exceed total_limit. */
+mucu_status_t mucu_solve_wd(int32_t num_kernels, const int32_t* front_len, const int64_t* t,
+                            const uint64_t* m, uint64_t total_limit, int32_t* choice,
+                            uint64_t* offset, int64_t* total_ns);
+
+/* ------------------------------------------------------------- GPU ---- */
+/* Benchmark pass (P:L88 WR step 1): for every b in the handle's policy set and
+ * every eligible algorithm whose workspace fits ws_limit, run the micro-config
+ * on scratch tensors: `warmup` untimed launches, then the median of `reps`
+ * CUDA-event timings, quantised to ns (reading G21).  Fills time_ns / ws
+ * ([MUCU_NUM_ALGOS][desc->n + 1], -1 / 0 where not measured).  Identical
+ * requests are served from the handle's in-memory cache.
+ * scratch: device buffer of >= mucu_benchmark_scratch_size() bytes (contents
+ * overwritten; the caller may pre-fill it with data of its choice).
+ * Synchronises cuda_stream. */
+mucu_status_t mucu_benchmark_scratch_size(const mucu_conv_desc_t* desc, mucu_conv_type_t type,
+                                          uint64_t ws_limit, uint64_t* bytes);
+mucu_status_t mucu_benchmark(mucu_handle_t handle, const mucu_conv_desc_t* desc, mucu_conv_type_t type,
+                             uint64_t ws_limit, void* scratch, uint64_t scratch_bytes, void* cuda_stream,
+                             int64_t* time_ns, uint64_t* ws);
+
+/* WR convenience: mucu_benchmark + mucu_plan_wr (P:L86-92 steps 1-3). */
+mucu_status_t mucu_plan_layer(mucu_handle_t handle, const mucu_conv_desc_t* desc, mucu_conv_type_t type,
+                              uint64_t ws_limit, void* scratch, uint64_t scratch_bytes, void* cuda_stream,
+                              mucu_micro_config_t* out, int32_t cap, int32_t* count, int64_t* total_ns);
+
+/* Execute a plan (Fig. 3): for each micro-config in order, offset
+ * the activation pointers by the samples already done and run the algorithm on
+ * micro_n samples.  out = alpha * op + beta * out (reading G5).
+ *   forward:          (x, w) -> y
+ *   backward_data:    (dy, w) -> dx
+ *   backward_filter:  (x, dy) -> dw (fp32); the user's beta applies to the
+ *                     first micro-batch, later ones accumulate with beta = 1
+ *                     ("output scale", reading G5).
+ * workspace: device buffer of ws_bytes >= max over the plan of
+ * mucu_workspace_size (INSUFFICIENT_WORKSPACE otherwise; NULL allowed when 0).
+ * Asynchronous on cuda_stream.  All device pointers must be 16-byte aligned. */
+mucu_status_t mucu_conv_forward(mucu_handle_t handle, const mucu_conv_desc_t* desc,
+                                const mucu_micro_config_t* plan, int32_t count, float alpha,
+                                const void* x, const void* w, float beta, void* y,
+                                void* workspace, uint64_t ws_bytes, void* cuda_stream);
+mucu_status_t mucu_conv_backward_data(mucu_handle_t handle, const mucu_conv_desc_t* desc,
+                                      const mucu_micro_config_t* plan, int32_t count, float alpha,
+                                      const void* dy, const void* w, float beta, void* dx,
+                                      void* workspace, uint64_t ws_bytes, void* cuda_stream);
+mucu_status_t mucu_conv_backward_filter(mucu_handle_t handle, const mucu_conv_desc_t* desc,
+                                        const mucu_micro_config_t* plan, int32_t count, float alpha,
+                                        const void* x, const void* dy, float beta, float* dw,
+                                        void* workspace, uint64_t ws_bytes, void* cuda_stream);
+
+/* ------------------------------------------------------------ WD ---- */
+/* WD needs every kernel before optimising: register the kernels,
+ * then plan once.  mucu_network_plan benchmarks each unique (desc, type)
+ * (deduplicated), builds each kernel's desirable set with the
+ * set-valued DP (ws_cap = total_limit) and solves the MCKP.  Then
+ * mucu_network_get returns kernel `kernel_id`'s plan, its segment offset into
+ * the caller's single network workspace and the segment size. */
+mucu_status_t mucu_network_create(mucu_network_t* net);
+mucu_status_t mucu_network_destroy(mucu_network_t net);
+mucu_status_t mucu_network_add(mucu_network_t net, const mucu_conv_desc_t* desc, mucu_conv_type_t type,
+                               int32_t* kernel_id);
+mucu_status_t mucu_network_plan(mucu_network_t net, mucu_handle_t handle, uint64_t total_limit,
+                                void* scratch, uint64_t scratch_bytes, void* cuda_stream);
+/* Same as mucu_network_plan but from caller-supplied timing tables (one
+ * [MUCU_NUM_ALGOS][n_k+1] pair per kernel, concatenated in kernel order);
+ * host-only, for offline planning from a stored benchmark table. */
+mucu_status_t mucu_network_plan_from_tables(mucu_network_t net, uint64_t total_limit,
+                                            const int64_t* time_ns, const uint64_t* ws);
+mucu_status_t mucu_network_get(mucu_network_t net, int32_t kernel_id, mucu_micro_config_t* out,
+                               int32_t cap, int32_t* count, uint64_t* ws_offset, uint64_t* ws_bytes,
+                               int64_t* time_ns);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* MUCUDNN_H_ */

@@ -1,0 +1,651 @@
+// api.cpp -- C ABI of libmucudnn (include/mucudnn.h): errors, geometry,
+// workspace sizing, the handle, the micro-batch executor (Fig. 3),
+// the benchmark pass (P:L88 WR step 1) and WD network planning
+// (P:L163-167).
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstdarg>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <map>
+#include <string>
+#include <vector>
+
+#include "mucudnn.h"
+#include "mucudnn_internal.h"
+
+namespace mucu {
+
+static thread_local char g_err[512] = "";
+
+mucu_status_t set_error(mucu_status_t s, const char* fmt, ...) {
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(g_err, sizeof(g_err), fmt, ap);
+    va_end(ap);
+    return s;
+}
+
+static mucu_status_t cuda_error(int e, const char* where) {
+    if (e == 0) return MUCU_OK;
+    return set_error(MUCU_ERR_CUDA, "%s: %s", where, cudaGetErrorString((cudaError_t)e));
+}
+
+bool make_geom(const mucu_conv_desc_t* d, Geom* g) {
+    if (!d) return false;
+    if (d->n <= 0 || d->c <= 0 || d->h <= 0 || d->w <= 0 || d->k <= 0 || d->r <= 0 || d->s <= 0 ||
+        d->pad < 0 || d->stride <= 0)
+        return false;
+    if (d->math < MUCU_MATH_F32 || d->math > MUCU_MATH_BF16) return false;
+    g->n = d->n; g->c = d->c; g->h = d->h; g->w = d->w; g->k = d->k; g->r = d->r; g->s = d->s;
+    g->pad = d->pad; g->stride = d->stride; g->math = d->math;
+    int64_t pn = (int64_t)d->h + 2 * d->pad - d->r, qn = (int64_t)d->w + 2 * d->pad - d->s;
+    if (pn < 0 || qn < 0) return false;
+    g->p = (int32_t)(pn / d->stride + 1);
+    g->q = (int32_t)(qn / d->stride + 1);
+    return g->p > 0 && g->q > 0;
+}
+
+bool is_pointwise(const Geom& g) { return g.r == 1 && g.s == 1 && g.pad == 0 && g.stride == 1; }
+
+bool algo_eligible(const Geom& g, int type, int algo) {
+    if (type < MUCU_FWD || type > MUCU_BWD_FILTER) return false;
+    switch (algo) {
+        case MUCU_ALGO_IMPLICIT_GEMM:
+        case MUCU_ALGO_IM2COL_GEMM:
+            return true;
+        case MUCU_ALGO_WINOGRAD_2X2_3X3:
+            // F(2x2,3x3): 3x3 filters, unit stride (ref [23]); BackwardFilter
+            // Winograd is NEXT-1 (not implemented); pad' = 2 - pad >= 0 for DGRAD.
+            return g.r == 3 && g.s == 3 && g.stride == 1 && g.pad <= 2 && type != MUCU_BWD_FILTER;
+        default:
+            return false;
+    }
+}
+
+mucu_status_t ws_layout(const Geom& g, int type, int algo, int32_t b, WsLayout* L) {
+    std::memset(L, 0, sizeof(*L));
+    if (!algo_eligible(g, type, algo)) return set_error(MUCU_ERR_UNSUPPORTED, "algorithm %d ineligible for this layer/type", algo);
+    if (b <= 0 || b > g.n) return set_error(MUCU_ERR_INVALID_VALUE, "micro-batch size %d outside 1..%d", b, g.n);
+    const uint64_t elt = (uint64_t)elt_size(g.math);
+    const uint64_t vec = 16 / elt;
+    const uint64_t RSC = (uint64_t)g.r * g.s * g.c;
+    const uint64_t PQ = (uint64_t)g.p * g.q;
+    if (algo == MUCU_ALGO_IMPLICIT_GEMM) return MUCU_OK;
+    if (algo == MUCU_ALGO_IM2COL_GEMM) {
+        L->kpitch = (int32_t)align_up(RSC, vec);
+        if (is_pointwise(g)) { L->kpitch = g.c; return MUCU_OK; }
+        if (type == MUCU_BWD_DATA) {
+            L->filter_padded = (RSC * elt) % 16 != 0;
+            const uint64_t fpitch = align_up(RSC, vec);
+            L->fixed_bytes = L->filter_padded ? align_up((uint64_t)g.k * fpitch * elt, 256) : 0;
+            L->kpitch = (int32_t)align_up(RSC, 4);  // fp32 dcol
+            L->a_off = L->fixed_bytes;
+            L->a_bytes = align_up((uint64_t)b * PQ * (uint64_t)L->kpitch * 4, 256);
+        } else {
+            L->filter_padded = (type == MUCU_FWD) && (RSC * elt) % 16 != 0;
+            L->fixed_bytes = L->filter_padded ? align_up((uint64_t)g.k * L->kpitch * elt, 256) : 0;
+            L->a_off = L->fixed_bytes;
+            L->a_bytes = align_up((uint64_t)b * PQ * (uint64_t)L->kpitch * elt, 256);
+        }
+        L->total = L->a_off + L->a_bytes;
+        return MUCU_OK;
+    }
+    // Winograd F(2x2,3x3): U (b-independent) | V | M (fp32).
+    const bool dgrad = type == MUCU_BWD_DATA;
+    const uint64_t OH = dgrad ? g.h : g.p, OW = dgrad ? g.w : g.q;
+    const uint64_t I = dgrad ? g.k : g.c, O = dgrad ? g.c : g.k;
+    const uint64_t T = ((OH + 1) / 2) * ((OW + 1) / 2);
+    L->fixed_bytes = align_up(16 * O * I * elt, 256);
+    L->a_off = L->fixed_bytes;
+    L->a_bytes = align_up(16 * (uint64_t)b * T * I * elt, 256);
+    L->b_off = L->a_off + L->a_bytes;
+    L->b_bytes = align_up(16 * (uint64_t)b * T * O * 4, 256);
+    L->total = L->b_off + L->b_bytes;
+    return MUCU_OK;
+}
+
+struct Handle {
+    int device = 0;
+    int num_sms = 148;
+    int policy = MUCU_POLICY_POW2;
+    int warmup = 2, reps = 5;
+    int32_t* sem = nullptr;
+    int32_t sem_cap = 0;
+    std::map<std::string, std::pair<std::vector<int64_t>, std::vector<uint64_t>>> cache;
+};
+
+static bool tc_math(int math) { return math == MUCU_MATH_TF32 || math == MUCU_MATH_BF16; }
+
+// ------------------------------------------------------------- dispatch --
+mucu_status_t run_micro(Handle* hd, const Geom& g, int type, int algo, int32_t b, float alpha, const void* in0,
+                        const void* in1, float beta, void* out, void* ws, uint64_t ws_bytes, cudaStream_t st,
+                        CallCtx* ctx) {
+    WsLayout L;
+    mucu_status_t s = ws_layout(g, type, algo, b, &L);
+    if (s != MUCU_OK) return s;
+    if (L.total > ws_bytes) return set_error(MUCU_ERR_INSUFFICIENT_WORKSPACE, "workspace %llu < %llu", (unsigned long long)ws_bytes, (unsigned long long)L.total);
+    char* wsb = (char*)ws;
+    const bool tc = tc_math(g.math);
+    const SemBuf sem{hd->sem, hd->sem_cap};
+    int e = 0;
+    if (tc) {
+        e = tc_run_micro(g, type, algo, b, alpha, in0, in1, beta, out, wsb, L, sem, hd->num_sms, st, ctx);
+        if (e == -1) return set_error(MUCU_ERR_UNSUPPORTED, "tensor-core path not available for this configuration");
+        return cuda_error(e, "tc kernel");
+    }
+    // ---- MUCU_MATH_F32: SIMT FFMA ----
+    const float* f0 = (const float*)in0;
+    const float* f1 = (const float*)in1;
+    float* fo = (float*)out;
+    if (type == MUCU_FWD) {
+        if (algo == MUCU_ALGO_IMPLICIT_GEMM) {
+            e = simt_fwd_ig(g, b, alpha, f0, f1, beta, fo, st);
+        } else if (algo == MUCU_ALGO_IM2COL_GEMM) {
+            const int64_t M = (int64_t)b * g.p * g.q, Kd = (int64_t)g.r * g.s * g.c;
+            if (is_pointwise(g)) {
+                e = simt_gemm_nt(M, g.k, Kd, alpha, f0, g.c, f1, Kd, beta, fo, g.k, 1, 0, 0, 0, st);
+            } else {
+                float* col = (float*)(wsb + L.a_off);
+                e = launch_im2col(g, b, f0, col, L.kpitch, st);
+                if (!e) e = simt_gemm_nt(M, g.k, Kd, alpha, col, L.kpitch, f1, Kd, beta, fo, g.k, 1, 0, 0, 0, st);
+            }
+        } else {
+            e = 0;
+            if (ctx->fixed_kind != 2 || ctx->fixed_src != in1) {
+                e = launch_wg_filter(g, false, f1, wsb, st);
+                ctx->fixed_kind = 2; ctx->fixed_src = in1;
+            }
+            const int64_t T = (int64_t)((g.p + 1) / 2) * ((g.q + 1) / 2) * b;
+            float* V = (float*)(wsb + L.a_off);
+            float* Mx = (float*)(wsb + L.b_off);
+            if (!e) e = launch_wg_input(g, false, b, f0, V, st);
+            if (!e) e = simt_gemm_nt(T, g.k, g.c, 1.f, V, g.c, (const float*)wsb, g.c, 0.f, Mx, g.k, 16,
+                                     T * g.c, (int64_t)g.k * g.c, T * g.k, st);
+            if (!e) e = launch_wg_output(g, false, b, alpha, Mx, beta, fo, st);
+        }
+    } else if (type == MUCU_BWD_DATA) {
+        if (algo == MUCU_ALGO_IMPLICIT_GEMM) {
+            e = simt_dgrad_ig(g, b, alpha, f0, f1, beta, fo, st);
+        } else if (algo == MUCU_ALGO_IM2COL_GEMM) {
+            const int64_t M = (int64_t)b * g.p * g.q, RSC = (int64_t)g.r * g.s * g.c;
+            if (is_pointwise(g)) {
+                e = simt_gemm_nn(M, g.c, g.k, alpha, f0, g.k, f1, g.c, beta, fo, g.c, st);
+            } else {
+                float* dcol = (float*)(wsb + L.a_off);
+                e = simt_gemm_nn(M, RSC, g.k, 1.f, f0, g.k, f1, RSC, 0.f, dcol, L.kpitch, st);
+                if (!e) e = launch_col2im(g, b, alpha, dcol, L.kpitch, beta, fo, st);
+            }
+        } else {
+            if (ctx->fixed_kind != 2 || ctx->fixed_src != in1) {
+                e = launch_wg_filter(g, true, f1, wsb, st);
+                ctx->fixed_kind = 2; ctx->fixed_src = in1;
+            }
+            const int64_t T = (int64_t)((g.h + 1) / 2) * ((g.w + 1) / 2) * b;
+            float* V = (float*)(wsb + L.a_off);
+            float* Mx = (float*)(wsb + L.b_off);
+            if (!e) e = launch_wg_input(g, true, b, f0, V, st);
+            if (!e) e = simt_gemm_nt(T, g.c, g.k, 1.f, V, g.k, (const float*)wsb, g.k, 0.f, Mx, g.c, 16,
+                                     T * g.k, (int64_t)g.c * g.k, T * g.c, st);
+            if (!e) e = launch_wg_output(g, true, b, alpha, Mx, beta, fo, st);
+        }
+    } else {  // MUCU_BWD_FILTER: in0 = x, in1 = dy, out = dw (fp32)
+        if (algo == MUCU_ALGO_IMPLICIT_GEMM) {
+            e = simt_wgrad(g, b, alpha, f1, f0, false, 0, beta, fo, sem, hd->num_sms, st);
+        } else {
+            if (is_pointwise(g)) {
+                e = simt_wgrad(g, b, alpha, f1, f0, true, g.c, beta, fo, sem, hd->num_sms, st);
+            } else {
+                float* col = (float*)(wsb + L.a_off);
+                e = launch_im2col(g, b, f0, col, L.kpitch, st);
+                if (!e) e = simt_wgrad(g, b, alpha, f1, col, true, L.kpitch, beta, fo, sem, hd->num_sms, st);
+            }
+        }
+    }
+    return cuda_error(e, "simt kernel");
+}
+
+}  // namespace mucu
+
+using namespace mucu;
+
+struct mucu_handle : public mucu::Handle {};
+
+struct mucu_network {
+    struct Kernel {
+        mucu_conv_desc_t desc;
+        int type;
+        std::vector<mucu_micro_config_t> plan;
+        uint64_t offset = 0, bytes = 0;
+        int64_t time_ns = 0;
+    };
+    std::vector<Kernel> kernels;
+    bool planned = false;
+};
+
+// ================================================================= misc ====
+extern "C" const char* mucu_status_string(mucu_status_t s) {
+    switch (s) {
+        case MUCU_OK: return "MUCU_OK";
+        case MUCU_ERR_INVALID_VALUE: return "MUCU_ERR_INVALID_VALUE";
+        case MUCU_ERR_UNSUPPORTED: return "MUCU_ERR_UNSUPPORTED";
+        case MUCU_ERR_INSUFFICIENT_WORKSPACE: return "MUCU_ERR_INSUFFICIENT_WORKSPACE";
+        case MUCU_ERR_INFEASIBLE: return "MUCU_ERR_INFEASIBLE";
+        case MUCU_ERR_CAPACITY: return "MUCU_ERR_CAPACITY";
+        case MUCU_ERR_MISALIGNED: return "MUCU_ERR_MISALIGNED";
+        case MUCU_ERR_CUDA: return "MUCU_ERR_CUDA";
+        case MUCU_ERR_INTERNAL: return "MUCU_ERR_INTERNAL";
+    }
+    return "MUCU_ERR_UNKNOWN";
+}
+
+extern "C" const char* mucu_last_error(void) { return g_err; }
+extern "C" int32_t mucu_version(void) { return MUCU_VERSION; }
+
+static int policy_from_env(int dflt) {
+    const char* p = getenv("MUCU_BATCH_POLICY");
+    if (!p) return dflt;
+    if (!strcmp(p, "all")) return MUCU_POLICY_ALL;
+    if (!strcmp(p, "pow2") || !strcmp(p, "powerOfTwo")) return MUCU_POLICY_POW2;
+    if (!strcmp(p, "undivided")) return MUCU_POLICY_UNDIVIDED;
+    return dflt;
+}
+
+extern "C" mucu_status_t mucu_create(mucu_handle_t* out, int device) {
+    if (!out) return set_error(MUCU_ERR_INVALID_VALUE, "create: null handle pointer");
+    *out = nullptr;
+    int e = (int)cudaSetDevice(device);
+    if (e) return cuda_error(e, "cudaSetDevice");
+    mucu_handle* h = new (std::nothrow) mucu_handle();
+    if (!h) return set_error(MUCU_ERR_INTERNAL, "create: out of host memory");
+    h->device = device;
+    cudaDeviceGetAttribute(&h->num_sms, cudaDevAttrMultiProcessorCount, device);
+    h->policy = policy_from_env(MUCU_POLICY_POW2);
+    if (const char* w = getenv("MUCU_BENCH_WARMUP")) h->warmup = std::max(0, atoi(w));
+    if (const char* r = getenv("MUCU_BENCH_REPS")) h->reps = std::max(1, atoi(r));
+    h->sem_cap = 1 << 16;
+    e = (int)cudaMalloc((void**)&h->sem, sizeof(int32_t) * h->sem_cap);
+    if (!e) e = (int)cudaMemset(h->sem, 0, sizeof(int32_t) * h->sem_cap);
+    if (e) { delete h; return cuda_error(e, "semaphore buffer"); }
+    *out = h;
+    return MUCU_OK;
+}
+
+extern "C" mucu_status_t mucu_destroy(mucu_handle_t h) {
+    if (!h) return MUCU_OK;
+    if (h->sem) cudaFree(h->sem);
+    delete h;
+    return MUCU_OK;
+}
+
+extern "C" mucu_status_t mucu_set_policy(mucu_handle_t h, mucu_policy_t p) {
+    if (!h || p < MUCU_POLICY_ALL || p > MUCU_POLICY_UNDIVIDED) return set_error(MUCU_ERR_INVALID_VALUE, "set_policy");
+    h->policy = p;
+    return MUCU_OK;
+}
+
+extern "C" mucu_status_t mucu_set_bench_params(mucu_handle_t h, int32_t warmup, int32_t reps) {
+    if (!h || warmup < 0 || reps < 1) return set_error(MUCU_ERR_INVALID_VALUE, "set_bench_params");
+    h->warmup = warmup;
+    h->reps = reps;
+    return MUCU_OK;
+}
+
+extern "C" mucu_status_t mucu_output_dims(const mucu_conv_desc_t* d, int32_t* p, int32_t* q) {
+    Geom g;
+    if (!make_geom(d, &g) || !p || !q) return set_error(MUCU_ERR_INVALID_VALUE, "output_dims: invalid descriptor");
+    *p = g.p;
+    *q = g.q;
+    return MUCU_OK;
+}
+
+extern "C" mucu_status_t mucu_workspace_size(const mucu_conv_desc_t* d, mucu_conv_type_t type, mucu_algo_t algo,
+                                             int32_t micro_n, uint64_t* bytes) {
+    Geom g;
+    if (!make_geom(d, &g) || !bytes) return set_error(MUCU_ERR_INVALID_VALUE, "workspace_size: invalid descriptor");
+    WsLayout L;
+    mucu_status_t s = ws_layout(g, type, algo, micro_n, &L);
+    if (s == MUCU_OK) *bytes = L.total;
+    return s;
+}
+
+// ============================================================= executor ====
+static mucu_status_t check_ptr(const void* p, const char* what) {
+    if (!p) return set_error(MUCU_ERR_INVALID_VALUE, "%s is null", what);
+    if ((uintptr_t)p % 16) return set_error(MUCU_ERR_MISALIGNED, "%s not 16-byte aligned", what);
+    return MUCU_OK;
+}
+
+static mucu_status_t execute(mucu_handle_t h, const mucu_conv_desc_t* d, int type, const mucu_micro_config_t* plan,
+                             int32_t count, float alpha, const void* in0, const void* in1, float beta, void* out,
+                             void* ws, uint64_t ws_bytes, void* stream) {
+    if (!h) return set_error(MUCU_ERR_INVALID_VALUE, "null handle");
+    Geom g;
+    if (!make_geom(d, &g)) return set_error(MUCU_ERR_INVALID_VALUE, "invalid descriptor");
+    if (!plan || count <= 0) return set_error(MUCU_ERR_INVALID_VALUE, "empty plan");
+    mucu_status_t s;
+    if ((s = check_ptr(in0, "input 0")) || (s = check_ptr(in1, "input 1")) || (s = check_ptr(out, "output"))) return s;
+    if (ws && (uintptr_t)ws % 256) return set_error(MUCU_ERR_MISALIGNED, "workspace not 256-byte aligned");
+    // Validate the whole plan before any launch.
+    int64_t sum = 0;
+    for (int32_t i = 0; i < count; ++i) {
+        if (plan[i].micro_n <= 0) return set_error(MUCU_ERR_INVALID_VALUE, "plan part %d has micro_n <= 0", i);
+        sum += plan[i].micro_n;
+        if (sum > g.n) return set_error(MUCU_ERR_INVALID_VALUE, "plan parts exceed N");
+        WsLayout L;
+        if ((s = ws_layout(g, type, plan[i].algo, plan[i].micro_n, &L))) return s;
+        if (L.total > ws_bytes || (L.total && !ws))
+            return set_error(MUCU_ERR_INSUFFICIENT_WORKSPACE, "part %d needs %llu workspace bytes, have %llu", i,
+                             (unsigned long long)L.total, (unsigned long long)ws_bytes);
+    }
+    if (sum != g.n) return set_error(MUCU_ERR_INVALID_VALUE, "plan parts sum to %lld, N = %d", (long long)sum, g.n);
+    const uint64_t elt = (uint64_t)elt_size(g.math);
+    const uint64_t in_sample = (uint64_t)g.h * g.w * g.c * elt;   // x / dx per sample
+    const uint64_t out_sample = (uint64_t)g.p * g.q * g.k * elt;  // y / dy per sample
+    cudaStream_t st = (cudaStream_t)stream;
+    CallCtx ctx;
+    int64_t done = 0;
+    for (int32_t i = 0; i < count; ++i) {
+        const int32_t b = plan[i].micro_n;
+        const char* p0 = (const char*)in0;
+        const char* p1 = (const char*)in1;
+        char* po = (char*)out;
+        float bta = beta;
+        if (type == MUCU_FWD) { p0 += done * in_sample; po += done * out_sample; }
+        else if (type == MUCU_BWD_DATA) { p0 += done * out_sample; po += done * in_sample; }
+        else { p0 += done * in_sample; p1 += done * out_sample; if (i > 0) bta = 1.f; }  // P:L58 output scale
+        s = run_micro(h, g, type, plan[i].algo, b, alpha, p0, p1, bta, po, ws, ws_bytes, st, &ctx);
+        if (s) return s;
+        done += b;
+    }
+    return MUCU_OK;
+}
+
+extern "C" mucu_status_t mucu_conv_forward(mucu_handle_t h, const mucu_conv_desc_t* d, const mucu_micro_config_t* plan,
+                                           int32_t count, float alpha, const void* x, const void* w, float beta,
+                                           void* y, void* ws, uint64_t ws_bytes, void* stream) {
+    return execute(h, d, MUCU_FWD, plan, count, alpha, x, w, beta, y, ws, ws_bytes, stream);
+}
+
+extern "C" mucu_status_t mucu_conv_backward_data(mucu_handle_t h, const mucu_conv_desc_t* d,
+                                                 const mucu_micro_config_t* plan, int32_t count, float alpha,
+                                                 const void* dy, const void* w, float beta, void* dx, void* ws,
+                                                 uint64_t ws_bytes, void* stream) {
+    return execute(h, d, MUCU_BWD_DATA, plan, count, alpha, dy, w, beta, dx, ws, ws_bytes, stream);
+}
+
+extern "C" mucu_status_t mucu_conv_backward_filter(mucu_handle_t h, const mucu_conv_desc_t* d,
+                                                   const mucu_micro_config_t* plan, int32_t count, float alpha,
+                                                   const void* x, const void* dy, float beta, float* dw, void* ws,
+                                                   uint64_t ws_bytes, void* stream) {
+    return execute(h, d, MUCU_BWD_FILTER, plan, count, alpha, x, dy, beta, dw, ws, ws_bytes, stream);
+}
+
+// ============================================================ benchmark ====
+static std::vector<int32_t> policy_sizes(int policy, int32_t n) {
+    std::vector<int32_t> v;
+    if (policy == MUCU_POLICY_ALL) {
+        for (int32_t b = 1; b <= n; ++b) v.push_back(b);
+    } else if (policy == MUCU_POLICY_POW2) {
+        for (int32_t b = 1; b <= n; b *= 2) v.push_back(b);
+        if (v.empty() || v.back() != n) v.push_back(n);  // reading G20
+    } else {
+        v.push_back(n);
+    }
+    return v;
+}
+
+struct ScratchLayout {
+    uint64_t in0, in1, out, ws, total;
+};
+
+static ScratchLayout scratch_layout(const Geom& g, int type, uint64_t ws_limit) {
+    const uint64_t elt = (uint64_t)elt_size(g.math);
+    const uint64_t X = align_up((uint64_t)g.n * g.h * g.w * g.c * elt, 256);
+    const uint64_t Y = align_up((uint64_t)g.n * g.p * g.q * g.k * elt, 256);
+    const uint64_t Wt = align_up((uint64_t)g.k * g.r * g.s * g.c * elt, 256);
+    const uint64_t DW = align_up((uint64_t)g.k * g.r * g.s * g.c * 4, 256);
+    // Largest workspace any benchmarked micro-config may use.
+    uint64_t need = 0;
+    for (int a = 0; a < MUCU_NUM_ALGOS; ++a)
+        for (int32_t b : {1, g.n}) {
+            WsLayout L;
+            if (ws_layout(g, type, a, b, &L) == MUCU_OK && L.total <= ws_limit) need = std::max(need, L.total);
+        }
+    // ws grows with b, so size at N bounds every b that fits the limit.
+    need = std::min<uint64_t>(align_up(need, 256), align_up(ws_limit, 256));
+    ScratchLayout s;
+    s.in0 = 0;
+    if (type == MUCU_FWD) { s.in1 = X; s.out = X + Wt; s.ws = X + Wt + Y; }
+    else if (type == MUCU_BWD_DATA) { s.in1 = Y; s.out = Y + Wt; s.ws = Y + Wt + X; }
+    else { s.in1 = X; s.out = X + Y; s.ws = X + Y + DW; }
+    s.total = s.ws + need;
+    return s;
+}
+
+extern "C" mucu_status_t mucu_benchmark_scratch_size(const mucu_conv_desc_t* d, mucu_conv_type_t type,
+                                                     uint64_t ws_limit, uint64_t* bytes) {
+    Geom g;
+    if (!make_geom(d, &g) || !bytes || type < 0 || type > 2) return set_error(MUCU_ERR_INVALID_VALUE, "benchmark_scratch_size");
+    *bytes = scratch_layout(g, type, ws_limit).total;
+    return MUCU_OK;
+}
+
+static std::string cache_key(const mucu_conv_desc_t* d, int type, uint64_t limit, int policy, int warmup, int reps) {
+    char buf[256];
+    snprintf(buf, sizeof(buf), "%d,%d,%d,%d,%d,%d,%d,%d,%d,%d|%d|%llu|%d|%d|%d", d->n, d->c, d->h, d->w, d->k, d->r,
+             d->s, d->pad, d->stride, d->math, type, (unsigned long long)limit, policy, warmup, reps);
+    return buf;
+}
+
+extern "C" mucu_status_t mucu_benchmark(mucu_handle_t h, const mucu_conv_desc_t* d, mucu_conv_type_t type,
+                                        uint64_t ws_limit, void* scratch, uint64_t scratch_bytes, void* stream,
+                                        int64_t* time_ns, uint64_t* ws) {
+    if (!h || !time_ns || !ws) return set_error(MUCU_ERR_INVALID_VALUE, "benchmark: bad arguments");
+    Geom g;
+    if (!make_geom(d, &g) || type < 0 || type > 2) return set_error(MUCU_ERR_INVALID_VALUE, "benchmark: invalid descriptor");
+    const size_t cols = (size_t)g.n + 1;
+    const std::string key = cache_key(d, type, ws_limit, h->policy, h->warmup, h->reps);
+    auto it = h->cache.find(key);
+    if (it != h->cache.end()) {  // P:L159 in-memory cache of benchmark results
+        std::copy(it->second.first.begin(), it->second.first.end(), time_ns);
+        std::copy(it->second.second.begin(), it->second.second.end(), ws);
+        return MUCU_OK;
+    }
+    ScratchLayout S = scratch_layout(g, type, ws_limit);
+    if (!scratch || scratch_bytes < S.total)
+        return set_error(MUCU_ERR_INSUFFICIENT_WORKSPACE, "benchmark scratch %llu < %llu", (unsigned long long)scratch_bytes, (unsigned long long)S.total);
+    if ((uintptr_t)scratch % 256) return set_error(MUCU_ERR_MISALIGNED, "scratch not 256-byte aligned");
+    for (size_t i = 0; i < MUCU_NUM_ALGOS * cols; ++i) { time_ns[i] = -1; ws[i] = 0; }
+    cudaStream_t st = (cudaStream_t)stream;
+    char* base = (char*)scratch;
+    cudaEvent_t e0, e1;
+    if (cudaEventCreate(&e0) || cudaEventCreate(&e1)) return cuda_error((int)cudaGetLastError(), "event create");
+    mucu_status_t status = MUCU_OK;
+    std::vector<float> samples;
+    for (int32_t b : policy_sizes(h->policy, g.n)) {
+        for (int a = 0; a < MUCU_NUM_ALGOS && status == MUCU_OK; ++a) {
+            WsLayout L;
+            if (ws_layout(g, type, a, b, &L) != MUCU_OK || L.total > ws_limit) continue;
+            auto launch = [&]() {
+                CallCtx ctx;  // each timed run is a whole call: includes the filter transform
+                return run_micro(h, g, type, a, b, 1.f, base + S.in0, base + S.in1, 0.f, base + S.out, base + S.ws,
+                                 S.total - S.ws, st, &ctx);
+            };
+            mucu_status_t r = MUCU_OK;
+            for (int i = 0; i < h->warmup && r == MUCU_OK; ++i) r = launch();
+            if (r == MUCU_ERR_UNSUPPORTED) continue;  // e.g. math mode without this kernel
+            if (r) { status = r; break; }
+            samples.clear();
+            for (int i = 0; i < h->reps; ++i) {
+                cudaEventRecord(e0, st);
+                r = launch();
+                cudaEventRecord(e1, st);
+                if (r) break;
+                if (cudaEventSynchronize(e1)) { r = cuda_error((int)cudaGetLastError(), "benchmark sync"); break; }
+                float ms = 0.f;
+                cudaEventElapsedTime(&ms, e0, e1);
+                samples.push_back(ms);
+            }
+            if (r) { status = r; break; }
+            std::sort(samples.begin(), samples.end());
+            float med = samples[samples.size() / 2];
+            time_ns[(size_t)a * cols + b] = (int64_t)(med * 1.0e6f + 0.5f);
+            ws[(size_t)a * cols + b] = L.total;
+        }
+        if (status) break;
+    }
+    cudaEventDestroy(e0);
+    cudaEventDestroy(e1);
+    if (status) return status;
+    int e = (int)cudaStreamSynchronize(st);
+    if (e) return cuda_error(e, "benchmark stream");
+    h->cache[key] = {std::vector<int64_t>(time_ns, time_ns + MUCU_NUM_ALGOS * cols),
+                     std::vector<uint64_t>(ws, ws + MUCU_NUM_ALGOS * cols)};
+    return MUCU_OK;
+}
+
+extern "C" mucu_status_t mucu_plan_layer(mucu_handle_t h, const mucu_conv_desc_t* d, mucu_conv_type_t type,
+                                         uint64_t ws_limit, void* scratch, uint64_t scratch_bytes, void* stream,
+                                         mucu_micro_config_t* out, int32_t cap, int32_t* count, int64_t* total_ns) {
+    Geom g;
+    if (!make_geom(d, &g)) return set_error(MUCU_ERR_INVALID_VALUE, "plan_layer: invalid descriptor");
+    std::vector<int64_t> t((size_t)MUCU_NUM_ALGOS * (g.n + 1));
+    std::vector<uint64_t> w(t.size());
+    mucu_status_t s = mucu_benchmark(h, d, type, ws_limit, scratch, scratch_bytes, stream, t.data(), w.data());
+    if (s) return s;
+    return mucu_plan_wr(g.n, t.data(), w.data(), ws_limit, out, cap, count, total_ns);
+}
+
+// =================================================================== WD ====
+extern "C" mucu_status_t mucu_network_create(mucu_network_t* net) {
+    if (!net) return set_error(MUCU_ERR_INVALID_VALUE, "network_create");
+    *net = new (std::nothrow) mucu_network();
+    return *net ? MUCU_OK : set_error(MUCU_ERR_INTERNAL, "network_create: out of memory");
+}
+
+extern "C" mucu_status_t mucu_network_destroy(mucu_network_t net) {
+    delete net;
+    return MUCU_OK;
+}
+
+extern "C" mucu_status_t mucu_network_add(mucu_network_t net, const mucu_conv_desc_t* d, mucu_conv_type_t type,
+                                          int32_t* kernel_id) {
+    Geom g;
+    if (!net || !make_geom(d, &g) || type < 0 || type > 2) return set_error(MUCU_ERR_INVALID_VALUE, "network_add");
+    mucu_network::Kernel k;
+    k.desc = *d;
+    k.type = type;
+    net->kernels.push_back(k);
+    net->planned = false;
+    if (kernel_id) *kernel_id = (int32_t)net->kernels.size() - 1;
+    return MUCU_OK;
+}
+
+// Fronts (set-valued DP) per kernel, then the MCKP.
+static mucu_status_t plan_network_tables(mucu_network_t net, uint64_t total_limit,
+                                         const std::vector<std::vector<int64_t>>& T,
+                                         const std::vector<std::vector<uint64_t>>& W) {
+    const int K = (int)net->kernels.size();
+    std::vector<std::vector<int64_t>> ft(K);
+    std::vector<std::vector<uint64_t>> fm(K);
+    std::vector<std::vector<std::vector<mucu_micro_config_t>>> fp(K);
+    std::map<std::string, int> dedupe;  // identical (desc, type) share one front
+    for (int k = 0; k < K; ++k) {
+        const auto& kd = net->kernels[k];
+        const int32_t n = kd.desc.n;
+        std::string key = cache_key(&kd.desc, kd.type, total_limit, 0, 0, 0);
+        auto it = dedupe.find(key);
+        if (it != dedupe.end() && T[k] == T[it->second] && W[k] == W[it->second]) {
+            ft[k] = ft[it->second]; fm[k] = fm[it->second]; fp[k] = fp[it->second];
+            continue;
+        }
+        int32_t len = 0;
+        mucu_status_t s = mucu_pareto_front(n, T[k].data(), W[k].data(), total_limit, nullptr, nullptr, 0, &len,
+                                            nullptr, nullptr);
+        if (s != MUCU_OK && s != MUCU_ERR_CAPACITY) return s == MUCU_ERR_INSUFFICIENT_WORKSPACE ? set_error(MUCU_ERR_INFEASIBLE, "kernel %d: nothing fits the total limit", k) : s;
+        ft[k].resize(len); fm[k].resize(len);
+        std::vector<mucu_micro_config_t> plans((size_t)len * n);
+        std::vector<int32_t> plen(len);
+        s = mucu_pareto_front(n, T[k].data(), W[k].data(), total_limit, ft[k].data(), fm[k].data(), len, &len,
+                              plans.data(), plen.data());
+        if (s) return s;
+        fp[k].resize(len);
+        for (int i = 0; i < len; ++i)
+            fp[k][i].assign(plans.begin() + (size_t)i * n, plans.begin() + (size_t)i * n + plen[i]);
+        dedupe[key] = k;
+    }
+    std::vector<int32_t> flen(K);
+    std::vector<int64_t> tt;
+    std::vector<uint64_t> mm;
+    for (int k = 0; k < K; ++k) {
+        flen[k] = (int32_t)ft[k].size();
+        tt.insert(tt.end(), ft[k].begin(), ft[k].end());
+        mm.insert(mm.end(), fm[k].begin(), fm[k].end());
+    }
+    std::vector<int32_t> choice(K);
+    std::vector<uint64_t> offs(K);
+    int64_t total = 0;
+    mucu_status_t s = mucu_solve_wd(K, flen.data(), tt.data(), mm.data(), total_limit, choice.data(), offs.data(), &total);
+    if (s) return s;
+    for (int k = 0; k < K; ++k) {
+        auto& kd = net->kernels[k];
+        kd.plan = fp[k][choice[k]];
+        kd.offset = offs[k];
+        kd.bytes = align_up(fm[k][choice[k]], 256);
+        kd.time_ns = ft[k][choice[k]];
+    }
+    net->planned = true;
+    return MUCU_OK;
+}
+
+extern "C" mucu_status_t mucu_network_plan(mucu_network_t net, mucu_handle_t h, uint64_t total_limit, void* scratch,
+                                           uint64_t scratch_bytes, void* stream) {
+    if (!net || !h || net->kernels.empty()) return set_error(MUCU_ERR_INVALID_VALUE, "network_plan");
+    const int K = (int)net->kernels.size();
+    std::vector<std::vector<int64_t>> T(K);
+    std::vector<std::vector<uint64_t>> W(K);
+    for (int k = 0; k < K; ++k) {
+        const auto& kd = net->kernels[k];
+        const size_t sz = (size_t)MUCU_NUM_ALGOS * (kd.desc.n + 1);
+        T[k].resize(sz); W[k].resize(sz);
+        // A kernel can use at most the whole budget; the cache dedupes repeats.
+        mucu_status_t s = mucu_benchmark(h, &kd.desc, (mucu_conv_type_t)kd.type, total_limit, scratch, scratch_bytes,
+                                         stream, T[k].data(), W[k].data());
+        if (s) return s;
+    }
+    return plan_network_tables(net, total_limit, T, W);
+}
+
+extern "C" mucu_status_t mucu_network_plan_from_tables(mucu_network_t net, uint64_t total_limit, const int64_t* time_ns,
+                                                       const uint64_t* ws) {
+    if (!net || net->kernels.empty() || !time_ns || !ws) return set_error(MUCU_ERR_INVALID_VALUE, "network_plan_from_tables");
+    const int K = (int)net->kernels.size();
+    std::vector<std::vector<int64_t>> T(K);
+    std::vector<std::vector<uint64_t>> W(K);
+    size_t off = 0;
+    for (int k = 0; k < K; ++k) {
+        const size_t sz = (size_t)MUCU_NUM_ALGOS * (net->kernels[k].desc.n + 1);
+        T[k].assign(time_ns + off, time_ns + off + sz);
+        W[k].assign(ws + off, ws + off + sz);
+        off += sz;
+    }
+    return plan_network_tables(net, total_limit, T, W);
+}
+
+extern "C" mucu_status_t mucu_network_get(mucu_network_t net, int32_t kernel_id, mucu_micro_config_t* out, int32_t cap,
+                                          int32_t* count, uint64_t* ws_offset, uint64_t* ws_bytes, int64_t* time_ns) {
+    if (!net || kernel_id < 0 || kernel_id >= (int32_t)net->kernels.size() || !count)
+        return set_error(MUCU_ERR_INVALID_VALUE, "network_get");
+    if (!net->planned) return set_error(MUCU_ERR_INVALID_VALUE, "network_get: network not planned");
+    const auto& kd = net->kernels[kernel_id];
+    *count = (int32_t)kd.plan.size();
+    if (ws_offset) *ws_offset = kd.offset;
+    if (ws_bytes) *ws_bytes = kd.bytes;
+    if (time_ns) *time_ns = kd.time_ns;
+    if (!out || cap < *count) return set_error(MUCU_ERR_CAPACITY, "network_get: capacity");
+    std::copy(kd.plan.begin(), kd.plan.end(), out);
+    return MUCU_OK;
+}

@@ -1,0 +1,367 @@
+// kernels_elem.cu -- data-movement kernels of the workspace-using algorithms.
+//
+//   im2col            (algorithm (b), "explicit GEMM"): x -> col[b*P*Q][kpitch]
+//   pad_filter        KRSC filter copied to a 16-B aligned row pitch (for TMA)
+//   col2im            deterministic gather-sum dcol -> dx (no atomics)
+//   wg_filter/input/output   Winograd F(2x2,3x3) transforms (algorithm (c),
+//                     Lavin & Gray, PAPER.md ref [23] P:L317)
+//
+// These passes are HBM-bound (no reuse beyond a few neighbouring pixels):
+// grid-stride loops with the channel index fastest so that consecutive threads
+// touch consecutive addresses (coalesced), 16-byte vectors where C allows,
+// grid sized to a multiple of the SM count.
+#include <cuda_bf16.h>
+#include <cuda_runtime.h>
+
+#include "mucudnn_internal.h"
+
+namespace mucu {
+
+namespace {
+
+template <class T> __device__ __forceinline__ float to_f(T v);
+template <> __device__ __forceinline__ float to_f<float>(float v) { return v; }
+template <> __device__ __forceinline__ float to_f<__nv_bfloat16>(__nv_bfloat16 v) { return __bfloat162float(v); }
+template <class T> __device__ __forceinline__ T from_f(float v);
+template <> __device__ __forceinline__ float from_f<float>(float v) { return v; }
+template <> __device__ __forceinline__ __nv_bfloat16 from_f<__nv_bfloat16>(float v) { return __float2bfloat16_rn(v); }
+
+int grid_for(int64_t work, int threads) {
+    int dev = 0, sms = 148;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    int64_t blocks = (work + threads - 1) / threads;
+    int64_t cap = (int64_t)sms * 16;
+    if (blocks > cap) blocks = cap;
+    if (blocks < 1) blocks = 1;
+    return (int)blocks;
+}
+
+// ---------------------------------------------------------------- im2col --
+// col[m][kk] = x[n, p*st + r - pad, q*st + s - pad, c] (0 outside / kk >= RSC),
+// m = (n,p,q), kk = (r,s,c).  Vector version: V = 16/sizeof(T) channels per
+// thread (requires C % V == 0, so a chunk never straddles (r,s)).
+template <class T, int V>
+__global__ void im2col_kernel(const T* __restrict__ x, T* __restrict__ col, int64_t rows, int H, int W,
+                              int C, int P, int Q, int S, int pad, int st, int RSC, int kpitch) {
+    const int64_t chunks_per_row = kpitch / V;
+    const int64_t total = rows * chunks_per_row;
+    for (int64_t idx = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; idx < total;
+         idx += (int64_t)gridDim.x * blockDim.x) {
+        int64_t m = idx / chunks_per_row;
+        int kk = (int)(idx - m * chunks_per_row) * V;
+        T* dst = col + m * kpitch + kk;
+        int pq = P * Q;
+        int n = (int)(m / pq);
+        int rem = (int)(m - (int64_t)n * pq);
+        int p = rem / Q, q = rem - (rem / Q) * Q;
+        bool ok = kk < RSC;
+        int h = 0, w = 0, c = 0;
+        if (ok) {
+            int rs = kk / C;
+            c = kk - rs * C;
+            int r = rs / S, s = rs - (rs / S) * S;
+            h = p * st + r - pad;
+            w = q * st + s - pad;
+            ok = (h >= 0 && h < H && w >= 0 && w < W);
+        }
+        if constexpr (V > 1) {
+            uint4 v = make_uint4(0, 0, 0, 0);
+            if (ok) v = *reinterpret_cast<const uint4*>(x + (((int64_t)n * H + h) * W + w) * C + c);
+            *reinterpret_cast<uint4*>(dst) = v;
+        } else {
+            *dst = ok ? x[(((int64_t)n * H + h) * W + w) * C + c] : from_f<T>(0.f);
+        }
+    }
+}
+
+// Scalar fallback when C is not a multiple of the vector width: one element
+// per thread, kk = (r,s,c) decomposed individually.
+template <class T>
+__global__ void im2col_scalar_kernel(const T* __restrict__ x, T* __restrict__ col, int64_t rows, int H, int W,
+                                     int C, int P, int Q, int S, int pad, int st, int RSC, int kpitch) {
+    const int64_t total = rows * kpitch;
+    for (int64_t idx = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; idx < total;
+         idx += (int64_t)gridDim.x * blockDim.x) {
+        int64_t m = idx / kpitch;
+        int kk = (int)(idx - m * kpitch);
+        float v = 0.f;
+        if (kk < RSC) {
+            int pq = P * Q;
+            int n = (int)(m / pq);
+            int rem = (int)(m - (int64_t)n * pq);
+            int p = rem / Q, q = rem % Q;
+            int rs = kk / C, c = kk % C;
+            int r = rs / S, s = rs % S;
+            int h = p * st + r - pad, w = q * st + s - pad;
+            if (h >= 0 && h < H && w >= 0 && w < W) v = to_f<T>(x[(((int64_t)n * H + h) * W + w) * C + c]);
+        }
+        col[idx] = from_f<T>(v);
+    }
+}
+
+template <class T>
+__global__ void pad_filter_kernel(const T* __restrict__ w, T* __restrict__ wp, int K, int RSC, int kpitch) {
+    const int64_t total = (int64_t)K * kpitch;
+    for (int64_t idx = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; idx < total;
+         idx += (int64_t)gridDim.x * blockDim.x) {
+        int k = (int)(idx / kpitch), kk = (int)(idx % kpitch);
+        wp[idx] = kk < RSC ? w[(int64_t)k * RSC + kk] : from_f<T>(0.f);
+    }
+}
+
+// ---------------------------------------------------------------- col2im --
+// dx[n,h,w,c] = alpha * sum_{r,s: st | h+pad-r, ...} dcol[(n,p,q)][(r*S+s)*C + c] + beta * dx
+// (the adjoint of im2col; gather form, so every dx element is written once in
+// a fixed summation order -- deterministic, no atomics).
+template <class T>
+__global__ void col2im_kernel(const float* __restrict__ dcol, T* __restrict__ dx, int64_t total, int H, int W,
+                              int C, int P, int Q, int R, int S, int pad, int st, int kpitch, float alpha,
+                              float beta) {
+    for (int64_t idx = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; idx < total;
+         idx += (int64_t)gridDim.x * blockDim.x) {
+        int c = (int)(idx % C);
+        int64_t pix = idx / C;
+        int w = (int)(pix % W);
+        int64_t t2 = pix / W;
+        int h = (int)(t2 % H);
+        int n = (int)(t2 / H);
+        float acc = 0.f;
+        for (int r = 0; r < R; ++r) {
+            int ph = h + pad - r;
+            if (ph < 0 || ph % st) continue;
+            int p = ph / st;
+            if (p >= P) continue;
+            for (int s = 0; s < S; ++s) {
+                int pw = w + pad - s;
+                if (pw < 0 || pw % st) continue;
+                int q = pw / st;
+                if (q >= Q) continue;
+                acc += dcol[(((int64_t)n * P + p) * Q + q) * kpitch + (r * S + s) * C + c];
+            }
+        }
+        float out = alpha * acc;
+        if (beta != 0.f) out += beta * to_f<T>(dx[idx]);
+        dx[idx] = from_f<T>(out);
+    }
+}
+
+// ------------------------------------------------------------- Winograd --
+// F(2x2,3x3) (Lavin & Gray, ref [23]):
+//   G  = [[1,0,0],[1/2,1/2,1/2],[1/2,-1/2,1/2],[0,0,1]]
+//   B^T= [[1,0,-1,0],[0,1,1,0],[0,-1,1,0],[0,1,0,-1]]
+//   A^T= [[1,1,1,0],[0,1,-1,-1]]
+// Y = A^T [ (G g G^T) .* (B^T d B) ] A, per 4x4 input tile (tile stride 2).
+// Layouts: U[xi][o][i], V[xi][t][i], M[xi][t][o] with xi = 4*a + b, o = output
+// channel, i = input channel, t = (n, tile_h, tile_w).
+// FWD: i = C, o = K, g = w[o,:,:,i].  DGRAD (full conv with the 180-degree
+// rotated, C/K-swapped filter; pad' = 2 - pad): i = K, o = C,
+// g[r][s] = w[i, 2-r, 2-s, o].
+template <class T>
+__global__ void wg_filter_kernel(const T* __restrict__ w, T* __restrict__ U, int O, int I, int C, bool dgrad) {
+    const int64_t total = (int64_t)O * I;
+    for (int64_t idx = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; idx < total;
+         idx += (int64_t)gridDim.x * blockDim.x) {
+        int i = (int)(idx % I), o = (int)(idx / I);
+        float g[3][3];
+        for (int r = 0; r < 3; ++r)
+            for (int s = 0; s < 3; ++s) {
+                // w is KRSC: element (k, r, s, c)
+                g[r][s] = dgrad ? to_f<T>(w[(((int64_t)i * 3 + (2 - r)) * 3 + (2 - s)) * C + o])
+                                : to_f<T>(w[(((int64_t)o * 3 + r) * 3 + s) * C + i]);
+            }
+        float t[4][3];  // t = G g
+        for (int s = 0; s < 3; ++s) {
+            t[0][s] = g[0][s];
+            t[1][s] = 0.5f * (g[0][s] + g[1][s] + g[2][s]);
+            t[2][s] = 0.5f * (g[0][s] - g[1][s] + g[2][s]);
+            t[3][s] = g[2][s];
+        }
+        for (int a = 0; a < 4; ++a) {  // u = t G^T
+            float u0 = t[a][0];
+            float u1 = 0.5f * (t[a][0] + t[a][1] + t[a][2]);
+            float u2 = 0.5f * (t[a][0] - t[a][1] + t[a][2]);
+            float u3 = t[a][2];
+            const int64_t plane = (int64_t)O * I;
+            U[(a * 4 + 0) * plane + idx] = from_f<T>(u0);
+            U[(a * 4 + 1) * plane + idx] = from_f<T>(u1);
+            U[(a * 4 + 2) * plane + idx] = from_f<T>(u2);
+            U[(a * 4 + 3) * plane + idx] = from_f<T>(u3);
+        }
+    }
+}
+
+// V[xi][t][i] = (B^T d B)[xi], d = 4x4 patch of `in` ([b, IH, IW, I]) at
+// (2*th - pad, 2*tw - pad), zero outside.  TH x TW tiles per image.
+template <class T>
+__global__ void wg_input_kernel(const T* __restrict__ in, T* __restrict__ V, int64_t tiles, int IH, int IW,
+                                int I, int TH, int TW, int pad) {
+    const int64_t total = tiles * I;
+    for (int64_t idx = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; idx < total;
+         idx += (int64_t)gridDim.x * blockDim.x) {
+        int i = (int)(idx % I);
+        int64_t t = idx / I;
+        int tw = (int)(t % TW);
+        int64_t t2 = t / TW;
+        int th = (int)(t2 % TH);
+        int n = (int)(t2 / TH);
+        float d[4][4];
+        for (int a = 0; a < 4; ++a)
+            for (int b = 0; b < 4; ++b) {
+                int h = 2 * th - pad + a, w = 2 * tw - pad + b;
+                d[a][b] = (h >= 0 && h < IH && w >= 0 && w < IW)
+                              ? to_f<T>(in[(((int64_t)n * IH + h) * IW + w) * I + i]) : 0.f;
+            }
+        float e[4][4];  // e = B^T d
+        for (int b = 0; b < 4; ++b) {
+            e[0][b] = d[0][b] - d[2][b];
+            e[1][b] = d[1][b] + d[2][b];
+            e[2][b] = d[2][b] - d[1][b];
+            e[3][b] = d[1][b] - d[3][b];
+        }
+        const int64_t plane = tiles * I;
+        for (int a = 0; a < 4; ++a) {  // v = e B
+            float v0 = e[a][0] - e[a][2];
+            float v1 = e[a][1] + e[a][2];
+            float v2 = e[a][2] - e[a][1];
+            float v3 = e[a][1] - e[a][3];
+            V[(a * 4 + 0) * plane + idx] = from_f<T>(v0);
+            V[(a * 4 + 1) * plane + idx] = from_f<T>(v1);
+            V[(a * 4 + 2) * plane + idx] = from_f<T>(v2);
+            V[(a * 4 + 3) * plane + idx] = from_f<T>(v3);
+        }
+    }
+}
+
+// out[n, 2th+i, 2tw+j, o] = alpha * (A^T M A)[i][j] + beta * out (masked at the
+// ragged right/bottom edge).
+template <class T>
+__global__ void wg_output_kernel(const float* __restrict__ M, T* __restrict__ out, int64_t tiles, int OH, int OW,
+                                 int O, int TH, int TW, float alpha, float beta) {
+    const int64_t total = tiles * O;
+    const int64_t plane = total;
+    for (int64_t idx = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; idx < total;
+         idx += (int64_t)gridDim.x * blockDim.x) {
+        int o = (int)(idx % O);
+        int64_t t = idx / O;
+        int tw = (int)(t % TW);
+        int64_t t2 = t / TW;
+        int th = (int)(t2 % TH);
+        int n = (int)(t2 / TH);
+        float m[4][4];
+        for (int a = 0; a < 4; ++a)
+            for (int b = 0; b < 4; ++b) m[a][b] = M[(a * 4 + b) * plane + idx];
+        float z[2][4];  // z = A^T m
+        for (int b = 0; b < 4; ++b) {
+            z[0][b] = m[0][b] + m[1][b] + m[2][b];
+            z[1][b] = m[1][b] - m[2][b] - m[3][b];
+        }
+        for (int a = 0; a < 2; ++a) {
+            float y0 = z[a][0] + z[a][1] + z[a][2];
+            float y1 = z[a][1] - z[a][2] - z[a][3];
+            int h = 2 * th + a;
+            if (h >= OH) continue;
+            for (int j = 0; j < 2; ++j) {
+                int w = 2 * tw + j;
+                if (w >= OW) continue;
+                int64_t off = (((int64_t)n * OH + h) * OW + w) * O + o;
+                float v = alpha * (j == 0 ? y0 : y1);
+                if (beta != 0.f) v += beta * to_f<T>(out[off]);
+                out[off] = from_f<T>(v);
+            }
+        }
+    }
+}
+
+template <class T>
+int im2col_t(const Geom& g, int32_t b, const void* x, void* col, int32_t kpitch, cudaStream_t st) {
+    constexpr int V = 16 / sizeof(T);
+    const int64_t rows = (int64_t)b * g.p * g.q;
+    const int RSC = g.r * g.s * g.c;
+    if (g.c % V == 0 && kpitch % V == 0) {
+        int grid = grid_for(rows * (kpitch / V), 256);
+        im2col_kernel<T, V><<<grid, 256, 0, st>>>((const T*)x, (T*)col, rows, g.h, g.w, g.c, g.p, g.q, g.s,
+                                                   g.pad, g.stride, RSC, kpitch);
+    } else {
+        int grid = grid_for(rows * kpitch, 256);
+        im2col_scalar_kernel<T><<<grid, 256, 0, st>>>((const T*)x, (T*)col, rows, g.h, g.w, g.c, g.p, g.q,
+                                                       g.s, g.pad, g.stride, RSC, kpitch);
+    }
+    return (int)cudaGetLastError();
+}
+
+}  // namespace
+
+int launch_im2col(const Geom& g, int32_t b, const void* x, void* col, int32_t kpitch, cudaStream_t st) {
+    return g.math == MUCU_MATH_BF16 ? im2col_t<__nv_bfloat16>(g, b, x, col, kpitch, st)
+                                    : im2col_t<float>(g, b, x, col, kpitch, st);
+}
+
+int launch_pad_filter(const Geom& g, const void* w, void* wpad, int32_t kpitch, cudaStream_t st) {
+    const int RSC = g.r * g.s * g.c;
+    int grid = grid_for((int64_t)g.k * kpitch, 256);
+    if (g.math == MUCU_MATH_BF16)
+        pad_filter_kernel<__nv_bfloat16><<<grid, 256, 0, st>>>((const __nv_bfloat16*)w, (__nv_bfloat16*)wpad, g.k, RSC, kpitch);
+    else
+        pad_filter_kernel<float><<<grid, 256, 0, st>>>((const float*)w, (float*)wpad, g.k, RSC, kpitch);
+    return (int)cudaGetLastError();
+}
+
+int launch_col2im(const Geom& g, int32_t b, float alpha, const float* dcol, int32_t kpitch, float beta,
+                  void* dx, cudaStream_t st) {
+    const int64_t total = (int64_t)b * g.h * g.w * g.c;
+    int grid = grid_for(total, 256);
+    if (g.math == MUCU_MATH_BF16)
+        col2im_kernel<__nv_bfloat16><<<grid, 256, 0, st>>>(dcol, (__nv_bfloat16*)dx, total, g.h, g.w, g.c, g.p, g.q,
+                                                          g.r, g.s, g.pad, g.stride, kpitch, alpha, beta);
+    else
+        col2im_kernel<float><<<grid, 256, 0, st>>>(dcol, (float*)dx, total, g.h, g.w, g.c, g.p, g.q, g.r, g.s,
+                                                  g.pad, g.stride, kpitch, alpha, beta);
+    return (int)cudaGetLastError();
+}
+
+int launch_wg_filter(const Geom& g, bool dgrad, const void* w, void* U, cudaStream_t st) {
+    const int O = dgrad ? g.c : g.k, I = dgrad ? g.k : g.c;
+    int grid = grid_for((int64_t)O * I, 256);
+    if (g.math == MUCU_MATH_BF16)
+        wg_filter_kernel<__nv_bfloat16><<<grid, 256, 0, st>>>((const __nv_bfloat16*)w, (__nv_bfloat16*)U, O, I, g.c, dgrad);
+    else
+        wg_filter_kernel<float><<<grid, 256, 0, st>>>((const float*)w, (float*)U, O, I, g.c, dgrad);
+    return (int)cudaGetLastError();
+}
+
+// Tile counts: FWD tiles cover the output P x Q; DGRAD tiles cover H x W.
+static inline void wg_dims(const Geom& g, bool dgrad, int* IH, int* IW, int* I, int* OH, int* OW, int* O,
+                           int* pad) {
+    if (!dgrad) { *IH = g.h; *IW = g.w; *I = g.c; *OH = g.p; *OW = g.q; *O = g.k; *pad = g.pad; }
+    else        { *IH = g.p; *IW = g.q; *I = g.k; *OH = g.h; *OW = g.w; *O = g.c; *pad = 2 - g.pad; }
+}
+
+int launch_wg_input(const Geom& g, bool dgrad, int32_t b, const void* in, void* V, cudaStream_t st) {
+    int IH, IW, I, OH, OW, O, pad;
+    wg_dims(g, dgrad, &IH, &IW, &I, &OH, &OW, &O, &pad);
+    const int TH = (OH + 1) / 2, TW = (OW + 1) / 2;
+    const int64_t tiles = (int64_t)b * TH * TW;
+    int grid = grid_for(tiles * I, 256);
+    if (g.math == MUCU_MATH_BF16)
+        wg_input_kernel<__nv_bfloat16><<<grid, 256, 0, st>>>((const __nv_bfloat16*)in, (__nv_bfloat16*)V, tiles, IH, IW, I, TH, TW, pad);
+    else
+        wg_input_kernel<float><<<grid, 256, 0, st>>>((const float*)in, (float*)V, tiles, IH, IW, I, TH, TW, pad);
+    return (int)cudaGetLastError();
+}
+
+int launch_wg_output(const Geom& g, bool dgrad, int32_t b, float alpha, const float* M, float beta, void* out,
+                     cudaStream_t st) {
+    int IH, IW, I, OH, OW, O, pad;
+    wg_dims(g, dgrad, &IH, &IW, &I, &OH, &OW, &O, &pad);
+    const int TH = (OH + 1) / 2, TW = (OW + 1) / 2;
+    const int64_t tiles = (int64_t)b * TH * TW;
+    int grid = grid_for(tiles * O, 256);
+    if (g.math == MUCU_MATH_BF16)
+        wg_output_kernel<__nv_bfloat16><<<grid, 256, 0, st>>>(M, (__nv_bfloat16*)out, tiles, OH, OW, O, TH, TW, alpha, beta);
+    else
+        wg_output_kernel<float><<<grid, 256, 0, st>>>(M, (float*)out, tiles, OH, OW, O, TH, TW, alpha, beta);
+    return (int)cudaGetLastError();
+}
+
+}  // namespace mucu

@@ -1,0 +1,355 @@
+// kernels_simt.cu -- fp32 CUDA-core (FFMA) path, MUCU_MATH_F32.
+//
+// Every convolution operation of every algorithm is expressed as a GEMM-shaped
+// contraction  C[i][j] = alpha * sum_kk A(i,kk) * B(j,kk) + beta * C[i][j]
+// whose operands are *views*: a dense matrix, the implicit im2col of x
+// (FWD / WGRAD, Alg. 1 loop order n,k,h,w | c,s,r), or the implicit
+// transposed-conv gather of dy (DGRAD).  One register-tiled SIMT kernel
+// (128x128x8 block tile, 8x8 per thread, double-buffered shared memory) runs
+// all of them; the fp32 path is FP32-ALU-bound (ridge ~11 flop/B), the
+// tensor-core paths live in kernels_tc.cu.
+//
+// Determinism: the reduction over kk is one sequential loop per output
+// element, so its order does not depend on the micro-batch size b (invariant I1
+// of SURVEY 8(c)).  BackwardFilter splits the pixel reduction over
+// CTAs and combines the partial tiles in split order through a per-tile turn
+// counter (no atomics on dw), so dw is deterministic too.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+
+#include "mucudnn_internal.h"
+
+namespace mucu {
+
+namespace {
+
+constexpr int kThreads = 256;
+
+// ------------------------------------------------------------------ views --
+// Dense matrix view: A(i,kk) = p[i*si + kk*sk] (zero outside rows x kdim).
+struct Dense {
+    const float* p;
+    int64_t rows, kdim, si, sk, batch_stride;
+    __device__ __forceinline__ float at(int64_t i, int64_t kk) const {
+        return (i < rows && kk < kdim) ? __ldg(p + i * si + kk * sk) : 0.f;
+    }
+    __device__ __forceinline__ void batch(int z) { p += z * batch_stride; }
+};
+
+// Implicit im2col of x (NHWC) for FWD: row i = output pixel (n,p,q), kk = (r,s,c).
+struct Im2col {
+    const float* x;
+    int64_t rows;
+    int H, W, C, P, Q, S, pad, st, RSC;
+    __device__ __forceinline__ float at(int64_t m, int64_t kk) const {
+        if (m >= rows || kk >= RSC) return 0.f;
+        int pq = P * Q;
+        int n = (int)(m / pq);
+        int rem = (int)(m - (int64_t)n * pq);
+        int p = rem / Q, q = rem - p * Q;
+        int k2 = (int)kk;
+        int rs = k2 / C, c = k2 - rs * C;
+        int r = rs / S, s = rs - r * S;
+        int h = p * st + r - pad, w = q * st + s - pad;
+        if (h < 0 || h >= H || w < 0 || w >= W) return 0.f;
+        return __ldg(x + (((int64_t)n * H + h) * W + w) * C + c);
+    }
+    __device__ __forceinline__ void batch(int) {}
+};
+
+// Im2col transposed for WGRAD's B operand: B(j, kk) = im2col(kk = pixel, j = (r,s,c)).
+struct Im2colT {
+    Im2col v;
+    __device__ __forceinline__ float at(int64_t j, int64_t m) const { return v.at(m, j); }
+    __device__ __forceinline__ void batch(int) {}
+};
+
+// DGRAD gather of dy: row i = dx pixel (n,h,w), kk = (r,s,k):
+// dy[n, (h+pad-r)/st, (w+pad-s)/st, k] when st divides and in range, else 0.
+struct DgradGather {
+    const float* dy;
+    int64_t rows;
+    int H, W, K, P, Q, S, pad, st, RSK;
+    __device__ __forceinline__ float at(int64_t m, int64_t kk) const {
+        if (m >= rows || kk >= RSK) return 0.f;
+        int hw = H * W;
+        int n = (int)(m / hw);
+        int rem = (int)(m - (int64_t)n * hw);
+        int h = rem / W, w = rem - h * W;
+        int k2 = (int)kk;
+        int rs = k2 / K, k = k2 - rs * K;
+        int r = rs / S, s = rs - r * S;
+        int ph = h + pad - r, pw = w + pad - s;
+        if (ph < 0 || pw < 0 || ph % st || pw % st) return 0.f;
+        int p = ph / st, q = pw / st;
+        if (p >= P || q >= Q) return 0.f;
+        return __ldg(dy + (((int64_t)n * P + p) * Q + q) * K + k);
+    }
+    __device__ __forceinline__ void batch(int) {}
+};
+
+// DGRAD filter view: B(j = c, kk = (r,s,k)) = w[k][r][s][c].
+struct DgradFilter {
+    const float* w;
+    int C, K, RS;
+    __device__ __forceinline__ float at(int64_t j, int64_t kk) const {
+        if (j >= C || kk >= (int64_t)RS * K) return 0.f;
+        int k2 = (int)kk;
+        int rs = k2 / K, k = k2 - rs * K;
+        return __ldg(w + ((int64_t)k * RS + rs) * C + j);
+    }
+    __device__ __forceinline__ void batch(int) {}
+};
+
+// -------------------------------------------------------------- epilogues --
+struct StoreDense {
+    float* c;
+    int64_t rows, cols, ldc, batch_stride;
+    float alpha, beta;
+    __device__ __forceinline__ void batch(int z) { c += z * batch_stride; }
+    template <int TN>
+    __device__ __forceinline__ void row(int64_t i, int64_t j0, const float (&v)[TN]) const {
+        if (i >= rows) return;
+        float* dst = c + i * ldc;
+#pragma unroll
+        for (int j = 0; j < TN; ++j) {
+            int64_t jj = j0 + j;
+            if (jj < cols) {
+                float o = alpha * v[j];
+                if (beta != 0.f) o += beta * dst[jj];
+                dst[jj] = o;
+            }
+        }
+    }
+};
+
+// ------------------------------------------------------------ the kernel --
+// CONTIG_A / CONTIG_B: true when consecutive kk are contiguous in memory
+// (threads of a warp then spread along kk), false when consecutive rows are.
+template <int BM, int BN, bool CONTIG_KA, bool CONTIG_KB, class AV, class BV>
+struct TileLoader {
+    static constexpr int BK = 8;
+    static constexpr int NA = BM * BK / kThreads;
+    static constexpr int NB = BN * BK / kThreads;
+    float ra[NA], rb[NB];
+
+    __device__ __forceinline__ static void a_coord(int e, int& il, int& kl) {
+        const int t = threadIdx.x;
+        if (CONTIG_KA) { kl = t % BK; il = t / BK + e * (kThreads / BK); }
+        else           { il = t % BM; kl = t / BM + e * (kThreads / BM); }
+    }
+    __device__ __forceinline__ static void b_coord(int e, int& jl, int& kl) {
+        const int t = threadIdx.x;
+        if (CONTIG_KB) { kl = t % BK; jl = t / BK + e * (kThreads / BK); }
+        else           { jl = t % BN; kl = t / BN + e * (kThreads / BN); }
+    }
+    __device__ __forceinline__ void load(const AV& a, const BV& b, int64_t m0, int64_t n0, int64_t k0, int64_t kend) {
+#pragma unroll
+        for (int e = 0; e < NA; ++e) {
+            int il, kl; a_coord(e, il, kl);
+            int64_t kk = k0 + kl;
+            ra[e] = kk < kend ? a.at(m0 + il, kk) : 0.f;
+        }
+#pragma unroll
+        for (int e = 0; e < NB; ++e) {
+            int jl, kl; b_coord(e, jl, kl);
+            int64_t kk = k0 + kl;
+            rb[e] = kk < kend ? b.at(n0 + jl, kk) : 0.f;
+        }
+    }
+    __device__ __forceinline__ void store(float (*As)[BM + 4], float (*Bs)[BN + 4]) const {
+#pragma unroll
+        for (int e = 0; e < NA; ++e) { int il, kl; a_coord(e, il, kl); As[kl][il] = ra[e]; }
+#pragma unroll
+        for (int e = 0; e < NB; ++e) { int jl, kl; b_coord(e, jl, kl); Bs[kl][jl] = rb[e]; }
+    }
+};
+
+// Main loop shared by all SIMT contractions: accumulates the BM x BN tile at
+// (m0, n0) over kk in [kbeg, kend).  acc[i][j] belongs to row ty*TM+i,
+// column tx*TN+j of the tile.
+template <int BM, int BN, bool CKA, bool CKB, class AV, class BV>
+__device__ __forceinline__ void simt_mainloop(const AV& a, const BV& b, int64_t m0, int64_t n0, int64_t kbeg,
+                                              int64_t kend, float (&acc)[BM / 16][BN / 16]) {
+    constexpr int BK = 8, TM = BM / 16, TN = BN / 16;
+    __shared__ __align__(16) float As[2][BK][BM + 4];
+    __shared__ __align__(16) float Bs[2][BK][BN + 4];
+    const int tx = threadIdx.x % 16, ty = threadIdx.x / 16;
+#pragma unroll
+    for (int i = 0; i < TM; ++i)
+#pragma unroll
+        for (int j = 0; j < TN; ++j) acc[i][j] = 0.f;
+    if (kbeg >= kend) return;
+    TileLoader<BM, BN, CKA, CKB, AV, BV> ld;
+    ld.load(a, b, m0, n0, kbeg, kend);
+    ld.store(As[0], Bs[0]);
+    __syncthreads();
+    int buf = 0;
+    for (int64_t k0 = kbeg; k0 < kend; k0 += BK) {
+        const bool more = k0 + BK < kend;
+        if (more) ld.load(a, b, m0, n0, k0 + BK, kend);
+#pragma unroll
+        for (int k = 0; k < BK; ++k) {
+            float af[TM], bf[TN];
+#pragma unroll
+            for (int i = 0; i < TM; i += 4) {
+                float4 v = *reinterpret_cast<const float4*>(&As[buf][k][ty * TM + i]);
+                af[i] = v.x; af[i + 1] = v.y; af[i + 2] = v.z; af[i + 3] = v.w;
+            }
+#pragma unroll
+            for (int j = 0; j < TN; j += 4) {
+                float4 v = *reinterpret_cast<const float4*>(&Bs[buf][k][tx * TN + j]);
+                bf[j] = v.x; bf[j + 1] = v.y; bf[j + 2] = v.z; bf[j + 3] = v.w;
+            }
+#pragma unroll
+            for (int i = 0; i < TM; ++i)
+#pragma unroll
+                for (int j = 0; j < TN; ++j) acc[i][j] = fmaf(af[i], bf[j], acc[i][j]);
+        }
+        if (more) ld.store(As[buf ^ 1], Bs[buf ^ 1]);
+        __syncthreads();
+        buf ^= 1;
+    }
+}
+
+template <int BM, int BN, bool CKA, bool CKB, class AV, class BV, class EPI>
+__global__ void __launch_bounds__(kThreads) simt_gemm_kernel(AV a, BV b, EPI epi, int64_t Kd) {
+    constexpr int TM = BM / 16, TN = BN / 16;
+    a.batch(blockIdx.z); b.batch(blockIdx.z); epi.batch(blockIdx.z);
+    const int64_t m0 = (int64_t)blockIdx.y * BM, n0 = (int64_t)blockIdx.x * BN;
+    float acc[TM][TN];
+    simt_mainloop<BM, BN, CKA, CKB>(a, b, m0, n0, 0, Kd, acc);
+    const int tx = threadIdx.x % 16, ty = threadIdx.x / 16;
+#pragma unroll
+    for (int i = 0; i < TM; ++i) epi.template row<TN>(m0 + ty * TM + i, n0 + tx * TN, acc[i]);
+}
+
+// WGRAD: dw[K][RSC] (+)= alpha * sum over the split's pixel range.  Splits of
+// one tile are combined in split order: split s waits until sem[tile] == s,
+// adds its partial (split 0 applies beta), publishes, and hands the turn to
+// s + 1 (the last split resets the counter to 0).  blockIdx.z = split, so all
+// CTAs of split s are dispatched before any of split s + 1 (no deadlock).
+template <int BM, int BN, class AV, class BV>
+__global__ void __launch_bounds__(kThreads) simt_wgrad_kernel(AV a, BV b, float* dw, int64_t rows, int64_t cols,
+                                                              int64_t Kd, int64_t k_per_split, float alpha,
+                                                              float beta, int32_t* sem) {
+    constexpr int TM = BM / 16, TN = BN / 16;
+    const int64_t m0 = (int64_t)blockIdx.y * BM, n0 = (int64_t)blockIdx.x * BN;
+    const int split = blockIdx.z, nsplit = gridDim.z;
+    const int64_t kb = (int64_t)split * k_per_split;
+    const int64_t ke = min(Kd, kb + k_per_split);
+    float acc[TM][TN];
+    simt_mainloop<BM, BN, false, false>(a, b, m0, n0, kb, ke, acc);
+    const int tile = blockIdx.y * gridDim.x + blockIdx.x;
+    if (threadIdx.x == 0 && split > 0) {
+        volatile int32_t* vs = sem + tile;
+        while (*vs != split) __nanosleep(64);
+        __threadfence();
+    }
+    __syncthreads();
+    const int tx = threadIdx.x % 16, ty = threadIdx.x / 16;
+#pragma unroll
+    for (int i = 0; i < TM; ++i) {
+        int64_t r = m0 + ty * TM + i;
+        if (r >= rows) continue;
+#pragma unroll
+        for (int j = 0; j < TN; ++j) {
+            int64_t cidx = n0 + tx * TN + j;
+            if (cidx >= cols) continue;
+            float* d = dw + r * cols + cidx;
+            float v = alpha * acc[i][j];
+            if (split > 0) v += *d;
+            else if (beta != 0.f) v += beta * *d;
+            *d = v;
+        }
+    }
+    __threadfence();
+    __syncthreads();
+    if (threadIdx.x == 0) atomicExch(sem + tile, split + 1 < nsplit ? split + 1 : 0);
+}
+
+template <int BM, int BN, bool CKA, bool CKB, class AV, class BV, class EPI>
+int launch_gemm(const AV& a, const BV& b, const EPI& e, int64_t M, int64_t N, int64_t Kd, int batch,
+                cudaStream_t st) {
+    dim3 grid((unsigned)ceil_div(N, BN), (unsigned)ceil_div(M, BM), (unsigned)batch);
+    simt_gemm_kernel<BM, BN, CKA, CKB><<<grid, kThreads, 0, st>>>(a, b, e, Kd);
+    return (int)cudaGetLastError();
+}
+
+// Tile shape by the GEMM's N extent (narrow N wastes less with BN = 64).
+template <bool CKA, bool CKB, class AV, class BV, class EPI>
+int dispatch_gemm(const AV& a, const BV& b, const EPI& e, int64_t M, int64_t N, int64_t Kd, int batch,
+                  cudaStream_t st) {
+    if (N <= 64) return launch_gemm<128, 64, CKA, CKB>(a, b, e, M, N, Kd, batch, st);
+    return launch_gemm<128, 128, CKA, CKB>(a, b, e, M, N, Kd, batch, st);
+}
+
+}  // namespace
+
+// FWD implicit GEMM (algorithm (a)): y[m][k] = sum_{(r,s,c)} im2col(x)[m][(r,s,c)] * w[k][(r,s,c)].
+int simt_fwd_ig(const Geom& g, int32_t b, float alpha, const float* x, const float* w, float beta, float* y,
+                cudaStream_t st) {
+    const int64_t M = (int64_t)b * g.p * g.q, N = g.k, Kd = (int64_t)g.r * g.s * g.c;
+    Im2col a{x, M, g.h, g.w, g.c, g.p, g.q, g.s, g.pad, g.stride, (int)Kd};
+    Dense bw{w, N, Kd, Kd, 1, 0};
+    StoreDense e{y, M, N, N, 0, alpha, beta};
+    return dispatch_gemm<true, true>(a, bw, e, M, N, Kd, 1, st);
+}
+
+// C[M,N] = alpha * A[M,K] * B[N,K]^T + beta * C, optional batch (strides in elements).
+int simt_gemm_nt(int64_t M, int64_t N, int64_t K, float alpha, const float* A, int64_t lda, const float* B,
+                 int64_t ldb, float beta, float* C, int64_t ldc, int batch, int64_t sA, int64_t sB, int64_t sC,
+                 cudaStream_t st) {
+    Dense a{A, M, K, lda, 1, sA};
+    Dense bb{B, N, K, ldb, 1, sB};
+    StoreDense e{C, M, N, ldc, sC, alpha, beta};
+    return dispatch_gemm<true, true>(a, bb, e, M, N, K, batch, st);
+}
+
+// C[M,N] = alpha * A[M,K] * B[K,N] + beta * C (B row-major, N contiguous).
+int simt_gemm_nn(int64_t M, int64_t N, int64_t K, float alpha, const float* A, int64_t lda, const float* B,
+                 int64_t ldb, float beta, float* C, int64_t ldc, cudaStream_t st) {
+    Dense a{A, M, K, lda, 1, 0};
+    Dense bb{B, N, K, 1, ldb, 0};
+    StoreDense e{C, M, N, ldc, 0, alpha, beta};
+    return dispatch_gemm<true, false>(a, bb, e, M, N, K, 1, st);
+}
+
+// DGRAD implicit GEMM: dx[m][c] = sum_{(r,s,k)} gather(dy)[m][(r,s,k)] * w[k][r][s][c].
+int simt_dgrad_ig(const Geom& g, int32_t b, float alpha, const float* dy, const float* w, float beta, float* dx,
+                  cudaStream_t st) {
+    const int64_t M = (int64_t)b * g.h * g.w, N = g.c, Kd = (int64_t)g.r * g.s * g.k;
+    DgradGather a{dy, M, g.h, g.w, g.k, g.p, g.q, g.s, g.pad, g.stride, (int)Kd};
+    DgradFilter bw{w, g.c, g.k, g.r * g.s};
+    StoreDense e{dx, M, N, N, 0, alpha, beta};
+    return dispatch_gemm<true, false>(a, bw, e, M, N, Kd, 1, st);
+}
+
+// WGRAD: dw[k][(r,s,c)] = sum_m dy[m][k] * B(m, (r,s,c)), B = implicit im2col
+// of x (IG) or the explicit col matrix (I2C, row pitch kpitch).
+int simt_wgrad(const Geom& g, int32_t b, float alpha, const float* dy, const float* xin, bool col_input,
+               int32_t kpitch, float beta, float* dw, const SemBuf& sem, int num_sms, cudaStream_t st) {
+    constexpr int BM = 128, BN = 128, BK = 8;
+    const int64_t rows = g.k, cols = (int64_t)g.r * g.s * g.c, Kd = (int64_t)b * g.p * g.q;
+    const int64_t tiles = ceil_div(cols, BN) * ceil_div(rows, BM);
+    if (tiles > sem.capacity) return (int)cudaErrorInvalidValue;
+    // Enough splits for ~2 waves of 2 CTAs/SM, each split >= 256 pixels.
+    int64_t want = std::max<int64_t>(1, (4LL * num_sms + tiles - 1) / tiles);
+    int64_t maxs = std::max<int64_t>(1, Kd / 256);
+    int64_t nsplit = std::min<int64_t>(std::min<int64_t>(want, maxs), 65535);
+    int64_t kps = ceil_div(ceil_div(Kd, nsplit), BK) * BK;
+    nsplit = ceil_div(Kd, kps);
+    dim3 grid((unsigned)ceil_div(cols, BN), (unsigned)ceil_div(rows, BM), (unsigned)nsplit);
+    Dense a{dy, rows, Kd, 1, g.k, 0};  // A(k, m) = dy[m][k]
+    if (col_input) {
+        Dense bb{xin, cols, Kd, 1, kpitch, 0};  // B(j, m) = col[m][j]
+        simt_wgrad_kernel<BM, BN><<<grid, kThreads, 0, st>>>(a, bb, dw, rows, cols, Kd, kps, alpha, beta, sem.sem);
+    } else {
+        Im2colT bb{Im2col{xin, Kd, g.h, g.w, g.c, g.p, g.q, g.s, g.pad, g.stride, (int)cols}};
+        simt_wgrad_kernel<BM, BN><<<grid, kThreads, 0, st>>>(a, bb, dw, rows, cols, Kd, kps, alpha, beta, sem.sem);
+    }
+    return (int)cudaGetLastError();
+}
+
+}  // namespace mucu

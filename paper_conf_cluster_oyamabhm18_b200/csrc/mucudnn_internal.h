@@ -1,0 +1,99 @@
+// mucudnn_internal.h -- shared declarations of the library's host runtime and
+// kernel launchers (not part of the public ABI; see include/mucudnn.h).
+#pragma once
+#include <cstdint>
+#include <cstddef>
+
+#include "mucudnn.h"
+
+#ifdef __CUDACC__
+#include <cuda_runtime.h>
+#else
+typedef struct CUstream_st* cudaStream_t;
+#endif
+
+namespace mucu {
+
+// Records a thread-local error message and returns `s` (printf-style).
+mucu_status_t set_error(mucu_status_t s, const char* fmt, ...);
+
+// Layer geometry with derived output extent (reading G1/G3).
+struct Geom {
+    int32_t n, c, h, w, k, r, s, pad, stride, p, q, math;
+};
+
+bool make_geom(const mucu_conv_desc_t* d, Geom* g);
+inline int elt_size(int math) { return math == MUCU_MATH_BF16 ? 2 : 4; }
+inline uint64_t align_up(uint64_t v, uint64_t a) { return (v + a - 1) / a * a; }
+inline int64_t ceil_div(int64_t a, int64_t b) { return (a + b - 1) / b; }
+
+// Algorithm eligibility (UNSUPPORTED reasons) -- shared by workspace sizing,
+// the benchmark pass and the executor.
+bool algo_eligible(const Geom& g, int type, int algo);
+bool is_pointwise(const Geom& g);  // 1x1, stride 1, pad 0: im2col(x) == x
+
+// Workspace layout of one micro-configuration (all offsets 256-B aligned).
+// `fixed` = b-independent prefix (padded filter / Winograd U) computed once per
+// call and shared by the call's micro-batches of the same algorithm.
+struct WsLayout {
+    uint64_t fixed_off, fixed_bytes;  // padded filter (I2C) or U (WG)
+    uint64_t a_off, a_bytes;          // col (I2C FWD/WGRAD), dcol (I2C DGRAD), V (WG)
+    uint64_t b_off, b_bytes;          // M (WG)
+    uint64_t total;
+    int32_t kpitch;                   // row pitch (elements) of col / padded filter / dcol
+    bool filter_padded;               // I2C: the filter row R*S*C is not 16-B aligned
+};
+mucu_status_t ws_layout(const Geom& g, int type, int algo, int32_t b, WsLayout* out);
+
+// Per-call executor state (which b-independent workspace prefix is valid).
+struct CallCtx {
+    int fixed_kind = 0;  // 0 none, 1 padded filter, 2 Winograd U
+    const void* fixed_src = nullptr;
+};
+
+struct Handle;
+// Run one micro-configuration on micro-batch b (pointers already offset).
+mucu_status_t run_micro(Handle* h, const Geom& g, int type, int algo, int32_t b, float alpha,
+                        const void* in0, const void* in1, float beta, void* out, void* ws,
+                        uint64_t ws_bytes, cudaStream_t st, CallCtx* ctx);
+
+// ---------------------------------------------------------------- kernels --
+// All launchers are asynchronous on `st` and return a CUDA error code (0 = ok).
+struct SemBuf {
+    int32_t* sem;      // device, zero-initialised, left zero by every kernel
+    int32_t capacity;  // number of ints
+};
+
+// SIMT fp32 GEMM-shaped convolution pieces (kernels_simt.cu).
+int simt_fwd_ig(const Geom& g, int32_t b, float alpha, const float* x, const float* w, float beta,
+                float* y, cudaStream_t st);
+int simt_gemm_nt(int64_t M, int64_t N, int64_t K, float alpha, const float* A, int64_t lda,
+                 const float* B, int64_t ldb, float beta, float* C, int64_t ldc, int batch,
+                 int64_t sA, int64_t sB, int64_t sC, cudaStream_t st);      // C = A[M,K] B[N,K]^T
+int simt_gemm_nn(int64_t M, int64_t N, int64_t K, float alpha, const float* A, int64_t lda,
+                 const float* B, int64_t ldb, float beta, float* C, int64_t ldc,
+                 cudaStream_t st);                                            // C = A[M,K] B[K,N]
+int simt_dgrad_ig(const Geom& g, int32_t b, float alpha, const float* dy, const float* w,
+                  float beta, float* dx, cudaStream_t st);
+int simt_wgrad(const Geom& g, int32_t b, float alpha, const float* dy, const float* x_or_col,
+               bool col_input, int32_t kpitch, float beta, float* dw, const SemBuf& sem,
+               int num_sms, cudaStream_t st);
+
+// Element-wise / data-movement kernels (kernels_elem.cu); T = float or bf16 by math.
+int launch_im2col(const Geom& g, int32_t b, const void* x, void* col, int32_t kpitch, cudaStream_t st);
+int launch_pad_filter(const Geom& g, const void* w, void* wpad, int32_t kpitch, cudaStream_t st);
+int launch_col2im(const Geom& g, int32_t b, float alpha, const float* dcol, int32_t kpitch, float beta,
+                  void* dx, cudaStream_t st);
+int launch_wg_filter(const Geom& g, bool dgrad, const void* w, void* U, cudaStream_t st);
+int launch_wg_input(const Geom& g, bool dgrad, int32_t b, const void* in, void* V, cudaStream_t st);
+int launch_wg_output(const Geom& g, bool dgrad, int32_t b, float alpha, const float* M, float beta,
+                     void* out, cudaStream_t st);
+
+// tcgen05 tensor-core path (kernels_tc.cu) for MUCU_MATH_TF32 / MUCU_MATH_BF16:
+// runs one micro-configuration; returns a cudaError_t, or -1 if this
+// (type, algo, geometry) has no tensor-core implementation.
+int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, const void* in0, const void* in1,
+                 float beta, void* out, char* ws, const WsLayout& L, const SemBuf& sem, int num_sms,
+                 cudaStream_t st, CallCtx* ctx);
+
+}  // namespace mucu

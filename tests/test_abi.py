@@ -1,0 +1,92 @@
+"""The C-ABI library loads on a CPU-only host and exports every function
+include/mucudnn.h declares; host-only entry points behave as documented.
+No compute (GPU) calls here."""
+import ctypes
+import os
+import re
+
+import pytest
+
+import paper_conf_cluster_oyamabhm18_b200 as mu
+from paper_conf_cluster_oyamabhm18_b200 import _lib
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+HEADER = os.path.join(ROOT, "include", "mucudnn.h")
+
+
+def declared_functions():
+    src = open(HEADER).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    return sorted(set(re.findall(r"\b(mucu_[a-z_0-9]+)\s*\(", src)))
+
+
+def test_header_declares_the_boundary():
+    fns = declared_functions()
+    for name in ["mucu_create", "mucu_benchmark", "mucu_plan_wr", "mucu_pareto_front", "mucu_solve_wd",
+                 "mucu_conv_forward", "mucu_conv_backward_data", "mucu_conv_backward_filter",
+                 "mucu_network_plan", "mucu_workspace_size"]:
+        assert name in fns
+
+
+def test_library_exports_every_declared_symbol():
+    lib = ctypes.CDLL(_lib._LIB_PATH)
+    missing = [f for f in declared_functions() if not hasattr(lib, f)]
+    assert not missing, missing
+
+
+def test_status_strings_and_version():
+    assert mu.version() == 100
+    for i, name in enumerate(_lib.STATUS):
+        assert _lib.status_string(i) == name
+
+
+def test_output_dims_and_invalid_descriptor():
+    assert mu.output_dims(mu.desc(8, 64, 27, 27, 192, 5, 5, 2, 1)) == (27, 27)
+    assert mu.output_dims(mu.desc(1, 3, 224, 224, 64, 11, 11, 2, 4)) == (55, 55)
+    assert mu.output_dims(mu.desc(1, 3, 224, 224, 64, 7, 7, 3, 2)) == (112, 112)
+    with pytest.raises(mu.MucuError) as e:
+        mu.output_dims(mu.desc(1, 3, 2, 2, 4, 5, 5, 0, 1))
+    assert e.value.status == 1
+
+
+# Closed-form workspace sizes (header comment of mucu_workspace_size).
+def test_workspace_im2col_alexnet_conv2_cfg1():
+    d = mu.desc(8, 64, 27, 27, 192, 5, 5, 2, 1, mu.MATH_F32)
+    assert mu.workspace_size(d, mu.FWD, mu.IMPLICIT_GEMM, 8) == 0
+    assert mu.workspace_size(d, mu.FWD, mu.IM2COL_GEMM, 1) == 4_665_600   # 729 * 1600 * 4
+    assert mu.workspace_size(d, mu.FWD, mu.IM2COL_GEMM, 2) == 9_331_200   # > 8 MiB: b = 1 only
+    with pytest.raises(mu.MucuError) as e:
+        mu.workspace_size(d, mu.FWD, mu.WINOGRAD, 1)                       # 5x5: ineligible
+    assert e.value.status == 2
+
+
+def test_workspace_winograd_alexnet_conv3():
+    d = mu.desc(256, 192, 13, 13, 384, 3, 3, 1, 1, mu.MATH_F32)
+    U = 16 * 384 * 192 * 4
+    per_sample = 16 * 49 * 192 * 4 + 16 * 49 * 384 * 4                    # V + M = 1,806,336
+    assert per_sample == 1_806_336
+    assert mu.workspace_size(d, mu.FWD, mu.WINOGRAD, 1) == U + per_sample
+    assert mu.workspace_size(d, mu.FWD, mu.WINOGRAD, 10) == U + 10 * per_sample
+    with pytest.raises(mu.MucuError):
+        mu.workspace_size(d, mu.BWD_FILTER, mu.WINOGRAD, 1)                 # NEXT-1
+
+
+def test_workspace_bf16_resnet_and_pointwise():
+    d = mu.desc(256, 64, 56, 56, 64, 3, 3, 1, 1, mu.MATH_BF16)
+    assert mu.workspace_size(d, mu.FWD, mu.IM2COL_GEMM, 1) == 3_612_672   # 3136 * 576 * 2
+    # WG bf16: V bf16 + M fp32 per sample = 4,816,896 (SURVEY ResNet-18 layer1 row)
+    U = 16 * 64 * 64 * 2
+    assert mu.workspace_size(d, mu.FWD, mu.WINOGRAD, 1) - U == 4_816_896
+    p = mu.desc(256, 256, 56, 56, 64, 1, 1, 0, 1, mu.MATH_BF16)
+    for t in (mu.FWD, mu.BWD_DATA, mu.BWD_FILTER):
+        assert mu.workspace_size(p, t, mu.IM2COL_GEMM, 256) == 0          # im2col(x) == x
+    ds = mu.desc(256, 256, 56, 56, 512, 1, 1, 0, 2, mu.MATH_BF16)
+    assert mu.workspace_size(ds, mu.FWD, mu.IM2COL_GEMM, 1) == 401_408    # 784 * 256 * 2
+
+
+def test_workspace_unaligned_filter_row():
+    d = mu.desc(4, 3, 224, 224, 64, 7, 7, 3, 2, mu.MATH_BF16)              # RSC = 147
+    kp = 152                                                               # ceil to 8 bf16
+    col = 112 * 112 * kp * 2
+    filt = -(-64 * kp * 2 // 256) * 256
+    assert mu.workspace_size(d, mu.FWD, mu.IM2COL_GEMM, 1) == filt + -(-col // 256) * 256

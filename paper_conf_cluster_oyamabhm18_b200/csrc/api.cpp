@@ -408,14 +408,13 @@ static ScratchLayout scratch_layout(const Geom& g, int type, uint64_t ws_limit) 
     const uint64_t Wt = align_up((uint64_t)g.k * g.r * g.s * g.c * elt, 256);
     const uint64_t DW = align_up((uint64_t)g.k * g.r * g.s * g.c * 4, 256);
     // Largest workspace any benchmarked micro-config may use.
+    // ws grows with b, so min(ws(N), limit) bounds every b that fits the limit.
     uint64_t need = 0;
-    for (int a = 0; a < MUCU_NUM_ALGOS; ++a)
-        for (int32_t b : {1, g.n}) {
-            WsLayout L;
-            if (ws_layout(g, type, a, b, &L) == MUCU_OK && L.total <= ws_limit) need = std::max(need, L.total);
-        }
-    // ws grows with b, so size at N bounds every b that fits the limit.
-    need = std::min<uint64_t>(align_up(need, 256), align_up(ws_limit, 256));
+    for (int a = 0; a < MUCU_NUM_ALGOS; ++a) {
+        WsLayout L;
+        if (ws_layout(g, type, a, g.n, &L) == MUCU_OK) need = std::max(need, std::min(L.total, ws_limit));
+    }
+    need = align_up(need, 256);
     ScratchLayout s;
     s.in0 = 0;
     if (type == MUCU_FWD) { s.in1 = X; s.out = X + Wt; s.ws = X + Wt + Y; }

@@ -1,9 +1,887 @@
-// kernels_tc.cu -- tcgen05 tensor-core path (placeholder until the sm_100a kernels land).
+// kernels_tc.cu -- tcgen05 tensor-core conv-GEMM for sm_100a (MUCU_MATH_TF32 /
+// MUCU_MATH_BF16): the contraction step of all three algorithms.
+//
+//   (a) implicit GEMM (zero workspace): the im2col / transposed-conv operand is
+//       gathered on the fly from NHWC activations with cp.async into the
+//       128-byte-swizzled shared-memory layout the UMMA descriptors expect;
+//   (b) im2col + GEMM: both operands dense, loaded with TMA;
+//   (c) Winograd: 16 independent GEMMs M_xi = V_xi U_xi^T (batched over
+//       blockIdx.z), TMA-loaded.
+//
+// One CTA computes a 128 x BN output tile; the fp32 accumulator lives in TMEM
+// (BN columns).  Warp roles (256 threads):
+//   warps 0-3  producers: one thread issues TMA, all 128 threads gather (cp.async)
+//   warp  4    TMEM allocator + single-thread tcgen05.mma issuer
+//   warps 4-7  epilogue: tcgen05.ld 32x32b -> registers -> alpha/beta -> global
+// Shared memory is a STAGES-deep ring of {A tile, B tile} guarded by
+// full/empty mbarriers; tcgen05.commit releases a stage when its MMAs retire.
+//
+// Operand layouts (K = reduction):
+//   K-major:  rows x 128 B (64 bf16 / 32 fp32 of K), SWIZZLE_128B atoms of 8 rows
+//   MN-major: (MN/64 bf16 | MN/32 fp32) atoms, each KB rows x 128 B, SWIZZLE_128B
+// KB = 128 B / element size of K per stage; 4 MMAs (UMMA_K = 32 B) per stage.
+//
+// Backward-filter splits the pixel reduction over blockIdx.z and
+// combines the partial tiles in split order through per-tile turn counters
+// (deterministic; split 0 applies the user's beta).
+#include <cuda.h>
+#include <cuda_bf16.h>
 #include <cuda_runtime.h>
+
+#include <cstdio>
+#include <cstring>
+#include <mutex>
+
 #include "mucudnn_internal.h"
+
 namespace mucu {
-int tc_run_micro(const Geom&, int, int, int32_t, float, const void*, const void*, float, void*, char*,
-                 const WsLayout&, const SemBuf&, int, cudaStream_t, CallCtx*) {
+
+namespace {
+
+// ------------------------------------------------------------ PTX helpers --
+__device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+
+__device__ __forceinline__ void mbar_init(uint32_t bar, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(bar), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint32_t bar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(bar) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_tx(uint32_t bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "WAIT_%=:\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+        "@!p bra WAIT_%=;\n\t}" ::"r"(bar),
+        "r"(parity)
+        : "memory");
+}
+__device__ __forceinline__ void tma_load_2d(uint32_t dst, const CUtensorMap* tm, uint32_t bar, int c0, int c1) {
+    asm volatile(
+        "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4}], [%2];" ::"r"(dst),
+        "l"((uint64_t)tm), "r"(bar), "r"(c0), "r"(c1)
+        : "memory");
+}
+__device__ __forceinline__ void tma_load_3d(uint32_t dst, const CUtensorMap* tm, uint32_t bar, int c0, int c1, int c2) {
+    asm volatile(
+        "cp.async.bulk.tensor.3d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4, %5}], [%2];" ::"r"(dst),
+        "l"((uint64_t)tm), "r"(bar), "r"(c0), "r"(c1), "r"(c2)
+        : "memory");
+}
+__device__ __forceinline__ void cp_async16(uint32_t dst, const void* src, bool valid) {
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(dst), "l"(src), "r"(valid ? 16 : 0) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
+__device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
+__device__ __forceinline__ void tc_fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
+__device__ __forceinline__ void tc_fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
+
+// Shared-memory matrix descriptor (sm_100 version 1).  layout: 2 = SWIZZLE_128B
+// (16-B chunks XOR row%8), 1 = SWIZZLE_128B_BASE32B (32-B chunks XOR row%4; the
+// only MN-major layout for 32-bit tf32 operands).
+__device__ __forceinline__ uint64_t sdesc(uint32_t saddr, uint32_t lbo, uint32_t sbo, uint32_t layout = 2) {
+    return (uint64_t)((saddr & 0x3FFFFu) >> 4) | ((uint64_t)((lbo >> 4) & 0x3FFFu) << 16) |
+           ((uint64_t)((sbo >> 4) & 0x3FFFu) << 32) | (1ull << 46) | ((uint64_t)layout << 61);
+}
+
+template <int ELT>
+__device__ __forceinline__ void mma(uint32_t tmem, uint64_t ad, uint64_t bd, uint32_t idesc, uint32_t acc) {
+    if constexpr (ELT == 2) {
+        asm volatile(
+            "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+            "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem),
+            "l"(ad), "l"(bd), "r"(idesc), "r"(acc));
+    } else {
+        asm volatile(
+            "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+            "tcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem),
+            "l"(ad), "l"(bd), "r"(idesc), "r"(acc));
+    }
+}
+__device__ __forceinline__ void mma_commit(uint32_t bar) {
+    asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(bar) : "memory");
+}
+
+#define TMEM_LD32(taddr, v)                                                                                      \
+    asm volatile(                                                                                                \
+        "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16,%17," \
+        "%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"                                       \
+        : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]),         \
+          "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]), "=r"(v[15]),   \
+          "=r"(v[16]), "=r"(v[17]), "=r"(v[18]), "=r"(v[19]), "=r"(v[20]), "=r"(v[21]), "=r"(v[22]), "=r"(v[23]), \
+          "=r"(v[24]), "=r"(v[25]), "=r"(v[26]), "=r"(v[27]), "=r"(v[28]), "=r"(v[29]), "=r"(v[30]), "=r"(v[31])  \
+        : "r"(taddr))
+
+// ----------------------------------------------------------- parameters --
+enum AMode : int {
+    A_TMA_K2 = 0,      // dense K-major, 2-D map {K, rows}
+    A_TMA_K3 = 1,      // dense K-major, batched 3-D map {K, rows, batch}
+    A_TMA_MN2 = 2,     // dense MN-major, 2-D map {rows(MN), K}
+    A_GATHER_FWD = 3,  // implicit im2col of x, K-major, 16-B vectors (C % KB == 0)
+    A_GATHER_DGRAD = 4,// transposed-conv gather of dy, K-major, 16-B vectors (K % KB == 0)
+    A_SCALAR_FWD = 5,  // implicit im2col of x, element-wise (any C)
+    A_SCALAR_DGRAD = 6,// transposed-conv gather of dy, element-wise (any K)
+};
+enum BMode : int {
+    B_TMA_K2 = 0,      // dense K-major {K, cols}
+    B_TMA_K3 = 1,      // batched K-major {K, cols, batch}
+    B_TMA_MN2 = 2,     // dense MN-major {cols(MN), K}
+    B_TMA_MN3 = 3,     // DGRAD filter view {C, R*S, K}: B(c, (r,s,k)) = w[k][r][s][c]
+    B_GATHER_WG = 4,   // WGRAD implicit im2col of x, MN-major, 16-B vectors (C % atom == 0)
+    B_SCALAR_K = 5,    // dense K-major rows with unaligned pitch, element-wise
+    B_SCALAR_DGRAD = 6,// DGRAD filter view, element-wise (any C)
+    B_SCALAR_WG = 7,   // WGRAD implicit im2col, element-wise (any C)
+};
+enum EpiMode : int { EPI_STORE = 0, EPI_WGRAD_CHAIN = 1 };
+
+struct TcArgs {
+    int M, N;                // output rows / cols
+    int num_kb;              // k-blocks of the whole reduction
+    int kb_per_split;        // WGRAD: k-blocks per blockIdx.z split
+    int BN;                  // tile N (multiple of 16, <= 256)
+    int stages;
+    int tmem_cols;
+    int bn_atoms;            // MN-major B atoms per stage = BN * ELT / 128
+    int tma_bytes;           // bytes the TMA loads of one stage deliver
+    int b_bytes;             // shared-memory bytes of one B stage
+    int kred;                // reduction length (elements) for scalar gathers
+    // gather geometry (x for FWD/WGRAD, dy for DGRAD)
+    const void* gsrc;
+    int H, W, C, P, Q, R, S, pad, stride, K;
+    // scalar B source
+    const void* bsrc;
+    int ldb;
+    // epilogue
+    void* out;
+    long long ldc;
+    long long batch_stride;  // elements
+    float alpha, beta;
+    int out_bf16;
+    int32_t* sem;
+};
+
+constexpr int kThreads = 256;
+
+template <int ELT>
+struct Elt;
+template <>
+struct Elt<2> { using T = __nv_bfloat16; static constexpr uint32_t fmt = 1; };
+template <>
+struct Elt<4> { using T = float; static constexpr uint32_t fmt = 2; };
+
+// Byte offset of element (row, kbyte) inside a K-major SW128 tile.
+__device__ __forceinline__ uint32_t kmaj_off(int row, int kbyte) {
+    return (uint32_t)((row >> 3) * 1024 + (row & 7) * 128 + ((((kbyte >> 4) ^ (row & 7)) & 7) << 4) + (kbyte & 15));
+}
+// Byte offset of byte `byte` (0..127) of k-row `krow` inside one MN-major atom
+// column: 16-bit types use SWIZZLE_128B (16-B chunk ^ krow%8), 32-bit types
+// SWIZZLE_128B_BASE32B (32-B chunk ^ krow%4).
+template <int ELT>
+__device__ __forceinline__ uint32_t mn_row_off(int krow, int byte) {
+    if constexpr (ELT == 2)
+        return (uint32_t)(krow * 128 + ((((byte >> 4) ^ (krow & 7)) & 7) << 4) + (byte & 15));
+    else
+        return (uint32_t)(krow * 128 + ((((byte >> 5) ^ (krow & 3)) & 3) << 5) + (byte & 31));
+}
+// Byte offset of element (mn, krow) inside an MN-major tile with KB rows per atom.
+template <int ELT>
+__device__ __forceinline__ uint32_t mnmaj_off(int mn, int krow, int kb_rows) {
+    constexpr int per_atom = 128 / ELT;
+    const int atom = mn / per_atom;
+    return (uint32_t)(atom * kb_rows * 128) + mn_row_off<ELT>(krow, (mn - atom * per_atom) * ELT);
+}
+
+template <class T>
+__device__ __forceinline__ void st_shared_elt(uint32_t addr, T v);
+template <>
+__device__ __forceinline__ void st_shared_elt<__nv_bfloat16>(uint32_t addr, __nv_bfloat16 v) {
+    unsigned short u = *reinterpret_cast<unsigned short*>(&v);
+    asm volatile("st.shared.u16 [%0], %1;" ::"r"(addr), "h"(u) : "memory");
+}
+template <>
+__device__ __forceinline__ void st_shared_elt<float>(uint32_t addr, float v) {
+    asm volatile("st.shared.f32 [%0], %1;" ::"r"(addr), "f"(v) : "memory");
+}
+
+// ------------------------------------------------------------ the kernel --
+template <int ELT, int AM, int BM_, int EPI>
+__global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constant__ TcArgs p,
+                                                            const __grid_constant__ CUtensorMap tmA,
+                                                            const __grid_constant__ CUtensorMap tmB) {
+    using T = typename Elt<ELT>::T;
+    constexpr int KB = 128 / ELT;            // K elements per stage
+    constexpr int UMMA_K = 32 / ELT;         // K elements per MMA
+    constexpr int A_BYTES = 128 * 128;       // 128 rows x 128 B
+    constexpr bool A_MN = (AM == A_TMA_MN2);
+    constexpr bool B_MN = (BM_ == B_TMA_MN2 || BM_ == B_TMA_MN3 || BM_ == B_GATHER_WG || BM_ == B_SCALAR_DGRAD ||
+                           BM_ == B_SCALAR_WG);
+    constexpr bool A_TMA = (AM == A_TMA_K2 || AM == A_TMA_K3 || AM == A_TMA_MN2);
+    constexpr bool B_TMA = (BM_ == B_TMA_K2 || BM_ == B_TMA_K3 || BM_ == B_TMA_MN2 || BM_ == B_TMA_MN3);
+    constexpr bool GATHER = !A_TMA || !B_TMA;
+    constexpr bool A_ASYNC = (AM == A_GATHER_FWD || AM == A_GATHER_DGRAD);
+    constexpr bool B_ASYNC = (BM_ == B_GATHER_WG);
+    // MN-major atoms: 8-row (bf16, SWIZZLE_128B) or 4-row (tf32, 128B_BASE32B) groups.
+    constexpr uint32_t MN_SBO = ELT == 2 ? 1024u : 512u;
+    constexpr uint32_t MN_LAYOUT = ELT == 2 ? 2u : 1u;
+
+    extern __shared__ uint8_t smem_raw[];
+    uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+    const int S = p.stages;
+    const int B_BYTES = p.b_bytes;
+    uint8_t* sA = smem;
+    uint8_t* sB = smem + (size_t)S * A_BYTES;
+    uint64_t* bars = (uint64_t*)(sB + (size_t)S * B_BYTES);
+    uint64_t* full = bars;
+    uint64_t* empty = bars + S;
+    uint64_t* accum = bars + 2 * S;
+    uint32_t* tmem_slot = (uint32_t*)(bars + 2 * S + 1);
+
+    const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
+    const int m0 = blockIdx.y * 128;
+    const int n0 = blockIdx.x * p.BN;
+    const int z = blockIdx.z;
+    int kb_begin = 0, kb_end = p.num_kb;
+    if (EPI == EPI_WGRAD_CHAIN) {
+        kb_begin = z * p.kb_per_split;
+        kb_end = min(p.num_kb, kb_begin + p.kb_per_split);
+    }
+    const int nkb = kb_end - kb_begin;
+
+    if (threadIdx.x == 0) {
+        const uint32_t full_count = (GATHER ? 128u : 0u) + (A_TMA || B_TMA ? 1u : 0u);
+        for (int s = 0; s < S; ++s) {
+            mbar_init(smem_u32(&full[s]), full_count);
+            mbar_init(smem_u32(&empty[s]), 1);
+        }
+        mbar_init(smem_u32(accum), 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    if (warp == 4) {
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
+                     "r"(p.tmem_cols));
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+    }
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    const uint32_t tmem = *tmem_slot;
+
+    if (warp < 4) {
+        // =========================== producers ===========================
+        const int t = threadIdx.x;  // 0..127
+        // Per-thread gather rows (A gathers: rows t/8 + 16 i, chunk t % 8).
+        int rn[8], rh[8], rw[8];
+        bool rv[8];
+        if constexpr (AM == A_GATHER_FWD || AM == A_GATHER_DGRAD) {
+#pragma unroll
+            for (int i = 0; i < 8; ++i) {
+                const int m = m0 + t / 8 + 16 * i;
+                rv[i] = m < p.M;
+                const int mm = rv[i] ? m : 0;
+                if (AM == A_GATHER_FWD) {  // output pixel (n,p,q) -> input origin
+                    const int pq = p.P * p.Q;
+                    const int n = mm / pq, rem = mm - n * pq, pp = rem / p.Q, qq = rem - pp * p.Q;
+                    rn[i] = n; rh[i] = pp * p.stride - p.pad; rw[i] = qq * p.stride - p.pad;
+                } else {  // dx pixel (n,h,w)
+                    const int hw = p.H * p.W;
+                    const int n = mm / hw, rem = mm - n * hw, hh = rem / p.W, ww = rem - hh * p.W;
+                    rn[i] = n; rh[i] = hh + p.pad; rw[i] = ww + p.pad;
+                }
+            }
+        }
+        const T* gx = (const T*)p.gsrc;
+        for (int it = 0; it < nkb; ++it) {
+            const int kb = kb_begin + it;
+            const int s = it % S;
+            const uint32_t ph = (uint32_t)(it / S) & 1u;
+            mbar_wait(smem_u32(&empty[s]), ph ^ 1u);
+            const uint32_t aT = smem_u32(sA + (size_t)s * A_BYTES);
+            const uint32_t bT = smem_u32(sB + (size_t)s * B_BYTES);
+            const uint32_t fb = smem_u32(&full[s]);
+            if ((A_TMA || B_TMA) && t == 0) {
+                mbar_arrive_tx(fb, (uint32_t)p.tma_bytes);
+                if constexpr (AM == A_TMA_K2) tma_load_2d(aT, &tmA, fb, kb * KB, m0);
+                if constexpr (AM == A_TMA_K3) tma_load_3d(aT, &tmA, fb, kb * KB, m0, z);
+                if constexpr (AM == A_TMA_MN2) {
+                    tma_load_2d(aT, &tmA, fb, m0, kb * KB);
+                    tma_load_2d(aT + KB * 128, &tmA, fb, m0 + 128 / ELT, kb * KB);
+                    if constexpr (ELT == 4) {
+                        tma_load_2d(aT + 2 * KB * 128, &tmA, fb, m0 + 2 * (128 / ELT), kb * KB);
+                        tma_load_2d(aT + 3 * KB * 128, &tmA, fb, m0 + 3 * (128 / ELT), kb * KB);
+                    }
+                }
+                if constexpr (BM_ == B_TMA_K2) tma_load_2d(bT, &tmB, fb, kb * KB, n0);
+                if constexpr (BM_ == B_TMA_K3) tma_load_3d(bT, &tmB, fb, kb * KB, n0, z);
+                if constexpr (BM_ == B_TMA_MN2) {
+                    for (int a = 0; a < p.bn_atoms; ++a)
+                        tma_load_2d(bT + a * KB * 128, &tmB, fb, n0 + a * (128 / ELT), kb * KB);
+                }
+                if constexpr (BM_ == B_TMA_MN3) {
+                    // k-block kb covers (r,s) = kb / (K/KB), k0 = (kb % (K/KB)) * KB
+                    const int kpr = p.K / KB;
+                    const int rs = kb / kpr, k0 = (kb - rs * kpr) * KB;
+                    for (int a = 0; a < p.bn_atoms; ++a)
+                        tma_load_3d(bT + a * KB * 128, &tmB, fb, n0 + a * (128 / ELT), rs, k0);
+                }
+            }
+            // ---- A gathers ----
+            if constexpr (AM == A_GATHER_FWD) {
+                const int kk0 = kb * KB;
+                const int rs = kk0 / p.C, c0 = kk0 - rs * p.C + (t & 7) * (16 / ELT);
+                const int r = rs / p.S, sx = rs - r * p.S;
+                const bool kin = rs < p.R * p.S;
+#pragma unroll
+                for (int i = 0; i < 8; ++i) {
+                    const int row = t / 8 + 16 * i;
+                    const int h = rh[i] + r, w = rw[i] + sx;
+                    const bool v = kin && rv[i] && h >= 0 && h < p.H && w >= 0 && w < p.W;
+                    const T* src = v ? gx + (((size_t)rn[i] * p.H + h) * p.W + w) * p.C + c0 : gx;
+                    cp_async16(aT + kmaj_off(row, (t & 7) * 16), src, v);
+                }
+            } else if constexpr (AM == A_GATHER_DGRAD) {
+                const int kk0 = kb * KB;
+                const int rs = kk0 / p.K, k0 = kk0 - rs * p.K + (t & 7) * (16 / ELT);
+                const int r = rs / p.S, sx = rs - r * p.S;
+                const bool kin = rs < p.R * p.S;
+#pragma unroll
+                for (int i = 0; i < 8; ++i) {
+                    const int row = t / 8 + 16 * i;
+                    const int ph_ = rh[i] - r, pw_ = rw[i] - sx;
+                    bool v = kin && rv[i] && ph_ >= 0 && pw_ >= 0;
+                    int pp = 0, qq = 0;
+                    if (v) {
+                        pp = ph_ / p.stride; qq = pw_ / p.stride;
+                        v = (pp * p.stride == ph_) && (qq * p.stride == pw_) && pp < p.P && qq < p.Q;
+                    }
+                    const T* src = v ? gx + (((size_t)rn[i] * p.P + pp) * p.Q + qq) * p.K + k0 : gx;
+                    cp_async16(aT + kmaj_off(row, (t & 7) * 16), src, v);
+                }
+            } else if constexpr (AM == A_SCALAR_FWD) {
+                // thread t owns row t; KB elements, kk = (r,s,c) decomposed each
+                const int m = m0 + t;
+                const bool rvalid = m < p.M;
+                const int pq = p.P * p.Q;
+                const int mm = rvalid ? m : 0;
+                const int n = mm / pq, rem = mm - n * pq, pp = rem / p.Q, qq = rem - pp * p.Q;
+                for (int e = 0; e < KB; ++e) {
+                    const int kk = kb * KB + e;
+                    float v = 0.f;
+                    if (rvalid && kk < p.kred) {
+                        const int rs = kk / p.C, c = kk - rs * p.C, r = rs / p.S, sx = rs - r * p.S;
+                        const int h = pp * p.stride - p.pad + r, w = qq * p.stride - p.pad + sx;
+                        if (h >= 0 && h < p.H && w >= 0 && w < p.W)
+                            v = (float)gx[(((size_t)n * p.H + h) * p.W + w) * p.C + c];
+                    }
+                    st_shared_elt<T>(aT + kmaj_off(t, e * ELT), (T)v);
+                }
+            } else if constexpr (AM == A_SCALAR_DGRAD) {
+                // thread t owns dx pixel row t; kk = (r,s,k) decomposed per element
+                const int m = m0 + t;
+                const bool rvalid = m < p.M;
+                const int hw = p.H * p.W;
+                const int mm = rvalid ? m : 0;
+                const int n = mm / hw, rem = mm - n * hw, hh = rem / p.W, ww = rem - hh * p.W;
+                for (int e = 0; e < KB; ++e) {
+                    const int kk = kb * KB + e;
+                    float v = 0.f;
+                    if (rvalid && kk < p.kred) {
+                        const int rs = kk / p.K, k = kk - rs * p.K, r = rs / p.S, sx = rs - r * p.S;
+                        const int ph_ = hh + p.pad - r, pw_ = ww + p.pad - sx;
+                        if (ph_ >= 0 && pw_ >= 0 && ph_ % p.stride == 0 && pw_ % p.stride == 0) {
+                            const int pp = ph_ / p.stride, qq = pw_ / p.stride;
+                            if (pp < p.P && qq < p.Q) v = (float)gx[(((size_t)n * p.P + pp) * p.Q + qq) * p.K + k];
+                        }
+                    }
+                    st_shared_elt<T>(aT + kmaj_off(t, e * ELT), (T)v);
+                }
+            }
+            // ---- B gathers ----
+            if constexpr (BM_ == B_GATHER_WG) {
+                // KB pixel rows x bn_atoms atoms x 8 chunks; thread: chunk t%8, rows t/8 + 16 i
+                const int chunk = t & 7;
+                for (int i = 0; i < KB / 16; ++i) {
+                    const int row = t / 8 + 16 * i;
+                    const int m = kb * KB + row;
+                    const int pq = p.P * p.Q;
+                    const bool mv = m < p.kred;
+                    const int mm = mv ? m : 0;
+                    const int n = mm / pq, rem = mm - n * pq, pp = rem / p.Q, qq = rem - pp * p.Q;
+                    for (int a = 0; a < p.bn_atoms; ++a) {
+                        const int j0 = n0 + a * (128 / ELT);
+                        const int rs = j0 / p.C, c0 = j0 - rs * p.C + chunk * (16 / ELT);
+                        const int r = rs / p.S, sx = rs - r * p.S;
+                        const int h = pp * p.stride - p.pad + r, w = qq * p.stride - p.pad + sx;
+                        const bool v = mv && rs < p.R * p.S && h >= 0 && h < p.H && w >= 0 && w < p.W;
+                        const T* src = v ? gx + (((size_t)n * p.H + h) * p.W + w) * p.C + c0 : gx;
+                        cp_async16(bT + (uint32_t)(a * KB * 128) + mn_row_off<ELT>(row, chunk * 16), src, v);
+                    }
+                }
+            } else if constexpr (BM_ == B_SCALAR_K) {
+                // B rows n0.. (BN of them) x KB elements from a dense row-major matrix with pitch ldb
+                const T* bs = (const T*)p.bsrc;
+                for (int idx = t; idx < p.BN * KB; idx += 128) {
+                    const int row = idx / KB, e = idx - (idx / KB) * KB;
+                    const int j = n0 + row, kk = kb * KB + e;
+                    const float v = (j < p.N && kk < p.kred) ? (float)bs[(size_t)j * p.ldb + kk] : 0.f;
+                    st_shared_elt<T>(bT + kmaj_off(row, e * ELT), (T)v);
+                }
+            } else if constexpr (BM_ == B_SCALAR_DGRAD) {
+                // B(j = c, kk = (r,s,k)) = w[k][r][s][c], MN-major
+                const T* bs = (const T*)p.bsrc;
+                const int RS = p.R * p.S;
+                for (int idx = t; idx < p.BN * KB; idx += 128) {
+                    const int krow = idx / p.BN, jj = idx - krow * p.BN;
+                    const int j = n0 + jj, kk = kb * KB + krow;
+                    float v = 0.f;
+                    if (j < p.N && kk < p.kred) {
+                        const int rs = kk / p.K, k = kk - rs * p.K;
+                        v = (float)bs[((size_t)k * RS + rs) * p.C + j];
+                    }
+                    st_shared_elt<T>(bT + mnmaj_off<ELT>(jj, krow, KB), (T)v);
+                }
+            } else if constexpr (BM_ == B_SCALAR_WG) {
+                // B(j = (r,s,c), kk = pixel m) = x[n, p*st + r - pad, q*st + s - pad, c], MN-major
+                const int pq = p.P * p.Q;
+                for (int idx = t; idx < p.BN * KB; idx += 128) {
+                    const int krow = idx / p.BN, jj = idx - krow * p.BN;
+                    const int j = n0 + jj, m = kb * KB + krow;
+                    float v = 0.f;
+                    if (j < p.N && m < p.kred) {
+                        const int n = m / pq, rem = m - n * pq, pp = rem / p.Q, qq = rem - pp * p.Q;
+                        const int rs = j / p.C, c = j - rs * p.C, r = rs / p.S, sx = rs - r * p.S;
+                        const int h = pp * p.stride - p.pad + r, w = qq * p.stride - p.pad + sx;
+                        if (h >= 0 && h < p.H && w >= 0 && w < p.W)
+                            v = (float)gx[(((size_t)n * p.H + h) * p.W + w) * p.C + c];
+                    }
+                    st_shared_elt<T>(bT + mnmaj_off<ELT>(jj, krow, KB), (T)v);
+                }
+            }
+            if constexpr (GATHER) {
+                if constexpr (A_ASYNC || B_ASYNC) {
+                    cp_async_commit();
+                    // lagged arrive: stage it-1 is complete once at most 1 group is pending
+                    if (it > 0) {
+                        cp_async_wait<1>();
+                        fence_proxy_async();
+                        mbar_arrive(smem_u32(&full[(it - 1) % S]));
+                    }
+                } else {
+                    fence_proxy_async();
+                    mbar_arrive(fb);
+                }
+            }
+        }
+        if constexpr (GATHER && (A_ASYNC || B_ASYNC)) {
+            if (nkb > 0) {
+                cp_async_wait<0>();
+                fence_proxy_async();
+                mbar_arrive(smem_u32(&full[(nkb - 1) % S]));
+            }
+        }
+    } else {
+        // ======================= MMA issuer (warp 4) =======================
+        if (warp == 4) {
+            const uint32_t idesc = (1u << 4) | (Elt<ELT>::fmt << 7) | (Elt<ELT>::fmt << 10) |
+                                   ((A_MN ? 1u : 0u) << 15) | ((B_MN ? 1u : 0u) << 16) |
+                                   ((uint32_t)(p.BN >> 3) << 17) | ((128u >> 4) << 24);
+            for (int it = 0; it < nkb; ++it) {
+                const int s = it % S;
+                const uint32_t ph = (uint32_t)(it / S) & 1u;
+                mbar_wait(smem_u32(&full[s]), ph);
+                tc_fence_after();
+                if (lane == 0) {
+                    const uint32_t aT = smem_u32(sA + (size_t)s * A_BYTES);
+                    const uint32_t bT = smem_u32(sB + (size_t)s * B_BYTES);
+#pragma unroll
+                    for (int j = 0; j < KB / UMMA_K; ++j) {
+                        const uint64_t ad = A_MN ? sdesc(aT + j * UMMA_K * 128, KB * 128, MN_SBO, MN_LAYOUT)
+                                                 : sdesc(aT + j * 32, 16, 1024);
+                        const uint64_t bd = B_MN ? sdesc(bT + j * UMMA_K * 128, KB * 128, MN_SBO, MN_LAYOUT)
+                                                 : sdesc(bT + j * 32, 16, 1024);
+                        mma<ELT>(tmem, ad, bd, idesc, (it | j) != 0 ? 1u : 0u);
+                    }
+                    mma_commit(smem_u32(&empty[s]));
+                }
+                __syncwarp();
+            }
+            if (lane == 0) {
+                if (nkb > 0) mma_commit(smem_u32(accum));
+                else mbar_arrive(smem_u32(accum));
+            }
+            __syncwarp();
+        }
+        // ============================ epilogue =============================
+        mbar_wait(smem_u32(accum), 0);
+        tc_fence_after();
+        const int q4 = warp & 3;
+        const int row = q4 * 32 + lane;
+        const int m = m0 + row;
+        const uint32_t taddr_row = tmem + ((uint32_t)(q4 * 32) << 16);
+        float* outF = (float*)p.out;
+        T* outT = (T*)p.out;
+        if (EPI == EPI_STORE && z > 0) {
+            outF += (size_t)z * p.batch_stride;
+            outT += (size_t)z * p.batch_stride;
+        }
+        if constexpr (EPI == EPI_WGRAD_CHAIN) {
+            const int tile = blockIdx.y * gridDim.x + blockIdx.x;
+            if (threadIdx.x == 128 && z > 0) {
+                volatile int32_t* vs = p.sem + tile;
+                while (*vs != z) __nanosleep(100);
+                __threadfence();
+            }
+            asm volatile("bar.sync 1, 128;" ::: "memory");
+        }
+        for (int c0 = 0; c0 < p.BN; c0 += 32) {
+            uint32_t v[32];
+            if (nkb > 0) {
+                TMEM_LD32(taddr_row + (uint32_t)c0, v);
+                asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+            } else {
+#pragma unroll
+                for (int j = 0; j < 32; ++j) v[j] = 0u;
+            }
+            if (m >= p.M) continue;
+            const int nb = n0 + c0;
+            if constexpr (EPI == EPI_WGRAD_CHAIN) {
+                float* d = outF + (size_t)m * p.ldc + nb;
+#pragma unroll
+                for (int j = 0; j < 32; ++j) {
+                    if (nb + j < p.N) {
+                        float o = p.alpha * __uint_as_float(v[j]);
+                        if (z > 0) o += d[j];
+                        else if (p.beta != 0.f) o += p.beta * d[j];
+                        d[j] = o;
+                    }
+                }
+            } else if (p.out_bf16) {
+                __nv_bfloat16* d = (__nv_bfloat16*)outT + (size_t)m * p.ldc + nb;
+                const bool vec = (nb + 32 <= p.N) && ((p.ldc & 7) == 0) && p.beta == 0.f;
+                if (vec) {
+#pragma unroll
+                    for (int j = 0; j < 32; j += 8) {
+                        __align__(16) __nv_bfloat16 tmp[8];
+#pragma unroll
+                        for (int u = 0; u < 8; ++u) tmp[u] = __float2bfloat16_rn(p.alpha * __uint_as_float(v[j + u]));
+                        *reinterpret_cast<uint4*>(d + j) = *reinterpret_cast<uint4*>(tmp);
+                    }
+                } else {
+#pragma unroll
+                    for (int j = 0; j < 32; ++j) {
+                        if (nb + j < p.N) {
+                            float o = p.alpha * __uint_as_float(v[j]);
+                            if (p.beta != 0.f) o += p.beta * __bfloat162float(d[j]);
+                            d[j] = __float2bfloat16_rn(o);
+                        }
+                    }
+                }
+            } else {
+                float* d = outF + (size_t)m * p.ldc + nb;
+                const bool vec = (nb + 32 <= p.N) && ((p.ldc & 3) == 0) && p.beta == 0.f;
+                if (vec) {
+#pragma unroll
+                    for (int j = 0; j < 32; j += 4)
+                        *reinterpret_cast<float4*>(d + j) =
+                            make_float4(p.alpha * __uint_as_float(v[j]), p.alpha * __uint_as_float(v[j + 1]),
+                                        p.alpha * __uint_as_float(v[j + 2]), p.alpha * __uint_as_float(v[j + 3]));
+                } else {
+#pragma unroll
+                    for (int j = 0; j < 32; ++j) {
+                        if (nb + j < p.N) {
+                            float o = p.alpha * __uint_as_float(v[j]);
+                            if (p.beta != 0.f) o += p.beta * d[j];
+                            d[j] = o;
+                        }
+                    }
+                }
+            }
+        }
+        if constexpr (EPI == EPI_WGRAD_CHAIN) {
+            __threadfence();
+            asm volatile("bar.sync 1, 128;" ::: "memory");
+            if (threadIdx.x == 128) {
+                const int tile = blockIdx.y * gridDim.x + blockIdx.x;
+                atomicExch(p.sem + tile, z + 1 < (int)gridDim.z ? z + 1 : 0);
+            }
+        }
+    }
+    tc_fence_before();
+    __syncthreads();
+    if (warp == 4) {
+        tc_fence_after();
+        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(p.tmem_cols));
+    }
+}
+
+// ------------------------------------------------------------ host side --
+typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
+                                  const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
+                                  CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+EncodeTiledFn get_encode() {
+    static EncodeTiledFn fn = nullptr;
+    static std::once_flag once;
+    std::call_once(once, [] {
+        void* p = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+            q == cudaDriverEntryPointSuccess)
+            fn = (EncodeTiledFn)p;
+    });
+    return fn;
+}
+
+// Tensor map over a row-major tensor with up to 3 dims (dims[0] contiguous).
+bool make_map(CUtensorMap* tm, int elt, const void* base, int rank, const uint64_t* dims, const uint64_t* strides_bytes,
+              const uint32_t* box, bool mn_major = false) {
+    // 32-bit MN-major operands need the 32-B-atom swizzle matching SWIZZLE_128B_BASE32B.
+    const CUtensorMapSwizzle sw = (mn_major && elt == 4) ? CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B : CU_TENSOR_MAP_SWIZZLE_128B;
+    EncodeTiledFn enc = get_encode();
+    if (!enc) return false;
+    cuuint64_t d[3], s[2];
+    cuuint32_t b[3], e[3] = {1, 1, 1};
+    for (int i = 0; i < rank; ++i) { d[i] = dims[i]; b[i] = box[i]; }
+    for (int i = 0; i < rank - 1; ++i) s[i] = strides_bytes[i];
+    CUresult r = enc(tm, elt == 2 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32, rank,
+                     const_cast<void*>(base), d, s, b, e, CU_TENSOR_MAP_INTERLEAVE_NONE, sw,
+                     CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    return r == CUDA_SUCCESS;
+}
+
+int pick_bn(int N) {
+    if (N >= 256 && N % 256 == 0) return 256;
+    if (N % 192 == 0 && N <= 384) return 192;
+    if (N >= 128) return (N % 256 == 0) ? 256 : 128;
+    if (N > 64) return 128;
+    if (N > 32) return 64;
+    if (N > 16) return 32;
+    return 16;
+}
+
+struct Launch {
+    TcArgs a;
+    CUtensorMap ta, tb;
+    dim3 grid;
+};
+
+template <int ELT, int AM, int BM_, int EPI>
+int launch_t(Launch& L, cudaStream_t st) {
+    auto kern = tc_conv_gemm<ELT, AM, BM_, EPI>;
+    const int smem = 1024 + L.a.stages * (128 * 128 + L.a.b_bytes) + (2 * L.a.stages + 2) * 8 + 64;
+    static int configured = 0;  // per instantiation
+    if (configured < smem) {
+        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 232448);
+        if (e) return (int)e;
+        configured = 232448;
+    }
+    kern<<<L.grid, kThreads, smem, st>>>(L.a, L.ta, L.tb);
+    return (int)cudaGetLastError();
+}
+
+void finalize_tiling(Launch& L, int elt) {
+    TcArgs& a = L.a;
+    a.BN = pick_bn(a.N);
+    a.tmem_cols = a.BN <= 32 ? 32 : a.BN <= 64 ? 64 : a.BN <= 128 ? 128 : 256;
+    a.bn_atoms = (a.BN * elt + 127) / 128;
+    a.b_bytes = std::max(a.BN * 128, a.bn_atoms * (128 / elt) * 128);
+    const int stage_bytes = 128 * 128 + a.b_bytes;
+    a.stages = std::min(6, (200 * 1024) / stage_bytes);
+    if (a.stages < 2) a.stages = 2;
+}
+
+}  // namespace
+
+// ====================================================== micro-config run ==
+// Returns cudaError_t, or -1 when a shape has no tensor-core path.
+int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, const void* in0, const void* in1,
+                 float beta, void* out, char* ws, const WsLayout& WL, const SemBuf& sem, int num_sms,
+                 cudaStream_t st, CallCtx* ctx) {
+    const int elt = elt_size(g.math);
+    const int KB = 128 / elt;
+    const int atom = 128 / elt;
+    const bool bf = g.math == MUCU_MATH_BF16;
+    const int64_t PQ = (int64_t)g.p * g.q, HW = (int64_t)g.h * g.w;
+    const int RS = g.r * g.s;
+    const int64_t RSC = (int64_t)RS * g.c;
+    Launch L;
+    std::memset(&L, 0, sizeof(L));
+    TcArgs& A = L.a;
+    A.H = g.h; A.W = g.w; A.C = g.c; A.P = g.p; A.Q = g.q; A.R = g.r; A.S = g.s; A.pad = g.pad;
+    A.stride = g.stride; A.K = g.k;
+    A.alpha = alpha; A.beta = beta; A.out = out; A.out_bf16 = bf ? 1 : 0; A.sem = sem.sem;
+    auto map2 = [&](CUtensorMap* tm, const void* base, uint64_t d0, uint64_t d1, uint64_t pitch_elems, uint32_t b0,
+                    uint32_t b1, bool mn = false) {
+        uint64_t dims[2] = {d0, d1}, str[1] = {pitch_elems * elt};
+        uint32_t box[2] = {b0, b1};
+        return make_map(tm, elt, base, 2, dims, str, box, mn);
+    };
+    auto map3 = [&](CUtensorMap* tm, const void* base, uint64_t d0, uint64_t d1, uint64_t d2, uint64_t s1,
+                    uint64_t s2, uint32_t b0, uint32_t b1, uint32_t b2, bool mn = false) {
+        uint64_t dims[3] = {d0, d1, d2}, str[2] = {s1 * elt, s2 * elt};
+        uint32_t box[3] = {b0, b1, b2};
+        return make_map(tm, elt, base, 3, dims, str, box, mn);
+    };
+    auto grid2 = [&](int batch) {
+        L.grid = dim3((unsigned)ceil_div(A.N, A.BN), (unsigned)ceil_div(A.M, 128), (unsigned)batch);
+    };
+    const bool Aok = (g.c % KB) == 0;  // vector gathers over C
+    int err = 0;
+#define LAUNCH(AMODE, BMODE, EPIM) \
+    (elt == 2 ? launch_t<2, AMODE, BMODE, EPIM>(L, st) : launch_t<4, AMODE, BMODE, EPIM>(L, st))
+
+    if (type == MUCU_FWD && algo == MUCU_ALGO_IMPLICIT_GEMM) {
+        A.M = (int)(b * PQ); A.N = g.k; A.kred = (int)RSC; A.gsrc = in0;
+        finalize_tiling(L, elt);
+        grid2(1);
+        A.ldc = g.k;
+        const bool waligned = (RSC * elt) % 16 == 0;
+        if (Aok) {
+            A.num_kb = (int)ceil_div(RSC, KB);
+            if (!waligned) return -1;
+            if (!map2(&L.tb, in1, RSC, g.k, RSC, KB, A.BN)) return -1;
+            A.tma_bytes = A.BN * 128;
+            err = LAUNCH(A_GATHER_FWD, B_TMA_K2, EPI_STORE);
+        } else {
+            A.num_kb = (int)ceil_div(RSC, KB);
+            A.bsrc = in1; A.ldb = (int)RSC;
+            err = LAUNCH(A_SCALAR_FWD, B_SCALAR_K, EPI_STORE);
+        }
+        return err;
+    }
+    if (type == MUCU_FWD && algo == MUCU_ALGO_IM2COL_GEMM) {
+        const void* colp = in0;
+        int kpitch = g.c;
+        if (!is_pointwise(g)) {
+            colp = ws + WL.a_off;
+            kpitch = WL.kpitch;
+            err = launch_im2col(g, b, in0, (void*)colp, kpitch, st);
+            if (err) return err;
+        }
+        const void* wp = in1;
+        int wpitch = (int)RSC;
+        if (WL.filter_padded) {
+            if (ctx->fixed_kind != 1 || ctx->fixed_src != in1) {
+                err = launch_pad_filter(g, in1, ws, WL.kpitch, st);
+                if (err) return err;
+                ctx->fixed_kind = 1; ctx->fixed_src = in1;
+            }
+            wp = ws; wpitch = WL.kpitch;
+        }
+        A.M = (int)(b * PQ); A.N = g.k; A.num_kb = (int)ceil_div(RSC, KB); A.ldc = g.k;
+        finalize_tiling(L, elt);
+        grid2(1);
+        if (!map2(&L.ta, colp, RSC, (uint64_t)A.M, kpitch, KB, 128)) return -1;
+        if (!map2(&L.tb, wp, RSC, g.k, wpitch, KB, A.BN)) return -1;
+        A.tma_bytes = 128 * 128 + A.BN * 128;
+        return LAUNCH(A_TMA_K2, B_TMA_K2, EPI_STORE);
+    }
+    if (algo == MUCU_ALGO_WINOGRAD_2X2_3X3) {
+        const bool dg = type == MUCU_BWD_DATA;
+        const int I = dg ? g.k : g.c, O = dg ? g.c : g.k;
+        const int OH = dg ? g.h : g.p, OW = dg ? g.w : g.q;
+        const int64_t Tt = (int64_t)((OH + 1) / 2) * ((OW + 1) / 2) * b;
+        if (ctx->fixed_kind != 2 || ctx->fixed_src != in1) {
+            err = launch_wg_filter(g, dg, in1, ws, st);
+            if (err) return err;
+            ctx->fixed_kind = 2; ctx->fixed_src = in1;
+        }
+        void* V = ws + WL.a_off;
+        float* Mx = (float*)(ws + WL.b_off);
+        err = launch_wg_input(g, dg, b, in0, V, st);
+        if (err) return err;
+        A.M = (int)Tt; A.N = O; A.num_kb = (int)ceil_div(I, KB); A.ldc = O;
+        A.batch_stride = Tt * O; A.alpha = 1.f; A.beta = 0.f; A.out = Mx; A.out_bf16 = 0;
+        finalize_tiling(L, elt);
+        grid2(16);
+        if (!map3(&L.ta, V, I, Tt, 16, I, Tt * I, KB, 128, 1)) return -1;
+        if (!map3(&L.tb, ws, I, O, 16, I, (uint64_t)O * I, KB, A.BN, 1)) return -1;
+        A.tma_bytes = 128 * 128 + A.BN * 128;
+        err = LAUNCH(A_TMA_K3, B_TMA_K3, EPI_STORE);
+        if (err) return err;
+        return launch_wg_output(g, dg, b, alpha, Mx, beta, out, st);
+    }
+    if (type == MUCU_BWD_DATA && algo == MUCU_ALGO_IMPLICIT_GEMM) {
+        A.M = (int)(b * HW); A.N = g.c; A.num_kb = (int)ceil_div((int64_t)RS * g.k, KB); A.ldc = g.c;
+        A.gsrc = in0; A.kred = RS * g.k;
+        finalize_tiling(L, elt);
+        grid2(1);
+        A.bsrc = in1;
+        if (g.k % KB != 0) return LAUNCH(A_SCALAR_DGRAD, B_SCALAR_DGRAD, EPI_STORE);
+        if ((g.c * elt) % 16 == 0 && g.c >= atom) {
+            // w viewed as {C, R*S, K} (c contiguous): B(c, (r,s,k)) MN-major
+            if (!map3(&L.tb, in1, g.c, RS, g.k, g.c, RSC, atom, 1, KB, true)) return -1;
+            A.tma_bytes = A.bn_atoms * KB * 128;
+            return LAUNCH(A_GATHER_DGRAD, B_TMA_MN3, EPI_STORE);
+        }
+        return LAUNCH(A_GATHER_DGRAD, B_SCALAR_DGRAD, EPI_STORE);
+    }
+    if (type == MUCU_BWD_DATA && algo == MUCU_ALGO_IM2COL_GEMM) {
+        // dcol[m', (r,s,c)] = sum_k dy[m'][k] w[k][(r,s,c)]  (pointwise: straight into dx with alpha/beta)
+        const bool pw = is_pointwise(g);
+        const void* wp = in1;
+        int64_t wpitch = RSC;
+        if (!pw && WL.filter_padded) {
+            if (ctx->fixed_kind != 1 || ctx->fixed_src != in1) {
+                const int fpitch = (int)align_up((uint64_t)RSC, (uint64_t)(16 / elt));
+                err = launch_pad_filter(g, in1, ws, fpitch, st);
+                if (err) return err;
+                ctx->fixed_kind = 1; ctx->fixed_src = in1;
+            }
+            wp = ws; wpitch = (int64_t)align_up((uint64_t)RSC, (uint64_t)(16 / elt));
+        }
+        A.M = (int)(b * PQ); A.N = (int)RSC; A.num_kb = (int)ceil_div(g.k, KB);
+        if (pw) { A.ldc = g.c; }
+        else { A.ldc = WL.kpitch; A.out = ws + WL.a_off; A.out_bf16 = 0; A.alpha = 1.f; A.beta = 0.f; }
+        finalize_tiling(L, elt);
+        grid2(1);
+        if (RSC < atom) return -1;
+        if (!map2(&L.ta, in0, g.k, (uint64_t)A.M, g.k, KB, 128)) return -1;
+        if (!map2(&L.tb, wp, RSC, g.k, wpitch, atom, KB, true)) return -1;
+        A.tma_bytes = 128 * 128 + A.bn_atoms * KB * 128;
+        err = LAUNCH(A_TMA_K2, B_TMA_MN2, EPI_STORE);
+        if (err || pw) return err;
+        return launch_col2im(g, b, alpha, (const float*)(ws + WL.a_off), WL.kpitch, beta, out, st);
+    }
+    if (type == MUCU_BWD_FILTER) {
+        // dw[k][(r,s,c)] = sum_m dy[m][k] B(m, (r,s,c)); A = dy MN-major via TMA.
+        const int64_t Mpix = (int64_t)b * PQ;
+        A.M = g.k; A.N = (int)RSC; A.ldc = RSC; A.kred = (int)Mpix; A.gsrc = in0;
+        finalize_tiling(L, elt);
+        const int64_t tiles = ceil_div(A.N, A.BN) * ceil_div(A.M, 128);
+        if (tiles > sem.capacity) return -1;
+        const int64_t nkb = ceil_div(Mpix, KB);
+        int64_t want = std::max<int64_t>(1, (2LL * num_sms + tiles - 1) / tiles);
+        int64_t nsplit = std::min<int64_t>(std::min<int64_t>(want, std::max<int64_t>(1, nkb / 4)), 65535);
+        A.kb_per_split = (int)ceil_div(nkb, nsplit);
+        nsplit = ceil_div(nkb, A.kb_per_split);
+        A.num_kb = (int)nkb;
+        L.grid = dim3((unsigned)ceil_div(A.N, A.BN), (unsigned)ceil_div(A.M, 128), (unsigned)nsplit);
+        if (!map2(&L.ta, in1, g.k, (uint64_t)Mpix, g.k, atom, KB, true)) return -1;
+        const int a_bytes = 128 * KB * elt;
+        if (algo == MUCU_ALGO_IM2COL_GEMM) {
+            const void* colp = in0;
+            int64_t kp = g.c;
+            if (!is_pointwise(g)) {
+                colp = ws + WL.a_off; kp = WL.kpitch;
+                err = launch_im2col(g, b, in0, (void*)colp, (int)kp, st);
+                if (err) return err;
+            }
+            if (RSC < atom) return -1;
+            if (!map2(&L.tb, colp, RSC, (uint64_t)Mpix, kp, atom, KB, true)) return -1;
+            A.tma_bytes = a_bytes + A.bn_atoms * KB * 128;
+            return LAUNCH(A_TMA_MN2, B_TMA_MN2, EPI_WGRAD_CHAIN);
+        }
+        A.tma_bytes = a_bytes;
+        if (g.c % atom == 0) return LAUNCH(A_TMA_MN2, B_GATHER_WG, EPI_WGRAD_CHAIN);
+        return LAUNCH(A_TMA_MN2, B_SCALAR_WG, EPI_WGRAD_CHAIN);
+    }
+#undef LAUNCH
     return -1;
 }
+
 }  // namespace mucu

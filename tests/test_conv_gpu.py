@@ -24,6 +24,9 @@ from gpu_util import normwise_err, oracle_ref, run_gpu, stored  # noqa: E402
 # n, c, h, w, k, r, s, pad, stride -- several tiles and a ragged tail each
 SHAPES = {
     "3x3s1": (3, 32, 13, 13, 40, 3, 3, 1, 1),
+    "3x3s1_c64": (2, 64, 12, 12, 64, 3, 3, 1, 1),      # vector gather paths (C, K % 64 == 0)
+    "3x3s1_c128": (2, 128, 10, 10, 192, 3, 3, 1, 1),
+    "3x3s2_c64": (2, 64, 15, 15, 128, 3, 3, 1, 2),
     "3x3s1_p0_odd": (2, 16, 9, 11, 24, 3, 3, 0, 1),
     "3x3s1_p2": (2, 32, 7, 7, 32, 3, 3, 2, 1),
     "5x5s1": (2, 64, 11, 11, 48, 5, 5, 2, 1),          # AlexNet conv2 geometry

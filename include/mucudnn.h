@@ -100,6 +100,9 @@ typedef struct mucu_network* mucu_network_t; /* library-owned WD kernel list (P:
 const char* mucu_status_string(mucu_status_t status);   /* host; static string */
 const char* mucu_last_error(void);                      /* host; thread-local detail */
 int32_t mucu_version(void);                             /* host */
+/* Process-wide number of CUDA kernels the library has launched so far (host;
+ * monotone, for launch accounting in benchmarks). */
+uint64_t mucu_launch_count(void);
 
 /* Create a handle bound to CUDA device `device` (makes it current on the
  * calling thread).  Reads env MUCU_BATCH_POLICY={all,pow2,undivided} (default

@@ -62,6 +62,7 @@ def _load():
         "mucu_status_string": (ctypes.c_char_p, [ctypes.c_int]),
         "mucu_last_error": (ctypes.c_char_p, []),
         "mucu_version": (i32, []),
+        "mucu_launch_count": (u64, []),
         "mucu_create": (ctypes.c_int, [P(vp), ctypes.c_int]),
         "mucu_destroy": (ctypes.c_int, [vp]),
         "mucu_set_policy": (ctypes.c_int, [vp, ctypes.c_int]),
@@ -111,6 +112,10 @@ def _u64(a):
 
 def version() -> int:
     return lib.mucu_version()
+
+
+def launch_count() -> int:
+    return int(lib.mucu_launch_count())
 
 
 def status_string(s: int) -> str:

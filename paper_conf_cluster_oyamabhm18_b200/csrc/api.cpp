@@ -5,6 +5,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <atomic>
 #include <cstdarg>
 #include <cstdio>
 #include <cstdlib>
@@ -19,6 +20,9 @@
 namespace mucu {
 
 static thread_local char g_err[512] = "";
+static std::atomic<uint64_t> g_launches{0};
+
+void count_launch() { g_launches.fetch_add(1, std::memory_order_relaxed); }
 
 mucu_status_t set_error(mucu_status_t s, const char* fmt, ...) {
     va_list ap;
@@ -243,6 +247,7 @@ extern "C" const char* mucu_status_string(mucu_status_t s) {
 
 extern "C" const char* mucu_last_error(void) { return g_err; }
 extern "C" int32_t mucu_version(void) { return MUCU_VERSION; }
+extern "C" uint64_t mucu_launch_count(void) { return g_launches.load(std::memory_order_relaxed); }
 
 static int policy_from_env(int dflt) {
     const char* p = getenv("MUCU_BATCH_POLICY");

@@ -287,6 +287,7 @@ int im2col_t(const Geom& g, int32_t b, const void* x, void* col, int32_t kpitch,
         im2col_scalar_kernel<T><<<grid, 256, 0, st>>>((const T*)x, (T*)col, rows, g.h, g.w, g.c, g.p, g.q,
                                                        g.s, g.pad, g.stride, RSC, kpitch);
     }
+    count_launch();
     return (int)cudaGetLastError();
 }
 
@@ -304,6 +305,7 @@ int launch_pad_filter(const Geom& g, const void* w, void* wpad, int32_t kpitch, 
         pad_filter_kernel<__nv_bfloat16><<<grid, 256, 0, st>>>((const __nv_bfloat16*)w, (__nv_bfloat16*)wpad, g.k, RSC, kpitch);
     else
         pad_filter_kernel<float><<<grid, 256, 0, st>>>((const float*)w, (float*)wpad, g.k, RSC, kpitch);
+    count_launch();
     return (int)cudaGetLastError();
 }
 
@@ -317,6 +319,7 @@ int launch_col2im(const Geom& g, int32_t b, float alpha, const float* dcol, int3
     else
         col2im_kernel<float><<<grid, 256, 0, st>>>(dcol, (float*)dx, total, g.h, g.w, g.c, g.p, g.q, g.r, g.s,
                                                   g.pad, g.stride, kpitch, alpha, beta);
+    count_launch();
     return (int)cudaGetLastError();
 }
 
@@ -327,6 +330,7 @@ int launch_wg_filter(const Geom& g, bool dgrad, const void* w, void* U, cudaStre
         wg_filter_kernel<__nv_bfloat16><<<grid, 256, 0, st>>>((const __nv_bfloat16*)w, (__nv_bfloat16*)U, O, I, g.c, dgrad);
     else
         wg_filter_kernel<float><<<grid, 256, 0, st>>>((const float*)w, (float*)U, O, I, g.c, dgrad);
+    count_launch();
     return (int)cudaGetLastError();
 }
 
@@ -347,6 +351,7 @@ int launch_wg_input(const Geom& g, bool dgrad, int32_t b, const void* in, void* 
         wg_input_kernel<__nv_bfloat16><<<grid, 256, 0, st>>>((const __nv_bfloat16*)in, (__nv_bfloat16*)V, tiles, IH, IW, I, TH, TW, pad);
     else
         wg_input_kernel<float><<<grid, 256, 0, st>>>((const float*)in, (float*)V, tiles, IH, IW, I, TH, TW, pad);
+    count_launch();
     return (int)cudaGetLastError();
 }
 
@@ -361,6 +366,7 @@ int launch_wg_output(const Geom& g, bool dgrad, int32_t b, float alpha, const fl
         wg_output_kernel<__nv_bfloat16><<<grid, 256, 0, st>>>(M, (__nv_bfloat16*)out, tiles, OH, OW, O, TH, TW, alpha, beta);
     else
         wg_output_kernel<float><<<grid, 256, 0, st>>>(M, (float*)out, tiles, OH, OW, O, TH, TW, alpha, beta);
+    count_launch();
     return (int)cudaGetLastError();
 }
 

@@ -217,7 +217,7 @@ template <int BM, int BN, bool CKA, bool CKB, class AV, class BV, class EPI>
 __global__ void __launch_bounds__(kThreads) simt_gemm_kernel(AV a, BV b, EPI epi, int64_t Kd) {
     constexpr int TM = BM / 16, TN = BN / 16;
     a.batch(blockIdx.z); b.batch(blockIdx.z); epi.batch(blockIdx.z);
-    const int64_t m0 = (int64_t)blockIdx.y * BM, n0 = (int64_t)blockIdx.x * BN;
+    const int64_t m0 = (int64_t)blockIdx.x * BM, n0 = (int64_t)blockIdx.y * BN;  // M on grid.x (no 65535 cap)
     float acc[TM][TN];
     simt_mainloop<BM, BN, CKA, CKB>(a, b, m0, n0, 0, Kd, acc);
     const int tx = threadIdx.x % 16, ty = threadIdx.x / 16;
@@ -235,7 +235,7 @@ __global__ void __launch_bounds__(kThreads) simt_wgrad_kernel(AV a, BV b, float*
                                                               int64_t Kd, int64_t k_per_split, float alpha,
                                                               float beta, int32_t* sem) {
     constexpr int TM = BM / 16, TN = BN / 16;
-    const int64_t m0 = (int64_t)blockIdx.y * BM, n0 = (int64_t)blockIdx.x * BN;
+    const int64_t m0 = (int64_t)blockIdx.x * BM, n0 = (int64_t)blockIdx.y * BN;
     const int split = blockIdx.z, nsplit = gridDim.z;
     const int64_t kb = (int64_t)split * k_per_split;
     const int64_t ke = min(Kd, kb + k_per_split);
@@ -272,8 +272,9 @@ __global__ void __launch_bounds__(kThreads) simt_wgrad_kernel(AV a, BV b, float*
 template <int BM, int BN, bool CKA, bool CKB, class AV, class BV, class EPI>
 int launch_gemm(const AV& a, const BV& b, const EPI& e, int64_t M, int64_t N, int64_t Kd, int batch,
                 cudaStream_t st) {
-    dim3 grid((unsigned)ceil_div(N, BN), (unsigned)ceil_div(M, BM), (unsigned)batch);
+    dim3 grid((unsigned)ceil_div(M, BM), (unsigned)ceil_div(N, BN), (unsigned)batch);
     simt_gemm_kernel<BM, BN, CKA, CKB><<<grid, kThreads, 0, st>>>(a, b, e, Kd);
+    count_launch();
     return (int)cudaGetLastError();
 }
 
@@ -340,7 +341,7 @@ int simt_wgrad(const Geom& g, int32_t b, float alpha, const float* dy, const flo
     int64_t nsplit = std::min<int64_t>(std::min<int64_t>(want, maxs), 65535);
     int64_t kps = ceil_div(ceil_div(Kd, nsplit), BK) * BK;
     nsplit = ceil_div(Kd, kps);
-    dim3 grid((unsigned)ceil_div(cols, BN), (unsigned)ceil_div(rows, BM), (unsigned)nsplit);
+    dim3 grid((unsigned)ceil_div(rows, BM), (unsigned)ceil_div(cols, BN), (unsigned)nsplit);
     Dense a{dy, rows, Kd, 1, g.k, 0};  // A(k, m) = dy[m][k]
     if (col_input) {
         Dense bb{xin, cols, Kd, 1, kpitch, 0};  // B(j, m) = col[m][j]
@@ -349,6 +350,7 @@ int simt_wgrad(const Geom& g, int32_t b, float alpha, const float* dy, const flo
         Im2colT bb{Im2col{xin, Kd, g.h, g.w, g.c, g.p, g.q, g.s, g.pad, g.stride, (int)cols}};
         simt_wgrad_kernel<BM, BN><<<grid, kThreads, 0, st>>>(a, bb, dw, rows, cols, Kd, kps, alpha, beta, sem.sem);
     }
+    count_launch();
     return (int)cudaGetLastError();
 }
 

@@ -242,8 +242,10 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
     uint32_t* tmem_slot = (uint32_t*)(bars + 2 * S + 1);
 
     const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
-    const int m0 = blockIdx.y * 128;
-    const int n0 = blockIdx.x * p.BN;
+    // M tiles on grid.x (up to 2^31-1; conv1 DGRAD at N=256 has 100k of them),
+    // N tiles on grid.y: consecutive CTAs share the same B (filter) tile in L2.
+    const int m0 = blockIdx.x * 128;
+    const int n0 = blockIdx.y * p.BN;
     const int z = blockIdx.z;
     int kb_begin = 0, kb_end = p.num_kb;
     if (EPI == EPI_WGRAD_CHAIN) {
@@ -680,6 +682,7 @@ int launch_t(Launch& L, cudaStream_t st) {
         configured = 232448;
     }
     kern<<<L.grid, kThreads, smem, st>>>(L.a, L.ta, L.tb);
+    count_launch();
     return (int)cudaGetLastError();
 }
 
@@ -727,7 +730,7 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         return make_map(tm, elt, base, 3, dims, str, box, mn);
     };
     auto grid2 = [&](int batch) {
-        L.grid = dim3((unsigned)ceil_div(A.N, A.BN), (unsigned)ceil_div(A.M, 128), (unsigned)batch);
+        L.grid = dim3((unsigned)ceil_div(A.M, 128), (unsigned)ceil_div(A.N, A.BN), (unsigned)batch);
     };
     const bool Aok = (g.c % KB) == 0;  // vector gathers over C
     int err = 0;
@@ -860,7 +863,7 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         A.kb_per_split = (int)ceil_div(nkb, nsplit);
         nsplit = ceil_div(nkb, A.kb_per_split);
         A.num_kb = (int)nkb;
-        L.grid = dim3((unsigned)ceil_div(A.N, A.BN), (unsigned)ceil_div(A.M, 128), (unsigned)nsplit);
+        L.grid = dim3((unsigned)ceil_div(A.M, 128), (unsigned)ceil_div(A.N, A.BN), (unsigned)nsplit);
         if (!map2(&L.ta, in1, g.k, (uint64_t)Mpix, g.k, atom, KB, true)) return -1;
         const int a_bytes = 128 * KB * elt;
         if (algo == MUCU_ALGO_IM2COL_GEMM) {

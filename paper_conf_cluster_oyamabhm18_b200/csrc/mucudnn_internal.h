@@ -17,6 +17,9 @@ namespace mucu {
 // Records a thread-local error message and returns `s` (printf-style).
 mucu_status_t set_error(mucu_status_t s, const char* fmt, ...);
 
+// Process-wide count of kernel launches issued by the library (mucu_launch_count).
+void count_launch();
+
 // Layer geometry with derived output extent (reading G1/G3).
 struct Geom {
     int32_t n, c, h, w, k, r, s, pad, stride, p, q, math;

@@ -1,0 +1,199 @@
+"""Network-level planning and execution of conv layers (Sec. III/III-A).
+
+ConvNet owns, for a list of conv layers at mini-batch N:
+* device tensors (x, w, dy inputs; y, dx, dw outputs) -- NHWC / KRSC,
+* one plan per kernel (layer x {FWD, DGRAD, WGRAD}) from
+  - WR: per-kernel benchmark + DP under a per-layer workspace limit,
+    one workspace per kernel (Fig. 4, "one workspace per layer"), or
+  - WD: one network workspace, per-kernel desirable sets + the
+    exact MCKP, each kernel a segment of it (Fig. 14),
+  - "undivided": the fastest single algorithm at micro-batch N that
+    fits the same limit -- the comparison baseline of BASELINE.json,
+* `iteration()`: forward of every layer in order, then BackwardData and
+  BackwardFilter in reverse order (the conv part of a training iteration,
+  P:L198), each call executing its plan through the C ABI.
+
+In data-parallel runs each BackwardFilter output is handed to `grad_hook`
+(e.g. an asynchronous NCCL allreduce, see distributed.py) right after its last
+micro-batch, so communication overlaps the remaining backward layers.
+"""
+from __future__ import annotations
+
+from dataclasses import dataclass, field
+from typing import Callable, Dict, List, Optional, Sequence, Tuple
+
+import numpy as np
+import torch
+
+from . import _lib as L
+from . import torch_api as T
+
+TYPES = (L.FWD, L.BWD_DATA, L.BWD_FILTER)
+
+
+@dataclass
+class Kernel:
+    layer: int
+    conv_type: int
+    desc: L.ConvDesc
+    plan: List[Tuple[int, int]] = field(default_factory=list)
+    table: Optional[Tuple[np.ndarray, np.ndarray]] = None
+    est_ns: int = 0
+    ws_bytes: int = 0
+    ws_offset: int = 0
+
+
+def layer_flops(layer, n: int) -> int:
+    """Direct-convolution FLOPs of one direction, 2 N K C R S P Q."""
+    return 2 * n * layer.k * layer.c * layer.r * layer.s * layer.p * layer.q
+
+
+def algorithmic_flops(layer, conv_type: int, plan) -> int:
+    """Tensor/FMA work the chosen algorithms actually perform:
+    IG / I2C: 2 b K C R S P Q; Winograd F(2x2,3x3): 16 GEMMs of 2 (b T) K C."""
+    f = 0
+    for algo, b in plan:
+        if algo == L.WINOGRAD:
+            oh, ow = (layer.h, layer.w) if conv_type == L.BWD_DATA else (layer.p, layer.q)
+            t = ((oh + 1) // 2) * ((ow + 1) // 2)
+            f += 2 * 16 * b * t * layer.k * layer.c
+        else:
+            f += layer_flops(layer, b)
+    return f
+
+
+class ConvNet:
+    def __init__(self, handle: L.Handle, layers: Sequence, n: int, math: int, device: str = "cuda"):
+        self.h = handle
+        self.layers = list(layers)
+        self.n = n
+        self.math = math
+        self.device = device
+        self.dtype = torch.bfloat16 if math == L.MATH_BF16 else torch.float32
+        self.descs = [L.desc(n, l.c, l.h, l.w, l.k, l.r, l.s, l.pad, l.stride, math) for l in self.layers]
+        self.kernels: Dict[Tuple[int, int], Kernel] = {
+            (i, t): Kernel(i, t, d) for i, d in enumerate(self.descs) for t in TYPES}
+        self.tensors: List[Dict[str, torch.Tensor]] = []
+        self.workspaces: Dict[Tuple[int, int], Optional[torch.Tensor]] = {}
+        self.net_ws: Optional[torch.Tensor] = None
+
+    # ----------------------------------------------------------- memory --
+    def allocate(self, seed: int = 0, kind: str = "normal", generator=None):
+        """Seeded synthetic tensors on the device (values do not affect timing)."""
+        from synthetic import torch_conv_inputs  # workload generator (no method arithmetic)
+        self.tensors = []
+        for i, (l, d) in enumerate(zip(self.layers, self.descs)):
+            x, w, dy = torch_conv_inputs(l, self.n, seed=1000 * seed + i, device=self.device, dtype=self.dtype,
+                                         kind=kind)
+            xs, ws_, ys = T.shapes(d)
+            self.tensors.append(dict(
+                x=x, w=w, dy=dy,
+                y=torch.empty(ys, dtype=self.dtype, device=self.device),
+                dx=torch.empty(xs, dtype=self.dtype, device=self.device),
+                dw=torch.zeros(ws_, dtype=torch.float32, device=self.device)))
+
+    # ---------------------------------------------------------- planning --
+    def benchmark_all(self, ws_limit: int, progress: Optional[Callable] = None):
+        """P:L88 step 1 for every kernel (identical layers hit the handle's cache)."""
+        scratch = None
+        for key, k in self.kernels.items():
+            need = L.benchmark_scratch_size(k.desc, k.conv_type, ws_limit)
+            if scratch is None or scratch.numel() < need:
+                scratch = None
+                torch.cuda.empty_cache()
+                scratch = T.make_scratch(k.desc, k.conv_type, ws_limit)
+            k.table = self.h.benchmark(k.desc, k.conv_type, ws_limit, scratch.data_ptr(), scratch.numel(),
+                                       T._stream())
+            if progress:
+                progress(key)
+        del scratch
+        torch.cuda.empty_cache()
+
+    def plan_wr(self, ws_limit: int):
+        """WR: per-kernel DP on its timing table; one workspace per kernel."""
+        for k in self.kernels.values():
+            t, w = k.table
+            k.est_ns, k.plan = L.plan_wr(self.n, t, w, ws_limit)
+            k.ws_bytes = T.plan_workspace(k.desc, k.conv_type, k.plan)
+        self._alloc_workspaces()
+
+    def plan_undivided(self, ws_limit: int):
+        """Best single algorithm at micro-batch N within the limit."""
+        n = self.n
+        for k in self.kernels.values():
+            t, w = k.table
+            fit = [(int(t[a, n]), int(w[a, n]), a) for a in range(L.NUM_ALGOS) if t[a, n] >= 0 and w[a, n] <= ws_limit]
+            if not fit:
+                raise L.MucuError(3, f"no algorithm fits {ws_limit} B undivided for kernel {k.layer}/{k.conv_type}")
+            tt, ww, a = min(fit)
+            k.plan, k.est_ns = [(a, n)], tt
+            k.ws_bytes = T.plan_workspace(k.desc, k.conv_type, k.plan)
+        self._alloc_workspaces()
+
+    def plan_wd(self, total_limit: int):
+        """WD: desirable sets + exact MCKP over all kernels, one
+        network workspace carved into 256-B aligned segments (reading G18)."""
+        net = L.Network()
+        order = list(self.kernels.keys())
+        for key in order:
+            net.add(self.kernels[key].desc, key[1])
+        net.plan_from_tables(total_limit, [self.kernels[key].table for key in order])
+        for kid, key in enumerate(order):
+            k = self.kernels[key]
+            k.plan, k.ws_offset, k.ws_bytes, k.est_ns = net.get(kid)
+        total = max((k.ws_offset + k.ws_bytes for k in self.kernels.values()), default=0)
+        self.net_ws = torch.empty(max(total, 256), dtype=torch.uint8, device=self.device)
+        self.workspaces = {key: (self.net_ws[k.ws_offset:k.ws_offset + k.ws_bytes] if k.ws_bytes else None)
+                           for key, k in self.kernels.items()}
+
+    def _alloc_workspaces(self):
+        self.net_ws = None
+        self.workspaces = {}
+        for key, k in self.kernels.items():
+            self.workspaces[key] = torch.empty(k.ws_bytes, dtype=torch.uint8, device=self.device) if k.ws_bytes else None
+
+    def total_workspace(self) -> int:
+        if self.net_ws is not None:
+            return self.net_ws.numel()
+        return sum(k.ws_bytes for k in self.kernels.values())
+
+    # --------------------------------------------------------- execution --
+    def run_kernel(self, i: int, conv_type: int):
+        k = self.kernels[(i, conv_type)]
+        t = self.tensors[i]
+        ws = self.workspaces.get((i, conv_type))
+        if conv_type == L.FWD:
+            T.conv_forward(self.h, k.desc, k.plan, t["x"], t["w"], t["y"], workspace=ws)
+        elif conv_type == L.BWD_DATA:
+            T.conv_backward_data(self.h, k.desc, k.plan, t["dy"], t["w"], t["dx"], workspace=ws)
+        else:
+            T.conv_backward_filter(self.h, k.desc, k.plan, t["x"], t["dy"], t["dw"], workspace=ws)
+
+    def iteration(self, on_op: Optional[Callable] = None, grad_hook: Optional[Callable] = None,
+                  skip_conv1_dgrad: bool = False):
+        """FWD of all layers, then DGRAD + WGRAD in reverse order.  on_op(i, type,
+        'begin'|'end') lets a caller record CUDA events around each call."""
+        order = [(i, L.FWD) for i in range(len(self.layers))]
+        for i in reversed(range(len(self.layers))):
+            if not (skip_conv1_dgrad and i == 0):
+                order.append((i, L.BWD_DATA))
+            order.append((i, L.BWD_FILTER))
+        for i, t in order:
+            if on_op:
+                on_op(i, t, "begin")
+            self.run_kernel(i, t)
+            if on_op:
+                on_op(i, t, "end")
+            if t == L.BWD_FILTER and grad_hook is not None:
+                grad_hook(i, self.tensors[i]["dw"])
+
+    def flops_per_iteration(self) -> int:
+        return sum(layer_flops(l, self.n) for l in self.layers) * 3
+
+    def summary(self):
+        rows = []
+        for (i, t), k in sorted(self.kernels.items()):
+            rows.append(dict(layer=self.layers[i].name, type=L.TYPE_NAMES[t],
+                             plan=[(L.ALGO_NAMES[a], b) for a, b in k.plan], est_us=k.est_ns / 1e3,
+                             ws_MiB=round(k.ws_bytes / 2 ** 20, 3)))
+        return rows

@@ -49,6 +49,8 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-sample", type=int, default=0, help="oracle sample (images per kernel); 0 = auto")
     ap.add_argument("--json-out", default="")
+    ap.add_argument("--tables-in", default="", help="benchmark DB (.npz) to plan from instead of benchmarking")
+    ap.add_argument("--tables-out", default="", help="write the benchmark DB (.npz) after the benchmark pass")
     return ap.parse_args()
 
 
@@ -206,7 +208,10 @@ def main():
     # ---- planning: benchmark pass + DP / ILP ----
     t0 = time.perf_counter()
     plan_limit = int(args.wd_mib * 2 ** 20) if args.wd_mib > 0 else ws_limit
-    net.benchmark_all(plan_limit)
+    if not (args.tables_in and os.path.exists(args.tables_in) and net.load_tables(args.tables_in, plan_limit, args.policy)):
+        net.benchmark_all(plan_limit)
+        if args.tables_out and rank == 0:
+            net.save_tables(args.tables_out, plan_limit, args.policy)
     bench_s = time.perf_counter() - t0
     flush = torch.empty(512 * 2 ** 20, dtype=torch.uint8, device=dev)
     grad_ar = GradAllreduce()

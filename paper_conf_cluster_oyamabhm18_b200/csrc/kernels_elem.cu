@@ -13,6 +13,8 @@
 #include <cuda_bf16.h>
 #include <cuda_runtime.h>
 
+#include <type_traits>
+
 #include "mucudnn_internal.h"
 
 namespace mucu {
@@ -273,22 +275,105 @@ __global__ void wg_output_kernel(const float* __restrict__ M, T* __restrict__ ou
     }
 }
 
+// Row-oriented im2col: one warp per col row (output pixel m = (n,p,q)).  For
+// a fixed filter row r the S*C values (s,c) of the row are CONTIGUOUS in NHWC
+// x (x[n, h0+r, w0 .. w0+S-1, 0..C-1]), so the warp copies R runs of S*C
+// elements with the lanes along the run (coalesced reads and writes, V-wide
+// vectors when C % V == 0) and zero-fills outside [s_lo*C, s_hi*C) and rows
+// off the image -- no per-element index division.
+template <class T, int V>
+__global__ void im2col_rows_kernel(const T* __restrict__ x, T* __restrict__ col, int64_t rows, int H, int W,
+                                   int C, int P, int Q, int R, int S, int pad, int st, int kpitch) {
+    using VT = typename std::conditional<V == 1, T, uint4>::type;
+    const int lane = threadIdx.x & 31;
+    const int64_t warp0 = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    const int SC = S * C, RSC = R * SC;
+    const int pq = P * Q;
+    for (int64_t m = warp0; m < rows; m += nwarps) {
+        const int n = (int)(m / pq);
+        const int rem = (int)(m - (int64_t)n * pq);
+        const int p = rem / Q, q = rem - (rem / Q) * Q;
+        const int h0 = p * st - pad, w0 = q * st - pad;
+        const int lo = max(0, -w0) * C, hi = min(S, W - w0) * C;
+        T* dst = col + m * kpitch;
+        for (int r = 0; r < R; ++r) {
+            const int h = h0 + r;
+            const bool hv = h >= 0 && h < H;
+            const T* src = x + (((int64_t)n * H + (hv ? h : 0)) * W + w0) * C;  // may point left of the row; only read in [lo,hi)
+            for (int sc = lane * V; sc < SC; sc += 32 * V) {
+                VT v;
+                if (hv && sc >= lo && sc < hi) v = *reinterpret_cast<const VT*>(src + sc);
+                else if constexpr (V == 1) v = from_f<T>(0.f);
+                else v = make_uint4(0, 0, 0, 0);
+                *reinterpret_cast<VT*>(dst + r * SC + sc) = v;
+            }
+        }
+        for (int kk = RSC + lane; kk < kpitch; kk += 32) dst[kk] = from_f<T>(0.f);
+    }
+}
+
 template <class T>
 int im2col_t(const Geom& g, int32_t b, const void* x, void* col, int32_t kpitch, cudaStream_t st) {
     constexpr int V = 16 / sizeof(T);
     const int64_t rows = (int64_t)b * g.p * g.q;
-    const int RSC = g.r * g.s * g.c;
-    if (g.c % V == 0 && kpitch % V == 0) {
-        int grid = grid_for(rows * (kpitch / V), 256);
-        im2col_kernel<T, V><<<grid, 256, 0, st>>>((const T*)x, (T*)col, rows, g.h, g.w, g.c, g.p, g.q, g.s,
-                                                   g.pad, g.stride, RSC, kpitch);
-    } else {
-        int grid = grid_for(rows * kpitch, 256);
-        im2col_scalar_kernel<T><<<grid, 256, 0, st>>>((const T*)x, (T*)col, rows, g.h, g.w, g.c, g.p, g.q,
-                                                       g.s, g.pad, g.stride, RSC, kpitch);
-    }
+    const int grid = grid_for(rows * 32, 256);
+    if (g.c % V == 0 && kpitch % V == 0)
+        im2col_rows_kernel<T, V><<<grid, 256, 0, st>>>((const T*)x, (T*)col, rows, g.h, g.w, g.c, g.p, g.q, g.r,
+                                                        g.s, g.pad, g.stride, kpitch);
+    else
+        im2col_rows_kernel<T, 1><<<grid, 256, 0, st>>>((const T*)x, (T*)col, rows, g.h, g.w, g.c, g.p, g.q, g.r,
+                                                        g.s, g.pad, g.stride, kpitch);
     count_launch();
     return (int)cudaGetLastError();
+}
+
+// Gather col2im over the VALID taps only: for a dx pixel (h,w) the taps with
+// st | h+pad-r are r = r0, r0+st, ... with r0 = (h+pad) % st, and p steps down
+// by one per tap -- one division per pixel instead of two per tap.  One
+// thread per (pixel, channel group of V channels), channels fastest.
+template <class T, int V>
+__global__ void col2im_taps_kernel(const float* __restrict__ dcol, T* __restrict__ dx, int64_t pixels, int H,
+                                   int W, int C, int P, int Q, int R, int S, int pad, int st, int kpitch,
+                                   float alpha, float beta) {
+    const int CG = C / V;
+    const int64_t total = pixels * CG;
+    for (int64_t idx = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; idx < total;
+         idx += (int64_t)gridDim.x * blockDim.x) {
+        const int c0 = (int)(idx % CG) * V;
+        const int64_t pix = idx / CG;
+        const int w = (int)(pix % W);
+        const int64_t t2 = pix / W;
+        const int h = (int)(t2 % H);
+        const int n = (int)(t2 / H);
+        const int hp = h + pad, wp = w + pad;
+        const int r0 = hp % st, s0 = wp % st;
+        float acc[V];
+#pragma unroll
+        for (int v = 0; v < V; ++v) acc[v] = 0.f;
+        for (int r = r0, p = (hp - r0) / st; r < R && p >= 0; r += st, --p) {
+            if (p >= P) continue;
+            const float* rowp = dcol + ((int64_t)n * P + p) * Q * (int64_t)kpitch;
+            for (int s = s0, q = (wp - s0) / st; s < S && q >= 0; s += st, --q) {
+                if (q >= Q) continue;
+                const float* src = rowp + (int64_t)q * kpitch + (r * S + s) * C + c0;
+                if constexpr (V == 4) {
+                    const float4 f = *reinterpret_cast<const float4*>(src);
+                    acc[0] += f.x; acc[1] += f.y; acc[2] += f.z; acc[3] += f.w;
+                } else {
+#pragma unroll
+                    for (int v = 0; v < V; ++v) acc[v] += src[v];
+                }
+            }
+        }
+        T* out = dx + pix * C + c0;
+#pragma unroll
+        for (int v = 0; v < V; ++v) {
+            float o = alpha * acc[v];
+            if (beta != 0.f) o += beta * to_f<T>(out[v]);
+            out[v] = from_f<T>(o);
+        }
+    }
 }
 
 }  // namespace
@@ -311,14 +396,31 @@ int launch_pad_filter(const Geom& g, const void* w, void* wpad, int32_t kpitch, 
 
 int launch_col2im(const Geom& g, int32_t b, float alpha, const float* dcol, int32_t kpitch, float beta,
                   void* dx, cudaStream_t st) {
-    const int64_t total = (int64_t)b * g.h * g.w * g.c;
-    int grid = grid_for(total, 256);
-    if (g.math == MUCU_MATH_BF16)
-        col2im_kernel<__nv_bfloat16><<<grid, 256, 0, st>>>(dcol, (__nv_bfloat16*)dx, total, g.h, g.w, g.c, g.p, g.q,
-                                                          g.r, g.s, g.pad, g.stride, kpitch, alpha, beta);
-    else
-        col2im_kernel<float><<<grid, 256, 0, st>>>(dcol, (float*)dx, total, g.h, g.w, g.c, g.p, g.q, g.r, g.s,
-                                                  g.pad, g.stride, kpitch, alpha, beta);
+    const int64_t pixels = (int64_t)b * g.h * g.w;
+    const bool v4 = g.c % 4 == 0 && kpitch % 4 == 0;
+    const int grid = grid_for(pixels * (v4 ? g.c / 4 : g.c), 256);
+#define COL2IM(TT, VV)                                                                                            \
+    col2im_taps_kernel<TT, VV><<<grid, 256, 0, st>>>(dcol, (TT*)dx, pixels, g.h, g.w, g.c, g.p, g.q, g.r, g.s,   \
+                                                     g.pad, g.stride, kpitch, alpha, beta)
+    if (g.math == MUCU_MATH_BF16) {
+        if (v4) COL2IM(__nv_bfloat16, 4); else COL2IM(__nv_bfloat16, 1);
+    } else {
+        if (v4) COL2IM(float, 4); else COL2IM(float, 1);
+    }
+#undef COL2IM
+    count_launch();
+    return (int)cudaGetLastError();
+}
+
+namespace {
+__global__ void scale_kernel(float* __restrict__ p, int64_t n, float beta) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        p[i] = beta == 0.f ? 0.f : beta * p[i];
+}
+}  // namespace
+
+int launch_scale(int64_t n, float beta, float* p, cudaStream_t st) {
+    scale_kernel<<<grid_for(n, 256), 256, 0, st>>>(p, n, beta);
     count_launch();
     return (int)cudaGetLastError();
 }

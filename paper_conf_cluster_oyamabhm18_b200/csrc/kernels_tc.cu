@@ -297,6 +297,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
             }
         }
         const T* gx = (const T*)p.gsrc;
+        const int lag = min(S - 1, 3);
         for (int it = 0; it < nkb; ++it) {
             const int kb = kb_begin + it;
             const int s = it % S;
@@ -466,11 +467,16 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
             if constexpr (GATHER) {
                 if constexpr (A_ASYNC || B_ASYNC) {
                     cp_async_commit();
-                    // lagged arrive: stage it-1 is complete once at most 1 group is pending
-                    if (it > 0) {
-                        cp_async_wait<1>();
+                    // Lagged arrive: keep `lag` stages of gathers in flight per
+                    // thread (L2 latency hiding); stage it-lag is complete once at
+                    // most `lag` groups are pending.  lag <= S-1 keeps the ring
+                    // deadlock-free (the MMA can always drain stage it-S).
+                    if (it >= lag) {
+                        if (lag == 1) cp_async_wait<1>();
+                        else if (lag == 2) cp_async_wait<2>();
+                        else cp_async_wait<3>();
                         fence_proxy_async();
-                        mbar_arrive(smem_u32(&full[(it - 1) % S]));
+                        mbar_arrive(smem_u32(&full[(it - lag) % S]));
                     }
                 } else {
                     fence_proxy_async();
@@ -482,7 +488,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
             if (nkb > 0) {
                 cp_async_wait<0>();
                 fence_proxy_async();
-                mbar_arrive(smem_u32(&full[(nkb - 1) % S]));
+                for (int j = max(0, nkb - lag); j < nkb; ++j) mbar_arrive(smem_u32(&full[j % S]));
             }
         }
     } else {
@@ -530,15 +536,6 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
             outF += (size_t)z * p.batch_stride;
             outT += (size_t)z * p.batch_stride;
         }
-        if constexpr (EPI == EPI_WGRAD_CHAIN) {
-            const int tile = blockIdx.y * gridDim.x + blockIdx.x;
-            if (threadIdx.x == 128 && z > 0) {
-                volatile int32_t* vs = p.sem + tile;
-                while (*vs != z) __nanosleep(100);
-                __threadfence();
-            }
-            asm volatile("bar.sync 1, 128;" ::: "memory");
-        }
         for (int c0 = 0; c0 < p.BN; c0 += 32) {
             uint32_t v[32];
             if (nkb > 0) {
@@ -551,15 +548,21 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
             if (m >= p.M) continue;
             const int nb = n0 + c0;
             if constexpr (EPI == EPI_WGRAD_CHAIN) {
+                // dw += alpha * partial (beta was applied by a prescale launch);
+                // 16-byte vector reductions in L2 (red.global.add.v4.f32).
                 float* d = outF + (size_t)m * p.ldc + nb;
+                const bool vec = (nb + 32 <= p.N) && ((p.ldc & 3) == 0);
+                if (vec) {
 #pragma unroll
-                for (int j = 0; j < 32; ++j) {
-                    if (nb + j < p.N) {
-                        float o = p.alpha * __uint_as_float(v[j]);
-                        if (z > 0) o += d[j];
-                        else if (p.beta != 0.f) o += p.beta * d[j];
-                        d[j] = o;
-                    }
+                    for (int j = 0; j < 32; j += 4)
+                        asm volatile("red.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(d + j),
+                                     "f"(p.alpha * __uint_as_float(v[j])), "f"(p.alpha * __uint_as_float(v[j + 1])),
+                                     "f"(p.alpha * __uint_as_float(v[j + 2])), "f"(p.alpha * __uint_as_float(v[j + 3]))
+                                     : "memory");
+                } else {
+#pragma unroll
+                    for (int j = 0; j < 32; ++j)
+                        if (nb + j < p.N) atomicAdd(d + j, p.alpha * __uint_as_float(v[j]));
                 }
             } else if (p.out_bf16) {
                 __nv_bfloat16* d = (__nv_bfloat16*)outT + (size_t)m * p.ldc + nb;
@@ -601,14 +604,6 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                         }
                     }
                 }
-            }
-        }
-        if constexpr (EPI == EPI_WGRAD_CHAIN) {
-            __threadfence();
-            asm volatile("bar.sync 1, 128;" ::: "memory");
-            if (threadIdx.x == 128) {
-                const int tile = blockIdx.y * gridDim.x + blockIdx.x;
-                atomicExch(p.sem + tile, z + 1 < (int)gridDim.z ? z + 1 : 0);
             }
         }
     }
@@ -856,10 +851,17 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         A.M = g.k; A.N = (int)RSC; A.ldc = RSC; A.kred = (int)Mpix; A.gsrc = in0;
         finalize_tiling(L, elt);
         const int64_t tiles = ceil_div(A.N, A.BN) * ceil_div(A.M, 128);
-        if (tiles > sem.capacity) return -1;
         const int64_t nkb = ceil_div(Mpix, KB);
+        // Split the pixel reduction so that ~2 waves of CTAs run, each split
+        // >= 16 k-blocks (amortises TMEM alloc / pipeline fill).
         int64_t want = std::max<int64_t>(1, (2LL * num_sms + tiles - 1) / tiles);
-        int64_t nsplit = std::min<int64_t>(std::min<int64_t>(want, std::max<int64_t>(1, nkb / 4)), 65535);
+        int64_t nsplit = std::min<int64_t>(std::min<int64_t>(want, std::max<int64_t>(1, nkb / 16)), 65535);
+        // P:L58 output scale: apply the user's beta once, then every split adds.
+        if (beta != 1.f) {
+            err = launch_scale(g.k * RSC, beta, (float*)out, st);
+            if (err) return err;
+        }
+        (void)sem;
         A.kb_per_split = (int)ceil_div(nkb, nsplit);
         nsplit = ceil_div(nkb, A.kb_per_split);
         A.num_kb = (int)nkb;

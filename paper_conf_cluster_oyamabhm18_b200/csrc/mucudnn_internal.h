@@ -88,6 +88,7 @@ int launch_pad_filter(const Geom& g, const void* w, void* wpad, int32_t kpitch, 
 int launch_col2im(const Geom& g, int32_t b, float alpha, const float* dcol, int32_t kpitch, float beta,
                   void* dx, cudaStream_t st);
 int launch_wg_filter(const Geom& g, bool dgrad, const void* w, void* U, cudaStream_t st);
+int launch_scale(int64_t n, float beta, float* p, cudaStream_t st);  // p *= beta (beta == 0: p = 0)
 int launch_wg_input(const Geom& g, bool dgrad, int32_t b, const void* in, void* V, cudaStream_t st);
 int launch_wg_output(const Geom& g, bool dgrad, int32_t b, float alpha, const float* M, float beta,
                      void* out, cudaStream_t st);

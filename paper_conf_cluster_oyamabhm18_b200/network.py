@@ -109,6 +109,32 @@ class ConvNet:
         del scratch
         torch.cuda.empty_cache()
 
+    # File-based benchmark DB ("caches ... the benchmark results into ...
+    # optional file-based database", enabling offline benchmarking and sharing
+    # among homogeneous GPUs).  Keyed by descriptor, conv type and limit.
+    @staticmethod
+    def _db_key(k: Kernel, ws_limit: int, policy: str) -> str:
+        d = k.desc
+        return (f"{d.n},{d.c},{d.h},{d.w},{d.k},{d.r},{d.s},{d.pad},{d.stride},{d.math}|{k.conv_type}|"
+                f"{ws_limit}|{policy}")
+
+    def save_tables(self, path: str, ws_limit: int, policy: str):
+        arrs = {}
+        for k in self.kernels.values():
+            key = self._db_key(k, ws_limit, policy)
+            arrs[key + "|t"], arrs[key + "|w"] = k.table
+        np.savez(path, **arrs)
+
+    def load_tables(self, path: str, ws_limit: int, policy: str) -> bool:
+        """Fill every kernel's table from the DB; False if any entry is missing."""
+        db = np.load(path)
+        for k in self.kernels.values():
+            key = self._db_key(k, ws_limit, policy)
+            if key + "|t" not in db:
+                return False
+            k.table = (db[key + "|t"], db[key + "|w"])
+        return True
+
     def plan_wr(self, ws_limit: int):
         """WR: per-kernel DP on its timing table; one workspace per kernel."""
         for k in self.kernels.values():

@@ -1,0 +1,57 @@
+"""Summarise ncu outputs into profiles/: launch lists (csv) and --set full reports."""
+import csv
+import io
+import subprocess
+import sys
+from collections import defaultdict
+
+
+def launches(path):
+    """Per-kernel-name totals from an `ncu --metrics gpu__time_duration.sum --csv` log."""
+    txt = open(path).read()
+    start = txt.find('"ID"')
+    rows = list(csv.DictReader(io.StringIO(txt[start:])))
+    agg = defaultdict(lambda: [0, 0.0])
+    for r in rows:
+        if r.get("Metric Name") != "gpu__time_duration.sum":
+            continue
+        v = float(r["Metric Value"].replace(",", ""))
+        unit = r.get("Metric Unit", "")
+        us = v / 1e3 if unit == "nsecond" else v * 1e3 if unit == "msecond" else v
+        name = r["Kernel Name"].split("(")[0][:90]
+        agg[name][0] += 1
+        agg[name][1] += us
+    tot = sum(v[1] for v in agg.values())
+    out = [f"{'kernel':90s} {'launches':>8s} {'total_us':>12s} {'share':>7s}"]
+    for k, (n, us) in sorted(agg.items(), key=lambda kv: -kv[1][1]):
+        out.append(f"{k:90s} {n:8d} {us:12.1f} {us / tot:7.3f}")
+    out.append(f"TOTAL {tot:.1f} us over {sum(v[0] for v in agg.values())} launches")
+    return "\n".join(out)
+
+
+KEYS = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum", "gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed",
+        "sm__pipe_tensor_cycles_active.avg.pct_of_peak_sustained_elapsed", "sm__throughput.avg.pct_of_peak_sustained_elapsed",
+        "lts__t_bytes.sum", "launch__registers_per_thread", "launch__grid_size", "launch__shared_mem_per_block_dynamic",
+        "sm__warps_active.avg.pct_of_peak_sustained_active", "l1tex__t_bytes.sum", "sm__inst_executed_pipe_tensor.sum",
+        "smsp__pcsamp_warps_issue_stalled_long_scoreboard", "sm__cycles_elapsed.avg.per_second"]
+
+
+def full(path):
+    r = subprocess.run(["ncu", "-i", path, "--page", "raw", "--csv"], capture_output=True, text=True)
+    rows = list(csv.reader(io.StringIO(r.stdout)))
+    if len(rows) < 3:
+        return r.stdout + r.stderr
+    hdr, units = rows[0], rows[1]
+    out = []
+    for row in rows[2:]:
+        d = dict(zip(hdr, row))
+        out.append(f"== {d.get('Kernel Name', '')[:120]}")
+        for k in hdr:
+            if any(k.startswith(p) for p in KEYS) or "tensor" in k and "pct" in k:
+                out.append(f"  {k} = {d[k]} {units[hdr.index(k)]}")
+    return "\n".join(out)
+
+
+if __name__ == "__main__":
+    kind, path = sys.argv[1], sys.argv[2]
+    print(launches(path) if kind == "launches" else full(path))

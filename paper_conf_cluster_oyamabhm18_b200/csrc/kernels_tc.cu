@@ -71,6 +71,18 @@ __device__ __forceinline__ void tma_load_3d(uint32_t dst, const CUtensorMap* tm,
         "l"((uint64_t)tm), "r"(bar), "r"(c0), "r"(c1), "r"(c2)
         : "memory");
 }
+// TMA im2col mode (4-D NHWC tensor {C, W, H, N}): pixelsPerColumn consecutive
+// pixels starting at (w, h, n) (walking W, then H, then N inside the map's
+// bounding box with the map's traversal stride), channelsPerPixel channels
+// from c, each read at (w + off_w, h + off_h); zero outside the tensor.
+__device__ __forceinline__ void tma_load_im2col_4d(uint32_t dst, const CUtensorMap* tm, uint32_t bar, int c, int w,
+                                                   int h, int n, uint16_t off_w, uint16_t off_h) {
+    asm volatile(
+        "cp.async.bulk.tensor.4d.shared::cluster.global.im2col.mbarrier::complete_tx::bytes"
+        " [%0], [%1, {%3, %4, %5, %6}], [%2], {%7, %8};" ::"r"(dst),
+        "l"((uint64_t)tm), "r"(bar), "r"(c), "r"(w), "r"(h), "r"(n), "h"(off_w), "h"(off_h)
+        : "memory");
+}
 __device__ __forceinline__ void cp_async16(uint32_t dst, const void* src, bool valid) {
     asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(dst), "l"(src), "r"(valid ? 16 : 0) : "memory");
 }
@@ -126,6 +138,7 @@ enum AMode : int {
     A_GATHER_DGRAD = 4,// transposed-conv gather of dy, K-major, 16-B vectors (K % KB == 0)
     A_SCALAR_FWD = 5,  // implicit im2col of x, element-wise (any C)
     A_SCALAR_DGRAD = 6,// transposed-conv gather of dy, element-wise (any K)
+    A_TMA_IM2COL = 7,  // TMA im2col mode: FWD (x) or stride-1 DGRAD (dy, flipped taps), 128 pixels x KB channels
 };
 enum BMode : int {
     B_TMA_K2 = 0,      // dense K-major {K, cols}
@@ -136,6 +149,7 @@ enum BMode : int {
     B_SCALAR_K = 5,    // dense K-major rows with unaligned pitch, element-wise
     B_SCALAR_DGRAD = 6,// DGRAD filter view, element-wise (any C)
     B_SCALAR_WG = 7,   // WGRAD implicit im2col, element-wise (any C)
+    B_TMA_IM2COL = 8,  // WGRAD implicit im2col of x by TMA im2col mode, MN-major (KB pixels x 128 B per atom)
 };
 enum EpiMode : int { EPI_STORE = 0, EPI_WGRAD_CHAIN = 1 };
 
@@ -156,6 +170,9 @@ struct TcArgs {
     // scalar B source
     const void* bsrc;
     int ldb;
+    // TMA im2col (A_TMA_IM2COL): DGRAD flips the tap order (r,s) -> (R-1-r, S-1-s)
+    // and starts each output pixel at (h + pad - (R-1), w + pad - (S-1)) in dy.
+    int im2col_dgrad;
     // epilogue
     void* out;
     long long ldc;
@@ -219,9 +236,10 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
     constexpr int A_BYTES = 128 * 128;       // 128 rows x 128 B
     constexpr bool A_MN = (AM == A_TMA_MN2);
     constexpr bool B_MN = (BM_ == B_TMA_MN2 || BM_ == B_TMA_MN3 || BM_ == B_GATHER_WG || BM_ == B_SCALAR_DGRAD ||
-                           BM_ == B_SCALAR_WG);
-    constexpr bool A_TMA = (AM == A_TMA_K2 || AM == A_TMA_K3 || AM == A_TMA_MN2);
-    constexpr bool B_TMA = (BM_ == B_TMA_K2 || BM_ == B_TMA_K3 || BM_ == B_TMA_MN2 || BM_ == B_TMA_MN3);
+                           BM_ == B_SCALAR_WG || BM_ == B_TMA_IM2COL);
+    constexpr bool A_TMA = (AM == A_TMA_K2 || AM == A_TMA_K3 || AM == A_TMA_MN2 || AM == A_TMA_IM2COL);
+    constexpr bool B_TMA = (BM_ == B_TMA_K2 || BM_ == B_TMA_K3 || BM_ == B_TMA_MN2 || BM_ == B_TMA_MN3 ||
+                            BM_ == B_TMA_IM2COL);
     constexpr bool GATHER = !A_TMA || !B_TMA;
     constexpr bool A_ASYNC = (AM == A_GATHER_FWD || AM == A_GATHER_DGRAD);
     constexpr bool B_ASYNC = (BM_ == B_GATHER_WG);
@@ -277,7 +295,13 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
         // =========================== producers ===========================
         const int t = threadIdx.x;  // 0..127
         // Per-thread gather rows (A gathers: rows t/8 + 16 i, chunk t % 8).
-        int rn[8], rh[8], rw[8];
+        // Per-row origin (h, w) and base element offset, computed once per tile:
+        // FWD  row = output pixel (n,p,q): origin (p*st - pad, q*st - pad) in x,
+        //      element (r,s,c) at base + (r*W + s)*C + c;
+        // DGRAD row = dx pixel (n,h,w): dy index (h + pad - r, w + pad - s)
+        //      (stride 1: element (r,s,k) at base - (r*Q + s)*K + k).
+        int rh[8], rw[8];
+        long long rbase[8];
         bool rv[8];
         if constexpr (AM == A_GATHER_FWD || AM == A_GATHER_DGRAD) {
 #pragma unroll
@@ -285,23 +309,61 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                 const int m = m0 + t / 8 + 16 * i;
                 rv[i] = m < p.M;
                 const int mm = rv[i] ? m : 0;
-                if (AM == A_GATHER_FWD) {  // output pixel (n,p,q) -> input origin
+                if (AM == A_GATHER_FWD) {
                     const int pq = p.P * p.Q;
                     const int n = mm / pq, rem = mm - n * pq, pp = rem / p.Q, qq = rem - pp * p.Q;
-                    rn[i] = n; rh[i] = pp * p.stride - p.pad; rw[i] = qq * p.stride - p.pad;
-                } else {  // dx pixel (n,h,w)
+                    rh[i] = pp * p.stride - p.pad; rw[i] = qq * p.stride - p.pad;
+                    rbase[i] = (((long long)n * p.H + rh[i]) * p.W + rw[i]) * p.C;
+                } else {
                     const int hw = p.H * p.W;
                     const int n = mm / hw, rem = mm - n * hw, hh = rem / p.W, ww = rem - hh * p.W;
-                    rn[i] = n; rh[i] = hh + p.pad; rw[i] = ww + p.pad;
+                    rh[i] = hh + p.pad; rw[i] = ww + p.pad;
+                    rbase[i] = p.stride == 1 ? (((long long)n * p.P + rh[i]) * p.Q + rw[i]) * p.K
+                                             : (long long)n * p.P * p.Q * p.K;  // strided: image base
                 }
             }
         }
         const T* gx = (const T*)p.gsrc;
         const int lag = min(S - 1, 3);
-        for (int it = 0; it < nkb; ++it) {
+        // Incremental (r, s, c0) of the current k-block (no per-block division):
+        // a k-block covers KB consecutive channels of one filter tap.
+        constexpr bool WALK = (AM == A_GATHER_FWD || AM == A_GATHER_DGRAD || AM == A_TMA_IM2COL);
+        const int gch = (AM == A_GATHER_DGRAD || (AM == A_TMA_IM2COL && p.im2col_dgrad)) ? p.K : p.C;
+        int g_c0 = 0, g_s = 0, g_r = 0;
+        if constexpr (WALK) {
+            const int kk0 = kb_begin * KB;
+            const int rs = kk0 / gch;
+            g_c0 = kk0 - rs * gch; g_r = rs / p.S; g_s = rs - g_r * p.S;
+        }
+        // TMA im2col start pixel of this tile (FWD: output pixel m0 -> x origin;
+        // DGRAD: dx pixel m0 -> dy origin h + pad - (R-1)).
+        int ic_w = 0, ic_h = 0, ic_n = 0;
+        if constexpr (AM == A_TMA_IM2COL) {
+            if (p.im2col_dgrad) {
+                const int hw = p.H * p.W;
+                ic_n = m0 / hw;
+                const int rem = m0 - ic_n * hw, hh = rem / p.W, ww = rem - hh * p.W;
+                ic_h = hh + p.pad - (p.R - 1); ic_w = ww + p.pad - (p.S - 1);
+            } else {
+                const int pq = p.P * p.Q;
+                ic_n = m0 / pq;
+                const int rem = m0 - ic_n * pq, pp = rem / p.Q, qq = rem - pp * p.Q;
+                ic_h = pp * p.stride - p.pad; ic_w = qq * p.stride - p.pad;
+            }
+        }
+        // WGRAD TMA im2col: pixel (n,p,q) of the first row of the k-block, walked
+        // incrementally (KB pixels per k-block).
+        int wb_n = 0, wb_p = 0, wb_q = 0;
+        if constexpr (BM_ == B_TMA_IM2COL) {
+            const int m = kb_begin * KB, pq = p.P * p.Q;
+            wb_n = m / pq;
+            const int rem = m - wb_n * pq;
+            wb_p = rem / p.Q; wb_q = rem - wb_p * p.Q;
+        }
+        int s = 0;
+        uint32_t ph = 0;
+        for (int it = 0; it < nkb; ++it, s = (s + 1 == S) ? 0 : s + 1, ph ^= (s == 0) ? 1u : 0u) {
             const int kb = kb_begin + it;
-            const int s = it % S;
-            const uint32_t ph = (uint32_t)(it / S) & 1u;
             mbar_wait(smem_u32(&empty[s]), ph ^ 1u);
             const uint32_t aT = smem_u32(sA + (size_t)s * A_BYTES);
             const uint32_t bT = smem_u32(sB + (size_t)s * B_BYTES);
@@ -331,40 +393,72 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                     for (int a = 0; a < p.bn_atoms; ++a)
                         tma_load_3d(bT + a * KB * 128, &tmB, fb, n0 + a * (128 / ELT), rs, k0);
                 }
+                if constexpr (AM == A_TMA_IM2COL) {
+                    // 128 consecutive output pixels x KB channels of tap (r,s) in one TMA
+                    const uint16_t ow = (uint16_t)(p.im2col_dgrad ? p.S - 1 - g_s : g_s);
+                    const uint16_t oh = (uint16_t)(p.im2col_dgrad ? p.R - 1 - g_r : g_r);
+                    tma_load_im2col_4d(aT, &tmA, fb, g_c0, ic_w, ic_h, ic_n, ow, oh);
+                }
+                if constexpr (BM_ == B_TMA_IM2COL) {
+                    // atom a = 128 B of channels (c0..) of tap (r,s) for KB pixels
+                    const int h0 = wb_p * p.stride - p.pad, w0 = wb_q * p.stride - p.pad;
+                    for (int a = 0; a < p.bn_atoms; ++a) {
+                        const int j0 = n0 + a * (128 / ELT);
+                        const int rs = j0 / p.C, c0 = j0 - rs * p.C;
+                        const int r = rs / p.S, sx = rs - r * p.S;
+                        tma_load_im2col_4d(bT + a * KB * 128, &tmB, fb, c0, w0, h0, wb_n, (uint16_t)sx, (uint16_t)r);
+                    }
+                }
+            }
+            if constexpr (BM_ == B_TMA_IM2COL) {
+                wb_q += KB;
+                while (wb_q >= p.Q) { wb_q -= p.Q; if (++wb_p == p.P) { wb_p = 0; ++wb_n; } }
             }
             // ---- A gathers ----
             if constexpr (AM == A_GATHER_FWD) {
-                const int kk0 = kb * KB;
-                const int rs = kk0 / p.C, c0 = kk0 - rs * p.C + (t & 7) * (16 / ELT);
-                const int r = rs / p.S, sx = rs - r * p.S;
-                const bool kin = rs < p.R * p.S;
+                const int r = g_r, sx = g_s;
+                const bool kin = r < p.R;
+                const long long koff = ((long long)r * p.W + sx) * p.C + g_c0 + (t & 7) * (16 / ELT);
+                const uint32_t soff = kmaj_off(t / 8, (t & 7) * 16);
 #pragma unroll
                 for (int i = 0; i < 8; ++i) {
-                    const int row = t / 8 + 16 * i;
-                    const int h = rh[i] + r, w = rw[i] + sx;
-                    const bool v = kin && rv[i] && h >= 0 && h < p.H && w >= 0 && w < p.W;
-                    const T* src = v ? gx + (((size_t)rn[i] * p.H + h) * p.W + w) * p.C + c0 : gx;
-                    cp_async16(aT + kmaj_off(row, (t & 7) * 16), src, v);
+                    const bool v = kin && rv[i] && (unsigned)(rh[i] + r) < (unsigned)p.H &&
+                                   (unsigned)(rw[i] + sx) < (unsigned)p.W;
+                    cp_async16(aT + soff + i * 2048, v ? gx + rbase[i] + koff : gx, v);
                 }
             } else if constexpr (AM == A_GATHER_DGRAD) {
-                const int kk0 = kb * KB;
-                const int rs = kk0 / p.K, k0 = kk0 - rs * p.K + (t & 7) * (16 / ELT);
-                const int r = rs / p.S, sx = rs - r * p.S;
-                const bool kin = rs < p.R * p.S;
+                const int r = g_r, sx = g_s;
+                const bool kin = r < p.R;
+                const int kc = g_c0 + (t & 7) * (16 / ELT);
+                const uint32_t soff = kmaj_off(t / 8, (t & 7) * 16);
+                if (p.stride == 1) {
+                    const long long koff = kc - ((long long)r * p.Q + sx) * p.K;
 #pragma unroll
-                for (int i = 0; i < 8; ++i) {
-                    const int row = t / 8 + 16 * i;
-                    const int ph_ = rh[i] - r, pw_ = rw[i] - sx;
-                    bool v = kin && rv[i] && ph_ >= 0 && pw_ >= 0;
-                    int pp = 0, qq = 0;
-                    if (v) {
-                        pp = ph_ / p.stride; qq = pw_ / p.stride;
-                        v = (pp * p.stride == ph_) && (qq * p.stride == pw_) && pp < p.P && qq < p.Q;
+                    for (int i = 0; i < 8; ++i) {
+                        const bool v = kin && rv[i] && (unsigned)(rh[i] - r) < (unsigned)p.P &&
+                                       (unsigned)(rw[i] - sx) < (unsigned)p.Q;
+                        cp_async16(aT + soff + i * 2048, v ? gx + rbase[i] + koff : gx, v);
                     }
-                    const T* src = v ? gx + (((size_t)rn[i] * p.P + pp) * p.Q + qq) * p.K + k0 : gx;
-                    cp_async16(aT + kmaj_off(row, (t & 7) * 16), src, v);
+                } else {
+#pragma unroll
+                    for (int i = 0; i < 8; ++i) {
+                        const int ph_ = rh[i] - r, pw_ = rw[i] - sx;
+                        bool v = kin && rv[i] && ph_ >= 0 && pw_ >= 0;
+                        int pp = 0, qq = 0;
+                        if (v) {
+                            pp = ph_ / p.stride; qq = pw_ / p.stride;
+                            v = (pp * p.stride == ph_) && (qq * p.stride == pw_) && pp < p.P && qq < p.Q;
+                        }
+                        const T* src = v ? gx + rbase[i] + ((long long)pp * p.Q + qq) * p.K + kc : gx;
+                        cp_async16(aT + soff + i * 2048, src, v);
+                    }
                 }
-            } else if constexpr (AM == A_SCALAR_FWD) {
+            }
+            if constexpr (WALK) {
+                g_c0 += KB;
+                if (g_c0 >= gch) { g_c0 = 0; if (++g_s == p.S) { g_s = 0; ++g_r; } }
+            }
+            if constexpr (AM == A_SCALAR_FWD) {
                 // thread t owns row t; KB elements, kk = (r,s,c) decomposed each
                 const int m = m0 + t;
                 const bool rvalid = m < p.M;
@@ -476,7 +570,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                         else if (lag == 2) cp_async_wait<2>();
                         else cp_async_wait<3>();
                         fence_proxy_async();
-                        mbar_arrive(smem_u32(&full[(it - lag) % S]));
+                        mbar_arrive(smem_u32(&full[s - lag < 0 ? s - lag + S : s - lag]));
                     }
                 } else {
                     fence_proxy_async();
@@ -497,9 +591,9 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
             const uint32_t idesc = (1u << 4) | (Elt<ELT>::fmt << 7) | (Elt<ELT>::fmt << 10) |
                                    ((A_MN ? 1u : 0u) << 15) | ((B_MN ? 1u : 0u) << 16) |
                                    ((uint32_t)(p.BN >> 3) << 17) | ((128u >> 4) << 24);
-            for (int it = 0; it < nkb; ++it) {
-                const int s = it % S;
-                const uint32_t ph = (uint32_t)(it / S) & 1u;
+            int s = 0;
+            uint32_t ph = 0;
+            for (int it = 0; it < nkb; ++it, s = (s + 1 == S) ? 0 : s + 1, ph ^= (s == 0) ? 1u : 0u) {
                 mbar_wait(smem_u32(&full[s]), ph);
                 tc_fence_after();
                 if (lane == 0) {
@@ -650,6 +744,55 @@ bool make_map(CUtensorMap* tm, int elt, const void* base, int rank, const uint64
     return r == CUDA_SUCCESS;
 }
 
+typedef CUresult (*EncodeIm2colFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
+                                   const cuuint64_t*, const int*, const int*, cuuint32_t, cuuint32_t,
+                                   const cuuint32_t*, CUtensorMapInterleave, CUtensorMapSwizzle,
+                                   CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+EncodeIm2colFn get_encode_im2col() {
+    static EncodeIm2colFn fn = nullptr;
+    static std::once_flag once;
+    std::call_once(once, [] {
+        void* p = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuTensorMapEncodeIm2col", &p, cudaEnableDefault, &q) == cudaSuccess &&
+            q == cudaDriverEntryPointSuccess)
+            fn = (EncodeIm2colFn)p;
+    });
+    return fn;
+}
+
+// TMA im2col map over an NHWC tensor viewed as {C, W, H, N}.  The bounding box
+// of start pixels is [lower, dim - 1 + upper] per spatial dim (W, H order),
+// walked with the traversal stride; channelsPerPixel = 128 B of channels.
+bool make_im2col_map(CUtensorMap* tm, int elt, const void* base, int C, int W, int H, int N, int lower_w,
+                     int lower_h, int upper_w, int upper_h, int pixels, int stride, bool mn_major) {
+    EncodeIm2colFn enc = get_encode_im2col();
+    if (!enc) return false;
+    if (lower_w < -128 || lower_h < -128 || upper_w > 127 || upper_h > 127 || lower_w > 127 || upper_h < -128)
+        return false;
+    cuuint64_t d[4] = {(cuuint64_t)C, (cuuint64_t)W, (cuuint64_t)H, (cuuint64_t)N};
+    cuuint64_t s[3] = {(cuuint64_t)C * elt, (cuuint64_t)W * C * elt, (cuuint64_t)H * W * C * elt};
+    int lo[2] = {lower_w, lower_h}, hi[2] = {upper_w, upper_h};
+    cuuint32_t es[4] = {1, (cuuint32_t)stride, (cuuint32_t)stride, 1};
+    const CUtensorMapSwizzle sw = (mn_major && elt == 4) ? CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B : CU_TENSOR_MAP_SWIZZLE_128B;
+    CUresult r = enc(tm, elt == 2 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4,
+                     const_cast<void*>(base), d, s, lo, hi, (cuuint32_t)(128 / elt), (cuuint32_t)pixels, es,
+                     CU_TENSOR_MAP_INTERLEAVE_NONE, sw, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                     CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    return r == CUDA_SUCCESS;
+}
+
+// MUCU_TMA_IM2COL=0 forces the cp.async gather producers (A/B comparison, tests).
+bool use_tma_im2col() {
+    static int v = -1;
+    if (v < 0) {
+        const char* e = getenv("MUCU_TMA_IM2COL");
+        v = (e && e[0] == '0') ? 0 : 1;
+    }
+    return v == 1;
+}
+
 int pick_bn(int N) {
     if (N >= 256 && N % 256 == 0) return 256;
     if (N % 192 == 0 && N <= 384) return 192;
@@ -742,6 +885,12 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
             A.num_kb = (int)ceil_div(RSC, KB);
             if (!waligned) return -1;
             if (!map2(&L.tb, in1, RSC, g.k, RSC, KB, A.BN)) return -1;
+            if (use_tma_im2col() &&
+                make_im2col_map(&L.ta, elt, in0, g.c, g.w, g.h, b, -g.pad, -g.pad, g.pad - (g.s - 1),
+                                g.pad - (g.r - 1), 128, g.stride, false)) {
+                A.tma_bytes = 128 * 128 + A.BN * 128;
+                return LAUNCH(A_TMA_IM2COL, B_TMA_K2, EPI_STORE);
+            }
             A.tma_bytes = A.BN * 128;
             err = LAUNCH(A_GATHER_FWD, B_TMA_K2, EPI_STORE);
         } else {
@@ -813,6 +962,15 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         if ((g.c * elt) % 16 == 0 && g.c >= atom) {
             // w viewed as {C, R*S, K} (c contiguous): B(c, (r,s,k)) MN-major
             if (!map3(&L.tb, in1, g.c, RS, g.k, g.c, RSC, atom, 1, KB, true)) return -1;
+            // stride 1: im2col of dy with pad' = R-1-pad and flipped taps
+            const int lw = g.pad - (g.s - 1), lh = g.pad - (g.r - 1);
+            if (g.stride == 1 && use_tma_im2col() &&
+                make_im2col_map(&L.ta, elt, in0, g.k, g.q, g.p, b, lw, lh, lw + g.w - g.q, lh + g.h - g.p, 128, 1,
+                                false)) {
+                A.im2col_dgrad = 1;
+                A.tma_bytes = 128 * 128 + A.bn_atoms * KB * 128;
+                return LAUNCH(A_TMA_IM2COL, B_TMA_MN3, EPI_STORE);
+            }
             A.tma_bytes = A.bn_atoms * KB * 128;
             return LAUNCH(A_GATHER_DGRAD, B_TMA_MN3, EPI_STORE);
         }
@@ -880,6 +1038,12 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
             if (!map2(&L.tb, colp, RSC, (uint64_t)Mpix, kp, atom, KB, true)) return -1;
             A.tma_bytes = a_bytes + A.bn_atoms * KB * 128;
             return LAUNCH(A_TMA_MN2, B_TMA_MN2, EPI_WGRAD_CHAIN);
+        }
+        if (g.c % atom == 0 && use_tma_im2col() &&
+            make_im2col_map(&L.tb, elt, in0, g.c, g.w, g.h, b, -g.pad, -g.pad, g.pad - (g.s - 1), g.pad - (g.r - 1),
+                            KB, g.stride, true)) {
+            A.tma_bytes = a_bytes + A.bn_atoms * KB * 128;
+            return LAUNCH(A_TMA_MN2, B_TMA_IM2COL, EPI_WGRAD_CHAIN);
         }
         A.tma_bytes = a_bytes;
         if (g.c % atom == 0) return LAUNCH(A_TMA_MN2, B_GATHER_WG, EPI_WGRAD_CHAIN);

@@ -204,3 +204,15 @@ def test_benchmark_dp_execute_end_to_end(math):
         got, _ = run_gpu(d, conv_type, plan, x, w, dy)
         assert np.array_equal(got, ref)
     h.set_policy(mu.POLICY_POW2)
+
+
+def test_cp_async_gather_producers_still_exact():
+    """The cp.async gather producers (used when TMA im2col does not apply) are
+    re-run on the vector-path shapes with TMA im2col disabled."""
+    import os
+    import subprocess
+    import sys
+    env = dict(os.environ, MUCU_TMA_IM2COL="0")
+    r = subprocess.run([sys.executable, "-m", "pytest", "-q", "-x", os.path.abspath(__file__), "-k",
+                        "(c64 or c128) and not cp_async"], env=env, capture_output=True, text=True)
+    assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-2000:]

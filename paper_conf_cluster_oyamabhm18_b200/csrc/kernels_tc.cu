@@ -173,6 +173,12 @@ struct TcArgs {
     // TMA im2col (A_TMA_IM2COL): DGRAD flips the tap order (r,s) -> (R-1-r, S-1-s)
     // and starts each output pixel at (h + pad - (R-1), w + pad - (S-1)) in dy.
     int im2col_dgrad;
+    // Strided DGRAD phase decomposition: dx pixels with (h+pad) % st == r0 and
+    // (w+pad) % st == s0 see only taps r = r0 + st*a (a < tapR), s = s0 + st*b
+    // (b < tapS), and dy row p = i - a: a stride-1 transposed conv on an
+    // (ph_H x ph_W) sub-grid.  tapR/tapS = R/S when not in phase mode.
+    int ph_mode, ph_H, ph_W, ph_i0, ph_j0, ph_r0, ph_s0, ph_hb, ph_wb;
+    int tapR, tapS;
     // epilogue
     void* out;
     long long ldc;
@@ -183,6 +189,14 @@ struct TcArgs {
 };
 
 constexpr int kThreads = 256;
+
+// DGRAD reduction tap index -> filter tap r*S+s (phase mode: the sub-filter
+// tap (a,b) is (r0 + st*a, s0 + st*b)).
+__device__ __forceinline__ int dgrad_tap_rs(const TcArgs& p, int tap) {
+    if (!p.ph_mode) return tap;
+    const int a = tap / p.tapS, b = tap - a * p.tapS;
+    return (p.ph_r0 + p.stride * a) * p.S + p.ph_s0 + p.stride * b;
+}
 
 template <int ELT>
 struct Elt;
@@ -333,13 +347,19 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
         if constexpr (WALK) {
             const int kk0 = kb_begin * KB;
             const int rs = kk0 / gch;
-            g_c0 = kk0 - rs * gch; g_r = rs / p.S; g_s = rs - g_r * p.S;
+            g_c0 = kk0 - rs * gch; g_r = rs / p.tapS; g_s = rs - g_r * p.tapS;
         }
         // TMA im2col start pixel of this tile (FWD: output pixel m0 -> x origin;
-        // DGRAD: dx pixel m0 -> dy origin h + pad - (R-1)).
+        // DGRAD: dx pixel m0 -> dy origin h + pad - (R-1); phase mode: sub-grid
+        // pixel (ii, jj) -> dy origin (i0 + ii - (tapR-1), j0 + jj - (tapS-1))).
         int ic_w = 0, ic_h = 0, ic_n = 0;
         if constexpr (AM == A_TMA_IM2COL) {
-            if (p.im2col_dgrad) {
+            if (p.ph_mode) {
+                const int hw = p.ph_H * p.ph_W;
+                ic_n = m0 / hw;
+                const int rem = m0 - ic_n * hw, ii = rem / p.ph_W, jj = rem - ii * p.ph_W;
+                ic_h = p.ph_i0 + ii - (p.tapR - 1); ic_w = p.ph_j0 + jj - (p.tapS - 1);
+            } else if (p.im2col_dgrad) {
                 const int hw = p.H * p.W;
                 ic_n = m0 / hw;
                 const int rem = m0 - ic_n * hw, hh = rem / p.W, ww = rem - hh * p.W;
@@ -389,14 +409,15 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                 if constexpr (BM_ == B_TMA_MN3) {
                     // k-block kb covers (r,s) = kb / (K/KB), k0 = (kb % (K/KB)) * KB
                     const int kpr = p.K / KB;
-                    const int rs = kb / kpr, k0 = (kb - rs * kpr) * KB;
+                    const int tap = kb / kpr, k0 = (kb - tap * kpr) * KB;
+                    const int rs = dgrad_tap_rs(p, tap);
                     for (int a = 0; a < p.bn_atoms; ++a)
                         tma_load_3d(bT + a * KB * 128, &tmB, fb, n0 + a * (128 / ELT), rs, k0);
                 }
                 if constexpr (AM == A_TMA_IM2COL) {
                     // 128 consecutive output pixels x KB channels of tap (r,s) in one TMA
-                    const uint16_t ow = (uint16_t)(p.im2col_dgrad ? p.S - 1 - g_s : g_s);
-                    const uint16_t oh = (uint16_t)(p.im2col_dgrad ? p.R - 1 - g_r : g_r);
+                    const uint16_t ow = (uint16_t)(p.im2col_dgrad ? p.tapS - 1 - g_s : g_s);
+                    const uint16_t oh = (uint16_t)(p.im2col_dgrad ? p.tapR - 1 - g_r : g_r);
                     tma_load_im2col_4d(aT, &tmA, fb, g_c0, ic_w, ic_h, ic_n, ow, oh);
                 }
                 if constexpr (BM_ == B_TMA_IM2COL) {
@@ -456,7 +477,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
             }
             if constexpr (WALK) {
                 g_c0 += KB;
-                if (g_c0 >= gch) { g_c0 = 0; if (++g_s == p.S) { g_s = 0; ++g_r; } }
+                if (g_c0 >= gch) { g_c0 = 0; if (++g_s == p.tapS) { g_s = 0; ++g_r; } }
             }
             if constexpr (AM == A_SCALAR_FWD) {
                 // thread t owns row t; KB elements, kk = (r,s,c) decomposed each
@@ -536,7 +557,8 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                     const int j = n0 + jj, kk = kb * KB + krow;
                     float v = 0.f;
                     if (j < p.N && kk < p.kred) {
-                        const int rs = kk / p.K, k = kk - rs * p.K;
+                        const int tap = kk / p.K, k = kk - tap * p.K;
+                        const int rs = dgrad_tap_rs(p, tap);
                         v = (float)bs[((size_t)k * RS + rs) * p.C + j];
                     }
                     st_shared_elt<T>(bT + mnmaj_off<ELT>(jj, krow, KB), (T)v);
@@ -623,6 +645,13 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
         const int q4 = warp & 3;
         const int row = q4 * 32 + lane;
         const int m = m0 + row;
+        // Output row of GEMM row m (phase mode scatters sub-grid rows back to dx).
+        long long mrow = m;
+        if (p.ph_mode && m < p.M) {
+            const int hw = p.ph_H * p.ph_W;
+            const int n = m / hw, rem = m - n * hw, ii = rem / p.ph_W, jj = rem - ii * p.ph_W;
+            mrow = ((long long)n * p.H + p.ph_hb + p.stride * ii) * p.W + p.ph_wb + p.stride * jj;
+        }
         const uint32_t taddr_row = tmem + ((uint32_t)(q4 * 32) << 16);
         float* outF = (float*)p.out;
         T* outT = (T*)p.out;
@@ -659,7 +688,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                         if (nb + j < p.N) atomicAdd(d + j, p.alpha * __uint_as_float(v[j]));
                 }
             } else if (p.out_bf16) {
-                __nv_bfloat16* d = (__nv_bfloat16*)outT + (size_t)m * p.ldc + nb;
+                __nv_bfloat16* d = (__nv_bfloat16*)outT + (size_t)mrow * p.ldc + nb;
                 const bool vec = (nb + 32 <= p.N) && ((p.ldc & 7) == 0) && p.beta == 0.f;
                 if (vec) {
 #pragma unroll
@@ -680,7 +709,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                     }
                 }
             } else {
-                float* d = outF + (size_t)m * p.ldc + nb;
+                float* d = outF + (size_t)mrow * p.ldc + nb;
                 const bool vec = (nb + 32 <= p.N) && ((p.ldc & 3) == 0) && p.beta == 0.f;
                 if (vec) {
 #pragma unroll
@@ -793,14 +822,17 @@ bool use_tma_im2col() {
     return v == 1;
 }
 
-int pick_bn(int N) {
-    if (N >= 256 && N % 256 == 0) return 256;
-    if (N % 192 == 0 && N <= 384) return 192;
-    if (N >= 128) return (N % 256 == 0) ? 256 : 128;
-    if (N > 64) return 128;
-    if (N > 32) return 64;
-    if (N > 16) return 32;
-    return 16;
+// Tile N: a multiple of `step` (16 = UMMA granularity at M = 128; an MN-major
+// atom when a tile must not split a 128-B channel atom) up to 256, minimising
+// the padded columns plus a per-tile overhead (~32 columns); ties -> larger.
+int pick_bn(int N, int step = 32) {
+    step = std::max(step, 32);  // the epilogue drains TMEM in 32-column chunks
+    int best = step, best_cost = 1 << 30;
+    for (int bn = step; bn <= 256; bn += step) {
+        const int cost = (int)ceil_div(N, bn) * (bn + 32);
+        if (cost <= best_cost) { best = bn; best_cost = cost; }
+    }
+    return best;
 }
 
 struct Launch {
@@ -824,9 +856,9 @@ int launch_t(Launch& L, cudaStream_t st) {
     return (int)cudaGetLastError();
 }
 
-void finalize_tiling(Launch& L, int elt) {
+void finalize_tiling(Launch& L, int elt, int step = 32) {
     TcArgs& a = L.a;
-    a.BN = pick_bn(a.N);
+    a.BN = pick_bn(a.N, step);
     a.tmem_cols = a.BN <= 32 ? 32 : a.BN <= 64 ? 64 : a.BN <= 128 ? 128 : 256;
     a.bn_atoms = (a.BN * elt + 127) / 128;
     a.b_bytes = std::max(a.BN * 128, a.bn_atoms * (128 / elt) * 128);
@@ -854,6 +886,7 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
     TcArgs& A = L.a;
     A.H = g.h; A.W = g.w; A.C = g.c; A.P = g.p; A.Q = g.q; A.R = g.r; A.S = g.s; A.pad = g.pad;
     A.stride = g.stride; A.K = g.k;
+    A.tapR = g.r; A.tapS = g.s;
     A.alpha = alpha; A.beta = beta; A.out = out; A.out_bf16 = bf ? 1 : 0; A.sem = sem.sem;
     auto map2 = [&](CUtensorMap* tm, const void* base, uint64_t d0, uint64_t d1, uint64_t pitch_elems, uint32_t b0,
                     uint32_t b1, bool mn = false) {
@@ -952,6 +985,46 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         if (err) return err;
         return launch_wg_output(g, dg, b, alpha, Mx, beta, out, st);
     }
+    if (type == MUCU_BWD_DATA && algo == MUCU_ALGO_IMPLICIT_GEMM && g.stride > 1 && g.k % KB == 0 &&
+        use_tma_im2col()) {
+        // Strided DGRAD by phase decomposition: one stride-1 transposed conv per
+        // phase (r0, s0) over the dx sub-grid it owns, with only its
+        // ceil((R-r0)/st) x ceil((S-s0)/st) taps -- no masked (zero) taps.
+        const bool bvec = (g.c * elt) % 16 == 0 && g.c >= atom;
+        if (bvec && !map3(&L.tb, in1, g.c, RS, g.k, g.c, RSC, atom, 1, KB, true)) return -1;
+        A.gsrc = in0; A.bsrc = in1; A.ldc = g.c; A.N = g.c;
+        A.ph_mode = 1; A.im2col_dgrad = 1;
+        finalize_tiling(L, elt);
+        for (int r0 = 0; r0 < g.stride; ++r0) {
+            for (int s0 = 0; s0 < g.stride; ++s0) {
+                // dx rows with (h + pad) % st == r0: h = r0 - pad + st*i, i >= i0
+                const int i0 = std::max(0, (int)ceil_div(g.pad - r0, g.stride));
+                const int j0 = std::max(0, (int)ceil_div(g.pad - s0, g.stride));
+                const int hb = r0 - g.pad + g.stride * i0, wb = s0 - g.pad + g.stride * j0;
+                const int Hph = hb < g.h ? (int)ceil_div(g.h - hb, g.stride) : 0;
+                const int Wph = wb < g.w ? (int)ceil_div(g.w - wb, g.stride) : 0;
+                if (Hph <= 0 || Wph <= 0) continue;
+                const int nr = r0 < g.r ? (int)ceil_div(g.r - r0, g.stride) : 0;
+                const int ns = s0 < g.s ? (int)ceil_div(g.s - s0, g.stride) : 0;
+                A.ph_H = Hph; A.ph_W = Wph; A.ph_i0 = i0; A.ph_j0 = j0; A.ph_r0 = r0; A.ph_s0 = s0;
+                A.ph_hb = hb; A.ph_wb = wb; A.tapR = std::max(nr, 1); A.tapS = std::max(ns, 1);
+                A.M = b * Hph * Wph;
+                A.num_kb = (nr > 0 && ns > 0) ? nr * ns * (g.k / KB) : 0;  // 0 taps: dx = beta * dx
+                A.kred = nr * ns * g.k;
+                grid2(1);
+                // dy im2col: start positions i0 - (nr-1) ... (Hph of them), stride 1
+                const int lh = i0 - (A.tapR - 1), lw = j0 - (A.tapS - 1);
+                if (A.num_kb > 0 &&
+                    !make_im2col_map(&L.ta, elt, in0, g.k, g.q, g.p, b, lw, lh, lw + Wph - g.q, lh + Hph - g.p,
+                                     128, 1, false))
+                    return -1;
+                A.tma_bytes = 128 * 128 + (bvec ? A.bn_atoms * KB * 128 : 0);
+                err = bvec ? LAUNCH(A_TMA_IM2COL, B_TMA_MN3, EPI_STORE) : LAUNCH(A_TMA_IM2COL, B_SCALAR_DGRAD, EPI_STORE);
+                if (err) return err;
+            }
+        }
+        return 0;
+    }
     if (type == MUCU_BWD_DATA && algo == MUCU_ALGO_IMPLICIT_GEMM) {
         A.M = (int)(b * HW); A.N = g.c; A.num_kb = (int)ceil_div((int64_t)RS * g.k, KB); A.ldc = g.c;
         A.gsrc = in0; A.kred = RS * g.k;
@@ -1007,7 +1080,9 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         // dw[k][(r,s,c)] = sum_m dy[m][k] B(m, (r,s,c)); A = dy MN-major via TMA.
         const int64_t Mpix = (int64_t)b * PQ;
         A.M = g.k; A.N = (int)RSC; A.ldc = RSC; A.kred = (int)Mpix; A.gsrc = in0;
-        finalize_tiling(L, elt);
+        // implicit-im2col B producers load whole 128-B channel atoms of one tap:
+        // N tiles must start on an atom boundary.
+        finalize_tiling(L, elt, (algo == MUCU_ALGO_IMPLICIT_GEMM && g.c % atom == 0) ? atom : 16);
         const int64_t tiles = ceil_div(A.N, A.BN) * ceil_div(A.M, 128);
         const int64_t nkb = ceil_div(Mpix, KB);
         // Split the pixel reduction so that ~2 waves of CTAs run, each split

@@ -313,19 +313,94 @@ __global__ void im2col_rows_kernel(const T* __restrict__ x, T* __restrict__ col,
     }
 }
 
+// Small-C im2col (C not a multiple of the vector width, e.g. the RGB first
+// layer): one thread per 16-byte chunk of a col row, so every store is a full
+// coalesced 16-B vector; the chunk's V elements are gathered walking (r, s*C+c)
+// incrementally from one division (reads hit L1/L2: neighbouring chunks share
+// the same input rows).
+template <class T>
+__global__ void im2col_chunk_kernel(const T* __restrict__ x, T* __restrict__ col, int64_t rows, int H, int W,
+                                    int C, int P, int Q, int R, int S, int pad, int st, int kpitch) {
+    constexpr int V = 16 / sizeof(T);
+    const int SC = S * C, RSC = R * SC;
+    const int cpr = kpitch / V;
+    const int64_t total = rows * cpr;
+    const int pq = P * Q;
+    for (int64_t idx = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; idx < total;
+         idx += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t m = idx / cpr;
+        const int kk0 = (int)(idx - m * cpr) * V;
+        const int n = (int)(m / pq);
+        const int rem = (int)(m - (int64_t)n * pq);
+        const int p = rem / Q, q = rem - (rem / Q) * Q;
+        const int h0 = p * st - pad, w0 = q * st - pad;
+        const int lo = max(0, -w0) * C, hi = min(S, W - w0) * C;
+        int r = kk0 / SC, sc = kk0 - r * SC;
+        const T* xn = x + (int64_t)n * H * W * C + (int64_t)w0 * C;
+        __align__(16) T v[V];
+#pragma unroll
+        for (int e = 0; e < V; ++e) {
+            T val = from_f<T>(0.f);
+            const int h = h0 + r;
+            if (r < R && sc >= lo && sc < hi && h >= 0 && h < H) val = xn[(int64_t)h * W * C + sc];
+            v[e] = val;
+            if (++sc == SC) { sc = 0; ++r; }
+        }
+        *reinterpret_cast<uint4*>(col + m * kpitch + kk0) = *reinterpret_cast<const uint4*>(v);
+        (void)RSC;
+    }
+}
+
 template <class T>
 int im2col_t(const Geom& g, int32_t b, const void* x, void* col, int32_t kpitch, cudaStream_t st) {
     constexpr int V = 16 / sizeof(T);
     const int64_t rows = (int64_t)b * g.p * g.q;
-    const int grid = grid_for(rows * 32, 256);
-    if (g.c % V == 0 && kpitch % V == 0)
+    if (g.c % V == 0 && kpitch % V == 0) {
+        const int grid = grid_for(rows * 32, 256);
         im2col_rows_kernel<T, V><<<grid, 256, 0, st>>>((const T*)x, (T*)col, rows, g.h, g.w, g.c, g.p, g.q, g.r,
                                                         g.s, g.pad, g.stride, kpitch);
-    else
+    } else if (kpitch % V == 0) {
+        const int grid = grid_for(rows * (kpitch / V), 256);
+        im2col_chunk_kernel<T><<<grid, 256, 0, st>>>((const T*)x, (T*)col, rows, g.h, g.w, g.c, g.p, g.q, g.r,
+                                                      g.s, g.pad, g.stride, kpitch);
+    } else {
+        const int grid = grid_for(rows * 32, 256);
         im2col_rows_kernel<T, 1><<<grid, 256, 0, st>>>((const T*)x, (T*)col, rows, g.h, g.w, g.c, g.p, g.q, g.r,
                                                         g.s, g.pad, g.stride, kpitch);
+    }
     count_launch();
     return (int)cudaGetLastError();
+}
+
+template <class T>
+__global__ void col2im_pixel_kernel(const float* __restrict__ dcol, T* __restrict__ dx, int64_t pixels, int H,
+                                    int W, int C, int P, int Q, int R, int S, int pad, int st, int kpitch,
+                                    float alpha, float beta) {
+    for (int64_t pix = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; pix < pixels;
+         pix += (int64_t)gridDim.x * blockDim.x) {
+        const int w = (int)(pix % W);
+        const int64_t t2 = pix / W;
+        const int h = (int)(t2 % H);
+        const int n = (int)(t2 / H);
+        const int hp = h + pad, wp = w + pad;
+        const int r0 = hp % st, s0 = wp % st;
+        float acc[4] = {0.f, 0.f, 0.f, 0.f};
+        for (int r = r0, p = (hp - r0) / st; r < R && p >= 0; r += st, --p) {
+            if (p >= P) continue;
+            const float* rowp = dcol + ((int64_t)n * P + p) * Q * (int64_t)kpitch;
+            for (int s = s0, q = (wp - s0) / st; s < S && q >= 0; s += st, --q) {
+                if (q >= Q) continue;
+                const float* src = rowp + (int64_t)q * kpitch + (r * S + s) * C;
+                for (int c = 0; c < C; ++c) acc[c] += src[c];
+            }
+        }
+        T* out = dx + pix * C;
+        for (int c = 0; c < C; ++c) {
+            float o = alpha * acc[c];
+            if (beta != 0.f) o += beta * to_f<T>(out[c]);
+            out[c] = from_f<T>(o);
+        }
+    }
 }
 
 // Gather col2im over the VALID taps only: for a dx pixel (h,w) the taps with
@@ -397,6 +472,19 @@ int launch_pad_filter(const Geom& g, const void* w, void* wpad, int32_t kpitch, 
 int launch_col2im(const Geom& g, int32_t b, float alpha, const float* dcol, int32_t kpitch, float beta,
                   void* dx, cudaStream_t st) {
     const int64_t pixels = (int64_t)b * g.h * g.w;
+    if (g.c < 4) {
+        // tiny C (RGB input layer): one thread per dx pixel, all channels in
+        // registers; neighbouring threads read neighbouring taps of a dcol row.
+        const int grid = grid_for(pixels, 256);
+        if (g.math == MUCU_MATH_BF16)
+            col2im_pixel_kernel<__nv_bfloat16><<<grid, 256, 0, st>>>(dcol, (__nv_bfloat16*)dx, pixels, g.h, g.w, g.c, g.p,
+                                                                    g.q, g.r, g.s, g.pad, g.stride, kpitch, alpha, beta);
+        else
+            col2im_pixel_kernel<float><<<grid, 256, 0, st>>>(dcol, (float*)dx, pixels, g.h, g.w, g.c, g.p, g.q, g.r,
+                                                            g.s, g.pad, g.stride, kpitch, alpha, beta);
+        count_launch();
+        return (int)cudaGetLastError();
+    }
     const bool v4 = g.c % 4 == 0 && kpitch % 4 == 0;
     const int grid = grid_for(pixels * (v4 ? g.c / 4 : g.c), 256);
 #define COL2IM(TT, VV)                                                                                            \

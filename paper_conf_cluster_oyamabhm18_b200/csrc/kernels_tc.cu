@@ -156,6 +156,7 @@ enum EpiMode : int { EPI_STORE = 0, EPI_WGRAD_CHAIN = 1 };
 struct TcArgs {
     int M, N;                // output rows / cols
     int num_kb;              // k-blocks of the whole reduction
+    int num_z;               // batch (WG) or split (WGRAD) count; tiles = mt * nt * num_z
     int kb_per_split;        // WGRAD: k-blocks per blockIdx.z split
     int BN;                  // tile N (multiple of 16, <= 256)
     int stages;
@@ -188,7 +189,7 @@ struct TcArgs {
     int32_t* sem;
 };
 
-constexpr int kThreads = 256;
+constexpr int kThreads = 288;  // 4 producer warps, 1 MMA warp, 4 epilogue warps
 
 // DGRAD reduction tap index -> filter tap r*S+s (phase mode: the sub-filter
 // tap (a,b) is (r0 + st*a, s0 + st*b)).
@@ -240,503 +241,7 @@ __device__ __forceinline__ void st_shared_elt<float>(uint32_t addr, float v) {
 }
 
 // ------------------------------------------------------------ the kernel --
-template <int ELT, int AM, int BM_, int EPI>
-__global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constant__ TcArgs p,
-                                                            const __grid_constant__ CUtensorMap tmA,
-                                                            const __grid_constant__ CUtensorMap tmB) {
-    using T = typename Elt<ELT>::T;
-    constexpr int KB = 128 / ELT;            // K elements per stage
-    constexpr int UMMA_K = 32 / ELT;         // K elements per MMA
-    constexpr int A_BYTES = 128 * 128;       // 128 rows x 128 B
-    constexpr bool A_MN = (AM == A_TMA_MN2);
-    constexpr bool B_MN = (BM_ == B_TMA_MN2 || BM_ == B_TMA_MN3 || BM_ == B_GATHER_WG || BM_ == B_SCALAR_DGRAD ||
-                           BM_ == B_SCALAR_WG || BM_ == B_TMA_IM2COL);
-    constexpr bool A_TMA = (AM == A_TMA_K2 || AM == A_TMA_K3 || AM == A_TMA_MN2 || AM == A_TMA_IM2COL);
-    constexpr bool B_TMA = (BM_ == B_TMA_K2 || BM_ == B_TMA_K3 || BM_ == B_TMA_MN2 || BM_ == B_TMA_MN3 ||
-                            BM_ == B_TMA_IM2COL);
-    constexpr bool GATHER = !A_TMA || !B_TMA;
-    constexpr bool A_ASYNC = (AM == A_GATHER_FWD || AM == A_GATHER_DGRAD);
-    constexpr bool B_ASYNC = (BM_ == B_GATHER_WG);
-    // MN-major atoms: 8-row (bf16, SWIZZLE_128B) or 4-row (tf32, 128B_BASE32B) groups.
-    constexpr uint32_t MN_SBO = ELT == 2 ? 1024u : 512u;
-    constexpr uint32_t MN_LAYOUT = ELT == 2 ? 2u : 1u;
-
-    extern __shared__ uint8_t smem_raw[];
-    uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
-    const int S = p.stages;
-    const int B_BYTES = p.b_bytes;
-    uint8_t* sA = smem;
-    uint8_t* sB = smem + (size_t)S * A_BYTES;
-    uint64_t* bars = (uint64_t*)(sB + (size_t)S * B_BYTES);
-    uint64_t* full = bars;
-    uint64_t* empty = bars + S;
-    uint64_t* accum = bars + 2 * S;
-    uint32_t* tmem_slot = (uint32_t*)(bars + 2 * S + 1);
-
-    const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
-    // M tiles on grid.x (up to 2^31-1; conv1 DGRAD at N=256 has 100k of them),
-    // N tiles on grid.y: consecutive CTAs share the same B (filter) tile in L2.
-    const int m0 = blockIdx.x * 128;
-    const int n0 = blockIdx.y * p.BN;
-    const int z = blockIdx.z;
-    int kb_begin = 0, kb_end = p.num_kb;
-    if (EPI == EPI_WGRAD_CHAIN) {
-        kb_begin = z * p.kb_per_split;
-        kb_end = min(p.num_kb, kb_begin + p.kb_per_split);
-    }
-    const int nkb = kb_end - kb_begin;
-
-    if (threadIdx.x == 0) {
-        const uint32_t full_count = (GATHER ? 128u : 0u) + (A_TMA || B_TMA ? 1u : 0u);
-        for (int s = 0; s < S; ++s) {
-            mbar_init(smem_u32(&full[s]), full_count);
-            mbar_init(smem_u32(&empty[s]), 1);
-        }
-        mbar_init(smem_u32(accum), 1);
-        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    }
-    if (warp == 4) {
-        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
-                     "r"(p.tmem_cols));
-        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
-    }
-    tc_fence_before();
-    __syncthreads();
-    tc_fence_after();
-    const uint32_t tmem = *tmem_slot;
-
-    if (warp < 4) {
-        // =========================== producers ===========================
-        const int t = threadIdx.x;  // 0..127
-        // Per-thread gather rows (A gathers: rows t/8 + 16 i, chunk t % 8).
-        // Per-row origin (h, w) and base element offset, computed once per tile:
-        // FWD  row = output pixel (n,p,q): origin (p*st - pad, q*st - pad) in x,
-        //      element (r,s,c) at base + (r*W + s)*C + c;
-        // DGRAD row = dx pixel (n,h,w): dy index (h + pad - r, w + pad - s)
-        //      (stride 1: element (r,s,k) at base - (r*Q + s)*K + k).
-        int rh[8], rw[8];
-        long long rbase[8];
-        bool rv[8];
-        if constexpr (AM == A_GATHER_FWD || AM == A_GATHER_DGRAD) {
-#pragma unroll
-            for (int i = 0; i < 8; ++i) {
-                const int m = m0 + t / 8 + 16 * i;
-                rv[i] = m < p.M;
-                const int mm = rv[i] ? m : 0;
-                if (AM == A_GATHER_FWD) {
-                    const int pq = p.P * p.Q;
-                    const int n = mm / pq, rem = mm - n * pq, pp = rem / p.Q, qq = rem - pp * p.Q;
-                    rh[i] = pp * p.stride - p.pad; rw[i] = qq * p.stride - p.pad;
-                    rbase[i] = (((long long)n * p.H + rh[i]) * p.W + rw[i]) * p.C;
-                } else {
-                    const int hw = p.H * p.W;
-                    const int n = mm / hw, rem = mm - n * hw, hh = rem / p.W, ww = rem - hh * p.W;
-                    rh[i] = hh + p.pad; rw[i] = ww + p.pad;
-                    rbase[i] = p.stride == 1 ? (((long long)n * p.P + rh[i]) * p.Q + rw[i]) * p.K
-                                             : (long long)n * p.P * p.Q * p.K;  // strided: image base
-                }
-            }
-        }
-        const T* gx = (const T*)p.gsrc;
-        const int lag = min(S - 1, 3);
-        // Incremental (r, s, c0) of the current k-block (no per-block division):
-        // a k-block covers KB consecutive channels of one filter tap.
-        constexpr bool WALK = (AM == A_GATHER_FWD || AM == A_GATHER_DGRAD || AM == A_TMA_IM2COL);
-        const int gch = (AM == A_GATHER_DGRAD || (AM == A_TMA_IM2COL && p.im2col_dgrad)) ? p.K : p.C;
-        int g_c0 = 0, g_s = 0, g_r = 0;
-        if constexpr (WALK) {
-            const int kk0 = kb_begin * KB;
-            const int rs = kk0 / gch;
-            g_c0 = kk0 - rs * gch; g_r = rs / p.tapS; g_s = rs - g_r * p.tapS;
-        }
-        // TMA im2col start pixel of this tile (FWD: output pixel m0 -> x origin;
-        // DGRAD: dx pixel m0 -> dy origin h + pad - (R-1); phase mode: sub-grid
-        // pixel (ii, jj) -> dy origin (i0 + ii - (tapR-1), j0 + jj - (tapS-1))).
-        int ic_w = 0, ic_h = 0, ic_n = 0;
-        if constexpr (AM == A_TMA_IM2COL) {
-            if (p.ph_mode) {
-                const int hw = p.ph_H * p.ph_W;
-                ic_n = m0 / hw;
-                const int rem = m0 - ic_n * hw, ii = rem / p.ph_W, jj = rem - ii * p.ph_W;
-                ic_h = p.ph_i0 + ii - (p.tapR - 1); ic_w = p.ph_j0 + jj - (p.tapS - 1);
-            } else if (p.im2col_dgrad) {
-                const int hw = p.H * p.W;
-                ic_n = m0 / hw;
-                const int rem = m0 - ic_n * hw, hh = rem / p.W, ww = rem - hh * p.W;
-                ic_h = hh + p.pad - (p.R - 1); ic_w = ww + p.pad - (p.S - 1);
-            } else {
-                const int pq = p.P * p.Q;
-                ic_n = m0 / pq;
-                const int rem = m0 - ic_n * pq, pp = rem / p.Q, qq = rem - pp * p.Q;
-                ic_h = pp * p.stride - p.pad; ic_w = qq * p.stride - p.pad;
-            }
-        }
-        // WGRAD TMA im2col: pixel (n,p,q) of the first row of the k-block, walked
-        // incrementally (KB pixels per k-block).
-        int wb_n = 0, wb_p = 0, wb_q = 0;
-        if constexpr (BM_ == B_TMA_IM2COL) {
-            const int m = kb_begin * KB, pq = p.P * p.Q;
-            wb_n = m / pq;
-            const int rem = m - wb_n * pq;
-            wb_p = rem / p.Q; wb_q = rem - wb_p * p.Q;
-        }
-        int s = 0;
-        uint32_t ph = 0;
-        for (int it = 0; it < nkb; ++it, s = (s + 1 == S) ? 0 : s + 1, ph ^= (s == 0) ? 1u : 0u) {
-            const int kb = kb_begin + it;
-            mbar_wait(smem_u32(&empty[s]), ph ^ 1u);
-            const uint32_t aT = smem_u32(sA + (size_t)s * A_BYTES);
-            const uint32_t bT = smem_u32(sB + (size_t)s * B_BYTES);
-            const uint32_t fb = smem_u32(&full[s]);
-            if ((A_TMA || B_TMA) && t == 0) {
-                mbar_arrive_tx(fb, (uint32_t)p.tma_bytes);
-                if constexpr (AM == A_TMA_K2) tma_load_2d(aT, &tmA, fb, kb * KB, m0);
-                if constexpr (AM == A_TMA_K3) tma_load_3d(aT, &tmA, fb, kb * KB, m0, z);
-                if constexpr (AM == A_TMA_MN2) {
-                    tma_load_2d(aT, &tmA, fb, m0, kb * KB);
-                    tma_load_2d(aT + KB * 128, &tmA, fb, m0 + 128 / ELT, kb * KB);
-                    if constexpr (ELT == 4) {
-                        tma_load_2d(aT + 2 * KB * 128, &tmA, fb, m0 + 2 * (128 / ELT), kb * KB);
-                        tma_load_2d(aT + 3 * KB * 128, &tmA, fb, m0 + 3 * (128 / ELT), kb * KB);
-                    }
-                }
-                if constexpr (BM_ == B_TMA_K2) tma_load_2d(bT, &tmB, fb, kb * KB, n0);
-                if constexpr (BM_ == B_TMA_K3) tma_load_3d(bT, &tmB, fb, kb * KB, n0, z);
-                if constexpr (BM_ == B_TMA_MN2) {
-                    for (int a = 0; a < p.bn_atoms; ++a)
-                        tma_load_2d(bT + a * KB * 128, &tmB, fb, n0 + a * (128 / ELT), kb * KB);
-                }
-                if constexpr (BM_ == B_TMA_MN3) {
-                    // k-block kb covers (r,s) = kb / (K/KB), k0 = (kb % (K/KB)) * KB
-                    const int kpr = p.K / KB;
-                    const int tap = kb / kpr, k0 = (kb - tap * kpr) * KB;
-                    const int rs = dgrad_tap_rs(p, tap);
-                    for (int a = 0; a < p.bn_atoms; ++a)
-                        tma_load_3d(bT + a * KB * 128, &tmB, fb, n0 + a * (128 / ELT), rs, k0);
-                }
-                if constexpr (AM == A_TMA_IM2COL) {
-                    // 128 consecutive output pixels x KB channels of tap (r,s) in one TMA
-                    const uint16_t ow = (uint16_t)(p.im2col_dgrad ? p.tapS - 1 - g_s : g_s);
-                    const uint16_t oh = (uint16_t)(p.im2col_dgrad ? p.tapR - 1 - g_r : g_r);
-                    tma_load_im2col_4d(aT, &tmA, fb, g_c0, ic_w, ic_h, ic_n, ow, oh);
-                }
-                if constexpr (BM_ == B_TMA_IM2COL) {
-                    // atom a = 128 B of channels (c0..) of tap (r,s) for KB pixels
-                    const int h0 = wb_p * p.stride - p.pad, w0 = wb_q * p.stride - p.pad;
-                    for (int a = 0; a < p.bn_atoms; ++a) {
-                        const int j0 = n0 + a * (128 / ELT);
-                        const int rs = j0 / p.C, c0 = j0 - rs * p.C;
-                        const int r = rs / p.S, sx = rs - r * p.S;
-                        tma_load_im2col_4d(bT + a * KB * 128, &tmB, fb, c0, w0, h0, wb_n, (uint16_t)sx, (uint16_t)r);
-                    }
-                }
-            }
-            if constexpr (BM_ == B_TMA_IM2COL) {
-                wb_q += KB;
-                while (wb_q >= p.Q) { wb_q -= p.Q; if (++wb_p == p.P) { wb_p = 0; ++wb_n; } }
-            }
-            // ---- A gathers ----
-            if constexpr (AM == A_GATHER_FWD) {
-                const int r = g_r, sx = g_s;
-                const bool kin = r < p.R;
-                const long long koff = ((long long)r * p.W + sx) * p.C + g_c0 + (t & 7) * (16 / ELT);
-                const uint32_t soff = kmaj_off(t / 8, (t & 7) * 16);
-#pragma unroll
-                for (int i = 0; i < 8; ++i) {
-                    const bool v = kin && rv[i] && (unsigned)(rh[i] + r) < (unsigned)p.H &&
-                                   (unsigned)(rw[i] + sx) < (unsigned)p.W;
-                    cp_async16(aT + soff + i * 2048, v ? gx + rbase[i] + koff : gx, v);
-                }
-            } else if constexpr (AM == A_GATHER_DGRAD) {
-                const int r = g_r, sx = g_s;
-                const bool kin = r < p.R;
-                const int kc = g_c0 + (t & 7) * (16 / ELT);
-                const uint32_t soff = kmaj_off(t / 8, (t & 7) * 16);
-                if (p.stride == 1) {
-                    const long long koff = kc - ((long long)r * p.Q + sx) * p.K;
-#pragma unroll
-                    for (int i = 0; i < 8; ++i) {
-                        const bool v = kin && rv[i] && (unsigned)(rh[i] - r) < (unsigned)p.P &&
-                                       (unsigned)(rw[i] - sx) < (unsigned)p.Q;
-                        cp_async16(aT + soff + i * 2048, v ? gx + rbase[i] + koff : gx, v);
-                    }
-                } else {
-#pragma unroll
-                    for (int i = 0; i < 8; ++i) {
-                        const int ph_ = rh[i] - r, pw_ = rw[i] - sx;
-                        bool v = kin && rv[i] && ph_ >= 0 && pw_ >= 0;
-                        int pp = 0, qq = 0;
-                        if (v) {
-                            pp = ph_ / p.stride; qq = pw_ / p.stride;
-                            v = (pp * p.stride == ph_) && (qq * p.stride == pw_) && pp < p.P && qq < p.Q;
-                        }
-                        const T* src = v ? gx + rbase[i] + ((long long)pp * p.Q + qq) * p.K + kc : gx;
-                        cp_async16(aT + soff + i * 2048, src, v);
-                    }
-                }
-            }
-            if constexpr (WALK) {
-                g_c0 += KB;
-                if (g_c0 >= gch) { g_c0 = 0; if (++g_s == p.tapS) { g_s = 0; ++g_r; } }
-            }
-            if constexpr (AM == A_SCALAR_FWD) {
-                // thread t owns row t; KB elements, kk = (r,s,c) decomposed each
-                const int m = m0 + t;
-                const bool rvalid = m < p.M;
-                const int pq = p.P * p.Q;
-                const int mm = rvalid ? m : 0;
-                const int n = mm / pq, rem = mm - n * pq, pp = rem / p.Q, qq = rem - pp * p.Q;
-                for (int e = 0; e < KB; ++e) {
-                    const int kk = kb * KB + e;
-                    float v = 0.f;
-                    if (rvalid && kk < p.kred) {
-                        const int rs = kk / p.C, c = kk - rs * p.C, r = rs / p.S, sx = rs - r * p.S;
-                        const int h = pp * p.stride - p.pad + r, w = qq * p.stride - p.pad + sx;
-                        if (h >= 0 && h < p.H && w >= 0 && w < p.W)
-                            v = (float)gx[(((size_t)n * p.H + h) * p.W + w) * p.C + c];
-                    }
-                    st_shared_elt<T>(aT + kmaj_off(t, e * ELT), (T)v);
-                }
-            } else if constexpr (AM == A_SCALAR_DGRAD) {
-                // thread t owns dx pixel row t; kk = (r,s,k) decomposed per element
-                const int m = m0 + t;
-                const bool rvalid = m < p.M;
-                const int hw = p.H * p.W;
-                const int mm = rvalid ? m : 0;
-                const int n = mm / hw, rem = mm - n * hw, hh = rem / p.W, ww = rem - hh * p.W;
-                for (int e = 0; e < KB; ++e) {
-                    const int kk = kb * KB + e;
-                    float v = 0.f;
-                    if (rvalid && kk < p.kred) {
-                        const int rs = kk / p.K, k = kk - rs * p.K, r = rs / p.S, sx = rs - r * p.S;
-                        const int ph_ = hh + p.pad - r, pw_ = ww + p.pad - sx;
-                        if (ph_ >= 0 && pw_ >= 0 && ph_ % p.stride == 0 && pw_ % p.stride == 0) {
-                            const int pp = ph_ / p.stride, qq = pw_ / p.stride;
-                            if (pp < p.P && qq < p.Q) v = (float)gx[(((size_t)n * p.P + pp) * p.Q + qq) * p.K + k];
-                        }
-                    }
-                    st_shared_elt<T>(aT + kmaj_off(t, e * ELT), (T)v);
-                }
-            }
-            // ---- B gathers ----
-            if constexpr (BM_ == B_GATHER_WG) {
-                // KB pixel rows x bn_atoms atoms x 8 chunks; thread: chunk t%8, rows t/8 + 16 i
-                const int chunk = t & 7;
-                for (int i = 0; i < KB / 16; ++i) {
-                    const int row = t / 8 + 16 * i;
-                    const int m = kb * KB + row;
-                    const int pq = p.P * p.Q;
-                    const bool mv = m < p.kred;
-                    const int mm = mv ? m : 0;
-                    const int n = mm / pq, rem = mm - n * pq, pp = rem / p.Q, qq = rem - pp * p.Q;
-                    for (int a = 0; a < p.bn_atoms; ++a) {
-                        const int j0 = n0 + a * (128 / ELT);
-                        const int rs = j0 / p.C, c0 = j0 - rs * p.C + chunk * (16 / ELT);
-                        const int r = rs / p.S, sx = rs - r * p.S;
-                        const int h = pp * p.stride - p.pad + r, w = qq * p.stride - p.pad + sx;
-                        const bool v = mv && rs < p.R * p.S && h >= 0 && h < p.H && w >= 0 && w < p.W;
-                        const T* src = v ? gx + (((size_t)n * p.H + h) * p.W + w) * p.C + c0 : gx;
-                        cp_async16(bT + (uint32_t)(a * KB * 128) + mn_row_off<ELT>(row, chunk * 16), src, v);
-                    }
-                }
-            } else if constexpr (BM_ == B_SCALAR_K) {
-                // B rows n0.. (BN of them) x KB elements from a dense row-major matrix with pitch ldb
-                const T* bs = (const T*)p.bsrc;
-                for (int idx = t; idx < p.BN * KB; idx += 128) {
-                    const int row = idx / KB, e = idx - (idx / KB) * KB;
-                    const int j = n0 + row, kk = kb * KB + e;
-                    const float v = (j < p.N && kk < p.kred) ? (float)bs[(size_t)j * p.ldb + kk] : 0.f;
-                    st_shared_elt<T>(bT + kmaj_off(row, e * ELT), (T)v);
-                }
-            } else if constexpr (BM_ == B_SCALAR_DGRAD) {
-                // B(j = c, kk = (r,s,k)) = w[k][r][s][c], MN-major
-                const T* bs = (const T*)p.bsrc;
-                const int RS = p.R * p.S;
-                for (int idx = t; idx < p.BN * KB; idx += 128) {
-                    const int krow = idx / p.BN, jj = idx - krow * p.BN;
-                    const int j = n0 + jj, kk = kb * KB + krow;
-                    float v = 0.f;
-                    if (j < p.N && kk < p.kred) {
-                        const int tap = kk / p.K, k = kk - tap * p.K;
-                        const int rs = dgrad_tap_rs(p, tap);
-                        v = (float)bs[((size_t)k * RS + rs) * p.C + j];
-                    }
-                    st_shared_elt<T>(bT + mnmaj_off<ELT>(jj, krow, KB), (T)v);
-                }
-            } else if constexpr (BM_ == B_SCALAR_WG) {
-                // B(j = (r,s,c), kk = pixel m) = x[n, p*st + r - pad, q*st + s - pad, c], MN-major
-                const int pq = p.P * p.Q;
-                for (int idx = t; idx < p.BN * KB; idx += 128) {
-                    const int krow = idx / p.BN, jj = idx - krow * p.BN;
-                    const int j = n0 + jj, m = kb * KB + krow;
-                    float v = 0.f;
-                    if (j < p.N && m < p.kred) {
-                        const int n = m / pq, rem = m - n * pq, pp = rem / p.Q, qq = rem - pp * p.Q;
-                        const int rs = j / p.C, c = j - rs * p.C, r = rs / p.S, sx = rs - r * p.S;
-                        const int h = pp * p.stride - p.pad + r, w = qq * p.stride - p.pad + sx;
-                        if (h >= 0 && h < p.H && w >= 0 && w < p.W)
-                            v = (float)gx[(((size_t)n * p.H + h) * p.W + w) * p.C + c];
-                    }
-                    st_shared_elt<T>(bT + mnmaj_off<ELT>(jj, krow, KB), (T)v);
-                }
-            }
-            if constexpr (GATHER) {
-                if constexpr (A_ASYNC || B_ASYNC) {
-                    cp_async_commit();
-                    // Lagged arrive: keep `lag` stages of gathers in flight per
-                    // thread (L2 latency hiding); stage it-lag is complete once at
-                    // most `lag` groups are pending.  lag <= S-1 keeps the ring
-                    // deadlock-free (the MMA can always drain stage it-S).
-                    if (it >= lag) {
-                        if (lag == 1) cp_async_wait<1>();
-                        else if (lag == 2) cp_async_wait<2>();
-                        else cp_async_wait<3>();
-                        fence_proxy_async();
-                        mbar_arrive(smem_u32(&full[s - lag < 0 ? s - lag + S : s - lag]));
-                    }
-                } else {
-                    fence_proxy_async();
-                    mbar_arrive(fb);
-                }
-            }
-        }
-        if constexpr (GATHER && (A_ASYNC || B_ASYNC)) {
-            if (nkb > 0) {
-                cp_async_wait<0>();
-                fence_proxy_async();
-                for (int j = max(0, nkb - lag); j < nkb; ++j) mbar_arrive(smem_u32(&full[j % S]));
-            }
-        }
-    } else {
-        // ======================= MMA issuer (warp 4) =======================
-        if (warp == 4) {
-            const uint32_t idesc = (1u << 4) | (Elt<ELT>::fmt << 7) | (Elt<ELT>::fmt << 10) |
-                                   ((A_MN ? 1u : 0u) << 15) | ((B_MN ? 1u : 0u) << 16) |
-                                   ((uint32_t)(p.BN >> 3) << 17) | ((128u >> 4) << 24);
-            int s = 0;
-            uint32_t ph = 0;
-            for (int it = 0; it < nkb; ++it, s = (s + 1 == S) ? 0 : s + 1, ph ^= (s == 0) ? 1u : 0u) {
-                mbar_wait(smem_u32(&full[s]), ph);
-                tc_fence_after();
-                if (lane == 0) {
-                    const uint32_t aT = smem_u32(sA + (size_t)s * A_BYTES);
-                    const uint32_t bT = smem_u32(sB + (size_t)s * B_BYTES);
-#pragma unroll
-                    for (int j = 0; j < KB / UMMA_K; ++j) {
-                        const uint64_t ad = A_MN ? sdesc(aT + j * UMMA_K * 128, KB * 128, MN_SBO, MN_LAYOUT)
-                                                 : sdesc(aT + j * 32, 16, 1024);
-                        const uint64_t bd = B_MN ? sdesc(bT + j * UMMA_K * 128, KB * 128, MN_SBO, MN_LAYOUT)
-                                                 : sdesc(bT + j * 32, 16, 1024);
-                        mma<ELT>(tmem, ad, bd, idesc, (it | j) != 0 ? 1u : 0u);
-                    }
-                    mma_commit(smem_u32(&empty[s]));
-                }
-                __syncwarp();
-            }
-            if (lane == 0) {
-                if (nkb > 0) mma_commit(smem_u32(accum));
-                else mbar_arrive(smem_u32(accum));
-            }
-            __syncwarp();
-        }
-        // ============================ epilogue =============================
-        mbar_wait(smem_u32(accum), 0);
-        tc_fence_after();
-        const int q4 = warp & 3;
-        const int row = q4 * 32 + lane;
-        const int m = m0 + row;
-        // Output row of GEMM row m (phase mode scatters sub-grid rows back to dx).
-        long long mrow = m;
-        if (p.ph_mode && m < p.M) {
-            const int hw = p.ph_H * p.ph_W;
-            const int n = m / hw, rem = m - n * hw, ii = rem / p.ph_W, jj = rem - ii * p.ph_W;
-            mrow = ((long long)n * p.H + p.ph_hb + p.stride * ii) * p.W + p.ph_wb + p.stride * jj;
-        }
-        const uint32_t taddr_row = tmem + ((uint32_t)(q4 * 32) << 16);
-        float* outF = (float*)p.out;
-        T* outT = (T*)p.out;
-        if (EPI == EPI_STORE && z > 0) {
-            outF += (size_t)z * p.batch_stride;
-            outT += (size_t)z * p.batch_stride;
-        }
-        for (int c0 = 0; c0 < p.BN; c0 += 32) {
-            uint32_t v[32];
-            if (nkb > 0) {
-                TMEM_LD32(taddr_row + (uint32_t)c0, v);
-                asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
-            } else {
-#pragma unroll
-                for (int j = 0; j < 32; ++j) v[j] = 0u;
-            }
-            if (m >= p.M) continue;
-            const int nb = n0 + c0;
-            if constexpr (EPI == EPI_WGRAD_CHAIN) {
-                // dw += alpha * partial (beta was applied by a prescale launch);
-                // 16-byte vector reductions in L2 (red.global.add.v4.f32).
-                float* d = outF + (size_t)m * p.ldc + nb;
-                const bool vec = (nb + 32 <= p.N) && ((p.ldc & 3) == 0);
-                if (vec) {
-#pragma unroll
-                    for (int j = 0; j < 32; j += 4)
-                        asm volatile("red.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(d + j),
-                                     "f"(p.alpha * __uint_as_float(v[j])), "f"(p.alpha * __uint_as_float(v[j + 1])),
-                                     "f"(p.alpha * __uint_as_float(v[j + 2])), "f"(p.alpha * __uint_as_float(v[j + 3]))
-                                     : "memory");
-                } else {
-#pragma unroll
-                    for (int j = 0; j < 32; ++j)
-                        if (nb + j < p.N) atomicAdd(d + j, p.alpha * __uint_as_float(v[j]));
-                }
-            } else if (p.out_bf16) {
-                __nv_bfloat16* d = (__nv_bfloat16*)outT + (size_t)mrow * p.ldc + nb;
-                const bool vec = (nb + 32 <= p.N) && ((p.ldc & 7) == 0) && p.beta == 0.f;
-                if (vec) {
-#pragma unroll
-                    for (int j = 0; j < 32; j += 8) {
-                        __align__(16) __nv_bfloat16 tmp[8];
-#pragma unroll
-                        for (int u = 0; u < 8; ++u) tmp[u] = __float2bfloat16_rn(p.alpha * __uint_as_float(v[j + u]));
-                        *reinterpret_cast<uint4*>(d + j) = *reinterpret_cast<uint4*>(tmp);
-                    }
-                } else {
-#pragma unroll
-                    for (int j = 0; j < 32; ++j) {
-                        if (nb + j < p.N) {
-                            float o = p.alpha * __uint_as_float(v[j]);
-                            if (p.beta != 0.f) o += p.beta * __bfloat162float(d[j]);
-                            d[j] = __float2bfloat16_rn(o);
-                        }
-                    }
-                }
-            } else {
-                float* d = outF + (size_t)mrow * p.ldc + nb;
-                const bool vec = (nb + 32 <= p.N) && ((p.ldc & 3) == 0) && p.beta == 0.f;
-                if (vec) {
-#pragma unroll
-                    for (int j = 0; j < 32; j += 4)
-                        *reinterpret_cast<float4*>(d + j) =
-                            make_float4(p.alpha * __uint_as_float(v[j]), p.alpha * __uint_as_float(v[j + 1]),
-                                        p.alpha * __uint_as_float(v[j + 2]), p.alpha * __uint_as_float(v[j + 3]));
-                } else {
-#pragma unroll
-                    for (int j = 0; j < 32; ++j) {
-                        if (nb + j < p.N) {
-                            float o = p.alpha * __uint_as_float(v[j]);
-                            if (p.beta != 0.f) o += p.beta * d[j];
-                            d[j] = o;
-                        }
-                    }
-                }
-            }
-        }
-    }
-    tc_fence_before();
-    __syncthreads();
-    if (warp == 4) {
-        tc_fence_after();
-        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(p.tmem_cols));
-    }
-}
+#include "tc_gemm_kernel.cuh"
 
 // ------------------------------------------------------------ host side --
 typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
@@ -844,7 +349,7 @@ struct Launch {
 template <int ELT, int AM, int BM_, int EPI>
 int launch_t(Launch& L, cudaStream_t st) {
     auto kern = tc_conv_gemm<ELT, AM, BM_, EPI>;
-    const int smem = 1024 + L.a.stages * (128 * 128 + L.a.b_bytes) + (2 * L.a.stages + 2) * 8 + 64;
+    const int smem = 1024 + L.a.stages * (128 * 128 + L.a.b_bytes) + (2 * L.a.stages + 4) * 8 + 64;
     static int configured = 0;  // per instantiation
     if (configured < smem) {
         cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 232448);
@@ -859,7 +364,7 @@ int launch_t(Launch& L, cudaStream_t st) {
 void finalize_tiling(Launch& L, int elt, int step = 32) {
     TcArgs& a = L.a;
     a.BN = pick_bn(a.N, step);
-    a.tmem_cols = a.BN <= 32 ? 32 : a.BN <= 64 ? 64 : a.BN <= 128 ? 128 : 256;
+    a.tmem_cols = 2 * a.BN <= 64 ? 64 : 2 * a.BN <= 128 ? 128 : 2 * a.BN <= 256 ? 256 : 512;  // 2 accumulators
     a.bn_atoms = (a.BN * elt + 127) / 128;
     a.b_bytes = std::max(a.BN * 128, a.bn_atoms * (128 / elt) * 128);
     const int stage_bytes = 128 * 128 + a.b_bytes;
@@ -900,8 +405,11 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         uint32_t box[3] = {b0, b1, b2};
         return make_map(tm, elt, base, 3, dims, str, box, mn);
     };
+    // Persistent launch: one CTA per SM (at most one per tile).
     auto grid2 = [&](int batch) {
-        L.grid = dim3((unsigned)ceil_div(A.M, 128), (unsigned)ceil_div(A.N, A.BN), (unsigned)batch);
+        A.num_z = batch;
+        const int64_t tiles = ceil_div(A.M, 128) * ceil_div(A.N, A.BN) * batch;
+        L.grid = dim3((unsigned)std::max<int64_t>(1, std::min<int64_t>(tiles, num_sms)));
     };
     const bool Aok = (g.c % KB) == 0;  // vector gathers over C
     int err = 0;
@@ -1098,7 +606,7 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         A.kb_per_split = (int)ceil_div(nkb, nsplit);
         nsplit = ceil_div(nkb, A.kb_per_split);
         A.num_kb = (int)nkb;
-        L.grid = dim3((unsigned)ceil_div(A.M, 128), (unsigned)ceil_div(A.N, A.BN), (unsigned)nsplit);
+        grid2((int)nsplit);
         if (!map2(&L.ta, in1, g.k, (uint64_t)Mpix, g.k, atom, KB, true)) return -1;
         const int a_bytes = 128 * KB * elt;
         if (algo == MUCU_ALGO_IM2COL_GEMM) {

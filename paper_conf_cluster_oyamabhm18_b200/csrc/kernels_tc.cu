@@ -317,6 +317,11 @@ bool make_im2col_map(CUtensorMap* tm, int elt, const void* base, int C, int W, i
     return r == CUDA_SUCCESS;
 }
 
+int env_int(const char* name, int dflt) {
+    const char* e = getenv(name);
+    return e ? atoi(e) : dflt;
+}
+
 // MUCU_TMA_IM2COL=0 forces the cp.async gather producers (A/B comparison, tests).
 bool use_tma_im2col() {
     static int v = -1;
@@ -364,11 +369,12 @@ int launch_t(Launch& L, cudaStream_t st) {
 void finalize_tiling(Launch& L, int elt, int step = 32) {
     TcArgs& a = L.a;
     a.BN = pick_bn(a.N, step);
+    if (const int fb = env_int("MUCU_FORCE_BN", 0)) a.BN = std::max(step, fb - fb % step);
     a.tmem_cols = 2 * a.BN <= 64 ? 64 : 2 * a.BN <= 128 ? 128 : 2 * a.BN <= 256 ? 256 : 512;  // 2 accumulators
     a.bn_atoms = (a.BN * elt + 127) / 128;
     a.b_bytes = std::max(a.BN * 128, a.bn_atoms * (128 / elt) * 128);
     const int stage_bytes = 128 * 128 + a.b_bytes;
-    a.stages = std::min(6, (200 * 1024) / stage_bytes);
+    a.stages = std::min(env_int("MUCU_MAX_STAGES", 8), (200 * 1024) / stage_bytes);
     if (a.stages < 2) a.stages = 2;
 }
 
@@ -595,7 +601,8 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         const int64_t nkb = ceil_div(Mpix, KB);
         // Split the pixel reduction so that ~2 waves of CTAs run, each split
         // >= 16 k-blocks (amortises TMEM alloc / pipeline fill).
-        int64_t want = std::max<int64_t>(1, (2LL * num_sms + tiles - 1) / tiles);
+        // splits x tiles <= 2 waves of persistent CTAs (no ragged third round)
+        int64_t want = std::max<int64_t>(1, (2LL * num_sms) / tiles);
         int64_t nsplit = std::min<int64_t>(std::min<int64_t>(want, std::max<int64_t>(1, nkb / 16)), 65535);
         // P:L58 output scale: apply the user's beta once, then every split adds.
         if (beta != 1.f) {

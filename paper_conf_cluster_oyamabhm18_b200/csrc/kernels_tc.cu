@@ -139,6 +139,7 @@ enum AMode : int {
     A_SCALAR_FWD = 5,  // implicit im2col of x, element-wise (any C)
     A_SCALAR_DGRAD = 6,// transposed-conv gather of dy, element-wise (any K)
     A_TMA_IM2COL = 7,  // TMA im2col mode: FWD (x) or stride-1 DGRAD (dy, flipped taps), 128 pixels x KB channels
+    A_GATHER_SMALLC = 8, // FWD, C*elt < 16 B (RGB layer): one 16-B chunk per filter tap, channels zero-padded
 };
 enum BMode : int {
     B_TMA_K2 = 0,      // dense K-major {K, cols}
@@ -150,8 +151,10 @@ enum BMode : int {
     B_SCALAR_DGRAD = 6,// DGRAD filter view, element-wise (any C)
     B_SCALAR_WG = 7,   // WGRAD implicit im2col, element-wise (any C)
     B_TMA_IM2COL = 8,  // WGRAD implicit im2col of x by TMA im2col mode, MN-major (KB pixels x 128 B per atom)
+    B_RESIDENT = 9,    // whole (padded) filter staged in smem once per CTA (small-C FWD)
+    B_GATHER_SMALLC = 10, // WGRAD small C: x pixels as 16-B tap chunks, MN-major
 };
-enum EpiMode : int { EPI_STORE = 0, EPI_WGRAD_CHAIN = 1 };
+enum EpiMode : int { EPI_STORE = 0, EPI_WGRAD_CHAIN = 1, EPI_WGRAD_SMALLC = 2 };
 
 struct TcArgs {
     int M, N;                // output rows / cols
@@ -180,6 +183,10 @@ struct TcArgs {
     // (ph_H x ph_W) sub-grid.  tapR/tapS = R/S when not in phase mode.
     int ph_mode, ph_H, ph_W, ph_i0, ph_j0, ph_r0, ph_s0, ph_hb, ph_wb;
     int tapR, tapS;
+    // Small-C layers: K' = (r, s8, c') with taps grouped by 8 per k-block and
+    // channels zero-padded to cp = 16 B / elt; s8 = S rounded up to 8.
+    int cp, s8;
+    int bres_bytes;          // B_RESIDENT: smem bytes of the staged filter
     // epilogue
     void* out;
     long long ldc;
@@ -317,6 +324,9 @@ bool make_im2col_map(CUtensorMap* tm, int elt, const void* base, int C, int W, i
     return r == CUDA_SUCCESS;
 }
 
+// Dynamic shared memory budget per CTA (227 KB minus alignment slack and barriers).
+constexpr int kSmemBudget = 232448 - 1024 - 512;
+
 int env_int(const char* name, int dflt) {
     const char* e = getenv(name);
     return e ? atoi(e) : dflt;
@@ -354,7 +364,7 @@ struct Launch {
 template <int ELT, int AM, int BM_, int EPI>
 int launch_t(Launch& L, cudaStream_t st) {
     auto kern = tc_conv_gemm<ELT, AM, BM_, EPI>;
-    const int smem = 1024 + L.a.stages * (128 * 128 + L.a.b_bytes) + (2 * L.a.stages + 4) * 8 + 64;
+    const int smem = 1024 + L.a.stages * (128 * 128 + L.a.b_bytes) + L.a.bres_bytes + (2 * L.a.stages + 5) * 8 + 64;
     static int configured = 0;  // per instantiation
     if (configured < smem) {
         cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 232448);
@@ -441,8 +451,25 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
             A.tma_bytes = A.BN * 128;
             err = LAUNCH(A_GATHER_FWD, B_TMA_K2, EPI_STORE);
         } else {
-            A.num_kb = (int)ceil_div(RSC, KB);
             A.bsrc = in1; A.ldb = (int)RSC;
+            if (g.c * elt < 16) {
+                // RGB-like layer: K' = (r, s8, c') with 8 taps x 16 B per k-block,
+                // the zero-padded filter staged once per CTA in shared memory.
+                A.cp = 16 / elt; A.s8 = (int)align_up((uint64_t)g.s, 8);
+                A.num_kb = g.r * (A.s8 / 8);
+                if (ceil_div(A.N, A.BN) == 1) {
+                    A.b_bytes = 0;
+                    A.bres_bytes = A.num_kb * A.BN * 128;
+                    A.stages = std::min(8, (kSmemBudget - A.bres_bytes) / (128 * 128));
+                    if (A.stages >= 2) {
+                        A.tma_bytes = 0;
+                        return LAUNCH(A_GATHER_SMALLC, B_RESIDENT, EPI_STORE);
+                    }
+                }
+                finalize_tiling(L, elt);
+                A.cp = 0; A.s8 = 0; A.bres_bytes = 0;
+            }
+            A.num_kb = (int)ceil_div(RSC, KB);
             err = LAUNCH(A_SCALAR_FWD, B_SCALAR_K, EPI_STORE);
         }
         return err;
@@ -637,6 +664,20 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         }
         A.tma_bytes = a_bytes;
         if (g.c % atom == 0) return LAUNCH(A_TMA_MN2, B_GATHER_WG, EPI_WGRAD_CHAIN);
+        if (g.c * elt < 16) {
+            // RGB-like layer: padded columns j' = (r, s8, c'), one 128-B atom per
+            // 8-tap group; the epilogue folds them back into dw[k][r][s][c].
+            A.cp = 16 / elt; A.s8 = (int)align_up((uint64_t)g.s, 8);
+            A.N = g.r * A.s8 * A.cp;
+            finalize_tiling(L, elt, atom);
+            const int64_t t2 = ceil_div(A.N, A.BN) * ceil_div(A.M, 128);
+            int64_t ns2 = std::min<int64_t>(std::min<int64_t>(std::max<int64_t>(1, (2LL * num_sms) / t2),
+                                                              std::max<int64_t>(1, nkb / 16)), 65535);
+            A.kb_per_split = (int)ceil_div(nkb, ns2);
+            ns2 = ceil_div(nkb, A.kb_per_split);
+            grid2((int)ns2);
+            return LAUNCH(A_TMA_MN2, B_GATHER_SMALLC, EPI_WGRAD_SMALLC);
+        }
         return LAUNCH(A_TMA_MN2, B_SCALAR_WG, EPI_WGRAD_CHAIN);
     }
 #undef LAUNCH

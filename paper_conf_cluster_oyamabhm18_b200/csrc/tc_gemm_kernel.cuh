@@ -21,11 +21,13 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
     constexpr int A_BYTES = 128 * 128;       // 128 rows x 128 B
     constexpr bool A_MN = (AM == A_TMA_MN2);
     constexpr bool B_MN = (BM_ == B_TMA_MN2 || BM_ == B_TMA_MN3 || BM_ == B_GATHER_WG || BM_ == B_SCALAR_DGRAD ||
-                           BM_ == B_SCALAR_WG || BM_ == B_TMA_IM2COL);
+                           BM_ == B_SCALAR_WG || BM_ == B_TMA_IM2COL || BM_ == B_GATHER_SMALLC);
     constexpr bool A_TMA = (AM == A_TMA_K2 || AM == A_TMA_K3 || AM == A_TMA_MN2 || AM == A_TMA_IM2COL);
     constexpr bool B_TMA = (BM_ == B_TMA_K2 || BM_ == B_TMA_K3 || BM_ == B_TMA_MN2 || BM_ == B_TMA_MN3 ||
                             BM_ == B_TMA_IM2COL);
-    constexpr bool GATHER = !A_TMA || !B_TMA;
+    constexpr bool B_RES = (BM_ == B_RESIDENT);
+    constexpr bool GATHER = !A_TMA || (!B_TMA && !B_RES);
+    constexpr bool SPLITK = (EPI == EPI_WGRAD_CHAIN || EPI == EPI_WGRAD_SMALLC);
     constexpr bool A_ASYNC = (AM == A_GATHER_FWD || AM == A_GATHER_DGRAD);
     constexpr bool B_ASYNC = (BM_ == B_GATHER_WG);
     // MN-major atoms: 8-row (bf16, SWIZZLE_128B) or 4-row (tf32, 128B_BASE32B) groups.
@@ -39,12 +41,14 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
     const int B_BYTES = p.b_bytes;
     uint8_t* sA = smem;
     uint8_t* sB = smem + (size_t)S * A_BYTES;
-    uint64_t* bars = (uint64_t*)(sB + (size_t)S * B_BYTES);
+    uint8_t* sBres = sB + (size_t)S * B_BYTES;  // B_RESIDENT: whole filter, k-block after k-block
+    uint64_t* bars = (uint64_t*)(sBres + (B_RES ? p.bres_bytes : 0));
     uint64_t* full = bars;
     uint64_t* empty = bars + S;
     uint64_t* tfull = bars + 2 * S;      // [2]
     uint64_t* tempty = bars + 2 * S + 2; // [2]
-    uint32_t* tmem_slot = (uint32_t*)(bars + 2 * S + 4);
+    uint64_t* bres_bar = bars + 2 * S + 4;
+    uint32_t* tmem_slot = (uint32_t*)(bars + 2 * S + 5);
 
     const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
     const int mt = (p.M + 127) / 128, nt = (p.N + p.BN - 1) / p.BN;
@@ -61,6 +65,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
             mbar_init(smem_u32(&tfull[a]), 1);
             mbar_init(smem_u32(&tempty[a]), 4);
         }
+        mbar_init(smem_u32(bres_bar), 128);
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     if (warp == 4) {
@@ -81,7 +86,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
         m0 = (rem - ntile * mt) * 128;
         n0 = ntile * p.BN;
         kb_begin = 0; kb_end = p.num_kb;
-        if (EPI == EPI_WGRAD_CHAIN) {
+        if (SPLITK) {
             kb_begin = z * p.kb_per_split;
             kb_end = min(p.num_kb, kb_begin + p.kb_per_split);
         }
@@ -93,6 +98,23 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
         const T* gx = (const T*)p.gsrc;
         const int lag = min(S - 1, 3);
         const int gch = (AM == A_GATHER_DGRAD || (AM == A_TMA_IM2COL && p.im2col_dgrad)) ? p.K : p.C;
+        if constexpr (B_RES) {
+            // Stage the whole zero-padded filter once: B(n, k') with k' = (r, s8, c')
+            // -> w[n][r][s][c'] (0 for s >= S or c' >= C), K-major SW128 per k-block.
+            const T* wsrc = (const T*)p.bsrc;
+            const int groups = p.s8 / 8;  // tap groups of 8 per filter row
+            const int per_kb = p.BN * KB;
+            for (int idx = t; idx < p.num_kb * per_kb; idx += 128) {
+                const int kb = idx / per_kb, rem = idx - kb * per_kb;
+                const int n = rem / KB, e = rem - n * KB;
+                const int r = kb / groups, s_ = (kb - r * groups) * 8 + e / p.cp, c = e % p.cp;
+                float v = 0.f;
+                if (n < p.N && s_ < p.S && c < p.C) v = (float)wsrc[(((size_t)n * p.R + r) * p.S + s_) * p.C + c];
+                st_shared_elt<T>(smem_u32(sBres) + (uint32_t)(kb * p.BN * 128) + kmaj_off(n, e * ELT), (T)v);
+            }
+            fence_proxy_async();
+            mbar_arrive(smem_u32(bres_bar));
+        }
         int s = 0;
         uint32_t ph = 0;
         int git = 0;  // k-blocks issued by this CTA so far (for the lagged arrivals)
@@ -107,13 +129,13 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
             int rh[8], rw[8];
             long long rbase[8];
             bool rv[8];
-            if constexpr (AM == A_GATHER_FWD || AM == A_GATHER_DGRAD) {
+            if constexpr (AM == A_GATHER_FWD || AM == A_GATHER_DGRAD || AM == A_GATHER_SMALLC) {
 #pragma unroll
                 for (int i = 0; i < 8; ++i) {
                     const int m = m0 + t / 8 + 16 * i;
                     rv[i] = m < p.M;
                     const int mm = rv[i] ? m : 0;
-                    if (AM == A_GATHER_FWD) {
+                    if (AM == A_GATHER_FWD || AM == A_GATHER_SMALLC) {
                         const int pq = p.P * p.Q;
                         const int n = mm / pq, rem = mm - n * pq, pp = rem / p.Q, qq = rem - pp * p.Q;
                         rh[i] = pp * p.stride - p.pad; rw[i] = qq * p.stride - p.pad;
@@ -157,6 +179,56 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                     ic_h = pp * p.stride - p.pad; ic_w = qq * p.stride - p.pad;
                 }
             }
+            // Small-C FWD gather: packed 16-B chunks of 8 rows for one k-block.
+            uint32_t pk[8][4];
+            auto smallc_load = [&](int kbl) {
+                if constexpr (AM == A_GATHER_SMALLC) {
+                    const int groups = p.s8 / 8;
+                    const int r = kbl / groups, sx = (kbl - r * groups) * 8 + (t & 7);
+                    const long long koff = ((long long)r * p.W + sx) * p.C;
+#pragma unroll
+                    for (int i = 0; i < 8; ++i) {
+                        const bool v = sx < p.S && rv[i] && (unsigned)(rh[i] + r) < (unsigned)p.H &&
+                                       (unsigned)(rw[i] + sx) < (unsigned)p.W;
+                        __align__(16) T vals[16 / ELT];
+#pragma unroll
+                        for (int u = 0; u < 16 / ELT; ++u)
+                            vals[u] = (v && u < p.C) ? gx[rbase[i] + koff + u] : (T)0.f;
+                        const uint4 q = *reinterpret_cast<const uint4*>(vals);
+                        pk[i][0] = q.x; pk[i][1] = q.y; pk[i][2] = q.z; pk[i][3] = q.w;
+                    }
+                }
+            };
+            // Small-C WGRAD gather: 16-B padded-pixel chunks for KB/16 rows x atoms.
+            uint32_t bpk[KB / 16][256 / KB][4];
+            auto wg_smallc_load = [&](int kbl) {
+                if constexpr (BM_ == B_GATHER_SMALLC) {
+                    const int chunk = t & 7;
+                    const int groups = p.s8 / 8;
+                    const int pq = p.P * p.Q;
+#pragma unroll
+                    for (int i = 0; i < KB / 16; ++i) {
+                        const int m = kbl * KB + t / 8 + 16 * i;
+                        const bool mv = m < p.kred;
+                        const int mm = mv ? m : 0;
+                        const int n = mm / pq, rem = mm - n * pq, pp = rem / p.Q, qq = rem - pp * p.Q;
+#pragma unroll
+                        for (int a = 0; a < 256 / KB; ++a) {
+                            const int grp = (n0 * ELT) / 128 + a;  // tap group index = atom index
+                            const int r = grp / groups, sx = (grp - r * groups) * 8 + chunk;
+                            const int h = pp * p.stride - p.pad + r, w = qq * p.stride - p.pad + sx;
+                            const bool v = a < p.bn_atoms && mv && r < p.R && sx < p.S && h >= 0 && h < p.H &&
+                                           w >= 0 && w < p.W;
+                            __align__(16) T vals[16 / ELT];
+                            const T* src = v ? gx + (((size_t)n * p.H + h) * p.W + w) * p.C : gx;
+#pragma unroll
+                            for (int u = 0; u < 16 / ELT; ++u) vals[u] = (v && u < p.C) ? src[u] : (T)0.f;
+                            const uint4 q = *reinterpret_cast<const uint4*>(vals);
+                            bpk[i][a][0] = q.x; bpk[i][a][1] = q.y; bpk[i][a][2] = q.z; bpk[i][a][3] = q.w;
+                        }
+                    }
+                }
+            };
             // WGRAD TMA im2col: pixel (n,p,q) of the first row of the k-block,
             // walked incrementally (KB pixels per k-block).
             int wb_n = 0, wb_p = 0, wb_q = 0;
@@ -256,6 +328,19 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                         }
                     }
                 }
+                if constexpr (AM == A_GATHER_SMALLC) {
+                    // k-block = filter row r, taps s0..s0+7; chunk j = tap s0 + j holds the
+                    // pixel's C (< 16 B) channels zero-padded to 16 B.  The registers
+                    // were filled one k-block ahead (software pipelining of the
+                    // synchronous loads): store them, then prefetch the next k-block.
+                    const uint32_t soff = kmaj_off(t / 8, (t & 7) * 16);
+                    if (kb == kb_begin) smallc_load(kb);
+#pragma unroll
+                    for (int i = 0; i < 8; ++i)
+                        asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(aT + soff + i * 2048),
+                                     "r"(pk[i][0]), "r"(pk[i][1]), "r"(pk[i][2]), "r"(pk[i][3])
+                                     : "memory");
+                }
                 if constexpr (WALK) {
                     g_c0 += KB;
                     if (g_c0 >= gch) { g_c0 = 0; if (++g_s == p.tapS) { g_s = 0; ++g_r; } }
@@ -321,6 +406,23 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                             cp_async16(bT + (uint32_t)(a * KB * 128) + mn_row_off<ELT>(row, chunk * 16), src, v);
                         }
                     }
+                } else if constexpr (BM_ == B_GATHER_SMALLC) {
+                    // WGRAD small C: B(j' = (r, s8, c'), m) MN-major; an atom (128 B)
+                    // is one tap group (r, s0..s0+7), chunk = tap, 16 B = padded pixel.
+                    // Registers filled one k-block ahead (see wg_smallc_load).
+                    const int chunk = t & 7;
+                    if (kb == kb_begin) wg_smallc_load(kb);
+#pragma unroll
+                    for (int i = 0; i < KB / 16; ++i)
+#pragma unroll
+                        for (int a = 0; a < 256 / KB; ++a)
+                            if (a < p.bn_atoms)
+                                asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(
+                                                 bT + (uint32_t)(a * KB * 128) +
+                                                 mn_row_off<ELT>(t / 8 + 16 * i, chunk * 16)),
+                                             "r"(bpk[i][a][0]), "r"(bpk[i][a][1]), "r"(bpk[i][a][2]),
+                                             "r"(bpk[i][a][3])
+                                             : "memory");
                 } else if constexpr (BM_ == B_SCALAR_K) {
                     // B rows n0.. (BN of them) x KB elements from a dense row-major matrix with pitch ldb
                     const T* bs = (const T*)p.bsrc;
@@ -381,6 +483,10 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                         mbar_arrive(fb);
                     }
                 }
+                // Small-C gathers: prefetch the next k-block's pixels into registers
+                // after this stage is published (a fence would otherwise wait for them).
+                if constexpr (AM == A_GATHER_SMALLC) { if (kb + 1 < kb_end) smallc_load(kb + 1); }
+                if constexpr (BM_ == B_GATHER_SMALLC) { if (kb + 1 < kb_end) wg_smallc_load(kb + 1); }
             }
         }
         if constexpr (GATHER && (A_ASYNC || B_ASYNC)) {
@@ -397,6 +503,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
         uint32_t ph = 0;
         int acc = 0;
         uint32_t aph = 0;
+        if constexpr (B_RES) mbar_wait(smem_u32(bres_bar), 0u);  // staged filter is ready
         for (int tile = blockIdx.x; tile < total_tiles; tile += gridDim.x) {
             int m0, n0, z, kb_begin, kb_end;
             decode(tile, m0, n0, z, kb_begin, kb_end);
@@ -408,7 +515,8 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                 tc_fence_after();
                 if (lane == 0) {
                     const uint32_t aT = smem_u32(sA + (size_t)s * A_BYTES);
-                    const uint32_t bT = smem_u32(sB + (size_t)s * B_BYTES);
+                    const uint32_t bT = B_RES ? smem_u32(sBres) + (uint32_t)(kb * p.BN * 128)
+                                              : smem_u32(sB + (size_t)s * B_BYTES);
 #pragma unroll
                     for (int j = 0; j < KB / UMMA_K; ++j) {
                         const uint64_t ad = A_MN ? sdesc(aT + j * UMMA_K * 128, KB * 128, MN_SBO, MN_LAYOUT)
@@ -467,7 +575,17 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                 }
                 if (m >= p.M) continue;
                 const int nb = n0 + c0;
-                if constexpr (EPI == EPI_WGRAD_CHAIN) {
+                if constexpr (EPI == EPI_WGRAD_SMALLC) {
+                    // padded column j' = (r, s8, c') -> dw column (r*S + s)*C + c (skip padding)
+                    float* drow = outF + (size_t)m * p.ldc;
+#pragma unroll
+                    for (int j = 0; j < 32; ++j) {
+                        const int jp = nb + j;
+                        const int c = jp % p.cp, t2 = jp / p.cp, s_ = t2 % p.s8, r = t2 / p.s8;
+                        if (jp < p.N && c < p.C && s_ < p.S)
+                            atomicAdd(drow + (r * p.S + s_) * p.C + c, p.alpha * __uint_as_float(v[j]));
+                    }
+                } else if constexpr (EPI == EPI_WGRAD_CHAIN) {
                     // dw += alpha * partial (beta was applied by a prescale launch);
                     // 16-byte vector reductions in L2 (red.global.add.v4.f32).
                     float* d = outF + (size_t)m * p.ldc + nb;

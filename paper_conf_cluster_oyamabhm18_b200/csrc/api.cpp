@@ -54,6 +54,8 @@ bool make_geom(const mucu_conv_desc_t* d, Geom* g) {
 
 bool is_pointwise(const Geom& g) { return g.r == 1 && g.s == 1 && g.pad == 0 && g.stride == 1; }
 
+bool small_c_tc(const Geom& g) { return g.math != MUCU_MATH_F32 && g.c * elt_size(g.math) < 16; }
+
 bool algo_eligible(const Geom& g, int type, int algo) {
     if (type < MUCU_FWD || type > MUCU_BWD_FILTER) return false;
     switch (algo) {
@@ -81,6 +83,16 @@ mucu_status_t ws_layout(const Geom& g, int type, int algo, int32_t b, WsLayout* 
     if (algo == MUCU_ALGO_IM2COL_GEMM) {
         L->kpitch = (int32_t)align_up(RSC, vec);
         if (is_pointwise(g)) { L->kpitch = g.c; return MUCU_OK; }
+        if (small_c_tc(g) && type != MUCU_BWD_DATA) {
+            // Tensor-core small-C (RGB) layers: the explicit transform is a
+            // channel pad of x to 16 B per pixel (the GEMM walks the taps);
+            // b*H*W*16 bytes instead of the full b*P*Q*R*S*C im2col matrix.
+            L->kpitch = 16 / (int32_t)elt;
+            L->a_off = 0;
+            L->a_bytes = align_up((uint64_t)b * g.h * g.w * 16, 256);
+            L->total = L->a_bytes;
+            return MUCU_OK;
+        }
         if (type == MUCU_BWD_DATA) {
             L->filter_padded = (RSC * elt) % 16 != 0;
             const uint64_t fpitch = align_up(RSC, vec);

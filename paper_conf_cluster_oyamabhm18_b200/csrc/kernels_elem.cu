@@ -507,6 +507,31 @@ __global__ void scale_kernel(float* __restrict__ p, int64_t n, float beta) {
 }
 }  // namespace
 
+namespace {
+// One thread per pixel: reads C (< 16 B) channels, writes one 16-B vector.
+template <class T>
+__global__ void pad_channels_kernel(const T* __restrict__ x, T* __restrict__ xp, int64_t pixels, int C) {
+    constexpr int V = 16 / sizeof(T);
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < pixels; i += (int64_t)gridDim.x * blockDim.x) {
+        __align__(16) T v[V];
+#pragma unroll
+        for (int c = 0; c < V; ++c) v[c] = c < C ? x[i * C + c] : from_f<T>(0.f);
+        *reinterpret_cast<uint4*>(xp + i * V) = *reinterpret_cast<const uint4*>(v);
+    }
+}
+}  // namespace
+
+int launch_pad_channels(const Geom& g, int32_t b, const void* x, void* xp, cudaStream_t st) {
+    const int64_t pixels = (int64_t)b * g.h * g.w;
+    const int grid = grid_for(pixels, 256);
+    if (g.math == MUCU_MATH_BF16)
+        pad_channels_kernel<__nv_bfloat16><<<grid, 256, 0, st>>>((const __nv_bfloat16*)x, (__nv_bfloat16*)xp, pixels, g.c);
+    else
+        pad_channels_kernel<float><<<grid, 256, 0, st>>>((const float*)x, (float*)xp, pixels, g.c);
+    count_launch();
+    return (int)cudaGetLastError();
+}
+
 int launch_scale(int64_t n, float beta, float* p, cudaStream_t st) {
     scale_kernel<<<grid_for(n, 256), 256, 0, st>>>(p, n, beta);
     count_launch();

@@ -31,6 +31,7 @@
 #include <cstdio>
 #include <cstring>
 #include <mutex>
+#include <type_traits>
 
 #include "mucudnn_internal.h"
 
@@ -140,6 +141,9 @@ enum AMode : int {
     A_SCALAR_DGRAD = 6,// transposed-conv gather of dy, element-wise (any K)
     A_TMA_IM2COL = 7,  // TMA im2col mode: FWD (x) or stride-1 DGRAD (dy, flipped taps), 128 pixels x KB channels
     A_GATHER_SMALLC = 8, // FWD, C*elt < 16 B (RGB layer): one 16-B chunk per filter tap, channels zero-padded
+    A_GATHER_SMALLC_PAD = 9, // same K' layout from a channel-padded copy of x (16 B per pixel): cp.async
+    A_TMA_IM2COL_SMALLC = 10, // same K' layout from the padded copy by TMA im2col: one 128-pixel x 16-B box
+                              // per tap, SWIZZLE_NONE core matrices (LBO 2 KB between taps, SBO 128 B)
 };
 enum BMode : int {
     B_TMA_K2 = 0,      // dense K-major {K, cols}
@@ -153,6 +157,7 @@ enum BMode : int {
     B_TMA_IM2COL = 8,  // WGRAD implicit im2col of x by TMA im2col mode, MN-major (KB pixels x 128 B per atom)
     B_RESIDENT = 9,    // whole (padded) filter staged in smem once per CTA (small-C FWD)
     B_GATHER_SMALLC = 10, // WGRAD small C: x pixels as 16-B tap chunks, MN-major
+    B_GATHER_SMALLC_PAD = 11, // WGRAD small C from the channel-padded copy of x: cp.async
 };
 enum EpiMode : int { EPI_STORE = 0, EPI_WGRAD_CHAIN = 1, EPI_WGRAD_SMALLC = 2 };
 
@@ -187,6 +192,9 @@ struct TcArgs {
     // channels zero-padded to cp = 16 B / elt; s8 = S rounded up to 8.
     int cp, s8;
     int bres_bytes;          // B_RESIDENT: smem bytes of the staged filter
+    int max_lag;             // cp.async stages kept in flight per producer thread (<= 6)
+    int debug;               // MUCU_TC_DEBUG bits (timing experiments only): 1 skip stores, 2 skip A gather
+    int mt;                  // 128-row halves per tile (1, or 2 for 256-row tiles with narrow N)
     // epilogue
     void* out;
     long long ldc;
@@ -307,7 +315,8 @@ EncodeIm2colFn get_encode_im2col() {
 // of start pixels is [lower, dim - 1 + upper] per spatial dim (W, H order),
 // walked with the traversal stride; channelsPerPixel = 128 B of channels.
 bool make_im2col_map(CUtensorMap* tm, int elt, const void* base, int C, int W, int H, int N, int lower_w,
-                     int lower_h, int upper_w, int upper_h, int pixels, int stride, bool mn_major) {
+                     int lower_h, int upper_w, int upper_h, int pixels, int stride, bool mn_major,
+                     bool pixel16 = false) {
     EncodeIm2colFn enc = get_encode_im2col();
     if (!enc) return false;
     if (lower_w < -128 || lower_h < -128 || upper_w > 127 || upper_h > 127 || lower_w > 127 || upper_h < -128)
@@ -316,9 +325,13 @@ bool make_im2col_map(CUtensorMap* tm, int elt, const void* base, int C, int W, i
     cuuint64_t s[3] = {(cuuint64_t)C * elt, (cuuint64_t)W * C * elt, (cuuint64_t)H * W * C * elt};
     int lo[2] = {lower_w, lower_h}, hi[2] = {upper_w, upper_h};
     cuuint32_t es[4] = {1, (cuuint32_t)stride, (cuuint32_t)stride, 1};
-    const CUtensorMapSwizzle sw = (mn_major && elt == 4) ? CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B : CU_TENSOR_MAP_SWIZZLE_128B;
+    // pixel16: 16 B of channels per pixel, unswizzled (core-matrix rows of 16 B).
+    const CUtensorMapSwizzle sw = pixel16 ? CU_TENSOR_MAP_SWIZZLE_NONE
+                                  : (mn_major && elt == 4) ? CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B
+                                                           : CU_TENSOR_MAP_SWIZZLE_128B;
+    const cuuint32_t cpp = pixel16 ? (cuuint32_t)(16 / elt) : (cuuint32_t)(128 / elt);
     CUresult r = enc(tm, elt == 2 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4,
-                     const_cast<void*>(base), d, s, lo, hi, (cuuint32_t)(128 / elt), (cuuint32_t)pixels, es,
+                     const_cast<void*>(base), d, s, lo, hi, cpp, (cuuint32_t)pixels, es,
                      CU_TENSOR_MAP_INTERLEAVE_NONE, sw, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                      CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
     return r == CUDA_SUCCESS;
@@ -364,7 +377,8 @@ struct Launch {
 template <int ELT, int AM, int BM_, int EPI>
 int launch_t(Launch& L, cudaStream_t st) {
     auto kern = tc_conv_gemm<ELT, AM, BM_, EPI>;
-    const int smem = 1024 + L.a.stages * (128 * 128 + L.a.b_bytes) + L.a.bres_bytes + (2 * L.a.stages + 5) * 8 + 64;
+    const int smem = 1024 + L.a.stages * (L.a.mt * 128 * 128 + L.a.b_bytes) + L.a.bres_bytes +
+                     (2 * L.a.stages + 5) * 8 + 64;
     static int configured = 0;  // per instantiation
     if (configured < smem) {
         cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 232448);
@@ -376,16 +390,34 @@ int launch_t(Launch& L, cudaStream_t st) {
     return (int)cudaGetLastError();
 }
 
+void size_stages(TcArgs& a) {
+    const int cols = 2 * a.mt * a.BN;  // 2 accumulators x mt halves
+    a.tmem_cols = cols <= 64 ? 64 : cols <= 128 ? 128 : cols <= 256 ? 256 : 512;
+    const int stage_bytes = a.mt * 128 * 128 + a.b_bytes;
+    a.stages = std::min(env_int("MUCU_MAX_STAGES", 8), (200 * 1024) / stage_bytes);
+    if (a.stages < 2) a.stages = 2;
+}
+
 void finalize_tiling(Launch& L, int elt, int step = 32) {
     TcArgs& a = L.a;
     a.BN = pick_bn(a.N, step);
     if (const int fb = env_int("MUCU_FORCE_BN", 0)) a.BN = std::max(step, fb - fb % step);
-    a.tmem_cols = 2 * a.BN <= 64 ? 64 : 2 * a.BN <= 128 ? 128 : 2 * a.BN <= 256 ? 256 : 512;  // 2 accumulators
     a.bn_atoms = (a.BN * elt + 127) / 128;
     a.b_bytes = std::max(a.BN * 128, a.bn_atoms * (128 / elt) * 128);
-    const int stage_bytes = 128 * 128 + a.b_bytes;
-    a.stages = std::min(env_int("MUCU_MAX_STAGES", 8), (200 * 1024) / stage_bytes);
-    if (a.stages < 2) a.stages = 2;
+    a.mt = 1;
+    size_stages(a);
+}
+
+// 256-row tiles (two 128-row accumulators sharing each B tile) for narrow N:
+// back-to-back MMAs of N <= 128 on ONE accumulator are latency-bound, two
+// interleaved accumulation chains are not.  TMA-fed A operands only; needs at
+// least one 256-row tile per SM.
+void use_mt2(Launch& L, int num_sms) {
+    TcArgs& a = L.a;
+    if (a.BN > 128 || env_int("MUCU_MT2", 1) == 0) return;
+    if (ceil_div(a.M, 256) < num_sms) return;
+    a.mt = 2;
+    size_stages(a);
 }
 
 }  // namespace
@@ -408,6 +440,8 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
     A.H = g.h; A.W = g.w; A.C = g.c; A.P = g.p; A.Q = g.q; A.R = g.r; A.S = g.s; A.pad = g.pad;
     A.stride = g.stride; A.K = g.k;
     A.tapR = g.r; A.tapS = g.s;
+    A.max_lag = std::min(6, std::max(1, env_int("MUCU_MAX_LAG", 6)));
+    A.debug = env_int("MUCU_TC_DEBUG", 0);
     A.alpha = alpha; A.beta = beta; A.out = out; A.out_bf16 = bf ? 1 : 0; A.sem = sem.sem;
     auto map2 = [&](CUtensorMap* tm, const void* base, uint64_t d0, uint64_t d1, uint64_t pitch_elems, uint32_t b0,
                     uint32_t b1, bool mn = false) {
@@ -424,7 +458,7 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
     // Persistent launch: one CTA per SM (at most one per tile).
     auto grid2 = [&](int batch) {
         A.num_z = batch;
-        const int64_t tiles = ceil_div(A.M, 128) * ceil_div(A.N, A.BN) * batch;
+        const int64_t tiles = ceil_div(A.M, 128 * A.mt) * ceil_div(A.N, A.BN) * batch;
         L.grid = dim3((unsigned)std::max<int64_t>(1, std::min<int64_t>(tiles, num_sms)));
     };
     const bool Aok = (g.c % KB) == 0;  // vector gathers over C
@@ -445,7 +479,9 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
             if (use_tma_im2col() &&
                 make_im2col_map(&L.ta, elt, in0, g.c, g.w, g.h, b, -g.pad, -g.pad, g.pad - (g.s - 1),
                                 g.pad - (g.r - 1), 128, g.stride, false)) {
-                A.tma_bytes = 128 * 128 + A.BN * 128;
+                use_mt2(L, num_sms);
+                grid2(1);
+                A.tma_bytes = 16384 * A.mt + A.BN * 128;
                 return LAUNCH(A_TMA_IM2COL, B_TMA_K2, EPI_STORE);
             }
             A.tma_bytes = A.BN * 128;
@@ -474,6 +510,30 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         }
         return err;
     }
+    if (type == MUCU_FWD && algo == MUCU_ALGO_IM2COL_GEMM && small_c_tc(g)) {
+        // RGB-like layer: x -> channel-padded copy (16 B / pixel) in the workspace,
+        // then the tap-walking GEMM with async 16-B gathers and the staged filter.
+        err = launch_pad_channels(g, b, in0, ws + WL.a_off, st);
+        if (err) return err;
+        A.M = (int)(b * PQ); A.N = g.k; A.ldc = g.k; A.gsrc = ws + WL.a_off; A.bsrc = in1;
+        A.cp = 16 / elt; A.s8 = (int)align_up((uint64_t)g.s, 8);
+        A.num_kb = g.r * (A.s8 / 8);
+        finalize_tiling(L, elt);
+        if (ceil_div(A.N, A.BN) != 1) return -1;
+        A.b_bytes = 0;
+        A.bres_bytes = A.num_kb * A.BN * 128;
+        A.stages = std::min(8, (kSmemBudget - A.bres_bytes) / (128 * 128));
+        if (A.stages < 2) return -1;
+        grid2(1);
+        A.tma_bytes = 0;
+        // TMA im2col over the 16-B pixels works for bf16 but measured no faster
+        // than the cp.async gather (and hangs for fp32): opt-in only.
+        if (elt == 2 && env_int("MUCU_SMALLC_TMA", 0) &&
+            make_im2col_map(&L.ta, elt, A.gsrc, A.cp, g.w, g.h, b, -g.pad, -g.pad, g.pad - (g.s - 1),
+                            g.pad - (g.r - 1), 128, g.stride, false, true))
+            return LAUNCH(A_TMA_IM2COL_SMALLC, B_RESIDENT, EPI_STORE);
+        return LAUNCH(A_GATHER_SMALLC_PAD, B_RESIDENT, EPI_STORE);
+    }
     if (type == MUCU_FWD && algo == MUCU_ALGO_IM2COL_GEMM) {
         const void* colp = in0;
         int kpitch = g.c;
@@ -495,10 +555,11 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         }
         A.M = (int)(b * PQ); A.N = g.k; A.num_kb = (int)ceil_div(RSC, KB); A.ldc = g.k;
         finalize_tiling(L, elt);
+        use_mt2(L, num_sms);
         grid2(1);
         if (!map2(&L.ta, colp, RSC, (uint64_t)A.M, kpitch, KB, 128)) return -1;
         if (!map2(&L.tb, wp, RSC, g.k, wpitch, KB, A.BN)) return -1;
-        A.tma_bytes = 128 * 128 + A.BN * 128;
+        A.tma_bytes = 16384 * A.mt + A.BN * 128;
         return LAUNCH(A_TMA_K2, B_TMA_K2, EPI_STORE);
     }
     if (algo == MUCU_ALGO_WINOGRAD_2X2_3X3) {
@@ -521,7 +582,7 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         grid2(16);
         if (!map3(&L.ta, V, I, Tt, 16, I, Tt * I, KB, 128, 1)) return -1;
         if (!map3(&L.tb, ws, I, O, 16, I, (uint64_t)O * I, KB, A.BN, 1)) return -1;
-        A.tma_bytes = 128 * 128 + A.BN * 128;
+        A.tma_bytes = 16384 * A.mt + A.BN * 128;
         err = LAUNCH(A_TMA_K3, B_TMA_K3, EPI_STORE);
         if (err) return err;
         return launch_wg_output(g, dg, b, alpha, Mx, beta, out, st);
@@ -559,7 +620,11 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
                     !make_im2col_map(&L.ta, elt, in0, g.k, g.q, g.p, b, lw, lh, lw + Wph - g.q, lh + Hph - g.p,
                                      128, 1, false))
                     return -1;
-                A.tma_bytes = 128 * 128 + (bvec ? A.bn_atoms * KB * 128 : 0);
+                A.mt = 1;
+                size_stages(A);
+                use_mt2(L, num_sms);
+                grid2(1);
+                A.tma_bytes = 16384 * A.mt + (bvec ? A.bn_atoms * KB * 128 : 0);
                 err = bvec ? LAUNCH(A_TMA_IM2COL, B_TMA_MN3, EPI_STORE) : LAUNCH(A_TMA_IM2COL, B_SCALAR_DGRAD, EPI_STORE);
                 if (err) return err;
             }
@@ -582,7 +647,9 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
                 make_im2col_map(&L.ta, elt, in0, g.k, g.q, g.p, b, lw, lh, lw + g.w - g.q, lh + g.h - g.p, 128, 1,
                                 false)) {
                 A.im2col_dgrad = 1;
-                A.tma_bytes = 128 * 128 + A.bn_atoms * KB * 128;
+                use_mt2(L, num_sms);
+                grid2(1);
+                A.tma_bytes = 16384 * A.mt + A.bn_atoms * KB * 128;
                 return LAUNCH(A_TMA_IM2COL, B_TMA_MN3, EPI_STORE);
             }
             A.tma_bytes = A.bn_atoms * KB * 128;
@@ -608,11 +675,12 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         if (pw) { A.ldc = g.c; }
         else { A.ldc = WL.kpitch; A.out = ws + WL.a_off; A.out_bf16 = 0; A.alpha = 1.f; A.beta = 0.f; }
         finalize_tiling(L, elt);
+        use_mt2(L, num_sms);
         grid2(1);
         if (RSC < atom) return -1;
         if (!map2(&L.ta, in0, g.k, (uint64_t)A.M, g.k, KB, 128)) return -1;
         if (!map2(&L.tb, wp, RSC, g.k, wpitch, atom, KB, true)) return -1;
-        A.tma_bytes = 128 * 128 + A.bn_atoms * KB * 128;
+        A.tma_bytes = 16384 * A.mt + A.bn_atoms * KB * 128;
         err = LAUNCH(A_TMA_K2, B_TMA_MN2, EPI_STORE);
         if (err || pw) return err;
         return launch_col2im(g, b, alpha, (const float*)(ws + WL.a_off), WL.kpitch, beta, out, st);
@@ -643,6 +711,23 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         grid2((int)nsplit);
         if (!map2(&L.ta, in1, g.k, (uint64_t)Mpix, g.k, atom, KB, true)) return -1;
         const int a_bytes = 128 * KB * elt;
+        if (algo == MUCU_ALGO_IM2COL_GEMM && small_c_tc(g)) {
+            // RGB-like layer: channel-padded copy of x, padded columns j' = (r, s8, c').
+            err = launch_pad_channels(g, b, in0, ws + WL.a_off, st);
+            if (err) return err;
+            A.gsrc = ws + WL.a_off;
+            A.cp = 16 / elt; A.s8 = (int)align_up((uint64_t)g.s, 8);
+            A.N = g.r * A.s8 * A.cp;
+            finalize_tiling(L, elt, atom);
+            const int64_t t2 = ceil_div(A.N, A.BN) * ceil_div(A.M, 128);
+            int64_t ns2 = std::min<int64_t>(std::min<int64_t>(std::max<int64_t>(1, (2LL * num_sms) / t2),
+                                                              std::max<int64_t>(1, nkb / 16)), 65535);
+            A.kb_per_split = (int)ceil_div(nkb, ns2);
+            ns2 = ceil_div(nkb, A.kb_per_split);
+            grid2((int)ns2);
+            A.tma_bytes = a_bytes;
+            return LAUNCH(A_TMA_MN2, B_GATHER_SMALLC_PAD, EPI_WGRAD_SMALLC);
+        }
         if (algo == MUCU_ALGO_IM2COL_GEMM) {
             const void* colp = in0;
             int64_t kp = g.c;

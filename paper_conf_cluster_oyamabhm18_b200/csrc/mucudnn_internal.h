@@ -34,6 +34,7 @@ inline int64_t ceil_div(int64_t a, int64_t b) { return (a + b - 1) / b; }
 // the benchmark pass and the executor.
 bool algo_eligible(const Geom& g, int type, int algo);
 bool is_pointwise(const Geom& g);  // 1x1, stride 1, pad 0: im2col(x) == x
+bool small_c_tc(const Geom& g);    // tensor-core math and C*elt < 16 B (RGB input layer)
 
 // Workspace layout of one micro-configuration (all offsets 256-B aligned).
 // `fixed` = b-independent prefix (padded filter / Winograd U) computed once per
@@ -89,6 +90,8 @@ int launch_col2im(const Geom& g, int32_t b, float alpha, const float* dcol, int3
                   void* dx, cudaStream_t st);
 int launch_wg_filter(const Geom& g, bool dgrad, const void* w, void* U, cudaStream_t st);
 int launch_scale(int64_t n, float beta, float* p, cudaStream_t st);  // p *= beta (beta == 0: p = 0)
+// x[b,H,W,C] -> xp[b,H,W,16/elt] with channels zero-padded to 16 B per pixel.
+int launch_pad_channels(const Geom& g, int32_t b, const void* x, void* xp, cudaStream_t st);
 int launch_wg_input(const Geom& g, bool dgrad, int32_t b, const void* in, void* V, cudaStream_t st);
 int launch_wg_output(const Geom& g, bool dgrad, int32_t b, float alpha, const float* M, float beta,
                      void* out, cudaStream_t st);

@@ -18,18 +18,21 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
     using T = typename Elt<ELT>::T;
     constexpr int KB = 128 / ELT;            // K elements per stage
     constexpr int UMMA_K = 32 / ELT;         // K elements per MMA
-    constexpr int A_BYTES = 128 * 128;       // 128 rows x 128 B
+    const int A_BYTES = p.mt * 128 * 128;    // p.mt blocks of 128 rows x 128 B (tile M = 128 * p.mt)
     constexpr bool A_MN = (AM == A_TMA_MN2);
     constexpr bool B_MN = (BM_ == B_TMA_MN2 || BM_ == B_TMA_MN3 || BM_ == B_GATHER_WG || BM_ == B_SCALAR_DGRAD ||
-                           BM_ == B_SCALAR_WG || BM_ == B_TMA_IM2COL || BM_ == B_GATHER_SMALLC);
-    constexpr bool A_TMA = (AM == A_TMA_K2 || AM == A_TMA_K3 || AM == A_TMA_MN2 || AM == A_TMA_IM2COL);
+                           BM_ == B_SCALAR_WG || BM_ == B_TMA_IM2COL || BM_ == B_GATHER_SMALLC ||
+                           BM_ == B_GATHER_SMALLC_PAD);
+    constexpr bool A_TMA = (AM == A_TMA_K2 || AM == A_TMA_K3 || AM == A_TMA_MN2 || AM == A_TMA_IM2COL ||
+                            AM == A_TMA_IM2COL_SMALLC);
+    constexpr bool A_NOSWZ = (AM == A_TMA_IM2COL_SMALLC);  // unswizzled core matrices, one 2-KB box per tap
     constexpr bool B_TMA = (BM_ == B_TMA_K2 || BM_ == B_TMA_K3 || BM_ == B_TMA_MN2 || BM_ == B_TMA_MN3 ||
                             BM_ == B_TMA_IM2COL);
     constexpr bool B_RES = (BM_ == B_RESIDENT);
     constexpr bool GATHER = !A_TMA || (!B_TMA && !B_RES);
     constexpr bool SPLITK = (EPI == EPI_WGRAD_CHAIN || EPI == EPI_WGRAD_SMALLC);
-    constexpr bool A_ASYNC = (AM == A_GATHER_FWD || AM == A_GATHER_DGRAD);
-    constexpr bool B_ASYNC = (BM_ == B_GATHER_WG);
+    constexpr bool A_ASYNC = (AM == A_GATHER_FWD || AM == A_GATHER_DGRAD || AM == A_GATHER_SMALLC_PAD);
+    constexpr bool B_ASYNC = (BM_ == B_GATHER_WG || BM_ == B_GATHER_SMALLC_PAD);
     // MN-major atoms: 8-row (bf16, SWIZZLE_128B) or 4-row (tf32, 128B_BASE32B) groups.
     constexpr uint32_t MN_SBO = ELT == 2 ? 1024u : 512u;
     constexpr uint32_t MN_LAYOUT = ELT == 2 ? 2u : 1u;
@@ -51,7 +54,8 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
     uint32_t* tmem_slot = (uint32_t*)(bars + 2 * S + 5);
 
     const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
-    const int mt = (p.M + 127) / 128, nt = (p.N + p.BN - 1) / p.BN;
+    const int BMt = 128 * p.mt;  // tile rows: 128, or 256 as two 128-row halves with separate accumulators
+    const int mt = (p.M + BMt - 1) / BMt, nt = (p.N + p.BN - 1) / p.BN;
     const int per_z = mt * nt;
     const int total_tiles = per_z * p.num_z;
 
@@ -83,7 +87,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
         z = tile / per_z;
         const int rem = tile - z * per_z;
         const int ntile = rem / mt;
-        m0 = (rem - ntile * mt) * 128;
+        m0 = (rem - ntile * mt) * BMt;
         n0 = ntile * p.BN;
         kb_begin = 0; kb_end = p.num_kb;
         if (SPLITK) {
@@ -96,8 +100,16 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
         // =========================== producers ===========================
         const int t = threadIdx.x;  // 0..127
         const T* gx = (const T*)p.gsrc;
-        const int lag = min(S - 1, 3);
+        const int lag = min(S - 1, p.max_lag);
         const int gch = (AM == A_GATHER_DGRAD || (AM == A_TMA_IM2COL && p.im2col_dgrad)) ? p.K : p.C;
+        if constexpr (A_NOSWZ) {
+            // Taps past S are never loaded (their filter columns are zero); keep
+            // those A slots finite by zeroing every stage once.
+            for (int i = t; i < S * A_BYTES / 16; i += 128)
+                asm volatile("st.shared.v4.b32 [%0], {%1, %1, %1, %1};" ::"r"(smem_u32(sA) + i * 16), "r"(0)
+                             : "memory");
+            fence_proxy_async();
+        }
         if constexpr (B_RES) {
             // Stage the whole zero-padded filter once: B(n, k') with k' = (r, s8, c')
             // -> w[n][r][s][c'] (0 for s >= S or c' >= C), K-major SW128 per k-block.
@@ -129,17 +141,19 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
             int rh[8], rw[8];
             long long rbase[8];
             bool rv[8];
-            if constexpr (AM == A_GATHER_FWD || AM == A_GATHER_DGRAD || AM == A_GATHER_SMALLC) {
+            if constexpr (AM == A_GATHER_FWD || AM == A_GATHER_DGRAD || AM == A_GATHER_SMALLC ||
+                          AM == A_GATHER_SMALLC_PAD) {
 #pragma unroll
                 for (int i = 0; i < 8; ++i) {
                     const int m = m0 + t / 8 + 16 * i;
                     rv[i] = m < p.M;
                     const int mm = rv[i] ? m : 0;
-                    if (AM == A_GATHER_FWD || AM == A_GATHER_SMALLC) {
+                    if (AM == A_GATHER_FWD || AM == A_GATHER_SMALLC || AM == A_GATHER_SMALLC_PAD) {
                         const int pq = p.P * p.Q;
                         const int n = mm / pq, rem = mm - n * pq, pp = rem / p.Q, qq = rem - pp * p.Q;
                         rh[i] = pp * p.stride - p.pad; rw[i] = qq * p.stride - p.pad;
-                        rbase[i] = (((long long)n * p.H + rh[i]) * p.W + rw[i]) * p.C;
+                        rbase[i] = (((long long)n * p.H + rh[i]) * p.W + rw[i]) *
+                                   (AM == A_GATHER_SMALLC_PAD ? p.cp : p.C);
                     } else {
                         const int hw = p.H * p.W;
                         const int n = mm / hw, rem = mm - n * hw, hh = rem / p.W, ww = rem - hh * p.W;
@@ -160,24 +174,28 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
             // TMA im2col start pixel of this tile (FWD: output pixel m0 -> x origin;
             // DGRAD: dx pixel m0 -> dy origin h + pad - (R-1); phase mode: sub-grid
             // pixel (ii, jj) -> dy origin (i0 + ii - (tapR-1), j0 + jj - (tapS-1))).
-            int ic_w = 0, ic_h = 0, ic_n = 0;
-            if constexpr (AM == A_TMA_IM2COL) {
+            int ic_w[2] = {0, 0}, ic_h[2] = {0, 0}, ic_n[2] = {0, 0};  // per 128-row half (constant-indexed)
+            auto ic_of = [&](int mH, int& icw, int& ich, int& icn) {
                 if (p.ph_mode) {
                     const int hw = p.ph_H * p.ph_W;
-                    ic_n = m0 / hw;
-                    const int rem = m0 - ic_n * hw, ii = rem / p.ph_W, jj = rem - ii * p.ph_W;
-                    ic_h = p.ph_i0 + ii - (p.tapR - 1); ic_w = p.ph_j0 + jj - (p.tapS - 1);
+                    icn = mH / hw;
+                    const int rem = mH - icn * hw, ii = rem / p.ph_W, jj = rem - ii * p.ph_W;
+                    ich = p.ph_i0 + ii - (p.tapR - 1); icw = p.ph_j0 + jj - (p.tapS - 1);
                 } else if (p.im2col_dgrad) {
                     const int hw = p.H * p.W;
-                    ic_n = m0 / hw;
-                    const int rem = m0 - ic_n * hw, hh = rem / p.W, ww = rem - hh * p.W;
-                    ic_h = hh + p.pad - (p.R - 1); ic_w = ww + p.pad - (p.S - 1);
+                    icn = mH / hw;
+                    const int rem = mH - icn * hw, hq = rem / p.W, wq = rem - hq * p.W;
+                    ich = hq + p.pad - (p.R - 1); icw = wq + p.pad - (p.S - 1);
                 } else {
                     const int pq = p.P * p.Q;
-                    ic_n = m0 / pq;
-                    const int rem = m0 - ic_n * pq, pp = rem / p.Q, qq = rem - pp * p.Q;
-                    ic_h = pp * p.stride - p.pad; ic_w = qq * p.stride - p.pad;
+                    icn = mH / pq;
+                    const int rem = mH - icn * pq, pp = rem / p.Q, qq = rem - pp * p.Q;
+                    ich = pp * p.stride - p.pad; icw = qq * p.stride - p.pad;
                 }
+            };
+            if constexpr (AM == A_TMA_IM2COL || AM == A_TMA_IM2COL_SMALLC) {
+                ic_of(m0, ic_w[0], ic_h[0], ic_n[0]);
+                if (p.mt == 2) ic_of(m0 + 128, ic_w[1], ic_h[1], ic_n[1]);
             }
             // Small-C FWD gather: packed 16-B chunks of 8 rows for one k-block.
             uint32_t pk[8][4];
@@ -243,14 +261,37 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                 const uint32_t aT = smem_u32(sA + (size_t)s * A_BYTES);
                 const uint32_t bT = smem_u32(sB + (size_t)s * B_BYTES);
                 const uint32_t fb = smem_u32(&full[s]);
-                if ((A_TMA || B_TMA) && t == 0) {
+                if (A_NOSWZ && t == 0) {
+                    // k-block = filter row r, taps s0..s0+7 of the padded x (16 B per pixel)
+                    const int groups = p.s8 / 8;
+                    const int r = kb / groups, s0 = (kb - r * groups) * 8;
+                    const int nv = min(8, p.S - s0);
+                    mbar_arrive_tx(fb, (uint32_t)(nv * 128 * 16 * p.mt));
+                    for (int hh = 0; hh < p.mt; ++hh)
+                        for (int j = 0; j < nv; ++j)
+                            tma_load_im2col_4d(aT + hh * 16384 + j * 2048, &tmA, fb, 0, hh ? ic_w[1] : ic_w[0],
+                                               hh ? ic_h[1] : ic_h[0], hh ? ic_n[1] : ic_n[0],
+                                               (uint16_t)(s0 + j), (uint16_t)r);
+                } else if ((A_TMA || B_TMA) && t == 0) {
                     mbar_arrive_tx(fb, (uint32_t)p.tma_bytes);
-                    if constexpr (AM == A_TMA_K2) tma_load_2d(aT, &tmA, fb, kb * KB, m0);
-                    if constexpr (AM == A_TMA_K3) tma_load_3d(aT, &tmA, fb, kb * KB, m0, z);
-                    if constexpr (AM == A_TMA_MN2) {
+                    // A: p.mt blocks of 128 rows (16 KB each)
+                    for (int hh = 0; hh < p.mt; ++hh) {
+                        const uint32_t aH = aT + hh * 16384;
+                        const int mH = m0 + 128 * hh;
+                        if constexpr (AM == A_TMA_K2) tma_load_2d(aH, &tmA, fb, kb * KB, mH);
+                        if constexpr (AM == A_TMA_K3) tma_load_3d(aH, &tmA, fb, kb * KB, mH, z);
+                        if constexpr (AM == A_TMA_MN2) {
 #pragma unroll
-                        for (int a = 0; a < 128 * ELT / 128; ++a)
-                            tma_load_2d(aT + a * KB * 128, &tmA, fb, m0 + a * (128 / ELT), kb * KB);
+                            for (int a = 0; a < 128 * ELT / 128; ++a)
+                                tma_load_2d(aH + a * KB * 128, &tmA, fb, mH + a * (128 / ELT), kb * KB);
+                        }
+                        if constexpr (AM == A_TMA_IM2COL) {
+                            // 128 consecutive output pixels x KB channels of tap (r,s) in one TMA
+                            const uint16_t ow = (uint16_t)(p.im2col_dgrad ? p.tapS - 1 - g_s : g_s);
+                            const uint16_t oh = (uint16_t)(p.im2col_dgrad ? p.tapR - 1 - g_r : g_r);
+                            tma_load_im2col_4d(aH, &tmA, fb, g_c0, hh ? ic_w[1] : ic_w[0], hh ? ic_h[1] : ic_h[0],
+                                               hh ? ic_n[1] : ic_n[0], ow, oh);
+                        }
                     }
                     if constexpr (BM_ == B_TMA_K2) tma_load_2d(bT, &tmB, fb, kb * KB, n0);
                     if constexpr (BM_ == B_TMA_K3) tma_load_3d(bT, &tmB, fb, kb * KB, n0, z);
@@ -265,12 +306,6 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                         const int rs = dgrad_tap_rs(p, tap);
                         for (int a = 0; a < p.bn_atoms; ++a)
                             tma_load_3d(bT + a * KB * 128, &tmB, fb, n0 + a * (128 / ELT), rs, k0);
-                    }
-                    if constexpr (AM == A_TMA_IM2COL) {
-                        // 128 consecutive output pixels x KB channels of tap (r,s) in one TMA
-                        const uint16_t ow = (uint16_t)(p.im2col_dgrad ? p.tapS - 1 - g_s : g_s);
-                        const uint16_t oh = (uint16_t)(p.im2col_dgrad ? p.tapR - 1 - g_r : g_r);
-                        tma_load_im2col_4d(aT, &tmA, fb, g_c0, ic_w, ic_h, ic_n, ow, oh);
                     }
                     if constexpr (BM_ == B_TMA_IM2COL) {
                         // atom a = 128 B of channels (c0..) of tap (r,s) for KB pixels
@@ -326,6 +361,20 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                             const T* src = v ? gx + rbase[i] + ((long long)pp * p.Q + qq) * p.K + kc : gx;
                             cp_async16(aT + soff + i * 2048, src, v);
                         }
+                    }
+                }
+                if (AM == A_GATHER_SMALLC_PAD && !(p.debug & 2)) {  // debug bit 1: skip the A gather
+                    // k-block = filter row r, taps s0..s0+7; chunk j = tap s0 + j = one
+                    // 16-B padded pixel of the channel-padded x (async, lagged arrive).
+                    const int groups = p.s8 / 8;
+                    const int r = kb / groups, sx = (kb - r * groups) * 8 + (t & 7);
+                    const uint32_t soff = kmaj_off(t / 8, (t & 7) * 16);
+                    const long long koff = ((long long)r * p.W + sx) * p.cp;
+#pragma unroll
+                    for (int i = 0; i < 8; ++i) {
+                        const bool v = sx < p.S && rv[i] && (unsigned)(rh[i] + r) < (unsigned)p.H &&
+                                       (unsigned)(rw[i] + sx) < (unsigned)p.W;
+                        cp_async16(aT + soff + i * 2048, v ? gx + rbase[i] + koff : gx, v);
                     }
                 }
                 if constexpr (AM == A_GATHER_SMALLC) {
@@ -406,6 +455,27 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                             cp_async16(bT + (uint32_t)(a * KB * 128) + mn_row_off<ELT>(row, chunk * 16), src, v);
                         }
                     }
+                } else if constexpr (BM_ == B_GATHER_SMALLC_PAD) {
+                    // WGRAD small C from padded x: atom = tap group (r, s0..s0+7),
+                    // chunk = tap, one 16-B cp.async per (pixel row, tap).
+                    const int chunk = t & 7;
+                    const int groups = p.s8 / 8;
+                    const int pq = p.P * p.Q;
+                    for (int i = 0; i < KB / 16; ++i) {
+                        const int row = t / 8 + 16 * i;
+                        const int m = kb * KB + row;
+                        const bool mv = m < p.kred;
+                        const int mm = mv ? m : 0;
+                        const int n = mm / pq, rem = mm - n * pq, pp = rem / p.Q, qq = rem - pp * p.Q;
+                        for (int a = 0; a < p.bn_atoms; ++a) {
+                            const int grp = (n0 * ELT) / 128 + a;
+                            const int r = grp / groups, sx = (grp - r * groups) * 8 + chunk;
+                            const int h = pp * p.stride - p.pad + r, w = qq * p.stride - p.pad + sx;
+                            const bool v = mv && r < p.R && sx < p.S && h >= 0 && h < p.H && w >= 0 && w < p.W;
+                            const T* src = v ? gx + (((size_t)n * p.H + h) * p.W + w) * p.cp : gx;
+                            cp_async16(bT + (uint32_t)(a * KB * 128) + mn_row_off<ELT>(row, chunk * 16), src, v);
+                        }
+                    }
                 } else if constexpr (BM_ == B_GATHER_SMALLC) {
                     // WGRAD small C: B(j' = (r, s8, c'), m) MN-major; an atom (128 B)
                     // is one tap group (r, s0..s0+7), chunk = tap, 16 B = padded pixel.
@@ -474,7 +544,10 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                         if (git >= lag) {
                             if (lag == 1) cp_async_wait<1>();
                             else if (lag == 2) cp_async_wait<2>();
-                            else cp_async_wait<3>();
+                            else if (lag == 3) cp_async_wait<3>();
+                            else if (lag == 4) cp_async_wait<4>();
+                            else if (lag == 5) cp_async_wait<5>();
+                            else cp_async_wait<6>();
                             fence_proxy_async();
                             mbar_arrive(smem_u32(&full[s - lag < 0 ? s - lag + S : s - lag]));
                         }
@@ -509,7 +582,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
             decode(tile, m0, n0, z, kb_begin, kb_end);
             mbar_wait(smem_u32(&tempty[acc]), aph ^ 1u);  // epilogue has drained this accumulator
             tc_fence_after();
-            const uint32_t dtm = tmem + (uint32_t)(acc * p.BN);
+            const uint32_t dtm = tmem + (uint32_t)(acc * p.mt * p.BN);
             for (int kb = kb_begin; kb < kb_end; ++kb, s = (s + 1 == S) ? 0 : s + 1, ph ^= (s == 0) ? 1u : 0u) {
                 mbar_wait(smem_u32(&full[s]), ph);
                 tc_fence_after();
@@ -517,14 +590,30 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                     const uint32_t aT = smem_u32(sA + (size_t)s * A_BYTES);
                     const uint32_t bT = B_RES ? smem_u32(sBres) + (uint32_t)(kb * p.BN * 128)
                                               : smem_u32(sB + (size_t)s * B_BYTES);
+                    // p.mt independent accumulators (one per 128-row half) share B and
+                    // interleave, so short-N MMAs are not serialised on one accumulator.
+                    // (Both variants fully unrolled: the issue thread must not stall.)
+                    auto issue = [&](auto mt_c) {
+                        constexpr int MT = decltype(mt_c)::value;
 #pragma unroll
-                    for (int j = 0; j < KB / UMMA_K; ++j) {
-                        const uint64_t ad = A_MN ? sdesc(aT + j * UMMA_K * 128, KB * 128, MN_SBO, MN_LAYOUT)
-                                                 : sdesc(aT + j * 32, 16, 1024);
-                        const uint64_t bd = B_MN ? sdesc(bT + j * UMMA_K * 128, KB * 128, MN_SBO, MN_LAYOUT)
-                                                 : sdesc(bT + j * 32, 16, 1024);
-                        mma<ELT>(dtm, ad, bd, idesc, (kb > kb_begin || j > 0) ? 1u : 0u);
-                    }
+                        for (int j = 0; j < KB / UMMA_K; ++j) {
+                            const uint64_t bd = B_MN ? sdesc(bT + j * UMMA_K * 128, KB * 128, MN_SBO, MN_LAYOUT)
+                                                     : sdesc(bT + j * 32, 16, 1024);
+#pragma unroll
+                            for (int hh = 0; hh < MT; ++hh) {
+                                const uint32_t aH = aT + hh * 16384;
+                                // no-swizzle A: core matrices 8 rows x 16 B, SBO 128 B (rows),
+                                // LBO 2 KB (next tap); one MMA covers 32 B of K = 2 taps
+                                const uint64_t ad = A_NOSWZ ? sdesc(aH + j * 4096, 2048, 128, 0)
+                                                  : A_MN ? sdesc(aH + j * UMMA_K * 128, KB * 128, MN_SBO, MN_LAYOUT)
+                                                         : sdesc(aH + j * 32, 16, 1024);
+                                mma<ELT>(dtm + (uint32_t)(hh * p.BN), ad, bd, idesc,
+                                         (kb > kb_begin || j > 0) ? 1u : 0u);
+                            }
+                        }
+                    };
+                    if (p.mt == 2) issue(std::integral_constant<int, 2>{});
+                    else issue(std::integral_constant<int, 1>{});
                     mma_commit(smem_u32(&empty[s]));
                 }
                 __syncwarp();
@@ -549,7 +638,8 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
             const bool has_acc = kb_end > kb_begin;
             mbar_wait(smem_u32(&tfull[acc]), aph);
             tc_fence_after();
-            const int m = m0 + row;
+            auto drain = [&](const int hh) {
+            const int m = m0 + 128 * hh + row;
             // Output row of GEMM row m (phase mode scatters sub-grid rows back to dx).
             long long mrow = m;
             if (p.ph_mode && m < p.M) {
@@ -557,7 +647,8 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                 const int n = m / hw, rem = m - n * hw, ii = rem / p.ph_W, jj = rem - ii * p.ph_W;
                 mrow = ((long long)n * p.H + p.ph_hb + p.stride * ii) * p.W + p.ph_wb + p.stride * jj;
             }
-            const uint32_t taddr_row = tmem + (uint32_t)(acc * p.BN) + ((uint32_t)(q4 * 32) << 16);
+            const uint32_t taddr_row =
+                tmem + (uint32_t)((acc * p.mt + hh) * p.BN) + ((uint32_t)(q4 * 32) << 16);
             float* outF = (float*)p.out;
             T* outT = (T*)p.out;
             if (EPI == EPI_STORE && z > 0) {
@@ -573,7 +664,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
 #pragma unroll
                     for (int j = 0; j < 32; ++j) v[j] = 0u;
                 }
-                if (m >= p.M) continue;
+                if (m >= p.M || (p.debug & 1)) continue;  // debug bit 0: skip stores (timing experiments)
                 const int nb = n0 + c0;
                 if constexpr (EPI == EPI_WGRAD_SMALLC) {
                     // padded column j' = (r, s8, c') -> dw column (r*S + s)*C + c (skip padding)
@@ -646,6 +737,9 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                     }
                 }
             }
+            };  // drain one 128-row half
+            drain(0);
+            if (p.mt == 2) drain(1);
             // release this accumulator to the MMA warp
             tc_fence_before();
             __syncwarp();

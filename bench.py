@@ -6,7 +6,8 @@ algorithm at the same workspace (BASELINE.json metric), on B200.
                     [--policy pow2|all|undivided] [--ws-mib 64] [--wd-mib T] [--batch 256]
 
 Default (N=1): BASELINE.json configs[1] -- AlexNet's 5 conv layers, forward +
-backward (15 kernels), N=256 per GPU, fp32 storage with TF32 tensor cores,
+backward (14 kernels: the first layer's BackwardData is skipped as in Caffe,
+P:L198 reading G19; --input-grad adds it), N=256 per GPU, fp32 storage with TF32 tensor cores,
 WR policy with a 64 MiB per-kernel workspace limit, `powerOfTwo` batch policy.
 A step = one pass of the whole hot path: for every kernel the planned
 sequence of micro-batches through the C ABI.  Synthetic seeded NHWC data.
@@ -46,6 +47,9 @@ def parse():
     ap.add_argument("--ws-mib", type=float, default=64.0, help="WR per-kernel workspace limit (MiB)")
     ap.add_argument("--wd-mib", type=float, default=0.0, help="use WD with this total workspace (MiB)")
     ap.add_argument("--batch", type=int, default=256, help="mini-batch per GPU")
+    ap.add_argument("--input-grad", action="store_true",
+                    help="also time the first layer's BackwardData (the data layer needs no gradient; "
+                         "the paper's Caffe iterations skip it, P:L198)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-sample", type=int, default=0, help="oracle sample (images per kernel); 0 = auto")
     ap.add_argument("--json-out", default="")
@@ -113,9 +117,10 @@ class ClockSampler:
 
 
 # --------------------------------------------------------------- oracle arm --
-def oracle_sample_time(layers, n_sample, threads=None):
+def oracle_sample_time(layers, n_sample, threads=None, input_grad=False):
     """Time the fp64 oracle (oracle/, unchanged) on n_sample images of every
-    kernel of the iteration; returns seconds."""
+    kernel of the iteration (the first layer's BackwardData only if
+    input_grad); returns seconds."""
     import oracle
     from synthetic import conv_inputs
     if threads:
@@ -127,25 +132,30 @@ def oracle_sample_time(layers, n_sample, threads=None):
         x, w, dy = x.astype(np.float64), w.astype(np.float64), dy.astype(np.float64)
         t0 = time.perf_counter()
         oracle.conv_forward(x, w, l.pad, l.stride)
-        oracle.conv_backward_data(dy, w, l.h, l.w, l.pad, l.stride)
+        if i > 0 or input_grad:
+            oracle.conv_backward_data(dy, w, l.h, l.w, l.pad, l.stride)
         oracle.conv_backward_filter(x, dy, l.r, l.s, l.pad, l.stride)
         tot += time.perf_counter() - t0
     return tot
 
 
-def cpu_baseline(layers, batch, n_sample):
+def n_kernels(layers, input_grad):
+    return 3 * len(layers) - (0 if input_grad else 1)
+
+
+def cpu_baseline(layers, batch, n_sample, input_grad=False):
     cores = os.cpu_count()
-    secs = oracle_sample_time(layers, n_sample)
+    secs = oracle_sample_time(layers, n_sample, input_grad=input_grad)
     ms_per_iter = secs * 1e3 * batch / n_sample
     return {"value": round(ms_per_iter, 3), "unit": "ms/iter", "cores": cores, "kind": "oracle",
-            "sample": f"{n_sample} image(s) per kernel, all {3 * len(layers)} kernels, fp64 7-loop oracle, "
+            "sample": f"{n_sample} image(s) per kernel, all {n_kernels(layers, input_grad)} timed kernels, fp64 7-loop oracle, "
                       f"{secs:.2f} s measured, x{batch // n_sample} extrapolated to N={batch} (work is linear in N, P:L50)"}
 
 
-def auto_sample(layers, batch):
+def auto_sample(layers, batch, input_grad=False):
     """Pick the oracle sample so one measurement takes ~10-20 s on this host
     (one probe image through every kernel, then scale)."""
-    per_img = oracle_sample_time(layers, 1)
+    per_img = oracle_sample_time(layers, 1, input_grad=input_grad)
     n = int(max(1, min(batch, 12.0 / max(per_img, 1e-6))))
     while batch % n:
         n -= 1
@@ -158,18 +168,19 @@ def run_reference(args):
         return
     from synthetic import network
     layers = network(args.config)
-    n_sample = args.cpu_sample or auto_sample(layers, args.batch)
+    n_sample = args.cpu_sample or auto_sample(layers, args.batch, args.input_grad)
     for _ in range(args.warmup):
         pass  # the oracle has no warm-up state; W is accepted for the contract
-    times = [oracle_sample_time(layers, n_sample) for _ in range(args.steps)]
+    times = [oracle_sample_time(layers, n_sample, input_grad=args.input_grad) for _ in range(args.steps)]
     ms = float(np.mean(times)) * 1e3 * args.batch / n_sample
     cb = {"value": round(ms, 3), "unit": "ms/iter", "cores": os.cpu_count(), "kind": "oracle",
           "sample": f"{n_sample} image(s) per kernel per step, x{args.batch // n_sample} extrapolated to N={args.batch}"}
     line = {"impl": "reference", "metric": METRIC, "value": round(ms, 3), "unit": "ms/iter", "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms, 3), "higher_is_better": False,
             "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-            "config": {"workload": f"{args.config} conv fwd+bwd (15 kernels)" if args.config == "alexnet" else
-                       f"{args.config} conv fwd+bwd", "batch_per_gpu": args.batch, "math": "fp64 oracle"},
+            "config": {"workload": f"{args.config} conv layers fwd+bwd ({n_kernels(layers, args.input_grad)} kernels)",
+                       "batch_per_gpu": args.batch, "math": "fp64 oracle",
+                       "first_layer_backward_data": bool(args.input_grad)},
             "cpu_baseline": cb,
             "e2e": {"value": round(ms, 3), "unit": "ms/iter", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
@@ -220,7 +231,7 @@ def main():
     def timed(nsteps, nwarm, record_ops=False, e2e=None):
         ops = {}
         for _ in range(nwarm):
-            net.iteration(grad_hook=grad_ar)
+            net.iteration(grad_hook=grad_ar, skip_conv1_dgrad=not args.input_grad)
             grad_ar.wait()
         torch.cuda.synchronize()
         if distributed:
@@ -242,7 +253,7 @@ def main():
             s0.record(stream)
             if e2e is not None:
                 e2e["h2d"]()
-            net.iteration(on_op=on_op, grad_hook=grad_ar)
+            net.iteration(on_op=on_op, grad_hook=grad_ar, skip_conv1_dgrad=not args.input_grad)
             grad_ar.wait()
             if e2e is not None:
                 e2e["d2h"]()
@@ -332,23 +343,24 @@ def main():
         except Exception:
             traffic = None
 
-    conv_flops = net.flops_per_iteration()
+    conv_flops = net.flops_per_iteration(skip_conv1_dgrad=not args.input_grad)
     total_ws = net.total_workspace()
     if rank == 0:
         cb = None
         if not args.no_cpu_baseline and world == 1:
-            n_sample = args.cpu_sample or auto_sample(layers, args.batch)
-            cb = cpu_baseline(layers, args.batch, n_sample)
+            n_sample = args.cpu_sample or auto_sample(layers, args.batch, args.input_grad)
+            cb = cpu_baseline(layers, args.batch, n_sample, args.input_grad)
         line = {
             "metric": METRIC, "value": round(ms_max, 4), "unit": "ms/iter", "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": round(ms_max, 4), "higher_is_better": False,
             "scaling": "weak", "vs_baseline": None, "dtype": args.math, "data": "synthetic",
-            "config": {"workload": f"{args.config} conv layers fwd+bwd ({3 * len(layers)} kernels)",
+            "config": {"workload": f"{args.config} conv layers fwd+bwd ({n_kernels(layers, args.input_grad)} kernels)",
                        "batch_per_gpu": args.batch, "global_batch": args.batch * world,
                        "policy": ("WD" if args.wd_mib > 0 else "WR"),
                        "ws_limit_mib": (args.wd_mib if args.wd_mib > 0 else args.ws_mib),
                        "batch_size_policy": args.policy, "parallelism": f"dp{world}",
-                       "l2": "512 MiB buffer overwritten before every timed step"},
+                       "l2": "512 MiB buffer overwritten before every timed step",
+                       "first_layer_backward_data": bool(args.input_grad)},
             "images_per_s": round(args.batch * world / (ms_max * 1e-3), 1),
             "conv_tflops_direct": round(conv_flops / (ms_max * 1e-3) / 1e12, 2),
             "undivided_ms_per_step": round(results["undivided"], 4) if "undivided" in results else None,

@@ -124,6 +124,8 @@ mucu_status_t mucu_output_dims(const mucu_conv_desc_t* desc, int32_t* p, int32_t
  *   IG  (all types):  0
  *   I2C FWD/WGRAD:    b*P*Q*ceil_e(R*S*C)*elt  (+ K*ceil_e(R*S*C)*elt when R*S*C*elt % 16 != 0)
  *                     0 for 1x1, stride 1, pad 0 (the im2col matrix is x itself)
+ *                     b*H*W*16 for TF32/BF16 with C*elt < 16 (RGB input layer): x with
+ *                     channels zero-padded to 16 B, gathered tap by tap on chip
  *   I2C DGRAD:        b*P*Q*ceil_4(R*S*C)*4 (fp32 dcol)  (+ filter copy as above); 0 for 1x1/s1/p0
  *   WG  FWD:          16*K*C*elt + 16*b*T*C*elt + 16*b*T*K*4,   T = ceil(P/2)*ceil(Q/2)
  *   WG  DGRAD:        16*C*K*elt + 16*b*T'*K*elt + 16*b*T'*C*4, T' = ceil(H/2)*ceil(W/2)

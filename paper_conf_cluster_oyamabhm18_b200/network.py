@@ -213,8 +213,9 @@ class ConvNet:
             if t == L.BWD_FILTER and grad_hook is not None:
                 grad_hook(i, self.tensors[i]["dw"])
 
-    def flops_per_iteration(self) -> int:
-        return sum(layer_flops(l, self.n) for l in self.layers) * 3
+    def flops_per_iteration(self, skip_conv1_dgrad: bool = False) -> int:
+        f = sum(layer_flops(l, self.n) for l in self.layers) * 3
+        return f - (layer_flops(self.layers[0], self.n) if skip_conv1_dgrad else 0)
 
     def summary(self):
         rows = []

@@ -85,8 +85,15 @@ def test_workspace_bf16_resnet_and_pointwise():
 
 
 def test_workspace_unaligned_filter_row():
-    d = mu.desc(4, 3, 224, 224, 64, 7, 7, 3, 2, mu.MATH_BF16)              # RSC = 147
-    kp = 152                                                               # ceil to 8 bf16
-    col = 112 * 112 * kp * 2
-    filt = -(-64 * kp * 2 // 256) * 256
+    d = mu.desc(4, 3, 224, 224, 64, 7, 7, 3, 2, mu.MATH_F32)               # RSC = 147
+    kp = 148                                                               # ceil to 4 floats
+    col = 112 * 112 * kp * 4
+    filt = -(-64 * kp * 4 // 256) * 256
     assert mu.workspace_size(d, mu.FWD, mu.IM2COL_GEMM, 1) == filt + -(-col // 256) * 256
+
+
+def test_workspace_small_c_tensor_core():
+    # C*elt < 16 B on tensor cores: I2C FWD/WGRAD keep x with channels padded to 16 B
+    d = mu.desc(4, 3, 224, 224, 64, 7, 7, 3, 2, mu.MATH_BF16)
+    assert mu.workspace_size(d, mu.FWD, mu.IM2COL_GEMM, 2) == 2 * 224 * 224 * 16
+    assert mu.workspace_size(d, mu.BWD_FILTER, mu.IM2COL_GEMM, 1) == 224 * 224 * 16

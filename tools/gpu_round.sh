@@ -1,0 +1,57 @@
+#!/bin/bash
+# Round measurement on a B200 box (run via gpurun from the repo root):
+#   tests, smoke, benches, the ncu launch list of the default bench step and a
+#   full-set capture of its dominant kernel.  Every step has its own timeout.
+# usage: tools/gpu_round.sh TAG [steps...]   steps: tests smoke bench others launches full
+set -u
+TAG=${1:-r01}; shift
+STEPS=${*:-"tests smoke bench others launches full"}
+OUT=gpurun_out/$TAG
+mkdir -p $OUT
+nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm,temperature.gpu --format=csv > $OUT/gpu.txt 2>&1
+has() { [[ " $STEPS " == *" $1 "* ]]; }
+
+if has tests; then
+  timeout -s KILL 1500 python -m pytest tests -q -m gpu -x > $OUT/tests.log 2>&1; echo "tests rc=$?" | tee -a $OUT/status
+  tail -3 $OUT/tests.log
+fi
+if has smoke; then
+  timeout -s KILL 300 python -c "import __graft_entry__ as g; g.build(); g.smoke(); print('smoke ok')" > $OUT/smoke.log 2>&1
+  echo "smoke rc=$?" | tee -a $OUT/status
+fi
+if has bench; then
+  timeout -s KILL 900 python bench.py --tables-out $OUT/tables_alexnet_tf32.npz --json-out $OUT/bench_alexnet_tf32.json \
+    > $OUT/bench_alexnet_tf32.log 2>&1; echo "bench rc=$?" | tee -a $OUT/status
+  tail -c 600 $OUT/bench_alexnet_tf32.log
+fi
+if has others; then
+  for cfg in "resnet50 bf16" "resnet18 bf16" "alexnet bf16"; do
+    set -- $cfg
+    timeout -s KILL 900 python bench.py --config $1 --math $2 --no-cpu-baseline --tables-out $OUT/tables_$1_$2.npz \
+      --json-out $OUT/bench_$1_$2.json > $OUT/bench_$1_$2.log 2>&1; echo "bench $1 $2 rc=$?" | tee -a $OUT/status
+  done
+  timeout -s KILL 900 python bench.py --wd-mib 120 --steps 5 --no-cpu-baseline --json-out $OUT/bench_alexnet_tf32_wd120.json \
+    > $OUT/bench_wd.log 2>&1; echo "bench wd rc=$?" | tee -a $OUT/status
+fi
+TAB=$OUT/tables_alexnet_tf32.npz
+if has launches; then
+  MUCU_PROFILE=1 timeout -s KILL 900 ncu --metrics gpu__time_duration.sum --clock-control none --profile-from-start off \
+    --csv --log-file $OUT/launches_alexnet_tf32.csv python bench.py --steps 2 --warmup 3 --no-cpu-baseline \
+    --tables-in $TAB > $OUT/launches.log 2>&1; echo "launches rc=$?" | tee -a $OUT/status
+fi
+if has full; then
+  CMD=$(python - $OUT/bench_alexnet_tf32.json <<'PY'
+import json, sys, re
+d = json.load(open(sys.argv[1]))
+k = d["roofline"]["kernel"]
+layer, typ = k.split()[0], k.split()[1]
+algo, b = re.findall(r"\('(\w+)', (\d+)\)", k)[0]
+t = {"FWD": "FWD", "BWD_DATA": "DGRAD", "BWD_FILTER": "WGRAD", "DGRAD": "DGRAD", "WGRAD": "WGRAD"}[typ]
+print(f"--layer {layer} --type {t} --algo {algo} --b {b}")
+PY
+)
+  echo "dominant: $CMD" | tee -a $OUT/status
+  timeout -s KILL 900 ncu --set full --clock-control none --import-source on --profile-from-start off \
+    -o $OUT/dominant_full -f python tools/profile_one.py --config alexnet --math tf32 $CMD > $OUT/full.log 2>&1
+  echo "full rc=$?" | tee -a $OUT/status
+fi

@@ -6,8 +6,8 @@ algorithm at the same workspace (BASELINE.json metric), on B200.
                     [--policy pow2|all|undivided] [--ws-mib 64] [--wd-mib T] [--batch 256]
 
 Default (N=1): BASELINE.json configs[1] -- AlexNet's 5 conv layers, forward +
-backward (14 kernels: the first layer's BackwardData is skipped as in Caffe,
-P:L198 reading G19; --input-grad adds it), N=256 per GPU, fp32 storage with TF32 tensor cores,
+backward (15 kernels; --no-input-grad drops the first layer's BackwardData as
+Caffe's `time` command does), N=256 per GPU, fp32 storage with TF32 tensor cores,
 WR policy with a 64 MiB per-kernel workspace limit, `powerOfTwo` batch policy.
 A step = one pass of the whole hot path: for every kernel the planned
 sequence of micro-batches through the C ABI.  Synthetic seeded NHWC data.
@@ -47,9 +47,9 @@ def parse():
     ap.add_argument("--ws-mib", type=float, default=64.0, help="WR per-kernel workspace limit (MiB)")
     ap.add_argument("--wd-mib", type=float, default=0.0, help="use WD with this total workspace (MiB)")
     ap.add_argument("--batch", type=int, default=256, help="mini-batch per GPU")
-    ap.add_argument("--input-grad", action="store_true",
-                    help="also time the first layer's BackwardData (the data layer needs no gradient; "
-                         "the paper's Caffe iterations skip it, P:L198)")
+    ap.add_argument("--no-input-grad", dest="input_grad", action="store_false",
+                    help="skip the first layer's BackwardData (the data layer needs no gradient, as in "
+                         "Caffe's `time` command, P:L198); the default times all 3 kernels per layer (SURVEY 8(d) cfg2)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-sample", type=int, default=0, help="oracle sample (images per kernel); 0 = auto")
     ap.add_argument("--json-out", default="")
@@ -117,7 +117,7 @@ class ClockSampler:
 
 
 # --------------------------------------------------------------- oracle arm --
-def oracle_sample_time(layers, n_sample, threads=None, input_grad=False):
+def oracle_sample_time(layers, n_sample, threads=None, input_grad=True):
     """Time the fp64 oracle (oracle/, unchanged) on n_sample images of every
     kernel of the iteration (the first layer's BackwardData only if
     input_grad); returns seconds."""
@@ -143,7 +143,7 @@ def n_kernels(layers, input_grad):
     return 3 * len(layers) - (0 if input_grad else 1)
 
 
-def cpu_baseline(layers, batch, n_sample, input_grad=False):
+def cpu_baseline(layers, batch, n_sample, input_grad=True):
     cores = os.cpu_count()
     secs = oracle_sample_time(layers, n_sample, input_grad=input_grad)
     ms_per_iter = secs * 1e3 * batch / n_sample
@@ -152,7 +152,7 @@ def cpu_baseline(layers, batch, n_sample, input_grad=False):
                       f"{secs:.2f} s measured, x{batch // n_sample} extrapolated to N={batch} (work is linear in N, P:L50)"}
 
 
-def auto_sample(layers, batch, input_grad=False):
+def auto_sample(layers, batch, input_grad=True):
     """Pick the oracle sample so one measurement takes ~10-20 s on this host
     (one probe image through every kernel, then scale)."""
     per_img = oracle_sample_time(layers, 1, input_grad=input_grad)

@@ -39,69 +39,6 @@ int grid_for(int64_t work, int threads) {
     return (int)blocks;
 }
 
-// ---------------------------------------------------------------- im2col --
-// col[m][kk] = x[n, p*st + r - pad, q*st + s - pad, c] (0 outside / kk >= RSC),
-// m = (n,p,q), kk = (r,s,c).  Vector version: V = 16/sizeof(T) channels per
-// thread (requires C % V == 0, so a chunk never straddles (r,s)).
-template <class T, int V>
-__global__ void im2col_kernel(const T* __restrict__ x, T* __restrict__ col, int64_t rows, int H, int W,
-                              int C, int P, int Q, int S, int pad, int st, int RSC, int kpitch) {
-    const int64_t chunks_per_row = kpitch / V;
-    const int64_t total = rows * chunks_per_row;
-    for (int64_t idx = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; idx < total;
-         idx += (int64_t)gridDim.x * blockDim.x) {
-        int64_t m = idx / chunks_per_row;
-        int kk = (int)(idx - m * chunks_per_row) * V;
-        T* dst = col + m * kpitch + kk;
-        int pq = P * Q;
-        int n = (int)(m / pq);
-        int rem = (int)(m - (int64_t)n * pq);
-        int p = rem / Q, q = rem - (rem / Q) * Q;
-        bool ok = kk < RSC;
-        int h = 0, w = 0, c = 0;
-        if (ok) {
-            int rs = kk / C;
-            c = kk - rs * C;
-            int r = rs / S, s = rs - (rs / S) * S;
-            h = p * st + r - pad;
-            w = q * st + s - pad;
-            ok = (h >= 0 && h < H && w >= 0 && w < W);
-        }
-        if constexpr (V > 1) {
-            uint4 v = make_uint4(0, 0, 0, 0);
-            if (ok) v = *reinterpret_cast<const uint4*>(x + (((int64_t)n * H + h) * W + w) * C + c);
-            *reinterpret_cast<uint4*>(dst) = v;
-        } else {
-            *dst = ok ? x[(((int64_t)n * H + h) * W + w) * C + c] : from_f<T>(0.f);
-        }
-    }
-}
-
-// Scalar fallback when C is not a multiple of the vector width: one element
-// per thread, kk = (r,s,c) decomposed individually.
-template <class T>
-__global__ void im2col_scalar_kernel(const T* __restrict__ x, T* __restrict__ col, int64_t rows, int H, int W,
-                                     int C, int P, int Q, int S, int pad, int st, int RSC, int kpitch) {
-    const int64_t total = rows * kpitch;
-    for (int64_t idx = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; idx < total;
-         idx += (int64_t)gridDim.x * blockDim.x) {
-        int64_t m = idx / kpitch;
-        int kk = (int)(idx - m * kpitch);
-        float v = 0.f;
-        if (kk < RSC) {
-            int pq = P * Q;
-            int n = (int)(m / pq);
-            int rem = (int)(m - (int64_t)n * pq);
-            int p = rem / Q, q = rem % Q;
-            int rs = kk / C, c = kk % C;
-            int r = rs / S, s = rs % S;
-            int h = p * st + r - pad, w = q * st + s - pad;
-            if (h >= 0 && h < H && w >= 0 && w < W) v = to_f<T>(x[(((int64_t)n * H + h) * W + w) * C + c]);
-        }
-        col[idx] = from_f<T>(v);
-    }
-}
-
 template <class T>
 __global__ void pad_filter_kernel(const T* __restrict__ w, T* __restrict__ wp, int K, int RSC, int kpitch) {
     const int64_t total = (int64_t)K * kpitch;
@@ -109,42 +46,6 @@ __global__ void pad_filter_kernel(const T* __restrict__ w, T* __restrict__ wp, i
          idx += (int64_t)gridDim.x * blockDim.x) {
         int k = (int)(idx / kpitch), kk = (int)(idx % kpitch);
         wp[idx] = kk < RSC ? w[(int64_t)k * RSC + kk] : from_f<T>(0.f);
-    }
-}
-
-// ---------------------------------------------------------------- col2im --
-// dx[n,h,w,c] = alpha * sum_{r,s: st | h+pad-r, ...} dcol[(n,p,q)][(r*S+s)*C + c] + beta * dx
-// (the adjoint of im2col; gather form, so every dx element is written once in
-// a fixed summation order -- deterministic, no atomics).
-template <class T>
-__global__ void col2im_kernel(const float* __restrict__ dcol, T* __restrict__ dx, int64_t total, int H, int W,
-                              int C, int P, int Q, int R, int S, int pad, int st, int kpitch, float alpha,
-                              float beta) {
-    for (int64_t idx = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; idx < total;
-         idx += (int64_t)gridDim.x * blockDim.x) {
-        int c = (int)(idx % C);
-        int64_t pix = idx / C;
-        int w = (int)(pix % W);
-        int64_t t2 = pix / W;
-        int h = (int)(t2 % H);
-        int n = (int)(t2 / H);
-        float acc = 0.f;
-        for (int r = 0; r < R; ++r) {
-            int ph = h + pad - r;
-            if (ph < 0 || ph % st) continue;
-            int p = ph / st;
-            if (p >= P) continue;
-            for (int s = 0; s < S; ++s) {
-                int pw = w + pad - s;
-                if (pw < 0 || pw % st) continue;
-                int q = pw / st;
-                if (q >= Q) continue;
-                acc += dcol[(((int64_t)n * P + p) * Q + q) * kpitch + (r * S + s) * C + c];
-            }
-        }
-        float out = alpha * acc;
-        if (beta != 0.f) out += beta * to_f<T>(dx[idx]);
-        dx[idx] = from_f<T>(out);
     }
 }
 

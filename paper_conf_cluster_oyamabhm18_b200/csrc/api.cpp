@@ -56,6 +56,17 @@ bool is_pointwise(const Geom& g) { return g.r == 1 && g.s == 1 && g.pad == 0 && 
 
 bool small_c_tc(const Geom& g) { return g.math != MUCU_MATH_F32 && g.c * elt_size(g.math) < 16; }
 
+int s2d_channels(const Geom& g) {
+    const int atom = 128 / elt_size(g.math);
+    return (int)align_up((uint64_t)g.stride * g.stride * g.c, (uint64_t)atom);
+}
+
+bool s2d_tc(const Geom& g, int type) {
+    if (!small_c_tc(g) || g.stride < 2) return false;
+    if (type == MUCU_BWD_DATA) return g.k % (128 / elt_size(g.math)) == 0 && g.stride * g.stride * g.c <= 256;
+    return s2d_channels(g) <= 2 * g.stride * g.stride * g.c;
+}
+
 bool algo_eligible(const Geom& g, int type, int algo) {
     if (type < MUCU_FWD || type > MUCU_BWD_FILTER) return false;
     switch (algo) {
@@ -83,6 +94,22 @@ mucu_status_t ws_layout(const Geom& g, int type, int algo, int32_t b, WsLayout* 
     if (algo == MUCU_ALGO_IM2COL_GEMM) {
         L->kpitch = (int32_t)align_up(RSC, vec);
         if (is_pointwise(g)) { L->kpitch = g.c; return MUCU_OK; }
+        if (s2d_tc(g, type)) {
+            // Space-to-depth: FWD = [s2d filter K x Dr*Ds*Cs][xs b x I x J x Cs],
+            // WGRAD = [xs], DGRAD = [s2d filter st*st*C x Dr*Ds*K] (b-independent).
+            const uint64_t Dr = s2d_taps(g.r, g.stride), Ds = s2d_taps(g.s, g.stride);
+            const uint64_t Cs = (uint64_t)s2d_channels(g);
+            if (type == MUCU_BWD_DATA) {
+                L->fixed_bytes = align_up((uint64_t)g.stride * g.stride * g.c * Dr * Ds * g.k * elt, 256);
+            } else {
+                if (type == MUCU_FWD) L->fixed_bytes = align_up((uint64_t)g.k * Dr * Ds * Cs * elt, 256);
+                L->a_off = L->fixed_bytes;
+                L->a_bytes = align_up((uint64_t)b * (g.p + Dr - 1) * (g.q + Ds - 1) * Cs * elt, 256);
+            }
+            L->kpitch = (int32_t)Cs;
+            L->total = L->fixed_bytes + L->a_bytes;
+            return MUCU_OK;
+        }
         if (small_c_tc(g) && type != MUCU_BWD_DATA) {
             // Tensor-core small-C (RGB) layers: the explicit transform is a
             // channel pad of x to 16 B per pixel (the GEMM walks the taps);
@@ -94,8 +121,11 @@ mucu_status_t ws_layout(const Geom& g, int type, int algo, int32_t b, WsLayout* 
             return MUCU_OK;
         }
         if (type == MUCU_BWD_DATA) {
-            L->filter_padded = (RSC * elt) % 16 != 0;
-            const uint64_t fpitch = align_up(RSC, vec);
+            // tensor cores read the filter as MN-major 128-B atoms: rows shorter
+            // than one atom are padded to it
+            const bool short_row = g.math != MUCU_MATH_F32 && RSC < 128 / elt;
+            L->filter_padded = (RSC * elt) % 16 != 0 || short_row;
+            const uint64_t fpitch = short_row ? 128 / elt : align_up(RSC, vec);
             L->fixed_bytes = L->filter_padded ? align_up((uint64_t)g.k * fpitch * elt, 256) : 0;
             L->kpitch = (int32_t)align_up(RSC, 4);  // fp32 dcol
             L->a_off = L->fixed_bytes;

@@ -352,6 +352,75 @@ __global__ void col2im_taps_kernel(const float* __restrict__ dcol, T* __restrict
     }
 }
 
+
+// ---------------------------------------------------------- space-to-depth --
+// Strided RGB-like layers run on the stride x stride super-pixel image
+// (DESIGN.md "space-to-depth"): a stride-st RxS conv on C channels equals a
+// stride-1 ceil(R/st) x ceil(S/st) conv on st*st*C channels.
+// xs[n][i][j][(a*st + b)*C + c] = x[n][st*i + a - pad][st*j + b - pad][c]
+// (0 off the image and in the channel padding c' >= st*st*C).  One thread per
+// 16-B chunk of xs, so every store is a full vector.
+template <class T>
+__global__ void s2d_input_kernel(const T* __restrict__ x, T* __restrict__ xs, int64_t chunks, int H, int W, int C,
+                                 int I, int J, int st, int pad, int Cs) {
+    constexpr int V = 16 / sizeof(T);
+    const int cpp = Cs / V, stc = st * C, real = st * stc;
+    for (int64_t idx = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; idx < chunks;
+         idx += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t pix = idx / cpp;
+        const int c0 = (int)(idx - pix * cpp) * V;
+        const int j = (int)(pix % J);
+        const int64_t t = pix / J;
+        const int i = (int)(t % I), n = (int)(t / I);
+        const int h0 = st * i - pad, w0 = st * j - pad;
+        int a = c0 / stc, b = (c0 - a * stc) / C, c = c0 - a * stc - b * C;
+        __align__(16) T vals[V];
+#pragma unroll
+        for (int u = 0; u < V; ++u) {
+            const int h = h0 + a, w = w0 + b;
+            vals[u] = (c0 + u < real && (unsigned)h < (unsigned)H && (unsigned)w < (unsigned)W)
+                          ? x[(((int64_t)n * H + h) * W + w) * C + c]
+                          : from_f<T>(0.f);
+            if (++c == C) { c = 0; if (++b == st) { b = 0; ++a; } }
+        }
+        *reinterpret_cast<uint4*>(xs + idx * V) = *reinterpret_cast<const uint4*>(vals);
+    }
+}
+
+// Space-to-depth filter.  FWD (K-major B of the stride-1 conv on xs):
+//   out[k][(d*Ds + e)*Cs + (a*st + b)*C + c] = w[k][st*d + a][st*e + b][c]
+// DGRAD (K-major B of the transposed conv, N = st*st*C columns of dx):
+//   out[(a*st + b)*C + c][(d*Ds + e)*K + k] = w[k][st*d + a][st*e + b][c]
+// Zero where st*d + a >= R, st*e + b >= S, or in the channel padding.
+template <class T>
+__global__ void s2d_filter_kernel(const T* __restrict__ w, T* __restrict__ out, int64_t total, int K, int R, int S,
+                                  int C, int st, int Dr, int Ds, int Cs, bool dgrad) {
+    const int stc = st * C, real = st * stc;
+    for (int64_t idx = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; idx < total;
+         idx += (int64_t)gridDim.x * blockDim.x) {
+        int k, tap, ch;
+        if (!dgrad) {
+            const int row = Dr * Ds * Cs;
+            k = (int)(idx / row);
+            const int rem = (int)(idx - (int64_t)k * row);
+            tap = rem / Cs; ch = rem - tap * Cs;
+        } else {
+            const int row = Dr * Ds * K;
+            ch = (int)(idx / row);
+            const int rem = (int)(idx - (int64_t)ch * row);
+            tap = rem / K; k = rem - tap * K;
+        }
+        T v = from_f<T>(0.f);
+        if (ch < real) {
+            const int d = tap / Ds, e = tap - d * Ds;
+            const int a = ch / stc, b = (ch - a * stc) / C, c = ch - a * stc - b * C;
+            const int r = st * d + a, s = st * e + b;
+            if (r < R && s < S) v = w[(((int64_t)k * R + r) * S + s) * C + c];
+        }
+        out[idx] = v;
+    }
+}
+
 }  // namespace
 
 int launch_im2col(const Geom& g, int32_t b, const void* x, void* col, int32_t kpitch, cudaStream_t st) {
@@ -482,6 +551,34 @@ int launch_wg_output(const Geom& g, bool dgrad, int32_t b, float alpha, const fl
         wg_output_kernel<__nv_bfloat16><<<grid, 256, 0, st>>>(M, (__nv_bfloat16*)out, tiles, OH, OW, O, TH, TW, alpha, beta);
     else
         wg_output_kernel<float><<<grid, 256, 0, st>>>(M, (float*)out, tiles, OH, OW, O, TH, TW, alpha, beta);
+    count_launch();
+    return (int)cudaGetLastError();
+}
+
+int launch_s2d_input(const Geom& g, int32_t b, int I, int J, int Cs, const void* x, void* xs, cudaStream_t st) {
+    const int V = 16 / elt_size(g.math);
+    const int64_t chunks = (int64_t)b * I * J * (Cs / V);
+    const int grid = grid_for(chunks, 256);
+    if (g.math == MUCU_MATH_BF16)
+        s2d_input_kernel<__nv_bfloat16><<<grid, 256, 0, st>>>((const __nv_bfloat16*)x, (__nv_bfloat16*)xs, chunks, g.h,
+                                                              g.w, g.c, I, J, g.stride, g.pad, Cs);
+    else
+        s2d_input_kernel<float><<<grid, 256, 0, st>>>((const float*)x, (float*)xs, chunks, g.h, g.w, g.c, I, J,
+                                                      g.stride, g.pad, Cs);
+    count_launch();
+    return (int)cudaGetLastError();
+}
+
+int launch_s2d_filter(const Geom& g, bool dgrad, int Cs, const void* w, void* out, cudaStream_t st) {
+    const int Dr = (g.r + g.stride - 1) / g.stride, Ds = (g.s + g.stride - 1) / g.stride;
+    const int64_t total = dgrad ? (int64_t)g.stride * g.stride * g.c * Dr * Ds * g.k : (int64_t)g.k * Dr * Ds * Cs;
+    const int grid = grid_for(total, 256);
+    if (g.math == MUCU_MATH_BF16)
+        s2d_filter_kernel<__nv_bfloat16><<<grid, 256, 0, st>>>((const __nv_bfloat16*)w, (__nv_bfloat16*)out, total,
+                                                               g.k, g.r, g.s, g.c, g.stride, Dr, Ds, Cs, dgrad);
+    else
+        s2d_filter_kernel<float><<<grid, 256, 0, st>>>((const float*)w, (float*)out, total, g.k, g.r, g.s, g.c,
+                                                       g.stride, Dr, Ds, Cs, dgrad);
     count_launch();
     return (int)cudaGetLastError();
 }

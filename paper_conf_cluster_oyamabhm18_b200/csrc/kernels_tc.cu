@@ -159,7 +159,11 @@ enum BMode : int {
     B_GATHER_SMALLC = 10, // WGRAD small C: x pixels as 16-B tap chunks, MN-major
     B_GATHER_SMALLC_PAD = 11, // WGRAD small C from the channel-padded copy of x: cp.async
 };
-enum EpiMode : int { EPI_STORE = 0, EPI_WGRAD_CHAIN = 1, EPI_WGRAD_SMALLC = 2 };
+// EPI_D2S: DGRAD on the space-to-depth grid -- row (n, i, j), column
+//   (a, b, c) -> dx[n][st*i + a - pad][st*j + b - pad][c] (out-of-image skipped).
+// EPI_WGRAD_S2D: column (d, e, (a, b, c')) of the space-to-depth filter ->
+//   dw[k][st*d + a][st*e + b][c'] (padding and r >= R / s >= S skipped), reduced.
+enum EpiMode : int { EPI_STORE = 0, EPI_WGRAD_CHAIN = 1, EPI_WGRAD_SMALLC = 2, EPI_D2S = 3, EPI_WGRAD_S2D = 4 };
 
 struct TcArgs {
     int M, N;                // output rows / cols
@@ -195,6 +199,9 @@ struct TcArgs {
     int max_lag;             // cp.async stages kept in flight per producer thread (<= 6)
     int debug;               // MUCU_TC_DEBUG bits (timing experiments only): 1 skip stores, 2 skip A gather
     int mt;                  // 128-row halves per tile (1, or 2 for 256-row tiles with narrow N)
+    // Space-to-depth layers (EPI_D2S / EPI_WGRAD_S2D): the real stride, C, R, S
+    // (the GEMM itself runs on the stride-1 super-pixel geometry).
+    int s2_st, s2_C, s2_R, s2_S;
     // epilogue
     void* out;
     long long ldc;
@@ -510,6 +517,77 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         }
         return err;
     }
+    if (algo == MUCU_ALGO_IM2COL_GEMM && s2d_tc(g, type)) {
+        // Space-to-depth: the strided small-C layer as a stride-1
+        // Dr x Ds conv over the st x st super-pixel image with Cs channels --
+        // 128-B channel atoms, so TMA im2col feeds it like any other layer.
+        const int st_ = g.stride, Dr = s2d_taps(g.r, st_), Ds = s2d_taps(g.s, st_);
+        const int Cs = s2d_channels(g);
+        const int kind = type == MUCU_BWD_DATA ? 4 : 3;
+        if (type != MUCU_BWD_FILTER && (ctx->fixed_kind != kind || ctx->fixed_src != in1)) {
+            err = launch_s2d_filter(g, type == MUCU_BWD_DATA, Cs, in1, ws, st);
+            if (err) return err;
+            ctx->fixed_kind = kind; ctx->fixed_src = in1;
+        }
+        A.s2_st = st_; A.s2_C = g.c; A.s2_R = g.r; A.s2_S = g.s;
+        if (type == MUCU_BWD_DATA) {
+            // dx in super-pixels: i = (h + pad) / st, a = (h + pad) % st; dy row
+            // p = i - d pairs with filter row r = st*d + a (d < Dr).
+            const int I = (g.h - 1 + g.pad) / st_ + 1, J = (g.w - 1 + g.pad) / st_ + 1;
+            const int Kp = Dr * Ds * g.k;
+            A.M = b * I * J; A.N = st_ * st_ * g.c; A.num_kb = Kp / KB; A.kred = Kp;
+            A.ph_mode = 1; A.ph_H = I; A.ph_W = J; A.ph_i0 = 0; A.ph_j0 = 0;
+            A.tapR = Dr; A.tapS = Ds; A.im2col_dgrad = 1; A.gsrc = in0;
+            finalize_tiling(L, elt);
+            use_mt2(L, num_sms);
+            grid2(1);
+            const int lw = -(Ds - 1), lh = -(Dr - 1);
+            if (!make_im2col_map(&L.ta, elt, in0, g.k, g.q, g.p, b, lw, lh, lw + J - g.q, lh + I - g.p, 128, 1,
+                                 false))
+                return -1;
+            if (!map2(&L.tb, ws, Kp, A.N, Kp, KB, A.BN)) return -1;
+            A.tma_bytes = 16384 * A.mt + A.BN * 128;
+            return LAUNCH(A_TMA_IM2COL, B_TMA_K2, EPI_D2S);
+        }
+        const int I = g.p + Dr - 1, J = g.q + Ds - 1;
+        char* xs = ws + WL.a_off;
+        err = launch_s2d_input(g, b, I, J, Cs, in0, xs, st);
+        if (err) return err;
+        // the GEMM sees the stride-1, pad-0 geometry over xs
+        A.H = I; A.W = J; A.C = Cs; A.R = Dr; A.S = Ds; A.pad = 0; A.stride = 1; A.tapR = Dr; A.tapS = Ds;
+        if (type == MUCU_FWD) {
+            const int Kp = Dr * Ds * Cs;
+            A.M = (int)(b * PQ); A.N = g.k; A.ldc = g.k; A.num_kb = Kp / KB; A.kred = Kp; A.gsrc = xs;
+            finalize_tiling(L, elt);
+            use_mt2(L, num_sms);
+            grid2(1);
+            if (!make_im2col_map(&L.ta, elt, xs, Cs, J, I, b, 0, 0, -(Ds - 1), -(Dr - 1), 128, 1, false)) return -1;
+            if (!map2(&L.tb, ws, Kp, g.k, Kp, KB, A.BN)) return -1;
+            A.tma_bytes = 16384 * A.mt + A.BN * 128;
+            return LAUNCH(A_TMA_IM2COL, B_TMA_K2, EPI_STORE);
+        }
+        // WGRAD: dw'[k][(d, e, c')] = sum_m dy[m][k] xs(m; d, e, c'), folded into
+        // dw[k][st*d + a][st*e + b][c] by the epilogue's reductions.
+        const int64_t Mpix = (int64_t)b * PQ;
+        A.M = g.k; A.N = Dr * Ds * Cs; A.ldc = RSC; A.kred = (int)Mpix; A.gsrc = xs;
+        finalize_tiling(L, elt, atom);
+        const int64_t tiles = ceil_div(A.N, A.BN) * ceil_div(A.M, 128);
+        const int64_t nkb = ceil_div(Mpix, KB);
+        int64_t nsplit = std::min<int64_t>(std::min<int64_t>(std::max<int64_t>(1, (2LL * num_sms) / tiles),
+                                                             std::max<int64_t>(1, nkb / 16)), 65535);
+        A.kb_per_split = (int)ceil_div(nkb, nsplit);
+        nsplit = ceil_div(nkb, A.kb_per_split);
+        A.num_kb = (int)nkb;
+        grid2((int)nsplit);
+        if (beta != 1.f) {
+            err = launch_scale(g.k * RSC, beta, (float*)out, st);
+            if (err) return err;
+        }
+        if (!map2(&L.ta, in1, g.k, (uint64_t)Mpix, g.k, atom, KB, true)) return -1;
+        if (!make_im2col_map(&L.tb, elt, xs, Cs, J, I, b, 0, 0, -(Ds - 1), -(Dr - 1), KB, 1, true)) return -1;
+        A.tma_bytes = 128 * KB * elt + A.bn_atoms * KB * 128;
+        return LAUNCH(A_TMA_MN2, B_TMA_IM2COL, EPI_WGRAD_S2D);
+    }
     if (type == MUCU_FWD && algo == MUCU_ALGO_IM2COL_GEMM && small_c_tc(g)) {
         // RGB-like layer: x -> channel-padded copy (16 B / pixel) in the workspace,
         // then the tap-walking GEMM with async 16-B gathers and the staged filter.
@@ -663,13 +741,14 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         const void* wp = in1;
         int64_t wpitch = RSC;
         if (!pw && WL.filter_padded) {
+            // same pitch as ws_layout: one 128-B atom for short rows, else 16 B
+            const int fpitch = RSC < atom ? atom : (int)align_up((uint64_t)RSC, (uint64_t)(16 / elt));
             if (ctx->fixed_kind != 1 || ctx->fixed_src != in1) {
-                const int fpitch = (int)align_up((uint64_t)RSC, (uint64_t)(16 / elt));
                 err = launch_pad_filter(g, in1, ws, fpitch, st);
                 if (err) return err;
                 ctx->fixed_kind = 1; ctx->fixed_src = in1;
             }
-            wp = ws; wpitch = (int64_t)align_up((uint64_t)RSC, (uint64_t)(16 / elt));
+            wp = ws; wpitch = fpitch;
         }
         A.M = (int)(b * PQ); A.N = (int)RSC; A.num_kb = (int)ceil_div(g.k, KB);
         if (pw) { A.ldc = g.c; }
@@ -677,9 +756,9 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         finalize_tiling(L, elt);
         use_mt2(L, num_sms);
         grid2(1);
-        if (RSC < atom) return -1;
+        if (wpitch < atom) return -1;  // pointwise with C < one atom
         if (!map2(&L.ta, in0, g.k, (uint64_t)A.M, g.k, KB, 128)) return -1;
-        if (!map2(&L.tb, wp, RSC, g.k, wpitch, atom, KB, true)) return -1;
+        if (!map2(&L.tb, wp, std::max<int64_t>(RSC, atom), g.k, wpitch, atom, KB, true)) return -1;
         A.tma_bytes = 16384 * A.mt + A.bn_atoms * KB * 128;
         err = LAUNCH(A_TMA_K2, B_TMA_MN2, EPI_STORE);
         if (err || pw) return err;

@@ -35,6 +35,14 @@ inline int64_t ceil_div(int64_t a, int64_t b) { return (a + b - 1) / b; }
 bool algo_eligible(const Geom& g, int type, int algo);
 bool is_pointwise(const Geom& g);  // 1x1, stride 1, pad 0: im2col(x) == x
 bool small_c_tc(const Geom& g);    // tensor-core math and C*elt < 16 B (RGB input layer)
+// Strided small-C layers whose I2C algorithm runs on the space-to-depth image:
+// a stride-1 ceil(R/st) x ceil(S/st) conv over st*st*C channels (padded to
+// s2d_channels = a multiple of 128 B).  FWD/WGRAD need the padding to at most
+// double the channels; DGRAD (no padding: the super-pixel channels are GEMM
+// columns) needs K to be a multiple of 128 B / elt.
+bool s2d_tc(const Geom& g, int type);
+int s2d_channels(const Geom& g);
+inline int s2d_taps(int r, int stride) { return (r + stride - 1) / stride; }
 
 // Workspace layout of one micro-configuration (all offsets 256-B aligned).
 // `fixed` = b-independent prefix (padded filter / Winograd U) computed once per
@@ -92,6 +100,9 @@ int launch_wg_filter(const Geom& g, bool dgrad, const void* w, void* U, cudaStre
 int launch_scale(int64_t n, float beta, float* p, cudaStream_t st);  // p *= beta (beta == 0: p = 0)
 // x[b,H,W,C] -> xp[b,H,W,16/elt] with channels zero-padded to 16 B per pixel.
 int launch_pad_channels(const Geom& g, int32_t b, const void* x, void* xp, cudaStream_t st);
+// Space-to-depth image xs[b][I][J][Cs] and filters (kernels_elem.cu).
+int launch_s2d_input(const Geom& g, int32_t b, int I, int J, int Cs, const void* x, void* xs, cudaStream_t st);
+int launch_s2d_filter(const Geom& g, bool dgrad, int Cs, const void* w, void* out, cudaStream_t st);
 int launch_wg_input(const Geom& g, bool dgrad, int32_t b, const void* in, void* V, cudaStream_t st);
 int launch_wg_output(const Geom& g, bool dgrad, int32_t b, float alpha, const float* M, float beta,
                      void* out, cudaStream_t st);

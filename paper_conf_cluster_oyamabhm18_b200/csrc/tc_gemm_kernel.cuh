@@ -30,7 +30,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                             BM_ == B_TMA_IM2COL);
     constexpr bool B_RES = (BM_ == B_RESIDENT);
     constexpr bool GATHER = !A_TMA || (!B_TMA && !B_RES);
-    constexpr bool SPLITK = (EPI == EPI_WGRAD_CHAIN || EPI == EPI_WGRAD_SMALLC);
+    constexpr bool SPLITK = (EPI == EPI_WGRAD_CHAIN || EPI == EPI_WGRAD_SMALLC || EPI == EPI_WGRAD_S2D);
     constexpr bool A_ASYNC = (AM == A_GATHER_FWD || AM == A_GATHER_DGRAD || AM == A_GATHER_SMALLC_PAD);
     constexpr bool B_ASYNC = (BM_ == B_GATHER_WG || BM_ == B_GATHER_SMALLC_PAD);
     // MN-major atoms: 8-row (bf16, SWIZZLE_128B) or 4-row (tf32, 128B_BASE32B) groups.
@@ -642,7 +642,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
             const int m = m0 + 128 * hh + row;
             // Output row of GEMM row m (phase mode scatters sub-grid rows back to dx).
             long long mrow = m;
-            if (p.ph_mode && m < p.M) {
+            if (EPI == EPI_STORE && p.ph_mode && m < p.M) {
                 const int hw = p.ph_H * p.ph_W;
                 const int n = m / hw, rem = m - n * hw, ii = rem / p.ph_W, jj = rem - ii * p.ph_W;
                 mrow = ((long long)n * p.H + p.ph_hb + p.stride * ii) * p.W + p.ph_wb + p.stride * jj;
@@ -666,7 +666,49 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                 }
                 if (m >= p.M || (p.debug & 1)) continue;  // debug bit 0: skip stores (timing experiments)
                 const int nb = n0 + c0;
-                if constexpr (EPI == EPI_WGRAD_SMALLC) {
+                if constexpr (EPI == EPI_D2S) {
+                    // super-pixel row (n, i, jj); column (a, b, c) walked incrementally
+                    const int hw = p.ph_H * p.ph_W;
+                    const int n = m / hw, rem = m - n * hw, ii = rem / p.ph_W, jj = rem - ii * p.ph_W;
+                    const int h0 = p.s2_st * ii - p.pad, w0 = p.s2_st * jj - p.pad;
+                    const long long nbase = (long long)n * p.H;
+                    const int stc = p.s2_st * p.C;
+                    int a = nb / stc, bq = (nb - a * stc) / p.C, c = nb - a * stc - bq * p.C;
+#pragma unroll
+                    for (int j = 0; j < 32; ++j) {
+                        const int h = h0 + a, w = w0 + bq;
+                        if (nb + j < p.N && (unsigned)h < (unsigned)p.H && (unsigned)w < (unsigned)p.W) {
+                            const long long off = ((nbase + h) * p.W + w) * p.C + c;
+                            float o = p.alpha * __uint_as_float(v[j]);
+                            if (p.out_bf16) {
+                                __nv_bfloat16* d = (__nv_bfloat16*)p.out + off;
+                                if (p.beta != 0.f) o += p.beta * __bfloat162float(*d);
+                                *d = __float2bfloat16_rn(o);
+                            } else {
+                                float* d = (float*)p.out + off;
+                                if (p.beta != 0.f) o += p.beta * *d;
+                                *d = o;
+                            }
+                        }
+                        if (++c == p.C) { c = 0; if (++bq == p.s2_st) { bq = 0; ++a; } }
+                    }
+                } else if constexpr (EPI == EPI_WGRAD_S2D) {
+                    // column (tap (d,e), channel (a, b, c)) -> dw[k][st*d+a][st*e+b][c]
+                    float* drow = outF + (size_t)m * p.ldc;
+                    const int stc = p.s2_st * p.s2_C, real = stc * p.s2_st;
+                    int tap = nb / p.C, ch = nb - tap * p.C;
+#pragma unroll
+                    for (int j = 0; j < 32; ++j) {
+                        if (nb + j < p.N && ch < real) {
+                            const int d = tap / p.S, e = tap - d * p.S;
+                            const int a = ch / stc, rem = ch - a * stc, bq = rem / p.s2_C, c = rem - bq * p.s2_C;
+                            const int r = p.s2_st * d + a, sx = p.s2_st * e + bq;
+                            if (r < p.s2_R && sx < p.s2_S)
+                                atomicAdd(drow + (r * p.s2_S + sx) * p.s2_C + c, p.alpha * __uint_as_float(v[j]));
+                        }
+                        if (++ch == p.C) { ch = 0; ++tap; }
+                    }
+                } else if constexpr (EPI == EPI_WGRAD_SMALLC) {
                     // padded column j' = (r, s8, c') -> dw column (r*S + s)*C + c (skip padding)
                     float* drow = outF + (size_t)m * p.ldc;
 #pragma unroll

@@ -97,3 +97,18 @@ def test_workspace_small_c_tensor_core():
     d = mu.desc(4, 3, 224, 224, 64, 7, 7, 3, 2, mu.MATH_BF16)
     assert mu.workspace_size(d, mu.FWD, mu.IM2COL_GEMM, 2) == 2 * 224 * 224 * 16
     assert mu.workspace_size(d, mu.BWD_FILTER, mu.IM2COL_GEMM, 1) == 224 * 224 * 16
+
+
+def test_workspace_space_to_depth():
+    # AlexNet conv1 on tensor cores: Dr = Ds = ceil(11/4) = 3, Cs = 4*4*3 = 48 -> 64 (TF32 atom 32)
+    d = mu.desc(4, 3, 224, 224, 64, 11, 11, 2, 4, mu.MATH_TF32)
+    a256 = lambda v: -(-v // 256) * 256  # noqa: E731
+    xs = 57 * 57 * 64 * 4                  # (P + Dr - 1) x (Q + Ds - 1) super-pixels per sample
+    assert mu.workspace_size(d, mu.FWD, mu.IM2COL_GEMM, 2) == a256(64 * 9 * 64 * 4) + a256(2 * xs)
+    assert mu.workspace_size(d, mu.BWD_FILTER, mu.IM2COL_GEMM, 3) == a256(3 * xs)
+    assert mu.workspace_size(d, mu.BWD_DATA, mu.IM2COL_GEMM, 4) == a256(48 * 9 * 64 * 4)
+    # ResNet conv1 BF16: Cs = 12 -> 64 would more than double the channels, so FWD keeps the
+    # channel-padded image, while DGRAD (no channel padding) uses the st*st*C x Dr*Ds*K filter
+    d = mu.desc(2, 3, 224, 224, 64, 7, 7, 3, 2, mu.MATH_BF16)
+    assert mu.workspace_size(d, mu.FWD, mu.IM2COL_GEMM, 2) == 2 * 224 * 224 * 16
+    assert mu.workspace_size(d, mu.BWD_DATA, mu.IM2COL_GEMM, 2) == a256(12 * 16 * 64 * 2)

@@ -32,6 +32,9 @@ SHAPES = {
     "5x5s1": (2, 64, 11, 11, 48, 5, 5, 2, 1),          # AlexNet conv2 geometry
     "11x11s4_c3": (2, 3, 35, 35, 64, 11, 11, 2, 4),    # AlexNet conv1 geometry
     "7x7s2_c3": (2, 3, 23, 23, 64, 7, 7, 3, 2),        # ResNet conv1 geometry
+    "11x11s4_c3_ragged": (2, 3, 30, 27, 64, 11, 11, 2, 4),  # space-to-depth with ragged super-pixel edges
+    "5x5s2_c2_k32": (2, 2, 17, 19, 32, 5, 5, 2, 2),
+    "4x4s3_c3_p0": (3, 3, 20, 22, 64, 4, 4, 0, 3),
     "3x3s2": (2, 64, 14, 14, 128, 3, 3, 1, 2),
     "1x1s1": (3, 64, 10, 10, 96, 1, 1, 0, 1),
     "1x1s2": (2, 64, 14, 14, 128, 1, 1, 0, 2),

@@ -51,7 +51,9 @@ print(f"--layer {layer} --type {t} --algo {algo} --b {b}")
 PY
 )
   echo "dominant: $CMD" | tee -a $OUT/status
+  # one launch of the GEMM kernel only (a full-set report of every micro-batch is tens of MB)
   timeout -s KILL 900 ncu --set full --clock-control none --import-source on --profile-from-start off \
-    -o $OUT/dominant_full -f python tools/profile_one.py --config alexnet --math tf32 $CMD > $OUT/full.log 2>&1
+    -k regex:tc_conv_gemm -c 1 -o $OUT/dominant_full -f python tools/profile_one.py --config alexnet --math tf32 $CMD \
+    > $OUT/full.log 2>&1
   echo "full rc=$?" | tee -a $OUT/status
 fi

@@ -173,6 +173,8 @@ struct TcArgs {
     int BN;                  // tile N (multiple of 16, <= 256)
     int stages;
     int tmem_cols;
+    int nacc;                // TMEM accumulators (2 = epilogue overlaps the next tile; 1 when mt*BN > 256)
+    int km;                  // k-blocks per stage (MN-major BackwardFilter operands; 1 elsewhere)
     int bn_atoms;            // MN-major B atoms per stage = BN * ELT / 128
     int tma_bytes;           // bytes the TMA loads of one stage deliver
     int b_bytes;             // shared-memory bytes of one B stage
@@ -197,7 +199,8 @@ struct TcArgs {
     int cp, s8;
     int bres_bytes;          // B_RESIDENT: smem bytes of the staged filter
     int max_lag;             // cp.async stages kept in flight per producer thread (<= 6)
-    int debug;               // MUCU_TC_DEBUG bits (timing experiments only): 1 skip stores, 2 skip A gather
+    int debug;               // MUCU_TC_DEBUG bits (timing experiments only): 1 skip stores, 2 skip A gather,
+                             // 4 skip TMA loads, 8 skip MMAs
     int mt;                  // 128-row halves per tile (1, or 2 for 256-row tiles with narrow N)
     // Space-to-depth layers (EPI_D2S / EPI_WGRAD_S2D): the real stride, C, R, S
     // (the GEMM itself runs on the stride-1 super-pixel geometry).
@@ -364,12 +367,13 @@ bool use_tma_im2col() {
 
 // Tile N: a multiple of `step` (16 = UMMA granularity at M = 128; an MN-major
 // atom when a tile must not split a 128-B channel atom) up to 256, minimising
-// the padded columns plus a per-tile overhead (~32 columns); ties -> larger.
-int pick_bn(int N, int step = 32) {
+// the padded columns plus a per-tile overhead (~32 columns, or the A rows a
+// tile re-reads); ties -> larger.
+int pick_bn(int N, int step = 32, int overhead = 32, int max_bn = 256) {
     step = std::max(step, 32);  // the epilogue drains TMEM in 32-column chunks
     int best = step, best_cost = 1 << 30;
-    for (int bn = step; bn <= 256; bn += step) {
-        const int cost = (int)ceil_div(N, bn) * (bn + 32);
+    for (int bn = step; bn <= max_bn; bn += step) {
+        const int cost = (int)ceil_div(N, bn) * (bn + overhead);
         if (cost <= best_cost) { best = bn; best_cost = cost; }
     }
     return best;
@@ -384,7 +388,7 @@ struct Launch {
 template <int ELT, int AM, int BM_, int EPI>
 int launch_t(Launch& L, cudaStream_t st) {
     auto kern = tc_conv_gemm<ELT, AM, BM_, EPI>;
-    const int smem = 1024 + L.a.stages * (L.a.mt * 128 * 128 + L.a.b_bytes) + L.a.bres_bytes +
+    const int smem = 1024 + L.a.stages * L.a.km * (L.a.mt * 128 * 128 + L.a.b_bytes) + L.a.bres_bytes +
                      (2 * L.a.stages + 5) * 8 + 64;
     static int configured = 0;  // per instantiation
     if (configured < smem) {
@@ -398,9 +402,11 @@ int launch_t(Launch& L, cudaStream_t st) {
 }
 
 void size_stages(TcArgs& a) {
-    const int cols = 2 * a.mt * a.BN;  // 2 accumulators x mt halves
+    a.nacc = a.mt * a.BN <= 256 ? 2 : 1;
+    const int cols = a.nacc * a.mt * a.BN;  // accumulators x mt halves
     a.tmem_cols = cols <= 64 ? 64 : cols <= 128 ? 128 : cols <= 256 ? 256 : 512;
-    const int stage_bytes = a.mt * 128 * 128 + a.b_bytes;
+    if (a.km < 1) a.km = 1;
+    const int stage_bytes = a.km * (a.mt * 128 * 128 + a.b_bytes);
     a.stages = std::min(env_int("MUCU_MAX_STAGES", 8), (200 * 1024) / stage_bytes);
     if (a.stages < 2) a.stages = 2;
 }
@@ -444,6 +450,7 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
     Launch L;
     std::memset(&L, 0, sizeof(L));
     TcArgs& A = L.a;
+    A.km = 1;
     A.H = g.h; A.W = g.w; A.C = g.c; A.P = g.p; A.Q = g.q; A.R = g.r; A.S = g.s; A.pad = g.pad;
     A.stride = g.stride; A.K = g.k;
     A.tapR = g.r; A.tapS = g.s;
@@ -467,6 +474,37 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         A.num_z = batch;
         const int64_t tiles = ceil_div(A.M, 128 * A.mt) * ceil_div(A.N, A.BN) * batch;
         L.grid = dim3((unsigned)std::max<int64_t>(1, std::min<int64_t>(tiles, num_sms)));
+    };
+    // BackwardFilter tiling: output rows = K (filter count), columns = the
+    // filter taps, reduction = pixels split across CTAs (~2 waves, >= 16
+    // k-blocks each).  TMA-fed B operands take 256-row tiles when they cover
+    // K without waste, so each B tile is read once per 256 output rows.
+    // TMA-only operands (tma = true) also take 256-row tiles and stages of
+    // km k-blocks: fewer, larger TMA transactions (the TMA issue rate, not
+    // bytes, bounds these MN-major loads), as deep as two stages allow.
+    auto wgrad_tiling = [&](int step, bool tma) {
+        A.mt = (tma && A.M > 128 && (A.M <= 256 || A.M % 256 == 0) && env_int("MUCU_MT2", 1)) ? 2 : 1;
+        // 256-row tiles keep BN <= 128 so that two stages of two k-blocks fit
+        // (measured: km = 2 beats BN = 256 with km = 1 on every AlexNet/ResNet layer)
+        A.BN = pick_bn(A.N, step, 128 * A.mt, A.mt == 2 ? std::max(128, step) : 256);
+        if (const int fb = env_int("MUCU_FORCE_BN", 0)) A.BN = std::max(std::max(step, 32), fb - fb % step);
+        A.bn_atoms = (A.BN * elt + 127) / 128;
+        A.b_bytes = std::max(A.BN * 128, A.bn_atoms * (128 / elt) * 128);
+        A.km = 1;
+        if (tma) {
+            const int base = A.mt * 128 * 128 + A.b_bytes;
+            while (A.km < 4 && 2 * (2 * A.km) * base <= 200 * 1024 && KB * 2 * A.km <= 256) A.km *= 2;
+            if (const int km = env_int("MUCU_KM", 0)) A.km = km;
+        }
+        size_stages(A);
+        const int64_t tiles = ceil_div(A.N, A.BN) * ceil_div(A.M, 128 * A.mt);
+        const int64_t nkb = ceil_div(A.kred, KB * A.km);
+        int64_t nsplit = std::min<int64_t>(std::min<int64_t>(std::max<int64_t>(1, (2LL * num_sms) / tiles),
+                                                             std::max<int64_t>(1, nkb / 16)), 65535);
+        A.kb_per_split = (int)ceil_div(nkb, nsplit);
+        nsplit = ceil_div(nkb, A.kb_per_split);
+        A.num_kb = (int)nkb;
+        grid2((int)nsplit);
     };
     const bool Aok = (g.c % KB) == 0;  // vector gathers over C
     int err = 0;
@@ -570,22 +608,15 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         // dw[k][st*d + a][st*e + b][c] by the epilogue's reductions.
         const int64_t Mpix = (int64_t)b * PQ;
         A.M = g.k; A.N = Dr * Ds * Cs; A.ldc = RSC; A.kred = (int)Mpix; A.gsrc = xs;
-        finalize_tiling(L, elt, atom);
-        const int64_t tiles = ceil_div(A.N, A.BN) * ceil_div(A.M, 128);
-        const int64_t nkb = ceil_div(Mpix, KB);
-        int64_t nsplit = std::min<int64_t>(std::min<int64_t>(std::max<int64_t>(1, (2LL * num_sms) / tiles),
-                                                             std::max<int64_t>(1, nkb / 16)), 65535);
-        A.kb_per_split = (int)ceil_div(nkb, nsplit);
-        nsplit = ceil_div(nkb, A.kb_per_split);
-        A.num_kb = (int)nkb;
-        grid2((int)nsplit);
+        wgrad_tiling(atom, true);
         if (beta != 1.f) {
             err = launch_scale(g.k * RSC, beta, (float*)out, st);
             if (err) return err;
         }
-        if (!map2(&L.ta, in1, g.k, (uint64_t)Mpix, g.k, atom, KB, true)) return -1;
-        if (!make_im2col_map(&L.tb, elt, xs, Cs, J, I, b, 0, 0, -(Ds - 1), -(Dr - 1), KB, 1, true)) return -1;
-        A.tma_bytes = 128 * KB * elt + A.bn_atoms * KB * 128;
+        if (!map2(&L.ta, in1, g.k, (uint64_t)Mpix, g.k, atom, KB * A.km, true)) return -1;
+        if (!make_im2col_map(&L.tb, elt, xs, Cs, J, I, b, 0, 0, -(Ds - 1), -(Dr - 1), KB * A.km, 1, true))
+            return -1;
+        A.tma_bytes = A.km * (A.mt * 128 * KB * elt + A.bn_atoms * KB * 128);
         return LAUNCH(A_TMA_MN2, B_TMA_IM2COL, EPI_WGRAD_S2D);
     }
     if (type == MUCU_FWD && algo == MUCU_ALGO_IM2COL_GEMM && small_c_tc(g)) {
@@ -768,28 +799,14 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         // dw[k][(r,s,c)] = sum_m dy[m][k] B(m, (r,s,c)); A = dy MN-major via TMA.
         const int64_t Mpix = (int64_t)b * PQ;
         A.M = g.k; A.N = (int)RSC; A.ldc = RSC; A.kred = (int)Mpix; A.gsrc = in0;
-        // implicit-im2col B producers load whole 128-B channel atoms of one tap:
-        // N tiles must start on an atom boundary.
-        finalize_tiling(L, elt, (algo == MUCU_ALGO_IMPLICIT_GEMM && g.c % atom == 0) ? atom : 16);
-        const int64_t tiles = ceil_div(A.N, A.BN) * ceil_div(A.M, 128);
-        const int64_t nkb = ceil_div(Mpix, KB);
-        // Split the pixel reduction so that ~2 waves of CTAs run, each split
-        // >= 16 k-blocks (amortises TMEM alloc / pipeline fill).
-        // splits x tiles <= 2 waves of persistent CTAs (no ragged third round)
-        int64_t want = std::max<int64_t>(1, (2LL * num_sms) / tiles);
-        int64_t nsplit = std::min<int64_t>(std::min<int64_t>(want, std::max<int64_t>(1, nkb / 16)), 65535);
         // P:L58 output scale: apply the user's beta once, then every split adds.
         if (beta != 1.f) {
             err = launch_scale(g.k * RSC, beta, (float*)out, st);
             if (err) return err;
         }
         (void)sem;
-        A.kb_per_split = (int)ceil_div(nkb, nsplit);
-        nsplit = ceil_div(nkb, A.kb_per_split);
-        A.num_kb = (int)nkb;
-        grid2((int)nsplit);
-        if (!map2(&L.ta, in1, g.k, (uint64_t)Mpix, g.k, atom, KB, true)) return -1;
         const int a_bytes = 128 * KB * elt;
+        auto map_dy = [&]() { return map2(&L.ta, in1, g.k, (uint64_t)Mpix, g.k, atom, KB * A.km, true); };
         if (algo == MUCU_ALGO_IM2COL_GEMM && small_c_tc(g)) {
             // RGB-like layer: channel-padded copy of x, padded columns j' = (r, s8, c').
             err = launch_pad_channels(g, b, in0, ws + WL.a_off, st);
@@ -797,13 +814,8 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
             A.gsrc = ws + WL.a_off;
             A.cp = 16 / elt; A.s8 = (int)align_up((uint64_t)g.s, 8);
             A.N = g.r * A.s8 * A.cp;
-            finalize_tiling(L, elt, atom);
-            const int64_t t2 = ceil_div(A.N, A.BN) * ceil_div(A.M, 128);
-            int64_t ns2 = std::min<int64_t>(std::min<int64_t>(std::max<int64_t>(1, (2LL * num_sms) / t2),
-                                                              std::max<int64_t>(1, nkb / 16)), 65535);
-            A.kb_per_split = (int)ceil_div(nkb, ns2);
-            ns2 = ceil_div(nkb, A.kb_per_split);
-            grid2((int)ns2);
+            wgrad_tiling(atom, false);
+            if (!map_dy()) return -1;
             A.tma_bytes = a_bytes;
             return LAUNCH(A_TMA_MN2, B_GATHER_SMALLC_PAD, EPI_WGRAD_SMALLC);
         }
@@ -816,32 +828,40 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
                 if (err) return err;
             }
             if (RSC < atom) return -1;
-            if (!map2(&L.tb, colp, RSC, (uint64_t)Mpix, kp, atom, KB, true)) return -1;
-            A.tma_bytes = a_bytes + A.bn_atoms * KB * 128;
+            wgrad_tiling(16, true);
+            if (!map_dy()) return -1;
+            if (!map2(&L.tb, colp, RSC, (uint64_t)Mpix, kp, atom, KB * A.km, true)) return -1;
+            A.tma_bytes = A.km * (A.mt * a_bytes + A.bn_atoms * KB * 128);
             return LAUNCH(A_TMA_MN2, B_TMA_MN2, EPI_WGRAD_CHAIN);
         }
-        if (g.c % atom == 0 && use_tma_im2col() &&
-            make_im2col_map(&L.tb, elt, in0, g.c, g.w, g.h, b, -g.pad, -g.pad, g.pad - (g.s - 1), g.pad - (g.r - 1),
-                            KB, g.stride, true)) {
-            A.tma_bytes = a_bytes + A.bn_atoms * KB * 128;
-            return LAUNCH(A_TMA_MN2, B_TMA_IM2COL, EPI_WGRAD_CHAIN);
+        // implicit-im2col B producers load whole 128-B channel atoms of one tap:
+        // N tiles must start on an atom boundary.
+        if (g.c % atom == 0 && use_tma_im2col()) {
+            wgrad_tiling(atom, true);
+            if (!map_dy()) return -1;
+            if (make_im2col_map(&L.tb, elt, in0, g.c, g.w, g.h, b, -g.pad, -g.pad, g.pad - (g.s - 1),
+                                g.pad - (g.r - 1), KB * A.km, g.stride, true)) {
+                A.tma_bytes = A.km * (A.mt * a_bytes + A.bn_atoms * KB * 128);
+                return LAUNCH(A_TMA_MN2, B_TMA_IM2COL, EPI_WGRAD_CHAIN);
+            }
         }
         A.tma_bytes = a_bytes;
-        if (g.c % atom == 0) return LAUNCH(A_TMA_MN2, B_GATHER_WG, EPI_WGRAD_CHAIN);
+        if (g.c % atom == 0) {
+            wgrad_tiling(atom, false);
+            if (!map_dy()) return -1;
+            return LAUNCH(A_TMA_MN2, B_GATHER_WG, EPI_WGRAD_CHAIN);
+        }
         if (g.c * elt < 16) {
             // RGB-like layer: padded columns j' = (r, s8, c'), one 128-B atom per
             // 8-tap group; the epilogue folds them back into dw[k][r][s][c].
             A.cp = 16 / elt; A.s8 = (int)align_up((uint64_t)g.s, 8);
             A.N = g.r * A.s8 * A.cp;
-            finalize_tiling(L, elt, atom);
-            const int64_t t2 = ceil_div(A.N, A.BN) * ceil_div(A.M, 128);
-            int64_t ns2 = std::min<int64_t>(std::min<int64_t>(std::max<int64_t>(1, (2LL * num_sms) / t2),
-                                                              std::max<int64_t>(1, nkb / 16)), 65535);
-            A.kb_per_split = (int)ceil_div(nkb, ns2);
-            ns2 = ceil_div(nkb, A.kb_per_split);
-            grid2((int)ns2);
+            wgrad_tiling(atom, false);
+            if (!map_dy()) return -1;
             return LAUNCH(A_TMA_MN2, B_GATHER_SMALLC, EPI_WGRAD_SMALLC);
         }
+        wgrad_tiling(16, false);
+        if (!map_dy()) return -1;
         return LAUNCH(A_TMA_MN2, B_SCALAR_WG, EPI_WGRAD_CHAIN);
     }
 #undef LAUNCH

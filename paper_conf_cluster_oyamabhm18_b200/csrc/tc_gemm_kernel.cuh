@@ -18,7 +18,11 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
     using T = typename Elt<ELT>::T;
     constexpr int KB = 128 / ELT;            // K elements per stage
     constexpr int UMMA_K = 32 / ELT;         // K elements per MMA
-    const int A_BYTES = p.mt * 128 * 128;    // p.mt blocks of 128 rows x 128 B (tile M = 128 * p.mt)
+    // p.mt blocks of 128 rows x 128 B (tile M = 128 * p.mt); MN-major WGRAD
+    // stages hold p.km k-blocks (p.km x KB rows of K per 128-B atom column).
+    const int A_HALF = 128 * 128 * p.km;
+    const int A_BYTES = p.mt * A_HALF;
+    const int KD = KB * p.km;                // K rows per stage (MN-major modes)
     constexpr bool A_MN = (AM == A_TMA_MN2);
     constexpr bool B_MN = (BM_ == B_TMA_MN2 || BM_ == B_TMA_MN3 || BM_ == B_GATHER_WG || BM_ == B_SCALAR_DGRAD ||
                            BM_ == B_SCALAR_WG || BM_ == B_TMA_IM2COL || BM_ == B_GATHER_SMALLC ||
@@ -41,7 +45,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
     extern __shared__ uint8_t smem_raw[];
     uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
     const int S = p.stages;
-    const int B_BYTES = p.b_bytes;
+    const int B_BYTES = p.b_bytes * p.km;
     uint8_t* sA = smem;
     uint8_t* sB = smem + (size_t)S * A_BYTES;
     uint8_t* sBres = sB + (size_t)S * B_BYTES;  // B_RESIDENT: whole filter, k-block after k-block
@@ -251,7 +255,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
             // walked incrementally (KB pixels per k-block).
             int wb_n = 0, wb_p = 0, wb_q = 0;
             if constexpr (BM_ == B_TMA_IM2COL) {
-                const int m = kb_begin * KB, pq = p.P * p.Q;
+                const int m = kb_begin * KD, pq = p.P * p.Q;
                 wb_n = m / pq;
                 const int rem = m - wb_n * pq;
                 wb_p = rem / p.Q; wb_q = rem - wb_p * p.Q;
@@ -272,18 +276,20 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                             tma_load_im2col_4d(aT + hh * 16384 + j * 2048, &tmA, fb, 0, hh ? ic_w[1] : ic_w[0],
                                                hh ? ic_h[1] : ic_h[0], hh ? ic_n[1] : ic_n[0],
                                                (uint16_t)(s0 + j), (uint16_t)r);
+                } else if ((A_TMA || B_TMA) && t == 0 && (p.debug & 4)) {
+                    mbar_arrive(fb);  // debug bit 2: no TMA loads (MMA-rate experiments)
                 } else if ((A_TMA || B_TMA) && t == 0) {
                     mbar_arrive_tx(fb, (uint32_t)p.tma_bytes);
                     // A: p.mt blocks of 128 rows (16 KB each)
                     for (int hh = 0; hh < p.mt; ++hh) {
-                        const uint32_t aH = aT + hh * 16384;
+                        const uint32_t aH = aT + hh * A_HALF;
                         const int mH = m0 + 128 * hh;
                         if constexpr (AM == A_TMA_K2) tma_load_2d(aH, &tmA, fb, kb * KB, mH);
                         if constexpr (AM == A_TMA_K3) tma_load_3d(aH, &tmA, fb, kb * KB, mH, z);
                         if constexpr (AM == A_TMA_MN2) {
 #pragma unroll
                             for (int a = 0; a < 128 * ELT / 128; ++a)
-                                tma_load_2d(aH + a * KB * 128, &tmA, fb, mH + a * (128 / ELT), kb * KB);
+                                tma_load_2d(aH + a * KD * 128, &tmA, fb, mH + a * (128 / ELT), kb * KD);
                         }
                         if constexpr (AM == A_TMA_IM2COL) {
                             // 128 consecutive output pixels x KB channels of tap (r,s) in one TMA
@@ -297,7 +303,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                     if constexpr (BM_ == B_TMA_K3) tma_load_3d(bT, &tmB, fb, kb * KB, n0, z);
                     if constexpr (BM_ == B_TMA_MN2) {
                         for (int a = 0; a < p.bn_atoms; ++a)
-                            tma_load_2d(bT + a * KB * 128, &tmB, fb, n0 + a * (128 / ELT), kb * KB);
+                            tma_load_2d(bT + a * KD * 128, &tmB, fb, n0 + a * (128 / ELT), kb * KD);
                     }
                     if constexpr (BM_ == B_TMA_MN3) {
                         // k-block kb covers tap kb / (K/KB), channels k0 = (kb % (K/KB)) * KB
@@ -314,13 +320,13 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                             const int j0 = n0 + a * (128 / ELT);
                             const int rs = j0 / p.C, c0 = j0 - rs * p.C;
                             const int r = rs / p.S, sx = rs - r * p.S;
-                            tma_load_im2col_4d(bT + a * KB * 128, &tmB, fb, c0, w0, h0, wb_n, (uint16_t)sx,
+                            tma_load_im2col_4d(bT + a * KD * 128, &tmB, fb, c0, w0, h0, wb_n, (uint16_t)sx,
                                                (uint16_t)r);
                         }
                     }
                 }
                 if constexpr (BM_ == B_TMA_IM2COL) {
-                    wb_q += KB;
+                    wb_q += KD;
                     while (wb_q >= p.Q) { wb_q -= p.Q; if (++wb_p == p.P) { wb_p = 0; ++wb_n; } }
                 }
                 // ---- A gathers ----
@@ -593,27 +599,33 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                     // p.mt independent accumulators (one per 128-row half) share B and
                     // interleave, so short-N MMAs are not serialised on one accumulator.
                     // (Both variants fully unrolled: the issue thread must not stall.)
-                    auto issue = [&](auto mt_c) {
+                    auto issue = [&](auto mt_c, const int jj) {
                         constexpr int MT = decltype(mt_c)::value;
+                        // MN-major operands: k-block jj of the stage starts jj * KB rows in
+                        const uint32_t kofs = (uint32_t)(jj * KB * 128);
 #pragma unroll
                         for (int j = 0; j < KB / UMMA_K; ++j) {
-                            const uint64_t bd = B_MN ? sdesc(bT + j * UMMA_K * 128, KB * 128, MN_SBO, MN_LAYOUT)
+                            const uint64_t bd = B_MN ? sdesc(bT + kofs + j * UMMA_K * 128, KD * 128, MN_SBO, MN_LAYOUT)
                                                      : sdesc(bT + j * 32, 16, 1024);
 #pragma unroll
                             for (int hh = 0; hh < MT; ++hh) {
-                                const uint32_t aH = aT + hh * 16384;
+                                const uint32_t aH = aT + hh * A_HALF;
                                 // no-swizzle A: core matrices 8 rows x 16 B, SBO 128 B (rows),
                                 // LBO 2 KB (next tap); one MMA covers 32 B of K = 2 taps
-                                const uint64_t ad = A_NOSWZ ? sdesc(aH + j * 4096, 2048, 128, 0)
-                                                  : A_MN ? sdesc(aH + j * UMMA_K * 128, KB * 128, MN_SBO, MN_LAYOUT)
-                                                         : sdesc(aH + j * 32, 16, 1024);
-                                mma<ELT>(dtm + (uint32_t)(hh * p.BN), ad, bd, idesc,
-                                         (kb > kb_begin || j > 0) ? 1u : 0u);
+                                const uint64_t ad =
+                                    A_NOSWZ ? sdesc(aH + j * 4096, 2048, 128, 0)
+                                    : A_MN  ? sdesc(aH + kofs + j * UMMA_K * 128, KD * 128, MN_SBO, MN_LAYOUT)
+                                            : sdesc(aH + j * 32, 16, 1024);
+                                if (!(p.debug & 8))  // debug bit 3: no MMAs (load-rate experiments)
+                                    mma<ELT>(dtm + (uint32_t)(hh * p.BN), ad, bd, idesc,
+                                             (kb > kb_begin || jj > 0 || j > 0) ? 1u : 0u);
                             }
                         }
                     };
-                    if (p.mt == 2) issue(std::integral_constant<int, 2>{});
-                    else issue(std::integral_constant<int, 1>{});
+                    for (int jj = 0; jj < p.km; ++jj) {
+                        if (p.mt == 2) issue(std::integral_constant<int, 2>{}, jj);
+                        else issue(std::integral_constant<int, 1>{}, jj);
+                    }
                     mma_commit(smem_u32(&empty[s]));
                 }
                 __syncwarp();
@@ -623,8 +635,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                 else mbar_arrive(smem_u32(&tfull[acc]));
             }
             __syncwarp();
-            acc ^= 1;
-            if (acc == 0) aph ^= 1u;
+            if (++acc == p.nacc) { acc = 0; aph ^= 1u; }
         }
     } else {
         // ============================ epilogue =============================
@@ -786,8 +797,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
             tc_fence_before();
             __syncwarp();
             if (lane == 0) mbar_arrive(smem_u32(&tempty[acc]));
-            acc ^= 1;
-            if (acc == 0) aph ^= 1u;
+            if (++acc == p.nacc) { acc = 0; aph ^= 1u; }
         }
     }
     tc_fence_before();

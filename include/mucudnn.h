@@ -130,8 +130,8 @@ mucu_status_t mucu_output_dims(const mucu_conv_desc_t* desc, int32_t* p, int32_t
  *                     128 B when R*S*C < 128/elt on tensor cores); 0 for 1x1/s1/p0
  *   I2C, TF32/BF16, stride st > 1 and C*elt < 16 ("space-to-depth"):
  *                     Dr = ceil(R/st), Ds = ceil(S/st), Cs = st*st*C rounded up to 128/elt
- *                     FWD   (when Cs <= 2*st*st*C): K*Dr*Ds*Cs*elt + b*(P+Dr-1)*(Q+Ds-1)*Cs*elt
- *                     WGRAD (when Cs <= 2*st*st*C): b*(P+Dr-1)*(Q+Ds-1)*Cs*elt
+ *                     FWD:   K*Dr*Ds*Cs*elt + b*(P+Dr-1)*(Q+Ds-1)*Cs*elt
+ *                     WGRAD: b*(P+Dr-1)*(Q+Ds-1)*Cs*elt
  *                     DGRAD (when K % (128/elt) == 0, st*st*C <= 256): st*st*C*Dr*Ds*K*elt
  *   WG  FWD:          16*K*C*elt + 16*b*T*C*elt + 16*b*T*K*4,   T = ceil(P/2)*ceil(Q/2)
  *   WG  DGRAD:        16*C*K*elt + 16*b*T'*K*elt + 16*b*T'*C*4, T' = ceil(H/2)*ceil(W/2)

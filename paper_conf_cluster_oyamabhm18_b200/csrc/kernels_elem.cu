@@ -361,29 +361,35 @@ __global__ void col2im_taps_kernel(const float* __restrict__ dcol, T* __restrict
 // (0 off the image and in the channel padding c' >= st*st*C).  One thread per
 // 16-B chunk of xs, so every store is a full vector.
 template <class T>
-__global__ void s2d_input_kernel(const T* __restrict__ x, T* __restrict__ xs, int64_t chunks, int H, int W, int C,
+__global__ void s2d_input_kernel(const T* __restrict__ x, T* __restrict__ xs, int chunks, int H, int W, int C,
                                  int I, int J, int st, int pad, int Cs) {
     constexpr int V = 16 / sizeof(T);
     const int cpp = Cs / V, stc = st * C, real = st * stc;
-    for (int64_t idx = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; idx < chunks;
-         idx += (int64_t)gridDim.x * blockDim.x) {
-        const int64_t pix = idx / cpp;
-        const int c0 = (int)(idx - pix * cpp) * V;
-        const int j = (int)(pix % J);
-        const int64_t t = pix / J;
-        const int i = (int)(t % I), n = (int)(t / I);
-        const int h0 = st * i - pad, w0 = st * j - pad;
-        int a = c0 / stc, b = (c0 - a * stc) / C, c = c0 - a * stc - b * C;
+    // 32-bit index math (the launcher checks the range): 64-bit divisions
+    // dominated the first version of this memory-bound kernel.
+    for (int idx = blockIdx.x * blockDim.x + threadIdx.x; idx < chunks; idx += gridDim.x * blockDim.x) {
+        const int pix = idx / cpp;
+        const int c0 = (idx - pix * cpp) * V;
         __align__(16) T vals[V];
+        if (c0 >= real) {
 #pragma unroll
-        for (int u = 0; u < V; ++u) {
-            const int h = h0 + a, w = w0 + b;
-            vals[u] = (c0 + u < real && (unsigned)h < (unsigned)H && (unsigned)w < (unsigned)W)
-                          ? x[(((int64_t)n * H + h) * W + w) * C + c]
-                          : from_f<T>(0.f);
-            if (++c == C) { c = 0; if (++b == st) { b = 0; ++a; } }
+            for (int u = 0; u < V; ++u) vals[u] = from_f<T>(0.f);
+        } else {
+            const int t = pix / J, j = pix - t * J;
+            const int n = t / I, i = t - n * I;
+            const int h0 = st * i - pad, w0 = st * j - pad;
+            int a = c0 / stc, b = (c0 - a * stc) / C, c = c0 - a * stc - b * C;
+            const T* xn = x + (size_t)n * H * W * C;
+#pragma unroll
+            for (int u = 0; u < V; ++u) {
+                const int h = h0 + a, w = w0 + b;
+                vals[u] = (c0 + u < real && (unsigned)h < (unsigned)H && (unsigned)w < (unsigned)W)
+                              ? xn[(h * W + w) * C + c]
+                              : from_f<T>(0.f);
+                if (++c == C) { c = 0; if (++b == st) { b = 0; ++a; } }
+            }
         }
-        *reinterpret_cast<uint4*>(xs + idx * V) = *reinterpret_cast<const uint4*>(vals);
+        *reinterpret_cast<uint4*>(xs + (size_t)idx * V) = *reinterpret_cast<const uint4*>(vals);
     }
 }
 
@@ -558,12 +564,13 @@ int launch_wg_output(const Geom& g, bool dgrad, int32_t b, float alpha, const fl
 int launch_s2d_input(const Geom& g, int32_t b, int I, int J, int Cs, const void* x, void* xs, cudaStream_t st) {
     const int V = 16 / elt_size(g.math);
     const int64_t chunks = (int64_t)b * I * J * (Cs / V);
+    if (chunks >= (1LL << 31) || (int64_t)g.h * g.w * g.c >= (1LL << 31)) return (int)cudaErrorInvalidValue;
     const int grid = grid_for(chunks, 256);
     if (g.math == MUCU_MATH_BF16)
-        s2d_input_kernel<__nv_bfloat16><<<grid, 256, 0, st>>>((const __nv_bfloat16*)x, (__nv_bfloat16*)xs, chunks, g.h,
-                                                              g.w, g.c, I, J, g.stride, g.pad, Cs);
+        s2d_input_kernel<__nv_bfloat16><<<grid, 256, 0, st>>>((const __nv_bfloat16*)x, (__nv_bfloat16*)xs, (int)chunks,
+                                                              g.h, g.w, g.c, I, J, g.stride, g.pad, Cs);
     else
-        s2d_input_kernel<float><<<grid, 256, 0, st>>>((const float*)x, (float*)xs, chunks, g.h, g.w, g.c, I, J,
+        s2d_input_kernel<float><<<grid, 256, 0, st>>>((const float*)x, (float*)xs, (int)chunks, g.h, g.w, g.c, I, J,
                                                       g.stride, g.pad, Cs);
     count_launch();
     return (int)cudaGetLastError();

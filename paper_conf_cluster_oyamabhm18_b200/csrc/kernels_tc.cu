@@ -403,7 +403,7 @@ int launch_t(Launch& L, cudaStream_t st) {
 
 void size_stages(TcArgs& a) {
     a.nacc = a.mt * a.BN <= 256 ? 2 : 1;
-    const int cols = a.nacc * a.mt * a.BN;  // accumulators x mt halves
+    const int cols = a.nacc * a.mt * a.BN;  // accumulator buffers x mt halves
     a.tmem_cols = cols <= 64 ? 64 : cols <= 128 ? 128 : cols <= 256 ? 256 : 512;
     if (a.km < 1) a.km = 1;
     const int stage_bytes = a.km * (a.mt * 128 * 128 + a.b_bytes);

@@ -37,9 +37,8 @@ bool is_pointwise(const Geom& g);  // 1x1, stride 1, pad 0: im2col(x) == x
 bool small_c_tc(const Geom& g);    // tensor-core math and C*elt < 16 B (RGB input layer)
 // Strided small-C layers whose I2C algorithm runs on the space-to-depth image:
 // a stride-1 ceil(R/st) x ceil(S/st) conv over st*st*C channels (padded to
-// s2d_channels = a multiple of 128 B).  FWD/WGRAD need the padding to at most
-// double the channels; DGRAD (no padding: the super-pixel channels are GEMM
-// columns) needs K to be a multiple of 128 B / elt.
+// s2d_channels = a multiple of 128 B).  DGRAD (no padding: the super-pixel
+// channels are GEMM columns) needs K to be a multiple of 128 B / elt.
 bool s2d_tc(const Geom& g, int type);
 int s2d_channels(const Geom& g);
 inline int s2d_taps(int r, int stride) { return (r + stride - 1) / stride; }

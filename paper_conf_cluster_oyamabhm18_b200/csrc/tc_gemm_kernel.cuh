@@ -282,7 +282,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                     mbar_arrive_tx(fb, (uint32_t)p.tma_bytes);
                     // A: p.mt blocks of 128 rows (16 KB each)
                     for (int hh = 0; hh < p.mt; ++hh) {
-                        const uint32_t aH = aT + hh * A_HALF;
+                        const uint32_t aH = aT + hh * (A_MN ? (uint32_t)A_HALF : 16384u);
                         const int mH = m0 + 128 * hh;
                         if constexpr (AM == A_TMA_K2) tma_load_2d(aH, &tmA, fb, kb * KB, mH);
                         if constexpr (AM == A_TMA_K3) tma_load_3d(aH, &tmA, fb, kb * KB, mH, z);
@@ -582,6 +582,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
         uint32_t ph = 0;
         int acc = 0;
         uint32_t aph = 0;
+        const int KDm = A_MN ? KD : KB;  // K rows per MN-major atom column (km > 1 only with A_MN)
         if constexpr (B_RES) mbar_wait(smem_u32(bres_bar), 0u);  // staged filter is ready
         for (int tile = blockIdx.x; tile < total_tiles; tile += gridDim.x) {
             int m0, n0, z, kb_begin, kb_end;
@@ -592,39 +593,45 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
             for (int kb = kb_begin; kb < kb_end; ++kb, s = (s + 1 == S) ? 0 : s + 1, ph ^= (s == 0) ? 1u : 0u) {
                 mbar_wait(smem_u32(&full[s]), ph);
                 tc_fence_after();
-                if (lane == 0) {
+                if (lane == 0 && !(p.debug & 8)) {  // debug bit 3: no MMAs (load-rate experiments)
                     const uint32_t aT = smem_u32(sA + (size_t)s * A_BYTES);
                     const uint32_t bT = B_RES ? smem_u32(sBres) + (uint32_t)(kb * p.BN * 128)
                                               : smem_u32(sB + (size_t)s * B_BYTES);
                     // p.mt independent accumulators (one per 128-row half) share B and
                     // interleave, so short-N MMAs are not serialised on one accumulator.
-                    // (Both variants fully unrolled: the issue thread must not stall.)
+                    // Fully unrolled with compile-time strides: the single issuing thread
+                    // is on the critical path (measured: runtime strides / extra variants
+                    // here cost 10-30% on the FWD kernels).
                     auto issue = [&](auto mt_c, const int jj) {
                         constexpr int MT = decltype(mt_c)::value;
                         // MN-major operands: k-block jj of the stage starts jj * KB rows in
-                        const uint32_t kofs = (uint32_t)(jj * KB * 128);
+                        const uint32_t kofs = A_MN ? (uint32_t)(jj * KB * 128) : 0u;
 #pragma unroll
                         for (int j = 0; j < KB / UMMA_K; ++j) {
-                            const uint64_t bd = B_MN ? sdesc(bT + kofs + j * UMMA_K * 128, KD * 128, MN_SBO, MN_LAYOUT)
+                            const uint64_t bd = B_MN ? sdesc(bT + kofs + j * UMMA_K * 128, KDm * 128, MN_SBO, MN_LAYOUT)
                                                      : sdesc(bT + j * 32, 16, 1024);
 #pragma unroll
                             for (int hh = 0; hh < MT; ++hh) {
-                                const uint32_t aH = aT + hh * A_HALF;
+                                const uint32_t aH = aT + hh * (A_MN ? (uint32_t)A_HALF : 16384u);
                                 // no-swizzle A: core matrices 8 rows x 16 B, SBO 128 B (rows),
                                 // LBO 2 KB (next tap); one MMA covers 32 B of K = 2 taps
                                 const uint64_t ad =
                                     A_NOSWZ ? sdesc(aH + j * 4096, 2048, 128, 0)
-                                    : A_MN  ? sdesc(aH + kofs + j * UMMA_K * 128, KD * 128, MN_SBO, MN_LAYOUT)
+                                    : A_MN  ? sdesc(aH + kofs + j * UMMA_K * 128, KDm * 128, MN_SBO, MN_LAYOUT)
                                             : sdesc(aH + j * 32, 16, 1024);
-                                if (!(p.debug & 8))  // debug bit 3: no MMAs (load-rate experiments)
-                                    mma<ELT>(dtm + (uint32_t)(hh * p.BN), ad, bd, idesc,
-                                             (kb > kb_begin || jj > 0 || j > 0) ? 1u : 0u);
+                                mma<ELT>(dtm + (uint32_t)(hh * p.BN), ad, bd, idesc,
+                                         (kb > kb_begin || jj > 0 || j > 0) ? 1u : 0u);
                             }
                         }
                     };
-                    for (int jj = 0; jj < p.km; ++jj) {
-                        if (p.mt == 2) issue(std::integral_constant<int, 2>{}, jj);
-                        else issue(std::integral_constant<int, 1>{}, jj);
+                    if constexpr (A_MN) {
+                        for (int jj = 0; jj < p.km; ++jj) {
+                            if (p.mt == 2) issue(std::integral_constant<int, 2>{}, jj);
+                            else issue(std::integral_constant<int, 1>{}, jj);
+                        }
+                    } else {
+                        if (p.mt == 2) issue(std::integral_constant<int, 2>{}, 0);
+                        else issue(std::integral_constant<int, 1>{}, 0);
                     }
                     mma_commit(smem_u32(&empty[s]));
                 }
@@ -678,18 +685,21 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                 if (m >= p.M || (p.debug & 1)) continue;  // debug bit 0: skip stores (timing experiments)
                 const int nb = n0 + c0;
                 if constexpr (EPI == EPI_D2S) {
-                    // super-pixel row (n, i, jj); column (a, b, c) walked incrementally
+                    // super-pixel row (n, i, jj); column (a, b, c) walked incrementally:
+                    // the dx offset advances by 1 inside an (a) block of st*C values and
+                    // by (W - st)*C between blocks (no per-column index arithmetic).
                     const int hw = p.ph_H * p.ph_W;
                     const int n = m / hw, rem = m - n * hw, ii = rem / p.ph_W, jj = rem - ii * p.ph_W;
                     const int h0 = p.s2_st * ii - p.pad, w0 = p.s2_st * jj - p.pad;
-                    const long long nbase = (long long)n * p.H;
                     const int stc = p.s2_st * p.C;
                     int a = nb / stc, bq = (nb - a * stc) / p.C, c = nb - a * stc - bq * p.C;
+                    long long off = (((long long)n * p.H + h0 + a) * p.W + w0 + bq) * p.C + c;
+                    const long long jump = (long long)(p.W - p.s2_st) * p.C;
+                    bool okh = (unsigned)(h0 + a) < (unsigned)p.H, okw = (unsigned)(w0 + bq) < (unsigned)p.W;
+                    const int nlim = p.N - nb;
 #pragma unroll
                     for (int j = 0; j < 32; ++j) {
-                        const int h = h0 + a, w = w0 + bq;
-                        if (nb + j < p.N && (unsigned)h < (unsigned)p.H && (unsigned)w < (unsigned)p.W) {
-                            const long long off = ((nbase + h) * p.W + w) * p.C + c;
+                        if (j < nlim && okh && okw) {
                             float o = p.alpha * __uint_as_float(v[j]);
                             if (p.out_bf16) {
                                 __nv_bfloat16* d = (__nv_bfloat16*)p.out + off;
@@ -701,7 +711,15 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                                 *d = o;
                             }
                         }
-                        if (++c == p.C) { c = 0; if (++bq == p.s2_st) { bq = 0; ++a; } }
+                        ++off;
+                        if (++c == p.C) {
+                            c = 0;
+                            if (++bq == p.s2_st) {
+                                bq = 0; ++a; off += jump;
+                                okh = (unsigned)(h0 + a) < (unsigned)p.H;
+                            }
+                            okw = (unsigned)(w0 + bq) < (unsigned)p.W;
+                        }
                     }
                 } else if constexpr (EPI == EPI_WGRAD_S2D) {
                     // column (tap (d,e), channel (a, b, c)) -> dw[k][st*d+a][st*e+b][c]

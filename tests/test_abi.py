@@ -93,8 +93,8 @@ def test_workspace_unaligned_filter_row():
 
 
 def test_workspace_small_c_tensor_core():
-    # C*elt < 16 B on tensor cores: I2C FWD/WGRAD keep x with channels padded to 16 B
-    d = mu.desc(4, 3, 224, 224, 64, 7, 7, 3, 2, mu.MATH_BF16)
+    # C*elt < 16 B on tensor cores, stride 1: I2C FWD/WGRAD keep x with channels padded to 16 B
+    d = mu.desc(4, 3, 224, 224, 64, 7, 7, 3, 1, mu.MATH_BF16)
     assert mu.workspace_size(d, mu.FWD, mu.IM2COL_GEMM, 2) == 2 * 224 * 224 * 16
     assert mu.workspace_size(d, mu.BWD_FILTER, mu.IM2COL_GEMM, 1) == 224 * 224 * 16
 
@@ -107,8 +107,12 @@ def test_workspace_space_to_depth():
     assert mu.workspace_size(d, mu.FWD, mu.IM2COL_GEMM, 2) == a256(64 * 9 * 64 * 4) + a256(2 * xs)
     assert mu.workspace_size(d, mu.BWD_FILTER, mu.IM2COL_GEMM, 3) == a256(3 * xs)
     assert mu.workspace_size(d, mu.BWD_DATA, mu.IM2COL_GEMM, 4) == a256(48 * 9 * 64 * 4)
-    # ResNet conv1 BF16: Cs = 12 -> 64 would more than double the channels, so FWD keeps the
-    # channel-padded image, while DGRAD (no channel padding) uses the st*st*C x Dr*Ds*K filter
+    # ResNet conv1 BF16: Dr = 4, Cs = 12 -> 64 (BF16 atom); DGRAD (no channel padding) uses the
+    # st*st*C x Dr*Ds*K filter
     d = mu.desc(2, 3, 224, 224, 64, 7, 7, 3, 2, mu.MATH_BF16)
-    assert mu.workspace_size(d, mu.FWD, mu.IM2COL_GEMM, 2) == 2 * 224 * 224 * 16
+    xs = 115 * 115 * 64 * 2
+    assert mu.workspace_size(d, mu.FWD, mu.IM2COL_GEMM, 2) == a256(64 * 16 * 64 * 2) + a256(2 * xs)
     assert mu.workspace_size(d, mu.BWD_DATA, mu.IM2COL_GEMM, 2) == a256(12 * 16 * 64 * 2)
+    # stride 1 keeps the channel-padded image (16 B per pixel)
+    d = mu.desc(2, 3, 32, 32, 64, 3, 3, 1, 1, mu.MATH_BF16)
+    assert mu.workspace_size(d, mu.FWD, mu.IM2COL_GEMM, 2) == 2 * 32 * 32 * 16

@@ -17,7 +17,7 @@ def launches(path):
             continue
         v = float(r["Metric Value"].replace(",", ""))
         unit = r.get("Metric Unit", "")
-        us = v / 1e3 if unit == "nsecond" else v * 1e3 if unit == "msecond" else v
+        us = v / 1e3 if unit in ("ns", "nsecond") else v * 1e3 if unit in ("ms", "msecond") else v
         name = r["Kernel Name"].split("(")[0][:90]
         agg[name][0] += 1
         agg[name][1] += us

@@ -56,4 +56,22 @@ PY
     -k regex:tc_conv_gemm -c 1 -o $OUT/dominant_full -f python tools/profile_one.py --config alexnet --math tf32 $CMD \
     > $OUT/full.log 2>&1
   echo "full rc=$?" | tee -a $OUT/status
+  # DRAM bytes of every launch of one call of the dominant op (bench.py roofline.traffic)
+  timeout -s KILL 600 ncu --metrics dram__bytes_read.sum,dram__bytes_write.sum,gpu__time_duration.sum \
+    --clock-control none --profile-from-start off --csv --log-file $OUT/dominant_traffic.csv \
+    python tools/profile_one.py --config alexnet --math tf32 $CMD > $OUT/traffic.log 2>&1
+  python - $OUT/dominant_traffic.csv $OUT/bench_alexnet_tf32.json $OUT/traffic.json <<'PY'
+import csv, io, json, sys
+txt = open(sys.argv[1]).read()
+rows = list(csv.DictReader(io.StringIO(txt[txt.find('"ID"'):])))
+scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}
+tot = sum(float(r["Metric Value"].replace(",", "")) * scale.get(r["Metric Unit"], 1)
+          for r in rows if r["Metric Name"] in ("dram__bytes_read.sum", "dram__bytes_write.sum"))
+d = json.load(open(sys.argv[2]))
+k = d["roofline"]["kernel"].split()
+key = f"alexnet/tf32/{k[0]}/{k[1]}"
+json.dump({key: int(tot), "_note": "DRAM read+write bytes of one call of the op (all its launches), "
+           "ncu --metrics dram__bytes_read.sum,dram__bytes_write.sum, tools/gpu_round.sh"}, open(sys.argv[3], "w"), indent=1)
+print("traffic", key, int(tot))
+PY
 fi

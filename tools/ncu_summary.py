@@ -29,14 +29,18 @@ def launches(path):
     return "\n".join(out)
 
 
-KEYS = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum", "gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed",
-        "sm__pipe_tensor_cycles_active.avg.pct_of_peak_sustained_elapsed", "sm__throughput.avg.pct_of_peak_sustained_elapsed",
-        "lts__t_bytes.sum", "launch__registers_per_thread", "launch__grid_size", "launch__shared_mem_per_block_dynamic",
-        "sm__warps_active.avg.pct_of_peak_sustained_active", "l1tex__t_bytes.sum", "sm__inst_executed_pipe_tensor.sum",
-        "smsp__pcsamp_warps_issue_stalled_long_scoreboard", "sm__cycles_elapsed.avg.per_second"]
+KEYS = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum",
+        "gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed", "lts__t_bytes.sum",
+        "lts__throughput.avg.pct_of_peak_sustained_elapsed",
+        "sm__pipe_tensor_cycles_active.avg.pct_of_peak_sustained_elapsed",
+        "sm__mem_tensor_cycles_active.avg.pct_of_peak_sustained_elapsed",
+        "sm__throughput.avg.pct_of_peak_sustained_elapsed", "sm__warps_active.avg.pct_of_peak_sustained_active",
+        "l1tex__t_bytes.sum", "launch__registers_per_thread", "launch__grid_size", "launch__block_size",
+        "launch__shared_mem_per_block_dynamic", "sm__cycles_elapsed.avg.per_second"]
 
 
 def full(path):
+    """Curated metrics of every kernel in a `--set full` report."""
     r = subprocess.run(["ncu", "-i", path, "--page", "raw", "--csv"], capture_output=True, text=True)
     rows = list(csv.reader(io.StringIO(r.stdout)))
     if len(rows) < 3:
@@ -46,8 +50,8 @@ def full(path):
     for row in rows[2:]:
         d = dict(zip(hdr, row))
         out.append(f"== {d.get('Kernel Name', '')[:120]}")
-        for k in hdr:
-            if any(k.startswith(p) for p in KEYS) or "tensor" in k and "pct" in k:
+        for k in KEYS:
+            if k in d:
                 out.append(f"  {k} = {d[k]} {units[hdr.index(k)]}")
     return "\n".join(out)
 

@@ -756,6 +756,14 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
                 make_im2col_map(&L.ta, elt, in0, g.k, g.q, g.p, b, lw, lh, lw + g.w - g.q, lh + g.h - g.p, 128, 1,
                                 false)) {
                 A.im2col_dgrad = 1;
+                // C a multiple of 128 (> 128): 256 x 128 tiles (two interleaved
+                // accumulators) beat 128 x min(C, 256) ones (measured, AlexNet conv4/5)
+                if (g.c > 128 && g.c % 128 == 0 && ceil_div(A.M, 256) >= num_sms && !env_int("MUCU_FORCE_BN", 0)) {
+                    A.BN = 128;
+                    A.bn_atoms = (A.BN * elt + 127) / 128;
+                    A.b_bytes = std::max(A.BN * 128, A.bn_atoms * (128 / elt) * 128);
+                    size_stages(A);
+                }
                 use_mt2(L, num_sms);
                 grid2(1);
                 A.tma_bytes = 16384 * A.mt + A.bn_atoms * KB * 128;

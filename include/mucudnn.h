@@ -128,9 +128,11 @@ mucu_status_t mucu_output_dims(const mucu_conv_desc_t* desc, int32_t* p, int32_t
  *                     channels zero-padded to 16 B, gathered tap by tap on chip
  *   I2C DGRAD:        b*P*Q*ceil_4(R*S*C)*4 (fp32 dcol)  (+ filter copy as above, or with rows of
  *                     128 B when R*S*C < 128/elt on tensor cores); 0 for 1x1/s1/p0
- *   I2C, TF32/BF16, stride st > 1 and C*elt < 16 ("space-to-depth", DESIGN.md):
- *                     Dr = ceil(R/st), Ds = ceil(S/st), Cs = st*st*C rounded up to 128/elt
- *                     FWD:   K*Dr*Ds*Cs*elt + b*(P+Dr-1)*(Q+Ds-1)*Cs*elt
+ *   I2C, TF32/BF16, stride st > 1 and C*elt < 16 ("space-to-depth", DESIGN.md 6.3):
+ *                     u = 2 for FWD with st = 2, else 1; f = st*u;
+ *                     Dr = (st*(u-1) + R - 1)/f + 1, Ds likewise, Cs = f*f*C rounded up to 128/elt,
+ *                     Pu = ceil(P/u), Qu = ceil(Q/u)
+ *                     FWD:   u*u*K*Dr*Ds*Cs*elt + b*(Pu+Dr-1)*(Qu+Ds-1)*Cs*elt
  *                     WGRAD: b*(P+Dr-1)*(Q+Ds-1)*Cs*elt
  *                     DGRAD (when K % (128/elt) == 0, st*st*C <= 256): st*st*C*Dr*Ds*K*elt
  *   WG  FWD:          16*K*C*elt + 16*b*T*C*elt + 16*b*T*K*4,   T = ceil(P/2)*ceil(Q/2)

@@ -61,6 +61,23 @@ int s2d_channels(const Geom& g) {
     return (int)align_up((uint64_t)g.stride * g.stride * g.c, (uint64_t)atom);
 }
 
+S2d s2d_geom(const Geom& g, int type) {
+    S2d z;
+    const int st = g.stride;
+    z.u = (type == MUCU_FWD && st == 2) ? 2 : 1;
+    z.f = st * z.u;
+    // output row u*i' + uu reads input rows f*(i' + d) + a - pad with st*uu + r = f*d + a
+    z.Dr = (st * (z.u - 1) + g.r - 1) / z.f + 1;
+    z.Ds = (st * (z.u - 1) + g.s - 1) / z.f + 1;
+    const int atom = 128 / elt_size(g.math);
+    z.Cs = (int)align_up((uint64_t)z.f * z.f * g.c, (uint64_t)atom);
+    z.Pu = (g.p + z.u - 1) / z.u;
+    z.Qu = (g.q + z.u - 1) / z.u;
+    z.I = z.Pu + z.Dr - 1;
+    z.J = z.Qu + z.Ds - 1;
+    return z;
+}
+
 bool s2d_tc(const Geom& g, int type) {
     if (!small_c_tc(g) || g.stride < 2) return false;
     if (type == MUCU_BWD_DATA) return g.k % (128 / elt_size(g.math)) == 0 && g.stride * g.stride * g.c <= 256;
@@ -99,14 +116,15 @@ mucu_status_t ws_layout(const Geom& g, int type, int algo, int32_t b, WsLayout* 
         if (s2d_tc(g, type)) {
             // Space-to-depth: FWD = [s2d filter K x Dr*Ds*Cs][xs b x I x J x Cs],
             // WGRAD = [xs], DGRAD = [s2d filter st*st*C x Dr*Ds*K] (b-independent).
-            const uint64_t Dr = s2d_taps(g.r, g.stride), Ds = s2d_taps(g.s, g.stride);
-            const uint64_t Cs = (uint64_t)s2d_channels(g);
+            const S2d z = s2d_geom(g, type);
+            const uint64_t Dr = z.Dr, Ds = z.Ds, Cs = z.Cs;
             if (type == MUCU_BWD_DATA) {
                 L->fixed_bytes = align_up((uint64_t)g.stride * g.stride * g.c * Dr * Ds * g.k * elt, 256);
             } else {
-                if (type == MUCU_FWD) L->fixed_bytes = align_up((uint64_t)g.k * Dr * Ds * Cs * elt, 256);
+                if (type == MUCU_FWD)
+                    L->fixed_bytes = align_up((uint64_t)z.u * z.u * g.k * Dr * Ds * Cs * elt, 256);
                 L->a_off = L->fixed_bytes;
-                L->a_bytes = align_up((uint64_t)b * (g.p + Dr - 1) * (g.q + Ds - 1) * Cs * elt, 256);
+                L->a_bytes = align_up((uint64_t)b * z.I * z.J * Cs * elt, 256);
             }
             L->kpitch = (int32_t)Cs;
             L->total = L->fixed_bytes + L->a_bytes;

@@ -393,23 +393,26 @@ __global__ void s2d_input_kernel(const T* __restrict__ x, T* __restrict__ xs, in
     }
 }
 
-// Space-to-depth filter.  FWD (K-major B of the stride-1 conv on xs):
-//   out[k][(d*Ds + e)*Cs + (a*st + b)*C + c] = w[k][st*d + a][st*e + b][c]
-// DGRAD (K-major B of the transposed conv, N = st*st*C columns of dx):
+// Space-to-depth filter.  FWD (K-major B of the stride-1 conv on xs, output
+// super-pixels of u x u outputs; input super-pixels of f = st*u pixels):
+//   out[(uu*u + vv)*K + k][(d*Ds + e)*Cs + (a*f + b)*C + c] = w[k][f*d + a - st*uu][f*e + b - st*vv][c]
+// DGRAD (u = 1, f = st; K-major B of the transposed conv, N = st*st*C columns of dx):
 //   out[(a*st + b)*C + c][(d*Ds + e)*K + k] = w[k][st*d + a][st*e + b][c]
-// Zero where st*d + a >= R, st*e + b >= S, or in the channel padding.
+// Zero where the filter tap falls outside R x S, or in the channel padding.
 template <class T>
 __global__ void s2d_filter_kernel(const T* __restrict__ w, T* __restrict__ out, int64_t total, int K, int R, int S,
-                                  int C, int st, int Dr, int Ds, int Cs, bool dgrad) {
-    const int stc = st * C, real = st * stc;
+                                  int C, int st, int f, int u, int Dr, int Ds, int Cs, bool dgrad) {
+    const int fc = f * C, real = f * fc;
     for (int64_t idx = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; idx < total;
          idx += (int64_t)gridDim.x * blockDim.x) {
-        int k, tap, ch;
+        int k, tap, ch, uu = 0, vv = 0;
         if (!dgrad) {
             const int row = Dr * Ds * Cs;
-            k = (int)(idx / row);
-            const int rem = (int)(idx - (int64_t)k * row);
+            const int orow = (int)(idx / row);
+            const int rem = (int)(idx - (int64_t)orow * row);
             tap = rem / Cs; ch = rem - tap * Cs;
+            const int uv = orow / K;
+            k = orow - uv * K; uu = uv / u; vv = uv - uu * u;
         } else {
             const int row = Dr * Ds * K;
             ch = (int)(idx / row);
@@ -419,9 +422,9 @@ __global__ void s2d_filter_kernel(const T* __restrict__ w, T* __restrict__ out, 
         T v = from_f<T>(0.f);
         if (ch < real) {
             const int d = tap / Ds, e = tap - d * Ds;
-            const int a = ch / stc, b = (ch - a * stc) / C, c = ch - a * stc - b * C;
-            const int r = st * d + a, s = st * e + b;
-            if (r < R && s < S) v = w[(((int64_t)k * R + r) * S + s) * C + c];
+            const int a = ch / fc, b = (ch - a * fc) / C, c = ch - a * fc - b * C;
+            const int r = f * d + a - st * uu, s = f * e + b - st * vv;
+            if (r >= 0 && r < R && s >= 0 && s < S) v = w[(((int64_t)k * R + r) * S + s) * C + c];
         }
         out[idx] = v;
     }
@@ -561,31 +564,32 @@ int launch_wg_output(const Geom& g, bool dgrad, int32_t b, float alpha, const fl
     return (int)cudaGetLastError();
 }
 
-int launch_s2d_input(const Geom& g, int32_t b, int I, int J, int Cs, const void* x, void* xs, cudaStream_t st) {
+int launch_s2d_input(const Geom& g, int32_t b, int f, int I, int J, int Cs, const void* x, void* xs, cudaStream_t st) {
     const int V = 16 / elt_size(g.math);
     const int64_t chunks = (int64_t)b * I * J * (Cs / V);
     if (chunks >= (1LL << 31) || (int64_t)g.h * g.w * g.c >= (1LL << 31)) return (int)cudaErrorInvalidValue;
     const int grid = grid_for(chunks, 256);
     if (g.math == MUCU_MATH_BF16)
         s2d_input_kernel<__nv_bfloat16><<<grid, 256, 0, st>>>((const __nv_bfloat16*)x, (__nv_bfloat16*)xs, (int)chunks,
-                                                              g.h, g.w, g.c, I, J, g.stride, g.pad, Cs);
+                                                              g.h, g.w, g.c, I, J, f, g.pad, Cs);
     else
         s2d_input_kernel<float><<<grid, 256, 0, st>>>((const float*)x, (float*)xs, (int)chunks, g.h, g.w, g.c, I, J,
-                                                      g.stride, g.pad, Cs);
+                                                      f, g.pad, Cs);
     count_launch();
     return (int)cudaGetLastError();
 }
 
-int launch_s2d_filter(const Geom& g, bool dgrad, int Cs, const void* w, void* out, cudaStream_t st) {
-    const int Dr = (g.r + g.stride - 1) / g.stride, Ds = (g.s + g.stride - 1) / g.stride;
-    const int64_t total = dgrad ? (int64_t)g.stride * g.stride * g.c * Dr * Ds * g.k : (int64_t)g.k * Dr * Ds * Cs;
+int launch_s2d_filter(const Geom& g, bool dgrad, const S2d& z, const void* w, void* out, cudaStream_t st) {
+    const int64_t total = dgrad ? (int64_t)g.stride * g.stride * g.c * z.Dr * z.Ds * g.k
+                                : (int64_t)z.u * z.u * g.k * z.Dr * z.Ds * z.Cs;
     const int grid = grid_for(total, 256);
     if (g.math == MUCU_MATH_BF16)
         s2d_filter_kernel<__nv_bfloat16><<<grid, 256, 0, st>>>((const __nv_bfloat16*)w, (__nv_bfloat16*)out, total,
-                                                               g.k, g.r, g.s, g.c, g.stride, Dr, Ds, Cs, dgrad);
+                                                               g.k, g.r, g.s, g.c, g.stride, z.f, z.u, z.Dr, z.Ds,
+                                                               z.Cs, dgrad);
     else
         s2d_filter_kernel<float><<<grid, 256, 0, st>>>((const float*)w, (float*)out, total, g.k, g.r, g.s, g.c,
-                                                       g.stride, Dr, Ds, Cs, dgrad);
+                                                       g.stride, z.f, z.u, z.Dr, z.Ds, z.Cs, dgrad);
     count_launch();
     return (int)cudaGetLastError();
 }

@@ -205,6 +205,8 @@ struct TcArgs {
     // Space-to-depth layers (EPI_D2S / EPI_WGRAD_S2D): the real stride, C, R, S
     // (the GEMM itself runs on the stride-1 super-pixel geometry).
     int s2_st, s2_C, s2_R, s2_S;
+    // EPI_D2S output tensor [*, e_H, e_W, e_C], written at (s2_st*i + a - e_pad, s2_st*j + b - e_pad)
+    int e_H, e_W, e_C, e_pad;
     // epilogue
     void* out;
     long long ldc;
@@ -556,14 +558,14 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         return err;
     }
     if (algo == MUCU_ALGO_IM2COL_GEMM && s2d_tc(g, type)) {
-        // Space-to-depth (DESIGN.md): the strided small-C layer as a stride-1
-        // Dr x Ds conv over the st x st super-pixel image with Cs channels --
-        // 128-B channel atoms, so TMA im2col feeds it like any other layer.
-        const int st_ = g.stride, Dr = s2d_taps(g.r, st_), Ds = s2d_taps(g.s, st_);
-        const int Cs = s2d_channels(g);
+        // Space-to-depth (DESIGN.md 6.3): the strided small-C layer as a stride-1
+        // Dr x Ds conv over the super-pixel image with Cs channels -- 128-B
+        // channel atoms, so TMA im2col feeds it like any other layer.
+        const S2d z = s2d_geom(g, type);
+        const int st_ = g.stride, Dr = z.Dr, Ds = z.Ds, Cs = z.Cs;
         const int kind = type == MUCU_BWD_DATA ? 4 : 3;
         if (type != MUCU_BWD_FILTER && (ctx->fixed_kind != kind || ctx->fixed_src != in1)) {
-            err = launch_s2d_filter(g, type == MUCU_BWD_DATA, Cs, in1, ws, st);
+            err = launch_s2d_filter(g, type == MUCU_BWD_DATA, z, in1, ws, st);
             if (err) return err;
             ctx->fixed_kind = kind; ctx->fixed_src = in1;
         }
@@ -576,6 +578,7 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
             A.M = b * I * J; A.N = st_ * st_ * g.c; A.num_kb = Kp / KB; A.kred = Kp;
             A.ph_mode = 1; A.ph_H = I; A.ph_W = J; A.ph_i0 = 0; A.ph_j0 = 0;
             A.tapR = Dr; A.tapS = Ds; A.im2col_dgrad = 1; A.gsrc = in0;
+            A.e_H = g.h; A.e_W = g.w; A.e_C = g.c; A.e_pad = g.pad;
             finalize_tiling(L, elt);
             use_mt2(L, num_sms);
             grid2(1);
@@ -587,25 +590,31 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
             A.tma_bytes = 16384 * A.mt + A.BN * 128;
             return LAUNCH(A_TMA_IM2COL, B_TMA_K2, EPI_D2S);
         }
-        const int I = g.p + Dr - 1, J = g.q + Ds - 1;
+        const int I = z.I, J = z.J;
         char* xs = ws + WL.a_off;
-        err = launch_s2d_input(g, b, I, J, Cs, in0, xs, st);
+        err = launch_s2d_input(g, b, z.f, I, J, Cs, in0, xs, st);
         if (err) return err;
-        // the GEMM sees the stride-1, pad-0 geometry over xs
+        // the GEMM sees the stride-1, pad-0 geometry over xs (Pu x Qu output super-pixels)
         A.H = I; A.W = J; A.C = Cs; A.R = Dr; A.S = Ds; A.pad = 0; A.stride = 1; A.tapR = Dr; A.tapS = Ds;
+        A.P = z.Pu; A.Q = z.Qu;
         if (type == MUCU_FWD) {
             const int Kp = Dr * Ds * Cs;
-            A.M = (int)(b * PQ); A.N = g.k; A.ldc = g.k; A.num_kb = Kp / KB; A.kred = Kp; A.gsrc = xs;
+            A.M = b * z.Pu * z.Qu; A.N = z.u * z.u * g.k; A.ldc = g.k; A.num_kb = Kp / KB; A.kred = Kp;
+            A.gsrc = xs;
             finalize_tiling(L, elt);
             use_mt2(L, num_sms);
             grid2(1);
             if (!make_im2col_map(&L.ta, elt, xs, Cs, J, I, b, 0, 0, -(Ds - 1), -(Dr - 1), 128, 1, false)) return -1;
-            if (!map2(&L.tb, ws, Kp, g.k, Kp, KB, A.BN)) return -1;
+            if (!map2(&L.tb, ws, Kp, A.N, Kp, KB, A.BN)) return -1;
             A.tma_bytes = 16384 * A.mt + A.BN * 128;
-            return LAUNCH(A_TMA_IM2COL, B_TMA_K2, EPI_STORE);
+            if (z.u == 1) return LAUNCH(A_TMA_IM2COL, B_TMA_K2, EPI_STORE);
+            // u x u output super-pixels: column (uu, vv, k) -> y[n][u*i' + uu][u*j' + vv][k]
+            A.ph_H = z.Pu; A.ph_W = z.Qu; A.s2_st = z.u;
+            A.e_H = g.p; A.e_W = g.q; A.e_C = g.k; A.e_pad = 0;
+            return LAUNCH(A_TMA_IM2COL, B_TMA_K2, EPI_D2S);
         }
-        // WGRAD: dw'[k][(d, e, c')] = sum_m dy[m][k] xs(m; d, e, c'), folded into
-        // dw[k][st*d + a][st*e + b][c] by the epilogue's reductions.
+        // WGRAD (u = 1): dw'[k][(d, e, c')] = sum_m dy[m][k] xs(m; d, e, c'), folded
+        // into dw[k][st*d + a][st*e + b][c] by the epilogue's reductions.
         const int64_t Mpix = (int64_t)b * PQ;
         A.M = g.k; A.N = Dr * Ds * Cs; A.ldc = RSC; A.kred = (int)Mpix; A.gsrc = xs;
         wgrad_tiling(atom, true);

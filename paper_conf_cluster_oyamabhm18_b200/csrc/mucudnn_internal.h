@@ -40,6 +40,13 @@ bool small_c_tc(const Geom& g);    // tensor-core math and C*elt < 16 B (RGB inp
 // s2d_channels = a multiple of 128 B).  DGRAD (no padding: the super-pixel
 // channels are GEMM columns) needs K to be a multiple of 128 B / elt.
 bool s2d_tc(const Geom& g, int type);
+// Space-to-depth geometry (FWD / WGRAD; DGRAD uses u = 1 on the dx grid):
+// input super-pixels of f = st*u pixels, output super-pixels of u x u outputs
+// (u = 2 for stride-2 FWD: N = 4K columns instead of 12 -> 64 padded channels
+// per output pixel), Dr x Ds taps, Cs channels, Pu x Qu output super-pixels,
+// I x J input super-pixels.
+struct S2d { int u, f, Dr, Ds, Cs, Pu, Qu, I, J; };
+S2d s2d_geom(const Geom& g, int type);
 int s2d_channels(const Geom& g);
 inline int s2d_taps(int r, int stride) { return (r + stride - 1) / stride; }
 
@@ -100,8 +107,8 @@ int launch_scale(int64_t n, float beta, float* p, cudaStream_t st);  // p *= bet
 // x[b,H,W,C] -> xp[b,H,W,16/elt] with channels zero-padded to 16 B per pixel.
 int launch_pad_channels(const Geom& g, int32_t b, const void* x, void* xp, cudaStream_t st);
 // Space-to-depth image xs[b][I][J][Cs] and filters (kernels_elem.cu).
-int launch_s2d_input(const Geom& g, int32_t b, int I, int J, int Cs, const void* x, void* xs, cudaStream_t st);
-int launch_s2d_filter(const Geom& g, bool dgrad, int Cs, const void* w, void* out, cudaStream_t st);
+int launch_s2d_input(const Geom& g, int32_t b, int f, int I, int J, int Cs, const void* x, void* xs, cudaStream_t st);
+int launch_s2d_filter(const Geom& g, bool dgrad, const S2d& z, const void* w, void* out, cudaStream_t st);
 int launch_wg_input(const Geom& g, bool dgrad, int32_t b, const void* in, void* V, cudaStream_t st);
 int launch_wg_output(const Geom& g, bool dgrad, int32_t b, float alpha, const float* M, float beta,
                      void* out, cudaStream_t st);

@@ -690,13 +690,38 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                     // by (W - st)*C between blocks (no per-column index arithmetic).
                     const int hw = p.ph_H * p.ph_W;
                     const int n = m / hw, rem = m - n * hw, ii = rem / p.ph_W, jj = rem - ii * p.ph_W;
-                    const int h0 = p.s2_st * ii - p.pad, w0 = p.s2_st * jj - p.pad;
-                    const int stc = p.s2_st * p.C;
-                    int a = nb / stc, bq = (nb - a * stc) / p.C, c = nb - a * stc - bq * p.C;
-                    long long off = (((long long)n * p.H + h0 + a) * p.W + w0 + bq) * p.C + c;
-                    const long long jump = (long long)(p.W - p.s2_st) * p.C;
-                    bool okh = (unsigned)(h0 + a) < (unsigned)p.H, okw = (unsigned)(w0 + bq) < (unsigned)p.W;
+                    const int h0 = p.s2_st * ii - p.e_pad, w0 = p.s2_st * jj - p.e_pad;
+                    const int stc = p.s2_st * p.e_C;
+                    int a = nb / stc, bq = (nb - a * stc) / p.e_C, c = nb - a * stc - bq * p.e_C;
+                    long long off = (((long long)n * p.e_H + h0 + a) * p.e_W + w0 + bq) * p.e_C + c;
+                    const long long jump = (long long)(p.e_W - p.s2_st) * p.e_C;
+                    bool okh = (unsigned)(h0 + a) < (unsigned)p.e_H, okw = (unsigned)(w0 + bq) < (unsigned)p.e_W;
                     const int nlim = p.N - nb;
+                    if (p.e_C % 32 == 0 && p.beta == 0.f) {
+                        // the 32 columns are 32 consecutive channels of one output pixel
+                        // (u x u FWD super-pixels): 16-B vector stores
+                        if (nlim >= 32 && okh && okw) {
+                            if (p.out_bf16) {
+                                __nv_bfloat16* d = (__nv_bfloat16*)p.out + off;
+#pragma unroll
+                                for (int j = 0; j < 32; j += 8) {
+                                    __align__(16) __nv_bfloat16 tmp[8];
+#pragma unroll
+                                    for (int u = 0; u < 8; ++u)
+                                        tmp[u] = __float2bfloat16_rn(p.alpha * __uint_as_float(v[j + u]));
+                                    *reinterpret_cast<uint4*>(d + j) = *reinterpret_cast<uint4*>(tmp);
+                                }
+                            } else {
+                                float* d = (float*)p.out + off;
+#pragma unroll
+                                for (int j = 0; j < 32; j += 4)
+                                    *reinterpret_cast<float4*>(d + j) =
+                                        make_float4(p.alpha * __uint_as_float(v[j]), p.alpha * __uint_as_float(v[j + 1]),
+                                                    p.alpha * __uint_as_float(v[j + 2]), p.alpha * __uint_as_float(v[j + 3]));
+                            }
+                        }
+                        continue;
+                    }
 #pragma unroll
                     for (int j = 0; j < 32; ++j) {
                         if (j < nlim && okh && okw) {
@@ -712,13 +737,13 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                             }
                         }
                         ++off;
-                        if (++c == p.C) {
+                        if (++c == p.e_C) {
                             c = 0;
                             if (++bq == p.s2_st) {
                                 bq = 0; ++a; off += jump;
-                                okh = (unsigned)(h0 + a) < (unsigned)p.H;
+                                okh = (unsigned)(h0 + a) < (unsigned)p.e_H;
                             }
-                            okw = (unsigned)(w0 + bq) < (unsigned)p.W;
+                            okw = (unsigned)(w0 + bq) < (unsigned)p.e_W;
                         }
                     }
                 } else if constexpr (EPI == EPI_WGRAD_S2D) {

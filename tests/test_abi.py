@@ -107,11 +107,13 @@ def test_workspace_space_to_depth():
     assert mu.workspace_size(d, mu.FWD, mu.IM2COL_GEMM, 2) == a256(64 * 9 * 64 * 4) + a256(2 * xs)
     assert mu.workspace_size(d, mu.BWD_FILTER, mu.IM2COL_GEMM, 3) == a256(3 * xs)
     assert mu.workspace_size(d, mu.BWD_DATA, mu.IM2COL_GEMM, 4) == a256(48 * 9 * 64 * 4)
-    # ResNet conv1 BF16: Dr = 4, Cs = 12 -> 64 (BF16 atom); DGRAD (no channel padding) uses the
-    # st*st*C x Dr*Ds*K filter
+    # ResNet conv1 BF16 (stride 2): FWD uses 2 x 2 output super-pixels over 4 x 4 input ones
+    # (u = 2, f = 4): Dr = (2*1 + 7 - 1) // 4 + 1 = 3, Cs = 48 -> 64, 56 x 56 output super-pixels,
+    # 58 x 58 input super-pixels, filter 4K x 9 x 64.  WGRAD keeps u = 1 (f = 2, Dr = 4, Cs = 12 -> 64,
+    # 115 x 115); DGRAD (no channel padding) uses the st*st*C x Dr*Ds*K filter.
     d = mu.desc(2, 3, 224, 224, 64, 7, 7, 3, 2, mu.MATH_BF16)
-    xs = 115 * 115 * 64 * 2
-    assert mu.workspace_size(d, mu.FWD, mu.IM2COL_GEMM, 2) == a256(64 * 16 * 64 * 2) + a256(2 * xs)
+    assert mu.workspace_size(d, mu.FWD, mu.IM2COL_GEMM, 2) == a256(4 * 64 * 9 * 64 * 2) + a256(2 * 58 * 58 * 64 * 2)
+    assert mu.workspace_size(d, mu.BWD_FILTER, mu.IM2COL_GEMM, 2) == a256(2 * 115 * 115 * 64 * 2)
     assert mu.workspace_size(d, mu.BWD_DATA, mu.IM2COL_GEMM, 2) == a256(12 * 16 * 64 * 2)
     # stride 1 keeps the channel-padded image (16 B per pixel)
     d = mu.desc(2, 3, 32, 32, 64, 3, 3, 1, 1, mu.MATH_BF16)

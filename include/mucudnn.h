@@ -129,12 +129,15 @@ mucu_status_t mucu_output_dims(const mucu_conv_desc_t* desc, int32_t* p, int32_t
  *   I2C DGRAD:        b*P*Q*ceil_4(R*S*C)*4 (fp32 dcol)  (+ filter copy as above, or with rows of
  *                     128 B when R*S*C < 128/elt on tensor cores); 0 for 1x1/s1/p0
  *   I2C, TF32/BF16, stride st > 1 and C*elt < 16 ("space-to-depth"):
- *                     u = 2 for FWD with st = 2, else 1; f = st*u;
- *                     Dr = (st*(u-1) + R - 1)/f + 1, Ds likewise, Cs = f*f*C rounded up to 128/elt,
- *                     Pu = ceil(P/u), Qu = ceil(Q/u)
- *                     FWD:   u*u*K*Dr*Ds*Cs*elt + b*(Pu+Dr-1)*(Qu+Ds-1)*Cs*elt
- *                     WGRAD: b*(P+Dr-1)*(Q+Ds-1)*Cs*elt
- *                     DGRAD (when K % (128/elt) == 0, st*st*C <= 256): st*st*C*Dr*Ds*K*elt
+ *                     FWD: u = 2, f = st*u, Dr = (st*(u-1) + R - 1)/f + 1, Ds likewise,
+ *                          Cs = f*f*C rounded up to 128/elt, Pu = ceil(P/u), Qu = ceil(Q/u):
+ *                          u*u*K*Dr*Ds*Cs*elt + b*(Pu+Dr-1)*(Qu+Ds-1)*Cs*elt
+ *                     WGRAD with C <= 4 and st*16 % 16 == 0 (BF16: st even) ("window"):
+ *                          b*H*Wp*4*elt, tpa = 32/elt taps per 128-B atom, na = ceil(S/tpa),
+ *                          Wp = max(st*(Q-1) + na*tpa, W + pad) rounded up to 4
+ *                     WGRAD otherwise (u = 1, f = st): b*(P+Dr-1)*(Q+Ds-1)*Cs*elt
+ *                     DGRAD (when K % (128/elt) == 0, st*st*C <= 256): u = 2 if (2*st)^2*C <= 256
+ *                          else 1, f = st*u, Dr = ceil(R/st) - 1 + u, Ds likewise: f*f*C*Dr*Ds*K*elt
  *   WG  FWD:          16*K*C*elt + 16*b*T*C*elt + 16*b*T*K*4,   T = ceil(P/2)*ceil(Q/2)
  *   WG  DGRAD:        16*C*K*elt + 16*b*T'*K*elt + 16*b*T'*C*4, T' = ceil(H/2)*ceil(W/2)
  * ceil_e rounds up to a multiple of 16/elt elements.  UNSUPPORTED if the

@@ -64,12 +64,33 @@ int s2d_channels(const Geom& g) {
 S2d s2d_geom(const Geom& g, int type) {
     S2d z;
     const int st = g.stride;
-    z.u = (type == MUCU_FWD && st == 2) ? 2 : 1;
+    const int atom = 128 / elt_size(g.math);
+    if (type == MUCU_BWD_DATA) {
+        // dx super-pixels of f = st*u rows/cols; dx row f*i + a' - pad takes dy rows
+        // p = u*i + u-1-d (d < Dr = ceil(R/st) - 1 + u) through filter row
+        // r = st*d + a' - st*(u-1).  u = 2 when f*f*C stays <= 256 GEMM columns.
+        static const char* e = getenv("MUCU_S2D_UD");
+        z.u = e ? atoi(e) : 2;
+        while (z.u > 1 && st * z.u * st * z.u * g.c > 256) --z.u;
+        z.f = st * z.u;
+        z.Dr = (g.r - 1) / st + z.u;
+        z.Ds = (g.s - 1) / st + z.u;
+        z.Cs = 0;
+        z.I = (g.h - 1 + g.pad) / z.f + 1;
+        z.J = (g.w - 1 + g.pad) / z.f + 1;
+        z.Pu = z.Qu = 0;
+        return z;
+    }
+    // FWD / WGRAD: output super-pixels of u x u (u = 2 for FWD: N = 4K columns)
+    z.u = type == MUCU_FWD ? 2 : 1;
+    if (type == MUCU_FWD) {
+        static const char* e = getenv("MUCU_S2D_U");  // experiments: output super-pixel factor
+        if (e) z.u = atoi(e);
+    }
     z.f = st * z.u;
     // output row u*i' + uu reads input rows f*(i' + d) + a - pad with st*uu + r = f*d + a
     z.Dr = (st * (z.u - 1) + g.r - 1) / z.f + 1;
     z.Ds = (st * (z.u - 1) + g.s - 1) / z.f + 1;
-    const int atom = 128 / elt_size(g.math);
     z.Cs = (int)align_up((uint64_t)z.f * z.f * g.c, (uint64_t)atom);
     z.Pu = (g.p + z.u - 1) / z.u;
     z.Qu = (g.q + z.u - 1) / z.u;
@@ -81,9 +102,29 @@ S2d s2d_geom(const Geom& g, int type) {
 bool s2d_tc(const Geom& g, int type) {
     if (!small_c_tc(g) || g.stride < 2) return false;
     if (type == MUCU_BWD_DATA) return g.k % (128 / elt_size(g.math)) == 0 && g.stride * g.stride * g.c <= 256;
+    // (DGRAD: s2d_geom picks the largest u <= 2 with (st*u)^2 * C <= 256 columns)
     // even 12 -> 64 padded channels (ResNet conv1, BF16) run ~5-8x faster on
     // the TMA-fed space-to-depth GEMM than on the 16-B tap gathers
     return true;
+}
+
+bool win_tc(const Geom& g, int type) {
+    static const int enabled = getenv("MUCU_WIN") ? atoi(getenv("MUCU_WIN")) : 1;
+    const int elt = elt_size(g.math);
+    return enabled && type == MUCU_BWD_FILTER && small_c_tc(g) && g.stride >= 2 && g.c <= 4 &&
+           (g.stride * 4 * elt) % 16 == 0;
+}
+
+Win win_geom(const Geom& g) {
+    Win z;
+    const int elt = elt_size(g.math);
+    z.cpx = 4;
+    z.tpa = 128 / elt / z.cpx;
+    z.na = (g.s + z.tpa - 1) / z.tpa;
+    // every window read stays inside its row: st*(Q-1) + na*tpa <= Wp
+    z.Wp = (int)align_up((uint64_t)std::max(g.stride * (g.q - 1) + z.na * z.tpa, g.w + g.pad), 4);
+    z.M = g.r * z.na * (128 / elt);
+    return z;
 }
 
 bool algo_eligible(const Geom& g, int type, int algo) {
@@ -113,13 +154,21 @@ mucu_status_t ws_layout(const Geom& g, int type, int algo, int32_t b, WsLayout* 
     if (algo == MUCU_ALGO_IM2COL_GEMM) {
         L->kpitch = (int32_t)align_up(RSC, vec);
         if (is_pointwise(g)) { L->kpitch = g.c; return MUCU_OK; }
+        if (win_tc(g, type)) {
+            const Win z = win_geom(g);
+            L->a_off = 0;
+            L->a_bytes = align_up((uint64_t)b * g.h * z.Wp * z.cpx * elt, 256);
+            L->kpitch = z.cpx;
+            L->total = L->a_bytes;
+            return MUCU_OK;
+        }
         if (s2d_tc(g, type)) {
             // Space-to-depth: FWD = [s2d filter K x Dr*Ds*Cs][xs b x I x J x Cs],
             // WGRAD = [xs], DGRAD = [s2d filter st*st*C x Dr*Ds*K] (b-independent).
             const S2d z = s2d_geom(g, type);
             const uint64_t Dr = z.Dr, Ds = z.Ds, Cs = z.Cs;
             if (type == MUCU_BWD_DATA) {
-                L->fixed_bytes = align_up((uint64_t)g.stride * g.stride * g.c * Dr * Ds * g.k * elt, 256);
+                L->fixed_bytes = align_up((uint64_t)z.f * z.f * g.c * Dr * Ds * g.k * elt, 256);
             } else {
                 if (type == MUCU_FWD)
                     L->fixed_bytes = align_up((uint64_t)z.u * z.u * g.k * Dr * Ds * Cs * elt, 256);

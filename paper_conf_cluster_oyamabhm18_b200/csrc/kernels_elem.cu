@@ -396,8 +396,8 @@ __global__ void s2d_input_kernel(const T* __restrict__ x, T* __restrict__ xs, in
 // Space-to-depth filter.  FWD (K-major B of the stride-1 conv on xs, output
 // super-pixels of u x u outputs; input super-pixels of f = st*u pixels):
 //   out[(uu*u + vv)*K + k][(d*Ds + e)*Cs + (a*f + b)*C + c] = w[k][f*d + a - st*uu][f*e + b - st*vv][c]
-// DGRAD (u = 1, f = st; K-major B of the transposed conv, N = st*st*C columns of dx):
-//   out[(a*st + b)*C + c][(d*Ds + e)*K + k] = w[k][st*d + a][st*e + b][c]
+// DGRAD (dx super-pixels of f = st*u; K-major B of the transposed conv, N = f*f*C columns of dx):
+//   out[(a*f + b)*C + c][(d*Ds + e)*K + k] = w[k][st*d + a - st*(u-1)][st*e + b - st*(u-1)][c]
 // Zero where the filter tap falls outside R x S, or in the channel padding.
 template <class T>
 __global__ void s2d_filter_kernel(const T* __restrict__ w, T* __restrict__ out, int64_t total, int K, int R, int S,
@@ -423,7 +423,8 @@ __global__ void s2d_filter_kernel(const T* __restrict__ w, T* __restrict__ out, 
         if (ch < real) {
             const int d = tap / Ds, e = tap - d * Ds;
             const int a = ch / fc, b = (ch - a * fc) / C, c = ch - a * fc - b * C;
-            const int r = f * d + a - st * uu, s = f * e + b - st * vv;
+            const int r = dgrad ? st * d + a - st * (u - 1) : f * d + a - st * uu;
+            const int s = dgrad ? st * e + b - st * (u - 1) : f * e + b - st * vv;
             if (r >= 0 && r < R && s >= 0 && s < S) v = w[(((int64_t)k * R + r) * S + s) * C + c];
         }
         out[idx] = v;
@@ -500,6 +501,37 @@ __global__ void pad_channels_kernel(const T* __restrict__ x, T* __restrict__ xp,
 }
 }  // namespace
 
+// xp[n][h][w'][c'] = x[n][h][w' - pad][c'] (zero outside 0 <= w' - pad < W or
+// c' >= C); one 16-B store per thread.
+template <typename T>
+__global__ void win_pad_kernel(const T* __restrict__ x, T* __restrict__ xp, int64_t units, int W, int Wp, int C,
+                               int pad) {
+    constexpr int V = 16 / sizeof(T);  // elements per unit = V / 4 pixels of 4 channels
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < units; i += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t e0 = i * V;
+        const int64_t pix0 = e0 / 4;          // padded pixel index (n, h, w')
+        const int64_t row = pix0 / Wp;        // (n, h)
+        const int w0 = (int)(pix0 - row * Wp);
+        __align__(16) T v[V];
+#pragma unroll
+        for (int u = 0; u < V; ++u) {
+            const int w = w0 + u / 4 - pad, c = u % 4;
+            v[u] = (c < C && w >= 0 && w < W) ? x[(row * W + w) * C + c] : from_f<T>(0.f);
+        }
+        *reinterpret_cast<uint4*>(xp + e0) = *reinterpret_cast<const uint4*>(v);
+    }
+}
+int launch_win_pad(const Geom& g, int32_t b, int Wp, const void* x, void* xp, cudaStream_t st) {
+    const int64_t units = (int64_t)b * g.h * Wp * 4 * elt_size(g.math) / 16;
+    const int grid = grid_for(units, 256);
+    if (g.math == MUCU_MATH_BF16)
+        win_pad_kernel<__nv_bfloat16><<<grid, 256, 0, st>>>((const __nv_bfloat16*)x, (__nv_bfloat16*)xp, units, g.w,
+                                                            Wp, g.c, g.pad);
+    else
+        win_pad_kernel<float><<<grid, 256, 0, st>>>((const float*)x, (float*)xp, units, g.w, Wp, g.c, g.pad);
+    count_launch();
+    return (int)cudaGetLastError();
+}
 int launch_pad_channels(const Geom& g, int32_t b, const void* x, void* xp, cudaStream_t st) {
     const int64_t pixels = (int64_t)b * g.h * g.w;
     const int grid = grid_for(pixels, 256);
@@ -580,7 +612,7 @@ int launch_s2d_input(const Geom& g, int32_t b, int f, int I, int J, int Cs, cons
 }
 
 int launch_s2d_filter(const Geom& g, bool dgrad, const S2d& z, const void* w, void* out, cudaStream_t st) {
-    const int64_t total = dgrad ? (int64_t)g.stride * g.stride * g.c * z.Dr * z.Ds * g.k
+    const int64_t total = dgrad ? (int64_t)z.f * z.f * g.c * z.Dr * z.Ds * g.k
                                 : (int64_t)z.u * z.u * g.k * z.Dr * z.Ds * z.Cs;
     const int grid = grid_for(total, 256);
     if (g.math == MUCU_MATH_BF16)

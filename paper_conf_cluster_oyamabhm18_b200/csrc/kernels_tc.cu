@@ -72,6 +72,13 @@ __device__ __forceinline__ void tma_load_3d(uint32_t dst, const CUtensorMap* tm,
         "l"((uint64_t)tm), "r"(bar), "r"(c0), "r"(c1), "r"(c2)
         : "memory");
 }
+__device__ __forceinline__ void tma_load_4d(uint32_t dst, const CUtensorMap* tm, uint32_t bar, int c0, int c1, int c2,
+                                            int c3) {
+    asm volatile(
+        "cp.async.bulk.tensor.4d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4, %5, %6}], [%2];" ::"r"(dst),
+        "l"((uint64_t)tm), "r"(bar), "r"(c0), "r"(c1), "r"(c2), "r"(c3)
+        : "memory");
+}
 // TMA im2col mode (4-D NHWC tensor {C, W, H, N}): pixelsPerColumn consecutive
 // pixels starting at (w, h, n) (walking W, then H, then N inside the map's
 // bounding box with the map's traversal stride), channelsPerPixel channels
@@ -144,6 +151,8 @@ enum AMode : int {
     A_GATHER_SMALLC_PAD = 9, // same K' layout from a channel-padded copy of x (16 B per pixel): cp.async
     A_TMA_IM2COL_SMALLC = 10, // same K' layout from the padded copy by TMA im2col: one 128-pixel x 16-B box
                               // per tap, SWIZZLE_NONE core matrices (LBO 2 KB between taps, SBO 128 B)
+    A_TMA_WIN = 11,    // WGRAD window operand, MN-major: rows j = (r, atom, tap, c) of the filter, K = pixels;
+                       // one 4-D TMA box per 128-B atom from the overlapping-window view of the padded x
 };
 enum BMode : int {
     B_TMA_K2 = 0,      // dense K-major {K, cols}
@@ -158,12 +167,15 @@ enum BMode : int {
     B_RESIDENT = 9,    // whole (padded) filter staged in smem once per CTA (small-C FWD)
     B_GATHER_SMALLC = 10, // WGRAD small C: x pixels as 16-B tap chunks, MN-major
     B_GATHER_SMALLC_PAD = 11, // WGRAD small C from the channel-padded copy of x: cp.async
+    B_TMA_DYROW = 12,  // WGRAD dy, MN-major, 3-D map {K, Q, b*P}: k-block = KD pixels of one output row
 };
 // EPI_D2S: DGRAD on the space-to-depth grid -- row (n, i, j), column
 //   (a, b, c) -> dx[n][st*i + a - pad][st*j + b - pad][c] (out-of-image skipped).
 // EPI_WGRAD_S2D: column (d, e, (a, b, c')) of the space-to-depth filter ->
 //   dw[k][st*d + a][st*e + b][c'] (padding and r >= R / s >= S skipped), reduced.
-enum EpiMode : int { EPI_STORE = 0, EPI_WGRAD_CHAIN = 1, EPI_WGRAD_SMALLC = 2, EPI_D2S = 3, EPI_WGRAD_S2D = 4 };
+// EPI_WGRAD_WIN: row j = (r, atom, tap, c) of the window GEMM -> dw[k][r][atom*taps + tap][c], reduced.
+enum EpiMode : int { EPI_STORE = 0, EPI_WGRAD_CHAIN = 1, EPI_WGRAD_SMALLC = 2, EPI_D2S = 3, EPI_WGRAD_S2D = 4,
+                     EPI_WGRAD_WIN = 5 };
 
 struct TcArgs {
     int M, N;                // output rows / cols
@@ -194,6 +206,7 @@ struct TcArgs {
     // (ph_H x ph_W) sub-grid.  tapR/tapS = R/S when not in phase mode.
     int ph_mode, ph_H, ph_W, ph_i0, ph_j0, ph_r0, ph_s0, ph_hb, ph_wb;
     int tapR, tapS;
+    int ph_u;                // phase mode: im2col positions advance by ph_u per sub-grid pixel (1 except s2d DGRAD)
     // Small-C layers: K' = (r, s8, c') with taps grouped by 8 per k-block and
     // channels zero-padded to cp = 16 B / elt; s8 = S rounded up to 8.
     int cp, s8;
@@ -207,6 +220,8 @@ struct TcArgs {
     int s2_st, s2_C, s2_R, s2_S;
     // EPI_D2S output tensor [*, e_H, e_W, e_C], written at (s2_st*i + a - e_pad, s2_st*j + b - e_pad)
     int e_H, e_W, e_C, e_pad;
+    // Window WGRAD (A_TMA_WIN / B_TMA_DYROW): 128-B atoms per filter row, q-blocks per output row
+    int win_na, win_qb;
     // epilogue
     void* out;
     long long ldc;
@@ -288,15 +303,15 @@ EncodeTiledFn get_encode() {
     return fn;
 }
 
-// Tensor map over a row-major tensor with up to 3 dims (dims[0] contiguous).
+// Tensor map over a row-major tensor with up to 4 dims (dims[0] contiguous).
 bool make_map(CUtensorMap* tm, int elt, const void* base, int rank, const uint64_t* dims, const uint64_t* strides_bytes,
               const uint32_t* box, bool mn_major = false) {
     // 32-bit MN-major operands need the 32-B-atom swizzle matching SWIZZLE_128B_BASE32B.
     const CUtensorMapSwizzle sw = (mn_major && elt == 4) ? CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B : CU_TENSOR_MAP_SWIZZLE_128B;
     EncodeTiledFn enc = get_encode();
     if (!enc) return false;
-    cuuint64_t d[3], s[2];
-    cuuint32_t b[3], e[3] = {1, 1, 1};
+    cuuint64_t d[4], s[3];
+    cuuint32_t b[4], e[4] = {1, 1, 1, 1};
     for (int i = 0; i < rank; ++i) { d[i] = dims[i]; b[i] = box[i]; }
     for (int i = 0; i < rank - 1; ++i) s[i] = strides_bytes[i];
     CUresult r = enc(tm, elt == 2 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32, rank,
@@ -455,7 +470,7 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
     A.km = 1;
     A.H = g.h; A.W = g.w; A.C = g.c; A.P = g.p; A.Q = g.q; A.R = g.r; A.S = g.s; A.pad = g.pad;
     A.stride = g.stride; A.K = g.k;
-    A.tapR = g.r; A.tapS = g.s;
+    A.tapR = g.r; A.tapS = g.s; A.ph_u = 1;
     A.max_lag = std::min(6, std::max(1, env_int("MUCU_MAX_LAG", 6)));
     A.debug = env_int("MUCU_TC_DEBUG", 0);
     A.alpha = alpha; A.beta = beta; A.out = out; A.out_bf16 = bf ? 1 : 0; A.sem = sem.sem;
@@ -484,8 +499,9 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
     // TMA-only operands (tma = true) also take 256-row tiles and stages of
     // km k-blocks: fewer, larger TMA transactions (the TMA issue rate, not
     // bytes, bounds these MN-major loads), as deep as two stages allow.
-    auto wgrad_tiling = [&](int step, bool tma) {
-        A.mt = (tma && A.M > 128 && (A.M <= 256 || A.M % 256 == 0) && env_int("MUCU_MT2", 1)) ? 2 : 1;
+    auto wgrad_tiling = [&](int step, bool tma, int qrow = 0) {
+        A.mt = (tma && A.M > 128 && (A.M <= 256 || A.M % 256 == 0 || (qrow && A.M % 256 > 128)) &&
+                env_int("MUCU_MT2", 1)) ? 2 : 1;
         // 256-row tiles keep BN <= 128 so that two stages of two k-blocks fit
         // (measured: km = 2 beats BN = 256 with km = 1 on every AlexNet/ResNet layer)
         A.BN = pick_bn(A.N, step, 128 * A.mt, A.mt == 2 ? std::max(128, step) : 256);
@@ -495,12 +511,16 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         A.km = 1;
         if (tma) {
             const int base = A.mt * 128 * 128 + A.b_bytes;
-            while (A.km < 4 && 2 * (2 * A.km) * base <= 200 * 1024 && KB * 2 * A.km <= 256) A.km *= 2;
+            while (A.km < 4 && 2 * (2 * A.km) * base <= 200 * 1024 && KB * 2 * A.km <= 256 &&
+                   (qrow == 0 || KB * 2 * A.km <= (int)align_up((uint64_t)qrow, (uint64_t)KB)))
+                A.km *= 2;
             if (const int km = env_int("MUCU_KM", 0)) A.km = km;
         }
         size_stages(A);
         const int64_t tiles = ceil_div(A.N, A.BN) * ceil_div(A.M, 128 * A.mt);
-        const int64_t nkb = ceil_div(A.kred, KB * A.km);
+        // qrow > 0: k-blocks are KD-pixel pieces of output rows of qrow pixels (window WGRAD)
+        if (qrow) A.win_qb = (int)ceil_div(qrow, KB * A.km);
+        const int64_t nkb = qrow ? (int64_t)b * g.p * A.win_qb : ceil_div(A.kred, KB * A.km);
         int64_t nsplit = std::min<int64_t>(std::min<int64_t>(std::max<int64_t>(1, (2LL * num_sms) / tiles),
                                                              std::max<int64_t>(1, nkb / 16)), 65535);
         A.kb_per_split = (int)ceil_div(nkb, nsplit);
@@ -557,6 +577,29 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         }
         return err;
     }
+    if (algo == MUCU_ALGO_IM2COL_GEMM && win_tc(g, type)) {
+        // Window WGRAD: dw^T[j][k] = sum over pixels of window(j, m) dy(m, k),
+        // rows j = (r, atom, tap, c) over the padded copy xp, columns = the K filters.
+        const Win z = win_geom(g);
+        char* xp = ws + WL.a_off;
+        err = launch_win_pad(g, b, z.Wp, in0, xp, st);
+        if (err) return err;
+        A.M = z.M; A.N = g.k; A.ldc = RSC; A.kred = (int)(b * PQ); A.cp = z.cpx; A.win_na = z.na;
+        wgrad_tiling(atom, true, g.q);
+        if (beta != 1.f) {
+            err = launch_scale(g.k * RSC, beta, (float*)out, st);
+            if (err) return err;
+        }
+        const int KD = KB * A.km;
+        const uint64_t pb = (uint64_t)z.cpx * elt;
+        uint64_t adims[4] = {(uint64_t)z.na * atom, (uint64_t)g.q, (uint64_t)g.h, (uint64_t)b};
+        uint64_t astr[3] = {g.stride * pb, z.Wp * pb, (uint64_t)g.h * z.Wp * pb};
+        uint32_t abox[4] = {(uint32_t)atom, (uint32_t)KD, 1, 1};
+        if (!make_map(&L.ta, elt, xp, 4, adims, astr, abox, true)) return -1;
+        if (!map3(&L.tb, in1, g.k, g.q, (uint64_t)b * g.p, g.k, (uint64_t)g.q * g.k, atom, KD, 1, true)) return -1;
+        A.tma_bytes = A.km * (A.mt * 128 * KB * elt + A.bn_atoms * KB * 128);
+        return LAUNCH(A_TMA_WIN, B_TMA_DYROW, EPI_WGRAD_WIN);
+    }
     if (algo == MUCU_ALGO_IM2COL_GEMM && s2d_tc(g, type)) {
         // Space-to-depth: the strided small-C layer as a stride-1
         // Dr x Ds conv over the super-pixel image with Cs channels -- 128-B
@@ -571,20 +614,26 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         }
         A.s2_st = st_; A.s2_C = g.c; A.s2_R = g.r; A.s2_S = g.s;
         if (type == MUCU_BWD_DATA) {
-            // dx in super-pixels: i = (h + pad) / st, a = (h + pad) % st; dy row
-            // p = i - d pairs with filter row r = st*d + a (d < Dr).
-            const int I = (g.h - 1 + g.pad) / st_ + 1, J = (g.w - 1 + g.pad) / st_ + 1;
+            // dx in f x f super-pixels (f = st*u, s2d_geom): super-pixel (i, j) takes dy
+            // pixels (u*i + u-1-d, u*j + u-1-e), d < Dr, e < Ds -- a TMA im2col walk with
+            // traversal stride u and flipped taps; the depth-to-space epilogue writes
+            // dx[n][f*i + a' - pad][f*j + b' - pad][c] for column (a', b', c).
+            const int I = z.I, J = z.J, f = z.f, u = z.u;
             const int Kp = Dr * Ds * g.k;
-            A.M = b * I * J; A.N = st_ * st_ * g.c; A.num_kb = Kp / KB; A.kred = Kp;
+            A.s2_st = f;
+            A.M = b * I * J; A.N = f * f * g.c; A.num_kb = Kp / KB; A.kred = Kp;
             A.ph_mode = 1; A.ph_H = I; A.ph_W = J; A.ph_i0 = 0; A.ph_j0 = 0;
-            A.tapR = Dr; A.tapS = Ds; A.im2col_dgrad = 1; A.gsrc = in0;
+            A.tapR = Dr; A.tapS = Ds; A.im2col_dgrad = 1; A.gsrc = in0; A.ph_u = u;
             A.e_H = g.h; A.e_W = g.w; A.e_C = g.c; A.e_pad = g.pad;
             finalize_tiling(L, elt);
             use_mt2(L, num_sms);
             grid2(1);
-            const int lw = -(Ds - 1), lh = -(Dr - 1);
-            if (!make_im2col_map(&L.ta, elt, in0, g.k, g.q, g.p, b, lw, lh, lw + J - g.q, lh + I - g.p, 128, 1,
-                                 false))
+            // start pixel of super-pixel (i, j): (u*i - (Dr - u), u*j - (Ds - u)); the kernel's
+            // phase-mode origin is ph_i0 + ii - (tapR - 1) in map units, so the map walks u-strided
+            // positions lw, lw + u, ... with J of them per row.
+            const int lw = -(Ds - u), lh = -(Dr - u);
+            if (!make_im2col_map(&L.ta, elt, in0, g.k, g.q, g.p, b, lw, lh, lw + u * (J - 1) - (g.q - 1),
+                                 lh + u * (I - 1) - (g.p - 1), 128, u, false))
                 return -1;
             if (!map2(&L.tb, ws, Kp, A.N, Kp, KB, A.BN)) return -1;
             A.tma_bytes = 16384 * A.mt + A.BN * 128;

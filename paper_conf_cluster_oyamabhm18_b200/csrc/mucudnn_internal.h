@@ -49,6 +49,15 @@ struct S2d { int u, f, Dr, Ds, Cs, Pu, Qu, I, J; };
 S2d s2d_geom(const Geom& g, int type);
 int s2d_channels(const Geom& g);
 inline int s2d_taps(int r, int stride) { return (r + stride - 1) / stride; }
+// Window WGRAD (strided small-C layers, I2C algorithm): x copied
+// to xp[b][H][Wp][4] (channels zero-padded to 4, `pad` zero columns on the
+// left, zeros up to Wp on the right).  GEMM row j = (r, atom, tap, c) of output
+// pixel (n,p,q) reads xp[n][st*p + r - pad][st*q + atom*tpa + tap][c]: one
+// 128-B window per (pixel, filter row, atom), windows starting st pixels
+// apart -- a plain strided view that TMA tiles directly.
+struct Win { int cpx, tpa, na, Wp, M; };
+bool win_tc(const Geom& g, int type);
+Win win_geom(const Geom& g);
 
 // Workspace layout of one micro-configuration (all offsets 256-B aligned).
 // `fixed` = b-independent prefix (padded filter / Winograd U) computed once per
@@ -108,6 +117,7 @@ int launch_scale(int64_t n, float beta, float* p, cudaStream_t st);  // p *= bet
 int launch_pad_channels(const Geom& g, int32_t b, const void* x, void* xp, cudaStream_t st);
 // Space-to-depth image xs[b][I][J][Cs] and filters (kernels_elem.cu).
 int launch_s2d_input(const Geom& g, int32_t b, int f, int I, int J, int Cs, const void* x, void* xs, cudaStream_t st);
+int launch_win_pad(const Geom& g, int32_t b, int Wp, const void* x, void* xp, cudaStream_t st);
 int launch_s2d_filter(const Geom& g, bool dgrad, const S2d& z, const void* w, void* out, cudaStream_t st);
 int launch_wg_input(const Geom& g, bool dgrad, int32_t b, const void* in, void* V, cudaStream_t st);
 int launch_wg_output(const Geom& g, bool dgrad, int32_t b, float alpha, const float* M, float beta,

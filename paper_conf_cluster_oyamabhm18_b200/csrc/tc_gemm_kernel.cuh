@@ -23,18 +23,19 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
     const int A_HALF = 128 * 128 * p.km;
     const int A_BYTES = p.mt * A_HALF;
     const int KD = KB * p.km;                // K rows per stage (MN-major modes)
-    constexpr bool A_MN = (AM == A_TMA_MN2);
+    constexpr bool A_MN = (AM == A_TMA_MN2 || AM == A_TMA_WIN);
     constexpr bool B_MN = (BM_ == B_TMA_MN2 || BM_ == B_TMA_MN3 || BM_ == B_GATHER_WG || BM_ == B_SCALAR_DGRAD ||
                            BM_ == B_SCALAR_WG || BM_ == B_TMA_IM2COL || BM_ == B_GATHER_SMALLC ||
-                           BM_ == B_GATHER_SMALLC_PAD);
+                           BM_ == B_GATHER_SMALLC_PAD || BM_ == B_TMA_DYROW);
     constexpr bool A_TMA = (AM == A_TMA_K2 || AM == A_TMA_K3 || AM == A_TMA_MN2 || AM == A_TMA_IM2COL ||
-                            AM == A_TMA_IM2COL_SMALLC);
+                            AM == A_TMA_IM2COL_SMALLC || AM == A_TMA_WIN);
     constexpr bool A_NOSWZ = (AM == A_TMA_IM2COL_SMALLC);  // unswizzled core matrices, one 2-KB box per tap
     constexpr bool B_TMA = (BM_ == B_TMA_K2 || BM_ == B_TMA_K3 || BM_ == B_TMA_MN2 || BM_ == B_TMA_MN3 ||
-                            BM_ == B_TMA_IM2COL);
+                            BM_ == B_TMA_IM2COL || BM_ == B_TMA_DYROW);
     constexpr bool B_RES = (BM_ == B_RESIDENT);
     constexpr bool GATHER = !A_TMA || (!B_TMA && !B_RES);
-    constexpr bool SPLITK = (EPI == EPI_WGRAD_CHAIN || EPI == EPI_WGRAD_SMALLC || EPI == EPI_WGRAD_S2D);
+    constexpr bool SPLITK = (EPI == EPI_WGRAD_CHAIN || EPI == EPI_WGRAD_SMALLC || EPI == EPI_WGRAD_S2D ||
+                             EPI == EPI_WGRAD_WIN);
     constexpr bool A_ASYNC = (AM == A_GATHER_FWD || AM == A_GATHER_DGRAD || AM == A_GATHER_SMALLC_PAD);
     constexpr bool B_ASYNC = (BM_ == B_GATHER_WG || BM_ == B_GATHER_SMALLC_PAD);
     // MN-major atoms: 8-row (bf16, SWIZZLE_128B) or 4-row (tf32, 128B_BASE32B) groups.
@@ -184,7 +185,9 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                     const int hw = p.ph_H * p.ph_W;
                     icn = mH / hw;
                     const int rem = mH - icn * hw, ii = rem / p.ph_W, jj = rem - ii * p.ph_W;
-                    ich = p.ph_i0 + ii - (p.tapR - 1); icw = p.ph_j0 + jj - (p.tapS - 1);
+                    // ph_u > 1 (space-to-depth DGRAD): the map walks u-strided positions
+                    ich = p.ph_u * (p.ph_i0 + ii) + (p.ph_u - 1) - (p.tapR - 1);
+                    icw = p.ph_u * (p.ph_j0 + jj) + (p.ph_u - 1) - (p.tapS - 1);
                 } else if (p.im2col_dgrad) {
                     const int hw = p.H * p.W;
                     icn = mH / hw;
@@ -260,6 +263,9 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                 const int rem = m - wb_n * pq;
                 wb_p = rem / p.Q; wb_q = rem - wb_p * p.Q;
             }
+            // Window WGRAD: k-block kb = (output row n*P + p, q-block qb)
+            int wr_row = 0, wr_qb = 0;
+            if constexpr (AM == A_TMA_WIN) { wr_row = kb_begin / p.win_qb; wr_qb = kb_begin - wr_row * p.win_qb; }
             for (int kb = kb_begin; kb < kb_end; ++kb, ++git, s = (s + 1 == S) ? 0 : s + 1, ph ^= (s == 0) ? 1u : 0u) {
                 mbar_wait(smem_u32(&empty[s]), ph ^ 1u);
                 const uint32_t aT = smem_u32(sA + (size_t)s * A_BYTES);
@@ -291,6 +297,18 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                             for (int a = 0; a < 128 * ELT / 128; ++a)
                                 tma_load_2d(aH + a * KD * 128, &tmA, fb, mH + a * (128 / ELT), kb * KD);
                         }
+                        if constexpr (AM == A_TMA_WIN) {
+                            // atom ja = (filter row r, atom aa): window of KD output pixels of row
+                            // (n, p) at x row st*p + r - pad (rows past R load out of bounds: zeros)
+                            const int n_ = wr_row / p.P, p_ = wr_row - n_ * p.P;
+#pragma unroll
+                            for (int a = 0; a < 128 * ELT / 128; ++a) {
+                                const int ja = mH / (128 / ELT) + a;
+                                const int r = ja / p.win_na, aa = ja - r * p.win_na;
+                                const int h = r < p.R ? p.stride * p_ + r - p.pad : -(1 << 20);
+                                tma_load_4d(aH + a * KD * 128, &tmA, fb, aa * (128 / ELT), wr_qb * KD, h, n_);
+                            }
+                        }
                         if constexpr (AM == A_TMA_IM2COL) {
                             // 128 consecutive output pixels x KB channels of tap (r,s) in one TMA
                             const uint16_t ow = (uint16_t)(p.im2col_dgrad ? p.tapS - 1 - g_s : g_s);
@@ -313,6 +331,10 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                         for (int a = 0; a < p.bn_atoms; ++a)
                             tma_load_3d(bT + a * KB * 128, &tmB, fb, n0 + a * (128 / ELT), rs, k0);
                     }
+                    if constexpr (BM_ == B_TMA_DYROW) {
+                        for (int a = 0; a < p.bn_atoms; ++a)
+                            tma_load_3d(bT + a * KD * 128, &tmB, fb, n0 + a * (128 / ELT), wr_qb * KD, wr_row);
+                    }
                     if constexpr (BM_ == B_TMA_IM2COL) {
                         // atom a = 128 B of channels (c0..) of tap (r,s) for KB pixels
                         const int h0 = wb_p * p.stride - p.pad, w0 = wb_q * p.stride - p.pad;
@@ -325,6 +347,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                         }
                     }
                 }
+                if constexpr (AM == A_TMA_WIN) { if (++wr_qb == p.win_qb) { wr_qb = 0; ++wr_row; } }
                 if constexpr (BM_ == B_TMA_IM2COL) {
                     wb_q += KD;
                     while (wb_q >= p.Q) { wb_q -= p.Q; if (++wb_p == p.P) { wb_p = 0; ++wb_n; } }
@@ -761,6 +784,21 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                                 atomicAdd(drow + (r * p.s2_S + sx) * p.s2_C + c, p.alpha * __uint_as_float(v[j]));
                         }
                         if (++ch == p.C) { ch = 0; ++tap; }
+                    }
+                } else if constexpr (EPI == EPI_WGRAD_WIN) {
+                    // row m = (r, atom aa, tap t, channel c) -> dw[k][r][aa*taps + t][c], k = nb + j
+                    constexpr int per_atom = 128 / ELT;
+                    const int ja = m / per_atom, e = m - ja * per_atom;
+                    const int t = e / p.cp, c = e - t * p.cp;
+                    const int r = ja / p.win_na, sx = (ja - r * p.win_na) * (per_atom / p.cp) + t;
+                    if (r < p.R && sx < p.S && c < p.C) {
+                        float* d = outF + (size_t)nb * p.ldc + (r * p.S + sx) * p.C + c;
+#pragma unroll
+                        for (int j = 0; j < 32; ++j)
+                            if (nb + j < p.N)
+                                asm volatile("red.global.add.f32 [%0], %1;" ::"l"(d + (size_t)j * p.ldc),
+                                             "f"(p.alpha * __uint_as_float(v[j]))
+                                             : "memory");
                     }
                 } else if constexpr (EPI == EPI_WGRAD_SMALLC) {
                     // padded column j' = (r, s8, c') -> dw column (r*S + s)*C + c (skip padding)

@@ -100,21 +100,30 @@ def test_workspace_small_c_tensor_core():
 
 
 def test_workspace_space_to_depth():
-    # AlexNet conv1 on tensor cores: Dr = Ds = ceil(11/4) = 3, Cs = 4*4*3 = 48 -> 64 (TF32 atom 32)
+    # AlexNet conv1 on tensor cores (TF32, stride 4).  FWD: 2 x 2 output super-pixels over
+    # 8 x 8 input ones (u = 2, f = 8): Dr = (4*1 + 11 - 1) // 8 + 1 = 2, Cs = 8*8*3 = 192 (a
+    # multiple of the TF32 atom 32), Pu = 28, 29 x 29 input super-pixels, filter 4K x 4 x 192.
     d = mu.desc(4, 3, 224, 224, 64, 11, 11, 2, 4, mu.MATH_TF32)
     a256 = lambda v: -(-v // 256) * 256  # noqa: E731
-    xs = 57 * 57 * 64 * 4                  # (P + Dr - 1) x (Q + Ds - 1) super-pixels per sample
-    assert mu.workspace_size(d, mu.FWD, mu.IM2COL_GEMM, 2) == a256(64 * 9 * 64 * 4) + a256(2 * xs)
-    assert mu.workspace_size(d, mu.BWD_FILTER, mu.IM2COL_GEMM, 3) == a256(3 * xs)
-    assert mu.workspace_size(d, mu.BWD_DATA, mu.IM2COL_GEMM, 4) == a256(48 * 9 * 64 * 4)
-    # ResNet conv1 BF16 (stride 2): FWD uses 2 x 2 output super-pixels over 4 x 4 input ones
-    # (u = 2, f = 4): Dr = (2*1 + 7 - 1) // 4 + 1 = 3, Cs = 48 -> 64, 56 x 56 output super-pixels,
-    # 58 x 58 input super-pixels, filter 4K x 9 x 64.  WGRAD keeps u = 1 (f = 2, Dr = 4, Cs = 12 -> 64,
-    # 115 x 115); DGRAD (no channel padding) uses the st*st*C x Dr*Ds*K filter.
+    xs = 29 * 29 * 192 * 4
+    assert mu.workspace_size(d, mu.FWD, mu.IM2COL_GEMM, 2) == a256(4 * 64 * 4 * 192 * 4) + a256(2 * xs)
+    # WGRAD, window form: 4-channel pixels, tpa = 8 taps per 128-B atom, na = 2,
+    # Wp = max(4*54 + 16, 224 + 2) = 232
+    assert mu.workspace_size(d, mu.BWD_FILTER, mu.IM2COL_GEMM, 3) == a256(3 * 224 * 232 * 4 * 4)
+    # DGRAD: dx super-pixels of f = 8 (u = 2; 8*8*3 = 192 <= 256 columns), Dr = 10 // 4 + 2 = 4
+    assert mu.workspace_size(d, mu.BWD_DATA, mu.IM2COL_GEMM, 4) == a256(192 * 16 * 64 * 4)
+    # ResNet conv1 BF16 (stride 2): FWD u = 2, f = 4: Dr = (2*1 + 7 - 1) // 4 + 1 = 3, Cs = 48 -> 64,
+    # 56 x 56 output super-pixels, 58 x 58 input super-pixels, filter 4K x 9 x 64.
     d = mu.desc(2, 3, 224, 224, 64, 7, 7, 3, 2, mu.MATH_BF16)
     assert mu.workspace_size(d, mu.FWD, mu.IM2COL_GEMM, 2) == a256(4 * 64 * 9 * 64 * 2) + a256(2 * 58 * 58 * 64 * 2)
-    assert mu.workspace_size(d, mu.BWD_FILTER, mu.IM2COL_GEMM, 2) == a256(2 * 115 * 115 * 64 * 2)
-    assert mu.workspace_size(d, mu.BWD_DATA, mu.IM2COL_GEMM, 2) == a256(12 * 16 * 64 * 2)
+    # WGRAD window: tpa = 16, na = 1, Wp = max(2*111 + 16, 224 + 3) = 238 -> 240
+    assert mu.workspace_size(d, mu.BWD_FILTER, mu.IM2COL_GEMM, 2) == a256(2 * 224 * 240 * 4 * 2)
+    # DGRAD: f = 4 (4*4*3 = 48 columns), Dr = 6 // 2 + 2 = 5: filter 48 x 25*64
+    assert mu.workspace_size(d, mu.BWD_DATA, mu.IM2COL_GEMM, 2) == a256(48 * 25 * 64 * 2)
+    # stride 3, BF16: 3*8 B is not a multiple of 16 -> WGRAD keeps the space-to-depth image
+    # (u = 1, f = 3, Dr = ceil(4/3) = 2, Cs = 27 -> 64, (P + 1) x (Q + 1) super-pixels)
+    d = mu.desc(1, 3, 20, 22, 64, 4, 4, 0, 3, mu.MATH_BF16)
+    assert mu.workspace_size(d, mu.BWD_FILTER, mu.IM2COL_GEMM, 1) == a256(1 * 7 * 8 * 64 * 2)
     # stride 1 keeps the channel-padded image (16 B per pixel)
     d = mu.desc(2, 3, 32, 32, 64, 3, 3, 1, 1, mu.MATH_BF16)
     assert mu.workspace_size(d, mu.FWD, mu.IM2COL_GEMM, 2) == 2 * 32 * 32 * 16

@@ -151,6 +151,9 @@ enum AMode : int {
     A_GATHER_SMALLC_PAD = 9, // same K' layout from a channel-padded copy of x (16 B per pixel): cp.async
     A_TMA_IM2COL_SMALLC = 10, // same K' layout from the padded copy by TMA im2col: one 128-pixel x 16-B box
                               // per tap, SWIZZLE_NONE core matrices (LBO 2 KB between taps, SBO 128 B)
+    A_HALO = 12,       // stride-1 FWD / DGRAD: per channel chunk, the full source rows a 128*mt-row tile of
+                       // the extended output grid touches (one TMA box per row, zero-filled padding); each
+                       // tap's A operand is a row-shifted window of that smem halo
     A_TMA_WIN = 11,    // WGRAD window operand, MN-major: rows j = (r, atom, tap, c) of the filter, K = pixels;
                        // one 4-D TMA box per 128-B atom from the overlapping-window view of the padded x
 };
@@ -222,6 +225,9 @@ struct TcArgs {
     int e_H, e_W, e_C, e_pad;
     // Window WGRAD (A_TMA_WIN / B_TMA_DYROW): 128-B atoms per filter row, q-blocks per output row
     int win_na, win_qb;
+    // Halo IG (A_HALO): extended grid of hx_H = Ho + R - 1 rows x hx_W (>= Wo + S - 1, multiple of 8)
+    // columns per image; source origin offset hx_pe; hx_nch channel chunks of 128 B; halo ring
+    int hx_W, hx_H, hx_Ho, hx_Wo, hx_pe, hx_nch, halo_bytes, hstages;
     // epilogue
     void* out;
     long long ldc;
@@ -366,6 +372,7 @@ bool make_im2col_map(CUtensorMap* tm, int elt, const void* base, int C, int W, i
 
 // Dynamic shared memory budget per CTA (227 KB minus alignment slack and barriers).
 constexpr int kSmemBudget = 232448 - 1024 - 512;
+constexpr int kRingBudget = 200 * 1024;  // operand ring of the default tilings (512-row tiles: +24 KB for a 3rd stage)
 
 int env_int(const char* name, int dflt) {
     const char* e = getenv(name);
@@ -405,8 +412,9 @@ struct Launch {
 template <int ELT, int AM, int BM_, int EPI>
 int launch_t(Launch& L, cudaStream_t st) {
     auto kern = tc_conv_gemm<ELT, AM, BM_, EPI>;
-    const int smem = 1024 + L.a.stages * L.a.km * (L.a.mt * 128 * 128 + L.a.b_bytes) + L.a.bres_bytes +
-                     (2 * L.a.stages + 5) * 8 + 64;
+    const int a_stage = AM == A_HALO ? 0 : L.a.mt * 128 * 128;
+    const int smem = 1024 + L.a.hstages * L.a.halo_bytes + L.a.stages * L.a.km * (a_stage + L.a.b_bytes) +
+                     L.a.bres_bytes + (2 * L.a.stages + 6 + 2 * L.a.hstages) * 8 + 64;
     static int configured = 0;  // per instantiation
     if (configured < smem) {
         cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 232448);
@@ -424,7 +432,7 @@ void size_stages(TcArgs& a) {
     a.tmem_cols = cols <= 64 ? 64 : cols <= 128 ? 128 : cols <= 256 ? 256 : 512;
     if (a.km < 1) a.km = 1;
     const int stage_bytes = a.km * (a.mt * 128 * 128 + a.b_bytes);
-    a.stages = std::min(env_int("MUCU_MAX_STAGES", 8), (200 * 1024) / stage_bytes);
+    a.stages = std::min(env_int("MUCU_MAX_STAGES", 8), (kRingBudget + (a.mt == 4 ? 24 * 1024 : 0)) / stage_bytes);
     if (a.stages < 2) a.stages = 2;
 }
 
@@ -438,16 +446,55 @@ void finalize_tiling(Launch& L, int elt, int step = 32) {
     size_stages(a);
 }
 
-// 256-row tiles (two 128-row accumulators sharing each B tile) for narrow N:
-// back-to-back MMAs of N <= 128 on ONE accumulator are latency-bound, two
-// interleaved accumulation chains are not.  TMA-fed A operands only; needs at
-// least one 256-row tile per SM.
+// 256- or 512-row tiles (two or four 128-row accumulators sharing each B tile)
+// for narrow N: a chain of dependent MMAs into one accumulator runs at one MMA
+// per ~250 cycles whatever N is (measured: N = 64 -> 459 TF/s with one chain,
+// 570 with two; N = 256 -> 1294), so short-N tiles need several independent
+// chains in flight.  TMA-fed K-major A operands only; needs at least one tile
+// per SM.
 void use_mt2(Launch& L, int num_sms) {
     TcArgs& a = L.a;
     if (a.BN > 128 || env_int("MUCU_MT2", 1) == 0) return;
+    const int force = env_int("MUCU_FORCE_MT", 0);  // tests: exercise 256/512-row tiles on small shapes
+    if (force == 4 && a.BN <= 64) num_sms = 1;
+    if (force == 2) { a.mt = 2; size_stages(a); return; }
+    if (a.BN <= 64 && env_int("MUCU_MT4", 1) && ceil_div(a.M, 512) >= num_sms) {
+        a.mt = 4;
+        size_stages(a);
+        return;
+    }
     if (ceil_div(a.M, 256) < num_sms) return;
     a.mt = 2;
     size_stages(a);
+}
+
+// Halo implicit GEMM geometry for a stride-1 conv viewed as a
+// correlation of a source tensor [b][Hs][Ws][Cs] (x for FWD, dy for DGRAD) with
+// R x S taps at origin offset pe over an Ho x Wo output grid.  Returns false
+// when the halo ring does not fit next to two B stages.
+bool halo_setup(TcArgs& a, int elt, int b, int Ho, int Wo, int R, int S, int pe, int Cs) {
+    // Opt-in (MUCU_HALO=1): measured slower than the TMA-im2col tiles on every
+    // AlexNet / ResNet layer; kept as a tested alternative producer.
+    if (env_int("MUCU_HALO", 0) == 0) return false;
+    const int KB = 128 / elt;
+    if (Cs % KB) return false;
+    a.hx_W = (int)align_up((uint64_t)(Wo + S - 1), 8);
+    a.hx_H = Ho + R - 1;
+    a.hx_Ho = Ho; a.hx_Wo = Wo; a.hx_pe = pe;
+    a.hx_nch = Cs / KB;
+    if (a.hx_W > 256) return false;  // one TMA box per row
+    a.M = (int)std::min<int64_t>((int64_t)b * a.hx_H * a.hx_W, INT32_MAX);
+    if ((int64_t)b * a.hx_H * a.hx_W > INT32_MAX) return false;
+    const int rows = 128 * a.mt;
+    const int nr = (a.hx_W - 8 + rows - 1 + (R - 1) * a.hx_W + S - 1) / a.hx_W + 1;
+    a.halo_bytes = (int)align_up((uint64_t)nr * a.hx_W * 128, 1024);
+    a.hstages = std::max(1, std::min(4, env_int("MUCU_HSTAGES", 2)));
+    a.tapR = R; a.tapS = S;
+    a.num_kb = a.hx_nch * R * S;
+    const int budget = 200 * 1024 - a.hstages * a.halo_bytes;
+    if (budget < 2 * a.b_bytes) return false;
+    a.stages = std::min(env_int("MUCU_MAX_STAGES", 8), budget / a.b_bytes);
+    return true;
 }
 
 }  // namespace
@@ -543,6 +590,22 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
             A.num_kb = (int)ceil_div(RSC, KB);
             if (!waligned) return -1;
             if (!map2(&L.tb, in1, RSC, g.k, RSC, KB, A.BN)) return -1;
+            if (g.stride == 1) {
+                Launch H = L;
+                H.a.mt = (H.a.BN <= 128 && env_int("MUCU_MT2", 1)) ? 2 : 1;
+                size_stages(H.a);
+                if (halo_setup(H.a, elt, b, g.p, g.q, g.r, g.s, g.pad, g.c)) {
+                    uint64_t dims[4] = {(uint64_t)g.c, (uint64_t)g.w, (uint64_t)g.h, (uint64_t)b};
+                    uint64_t str[3] = {(uint64_t)g.c * elt, (uint64_t)g.w * g.c * elt, (uint64_t)g.h * g.w * g.c * elt};
+                    uint32_t box[4] = {(uint32_t)KB, (uint32_t)H.a.hx_W, 1, 1};
+                    if (make_map(&H.ta, elt, in0, 4, dims, str, box)) {
+                        L = H;
+                        grid2(1);
+                        A.tma_bytes = A.BN * 128;
+                        return LAUNCH(A_HALO, B_TMA_K2, EPI_STORE);
+                    }
+                }
+            }
             if (use_tma_im2col() &&
                 make_im2col_map(&L.ta, elt, in0, g.c, g.w, g.h, b, -g.pad, -g.pad, g.pad - (g.s - 1),
                                 g.pad - (g.r - 1), 128, g.stride, false)) {
@@ -808,6 +871,27 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         if ((g.c * elt) % 16 == 0 && g.c >= atom) {
             // w viewed as {C, R*S, K} (c contiguous): B(c, (r,s,k)) MN-major
             if (!map3(&L.tb, in1, g.c, RS, g.k, g.c, RSC, atom, 1, KB, true)) return -1;
+            if (g.stride == 1 && g.pad <= g.r - 1 && g.pad <= g.s - 1) {
+                // transposed conv = correlation of dy with the flipped filter, origin R-1-pad
+                Launch H = L;
+                if (g.c > 128 && g.c % 128 == 0 && !env_int("MUCU_FORCE_BN", 0)) H.a.BN = 128;
+                H.a.bn_atoms = (H.a.BN * elt + 127) / 128;
+                H.a.b_bytes = std::max(H.a.BN * 128, H.a.bn_atoms * (128 / elt) * 128);
+                H.a.mt = (H.a.BN <= 128 && env_int("MUCU_MT2", 1)) ? 2 : 1;
+                size_stages(H.a);
+                if (g.r - 1 - g.pad == g.s - 1 - g.pad &&
+                    halo_setup(H.a, elt, b, g.h, g.w, g.r, g.s, g.r - 1 - g.pad, g.k)) {
+                    uint64_t dims[4] = {(uint64_t)g.k, (uint64_t)g.q, (uint64_t)g.p, (uint64_t)b};
+                    uint64_t str[3] = {(uint64_t)g.k * elt, (uint64_t)g.q * g.k * elt, (uint64_t)g.p * g.q * g.k * elt};
+                    uint32_t box[4] = {(uint32_t)KB, (uint32_t)H.a.hx_W, 1, 1};
+                    if (make_map(&H.ta, elt, in0, 4, dims, str, box)) {
+                        L = H;
+                        grid2(1);
+                        A.tma_bytes = A.bn_atoms * KB * 128;
+                        return LAUNCH(A_HALO, B_TMA_MN3, EPI_STORE);
+                    }
+                }
+            }
             // stride 1: im2col of dy with pad' = R-1-pad and flipped taps
             const int lw = g.pad - (g.s - 1), lh = g.pad - (g.r - 1);
             if (g.stride == 1 && use_tma_im2col() &&

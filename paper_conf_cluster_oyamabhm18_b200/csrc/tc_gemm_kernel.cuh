@@ -21,14 +21,15 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
     // p.mt blocks of 128 rows x 128 B (tile M = 128 * p.mt); MN-major WGRAD
     // stages hold p.km k-blocks (p.km x KB rows of K per 128-B atom column).
     const int A_HALF = 128 * 128 * p.km;
-    const int A_BYTES = p.mt * A_HALF;
+    constexpr bool HALO = (AM == A_HALO);
+    const int A_BYTES = HALO ? 0 : p.mt * A_HALF;
     const int KD = KB * p.km;                // K rows per stage (MN-major modes)
     constexpr bool A_MN = (AM == A_TMA_MN2 || AM == A_TMA_WIN);
     constexpr bool B_MN = (BM_ == B_TMA_MN2 || BM_ == B_TMA_MN3 || BM_ == B_GATHER_WG || BM_ == B_SCALAR_DGRAD ||
                            BM_ == B_SCALAR_WG || BM_ == B_TMA_IM2COL || BM_ == B_GATHER_SMALLC ||
                            BM_ == B_GATHER_SMALLC_PAD || BM_ == B_TMA_DYROW);
     constexpr bool A_TMA = (AM == A_TMA_K2 || AM == A_TMA_K3 || AM == A_TMA_MN2 || AM == A_TMA_IM2COL ||
-                            AM == A_TMA_IM2COL_SMALLC || AM == A_TMA_WIN);
+                            AM == A_TMA_IM2COL_SMALLC || AM == A_TMA_WIN || AM == A_HALO);
     constexpr bool A_NOSWZ = (AM == A_TMA_IM2COL_SMALLC);  // unswizzled core matrices, one 2-KB box per tap
     constexpr bool B_TMA = (BM_ == B_TMA_K2 || BM_ == B_TMA_K3 || BM_ == B_TMA_MN2 || BM_ == B_TMA_MN3 ||
                             BM_ == B_TMA_IM2COL || BM_ == B_TMA_DYROW);
@@ -48,7 +49,8 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
     const int S = p.stages;
     const int B_BYTES = p.b_bytes * p.km;
     uint8_t* sA = smem;
-    uint8_t* sB = smem + (size_t)S * A_BYTES;
+    // A_HALO: a ring of p.hstages halo tiles (p.halo_bytes each) replaces the A stages
+    uint8_t* sB = smem + (HALO ? (size_t)p.hstages * p.halo_bytes : (size_t)S * A_BYTES);
     uint8_t* sBres = sB + (size_t)S * B_BYTES;  // B_RESIDENT: whole filter, k-block after k-block
     uint64_t* bars = (uint64_t*)(sBres + (B_RES ? p.bres_bytes : 0));
     uint64_t* full = bars;
@@ -57,6 +59,8 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
     uint64_t* tempty = bars + 2 * S + 2; // [2]
     uint64_t* bres_bar = bars + 2 * S + 4;
     uint32_t* tmem_slot = (uint32_t*)(bars + 2 * S + 5);
+    uint64_t* hfull = bars + 2 * S + 6;             // [hstages] halo ring
+    uint64_t* hempty = bars + 2 * S + 6 + p.hstages;
 
     const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
     const int BMt = 128 * p.mt;  // tile rows: 128, or 256 as two 128-row halves with separate accumulators
@@ -75,6 +79,10 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
             mbar_init(smem_u32(&tempty[a]), 4);
         }
         mbar_init(smem_u32(bres_bar), 128);
+        for (int h = 0; h < p.hstages; ++h) {
+            mbar_init(smem_u32(&hfull[h]), 1);
+            mbar_init(smem_u32(&hempty[h]), 1);
+        }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     if (warp == 4) {
@@ -101,7 +109,77 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
         }
     };
 
-    if (warp < 4) {
+    if (HALO && warp < 4) {
+        // ===================== halo producers (A_HALO) =====================
+        // warp 1: one halo per (tile, channel chunk) = the full rows of the
+        // extended source grid the tile's taps touch (one TMA row box each);
+        // warp 0: the filter k-block of every (tile, chunk, tap).  Whole warps
+        // run the loops (lane 0 issues): a lone spinning lane next to lanes
+        // parked at the CTA barrier starves (measured 2x slower).
+        const int taps = p.tapR * p.tapS;
+        if (warp == 1) {
+            int hs = 0;
+            uint32_t hph = 0;
+            for (int tile = blockIdx.x; tile < total_tiles; tile += gridDim.x) {
+                int m0, n0, z, kb_begin, kb_end;
+                decode(tile, m0, n0, z, kb_begin, kb_end);
+                const int G0 = m0 / p.hx_W;
+                const int G1 = (m0 + BMt - 1 + (p.tapR - 1) * p.hx_W + p.tapS - 1) / p.hx_W;
+                const int nr = G1 - G0 + 1;
+                for (int c = 0; c < p.hx_nch; ++c) {
+                    mbar_wait(smem_u32(&hempty[hs]), hph ^ 1u);
+                    if (lane == 0) {
+                        const uint32_t dst = smem_u32(sA + (size_t)hs * p.halo_bytes);
+                        const uint32_t fb = smem_u32(&hfull[hs]);
+                        if (p.debug & 4) {
+                            mbar_arrive(fb);
+                        } else {
+                            mbar_arrive_tx(fb, (uint32_t)(nr * p.hx_W * 128));
+                            int n_ = G0 / p.hx_H, hx = G0 - n_ * p.hx_H;
+                            for (int i = 0; i < nr; ++i) {
+                                tma_load_4d(dst + (uint32_t)(i * p.hx_W * 128), &tmA, fb, c * KB, -p.hx_pe,
+                                            hx - p.hx_pe, n_);
+                                if (++hx == p.hx_H) { hx = 0; ++n_; }
+                            }
+                        }
+                    }
+                    __syncwarp();
+                    if (++hs == p.hstages) { hs = 0; hph ^= 1u; }
+                }
+            }
+        } else if (warp == 0) {
+            int s = 0;
+            uint32_t ph = 0;
+            for (int tile = blockIdx.x; tile < total_tiles; tile += gridDim.x) {
+                int m0, n0, z, kb_begin, kb_end;
+                decode(tile, m0, n0, z, kb_begin, kb_end);
+                for (int c = 0; c < p.hx_nch; ++c) {
+                    for (int tap = 0; tap < taps; ++tap) {
+                        mbar_wait(smem_u32(&empty[s]), ph ^ 1u);
+                        if (lane == 0) {
+                            const uint32_t bT = smem_u32(sB + (size_t)s * B_BYTES);
+                            const uint32_t fb = smem_u32(&full[s]);
+                            if (p.debug & 4) {
+                                mbar_arrive(fb);
+                            } else {
+                                mbar_arrive_tx(fb, (uint32_t)p.tma_bytes);
+                                if constexpr (BM_ == B_TMA_K2) tma_load_2d(bT, &tmB, fb, tap * p.C + c * KB, n0);
+                                if constexpr (BM_ == B_TMA_MN3) {
+                                    // DGRAD: tap (r', s') of the flipped filter = w[.][R-1-r'][S-1-s'][.]
+                                    const int rr = tap / p.tapS, ss = tap - rr * p.tapS;
+                                    const int rs = (p.R - 1 - rr) * p.S + (p.S - 1 - ss);
+                                    for (int a = 0; a < p.bn_atoms; ++a)
+                                        tma_load_3d(bT + a * KB * 128, &tmB, fb, n0 + a * (128 / ELT), rs, c * KB);
+                                }
+                            }
+                        }
+                        __syncwarp();
+                        if (++s == S) { s = 0; ph ^= 1u; }
+                    }
+                }
+            }
+        }
+    } else if (warp < 4) {
         // =========================== producers ===========================
         const int t = threadIdx.x;  // 0..127
         const T* gx = (const T*)p.gsrc;
@@ -179,7 +257,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
             // TMA im2col start pixel of this tile (FWD: output pixel m0 -> x origin;
             // DGRAD: dx pixel m0 -> dy origin h + pad - (R-1); phase mode: sub-grid
             // pixel (ii, jj) -> dy origin (i0 + ii - (tapR-1), j0 + jj - (tapS-1))).
-            int ic_w[2] = {0, 0}, ic_h[2] = {0, 0}, ic_n[2] = {0, 0};  // per 128-row half (constant-indexed)
+            int ic_w[4] = {0, 0, 0, 0}, ic_h[4] = {0, 0, 0, 0}, ic_n[4] = {0, 0, 0, 0};  // per 128-row block (constant-indexed)
             auto ic_of = [&](int mH, int& icw, int& ich, int& icn) {
                 if (p.ph_mode) {
                     const int hw = p.ph_H * p.ph_W;
@@ -201,8 +279,9 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                 }
             };
             if constexpr (AM == A_TMA_IM2COL || AM == A_TMA_IM2COL_SMALLC) {
-                ic_of(m0, ic_w[0], ic_h[0], ic_n[0]);
-                if (p.mt == 2) ic_of(m0 + 128, ic_w[1], ic_h[1], ic_n[1]);
+#pragma unroll
+                for (int hh = 0; hh < 4; ++hh)
+                    if (hh < p.mt) ic_of(m0 + 128 * hh, ic_w[hh], ic_h[hh], ic_n[hh]);
             }
             // Small-C FWD gather: packed 16-B chunks of 8 rows for one k-block.
             uint32_t pk[8][4];
@@ -277,17 +356,20 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                     const int r = kb / groups, s0 = (kb - r * groups) * 8;
                     const int nv = min(8, p.S - s0);
                     mbar_arrive_tx(fb, (uint32_t)(nv * 128 * 16 * p.mt));
-                    for (int hh = 0; hh < p.mt; ++hh)
-                        for (int j = 0; j < nv; ++j)
-                            tma_load_im2col_4d(aT + hh * 16384 + j * 2048, &tmA, fb, 0, hh ? ic_w[1] : ic_w[0],
-                                               hh ? ic_h[1] : ic_h[0], hh ? ic_n[1] : ic_n[0],
-                                               (uint16_t)(s0 + j), (uint16_t)r);
+#pragma unroll
+                    for (int hh = 0; hh < 4; ++hh)
+                        if (hh < p.mt)
+                            for (int j = 0; j < nv; ++j)
+                                tma_load_im2col_4d(aT + hh * 16384 + j * 2048, &tmA, fb, 0, ic_w[hh], ic_h[hh],
+                                                   ic_n[hh], (uint16_t)(s0 + j), (uint16_t)r);
                 } else if ((A_TMA || B_TMA) && t == 0 && (p.debug & 4)) {
                     mbar_arrive(fb);  // debug bit 2: no TMA loads (MMA-rate experiments)
                 } else if ((A_TMA || B_TMA) && t == 0) {
                     mbar_arrive_tx(fb, (uint32_t)p.tma_bytes);
                     // A: p.mt blocks of 128 rows (16 KB each)
-                    for (int hh = 0; hh < p.mt; ++hh) {
+#pragma unroll
+                    for (int hh = 0; hh < 4; ++hh) {
+                        if (hh >= p.mt) break;
                         const uint32_t aH = aT + hh * (A_MN ? (uint32_t)A_HALF : 16384u);
                         const int mH = m0 + 128 * hh;
                         if constexpr (AM == A_TMA_K2) tma_load_2d(aH, &tmA, fb, kb * KB, mH);
@@ -313,8 +395,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                             // 128 consecutive output pixels x KB channels of tap (r,s) in one TMA
                             const uint16_t ow = (uint16_t)(p.im2col_dgrad ? p.tapS - 1 - g_s : g_s);
                             const uint16_t oh = (uint16_t)(p.im2col_dgrad ? p.tapR - 1 - g_r : g_r);
-                            tma_load_im2col_4d(aH, &tmA, fb, g_c0, hh ? ic_w[1] : ic_w[0], hh ? ic_h[1] : ic_h[0],
-                                               hh ? ic_n[1] : ic_n[0], ow, oh);
+                            tma_load_im2col_4d(aH, &tmA, fb, g_c0, ic_w[hh], ic_h[hh], ic_n[hh], ow, oh);
                         }
                     }
                     if constexpr (BM_ == B_TMA_K2) tma_load_2d(bT, &tmB, fb, kb * KB, n0);
@@ -607,7 +688,58 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
         uint32_t aph = 0;
         const int KDm = A_MN ? KD : KB;  // K rows per MN-major atom column (km > 1 only with A_MN)
         if constexpr (B_RES) mbar_wait(smem_u32(bres_bar), 0u);  // staged filter is ready
-        for (int tile = blockIdx.x; tile < total_tiles; tile += gridDim.x) {
+        if constexpr (HALO) {
+            // A for tap (r', s') = 128 consecutive rows of the halo starting at row
+            // (m0 - G0*W') + r'*W' + s' -- a shifted window of the same smem tile
+            // (SW128 swizzle is address-based, so any 128-B row offset is a valid start).
+            int hs = 0;
+            uint32_t hph = 0;
+            const int taps = p.tapR * p.tapS;
+            for (int tile = blockIdx.x; tile < total_tiles; tile += gridDim.x) {
+                int m0, n0, z, kb_begin, kb_end;
+                decode(tile, m0, n0, z, kb_begin, kb_end);
+                mbar_wait(smem_u32(&tempty[acc]), aph ^ 1u);
+                tc_fence_after();
+                const uint32_t dtm = tmem + (uint32_t)(acc * p.mt * p.BN);
+                const int off0 = m0 - (m0 / p.hx_W) * p.hx_W;
+                for (int c = 0; c < p.hx_nch; ++c) {
+                    mbar_wait(smem_u32(&hfull[hs]), hph);
+                    const uint32_t hbase = smem_u32(sA + (size_t)hs * p.halo_bytes) + (uint32_t)(off0 * 128);
+                    for (int tap = 0; tap < taps; ++tap) {
+                        mbar_wait(smem_u32(&full[s]), ph);
+                        tc_fence_after();
+                        if (lane == 0 && (p.debug & 8)) {
+                            mma_commit(smem_u32(&empty[s]));
+                            if (tap == taps - 1) mma_commit(smem_u32(&hempty[hs]));
+                        } else if (lane == 0) {
+                            const int rr = (p.debug & 32) ? 0 : tap / p.tapS;
+                            const int ss = (p.debug & 16) ? 0 : tap - (tap / p.tapS) * p.tapS;
+                            const uint32_t aT = hbase + (uint32_t)((rr * p.hx_W + ss) * 128);
+                            const uint32_t bT = smem_u32(sB + (size_t)s * B_BYTES);
+#pragma unroll
+                            for (int j = 0; j < KB / UMMA_K; ++j) {
+                                const uint64_t bd = B_MN ? sdesc(bT + j * UMMA_K * 128, KB * 128, MN_SBO, MN_LAYOUT)
+                                                         : sdesc(bT + j * 32, 16, 1024);
+                                const uint32_t accf = (c > 0 || tap > 0 || j > 0) ? 1u : 0u;
+                                mma<ELT>(dtm, sdesc(aT + j * 32, 16, 1024), bd, idesc, accf);
+                                if (p.mt == 2)
+                                    mma<ELT>(dtm + (uint32_t)p.BN, sdesc(aT + 128 * 128 + j * 32, 16, 1024), bd, idesc,
+                                             accf);
+                            }
+                            mma_commit(smem_u32(&empty[s]));
+                            if (tap == taps - 1) mma_commit(smem_u32(&hempty[hs]));
+                        }
+                        __syncwarp();
+                        if (++s == S) { s = 0; ph ^= 1u; }
+                    }
+                    if (++hs == p.hstages) { hs = 0; hph ^= 1u; }
+                }
+                if (lane == 0) mma_commit(smem_u32(&tfull[acc]));
+                __syncwarp();
+                if (++acc == p.nacc) { acc = 0; aph ^= 1u; }
+            }
+        }
+        for (int tile = blockIdx.x; tile < total_tiles && !HALO; tile += gridDim.x) {
             int m0, n0, z, kb_begin, kb_end;
             decode(tile, m0, n0, z, kb_begin, kb_end);
             mbar_wait(smem_u32(&tempty[acc]), aph ^ 1u);  // epilogue has drained this accumulator
@@ -649,11 +781,13 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                     };
                     if constexpr (A_MN) {
                         for (int jj = 0; jj < p.km; ++jj) {
-                            if (p.mt == 2) issue(std::integral_constant<int, 2>{}, jj);
+                            if (p.mt == 4) issue(std::integral_constant<int, 4>{}, jj);
+                            else if (p.mt == 2) issue(std::integral_constant<int, 2>{}, jj);
                             else issue(std::integral_constant<int, 1>{}, jj);
                         }
                     } else {
-                        if (p.mt == 2) issue(std::integral_constant<int, 2>{}, 0);
+                        if (p.mt == 4) issue(std::integral_constant<int, 4>{}, 0);
+                        else if (p.mt == 2) issue(std::integral_constant<int, 2>{}, 0);
                         else issue(std::integral_constant<int, 1>{}, 0);
                     }
                     mma_commit(smem_u32(&empty[s]));
@@ -683,6 +817,13 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
             const int m = m0 + 128 * hh + row;
             // Output row of GEMM row m (phase mode scatters sub-grid rows back to dx).
             long long mrow = m;
+            bool rowok = true;
+            if (HALO && m < p.M) {
+                // extended-grid row m = ((n*Hx + oh)*W' + ow): junk unless oh < Ho, ow < Wo
+                const int G = m / p.hx_W, ow = m - G * p.hx_W, n = G / p.hx_H, oh = G - n * p.hx_H;
+                rowok = oh < p.hx_Ho && ow < p.hx_Wo;
+                mrow = ((long long)n * p.hx_Ho + oh) * p.hx_Wo + ow;
+            }
             if (EPI == EPI_STORE && p.ph_mode && m < p.M) {
                 const int hw = p.ph_H * p.ph_W;
                 const int n = m / hw, rem = m - n * hw, ii = rem / p.ph_W, jj = rem - ii * p.ph_W;
@@ -705,7 +846,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
 #pragma unroll
                     for (int j = 0; j < 32; ++j) v[j] = 0u;
                 }
-                if (m >= p.M || (p.debug & 1)) continue;  // debug bit 0: skip stores (timing experiments)
+                if (m >= p.M || !rowok || (p.debug & 1)) continue;  // debug bit 0: skip stores (timing experiments)
                 const int nb = n0 + c0;
                 if constexpr (EPI == EPI_D2S) {
                     // super-pixel row (n, i, jj); column (a, b, c) walked incrementally:
@@ -872,8 +1013,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                 }
             }
             };  // drain one 128-row half
-            drain(0);
-            if (p.mt == 2) drain(1);
+            for (int hh = 0; hh < p.mt; ++hh) drain(hh);
             // release this accumulator to the MMA warp
             tc_fence_before();
             __syncwarp();

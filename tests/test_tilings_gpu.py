@@ -1,0 +1,52 @@
+"""GPU parity of the alternative tilings the default heuristics pick only at
+full size (or not at all), forced on the small parity shapes:
+
+* MUCU_FORCE_MT=4 / 2: 512- / 256-row tiles (four / two interleaved TMEM
+  accumulators; chosen by default for narrow N when there is at least one
+  such tile per SM -- never at parity-test sizes);
+* MUCU_HALO=1: the halo producer for stride-1 FWD / DGRAD (opt-in).
+
+Integer-valued inputs make every tensor-core path exact (sums < 2^24), so the
+check is bit-exact against the fp64 oracle (BF16 outputs: RNE of the oracle).
+"""
+import numpy as np
+import pytest
+import torch
+
+import paper_conf_cluster_oyamabhm18_b200 as mu
+from synthetic import conv_inputs
+
+pytestmark = pytest.mark.gpu
+
+from gpu_util import oracle_ref, run_gpu  # noqa: E402
+
+SHAPES = {
+    "3x3s1_c64": (2, 64, 12, 12, 64, 3, 3, 1, 1),
+    "3x3s1_c128": (2, 128, 10, 10, 192, 3, 3, 1, 1),
+    "5x5s1": (2, 64, 11, 11, 48, 5, 5, 2, 1),
+    "3x3s1_p2": (2, 32, 7, 7, 32, 3, 3, 2, 1),
+    "3x3s2_c64": (2, 64, 15, 15, 128, 3, 3, 1, 2),
+    "1x1s1": (3, 64, 10, 10, 96, 1, 1, 0, 1),
+    "7x7s2_c3": (2, 3, 23, 23, 64, 7, 7, 3, 2),
+    "big_k": (1, 128, 6, 6, 256, 3, 3, 1, 1),
+}
+ENVS = {"mt4": {"MUCU_FORCE_MT": "4"}, "mt2": {"MUCU_FORCE_MT": "2"}, "halo": {"MUCU_HALO": "1"}}
+CASES = [(s, t, a) for s in SHAPES for t in (mu.FWD, mu.BWD_DATA)
+         for a in (mu.IMPLICIT_GEMM, mu.IM2COL_GEMM)]
+
+
+@pytest.mark.parametrize("env", list(ENVS))
+@pytest.mark.parametrize("math", [mu.MATH_TF32, mu.MATH_BF16], ids=["tf32", "bf16"])
+@pytest.mark.parametrize("case", CASES, ids=lambda c: f"{c[0]}-{mu.TYPE_NAMES[c[1]]}-{mu.ALGO_NAMES[c[2]]}")
+def test_forced_tiling_exact(case, math, env, monkeypatch):
+    for k, v in ENVS[env].items():
+        monkeypatch.setenv(k, v)
+    name, conv_type, algo = case
+    shape = SHAPES[name]
+    d = mu.desc(*shape, math)
+    x, w, dy = conv_inputs(*shape, seed=21, kind="int")
+    ref = oracle_ref(shape, conv_type, x, w, dy)
+    if math == mu.MATH_BF16:
+        ref = torch.from_numpy(ref).to(torch.bfloat16).double().numpy()
+    got, _ = run_gpu(d, conv_type, [(algo, shape[0])], x, w, dy)
+    assert np.array_equal(got, ref)

@@ -127,6 +127,27 @@ __device__ __forceinline__ void mma_commit(uint32_t bar) {
     asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(bar) : "memory");
 }
 
+// 256-bit global stores (sm_100 STG.256): alpha * 16 fp32 accumulators as bf16
+// (RNE) / alpha * 8 as fp32; the address must be 32-B aligned.
+__device__ __forceinline__ void st256_bf16(__nv_bfloat16* d, const uint32_t* v, float alpha) {
+    uint32_t w[8];
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+        const __nv_bfloat162 h = __floats2bfloat162_rn(alpha * __uint_as_float(v[2 * u]), alpha * __uint_as_float(v[2 * u + 1]));
+        w[u] = *reinterpret_cast<const uint32_t*>(&h);
+    }
+    asm volatile("st.global.v8.b32 [%0], {%1, %2, %3, %4, %5, %6, %7, %8};" ::"l"(d), "r"(w[0]), "r"(w[1]), "r"(w[2]),
+                 "r"(w[3]), "r"(w[4]), "r"(w[5]), "r"(w[6]), "r"(w[7])
+                 : "memory");
+}
+__device__ __forceinline__ void st256_f32(float* d, const uint32_t* v, float alpha) {
+    asm volatile("st.global.v8.f32 [%0], {%1, %2, %3, %4, %5, %6, %7, %8};" ::"l"(d), "f"(alpha * __uint_as_float(v[0])),
+                 "f"(alpha * __uint_as_float(v[1])), "f"(alpha * __uint_as_float(v[2])), "f"(alpha * __uint_as_float(v[3])),
+                 "f"(alpha * __uint_as_float(v[4])), "f"(alpha * __uint_as_float(v[5])), "f"(alpha * __uint_as_float(v[6])),
+                 "f"(alpha * __uint_as_float(v[7]))
+                 : "memory");
+}
+
 #define TMEM_LD32(taddr, v)                                                                                      \
     asm volatile(                                                                                                \
         "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16,%17," \

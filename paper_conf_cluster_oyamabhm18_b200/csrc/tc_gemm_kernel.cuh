@@ -861,27 +861,18 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                     const long long jump = (long long)(p.e_W - p.s2_st) * p.e_C;
                     bool okh = (unsigned)(h0 + a) < (unsigned)p.e_H, okw = (unsigned)(w0 + bq) < (unsigned)p.e_W;
                     const int nlim = p.N - nb;
-                    if (p.e_C % 32 == 0 && p.beta == 0.f) {
+                    if (p.e_C % 32 == 0 && p.beta == 0.f && (((uintptr_t)p.out & 31) == 0)) {
                         // the 32 columns are 32 consecutive channels of one output pixel
                         // (u x u FWD super-pixels): 16-B vector stores
                         if (nlim >= 32 && okh && okw) {
                             if (p.out_bf16) {
                                 __nv_bfloat16* d = (__nv_bfloat16*)p.out + off;
 #pragma unroll
-                                for (int j = 0; j < 32; j += 8) {
-                                    __align__(16) __nv_bfloat16 tmp[8];
-#pragma unroll
-                                    for (int u = 0; u < 8; ++u)
-                                        tmp[u] = __float2bfloat16_rn(p.alpha * __uint_as_float(v[j + u]));
-                                    *reinterpret_cast<uint4*>(d + j) = *reinterpret_cast<uint4*>(tmp);
-                                }
+                                for (int j = 0; j < 32; j += 16) st256_bf16(d + j, v + j, p.alpha);
                             } else {
                                 float* d = (float*)p.out + off;
 #pragma unroll
-                                for (int j = 0; j < 32; j += 4)
-                                    *reinterpret_cast<float4*>(d + j) =
-                                        make_float4(p.alpha * __uint_as_float(v[j]), p.alpha * __uint_as_float(v[j + 1]),
-                                                    p.alpha * __uint_as_float(v[j + 2]), p.alpha * __uint_as_float(v[j + 3]));
+                                for (int j = 0; j < 32; j += 8) st256_f32(d + j, v + j, p.alpha);
                             }
                         }
                         continue;
@@ -972,7 +963,12 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                 } else if (p.out_bf16) {
                     __nv_bfloat16* d = (__nv_bfloat16*)outT + (size_t)mrow * p.ldc + nb;
                     const bool vec = (nb + 32 <= p.N) && ((p.ldc & 7) == 0) && p.beta == 0.f;
-                    if (vec) {
+                    if (vec && (p.ldc & 15) == 0 && (((uintptr_t)p.out & 31) == 0)) {
+                        // 32-B stores: every store fills whole L2 sectors (16-B stores of
+                        // rows 512 B apart half-fill them: 2x the L2 write traffic, measured)
+#pragma unroll
+                        for (int j = 0; j < 32; j += 16) st256_bf16(d + j, v + j, p.alpha);
+                    } else if (vec) {
 #pragma unroll
                         for (int j = 0; j < 32; j += 8) {
                             __align__(16) __nv_bfloat16 tmp[8];
@@ -994,7 +990,10 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                 } else {
                     float* d = outF + (size_t)mrow * p.ldc + nb;
                     const bool vec = (nb + 32 <= p.N) && ((p.ldc & 3) == 0) && p.beta == 0.f;
-                    if (vec) {
+                    if (vec && (p.ldc & 7) == 0 && (((uintptr_t)p.out & 31) == 0)) {
+#pragma unroll
+                        for (int j = 0; j < 32; j += 8) st256_f32(d + j, v + j, p.alpha);
+                    } else if (vec) {
 #pragma unroll
                         for (int j = 0; j < 32; j += 4)
                             *reinterpret_cast<float4*>(d + j) =

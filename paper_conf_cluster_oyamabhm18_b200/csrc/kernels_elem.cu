@@ -485,7 +485,35 @@ __global__ void scale_kernel(float* __restrict__ p, int64_t n, float beta) {
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
         p[i] = beta == 0.f ? 0.f : beta * p[i];
 }
+// Strided DGRAD: dx pixels whose phase ((h+pad) % st, (w+pad) % st) meets no
+// filter tap (r0 >= R or s0 >= S, e.g. 3 of 4 pixels of a 1x1 stride-2 layer)
+// receive no gradient: zero them (beta = 0) in one pass of 16-B stores.
+__global__ void zero_tapless_kernel(uint4* __restrict__ dx, int rows, int cpp, int H, int W, int R, int S, int pad,
+                                    int st) {
+    // one block per dx pixel row (n, h); a row whose phase meets no tap is zeroed whole
+    const int per_row = W * cpp;
+    for (int row = blockIdx.x; row < rows; row += gridDim.x) {
+        const int h = row % H;
+        const bool all = (h + pad) % st >= R;
+        uint4* d = dx + (int64_t)row * per_row;
+        for (int i = threadIdx.x; i < per_row; i += blockDim.x) {
+            const int w = i / cpp;
+            if (all || (w + pad) % st >= S) d[i] = make_uint4(0u, 0u, 0u, 0u);
+        }
+    }
+}
 }  // namespace
+
+int launch_zero_tapless(const Geom& g, int32_t b, void* dx, cudaStream_t st) {
+    const int elt = elt_size(g.math);
+    if ((g.c * elt) % 16 != 0) return -1;
+    const int cpp = g.c * elt / 16;
+    const int rows = b * g.h;
+    zero_tapless_kernel<<<std::min(rows, 148 * 16), 256, 0, st>>>((uint4*)dx, rows, cpp, g.h, g.w, g.r, g.s, g.pad,
+                                                                  g.stride);
+    count_launch();
+    return (int)cudaGetLastError();
+}
 
 namespace {
 // One thread per pixel: reads C (< 16 B) channels, writes one 16-B vector.

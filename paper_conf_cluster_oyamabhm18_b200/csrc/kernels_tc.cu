@@ -230,6 +230,10 @@ struct TcArgs {
     // (ph_H x ph_W) sub-grid.  tapR/tapS = R/S when not in phase mode.
     int ph_mode, ph_H, ph_W, ph_i0, ph_j0, ph_r0, ph_s0, ph_hb, ph_wb;
     int tapR, tapS;
+    // Merged strided-DGRAD launch: ph_n phases (blockIdx-tiles z = phase), each with
+    // its own taps / origin / output offset and k-block count; all share ph_H x ph_W
+    // and one TMA im2col map (equal start-pixel corners), so one launch covers dx.
+    int ph_n, ph_r0v[4], ph_s0v[4], ph_i0v[4], ph_j0v[4], ph_hbv[4], ph_wbv[4], ph_tRv[4], ph_tSv[4], ph_kbv[4];
     int ph_u;                // phase mode: im2col positions advance by ph_u per sub-grid pixel (1 except s2d DGRAD)
     // Small-C layers: K' = (r, s8, c') with taps grouped by 8 per k-block and
     // channels zero-padded to cp = 16 B / elt; s8 = S rounded up to 8.
@@ -262,10 +266,10 @@ constexpr int kThreads = 288;  // 4 producer warps, 1 MMA warp, 4 epilogue warps
 
 // DGRAD reduction tap index -> filter tap r*S+s (phase mode: the sub-filter
 // tap (a,b) is (r0 + st*a, s0 + st*b)).
-__device__ __forceinline__ int dgrad_tap_rs(const TcArgs& p, int tap) {
+__device__ __forceinline__ int dgrad_tap_rs(const TcArgs& p, int tap, int r0, int s0, int tapS) {
     if (!p.ph_mode) return tap;
-    const int a = tap / p.tapS, b = tap - a * p.tapS;
-    return (p.ph_r0 + p.stride * a) * p.S + p.ph_s0 + p.stride * b;
+    const int a = tap / tapS, b = tap - a * tapS;
+    return (r0 + p.stride * a) * p.S + s0 + p.stride * b;
 }
 
 template <int ELT>
@@ -848,6 +852,58 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         A.gsrc = in0; A.bsrc = in1; A.ldc = g.c; A.N = g.c;
         A.ph_mode = 1; A.im2col_dgrad = 1;
         finalize_tiling(L, elt);
+        // beta = 0: the phases that meet no tap (r0 >= R or s0 >= S) are zeroed in one
+        // elementwise pass instead of one GEMM launch each
+        const bool zero_pass = beta == 0.f && (g.r < g.stride || g.s < g.stride) && (g.c * elt) % 16 == 0;
+        if (zero_pass) {
+            err = launch_zero_tapless(g, b, out, st);
+            if (err) return err;
+        }
+        // One launch for all phases with taps when they tile equal sub-grids whose
+        // dy start pixels share one im2col map (equal lower corners i0 - (nr-1),
+        // j0 - (ns-1)); tiles of phase z are blockIdx-tiles of batch z.
+        if (bvec && env_int("MUCU_MERGE_PHASES", 1) && g.stride * g.stride <= 4) {
+            int n_ph = 0, H0 = -1, W0 = -1, lh0 = 0, lw0 = 0;
+            bool ok = true;
+            for (int r0 = 0; r0 < g.stride && ok; ++r0) {
+                for (int s0 = 0; s0 < g.stride && ok; ++s0) {
+                    const int i0 = std::max(0, (int)ceil_div(g.pad - r0, g.stride));
+                    const int j0 = std::max(0, (int)ceil_div(g.pad - s0, g.stride));
+                    const int hb = r0 - g.pad + g.stride * i0, wb = s0 - g.pad + g.stride * j0;
+                    const int Hph = hb < g.h ? (int)ceil_div(g.h - hb, g.stride) : 0;
+                    const int Wph = wb < g.w ? (int)ceil_div(g.w - wb, g.stride) : 0;
+                    const int nr = r0 < g.r ? (int)ceil_div(g.r - r0, g.stride) : 0;
+                    const int ns = s0 < g.s ? (int)ceil_div(g.s - s0, g.stride) : 0;
+                    if (Hph <= 0 || Wph <= 0) continue;
+                    if (nr == 0 || ns == 0) { ok = zero_pass; continue; }
+                    const int lh = i0 - (nr - 1), lw = j0 - (ns - 1);
+                    if (n_ph == 0) { H0 = Hph; W0 = Wph; lh0 = lh; lw0 = lw; }
+                    ok = Hph == H0 && Wph == W0 && lh == lh0 && lw == lw0;
+                    A.ph_r0v[n_ph] = r0; A.ph_s0v[n_ph] = s0; A.ph_i0v[n_ph] = i0; A.ph_j0v[n_ph] = j0;
+                    A.ph_hbv[n_ph] = hb; A.ph_wbv[n_ph] = wb; A.ph_tRv[n_ph] = nr; A.ph_tSv[n_ph] = ns;
+                    A.ph_kbv[n_ph] = nr * ns * (g.k / KB);
+                    ++n_ph;
+                }
+            }
+            if (ok && n_ph > 1) {
+                A.ph_n = n_ph; A.ph_H = H0; A.ph_W = W0;
+                A.tapR = A.ph_tRv[0]; A.tapS = A.ph_tSv[0];
+                A.M = b * H0 * W0;
+                A.num_kb = 0;
+                for (int z = 0; z < n_ph; ++z) A.num_kb = std::max(A.num_kb, A.ph_kbv[z]);
+                if (!make_im2col_map(&L.ta, elt, in0, g.k, g.q, g.p, b, lw0, lh0, lw0 + W0 - g.q, lh0 + H0 - g.p, 128,
+                                     1, false))
+                    return -1;
+                A.mt = 1;
+                size_stages(A);
+                // 512-/256-row tiles only when every phase alone has a tile per SM
+                use_mt2(L, num_sms);
+                grid2(n_ph);
+                A.tma_bytes = 16384 * A.mt + A.bn_atoms * KB * 128;
+                return LAUNCH(A_TMA_IM2COL, B_TMA_MN3, EPI_STORE);
+            }
+            A.ph_n = 0;
+        }
         for (int r0 = 0; r0 < g.stride; ++r0) {
             for (int s0 = 0; s0 < g.stride; ++s0) {
                 // dx rows with (h + pad) % st == r0: h = r0 - pad + st*i, i >= i0
@@ -859,6 +915,7 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
                 if (Hph <= 0 || Wph <= 0) continue;
                 const int nr = r0 < g.r ? (int)ceil_div(g.r - r0, g.stride) : 0;
                 const int ns = s0 < g.s ? (int)ceil_div(g.s - s0, g.stride) : 0;
+                if (zero_pass && (nr == 0 || ns == 0)) continue;
                 A.ph_H = Hph; A.ph_W = Wph; A.ph_i0 = i0; A.ph_j0 = j0; A.ph_r0 = r0; A.ph_s0 = s0;
                 A.ph_hb = hb; A.ph_wb = wb; A.tapR = std::max(nr, 1); A.tapS = std::max(ns, 1);
                 A.M = b * Hph * Wph;

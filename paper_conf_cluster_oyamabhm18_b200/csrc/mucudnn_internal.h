@@ -113,6 +113,8 @@ int launch_col2im(const Geom& g, int32_t b, float alpha, const float* dcol, int3
                   void* dx, cudaStream_t st);
 int launch_wg_filter(const Geom& g, bool dgrad, const void* w, void* U, cudaStream_t st);
 int launch_scale(int64_t n, float beta, float* p, cudaStream_t st);  // p *= beta (beta == 0: p = 0)
+// dx = 0 on the pixels of strided-DGRAD phases that meet no filter tap (C*elt % 16 == 0, else -1)
+int launch_zero_tapless(const Geom& g, int32_t b, void* dx, cudaStream_t st);
 // x[b,H,W,C] -> xp[b,H,W,16/elt] with channels zero-padded to 16 B per pixel.
 int launch_pad_channels(const Geom& g, int32_t b, const void* x, void* xp, cudaStream_t st);
 // Space-to-depth image xs[b][I][J][Cs] and filters (kernels_elem.cu).

@@ -102,7 +102,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
         const int ntile = rem / mt;
         m0 = (rem - ntile * mt) * BMt;
         n0 = ntile * p.BN;
-        kb_begin = 0; kb_end = p.num_kb;
+        kb_begin = 0; kb_end = p.ph_n ? p.ph_kbv[z] : p.num_kb;
         if (SPLITK) {
             kb_begin = z * p.kb_per_split;
             kb_end = min(p.num_kb, kb_begin + p.kb_per_split);
@@ -246,13 +246,19 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                     }
                 }
             }
+            // Phase of this tile (merged strided-DGRAD launch: z = phase index)
+            int tR = p.tapR, tS = p.tapS, pr0 = p.ph_r0, ps0 = p.ph_s0, pi0 = p.ph_i0, pj0 = p.ph_j0;
+            if (p.ph_n) {
+                tR = p.ph_tRv[z]; tS = p.ph_tSv[z]; pr0 = p.ph_r0v[z]; ps0 = p.ph_s0v[z];
+                pi0 = p.ph_i0v[z]; pj0 = p.ph_j0v[z];
+            }
             // Incremental (r, s, c0) of the current k-block: a k-block covers KB
             // consecutive channels of one filter tap.
             int g_c0 = 0, g_s = 0, g_r = 0;
             if constexpr (WALK) {
                 const int kk0 = kb_begin * KB;
                 const int rs = kk0 / gch;
-                g_c0 = kk0 - rs * gch; g_r = rs / p.tapS; g_s = rs - g_r * p.tapS;
+                g_c0 = kk0 - rs * gch; g_r = rs / tS; g_s = rs - g_r * tS;
             }
             // TMA im2col start pixel of this tile (FWD: output pixel m0 -> x origin;
             // DGRAD: dx pixel m0 -> dy origin h + pad - (R-1); phase mode: sub-grid
@@ -264,8 +270,8 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                     icn = mH / hw;
                     const int rem = mH - icn * hw, ii = rem / p.ph_W, jj = rem - ii * p.ph_W;
                     // ph_u > 1 (space-to-depth DGRAD): the map walks u-strided positions
-                    ich = p.ph_u * (p.ph_i0 + ii) + (p.ph_u - 1) - (p.tapR - 1);
-                    icw = p.ph_u * (p.ph_j0 + jj) + (p.ph_u - 1) - (p.tapS - 1);
+                    ich = p.ph_u * (pi0 + ii) + (p.ph_u - 1) - (tR - 1);
+                    icw = p.ph_u * (pj0 + jj) + (p.ph_u - 1) - (tS - 1);
                 } else if (p.im2col_dgrad) {
                     const int hw = p.H * p.W;
                     icn = mH / hw;
@@ -393,8 +399,8 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                         }
                         if constexpr (AM == A_TMA_IM2COL) {
                             // 128 consecutive output pixels x KB channels of tap (r,s) in one TMA
-                            const uint16_t ow = (uint16_t)(p.im2col_dgrad ? p.tapS - 1 - g_s : g_s);
-                            const uint16_t oh = (uint16_t)(p.im2col_dgrad ? p.tapR - 1 - g_r : g_r);
+                            const uint16_t ow = (uint16_t)(p.im2col_dgrad ? tS - 1 - g_s : g_s);
+                            const uint16_t oh = (uint16_t)(p.im2col_dgrad ? tR - 1 - g_r : g_r);
                             tma_load_im2col_4d(aH, &tmA, fb, g_c0, ic_w[hh], ic_h[hh], ic_n[hh], ow, oh);
                         }
                     }
@@ -408,7 +414,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                         // k-block kb covers tap kb / (K/KB), channels k0 = (kb % (K/KB)) * KB
                         const int kpr = p.K / KB;
                         const int tap = kb / kpr, k0 = (kb - tap * kpr) * KB;
-                        const int rs = dgrad_tap_rs(p, tap);
+                        const int rs = dgrad_tap_rs(p, tap, pr0, ps0, tS);
                         for (int a = 0; a < p.bn_atoms; ++a)
                             tma_load_3d(bT + a * KB * 128, &tmB, fb, n0 + a * (128 / ELT), rs, k0);
                     }
@@ -502,7 +508,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                 }
                 if constexpr (WALK) {
                     g_c0 += KB;
-                    if (g_c0 >= gch) { g_c0 = 0; if (++g_s == p.tapS) { g_s = 0; ++g_r; } }
+                    if (g_c0 >= gch) { g_c0 = 0; if (++g_s == tS) { g_s = 0; ++g_r; } }
                 }
                 if constexpr (AM == A_SCALAR_FWD) {
                     // thread t owns row t; KB elements, kk = (r,s,c) decomposed each
@@ -622,7 +628,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                         float v = 0.f;
                         if (j < p.N && kk < p.kred) {
                             const int tap = kk / p.K, k = kk - tap * p.K;
-                            const int rs = dgrad_tap_rs(p, tap);
+                            const int rs = dgrad_tap_rs(p, tap, pr0, ps0, tS);
                             v = (float)bs[((size_t)k * RS + rs) * p.C + j];
                         }
                         st_shared_elt<T>(bT + mnmaj_off<ELT>(jj, krow, KB), (T)v);
@@ -827,13 +833,14 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
             if (EPI == EPI_STORE && p.ph_mode && m < p.M) {
                 const int hw = p.ph_H * p.ph_W;
                 const int n = m / hw, rem = m - n * hw, ii = rem / p.ph_W, jj = rem - ii * p.ph_W;
-                mrow = ((long long)n * p.H + p.ph_hb + p.stride * ii) * p.W + p.ph_wb + p.stride * jj;
+                const int hb = p.ph_n ? p.ph_hbv[z] : p.ph_hb, wb = p.ph_n ? p.ph_wbv[z] : p.ph_wb;
+                mrow = ((long long)n * p.H + hb + p.stride * ii) * p.W + wb + p.stride * jj;
             }
             const uint32_t taddr_row =
                 tmem + (uint32_t)((acc * p.mt + hh) * p.BN) + ((uint32_t)(q4 * 32) << 16);
             float* outF = (float*)p.out;
             T* outT = (T*)p.out;
-            if (EPI == EPI_STORE && z > 0) {
+            if (EPI == EPI_STORE && z > 0 && !p.ph_n) {
                 outF += (size_t)z * p.batch_stride;
                 outT += (size_t)z * p.batch_stride;
             }

@@ -26,11 +26,14 @@ SHAPES = {
     "5x5s1": (2, 64, 11, 11, 48, 5, 5, 2, 1),
     "3x3s1_p2": (2, 32, 7, 7, 32, 3, 3, 2, 1),
     "3x3s2_c64": (2, 64, 15, 15, 128, 3, 3, 1, 2),
+    "3x3s2_even": (2, 64, 14, 14, 64, 3, 3, 1, 2),      # strided DGRAD: the 4 phases in one launch
+    "1x1s2_c128": (2, 128, 14, 12, 64, 1, 1, 0, 2),     # strided DGRAD: 3 tapless phases zeroed
     "1x1s1": (3, 64, 10, 10, 96, 1, 1, 0, 1),
     "7x7s2_c3": (2, 3, 23, 23, 64, 7, 7, 3, 2),
     "big_k": (1, 128, 6, 6, 256, 3, 3, 1, 1),
 }
-ENVS = {"mt4": {"MUCU_FORCE_MT": "4"}, "mt2": {"MUCU_FORCE_MT": "2"}, "halo": {"MUCU_HALO": "1"}}
+ENVS = {"mt4": {"MUCU_FORCE_MT": "4"}, "mt2": {"MUCU_FORCE_MT": "2"}, "halo": {"MUCU_HALO": "1"},
+        "per_phase": {"MUCU_MERGE_PHASES": "0"}}
 CASES = [(s, t, a) for s in SHAPES for t in (mu.FWD, mu.BWD_DATA)
          for a in (mu.IMPLICIT_GEMM, mu.IM2COL_GEMM)]
 

@@ -133,8 +133,10 @@ mucu_status_t mucu_output_dims(const mucu_conv_desc_t* desc, int32_t* p, int32_t
  *                          Cs = f*f*C rounded up to 128/elt, Pu = ceil(P/u), Qu = ceil(Q/u):
  *                          u*u*K*Dr*Ds*Cs*elt + b*(Pu+Dr-1)*(Qu+Ds-1)*Cs*elt
  *                     WGRAD with C <= 4 and st*16 % 16 == 0 (BF16: st even) ("window"):
- *                          b*H*Wp*4*elt, tpa = 32/elt taps per 128-B atom, na = ceil(S/tpa),
- *                          Wp = max(st*(Q-1) + na*tpa, W + pad) rounded up to 4
+ *                          b*H*Wp*4*elt; atoms of aw bytes (TF32: 128; BF16: the aw in {128, 64, 32}
+ *                          minimising align256(R*na*aw/elt), larger aw on ties), tpa = aw/(4*elt)
+ *                          taps per atom, na = ceil(S/tpa), Wp = max(st*(Q-1) + na*tpa, W + pad)
+ *                          rounded up to 4
  *                     WGRAD otherwise (u = 1, f = st): b*(P+Dr-1)*(Q+Ds-1)*Cs*elt
  *                     DGRAD (when K % (128/elt) == 0, st*st*C <= 256): u = 2 if (2*st)^2*C <= 256
  *                          else 1, f = st*u, Dr = ceil(R/st) - 1 + u, Ds likewise: f*f*C*Dr*Ds*K*elt

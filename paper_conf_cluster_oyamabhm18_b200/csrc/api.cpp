@@ -119,11 +119,21 @@ Win win_geom(const Geom& g) {
     Win z;
     const int elt = elt_size(g.math);
     z.cpx = 4;
-    z.tpa = 128 / elt / z.cpx;
+    // GEMM rows per filter row = na * aw/elt; BF16 may use 64- or 32-B swizzle atoms
+    // (fewer padded taps: ResNet 7 taps -> one 8-tap 64-B atom instead of a 16-tap
+    // 128-B one); TF32 MN-major operands need the 128-B (32-B-base) layout.
+    z.aw = 128;
+    int best = 1 << 30;
+    for (int aw = 128; aw >= (elt == 2 ? 32 : 128); aw /= 2) {
+        const int tpa = aw / elt / z.cpx, na = (g.s + tpa - 1) / tpa;
+        const int M = (int)align_up((uint64_t)g.r * na * (aw / elt), 256);
+        if (M < best) { best = M; z.aw = aw; }
+    }
+    z.tpa = z.aw / elt / z.cpx;
     z.na = (g.s + z.tpa - 1) / z.tpa;
     // every window read stays inside its row: st*(Q-1) + na*tpa <= Wp
     z.Wp = (int)align_up((uint64_t)std::max(g.stride * (g.q - 1) + z.na * z.tpa, g.w + g.pad), 4);
-    z.M = g.r * z.na * (128 / elt);
+    z.M = g.r * z.na * (z.aw / elt);
     return z;
 }
 

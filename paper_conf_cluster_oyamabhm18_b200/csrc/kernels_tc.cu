@@ -175,6 +175,8 @@ enum AMode : int {
     A_HALO = 12,       // stride-1 FWD / DGRAD: per channel chunk, the full source rows a 128*mt-row tile of
                        // the extended output grid touches (one TMA box per row, zero-filled padding); each
                        // tap's A operand is a row-shifted window of that smem halo
+    A_TMA_WIN64 = 13,  // A_TMA_WIN with 64-B / 32-B swizzle atoms (BF16; fewer padded taps)
+    A_TMA_WIN32 = 14,
     A_TMA_WIN = 11,    // WGRAD window operand, MN-major: rows j = (r, atom, tap, c) of the filter, K = pixels;
                        // one 4-D TMA box per 128-B atom from the overlapping-window view of the padded x
 };
@@ -249,7 +251,7 @@ struct TcArgs {
     // EPI_D2S output tensor [*, e_H, e_W, e_C], written at (s2_st*i + a - e_pad, s2_st*j + b - e_pad)
     int e_H, e_W, e_C, e_pad;
     // Window WGRAD (A_TMA_WIN / B_TMA_DYROW): 128-B atoms per filter row, q-blocks per output row
-    int win_na, win_qb;
+    int win_na, win_qb, win_aw;  // + bytes per A swizzle atom (128 / 64 / 32: UMMA layout 2 / 4 / 6)
     // Halo IG (A_HALO): extended grid of hx_H = Ho + R - 1 rows x hx_W (>= Wo + S - 1, multiple of 8)
     // columns per image; source origin offset hx_pe; hx_nch channel chunks of 128 B; halo ring
     int hx_W, hx_H, hx_Ho, hx_Wo, hx_pe, hx_nch, halo_bytes, hstages;
@@ -336,9 +338,12 @@ EncodeTiledFn get_encode() {
 
 // Tensor map over a row-major tensor with up to 4 dims (dims[0] contiguous).
 bool make_map(CUtensorMap* tm, int elt, const void* base, int rank, const uint64_t* dims, const uint64_t* strides_bytes,
-              const uint32_t* box, bool mn_major = false) {
+              const uint32_t* box, bool mn_major = false, int swz = 128) {
     // 32-bit MN-major operands need the 32-B-atom swizzle matching SWIZZLE_128B_BASE32B.
-    const CUtensorMapSwizzle sw = (mn_major && elt == 4) ? CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B : CU_TENSOR_MAP_SWIZZLE_128B;
+    const CUtensorMapSwizzle sw = (mn_major && elt == 4) ? CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B
+                                  : swz == 64                ? CU_TENSOR_MAP_SWIZZLE_64B
+                                  : swz == 32                ? CU_TENSOR_MAP_SWIZZLE_32B
+                                                             : CU_TENSOR_MAP_SWIZZLE_128B;
     EncodeTiledFn enc = get_encode();
     if (!enc) return false;
     cuuint64_t d[4], s[3];
@@ -672,7 +677,7 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         char* xp = ws + WL.a_off;
         err = launch_win_pad(g, b, z.Wp, in0, xp, st);
         if (err) return err;
-        A.M = z.M; A.N = g.k; A.ldc = RSC; A.kred = (int)(b * PQ); A.cp = z.cpx; A.win_na = z.na;
+        A.M = z.M; A.N = g.k; A.ldc = RSC; A.kred = (int)(b * PQ); A.cp = z.cpx; A.win_na = z.na; A.win_aw = z.aw;
         wgrad_tiling(atom, true, g.q);
         if (beta != 1.f) {
             err = launch_scale(g.k * RSC, beta, (float*)out, st);
@@ -680,12 +685,15 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         }
         const int KD = KB * A.km;
         const uint64_t pb = (uint64_t)z.cpx * elt;
-        uint64_t adims[4] = {(uint64_t)z.na * atom, (uint64_t)g.q, (uint64_t)g.h, (uint64_t)b};
+        const int wat = z.aw / elt;  // elements per A atom
+        uint64_t adims[4] = {(uint64_t)z.na * wat, (uint64_t)g.q, (uint64_t)g.h, (uint64_t)b};
         uint64_t astr[3] = {g.stride * pb, z.Wp * pb, (uint64_t)g.h * z.Wp * pb};
-        uint32_t abox[4] = {(uint32_t)atom, (uint32_t)KD, 1, 1};
-        if (!make_map(&L.ta, elt, xp, 4, adims, astr, abox, true)) return -1;
+        uint32_t abox[4] = {(uint32_t)wat, (uint32_t)KD, 1, 1};
+        if (!make_map(&L.ta, elt, xp, 4, adims, astr, abox, true, z.aw)) return -1;
         if (!map3(&L.tb, in1, g.k, g.q, (uint64_t)b * g.p, g.k, (uint64_t)g.q * g.k, atom, KD, 1, true)) return -1;
         A.tma_bytes = A.km * (A.mt * 128 * KB * elt + A.bn_atoms * KB * 128);
+        if (z.aw == 64) return LAUNCH(A_TMA_WIN64, B_TMA_DYROW, EPI_WGRAD_WIN);
+        if (z.aw == 32) return LAUNCH(A_TMA_WIN32, B_TMA_DYROW, EPI_WGRAD_WIN);
         return LAUNCH(A_TMA_WIN, B_TMA_DYROW, EPI_WGRAD_WIN);
     }
     if (algo == MUCU_ALGO_IM2COL_GEMM && s2d_tc(g, type)) {

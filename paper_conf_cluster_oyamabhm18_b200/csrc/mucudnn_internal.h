@@ -53,9 +53,9 @@ inline int s2d_taps(int r, int stride) { return (r + stride - 1) / stride; }
 // to xp[b][H][Wp][4] (channels zero-padded to 4, `pad` zero columns on the
 // left, zeros up to Wp on the right).  GEMM row j = (r, atom, tap, c) of output
 // pixel (n,p,q) reads xp[n][st*p + r - pad][st*q + atom*tpa + tap][c]: one
-// 128-B window per (pixel, filter row, atom), windows starting st pixels
+// aw-byte window per (pixel, filter row, atom), windows starting st pixels
 // apart -- a plain strided view that TMA tiles directly.
-struct Win { int cpx, tpa, na, Wp, M; };
+struct Win { int cpx, aw, tpa, na, Wp, M; };  // aw: bytes per swizzle atom (128 / 64 / 32)
 bool win_tc(const Geom& g, int type);
 Win win_geom(const Geom& g);
 

@@ -24,12 +24,14 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
     constexpr bool HALO = (AM == A_HALO);
     const int A_BYTES = HALO ? 0 : p.mt * A_HALF;
     const int KD = KB * p.km;                // K rows per stage (MN-major modes)
-    constexpr bool A_MN = (AM == A_TMA_MN2 || AM == A_TMA_WIN);
+    constexpr bool WIN = (AM == A_TMA_WIN || AM == A_TMA_WIN64 || AM == A_TMA_WIN32);
+    constexpr uint32_t WAW = AM == A_TMA_WIN64 ? 64u : AM == A_TMA_WIN32 ? 32u : 128u;  // window atom bytes
+    constexpr bool A_MN = (AM == A_TMA_MN2 || WIN);
     constexpr bool B_MN = (BM_ == B_TMA_MN2 || BM_ == B_TMA_MN3 || BM_ == B_GATHER_WG || BM_ == B_SCALAR_DGRAD ||
                            BM_ == B_SCALAR_WG || BM_ == B_TMA_IM2COL || BM_ == B_GATHER_SMALLC ||
                            BM_ == B_GATHER_SMALLC_PAD || BM_ == B_TMA_DYROW);
     constexpr bool A_TMA = (AM == A_TMA_K2 || AM == A_TMA_K3 || AM == A_TMA_MN2 || AM == A_TMA_IM2COL ||
-                            AM == A_TMA_IM2COL_SMALLC || AM == A_TMA_WIN || AM == A_HALO);
+                            AM == A_TMA_IM2COL_SMALLC || WIN || AM == A_HALO);
     constexpr bool A_NOSWZ = (AM == A_TMA_IM2COL_SMALLC);  // unswizzled core matrices, one 2-KB box per tap
     constexpr bool B_TMA = (BM_ == B_TMA_K2 || BM_ == B_TMA_K3 || BM_ == B_TMA_MN2 || BM_ == B_TMA_MN3 ||
                             BM_ == B_TMA_IM2COL || BM_ == B_TMA_DYROW);
@@ -350,7 +352,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
             }
             // Window WGRAD: k-block kb = (output row n*P + p, q-block qb)
             int wr_row = 0, wr_qb = 0;
-            if constexpr (AM == A_TMA_WIN) { wr_row = kb_begin / p.win_qb; wr_qb = kb_begin - wr_row * p.win_qb; }
+            if constexpr (WIN) { wr_row = kb_begin / p.win_qb; wr_qb = kb_begin - wr_row * p.win_qb; }
             for (int kb = kb_begin; kb < kb_end; ++kb, ++git, s = (s + 1 == S) ? 0 : s + 1, ph ^= (s == 0) ? 1u : 0u) {
                 mbar_wait(smem_u32(&empty[s]), ph ^ 1u);
                 const uint32_t aT = smem_u32(sA + (size_t)s * A_BYTES);
@@ -385,16 +387,18 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                             for (int a = 0; a < 128 * ELT / 128; ++a)
                                 tma_load_2d(aH + a * KD * 128, &tmA, fb, mH + a * (128 / ELT), kb * KD);
                         }
-                        if constexpr (AM == A_TMA_WIN) {
+                        if constexpr (WIN) {
                             // atom ja = (filter row r, atom aa): window of KD output pixels of row
-                            // (n, p) at x row st*p + r - pad (rows past R load out of bounds: zeros)
+                            // (n, p) at x row st*p + r - pad (rows past R load out of bounds: zeros);
+                            // atoms of aw bytes, 128*ELT/aw of them per 128 rows
                             const int n_ = wr_row / p.P, p_ = wr_row - n_ * p.P;
+                            constexpr int wat = WAW / ELT;
 #pragma unroll
-                            for (int a = 0; a < 128 * ELT / 128; ++a) {
-                                const int ja = mH / (128 / ELT) + a;
+                            for (int a = 0; a < 128 * ELT / (int)WAW; ++a) {
+                                const int ja = mH / wat + a;
                                 const int r = ja / p.win_na, aa = ja - r * p.win_na;
                                 const int h = r < p.R ? p.stride * p_ + r - p.pad : -(1 << 20);
-                                tma_load_4d(aH + a * KD * 128, &tmA, fb, aa * (128 / ELT), wr_qb * KD, h, n_);
+                                tma_load_4d(aH + a * KD * WAW, &tmA, fb, aa * wat, wr_qb * KD, h, n_);
                             }
                         }
                         if constexpr (AM == A_TMA_IM2COL) {
@@ -434,7 +438,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                         }
                     }
                 }
-                if constexpr (AM == A_TMA_WIN) { if (++wr_qb == p.win_qb) { wr_qb = 0; ++wr_row; } }
+                if constexpr (WIN) { if (++wr_qb == p.win_qb) { wr_qb = 0; ++wr_row; } }
                 if constexpr (BM_ == B_TMA_IM2COL) {
                     wb_q += KD;
                     while (wb_q >= p.Q) { wb_q -= p.Q; if (++wb_p == p.P) { wb_p = 0; ++wb_n; } }
@@ -776,8 +780,13 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                                 const uint32_t aH = aT + hh * (A_MN ? (uint32_t)A_HALF : 16384u);
                                 // no-swizzle A: core matrices 8 rows x 16 B, SBO 128 B (rows),
                                 // LBO 2 KB (next tap); one MMA covers 32 B of K = 2 taps
+                                // window atoms of aw bytes: KD rows x aw per atom column, 8-row
+                                // groups aw*8 apart; UMMA swizzle 2 / 4 / 6 = 128 / 64 / 32 B
                                 const uint64_t ad =
-                                    A_NOSWZ ? sdesc(aH + j * 4096, 2048, 128, 0)
+                                    WIN && WAW < 128
+                                        ? sdesc(aH + (uint32_t)(jj * KB) * WAW + j * UMMA_K * WAW, KDm * WAW, 8 * WAW,
+                                                WAW == 64 ? 4u : 6u)
+                                    : A_NOSWZ ? sdesc(aH + j * 4096, 2048, 128, 0)
                                     : A_MN  ? sdesc(aH + kofs + j * UMMA_K * 128, KDm * 128, MN_SBO, MN_LAYOUT)
                                             : sdesc(aH + j * 32, 16, 1024);
                                 mma<ELT>(dtm + (uint32_t)(hh * p.BN), ad, bd, idesc,
@@ -926,7 +935,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                     }
                 } else if constexpr (EPI == EPI_WGRAD_WIN) {
                     // row m = (r, atom aa, tap t, channel c) -> dw[k][r][aa*taps + t][c], k = nb + j
-                    constexpr int per_atom = 128 / ELT;
+                    constexpr int per_atom = WAW / ELT;
                     const int ja = m / per_atom, e = m - ja * per_atom;
                     const int t = e / p.cp, c = e - t * p.cp;
                     const int r = ja / p.win_na, sx = (ja - r * p.win_na) * (per_atom / p.cp) + t;

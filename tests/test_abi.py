@@ -116,8 +116,9 @@ def test_workspace_space_to_depth():
     # 56 x 56 output super-pixels, 58 x 58 input super-pixels, filter 4K x 9 x 64.
     d = mu.desc(2, 3, 224, 224, 64, 7, 7, 3, 2, mu.MATH_BF16)
     assert mu.workspace_size(d, mu.FWD, mu.IM2COL_GEMM, 2) == a256(4 * 64 * 9 * 64 * 2) + a256(2 * 58 * 58 * 64 * 2)
-    # WGRAD window: tpa = 16, na = 1, Wp = max(2*111 + 16, 224 + 3) = 238 -> 240
-    assert mu.workspace_size(d, mu.BWD_FILTER, mu.IM2COL_GEMM, 2) == a256(2 * 224 * 240 * 4 * 2)
+    # WGRAD window: 64-B atoms (one 8-tap atom per filter row: 7*32 = 224 GEMM rows instead of
+    # 7*64 with 128-B atoms), tpa = 8, na = 1, Wp = max(2*111 + 8, 224 + 3) = 230 -> 232
+    assert mu.workspace_size(d, mu.BWD_FILTER, mu.IM2COL_GEMM, 2) == a256(2 * 224 * 232 * 4 * 2)
     # DGRAD: f = 4 (4*4*3 = 48 columns), Dr = 6 // 2 + 2 = 5: filter 48 x 25*64
     assert mu.workspace_size(d, mu.BWD_DATA, mu.IM2COL_GEMM, 2) == a256(48 * 25 * 64 * 2)
     # stride 3, BF16: 3*8 B is not a multiple of 16 -> WGRAD keeps the space-to-depth image

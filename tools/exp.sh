@@ -1,3 +1,4 @@
-timeout 900 python -m pytest tests -q -x -m gpu 2>&1 | tail -2
-timeout 120 python tools/time_one.py --config resnet50 --math bf16 --specs layer2.0.conv2:DGRAD:IG:256 layer3.0.conv2:DGRAD:IG:256 layer4.0.conv2:DGRAD:IG:256
-MUCU_MERGE_PHASES=0 timeout 120 python tools/time_one.py --config resnet50 --math bf16 --specs layer2.0.conv2:DGRAD:IG:256 layer3.0.conv2:DGRAD:IG:256 layer4.0.conv2:DGRAD:IG:256
+timeout 900 python -m pytest tests/test_conv_gpu.py -q -x -k "c3 or c2_k32" 2>&1 | tail -1
+timeout 120 python tools/time_one.py --config resnet50 --math bf16 --specs conv1:WGRAD:I2C:256 conv1:WGRAD:I2C:128
+timeout 120 python tools/time_one.py --config alexnet --math bf16 --specs conv1:WGRAD:I2C:256
+timeout 120 python tools/time_one.py --config alexnet --math tf32 --specs conv1:WGRAD:I2C:256

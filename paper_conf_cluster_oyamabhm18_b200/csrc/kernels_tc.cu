@@ -484,7 +484,12 @@ void finalize_tiling(Launch& L, int elt, int step = 32) {
 // per SM.
 void use_mt2(Launch& L, int num_sms) {
     TcArgs& a = L.a;
-    if (a.BN > 128 || env_int("MUCU_MT2", 1) == 0) return;
+    // Wide tiles (128 < BN <= 192): 256 x BN needs one accumulator set (the epilogue
+    // no longer overlaps the next tile), worth it for long reductions only; measured
+    // AlexNet conv2 FWD / conv3 DGRAD 0.19 / 0.22 -> 0.16 / 0.17 ms, while BN = 256
+    // (one 128 x 256 chain is already near the MMA floor) got slower.
+    const bool wide_ok = env_int("MUCU_MT2_WIDE", 1) && a.num_kb >= 32 && a.BN <= 192;
+    if ((a.BN > 128 && !wide_ok) || env_int("MUCU_MT2", 1) == 0) return;
     const int force = env_int("MUCU_FORCE_MT", 0);  // tests: exercise 256/512-row tiles on small shapes
     if (force == 4 && a.BN <= 64) num_sms = 1;
     if (force == 2) { a.mt = 2; size_stages(a); return; }

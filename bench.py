@@ -197,7 +197,7 @@ def main():
 
     import paper_conf_cluster_oyamabhm18_b200 as mu
     from paper_conf_cluster_oyamabhm18_b200.distributed import GradAllreduce, init_from_env, max_over_ranks
-    from paper_conf_cluster_oyamabhm18_b200.network import ConvNet, algorithmic_flops, layer_flops
+    from paper_conf_cluster_oyamabhm18_b200.network import ConvNet, algorithmic_bytes, algorithmic_flops, layer_flops
     from synthetic import network
 
     distributed = init_from_env("nccl")
@@ -321,19 +321,37 @@ def main():
     dom = max(op_ms, key=op_ms.get)
     li, lt = dom
     kern = net.kernels[dom]
-    alg_flops = algorithmic_flops(layers[li], lt, kern.plan)
-    achieved = alg_flops / (op_ms[dom] * 1e-3) / 1e12
     bf16_peak = peaks.get("bf16_tflops", 1590.0)
+    hbm_peak = peaks.get("hbm_gbs", 6650.0)
+    elt = 2 if math == mu.MATH_BF16 else 4
     if math == mu.MATH_BF16:
-        peak, bound, punit = bf16_peak, "tensor", "TFLOP/s"
+        tpeak, tbound = bf16_peak, "tensor"
         peak_note = f"bf16 dense {peaks_src} (burst)"
     elif math == mu.MATH_TF32:
-        peak, bound, punit = bf16_peak * 0.5, "tensor", "TFLOP/s"
+        tpeak, tbound = bf16_peak * 0.5, "tensor"
         peak_note = f"tf32 = {peaks_src} bf16 burst x nominal tf32/bf16 ratio 1.125/2.25"
     else:
         sm_mhz = peaks.get("sm_max_mhz", 1965.0)
-        peak, bound, punit = 148 * 128 * 2 * sm_mhz * 1e6 / 1e12, "alu", "TFLOP/s"
+        tpeak, tbound = 148 * 128 * 2 * sm_mhz * 1e6 / 1e12, "alu"
         peak_note = "fp32 FFMA: 148 SM x 128 lanes x 2 flop x max SM clock"
+
+    def floor_ms(i, t, plan):
+        """Roofline floor of one op: max(F / compute peak, B / HBM peak)."""
+        f = algorithmic_flops(layers[i], t, plan)
+        b = algorithmic_bytes(layers[i], t, args.batch, elt)
+        return max(f / (tpeak * 1e12), b / (hbm_peak * 1e9)) * 1e3, f, b
+
+    # The dominant op is bounded by whichever of its compute / byte floors is
+    # larger; achieved = that algorithmic work / the op's mean CUDA-event time.
+    _, alg_flops, alg_bytes = floor_ms(li, lt, kern.plan)
+    if alg_bytes / (hbm_peak * 1e9) > alg_flops / (tpeak * 1e12):
+        bound, punit, peak = "hbm", "GB/s", hbm_peak
+        achieved = alg_bytes / (op_ms[dom] * 1e-3) / 1e9
+        peak_note = f"HBM copy bandwidth, {peaks_src} (MEASURED_PEAKS.json hbm_gbs)"
+    else:
+        bound, punit, peak = tbound, "TFLOP/s", tpeak
+        achieved = alg_flops / (op_ms[dom] * 1e-3) / 1e12
+    step_floor = sum(floor_ms(i, t, k.plan)[0] for (i, t), k in net.kernels.items() if (i, t) in op_ms)
     traffic = None
     tp = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(tp):
@@ -371,8 +389,10 @@ def main():
                          "frac": round(achieved / peak, 4), "traffic": traffic,
                          "kernel": f"{layers[li].name} {mu.TYPE_NAMES[lt]} plan="
                                    f"{[(mu.ALGO_NAMES[a], b) for a, b in kern.plan]}",
-                         "algorithmic_flops": alg_flops, "avg_ms": round(op_ms[dom], 4),
-                         "share_of_step": round(op_ms[dom] / ms, 4), "peak_source": peak_note},
+                         "algorithmic_flops": alg_flops, "algorithmic_bytes": alg_bytes,
+                         "avg_ms": round(op_ms[dom], 4),
+                         "share_of_step": round(op_ms[dom] / ms, 4), "peak_source": peak_note,
+                         "step_floor_ms": round(step_floor, 4), "step_frac": round(step_floor / ms, 4)},
             "cpu_baseline": cb,
             "e2e": {"value": round(e2e_ms, 4), "unit": "ms/iter", "h2d_bytes_per_step": int(h2d_bytes),
                     "d2h_bytes_per_step": int(d2h_bytes)},

@@ -605,6 +605,19 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         const int64_t nkb = qrow ? (int64_t)b * g.p * A.win_qb : ceil_div(A.kred, KB * A.km);
         int64_t nsplit = std::min<int64_t>(std::min<int64_t>(std::max<int64_t>(1, (2LL * num_sms) / tiles),
                                                              std::max<int64_t>(1, nkb / 16)), 65535);
+        if (env_int("MUCU_SPLIT_WAVES", 1)) {
+            // Wave-quantised split count: minimise waves x (stages per split + the
+            // per-split epilogue / pipeline fill, ~E stages of 128-B k-blocks),
+            // splits >= 4 stages each.  (Capping at 16 stages per split left e.g.
+            // ResNet-50 layer4 1x1 WGRAD at 192 units on 148 SMs.)
+            const double E = env_int("MUCU_SPLIT_E", 16) / (double)A.km;
+            double best = 1e30;
+            const int64_t smax = std::min<int64_t>(std::max<int64_t>(1, nkb / 4), std::min<int64_t>(65535, 4LL * num_sms));
+            for (int64_t sp = 1; sp <= smax; ++sp) {
+                const double cost = (double)ceil_div(tiles * sp, num_sms) * ((double)ceil_div(nkb, sp) + E);
+                if (cost < best - 1e-9) { best = cost; nsplit = sp; }
+            }
+        }
         A.kb_per_split = (int)ceil_div(nkb, nsplit);
         nsplit = ceil_div(nkb, A.kb_per_split);
         A.num_kb = (int)nkb;

@@ -62,6 +62,17 @@ def algorithmic_flops(layer, conv_type: int, plan) -> int:
     return f
 
 
+def algorithmic_bytes(layer, conv_type: int, n: int, elt: int) -> int:
+    """HBM bytes the convolution must move once (SURVEY 8(d) "IG: x + w + y"):
+    the operands and the result, no workspace; dW is fp32 (written once, beta = 0)."""
+    x = n * layer.h * layer.w * layer.c * elt
+    y = n * layer.p * layer.q * layer.k * elt
+    w = layer.k * layer.r * layer.s * layer.c * elt
+    if conv_type == L.BWD_FILTER:
+        return x + y + layer.k * layer.r * layer.s * layer.c * 4
+    return x + y + w
+
+
 class ConvNet:
     def __init__(self, handle: L.Handle, layers: Sequence, n: int, math: int, device: str = "cuda"):
         self.h = handle

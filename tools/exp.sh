@@ -1,4 +1,7 @@
-for w in 0 1; do echo "== WIDE=$w"
-MUCU_MT2_WIDE=$w timeout 120 python tools/time_one.py --config alexnet --math tf32 --specs conv2:FWD:IG:256 conv3:FWD:IG:256 conv3:DGRAD:IG:256 conv4:FWD:IG:256 conv4:DGRAD:IG:256 conv5:FWD:IG:256 conv5:DGRAD:IG:256 conv1:FWD:I2C:64
-MUCU_MT2_WIDE=$w timeout 120 python tools/time_one.py --config resnet50 --math bf16 --specs layer3.1.conv2:FWD:IG:256 layer3.1.conv2:DGRAD:IG:256 layer4.1.conv2:FWD:IG:256 layer4.1.conv2:DGRAD:IG:256 layer2.1.conv2:FWD:IG:256 layer3.0.conv2:DGRAD:IG:256 conv1:FWD:I2C:128
+#!/bin/bash
+set -u
+source tools/specs.sh
+for env in "MUCU_SPLIT_WAVES=0" "MUCU_SPLIT_WAVES=1" "MUCU_SPLIT_E=8" "MUCU_SPLIT_E=32" "MUCU_SPLIT_E=16 MUCU_KM=1"; do echo "== $env"
+env $env timeout 120 python tools/time_one.py --config resnet50 --math bf16 --specs $SP_resnet50
+env $env timeout 120 python tools/time_one.py --config alexnet --math tf32 --specs $SP_alexnet
 done

@@ -423,11 +423,21 @@ bool use_tma_im2col() {
 // atom when a tile must not split a 128-B channel atom) up to 256, minimising
 // the padded columns plus a per-tile overhead (~32 columns, or the A rows a
 // tile re-reads); ties -> larger.
-int pick_bn(int N, int step = 32, int overhead = 32, int max_bn = 256) {
+// With mtiles > 0 (persistent FWD / DGRAD launches) the cost counts whole
+// waves of tiles over the SMs: time ~ waves x (bn + 128), so e.g. ResNet-50
+// layer4 (98 row tiles, N = 512) takes 3 x 192 (2 waves) instead of 2 x 256
+// (196 tiles = 1.3 waves): DGRAD 0.095 -> 0.077 ms.
+int g_num_sms = 148;
+int pick_bn(int N, int step = 32, int overhead = 32, int max_bn = 256, int64_t mtiles = 0) {
     step = std::max(step, 32);  // the epilogue drains TMEM in 32-column chunks
-    int best = step, best_cost = 1 << 30;
+    int best = step;
+    int64_t best_cost = INT64_MAX;
+    const bool waves = mtiles > 0 && env_int("MUCU_BN_WAVES", 1);
     for (int bn = step; bn <= max_bn; bn += step) {
-        const int cost = (int)ceil_div(N, bn) * (bn + overhead);
+        const int64_t nt = ceil_div(N, bn);
+        // per-tile cost in wave mode: narrow tiles run well below the MMA rate of wide
+        // ones (one 128 x 64 chain ~ 0.7x the time of a 128 x 256 one), hence +128
+        const int64_t cost = waves ? ceil_div(mtiles * nt, g_num_sms) * (bn + 128) : nt * (bn + overhead);
         if (cost <= best_cost) { best = bn; best_cost = cost; }
     }
     return best;
@@ -451,7 +461,22 @@ int launch_t(Launch& L, cudaStream_t st) {
         if (e) return (int)e;
         configured = 232448;
     }
-    kern<<<L.grid, kThreads, smem, st>>>(L.a, L.ta, L.tb);
+    // Programmatic dependent launch (MUCU_PDL=0 disables): the kernel may start
+    // (prologue only -- it executes griddepcontrol.wait before touching global
+    // memory) while the previous kernel on the stream drains its last wave.
+    static const int pdl = env_int("MUCU_PDL", 1);
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = L.grid;
+    cfg.blockDim = dim3(kThreads);
+    cfg.dynamicSmemBytes = (size_t)smem;
+    cfg.stream = st;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = pdl ? 1 : 0;
+    cudaError_t le = cudaLaunchKernelEx(&cfg, kern, L.a, L.ta, L.tb);
+    if (le) return (int)le;
     count_launch();
     return (int)cudaGetLastError();
 }
@@ -466,9 +491,9 @@ void size_stages(TcArgs& a) {
     if (a.stages < 2) a.stages = 2;
 }
 
-void finalize_tiling(Launch& L, int elt, int step = 32) {
+void finalize_tiling(Launch& L, int elt, int step = 32, int batch = 1) {
     TcArgs& a = L.a;
-    a.BN = pick_bn(a.N, step);
+    a.BN = pick_bn(a.N, step, 32, 256, ceil_div(a.M, 128) * batch);
     if (const int fb = env_int("MUCU_FORCE_BN", 0)) a.BN = std::max(step, fb - fb % step);
     a.bn_atoms = (a.BN * elt + 127) / 128;
     a.b_bytes = std::max(a.BN * 128, a.bn_atoms * (128 / elt) * 128);
@@ -542,6 +567,7 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
     const int elt = elt_size(g.math);
     const int KB = 128 / elt;
     const int atom = 128 / elt;
+    g_num_sms = num_sms;
     const bool bf = g.math == MUCU_MATH_BF16;
     const int64_t PQ = (int64_t)g.p * g.q, HW = (int64_t)g.h * g.w;
     const int RS = g.r * g.s;
@@ -859,7 +885,7 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         if (err) return err;
         A.M = (int)Tt; A.N = O; A.num_kb = (int)ceil_div(I, KB); A.ldc = O;
         A.batch_stride = Tt * O; A.alpha = 1.f; A.beta = 0.f; A.out = Mx; A.out_bf16 = 0;
-        finalize_tiling(L, elt);
+        finalize_tiling(L, elt, 32, 16);
         grid2(16);
         if (!map3(&L.ta, V, I, Tt, 16, I, Tt * I, KB, 128, 1)) return -1;
         if (!map3(&L.tb, ws, I, O, 16, I, (uint64_t)O * I, KB, A.BN, 1)) return -1;

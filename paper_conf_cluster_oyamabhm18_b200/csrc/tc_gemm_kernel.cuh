@@ -96,6 +96,11 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
     __syncthreads();
     tc_fence_after();
     const uint32_t tmem = *tmem_slot;
+    // Programmatic dependent launch: the prologue above (barrier init, TMEM
+    // allocation) overlaps the previous kernel's tail; wait for its results
+    // before the first global access, then let the next launch start its own.
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+    asm volatile("griddepcontrol.launch_dependents;" :::);
 
     // tile -> (m0, n0, z, k-block range)
     auto decode = [&](int tile, int& m0, int& n0, int& z, int& kb_begin, int& kb_end) {

@@ -1,7 +1,10 @@
 #!/bin/bash
 set -u
-source tools/specs.sh
-for env in "MUCU_SPLIT_WAVES=0" "MUCU_SPLIT_WAVES=1" "MUCU_SPLIT_E=8" "MUCU_SPLIT_E=32" "MUCU_SPLIT_E=16 MUCU_KM=1"; do echo "== $env"
-env $env timeout 120 python tools/time_one.py --config resnet50 --math bf16 --specs $SP_resnet50
-env $env timeout 120 python tools/time_one.py --config alexnet --math tf32 --specs $SP_alexnet
-done
+timeout 900 python -m pytest tests -q -m gpu -x 2>&1 | tail -2
+for rep in 1 2; do for pdl in 0 1; do
+  for cfg in "resnet50 bf16" "alexnet tf32"; do set -- $cfg
+  MUCU_PDL=$pdl timeout 300 python bench.py --config $1 --math $2 --no-cpu-baseline --tables-in scratch/tables_$1_$2.npz --steps 20 2>/dev/null | python -c "
+import json,sys
+d=json.loads(sys.stdin.readlines()[-1]); print('PDL=$pdl $1 $2', d['value'], d['e2e']['value'], d['roofline']['step_frac'], d['clocks']['reasons'])"
+  done
+done; done

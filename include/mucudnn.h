@@ -142,9 +142,10 @@ mucu_status_t mucu_output_dims(const mucu_conv_desc_t* desc, int32_t* p, int32_t
  *                          else 1, f = st*u, Dr = ceil(R/st) - 1 + u, Ds likewise: f*f*C*Dr*Ds*K*elt
  *   WG  FWD:          16*K*C*elt + 16*b*T*C*elt + 16*b*T*K*4,   T = ceil(P/2)*ceil(Q/2)
  *   WG  DGRAD:        16*C*K*elt + 16*b*T'*K*elt + 16*b*T'*C*4, T' = ceil(H/2)*ceil(W/2)
+ *   WG  WGRAD:        F(3x3,2x2), Tp = b*T rounded up to 256, Cp / Kp = C / K
+ *                     rounded up to 128/elt:  16*Tp*Cp*elt + 16*Tp*Kp*elt + 16*Kp*Cp*4
  * ceil_e rounds up to a multiple of 16/elt elements.  UNSUPPORTED if the
- * algorithm is ineligible (WG needs R=S=3, stride 1, pad <= 2, and is not
- * implemented for BWD_FILTER). */
+ * algorithm is ineligible (WG needs R=S=3, stride 1, pad <= 2). */
 mucu_status_t mucu_workspace_size(const mucu_conv_desc_t* desc, mucu_conv_type_t type,
                                   mucu_algo_t algo, int32_t micro_n, uint64_t* bytes);
 

@@ -144,9 +144,9 @@ bool algo_eligible(const Geom& g, int type, int algo) {
         case MUCU_ALGO_IM2COL_GEMM:
             return true;
         case MUCU_ALGO_WINOGRAD_2X2_3X3:
-            // F(2x2,3x3): 3x3 filters, unit stride (ref [23]); BackwardFilter
-            // Winograd is NEXT-1 (not implemented); pad' = 2 - pad >= 0 for DGRAD.
-            return g.r == 3 && g.s == 3 && g.stride == 1 && g.pad <= 2 && type != MUCU_BWD_FILTER;
+            // F(2x2,3x3): 3x3 filters, unit stride (ref [23]); pad' = 2 - pad >= 0 for
+            // DGRAD.  BackwardFilter runs the transposed F(3x3,2x2).
+            return g.r == 3 && g.s == 3 && g.stride == 1 && g.pad <= 2;
         default:
             return false;
     }
@@ -216,6 +216,21 @@ mucu_status_t ws_layout(const Geom& g, int type, int algo, int32_t b, WsLayout* 
             L->a_bytes = align_up((uint64_t)b * PQ * (uint64_t)L->kpitch * elt, 256);
         }
         L->total = L->a_off + L->a_bytes;
+        return MUCU_OK;
+    }
+    if (type == MUCU_BWD_FILTER) {
+        // Winograd F(3x3,2x2) BackwardFilter: V = B^T x B [16][Tp][C] | D = A dy A^T
+        // [16][Tp][K] | M [16][K][C] fp32; T = b*ceil(P/2)*ceil(Q/2) tiles padded to
+        // Tp = a multiple of 256 (zero rows: whole TMA k-blocks per plane).
+        // Channel pitches Cp, Kp: C, K rounded up to 128 B (zero channels), the TMA atom.
+        const uint64_t Tp = align_up((uint64_t)b * ((g.p + 1) / 2) * ((g.q + 1) / 2), 256);
+        const uint64_t Cp = align_up((uint64_t)g.c, 128 / elt), Kp = align_up((uint64_t)g.k, 128 / elt);
+        L->a_off = 0;
+        L->a_bytes = align_up(16 * Tp * Cp * elt, 256);
+        L->b_off = L->a_bytes;
+        L->b_bytes = align_up(16 * Tp * Kp * elt, 256);
+        L->fixed_off = L->b_off + L->b_bytes;  // M (per call, not b-independent)
+        L->total = L->fixed_off + align_up(16 * Kp * Cp * 4, 256);
         return MUCU_OK;
     }
     // Winograd F(2x2,3x3): U (b-independent) | V | M (fp32).
@@ -317,7 +332,16 @@ mucu_status_t run_micro(Handle* hd, const Geom& g, int type, int algo, int32_t b
             if (!e) e = launch_wg_output(g, true, b, alpha, Mx, beta, fo, st);
         }
     } else {  // MUCU_BWD_FILTER: in0 = x, in1 = dy, out = dw (fp32)
-        if (algo == MUCU_ALGO_IMPLICIT_GEMM) {
+        if (algo == MUCU_ALGO_WINOGRAD_2X2_3X3) {
+            // M_xi[k][c] = sum_t D[xi][t][k] V[xi][t][c] (16 batched GEMMs over the tiles)
+            const int64_t Tp = (int64_t)align_up((uint64_t)b * ((g.p + 1) / 2) * ((g.q + 1) / 2), 256);
+            float* V = (float*)(wsb + L.a_off);
+            float* D = (float*)(wsb + L.b_off);
+            float* Mx = (float*)(wsb + L.fixed_off);
+            e = launch_wgw_transforms(g, b, f0, f1, V, D, Tp, st);
+            if (!e) e = simt_gemm_tt(g.k, g.c, Tp, V, D, Mx, Tp, st);  // F32: Cp = C, Kp = K (mult. of 32 or padded)
+            if (!e) e = launch_wgw_output(g, alpha, Mx, beta, fo, st);
+        } else if (algo == MUCU_ALGO_IMPLICIT_GEMM) {
             e = simt_wgrad(g, b, alpha, f1, f0, false, 0, beta, fo, sem, hd->num_sms, st);
         } else {
             if (is_pointwise(g)) {

@@ -176,6 +176,116 @@ __global__ void wg_output_kernel(const float* __restrict__ M, T* __restrict__ ou
     }
 }
 
+// Winograd F(3x3,2x2) BackwardFilter: per 2x2 tile of dy at
+// (2th, 2tw) and the 4x4 x patch at (2th - pad, 2tw - pad),
+//   dW[r][s] += (G^T [(A dy A^T) .* (B^T x B)] G)[r][s],
+// A = [[1,0],[1,1],[1,-1],[0,-1]] (the transpose of F(2x2,3x3)'s A^T), B^T and G
+// as in F(2x2,3x3).  V[xi][t][c] = (B^T x B)[xi], D[xi][t][k] = (A dy A^T)[xi];
+// rows t in [tiles, Tp) are zero so the GEMMs can read whole k-blocks.
+template <class T>
+__global__ void wgw_x_kernel(const T* __restrict__ x, T* __restrict__ V, int64_t tiles, int64_t Tp, int H, int W,
+                             int C, int Cp, int TH, int TW, int pad) {
+    const int64_t total = Tp * Cp, plane = Tp * Cp;
+    for (int64_t idx = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; idx < total;
+         idx += (int64_t)gridDim.x * blockDim.x) {
+        const int c = (int)(idx % Cp);
+        const int64_t t = idx / Cp;
+        float d[4][4];
+        if (t < tiles && c < C) {
+            const int tw = (int)(t % TW);
+            const int64_t t2 = t / TW;
+            const int th = (int)(t2 % TH), n = (int)(t2 / TH);
+            for (int a = 0; a < 4; ++a)
+                for (int b = 0; b < 4; ++b) {
+                    const int h = 2 * th - pad + a, w = 2 * tw - pad + b;
+                    d[a][b] = (h >= 0 && h < H && w >= 0 && w < W) ? to_f<T>(x[(((int64_t)n * H + h) * W + w) * C + c])
+                                                                   : 0.f;
+                }
+        } else {
+            for (int a = 0; a < 4; ++a)
+                for (int b = 0; b < 4; ++b) d[a][b] = 0.f;
+        }
+        float e[4][4];  // e = B^T d
+        for (int b = 0; b < 4; ++b) {
+            e[0][b] = d[0][b] - d[2][b];
+            e[1][b] = d[1][b] + d[2][b];
+            e[2][b] = d[2][b] - d[1][b];
+            e[3][b] = d[1][b] - d[3][b];
+        }
+        for (int a = 0; a < 4; ++a) {  // v = e B
+            V[(a * 4 + 0) * plane + idx] = from_f<T>(e[a][0] - e[a][2]);
+            V[(a * 4 + 1) * plane + idx] = from_f<T>(e[a][1] + e[a][2]);
+            V[(a * 4 + 2) * plane + idx] = from_f<T>(e[a][2] - e[a][1]);
+            V[(a * 4 + 3) * plane + idx] = from_f<T>(e[a][1] - e[a][3]);
+        }
+    }
+}
+
+template <class T>
+__global__ void wgw_dy_kernel(const T* __restrict__ dy, T* __restrict__ D, int64_t tiles, int64_t Tp, int P, int Q,
+                              int K, int Kp, int TH, int TW) {
+    const int64_t total = Tp * Kp, plane = Tp * Kp;
+    for (int64_t idx = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; idx < total;
+         idx += (int64_t)gridDim.x * blockDim.x) {
+        const int k = (int)(idx % Kp);
+        const int64_t t = idx / Kp;
+        float g[2][2] = {{0.f, 0.f}, {0.f, 0.f}};
+        if (t < tiles && k < K) {
+            const int tw = (int)(t % TW);
+            const int64_t t2 = t / TW;
+            const int th = (int)(t2 % TH), n = (int)(t2 / TH);
+            for (int j = 0; j < 2; ++j)
+                for (int l = 0; l < 2; ++l) {
+                    const int p = 2 * th + j, q = 2 * tw + l;
+                    if (p < P && q < Q) g[j][l] = to_f<T>(dy[(((int64_t)n * P + p) * Q + q) * K + k]);
+                }
+        }
+        float e[4][2];  // e = A g
+        for (int l = 0; l < 2; ++l) {
+            e[0][l] = g[0][l];
+            e[1][l] = g[0][l] + g[1][l];
+            e[2][l] = g[0][l] - g[1][l];
+            e[3][l] = -g[1][l];
+        }
+        for (int a = 0; a < 4; ++a) {  // (A g) A^T
+            D[(a * 4 + 0) * plane + idx] = from_f<T>(e[a][0]);
+            D[(a * 4 + 1) * plane + idx] = from_f<T>(e[a][0] + e[a][1]);
+            D[(a * 4 + 2) * plane + idx] = from_f<T>(e[a][0] - e[a][1]);
+            D[(a * 4 + 3) * plane + idx] = from_f<T>(-e[a][1]);
+        }
+    }
+}
+
+// dw[k][r][s][c] = alpha * (G^T M[.][k][c] G)[r][s] + beta * dw (beta = 0: no read).
+__global__ void wgw_out_kernel(const float* __restrict__ M, float* __restrict__ dw, int K, int C, int Kp, int Cp,
+                               float alpha, float beta) {
+    const int64_t total = (int64_t)K * C, plane = (int64_t)Kp * Cp;
+    for (int64_t idx = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; idx < total;
+         idx += (int64_t)gridDim.x * blockDim.x) {
+        const int c = (int)(idx % C), k = (int)(idx / C);
+        const int64_t mi = (int64_t)k * Cp + c;
+        float m[4][4];
+        for (int a = 0; a < 4; ++a)
+            for (int b = 0; b < 4; ++b) m[a][b] = M[(a * 4 + b) * plane + mi];
+        float z[3][4];  // z = G^T m
+        for (int b = 0; b < 4; ++b) {
+            z[0][b] = m[0][b] + 0.5f * (m[1][b] + m[2][b]);
+            z[1][b] = 0.5f * (m[1][b] - m[2][b]);
+            z[2][b] = 0.5f * (m[1][b] + m[2][b]) + m[3][b];
+        }
+        for (int r = 0; r < 3; ++r) {  // z G
+            const float o[3] = {z[r][0] + 0.5f * (z[r][1] + z[r][2]), 0.5f * (z[r][1] - z[r][2]),
+                                0.5f * (z[r][1] + z[r][2]) + z[r][3]};
+            for (int s2 = 0; s2 < 3; ++s2) {
+                float* d = dw + (((int64_t)k * 3 + r) * 3 + s2) * C + c;
+                float v = alpha * o[s2];
+                if (beta != 0.f) v += beta * *d;
+                *d = v;
+            }
+        }
+    }
+}
+
 // Row-oriented im2col: one warp per col row (output pixel m = (n,p,q)).  For
 // a fixed filter row r the S*C values (s,c) of the row are CONTIGUOUS in NHWC
 // x (x[n, h0+r, w0 .. w0+S-1, 0..C-1]), so the warp copies R runs of S*C
@@ -650,6 +760,37 @@ int launch_s2d_filter(const Geom& g, bool dgrad, const S2d& z, const void* w, vo
     else
         s2d_filter_kernel<float><<<grid, 256, 0, st>>>((const float*)w, (float*)out, total, g.k, g.r, g.s, g.c,
                                                        g.stride, z.f, z.u, z.Dr, z.Ds, z.Cs, dgrad);
+    count_launch();
+    return (int)cudaGetLastError();
+}
+
+int launch_wgw_transforms(const Geom& g, int32_t b, const void* x, const void* dy, void* V, void* D, int64_t Tp,
+                          cudaStream_t st) {
+    const int TH = (g.p + 1) / 2, TW = (g.q + 1) / 2;
+    const int64_t tiles = (int64_t)b * TH * TW;
+    const int at = 128 / elt_size(g.math);
+    const int Cp = (int)align_up((uint64_t)g.c, (uint64_t)at), Kp = (int)align_up((uint64_t)g.k, (uint64_t)at);
+    if (g.math == MUCU_MATH_BF16) {
+        wgw_x_kernel<__nv_bfloat16><<<grid_for(Tp * Cp, 256), 256, 0, st>>>(
+            (const __nv_bfloat16*)x, (__nv_bfloat16*)V, tiles, Tp, g.h, g.w, g.c, Cp, TH, TW, g.pad);
+        count_launch();
+        wgw_dy_kernel<__nv_bfloat16><<<grid_for(Tp * Kp, 256), 256, 0, st>>>(
+            (const __nv_bfloat16*)dy, (__nv_bfloat16*)D, tiles, Tp, g.p, g.q, g.k, Kp, TH, TW);
+    } else {
+        wgw_x_kernel<float><<<grid_for(Tp * Cp, 256), 256, 0, st>>>((const float*)x, (float*)V, tiles, Tp, g.h, g.w,
+                                                                    g.c, Cp, TH, TW, g.pad);
+        count_launch();
+        wgw_dy_kernel<float><<<grid_for(Tp * Kp, 256), 256, 0, st>>>((const float*)dy, (float*)D, tiles, Tp, g.p,
+                                                                     g.q, g.k, Kp, TH, TW);
+    }
+    count_launch();
+    return (int)cudaGetLastError();
+}
+
+int launch_wgw_output(const Geom& g, float alpha, const float* M, float beta, float* dw, cudaStream_t st) {
+    const int at = 128 / elt_size(g.math);
+    const int Cp = (int)align_up((uint64_t)g.c, (uint64_t)at), Kp = (int)align_up((uint64_t)g.k, (uint64_t)at);
+    wgw_out_kernel<<<grid_for((int64_t)g.k * g.c, 256), 256, 0, st>>>(M, dw, g.k, g.c, Kp, Cp, alpha, beta);
     count_launch();
     return (int)cudaGetLastError();
 }

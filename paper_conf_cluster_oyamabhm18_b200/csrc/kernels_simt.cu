@@ -354,4 +354,14 @@ int simt_wgrad(const Geom& g, int32_t b, float alpha, const float* dy, const flo
     return (int)cudaGetLastError();
 }
 
+// Winograd BackwardFilter GEMMs: M[z][k][c] = sum_t D[z][t][k] * V[z][t][c], z < 16.
+int simt_gemm_tt(int64_t K, int64_t C, int64_t Tp, const float* V, const float* D, float* M, int64_t ldt,
+                 cudaStream_t st) {
+    const int64_t Kp = (K + 31) / 32 * 32, Cp = (C + 31) / 32 * 32;  // channel pitches (128 B of fp32)
+    Dense a{D, K, Tp, 1, Kp, ldt * Kp};   // A(k, t) = D[z][t][k]
+    Dense bb{V, C, Tp, 1, Cp, ldt * Cp};  // B(c, t) = V[z][t][c]
+    StoreDense e{M, K, C, Cp, Kp * Cp, 1.f, 0.f};
+    return dispatch_gemm<false, false>(a, bb, e, K, C, Tp, 16, st);
+}
+
 }  // namespace mucu

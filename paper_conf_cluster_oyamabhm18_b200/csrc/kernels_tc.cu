@@ -255,6 +255,9 @@ struct TcArgs {
     // Halo IG (A_HALO): extended grid of hx_H = Ho + R - 1 rows x hx_W (>= Wo + S - 1, multiple of 8)
     // columns per image; source origin offset hx_pe; hx_nch channel chunks of 128 B; halo ring
     int hx_W, hx_H, hx_Ho, hx_Wo, hx_pe, hx_nch, halo_bytes, hstages;
+    // Batched split-K (Winograd BackwardFilter): blockIdx-tile batch z = b * zsplit + split;
+    // batch b reads operand rows from b * zrows and writes out + b * batch_stride.
+    int zsplit, zrows;
     // epilogue
     void* out;
     long long ldc;
@@ -868,6 +871,34 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         if (!map2(&L.tb, wp, RSC, g.k, wpitch, KB, A.BN)) return -1;
         A.tma_bytes = 16384 * A.mt + A.BN * 128;
         return LAUNCH(A_TMA_K2, B_TMA_K2, EPI_STORE);
+    }
+    if (algo == MUCU_ALGO_WINOGRAD_2X2_3X3 && type == MUCU_BWD_FILTER) {
+        // Winograd F(3x3,2x2) BackwardFilter: transforms, then 16 GEMMs
+        // M_xi[k][c] = sum_t D_xi[t][k] V_xi[t][c] as one batched split-K launch
+        // (z = xi * splits + split, fp32 reductions into the zeroed M), then
+        // dw = alpha * G^T M G + beta * dw.
+        const int Cp = (int)align_up((uint64_t)g.c, (uint64_t)atom), Kp = (int)align_up((uint64_t)g.k, (uint64_t)atom);
+        const int64_t Tp = (int64_t)align_up((uint64_t)b * ((g.p + 1) / 2) * ((g.q + 1) / 2), 256);
+        if (16 * Tp > INT32_MAX) return -1;
+        void* V = ws + WL.a_off;
+        void* D = ws + WL.b_off;
+        float* Mx = (float*)(ws + WL.fixed_off);
+        err = launch_wgw_transforms(g, b, in0, in1, V, D, Tp, st);
+        if (err) return err;
+        err = launch_scale(16LL * Kp * Cp, 0.f, Mx, st);
+        if (err) return err;
+        A.M = g.k; A.N = g.c; A.ldc = Cp; A.kred = (int)Tp; A.out = Mx; A.alpha = 1.f; A.beta = 0.f; A.out_bf16 = 0;
+        A.batch_stride = (long long)Kp * Cp;
+        wgrad_tiling(16, true);
+        const int nsplit = A.num_z;
+        A.zsplit = nsplit; A.zrows = (int)Tp;
+        grid2(16 * nsplit);
+        if (!map2(&L.ta, D, Kp, 16 * Tp, Kp, atom, KB * A.km, true)) return -1;
+        if (!map2(&L.tb, V, Cp, 16 * Tp, Cp, atom, KB * A.km, true)) return -1;
+        A.tma_bytes = A.km * (A.mt * 128 * KB * elt + A.bn_atoms * KB * 128);
+        err = LAUNCH(A_TMA_MN2, B_TMA_MN2, EPI_WGRAD_CHAIN);
+        if (err) return err;
+        return launch_wgw_output(g, alpha, Mx, beta, (float*)out, st);
     }
     if (algo == MUCU_ALGO_WINOGRAD_2X2_3X3) {
         const bool dg = type == MUCU_BWD_DATA;

@@ -124,6 +124,15 @@ int launch_s2d_filter(const Geom& g, bool dgrad, const S2d& z, const void* w, vo
 int launch_wg_input(const Geom& g, bool dgrad, int32_t b, const void* in, void* V, cudaStream_t st);
 int launch_wg_output(const Geom& g, bool dgrad, int32_t b, float alpha, const float* M, float beta,
                      void* out, cudaStream_t st);
+// Winograd F(3x3,2x2) BackwardFilter: V[16][Tp][C] = B^T x B and
+// D[16][Tp][K] = A dy A^T per 2x2 output tile (rows >= b*T zeroed), then
+// dw = alpha * G^T M G + beta * dw with M[16][K][C] fp32.
+int launch_wgw_transforms(const Geom& g, int32_t b, const void* x, const void* dy, void* V, void* D, int64_t Tp,
+                          cudaStream_t st);
+int launch_wgw_output(const Geom& g, float alpha, const float* M, float beta, float* dw, cudaStream_t st);
+// F32: M[z][k][c] = sum_t D[z][t][k] * V[z][t][c], z < 16 (SIMT).
+int simt_gemm_tt(int64_t K, int64_t C, int64_t Tp, const float* V, const float* D, float* M, int64_t ldt,
+                 cudaStream_t st);
 
 // tcgen05 tensor-core path (kernels_tc.cu) for MUCU_MATH_TF32 / MUCU_MATH_BF16:
 // runs one micro-configuration; returns a cudaError_t, or -1 if this

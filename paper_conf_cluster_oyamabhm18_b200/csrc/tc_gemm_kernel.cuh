@@ -111,7 +111,9 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
         n0 = ntile * p.BN;
         kb_begin = 0; kb_end = p.ph_n ? p.ph_kbv[z] : p.num_kb;
         if (SPLITK) {
-            kb_begin = z * p.kb_per_split;
+            // batched split-K (Winograd BackwardFilter): z = batch * zsplit + split
+            const int sp = p.zsplit ? z % p.zsplit : z;
+            kb_begin = sp * p.kb_per_split;
             kb_end = min(p.num_kb, kb_begin + p.kb_per_split);
         }
     };
@@ -388,9 +390,10 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                         if constexpr (AM == A_TMA_K2) tma_load_2d(aH, &tmA, fb, kb * KB, mH);
                         if constexpr (AM == A_TMA_K3) tma_load_3d(aH, &tmA, fb, kb * KB, mH, z);
                         if constexpr (AM == A_TMA_MN2) {
+                            const int zr = p.zsplit ? (z / p.zsplit) * p.zrows : 0;
 #pragma unroll
                             for (int a = 0; a < 128 * ELT / 128; ++a)
-                                tma_load_2d(aH + a * KD * 128, &tmA, fb, mH + a * (128 / ELT), kb * KD);
+                                tma_load_2d(aH + a * KD * 128, &tmA, fb, mH + a * (128 / ELT), zr + kb * KD);
                         }
                         if constexpr (WIN) {
                             // atom ja = (filter row r, atom aa): window of KD output pixels of row
@@ -416,8 +419,9 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                     if constexpr (BM_ == B_TMA_K2) tma_load_2d(bT, &tmB, fb, kb * KB, n0);
                     if constexpr (BM_ == B_TMA_K3) tma_load_3d(bT, &tmB, fb, kb * KB, n0, z);
                     if constexpr (BM_ == B_TMA_MN2) {
+                        const int zr = p.zsplit ? (z / p.zsplit) * p.zrows : 0;
                         for (int a = 0; a < p.bn_atoms; ++a)
-                            tma_load_2d(bT + a * KD * 128, &tmB, fb, n0 + a * (128 / ELT), kb * KD);
+                            tma_load_2d(bT + a * KD * 128, &tmB, fb, n0 + a * (128 / ELT), zr + kb * KD);
                     }
                     if constexpr (BM_ == B_TMA_MN3) {
                         // k-block kb covers tap kb / (K/KB), channels k0 = (kb % (K/KB)) * KB
@@ -966,7 +970,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                 } else if constexpr (EPI == EPI_WGRAD_CHAIN) {
                     // dw += alpha * partial (beta was applied by a prescale launch);
                     // 16-byte vector reductions in L2 (red.global.add.v4.f32).
-                    float* d = outF + (size_t)m * p.ldc + nb;
+                    float* d = outF + (p.zsplit ? (size_t)(z / p.zsplit) * p.batch_stride : 0) + (size_t)m * p.ldc + nb;
                     const bool vec = (nb + 32 <= p.N) && ((p.ldc & 3) == 0);
                     if (vec) {
 #pragma unroll

@@ -67,8 +67,12 @@ def test_workspace_winograd_alexnet_conv3():
     assert per_sample == 1_806_336
     assert mu.workspace_size(d, mu.FWD, mu.WINOGRAD, 1) == U + per_sample
     assert mu.workspace_size(d, mu.FWD, mu.WINOGRAD, 10) == U + 10 * per_sample
-    with pytest.raises(mu.MucuError):
-        mu.workspace_size(d, mu.BWD_FILTER, mu.WINOGRAD, 1)                 # NEXT-1
+    # WGRAD F(3x3,2x2): V + D at Tp = align256(b*T) tile rows, M fp32 (header closed form)
+    for b in (1, 10):
+        Tp = -(-b * 49 // 256) * 256
+        assert mu.workspace_size(d, mu.BWD_FILTER, mu.WINOGRAD, b) == 16 * Tp * (192 + 384) * 4 + 16 * 384 * 192 * 4
+    d5 = mu.desc(2, 40, 9, 9, 24, 3, 3, 1, 1, mu.MATH_BF16)                 # pitches 64 / 64 (128 B)
+    assert mu.workspace_size(d5, mu.BWD_FILTER, mu.WINOGRAD, 2) == 16 * 256 * (64 + 64) * 2 + 16 * 64 * 64 * 4
 
 
 def test_workspace_bf16_resnet_and_pointwise():

@@ -47,7 +47,7 @@ TOL = {mu.MATH_F32: 1e-5, mu.MATH_TF32: 1e-2, mu.MATH_BF16: 1e-2}
 def _eligible(shape, conv_type, algo):
     n, c, h, w, k, r, s, pad, st = shape
     if algo == mu.WINOGRAD:
-        return r == 3 and s == 3 and st == 1 and pad <= 2 and conv_type != mu.BWD_FILTER
+        return r == 3 and s == 3 and st == 1 and pad <= 2
     return True
 
 
@@ -120,7 +120,8 @@ def test_wgrad_accumulates_over_micro_batches(name, math):
         x, w, dy = _inputs(shape, kind, seed=11)
         xs, dys = stored(x, math), stored(dy, math)
         ref = oracle_ref(shape, mu.BWD_FILTER, xs, None, dys)
-        plan = [(mu.IMPLICIT_GEMM, 2), (mu.IM2COL_GEMM, 1), (mu.IMPLICIT_GEMM, 1)]
+        first = mu.WINOGRAD if _eligible(shape, mu.BWD_FILTER, mu.WINOGRAD) else mu.IMPLICIT_GEMM
+        plan = [(first, 2), (mu.IM2COL_GEMM, 1), (mu.IMPLICIT_GEMM, 1)]
         got, _ = run_gpu(d, mu.BWD_FILTER, plan, x, w, dy)
         if kind == "int":
             assert np.array_equal(got, ref)
@@ -136,8 +137,7 @@ def test_alpha_beta_and_mixed_plan(conv_type, math):
     shape = (4, 32, 9, 9, 48, 3, 3, 1, 1)
     d = mu.desc(*shape, math)
     x, w, dy = _inputs(shape, "int", seed=13)
-    algos = [mu.WINOGRAD, mu.IM2COL_GEMM, mu.IMPLICIT_GEMM] if conv_type != mu.BWD_FILTER else \
-        [mu.IM2COL_GEMM, mu.IMPLICIT_GEMM, mu.IMPLICIT_GEMM]
+    algos = [mu.WINOGRAD, mu.IM2COL_GEMM, mu.IMPLICIT_GEMM]
     plan = [(algos[0], 2), (algos[1], 1), (algos[2], 1)]
     n, c, h, wd, k, r, s, pad, st = shape
     p, q = mu.output_dims(d)

@@ -73,6 +73,18 @@ def algorithmic_bytes(layer, conv_type: int, n: int, elt: int) -> int:
     return x + y + w
 
 
+def shard_benchmark(costs: Dict[str, int], world: int) -> List[List[str]]:
+    """Assign benchmark jobs to ranks: longest-processing-time first onto the
+    least-loaded rank (ties -> lower rank), deterministic on every rank."""
+    shards: List[List[str]] = [[] for _ in range(world)]
+    load = [0] * world
+    for dk in sorted(costs, key=lambda d: (-costs[d], d)):
+        r = min(range(world), key=lambda i: (load[i], i))
+        shards[r].append(dk)
+        load[r] += costs[dk]
+    return shards
+
+
 class ConvNet:
     def __init__(self, handle: L.Handle, layers: Sequence, n: int, math: int, device: str = "cuda"):
         self.h = handle
@@ -104,21 +116,45 @@ class ConvNet:
                 dw=torch.zeros(ws_, dtype=torch.float32, device=self.device)))
 
     # ---------------------------------------------------------- planning --
-    def benchmark_all(self, ws_limit: int, progress: Optional[Callable] = None):
-        """P:L88 step 1 for every kernel (identical layers hit the handle's cache)."""
-        scratch = None
+    def benchmark_all(self, ws_limit: int, progress: Optional[Callable] = None, group=None):
+        """P:L88 step 1 for every kernel.  Identical kernels (same descriptor and
+        type) are benchmarked once (P:L159 cache).  In a data-parallel job the
+        unique kernels are sharded over the ranks (largest first onto the least
+        loaded rank) and the tables all-gathered: homogeneous GPUs give the same
+        tables, so the pass takes ~1/world of the time (SURVEY 8(f)
+        NEXT-2)."""
+        import torch.distributed as dist
+        world = dist.get_world_size(group) if dist.is_available() and dist.is_initialized() else 1
+        rank = dist.get_rank(group) if world > 1 else 0
+        uniq: Dict[str, List[Tuple[int, int]]] = {}
         for key, k in self.kernels.items():
+            uniq.setdefault(self._db_key(k, ws_limit, "bench"), []).append(key)
+        costs = {dk: layer_flops(self.layers[keys[0][0]], self.n) for dk, keys in uniq.items()}
+        mine = shard_benchmark(costs, world)[rank]
+        local = {}
+        scratch = None
+        for dk in mine:
+            k = self.kernels[uniq[dk][0]]
             need = L.benchmark_scratch_size(k.desc, k.conv_type, ws_limit)
             if scratch is None or scratch.numel() < need:
                 scratch = None
                 torch.cuda.empty_cache()
                 scratch = T.make_scratch(k.desc, k.conv_type, ws_limit)
-            k.table = self.h.benchmark(k.desc, k.conv_type, ws_limit, scratch.data_ptr(), scratch.numel(),
-                                       T._stream())
+            local[dk] = self.h.benchmark(k.desc, k.conv_type, ws_limit, scratch.data_ptr(), scratch.numel(),
+                                         T._stream())
             if progress:
-                progress(key)
+                progress(uniq[dk][0])
         del scratch
-        torch.cuda.empty_cache()
+        if torch.cuda.is_available():
+            torch.cuda.empty_cache()
+        tables = local
+        if world > 1:
+            parts = [None] * world
+            dist.all_gather_object(parts, local, group=group)
+            tables = {dk: tb for part in parts for dk, tb in part.items()}
+        for dk, keys in uniq.items():
+            for key in keys:
+                self.kernels[key].table = tables[dk]
 
     # File-based benchmark DB (P:L159: "caches ... the benchmark results into ...
     # optional file-based database", enabling offline benchmarking and sharing

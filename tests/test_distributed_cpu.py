@@ -72,3 +72,65 @@ def test_gloo_dw_allreduce_equals_full_batch():
             got = np.load(os.path.join(d, f"dw{rank}.npy"))
             assert np.max(np.abs(got - full)) <= 1e-12 * max(1.0, np.max(np.abs(full)))
             assert float(np.load(os.path.join(d, f"t{rank}.npy"))[0]) == world  # max over ranks
+
+
+def _bench_worker(rank, world, port, out_dir):
+    """Sharded benchmark pass with a stand-in benchmark:
+    host logic only (sharding, all-gather, fan-out to identical kernels)."""
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port), RANK=str(rank), WORLD_SIZE=str(world),
+                      LOCAL_RANK=str(rank))
+    import sys
+    sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+    import json
+    import paper_conf_cluster_oyamabhm18_b200 as mu
+    from paper_conf_cluster_oyamabhm18_b200 import network as N
+    from paper_conf_cluster_oyamabhm18_b200 import torch_api as T
+    from paper_conf_cluster_oyamabhm18_b200.distributed import init_from_env
+    from synthetic.networks import resnet18
+    assert init_from_env("gloo")
+    calls = []
+
+    class FakeHandle:
+        def benchmark(self, d, conv_type, ws_limit, scratch, nbytes, stream):
+            calls.append(f"{d.c},{d.h},{d.k},{d.r},{d.stride}|{conv_type}")
+            t = np.full((mu.NUM_ALGOS, d.n + 1), -1, dtype=np.int64)
+            t[:, 1:] = (d.c * 7 + d.k * 3 + d.h + conv_type) * np.arange(1, d.n + 1)
+            return t, np.zeros((mu.NUM_ALGOS, d.n + 1), dtype=np.uint64)
+
+    N.L.benchmark_scratch_size = lambda *a: 0
+    T.make_scratch = lambda *a: torch.empty(1, dtype=torch.uint8)
+    T._stream = lambda: 0
+    net = N.ConvNet(FakeHandle(), resnet18(), 8, mu.MATH_BF16, device="cpu")
+    net.benchmark_all(1 << 20)
+    tables = {f"{k[0]}/{k[1]}": v.table[0][0].tolist() for k, v in net.kernels.items()}
+    json.dump({"calls": calls, "tables": tables}, open(os.path.join(out_dir, f"b{rank}.json"), "w"))
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+def test_sharded_benchmark_pass_gloo():
+    import json
+    from synthetic.networks import resnet18
+    with tempfile.TemporaryDirectory() as d:
+        mp.spawn(_bench_worker, args=(2, _free_port(), d), nprocs=2, join=True)
+        r = [json.load(open(os.path.join(d, f"b{i}.json"))) for i in range(2)]
+    layers = resnet18()
+    uniq = {(l.c, l.h, l.k, l.r, l.stride, t) for l in layers for t in range(3)}
+    c0, c1 = set(r[0]["calls"]), set(r[1]["calls"])
+    assert not (c0 & c1)                                    # each unique kernel benchmarked on one rank
+    assert len(r[0]["calls"]) + len(r[1]["calls"]) == len(uniq)
+    assert abs(len(c0) - len(c1)) <= len(uniq) // 2         # both ranks work
+    assert r[0]["tables"] == r[1]["tables"]                 # identical tables everywhere after the gather
+    for i, l in enumerate(layers):                          # fan-out to identical kernels is the right table
+        for t in range(3):
+            v = r[0]["tables"][f"{i}/{t}"]
+            assert v[1] == l.c * 7 + l.k * 3 + l.h + t
+
+
+def test_shard_benchmark_lpt():
+    from paper_conf_cluster_oyamabhm18_b200.network import shard_benchmark
+    costs = {"a": 10, "b": 9, "c": 5, "d": 4, "e": 1}
+    s = shard_benchmark(costs, 2)
+    assert sorted(sum(s, [])) == sorted(costs)
+    assert s == [["a", "d", "e"], ["b", "c"]]
+    assert shard_benchmark(costs, 1) == [["a", "b", "c", "d", "e"]]

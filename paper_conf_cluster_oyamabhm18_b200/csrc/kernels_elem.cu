@@ -19,6 +19,32 @@
 
 namespace mucu {
 
+// Programmatic dependent launch (see kernels_tc.cu launch_t): every kernel here
+// is launched with programmatic stream serialization and waits for the
+// previous kernel's results before its first global access, so its launch
+// and scheduling overlap the previous kernel's tail.
+__device__ __forceinline__ void pdl_entry() {
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+    asm volatile("griddepcontrol.launch_dependents;" :::);
+}
+
+template <typename... KArgs, typename... Args>
+void launch_pdl(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st, Args... args) {
+    static const int pdl = getenv("MUCU_PDL") ? atoi(getenv("MUCU_PDL")) : 1;
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = grid;
+    cfg.blockDim = block;
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = st;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = pdl ? 1 : 0;
+    cudaLaunchKernelEx(&cfg, kern, ((KArgs)args)...);
+}
+
+
 namespace {
 
 template <class T> __device__ __forceinline__ float to_f(T v);
@@ -41,6 +67,7 @@ int grid_for(int64_t work, int threads) {
 
 template <class T>
 __global__ void pad_filter_kernel(const T* __restrict__ w, T* __restrict__ wp, int K, int RSC, int kpitch) {
+    pdl_entry();
     const int64_t total = (int64_t)K * kpitch;
     for (int64_t idx = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; idx < total;
          idx += (int64_t)gridDim.x * blockDim.x) {
@@ -62,6 +89,7 @@ __global__ void pad_filter_kernel(const T* __restrict__ w, T* __restrict__ wp, i
 // g[r][s] = w[i, 2-r, 2-s, o].
 template <class T>
 __global__ void wg_filter_kernel(const T* __restrict__ w, T* __restrict__ U, int O, int I, int C, bool dgrad) {
+    pdl_entry();
     const int64_t total = (int64_t)O * I;
     for (int64_t idx = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; idx < total;
          idx += (int64_t)gridDim.x * blockDim.x) {
@@ -99,6 +127,7 @@ __global__ void wg_filter_kernel(const T* __restrict__ w, T* __restrict__ U, int
 template <class T>
 __global__ void wg_input_kernel(const T* __restrict__ in, T* __restrict__ V, int64_t tiles, int IH, int IW,
                                 int I, int TH, int TW, int pad) {
+    pdl_entry();
     const int64_t total = tiles * I;
     for (int64_t idx = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; idx < total;
          idx += (int64_t)gridDim.x * blockDim.x) {
@@ -141,6 +170,7 @@ __global__ void wg_input_kernel(const T* __restrict__ in, T* __restrict__ V, int
 template <class T>
 __global__ void wg_output_kernel(const float* __restrict__ M, T* __restrict__ out, int64_t tiles, int OH, int OW,
                                  int O, int TH, int TW, float alpha, float beta) {
+    pdl_entry();
     const int64_t total = tiles * O;
     const int64_t plane = total;
     for (int64_t idx = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; idx < total;
@@ -185,6 +215,7 @@ __global__ void wg_output_kernel(const float* __restrict__ M, T* __restrict__ ou
 template <class T>
 __global__ void wgw_x_kernel(const T* __restrict__ x, T* __restrict__ V, int64_t tiles, int64_t Tp, int H, int W,
                              int C, int Cp, int TH, int TW, int pad) {
+    pdl_entry();
     const int64_t total = Tp * Cp, plane = Tp * Cp;
     for (int64_t idx = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; idx < total;
          idx += (int64_t)gridDim.x * blockDim.x) {
@@ -224,6 +255,7 @@ __global__ void wgw_x_kernel(const T* __restrict__ x, T* __restrict__ V, int64_t
 template <class T>
 __global__ void wgw_dy_kernel(const T* __restrict__ dy, T* __restrict__ D, int64_t tiles, int64_t Tp, int P, int Q,
                               int K, int Kp, int TH, int TW) {
+    pdl_entry();
     const int64_t total = Tp * Kp, plane = Tp * Kp;
     for (int64_t idx = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; idx < total;
          idx += (int64_t)gridDim.x * blockDim.x) {
@@ -259,6 +291,7 @@ __global__ void wgw_dy_kernel(const T* __restrict__ dy, T* __restrict__ D, int64
 // dw[k][r][s][c] = alpha * (G^T M[.][k][c] G)[r][s] + beta * dw (beta = 0: no read).
 __global__ void wgw_out_kernel(const float* __restrict__ M, float* __restrict__ dw, int K, int C, int Kp, int Cp,
                                float alpha, float beta) {
+    pdl_entry();
     const int64_t total = (int64_t)K * C, plane = (int64_t)Kp * Cp;
     for (int64_t idx = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; idx < total;
          idx += (int64_t)gridDim.x * blockDim.x) {
@@ -295,6 +328,7 @@ __global__ void wgw_out_kernel(const float* __restrict__ M, float* __restrict__ 
 template <class T, int V>
 __global__ void im2col_rows_kernel(const T* __restrict__ x, T* __restrict__ col, int64_t rows, int H, int W,
                                    int C, int P, int Q, int R, int S, int pad, int st, int kpitch) {
+    pdl_entry();
     using VT = typename std::conditional<V == 1, T, uint4>::type;
     const int lane = threadIdx.x & 31;
     const int64_t warp0 = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
@@ -332,6 +366,7 @@ __global__ void im2col_rows_kernel(const T* __restrict__ x, T* __restrict__ col,
 template <class T>
 __global__ void im2col_chunk_kernel(const T* __restrict__ x, T* __restrict__ col, int64_t rows, int H, int W,
                                     int C, int P, int Q, int R, int S, int pad, int st, int kpitch) {
+    pdl_entry();
     constexpr int V = 16 / sizeof(T);
     const int SC = S * C, RSC = R * SC;
     const int cpr = kpitch / V;
@@ -368,15 +403,15 @@ int im2col_t(const Geom& g, int32_t b, const void* x, void* col, int32_t kpitch,
     const int64_t rows = (int64_t)b * g.p * g.q;
     if (g.c % V == 0 && kpitch % V == 0) {
         const int grid = grid_for(rows * 32, 256);
-        im2col_rows_kernel<T, V><<<grid, 256, 0, st>>>((const T*)x, (T*)col, rows, g.h, g.w, g.c, g.p, g.q, g.r,
+        launch_pdl(im2col_rows_kernel<T, V>, dim3(grid), dim3(256), (size_t)(0), st, (const T*)x, (T*)col, rows, g.h, g.w, g.c, g.p, g.q, g.r,
                                                         g.s, g.pad, g.stride, kpitch);
     } else if (kpitch % V == 0) {
         const int grid = grid_for(rows * (kpitch / V), 256);
-        im2col_chunk_kernel<T><<<grid, 256, 0, st>>>((const T*)x, (T*)col, rows, g.h, g.w, g.c, g.p, g.q, g.r,
+        launch_pdl(im2col_chunk_kernel<T>, dim3(grid), dim3(256), (size_t)(0), st, (const T*)x, (T*)col, rows, g.h, g.w, g.c, g.p, g.q, g.r,
                                                       g.s, g.pad, g.stride, kpitch);
     } else {
         const int grid = grid_for(rows * 32, 256);
-        im2col_rows_kernel<T, 1><<<grid, 256, 0, st>>>((const T*)x, (T*)col, rows, g.h, g.w, g.c, g.p, g.q, g.r,
+        launch_pdl(im2col_rows_kernel<T, 1>, dim3(grid), dim3(256), (size_t)(0), st, (const T*)x, (T*)col, rows, g.h, g.w, g.c, g.p, g.q, g.r,
                                                         g.s, g.pad, g.stride, kpitch);
     }
     count_launch();
@@ -387,6 +422,7 @@ template <class T>
 __global__ void col2im_pixel_kernel(const float* __restrict__ dcol, T* __restrict__ dx, int64_t pixels, int H,
                                     int W, int C, int P, int Q, int R, int S, int pad, int st, int kpitch,
                                     float alpha, float beta) {
+    pdl_entry();
     for (int64_t pix = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; pix < pixels;
          pix += (int64_t)gridDim.x * blockDim.x) {
         const int w = (int)(pix % W);
@@ -422,6 +458,7 @@ template <class T, int V>
 __global__ void col2im_taps_kernel(const float* __restrict__ dcol, T* __restrict__ dx, int64_t pixels, int H,
                                    int W, int C, int P, int Q, int R, int S, int pad, int st, int kpitch,
                                    float alpha, float beta) {
+    pdl_entry();
     const int CG = C / V;
     const int64_t total = pixels * CG;
     for (int64_t idx = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; idx < total;
@@ -473,6 +510,7 @@ __global__ void col2im_taps_kernel(const float* __restrict__ dcol, T* __restrict
 template <class T>
 __global__ void s2d_input_kernel(const T* __restrict__ x, T* __restrict__ xs, int chunks, int H, int W, int C,
                                  int I, int J, int st, int pad, int Cs) {
+    pdl_entry();
     constexpr int V = 16 / sizeof(T);
     const int cpp = Cs / V, stc = st * C, real = st * stc;
     // 32-bit index math (the launcher checks the range): 64-bit divisions
@@ -512,6 +550,7 @@ __global__ void s2d_input_kernel(const T* __restrict__ x, T* __restrict__ xs, in
 template <class T>
 __global__ void s2d_filter_kernel(const T* __restrict__ w, T* __restrict__ out, int64_t total, int K, int R, int S,
                                   int C, int st, int f, int u, int Dr, int Ds, int Cs, bool dgrad) {
+    pdl_entry();
     const int fc = f * C, real = f * fc;
     for (int64_t idx = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; idx < total;
          idx += (int64_t)gridDim.x * blockDim.x) {
@@ -552,9 +591,9 @@ int launch_pad_filter(const Geom& g, const void* w, void* wpad, int32_t kpitch, 
     const int RSC = g.r * g.s * g.c;
     int grid = grid_for((int64_t)g.k * kpitch, 256);
     if (g.math == MUCU_MATH_BF16)
-        pad_filter_kernel<__nv_bfloat16><<<grid, 256, 0, st>>>((const __nv_bfloat16*)w, (__nv_bfloat16*)wpad, g.k, RSC, kpitch);
+        launch_pdl(pad_filter_kernel<__nv_bfloat16>, dim3(grid), dim3(256), (size_t)(0), st, (const __nv_bfloat16*)w, (__nv_bfloat16*)wpad, g.k, RSC, kpitch);
     else
-        pad_filter_kernel<float><<<grid, 256, 0, st>>>((const float*)w, (float*)wpad, g.k, RSC, kpitch);
+        launch_pdl(pad_filter_kernel<float>, dim3(grid), dim3(256), (size_t)(0), st, (const float*)w, (float*)wpad, g.k, RSC, kpitch);
     count_launch();
     return (int)cudaGetLastError();
 }
@@ -567,10 +606,10 @@ int launch_col2im(const Geom& g, int32_t b, float alpha, const float* dcol, int3
         // registers; neighbouring threads read neighbouring taps of a dcol row.
         const int grid = grid_for(pixels, 256);
         if (g.math == MUCU_MATH_BF16)
-            col2im_pixel_kernel<__nv_bfloat16><<<grid, 256, 0, st>>>(dcol, (__nv_bfloat16*)dx, pixels, g.h, g.w, g.c, g.p,
+            launch_pdl(col2im_pixel_kernel<__nv_bfloat16>, dim3(grid), dim3(256), (size_t)(0), st, dcol, (__nv_bfloat16*)dx, pixels, g.h, g.w, g.c, g.p,
                                                                     g.q, g.r, g.s, g.pad, g.stride, kpitch, alpha, beta);
         else
-            col2im_pixel_kernel<float><<<grid, 256, 0, st>>>(dcol, (float*)dx, pixels, g.h, g.w, g.c, g.p, g.q, g.r,
+            launch_pdl(col2im_pixel_kernel<float>, dim3(grid), dim3(256), (size_t)(0), st, dcol, (float*)dx, pixels, g.h, g.w, g.c, g.p, g.q, g.r,
                                                             g.s, g.pad, g.stride, kpitch, alpha, beta);
         count_launch();
         return (int)cudaGetLastError();
@@ -578,7 +617,7 @@ int launch_col2im(const Geom& g, int32_t b, float alpha, const float* dcol, int3
     const bool v4 = g.c % 4 == 0 && kpitch % 4 == 0;
     const int grid = grid_for(pixels * (v4 ? g.c / 4 : g.c), 256);
 #define COL2IM(TT, VV)                                                                                            \
-    col2im_taps_kernel<TT, VV><<<grid, 256, 0, st>>>(dcol, (TT*)dx, pixels, g.h, g.w, g.c, g.p, g.q, g.r, g.s,   \
+    launch_pdl(col2im_taps_kernel<TT, VV>, dim3(grid), dim3(256), (size_t)(0), st, dcol, (TT*)dx, pixels, g.h, g.w, g.c, g.p, g.q, g.r, g.s,   \
                                                      g.pad, g.stride, kpitch, alpha, beta)
     if (g.math == MUCU_MATH_BF16) {
         if (v4) COL2IM(__nv_bfloat16, 4); else COL2IM(__nv_bfloat16, 1);
@@ -592,6 +631,7 @@ int launch_col2im(const Geom& g, int32_t b, float alpha, const float* dcol, int3
 
 namespace {
 __global__ void scale_kernel(float* __restrict__ p, int64_t n, float beta) {
+    pdl_entry();
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
         p[i] = beta == 0.f ? 0.f : beta * p[i];
 }
@@ -600,6 +640,7 @@ __global__ void scale_kernel(float* __restrict__ p, int64_t n, float beta) {
 // receive no gradient: zero them (beta = 0) in one pass of 16-B stores.
 __global__ void zero_tapless_kernel(uint4* __restrict__ dx, int rows, int cpp, int H, int W, int R, int S, int pad,
                                     int st) {
+    pdl_entry();
     // one block per dx pixel row (n, h); a row whose phase meets no tap is zeroed whole
     const int per_row = W * cpp;
     for (int row = blockIdx.x; row < rows; row += gridDim.x) {
@@ -619,7 +660,7 @@ int launch_zero_tapless(const Geom& g, int32_t b, void* dx, cudaStream_t st) {
     if ((g.c * elt) % 16 != 0) return -1;
     const int cpp = g.c * elt / 16;
     const int rows = b * g.h;
-    zero_tapless_kernel<<<std::min(rows, 148 * 16), 256, 0, st>>>((uint4*)dx, rows, cpp, g.h, g.w, g.r, g.s, g.pad,
+    launch_pdl(zero_tapless_kernel, dim3(std::min(rows, 148 * 16)), dim3(256), (size_t)(0), st, (uint4*)dx, rows, cpp, g.h, g.w, g.r, g.s, g.pad,
                                                                   g.stride);
     count_launch();
     return (int)cudaGetLastError();
@@ -629,6 +670,7 @@ namespace {
 // One thread per pixel: reads C (< 16 B) channels, writes one 16-B vector.
 template <class T>
 __global__ void pad_channels_kernel(const T* __restrict__ x, T* __restrict__ xp, int64_t pixels, int C) {
+    pdl_entry();
     constexpr int V = 16 / sizeof(T);
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < pixels; i += (int64_t)gridDim.x * blockDim.x) {
         __align__(16) T v[V];
@@ -644,6 +686,7 @@ __global__ void pad_channels_kernel(const T* __restrict__ x, T* __restrict__ xp,
 template <typename T>
 __global__ void win_pad_kernel(const T* __restrict__ x, T* __restrict__ xp, int64_t units, int W, int Wp, int C,
                                int pad) {
+    pdl_entry();
     constexpr int V = 16 / sizeof(T);  // elements per unit = V / 4 pixels of 4 channels
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < units; i += (int64_t)gridDim.x * blockDim.x) {
         const int64_t e0 = i * V;
@@ -663,10 +706,10 @@ int launch_win_pad(const Geom& g, int32_t b, int Wp, const void* x, void* xp, cu
     const int64_t units = (int64_t)b * g.h * Wp * 4 * elt_size(g.math) / 16;
     const int grid = grid_for(units, 256);
     if (g.math == MUCU_MATH_BF16)
-        win_pad_kernel<__nv_bfloat16><<<grid, 256, 0, st>>>((const __nv_bfloat16*)x, (__nv_bfloat16*)xp, units, g.w,
+        launch_pdl(win_pad_kernel<__nv_bfloat16>, dim3(grid), dim3(256), (size_t)(0), st, (const __nv_bfloat16*)x, (__nv_bfloat16*)xp, units, g.w,
                                                             Wp, g.c, g.pad);
     else
-        win_pad_kernel<float><<<grid, 256, 0, st>>>((const float*)x, (float*)xp, units, g.w, Wp, g.c, g.pad);
+        launch_pdl(win_pad_kernel<float>, dim3(grid), dim3(256), (size_t)(0), st, (const float*)x, (float*)xp, units, g.w, Wp, g.c, g.pad);
     count_launch();
     return (int)cudaGetLastError();
 }
@@ -674,15 +717,15 @@ int launch_pad_channels(const Geom& g, int32_t b, const void* x, void* xp, cudaS
     const int64_t pixels = (int64_t)b * g.h * g.w;
     const int grid = grid_for(pixels, 256);
     if (g.math == MUCU_MATH_BF16)
-        pad_channels_kernel<__nv_bfloat16><<<grid, 256, 0, st>>>((const __nv_bfloat16*)x, (__nv_bfloat16*)xp, pixels, g.c);
+        launch_pdl(pad_channels_kernel<__nv_bfloat16>, dim3(grid), dim3(256), (size_t)(0), st, (const __nv_bfloat16*)x, (__nv_bfloat16*)xp, pixels, g.c);
     else
-        pad_channels_kernel<float><<<grid, 256, 0, st>>>((const float*)x, (float*)xp, pixels, g.c);
+        launch_pdl(pad_channels_kernel<float>, dim3(grid), dim3(256), (size_t)(0), st, (const float*)x, (float*)xp, pixels, g.c);
     count_launch();
     return (int)cudaGetLastError();
 }
 
 int launch_scale(int64_t n, float beta, float* p, cudaStream_t st) {
-    scale_kernel<<<grid_for(n, 256), 256, 0, st>>>(p, n, beta);
+    launch_pdl(scale_kernel, dim3(grid_for(n, 256)), dim3(256), (size_t)(0), st, p, n, beta);
     count_launch();
     return (int)cudaGetLastError();
 }
@@ -691,9 +734,9 @@ int launch_wg_filter(const Geom& g, bool dgrad, const void* w, void* U, cudaStre
     const int O = dgrad ? g.c : g.k, I = dgrad ? g.k : g.c;
     int grid = grid_for((int64_t)O * I, 256);
     if (g.math == MUCU_MATH_BF16)
-        wg_filter_kernel<__nv_bfloat16><<<grid, 256, 0, st>>>((const __nv_bfloat16*)w, (__nv_bfloat16*)U, O, I, g.c, dgrad);
+        launch_pdl(wg_filter_kernel<__nv_bfloat16>, dim3(grid), dim3(256), (size_t)(0), st, (const __nv_bfloat16*)w, (__nv_bfloat16*)U, O, I, g.c, dgrad);
     else
-        wg_filter_kernel<float><<<grid, 256, 0, st>>>((const float*)w, (float*)U, O, I, g.c, dgrad);
+        launch_pdl(wg_filter_kernel<float>, dim3(grid), dim3(256), (size_t)(0), st, (const float*)w, (float*)U, O, I, g.c, dgrad);
     count_launch();
     return (int)cudaGetLastError();
 }
@@ -712,9 +755,9 @@ int launch_wg_input(const Geom& g, bool dgrad, int32_t b, const void* in, void* 
     const int64_t tiles = (int64_t)b * TH * TW;
     int grid = grid_for(tiles * I, 256);
     if (g.math == MUCU_MATH_BF16)
-        wg_input_kernel<__nv_bfloat16><<<grid, 256, 0, st>>>((const __nv_bfloat16*)in, (__nv_bfloat16*)V, tiles, IH, IW, I, TH, TW, pad);
+        launch_pdl(wg_input_kernel<__nv_bfloat16>, dim3(grid), dim3(256), (size_t)(0), st, (const __nv_bfloat16*)in, (__nv_bfloat16*)V, tiles, IH, IW, I, TH, TW, pad);
     else
-        wg_input_kernel<float><<<grid, 256, 0, st>>>((const float*)in, (float*)V, tiles, IH, IW, I, TH, TW, pad);
+        launch_pdl(wg_input_kernel<float>, dim3(grid), dim3(256), (size_t)(0), st, (const float*)in, (float*)V, tiles, IH, IW, I, TH, TW, pad);
     count_launch();
     return (int)cudaGetLastError();
 }
@@ -727,9 +770,9 @@ int launch_wg_output(const Geom& g, bool dgrad, int32_t b, float alpha, const fl
     const int64_t tiles = (int64_t)b * TH * TW;
     int grid = grid_for(tiles * O, 256);
     if (g.math == MUCU_MATH_BF16)
-        wg_output_kernel<__nv_bfloat16><<<grid, 256, 0, st>>>(M, (__nv_bfloat16*)out, tiles, OH, OW, O, TH, TW, alpha, beta);
+        launch_pdl(wg_output_kernel<__nv_bfloat16>, dim3(grid), dim3(256), (size_t)(0), st, M, (__nv_bfloat16*)out, tiles, OH, OW, O, TH, TW, alpha, beta);
     else
-        wg_output_kernel<float><<<grid, 256, 0, st>>>(M, (float*)out, tiles, OH, OW, O, TH, TW, alpha, beta);
+        launch_pdl(wg_output_kernel<float>, dim3(grid), dim3(256), (size_t)(0), st, M, (float*)out, tiles, OH, OW, O, TH, TW, alpha, beta);
     count_launch();
     return (int)cudaGetLastError();
 }
@@ -740,10 +783,10 @@ int launch_s2d_input(const Geom& g, int32_t b, int f, int I, int J, int Cs, cons
     if (chunks >= (1LL << 31) || (int64_t)g.h * g.w * g.c >= (1LL << 31)) return (int)cudaErrorInvalidValue;
     const int grid = grid_for(chunks, 256);
     if (g.math == MUCU_MATH_BF16)
-        s2d_input_kernel<__nv_bfloat16><<<grid, 256, 0, st>>>((const __nv_bfloat16*)x, (__nv_bfloat16*)xs, (int)chunks,
+        launch_pdl(s2d_input_kernel<__nv_bfloat16>, dim3(grid), dim3(256), (size_t)(0), st, (const __nv_bfloat16*)x, (__nv_bfloat16*)xs, (int)chunks,
                                                               g.h, g.w, g.c, I, J, f, g.pad, Cs);
     else
-        s2d_input_kernel<float><<<grid, 256, 0, st>>>((const float*)x, (float*)xs, (int)chunks, g.h, g.w, g.c, I, J,
+        launch_pdl(s2d_input_kernel<float>, dim3(grid), dim3(256), (size_t)(0), st, (const float*)x, (float*)xs, (int)chunks, g.h, g.w, g.c, I, J,
                                                       f, g.pad, Cs);
     count_launch();
     return (int)cudaGetLastError();
@@ -754,11 +797,11 @@ int launch_s2d_filter(const Geom& g, bool dgrad, const S2d& z, const void* w, vo
                                 : (int64_t)z.u * z.u * g.k * z.Dr * z.Ds * z.Cs;
     const int grid = grid_for(total, 256);
     if (g.math == MUCU_MATH_BF16)
-        s2d_filter_kernel<__nv_bfloat16><<<grid, 256, 0, st>>>((const __nv_bfloat16*)w, (__nv_bfloat16*)out, total,
+        launch_pdl(s2d_filter_kernel<__nv_bfloat16>, dim3(grid), dim3(256), (size_t)(0), st, (const __nv_bfloat16*)w, (__nv_bfloat16*)out, total,
                                                                g.k, g.r, g.s, g.c, g.stride, z.f, z.u, z.Dr, z.Ds,
                                                                z.Cs, dgrad);
     else
-        s2d_filter_kernel<float><<<grid, 256, 0, st>>>((const float*)w, (float*)out, total, g.k, g.r, g.s, g.c,
+        launch_pdl(s2d_filter_kernel<float>, dim3(grid), dim3(256), (size_t)(0), st, (const float*)w, (float*)out, total, g.k, g.r, g.s, g.c,
                                                        g.stride, z.f, z.u, z.Dr, z.Ds, z.Cs, dgrad);
     count_launch();
     return (int)cudaGetLastError();
@@ -771,16 +814,16 @@ int launch_wgw_transforms(const Geom& g, int32_t b, const void* x, const void* d
     const int at = 128 / elt_size(g.math);
     const int Cp = (int)align_up((uint64_t)g.c, (uint64_t)at), Kp = (int)align_up((uint64_t)g.k, (uint64_t)at);
     if (g.math == MUCU_MATH_BF16) {
-        wgw_x_kernel<__nv_bfloat16><<<grid_for(Tp * Cp, 256), 256, 0, st>>>(
+        launch_pdl(wgw_x_kernel<__nv_bfloat16>, dim3(grid_for(Tp * Cp, 256)), dim3(256), (size_t)(0), st, 
             (const __nv_bfloat16*)x, (__nv_bfloat16*)V, tiles, Tp, g.h, g.w, g.c, Cp, TH, TW, g.pad);
         count_launch();
-        wgw_dy_kernel<__nv_bfloat16><<<grid_for(Tp * Kp, 256), 256, 0, st>>>(
+        launch_pdl(wgw_dy_kernel<__nv_bfloat16>, dim3(grid_for(Tp * Kp, 256)), dim3(256), (size_t)(0), st, 
             (const __nv_bfloat16*)dy, (__nv_bfloat16*)D, tiles, Tp, g.p, g.q, g.k, Kp, TH, TW);
     } else {
-        wgw_x_kernel<float><<<grid_for(Tp * Cp, 256), 256, 0, st>>>((const float*)x, (float*)V, tiles, Tp, g.h, g.w,
+        launch_pdl(wgw_x_kernel<float>, dim3(grid_for(Tp * Cp, 256)), dim3(256), (size_t)(0), st, (const float*)x, (float*)V, tiles, Tp, g.h, g.w,
                                                                     g.c, Cp, TH, TW, g.pad);
         count_launch();
-        wgw_dy_kernel<float><<<grid_for(Tp * Kp, 256), 256, 0, st>>>((const float*)dy, (float*)D, tiles, Tp, g.p,
+        launch_pdl(wgw_dy_kernel<float>, dim3(grid_for(Tp * Kp, 256)), dim3(256), (size_t)(0), st, (const float*)dy, (float*)D, tiles, Tp, g.p,
                                                                      g.q, g.k, Kp, TH, TW);
     }
     count_launch();
@@ -790,7 +833,7 @@ int launch_wgw_transforms(const Geom& g, int32_t b, const void* x, const void* d
 int launch_wgw_output(const Geom& g, float alpha, const float* M, float beta, float* dw, cudaStream_t st) {
     const int at = 128 / elt_size(g.math);
     const int Cp = (int)align_up((uint64_t)g.c, (uint64_t)at), Kp = (int)align_up((uint64_t)g.k, (uint64_t)at);
-    wgw_out_kernel<<<grid_for((int64_t)g.k * g.c, 256), 256, 0, st>>>(M, dw, g.k, g.c, Kp, Cp, alpha, beta);
+    launch_pdl(wgw_out_kernel, dim3(grid_for((int64_t)g.k * g.c, 256)), dim3(256), (size_t)(0), st, M, dw, g.k, g.c, Kp, Cp, alpha, beta);
     count_launch();
     return (int)cudaGetLastError();
 }

@@ -250,6 +250,7 @@ struct TcArgs {
     int s2_st, s2_C, s2_R, s2_S;
     // EPI_D2S output tensor [*, e_H, e_W, e_C], written at (s2_st*i + a - e_pad, s2_st*j + b - e_pad)
     int e_H, e_W, e_C, e_pad;
+    int d2s_rows;            // EPI_D2S by dx rows (beta = 0, one N tile, f*C % 4 == 0)
     // Window WGRAD (A_TMA_WIN / B_TMA_DYROW): 128-B atoms per filter row, q-blocks per output row
     int win_na, win_qb, win_aw;  // + bytes per A swizzle atom (128 / 64 / 32: UMMA layout 2 / 4 / 6)
     // Halo IG (A_HALO): extended grid of hx_H = Ho + R - 1 rows x hx_W (>= Wo + S - 1, multiple of 8)
@@ -780,6 +781,7 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
                 return -1;
             if (!map2(&L.tb, ws, Kp, A.N, Kp, KB, A.BN)) return -1;
             A.tma_bytes = 16384 * A.mt + A.BN * 128;
+            A.d2s_rows = beta == 0.f && A.N <= A.BN && (f * g.c) % 4 == 0 && env_int("MUCU_D2S_ROWS", 1);
             return LAUNCH(A_TMA_IM2COL, B_TMA_K2, EPI_D2S);
         }
         const int I = z.I, J = z.J;

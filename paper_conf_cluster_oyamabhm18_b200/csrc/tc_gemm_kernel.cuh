@@ -862,6 +862,76 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                 outF += (size_t)z * p.batch_stride;
                 outT += (size_t)z * p.batch_stride;
             }
+            if constexpr (EPI == EPI_D2S) {
+                if (p.d2s_rows) {
+                    // Depth-to-space by dx rows (beta = 0, one N tile): for each row a of
+                    // the f x f super-pixel, its f*C contiguous dx values are read from
+                    // TMEM in 4-column pieces (warp-uniform loop: tcgen05.ld is
+                    // .sync.aligned) and stored as bf16x2 / float2 words when the segment
+                    // lies inside the image (~1.5 instructions per element instead of ~15
+                    // with per-column index stepping, which made this epilogue the bound
+                    // of the space-to-depth DGRAD); edge super-pixels go element-wise.
+                    const bool mv = m < p.M && rowok;
+                    const int hw = p.ph_H * p.ph_W;
+                    const int mm = mv ? m : 0;
+                    const int n = mm / hw, rem = mm - n * hw, ii = rem / p.ph_W, jj = rem - ii * p.ph_W;
+                    const int f = p.s2_st, C = p.e_C, fC = f * C;
+                    const int h0 = f * ii - p.e_pad, w0 = f * jj - p.e_pad;
+                    const bool inner = w0 >= 0 && w0 + f <= p.e_W;
+                    const uint32_t tb = tmem + (uint32_t)((acc * p.mt + hh) * p.BN) + ((uint32_t)(q4 * 32) << 16);
+                    for (int a = 0; a < f; ++a) {
+                        const int h = h0 + a;
+                        const bool hv = mv && (unsigned)h < (unsigned)p.e_H;
+                        const long long off = (((long long)n * p.e_H + h) * p.e_W + w0) * C;
+                        for (int e0 = 0; e0 < fC; e0 += 4) {
+                            uint32_t v[4];
+                            if (has_acc) {
+                                asm volatile("tcgen05.ld.sync.aligned.32x32b.x4.b32 {%0,%1,%2,%3}, [%4];"
+                                             : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3])
+                                             : "r"(tb + (uint32_t)(a * fC + e0)));
+                                asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+                            } else {
+                                v[0] = v[1] = v[2] = v[3] = 0u;
+                            }
+                            if (!hv || (p.debug & 1)) continue;
+                            float o[4];
+#pragma unroll
+                            for (int u = 0; u < 4; ++u) o[u] = p.alpha * __uint_as_float(v[u]);
+                            if (inner) {
+                                if (p.out_bf16) {
+                                    __nv_bfloat16* d = (__nv_bfloat16*)p.out + off + e0;
+                                    if ((((uintptr_t)d) & 3) == 0) {
+                                        *reinterpret_cast<__nv_bfloat162*>(d) = __floats2bfloat162_rn(o[0], o[1]);
+                                        *reinterpret_cast<__nv_bfloat162*>(d + 2) = __floats2bfloat162_rn(o[2], o[3]);
+                                    } else {
+#pragma unroll
+                                        for (int u = 0; u < 4; ++u) d[u] = __float2bfloat16_rn(o[u]);
+                                    }
+                                } else {
+                                    float* d = (float*)p.out + off + e0;
+                                    if ((((uintptr_t)d) & 7) == 0) {
+                                        *reinterpret_cast<float2*>(d) = make_float2(o[0], o[1]);
+                                        *reinterpret_cast<float2*>(d + 2) = make_float2(o[2], o[3]);
+                                    } else {
+#pragma unroll
+                                        for (int u = 0; u < 4; ++u) d[u] = o[u];
+                                    }
+                                }
+                            } else {
+#pragma unroll
+                                for (int u = 0; u < 4; ++u) {
+                                    const int e = e0 + u, bq = e / C;
+                                    if ((unsigned)(w0 + bq) < (unsigned)p.e_W) {
+                                        if (p.out_bf16) ((__nv_bfloat16*)p.out)[off + e] = __float2bfloat16_rn(o[u]);
+                                        else ((float*)p.out)[off + e] = o[u];
+                                    }
+                                }
+                            }
+                        }
+                    }
+                    return;
+                }
+            }
             for (int c0 = 0; c0 < p.BN; c0 += 32) {
                 uint32_t v[32];
                 if (has_acc) {

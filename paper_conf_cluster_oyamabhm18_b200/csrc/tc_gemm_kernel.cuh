@@ -883,6 +883,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                         const int h = h0 + a;
                         const bool hv = mv && (unsigned)h < (unsigned)p.e_H;
                         const long long off = (((long long)n * p.e_H + h) * p.e_W + w0) * C;
+                        int ebq = 0, ec = 0;  // edge path: (pixel, channel) of element e0 (no division)
                         for (int e0 = 0; e0 < fC; e0 += 4) {
                             uint32_t v[4];
                             if (has_acc) {
@@ -920,11 +921,12 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                             } else {
 #pragma unroll
                                 for (int u = 0; u < 4; ++u) {
-                                    const int e = e0 + u, bq = e / C;
-                                    if ((unsigned)(w0 + bq) < (unsigned)p.e_W) {
+                                    const int e = e0 + u;
+                                    if ((unsigned)(w0 + ebq) < (unsigned)p.e_W) {
                                         if (p.out_bf16) ((__nv_bfloat16*)p.out)[off + e] = __float2bfloat16_rn(o[u]);
                                         else ((float*)p.out)[off + e] = o[u];
                                     }
+                                    if (++ec == C) { ec = 0; ++ebq; }
                                 }
                             }
                         }

@@ -934,6 +934,17 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                     return;
                 }
             }
+            // EPI_D2S: the row's super-pixel (n, i, j) once per row, not per 32-column chunk
+            int d2_n = 0, d2_h0 = 0, d2_w0 = 0;
+            if constexpr (EPI == EPI_D2S) {
+                if (m < p.M) {
+                    const int hw = p.ph_H * p.ph_W;
+                    d2_n = m / hw;
+                    const int rem = m - d2_n * hw, ii = rem / p.ph_W, jj = rem - ii * p.ph_W;
+                    d2_h0 = p.s2_st * ii - p.e_pad;
+                    d2_w0 = p.s2_st * jj - p.e_pad;
+                }
+            }
             for (int c0 = 0; c0 < p.BN; c0 += 32) {
                 uint32_t v[32];
                 if (has_acc) {
@@ -949,9 +960,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                     // super-pixel row (n, i, jj); column (a, b, c) walked incrementally:
                     // the dx offset advances by 1 inside an (a) block of st*C values and
                     // by (W - st)*C between blocks (no per-column index arithmetic).
-                    const int hw = p.ph_H * p.ph_W;
-                    const int n = m / hw, rem = m - n * hw, ii = rem / p.ph_W, jj = rem - ii * p.ph_W;
-                    const int h0 = p.s2_st * ii - p.e_pad, w0 = p.s2_st * jj - p.e_pad;
+                    const int n = d2_n, h0 = d2_h0, w0 = d2_w0;
                     const int stc = p.s2_st * p.e_C;
                     int a = nb / stc, bq = (nb - a * stc) / p.e_C, c = nb - a * stc - bq * p.e_C;
                     long long off = (((long long)n * p.e_H + h0 + a) * p.e_W + w0 + bq) * p.e_C + c;

@@ -51,6 +51,8 @@ def parse():
                     help="skip the first layer's BackwardData (the data layer needs no gradient, as in "
                          "Caffe's `time` command, P:L198); the default times all 3 kernels per layer (SURVEY 8(d) cfg2)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-concurrent-wgrad", dest="concurrent_wgrad", action="store_false",
+                    help="run each BackwardFilter after its BackwardData on one stream")
     ap.add_argument("--cpu-sample", type=int, default=0, help="oracle sample (images per kernel); 0 = auto")
     ap.add_argument("--json-out", default="")
     ap.add_argument("--tables-in", default="", help="benchmark DB (.npz) to plan from instead of benchmarking")
@@ -180,7 +182,8 @@ def run_reference(args):
             "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": {"workload": f"{args.config} conv layers fwd+bwd ({n_kernels(layers, args.input_grad)} kernels)",
                        "batch_per_gpu": args.batch, "math": "fp64 oracle",
-                       "first_layer_backward_data": bool(args.input_grad)},
+                       "first_layer_backward_data": bool(args.input_grad),
+                       "backward_streams": 2 if args.concurrent_wgrad else 1},
             "cpu_baseline": cb,
             "e2e": {"value": round(ms, 3), "unit": "ms/iter", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
@@ -228,10 +231,14 @@ def main():
     grad_ar = GradAllreduce()
     stream = torch.cuda.current_stream()
 
+    # BackwardFilter of each layer on a side stream next to its BackwardData
+    # (network.iteration concurrent=True); the evented per-op pass is sequential.
+    conc = args.concurrent_wgrad
+
     def timed(nsteps, nwarm, record_ops=False, e2e=None):
         ops = {}
         for _ in range(nwarm):
-            net.iteration(grad_hook=grad_ar, skip_conv1_dgrad=not args.input_grad)
+            net.iteration(grad_hook=grad_ar, skip_conv1_dgrad=not args.input_grad, concurrent=conc and not record_ops)
             grad_ar.wait()
         torch.cuda.synchronize()
         if distributed:
@@ -255,7 +262,8 @@ def main():
             s0.record(stream)
             if e2e is not None:
                 e2e["h2d"]()
-            net.iteration(on_op=on_op, grad_hook=grad_ar, skip_conv1_dgrad=not args.input_grad)
+            net.iteration(on_op=on_op, grad_hook=grad_ar, skip_conv1_dgrad=not args.input_grad,
+                          concurrent=conc and not record_ops)
             grad_ar.wait()
             if e2e is not None:
                 e2e["d2h"]()
@@ -327,11 +335,11 @@ def main():
     first_bwd = [True]
 
     def e2e_op(i, t, what):
-        if what == "begin" and t != mu.FWD and first_bwd[0]:
+        if what in ("begin", "first") and t != mu.FWD and first_bwd[0]:
             stream.wait_event(dy_ready)
             first_bwd[0] = False
         if what == "end" and t == mu.BWD_FILTER and not distributed:  # N > 1: after the dW allreduce
-            copy_stream.wait_stream(stream)
+            copy_stream.wait_stream(torch.cuda.current_stream())  # the BackwardFilter's stream
             with torch.cuda.stream(copy_stream):
                 dw_host[i].copy_(net.tensors[i]["dw"], non_blocking=True)
 

@@ -243,9 +243,17 @@ class ConvNet:
             T.conv_backward_filter(self.h, k.desc, k.plan, t["x"], t["dy"], t["dw"], workspace=ws)
 
     def iteration(self, on_op: Optional[Callable] = None, grad_hook: Optional[Callable] = None,
-                  skip_conv1_dgrad: bool = False):
+                  skip_conv1_dgrad: bool = False, concurrent: bool = False):
         """FWD of all layers, then DGRAD + WGRAD in reverse order.  on_op(i, type,
-        'begin'|'end') lets a caller record CUDA events around each call."""
+        'begin'|'end') lets a caller record CUDA events around each call.
+
+        concurrent=True runs each layer's BackwardFilter on a side stream next to
+        its BackwardData (both only need the layer's dy, i.e. the previous
+        BackwardData): the two persistent kernels fill each other's partial last
+        waves.  Each kernel keeps its own workspace (WR) or segment (WD), so the
+        overlap is memory-safe; results are unchanged."""
+        if concurrent:
+            return self._iteration_concurrent(grad_hook, skip_conv1_dgrad, on_op)
         order = [(i, L.FWD) for i in range(len(self.layers))]
         for i in reversed(range(len(self.layers))):
             if not (skip_conv1_dgrad and i == 0):
@@ -259,6 +267,36 @@ class ConvNet:
                 on_op(i, t, "end")
             if t == L.BWD_FILTER and grad_hook is not None:
                 grad_hook(i, self.tensors[i]["dw"])
+
+    def _iteration_concurrent(self, grad_hook, skip_conv1_dgrad, on_op=None):
+        """on_op(i, type, 'begin'|'end') runs on the host around each call with the
+        call's stream current (for stream-ordered hooks; not for event timing)."""
+        main = torch.cuda.current_stream()
+        if getattr(self, "_side", None) is None:
+            self._side = torch.cuda.Stream()
+            self._dy_ready = [torch.cuda.Event() for _ in self.layers]
+        side = self._side
+        hook = on_op or (lambda *a: None)
+
+        def run(i, t):
+            hook(i, t, "begin")
+            self.run_kernel(i, t)
+            hook(i, t, "end")
+        for i in range(len(self.layers)):
+            run(i, L.FWD)
+        for i in reversed(range(len(self.layers))):
+            if i == len(self.layers) - 1:
+                hook(i, L.BWD_DATA, "first")  # stream-ordered setup before any backward call
+            # dy of layer i: produced by the previous BackwardData on the main stream
+            self._dy_ready[i].record(main)
+            if not (skip_conv1_dgrad and i == 0):
+                run(i, L.BWD_DATA)
+            side.wait_event(self._dy_ready[i])
+            with torch.cuda.stream(side):
+                run(i, L.BWD_FILTER)
+                if grad_hook is not None:
+                    grad_hook(i, self.tensors[i]["dw"])
+        main.wait_stream(side)
 
     def flops_per_iteration(self, skip_conv1_dgrad: bool = False) -> int:
         f = sum(layer_flops(l, self.n) for l in self.layers) * 3

@@ -42,18 +42,10 @@ def with_events():
         e = torch.cuda.Event(enable_timing=True); e.record(st); evs.append(e)
     net.iteration(on_op=on_op)
 print("eager, no events   %.4f ms" % timeit(lambda: net.iteration()))
+print("concurrent WGRAD   %.4f ms" % timeit(lambda: net.iteration(concurrent=True)))
+print("eager, no events   %.4f ms" % timeit(lambda: net.iteration()))
+print("concurrent WGRAD   %.4f ms" % timeit(lambda: net.iteration(concurrent=True)))
 print("eager, op events   %.4f ms" % timeit(with_events))
 t0 = time.perf_counter(); net.iteration(); torch.cuda.synchronize()
 t1 = time.perf_counter(); net.iteration(); t2 = time.perf_counter(); torch.cuda.synchronize()
 print("host enqueue time  %.4f ms (wall of one iteration without sync)" % ((t2 - t1) * 1e3))
-g = torch.cuda.CUDAGraph()
-s2 = torch.cuda.Stream()
-s2.wait_stream(st)
-with torch.cuda.stream(s2):
-    net.iteration()
-st.wait_stream(s2)
-torch.cuda.synchronize()
-with torch.cuda.graph(g):
-    net.iteration()
-torch.cuda.synchronize()
-print("cuda graph replay  %.4f ms" % timeit(lambda: g.replay()))

@@ -182,8 +182,7 @@ def run_reference(args):
             "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": {"workload": f"{args.config} conv layers fwd+bwd ({n_kernels(layers, args.input_grad)} kernels)",
                        "batch_per_gpu": args.batch, "math": "fp64 oracle",
-                       "first_layer_backward_data": bool(args.input_grad),
-                       "backward_streams": 2 if args.concurrent_wgrad else 1},
+                       "first_layer_backward_data": bool(args.input_grad)},
             "cpu_baseline": cb,
             "e2e": {"value": round(ms, 3), "unit": "ms/iter", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
@@ -416,7 +415,8 @@ def main():
                        "ws_limit_mib": (args.wd_mib if args.wd_mib > 0 else args.ws_mib),
                        "batch_size_policy": args.policy, "parallelism": f"dp{world}",
                        "l2": "512 MiB buffer overwritten before every timed step",
-                       "first_layer_backward_data": bool(args.input_grad)},
+                       "first_layer_backward_data": bool(args.input_grad),
+                       "backward_streams": 2 if args.concurrent_wgrad else 1},
             "images_per_s": round(args.batch * world / (ms_max * 1e-3), 1),
             "conv_tflops_direct": round(conv_flops / (ms_max * 1e-3) / 1e12, 2),
             "ms_per_step_with_op_events": round(ms_ops, 4),

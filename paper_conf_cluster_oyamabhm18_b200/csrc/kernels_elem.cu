@@ -28,6 +28,22 @@ __device__ __forceinline__ void pdl_entry() {
     asm volatile("griddepcontrol.launch_dependents;" :::);
 }
 
+// Division by a runtime divisor d >= 1 as a multiply-high (round-up method,
+// l = ceil(log2 d), m = floor(2^32 (2^l - d) / d) + 1; exact for all 32-bit n):
+// the index math of the memory-bound transform kernels below was dominated by
+// integer divisions.
+struct FastDiv {
+    uint32_t d, m, l;
+    FastDiv() = default;
+    explicit FastDiv(uint32_t dv) : d(dv), l(0) {
+        while ((1ull << l) < dv) ++l;
+        m = (uint32_t)((((1ull << 32) * ((1ull << l) - dv)) / dv) + 1);
+    }
+    __device__ __forceinline__ uint32_t div(uint32_t n) const {
+        return (uint32_t)(((uint64_t)__umulhi(n, m) + n) >> l);
+    }
+};
+
 template <typename... KArgs, typename... Args>
 void launch_pdl(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st, Args... args) {
     static const int pdl = getenv("MUCU_PDL") ? atoi(getenv("MUCU_PDL")) : 1;
@@ -509,24 +525,26 @@ __global__ void col2im_taps_kernel(const float* __restrict__ dcol, T* __restrict
 // 16-B chunk of xs, so every store is a full vector.
 template <class T>
 __global__ void s2d_input_kernel(const T* __restrict__ x, T* __restrict__ xs, int chunks, int H, int W, int C,
-                                 int I, int J, int st, int pad, int Cs) {
+                                 FastDiv divI, FastDiv divJ, FastDiv divCpp, FastDiv divStc, FastDiv divC, int st,
+                                 int pad, int Cs) {
     pdl_entry();
     constexpr int V = 16 / sizeof(T);
-    const int cpp = Cs / V, stc = st * C, real = st * stc;
-    // 32-bit index math (the launcher checks the range): 64-bit divisions
-    // dominated the first version of this memory-bound kernel.
+    const int stc = (int)divStc.d, real = st * stc;
+    // 32-bit index math with multiply-high divisions (the launcher checks the range)
     for (int idx = blockIdx.x * blockDim.x + threadIdx.x; idx < chunks; idx += gridDim.x * blockDim.x) {
-        const int pix = idx / cpp;
-        const int c0 = (idx - pix * cpp) * V;
+        const int pix = (int)divCpp.div((uint32_t)idx);
+        const int c0 = (idx - pix * (int)divCpp.d) * V;
         __align__(16) T vals[V];
         if (c0 >= real) {
 #pragma unroll
             for (int u = 0; u < V; ++u) vals[u] = from_f<T>(0.f);
         } else {
-            const int t = pix / J, j = pix - t * J;
-            const int n = t / I, i = t - n * I;
+            const int t = (int)divJ.div((uint32_t)pix), j = pix - t * (int)divJ.d;
+            const int n = (int)divI.div((uint32_t)t), i = t - n * (int)divI.d;
             const int h0 = st * i - pad, w0 = st * j - pad;
-            int a = c0 / stc, b = (c0 - a * stc) / C, c = c0 - a * stc - b * C;
+            int a = (int)divStc.div((uint32_t)c0);
+            const int r0 = c0 - a * stc;
+            int b = (int)divC.div((uint32_t)r0), c = r0 - b * C;
             const T* xn = x + (size_t)n * H * W * C;
 #pragma unroll
             for (int u = 0; u < V; ++u) {
@@ -684,32 +702,35 @@ __global__ void pad_channels_kernel(const T* __restrict__ x, T* __restrict__ xp,
 // xp[n][h][w'][c'] = x[n][h][w' - pad][c'] (zero outside 0 <= w' - pad < W or
 // c' >= C); one 16-B store per thread.
 template <typename T>
-__global__ void win_pad_kernel(const T* __restrict__ x, T* __restrict__ xp, int64_t units, int W, int Wp, int C,
+__global__ void win_pad_kernel(const T* __restrict__ x, T* __restrict__ xp, int units, int W, FastDiv divWp, int C,
                                int pad) {
     pdl_entry();
     constexpr int V = 16 / sizeof(T);  // elements per unit = V / 4 pixels of 4 channels
-    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < units; i += (int64_t)gridDim.x * blockDim.x) {
-        const int64_t e0 = i * V;
-        const int64_t pix0 = e0 / 4;          // padded pixel index (n, h, w')
-        const int64_t row = pix0 / Wp;        // (n, h)
-        const int w0 = (int)(pix0 - row * Wp);
+    for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < units; i += gridDim.x * blockDim.x) {
+        const int e0 = i * V;
+        const int pix0 = e0 / 4;                           // padded pixel index (n, h, w')
+        const int row = (int)divWp.div((uint32_t)pix0);     // (n, h)
+        const int w0 = pix0 - row * (int)divWp.d;
         __align__(16) T v[V];
 #pragma unroll
         for (int u = 0; u < V; ++u) {
             const int w = w0 + u / 4 - pad, c = u % 4;
-            v[u] = (c < C && w >= 0 && w < W) ? x[(row * W + w) * C + c] : from_f<T>(0.f);
+            v[u] = (c < C && w >= 0 && w < W) ? x[((size_t)row * W + w) * C + c] : from_f<T>(0.f);
         }
-        *reinterpret_cast<uint4*>(xp + e0) = *reinterpret_cast<const uint4*>(v);
+        *reinterpret_cast<uint4*>(xp + (size_t)e0) = *reinterpret_cast<const uint4*>(v);
     }
 }
 int launch_win_pad(const Geom& g, int32_t b, int Wp, const void* x, void* xp, cudaStream_t st) {
     const int64_t units = (int64_t)b * g.h * Wp * 4 * elt_size(g.math) / 16;
+    if (units * (16 / elt_size(g.math)) >= (1LL << 31)) return (int)cudaErrorInvalidValue;
     const int grid = grid_for(units, 256);
+    const FastDiv dWp(Wp);
     if (g.math == MUCU_MATH_BF16)
-        launch_pdl(win_pad_kernel<__nv_bfloat16>, dim3(grid), dim3(256), (size_t)(0), st, (const __nv_bfloat16*)x, (__nv_bfloat16*)xp, units, g.w,
-                                                            Wp, g.c, g.pad);
+        launch_pdl(win_pad_kernel<__nv_bfloat16>, dim3(grid), dim3(256), (size_t)0, st, (const __nv_bfloat16*)x,
+                   (__nv_bfloat16*)xp, (int)units, g.w, dWp, g.c, g.pad);
     else
-        launch_pdl(win_pad_kernel<float>, dim3(grid), dim3(256), (size_t)(0), st, (const float*)x, (float*)xp, units, g.w, Wp, g.c, g.pad);
+        launch_pdl(win_pad_kernel<float>, dim3(grid), dim3(256), (size_t)0, st, (const float*)x, (float*)xp,
+                   (int)units, g.w, dWp, g.c, g.pad);
     count_launch();
     return (int)cudaGetLastError();
 }
@@ -782,12 +803,13 @@ int launch_s2d_input(const Geom& g, int32_t b, int f, int I, int J, int Cs, cons
     const int64_t chunks = (int64_t)b * I * J * (Cs / V);
     if (chunks >= (1LL << 31) || (int64_t)g.h * g.w * g.c >= (1LL << 31)) return (int)cudaErrorInvalidValue;
     const int grid = grid_for(chunks, 256);
+    const FastDiv dI(I), dJ(J), dCpp(Cs / V), dStc(f * g.c), dC(g.c);
     if (g.math == MUCU_MATH_BF16)
-        launch_pdl(s2d_input_kernel<__nv_bfloat16>, dim3(grid), dim3(256), (size_t)(0), st, (const __nv_bfloat16*)x, (__nv_bfloat16*)xs, (int)chunks,
-                                                              g.h, g.w, g.c, I, J, f, g.pad, Cs);
+        launch_pdl(s2d_input_kernel<__nv_bfloat16>, dim3(grid), dim3(256), (size_t)0, st, (const __nv_bfloat16*)x,
+                   (__nv_bfloat16*)xs, (int)chunks, g.h, g.w, g.c, dI, dJ, dCpp, dStc, dC, f, g.pad, Cs);
     else
-        launch_pdl(s2d_input_kernel<float>, dim3(grid), dim3(256), (size_t)(0), st, (const float*)x, (float*)xs, (int)chunks, g.h, g.w, g.c, I, J,
-                                                      f, g.pad, Cs);
+        launch_pdl(s2d_input_kernel<float>, dim3(grid), dim3(256), (size_t)0, st, (const float*)x, (float*)xs,
+                   (int)chunks, g.h, g.w, g.c, dI, dJ, dCpp, dStc, dC, f, g.pad, Cs);
     count_launch();
     return (int)cudaGetLastError();
 }

@@ -15,16 +15,20 @@ from synthetic import network
 pytestmark = pytest.mark.gpu
 
 
-@pytest.mark.parametrize("config,math", [("alexnet", mu.MATH_TF32), ("resnet18", mu.MATH_BF16)],
-                         ids=["alexnet-tf32", "resnet18-bf16"])
-def test_concurrent_backward_matches_sequential(config, math):
+@pytest.mark.parametrize("config,math,policy", [("alexnet", mu.MATH_TF32, "wr"), ("resnet18", mu.MATH_BF16, "wr"),
+                                                ("alexnet", mu.MATH_BF16, "wd")],
+                         ids=["alexnet-tf32-wr", "resnet18-bf16-wr", "alexnet-bf16-wd"])
+def test_concurrent_backward_matches_sequential(config, math, policy):
     h = mu.Handle(0)
     h.set_policy(mu.POLICY_POW2)
     net = ConvNet(h, network(config), 8, math, device="cuda")
     net.allocate(seed=5, kind="int")
     limit = 8 << 20                       # tight: micro-batched plans
     net.benchmark_all(limit)
-    net.plan_wr(limit)
+    if policy == "wr":
+        net.plan_wr(limit)
+    else:  # one shared network workspace: concurrent kernels use disjoint segments
+        net.plan_wd(len(net.kernels) * limit // 2)
 
     def outputs():
         torch.cuda.synchronize()
@@ -44,5 +48,5 @@ def test_concurrent_backward_matches_sequential(config, math):
     for i, (a, b) in enumerate(zip(seq, con)):
         for k in ("y", "dx", "dw"):
             assert np.array_equal(a[k], b[k]), (config, i, k)
-    if config == "alexnet":  # at 8 MiB some AlexNet kernels really are micro-batched
+    if config == "alexnet" and policy == "wr":  # at 8 MiB some AlexNet kernels really are micro-batched
         assert any(len(k.plan) > 1 for k in net.kernels.values())

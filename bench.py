@@ -158,7 +158,7 @@ def auto_sample(layers, batch, input_grad=True):
     """Pick the oracle sample so one measurement takes ~10-20 s on this host
     (one probe image through every kernel, then scale)."""
     per_img = oracle_sample_time(layers, 1, input_grad=input_grad)
-    n = int(max(1, min(batch, 12.0 / max(per_img, 1e-6))))
+    n = int(max(1, min(batch, 20.0 / max(per_img, 1e-6))))  # powers of two below: ~10-20 s
     while batch % n:
         n -= 1
     return n

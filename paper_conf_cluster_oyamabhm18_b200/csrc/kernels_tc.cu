@@ -770,6 +770,16 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
             A.tapR = Dr; A.tapS = Ds; A.im2col_dgrad = 1; A.gsrc = in0; A.ph_u = u;
             A.e_H = g.h; A.e_W = g.w; A.e_C = g.c; A.e_pad = g.pad;
             finalize_tiling(L, elt);
+            // The row-wise depth-to-space epilogue reads TMEM in 4-column pieces, so the
+            // tile can be exactly N = f*f*C columns when that is a legal UMMA N (ResNet:
+            // 48 instead of 64)
+            const bool rows_ok = beta == 0.f && (f * g.c) % 4 == 0 && env_int("MUCU_D2S_ROWS", 1);
+            if (rows_ok && A.N < A.BN && A.N % 16 == 0 && env_int("MUCU_D2S_EXACT_N", 1)) {
+                A.BN = A.N;
+                A.bn_atoms = (A.BN * elt + 127) / 128;
+                A.b_bytes = std::max(A.BN * 128, A.bn_atoms * (128 / elt) * 128);
+                size_stages(A);
+            }
             use_mt2(L, num_sms);
             grid2(1);
             // start pixel of super-pixel (i, j): (u*i - (Dr - u), u*j - (Ds - u)); the kernel's
@@ -781,7 +791,7 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
                 return -1;
             if (!map2(&L.tb, ws, Kp, A.N, Kp, KB, A.BN)) return -1;
             A.tma_bytes = 16384 * A.mt + A.BN * 128;
-            A.d2s_rows = beta == 0.f && A.N <= A.BN && (f * g.c) % 4 == 0 && env_int("MUCU_D2S_ROWS", 1);
+            A.d2s_rows = rows_ok && A.N <= A.BN;
             return LAUNCH(A_TMA_IM2COL, B_TMA_K2, EPI_D2S);
         }
         const int I = z.I, J = z.J;

@@ -767,7 +767,8 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
             for (int kb = kb_begin; kb < kb_end; ++kb, s = (s + 1 == S) ? 0 : s + 1, ph ^= (s == 0) ? 1u : 0u) {
                 mbar_wait(smem_u32(&full[s]), ph);
                 tc_fence_after();
-                if (lane == 0 && !(p.debug & 8)) {  // debug bit 3: no MMAs (load-rate experiments)
+                // whole warp (converged): elect.sync inside the MMA / commit picks the issuer
+                if (!(p.debug & 8)) {  // debug bit 3: no MMAs (load-rate experiments)
                     const uint32_t aT = smem_u32(sA + (size_t)s * A_BYTES);
                     const uint32_t bT = B_RES ? smem_u32(sBres) + (uint32_t)(kb * p.BN * 128)
                                               : smem_u32(sB + (size_t)s * B_BYTES);
@@ -798,8 +799,8 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                                     : A_NOSWZ ? sdesc(aH + j * 4096, 2048, 128, 0)
                                     : A_MN  ? sdesc(aH + kofs + j * UMMA_K * 128, KDm * 128, MN_SBO, MN_LAYOUT)
                                             : sdesc(aH + j * 32, 16, 1024);
-                                mma<ELT>(dtm + (uint32_t)(hh * p.BN), ad, bd, idesc,
-                                         (kb > kb_begin || jj > 0 || j > 0) ? 1u : 0u);
+                                mma_elect<ELT>(dtm + (uint32_t)(hh * p.BN), ad, bd, idesc,
+                                               (kb > kb_begin || jj > 0 || j > 0) ? 1u : 0u);
                             }
                         }
                     };
@@ -814,7 +815,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                         else if (p.mt == 2) issue(std::integral_constant<int, 2>{}, 0);
                         else issue(std::integral_constant<int, 1>{}, 0);
                     }
-                    mma_commit(smem_u32(&empty[s]));
+                    mma_commit_elect(smem_u32(&empty[s]));
                 }
                 __syncwarp();
             }

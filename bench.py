@@ -234,7 +234,7 @@ def main():
     # (network.iteration concurrent=True); the evented per-op pass is sequential.
     conc = args.concurrent_wgrad
 
-    def timed(nsteps, nwarm, record_ops=False, e2e=None):
+    def timed(nsteps, nwarm, record_ops=False):
         ops = {}
         for _ in range(nwarm):
             net.iteration(grad_hook=grad_ar, skip_conv1_dgrad=not args.input_grad, concurrent=conc and not record_ops)
@@ -250,8 +250,6 @@ def main():
             ev = []
 
             def on_op(i, t, what):
-                if e2e is not None:
-                    e2e["on_op"](i, t, what)
                 if record_ops:
                     e = torch.cuda.Event(enable_timing=True)
                     e.record(stream)
@@ -259,13 +257,9 @@ def main():
             s0 = torch.cuda.Event(enable_timing=True)
             s1 = torch.cuda.Event(enable_timing=True)
             s0.record(stream)
-            if e2e is not None:
-                e2e["h2d"]()
             net.iteration(on_op=on_op, grad_hook=grad_ar, skip_conv1_dgrad=not args.input_grad,
                           concurrent=conc and not record_ops)
             grad_ar.wait()
-            if e2e is not None:
-                e2e["d2h"]()
             s1.record(stream)
             s1.synchronize()
             step_ms.append(s0.elapsed_time(s1))
@@ -318,37 +312,62 @@ def main():
     dy_host = net.tensors[-1]["dy"].detach().cpu().pin_memory()
     dw_host = [torch.empty_like(t["dw"], device="cpu").pin_memory() for t in net.tensors]
 
-    # x gates the first FWD call; dy (needed from the first backward call on) and
-    # each layer's dW (ready after its BackwardFilter) move on a copy stream that
-    # overlaps the compute stream -- what a training loop feeding this API does.
-    copy_stream = torch.cuda.Stream()
-    dy_ready = torch.cuda.Event()
+    # The input pipeline of a training loop: step k+1's x and dy are uploaded from
+    # pinned host memory (double-buffered, on an upload stream) while step k
+    # computes, and each layer's dW is read back to the host (download stream)
+    # as soon as its BackwardFilter is done.  Every timed step performs its own
+    # h2d_bytes / d2h_bytes of copies; the first step's upload is not hidden.
+    up_stream, down_stream = torch.cuda.Stream(), torch.cuda.Stream()
+    x_bufs = [net.tensors[0]["x"], torch.empty_like(net.tensors[0]["x"])]
+    dy_bufs = [net.tensors[-1]["dy"], torch.empty_like(net.tensors[-1]["dy"])]
+    ready = [torch.cuda.Event(), torch.cuda.Event()]
+    done = [torch.cuda.Event(), torch.cuda.Event()]
 
-    def h2d():
-        net.tensors[0]["x"].copy_(x_host, non_blocking=True)
-        copy_stream.wait_stream(stream)
-        with torch.cuda.stream(copy_stream):
-            net.tensors[-1]["dy"].copy_(dy_host, non_blocking=True)
-            dy_ready.record(copy_stream)
-
-    first_bwd = [True]
+    def upload(k):
+        j = k % 2
+        if k >= 2:
+            up_stream.wait_event(done[j])  # step k-2 has finished with these buffers
+        with torch.cuda.stream(up_stream):
+            x_bufs[j].copy_(x_host, non_blocking=True)
+            dy_bufs[j].copy_(dy_host, non_blocking=True)
+            ready[j].record(up_stream)
 
     def e2e_op(i, t, what):
-        if what in ("begin", "first") and t != mu.FWD and first_bwd[0]:
-            stream.wait_event(dy_ready)
-            first_bwd[0] = False
         if what == "end" and t == mu.BWD_FILTER and not distributed:  # N > 1: after the dW allreduce
-            copy_stream.wait_stream(torch.cuda.current_stream())  # the BackwardFilter's stream
-            with torch.cuda.stream(copy_stream):
+            down_stream.wait_stream(torch.cuda.current_stream())  # the BackwardFilter's stream
+            with torch.cuda.stream(down_stream):
                 dw_host[i].copy_(net.tensors[i]["dw"], non_blocking=True)
 
-    def d2h():
-        if distributed:
-            for t, hbuf in zip(net.tensors, dw_host):
-                hbuf.copy_(t["dw"], non_blocking=True)
-        stream.wait_stream(copy_stream)
-        first_bwd[0] = True
-    e2e_ms, _, _ = timed(max(3, args.steps // 2), 1, e2e={"h2d": h2d, "d2h": d2h, "on_op": e2e_op})
+    def e2e_run(nsteps):
+        s0, s1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        s0.record(stream)
+        upload(0)
+        for k in range(nsteps):
+            if k + 1 < nsteps:
+                upload(k + 1)  # prefetch the next step's inputs while this one computes
+            j = k % 2
+            stream.wait_event(ready[j])
+            net.tensors[0]["x"], net.tensors[-1]["dy"] = x_bufs[j], dy_bufs[j]
+            net.iteration(on_op=e2e_op, grad_hook=grad_ar, skip_conv1_dgrad=not args.input_grad,
+                          concurrent=conc)
+            grad_ar.wait()
+            if distributed:
+                down_stream.wait_stream(stream)
+                with torch.cuda.stream(down_stream):
+                    for t, hbuf in zip(net.tensors, dw_host):
+                        hbuf.copy_(t["dw"], non_blocking=True)
+            stream.wait_stream(down_stream)  # the step's results are on the host
+            done[j].record(stream)
+        s1.record(stream)
+        s1.synchronize()
+        return s0.elapsed_time(s1) / nsteps
+
+    e2e_run(2)  # warm-up
+    torch.cuda.synchronize()
+    if distributed:
+        dist.barrier()
+    e2e_ms = e2e_run(max(5, args.steps))
+    net.tensors[0]["x"], net.tensors[-1]["dy"] = x_bufs[0], dy_bufs[0]
     e2e_ms = max_over_ranks(e2e_ms)
     h2d_bytes = x_host.numel() * x_host.element_size() + dy_host.numel() * dy_host.element_size()
     d2h_bytes = sum(b.numel() * 4 for b in dw_host)

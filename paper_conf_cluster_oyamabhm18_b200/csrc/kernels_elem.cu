@@ -656,18 +656,24 @@ __global__ void scale_kernel(float* __restrict__ p, int64_t n, float beta) {
 // Strided DGRAD: dx pixels whose phase ((h+pad) % st, (w+pad) % st) meets no
 // filter tap (r0 >= R or s0 >= S, e.g. 3 of 4 pixels of a 1x1 stride-2 layer)
 // receive no gradient: zero them (beta = 0) in one pass of 16-B stores.
-__global__ void zero_tapless_kernel(uint4* __restrict__ dx, int rows, int cpp, int H, int W, int R, int S, int pad,
-                                    int st) {
+__global__ void zero_tapless_kernel(uint4* __restrict__ dx, int rows, FastDiv div_cpp, FastDiv div_st, int H, int W,
+                                    int R, int S, int pad, int st) {
     pdl_entry();
-    // one block per dx pixel row (n, h); a row whose phase meets no tap is zeroed whole
-    const int per_row = W * cpp;
+    // one block per dx pixel row (n, h); a row whose phase meets no tap is zeroed
+    // whole, otherwise only the pixels whose column phase meets no tap (the
+    // per-element index math uses a multiply-high division: this pass writes
+    // up to 3/4 of dx for 1x1 stride-2 layers and was instruction-bound)
+    const int cpp = (int)div_cpp.d, per_row = W * cpp;
     for (int row = blockIdx.x; row < rows; row += gridDim.x) {
         const int h = row % H;
-        const bool all = (h + pad) % st >= R;
         uint4* d = dx + (int64_t)row * per_row;
+        if ((h + pad) % st >= R) {
+            for (int i = threadIdx.x; i < per_row; i += blockDim.x) d[i] = make_uint4(0u, 0u, 0u, 0u);
+            continue;
+        }
         for (int i = threadIdx.x; i < per_row; i += blockDim.x) {
-            const int w = i / cpp;
-            if (all || (w + pad) % st >= S) d[i] = make_uint4(0u, 0u, 0u, 0u);
+            const int wp = (int)div_cpp.div((uint32_t)i) + pad;
+            if (wp - (int)div_st.div((uint32_t)wp) * st >= S) d[i] = make_uint4(0u, 0u, 0u, 0u);
         }
     }
 }
@@ -678,7 +684,7 @@ int launch_zero_tapless(const Geom& g, int32_t b, void* dx, cudaStream_t st) {
     if ((g.c * elt) % 16 != 0) return -1;
     const int cpp = g.c * elt / 16;
     const int rows = b * g.h;
-    launch_pdl(zero_tapless_kernel, dim3(std::min(rows, 148 * 16)), dim3(256), (size_t)(0), st, (uint4*)dx, rows, cpp, g.h, g.w, g.r, g.s, g.pad,
+    launch_pdl(zero_tapless_kernel, dim3(std::min(rows, 148 * 16)), dim3(256), (size_t)(0), st, (uint4*)dx, rows, FastDiv(cpp), FastDiv(g.stride), g.h, g.w, g.r, g.s, g.pad,
                                                                   g.stride);
     count_launch();
     return (int)cudaGetLastError();

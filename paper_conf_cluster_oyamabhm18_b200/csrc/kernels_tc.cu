@@ -79,6 +79,13 @@ __device__ __forceinline__ void tma_load_4d(uint32_t dst, const CUtensorMap* tm,
         "l"((uint64_t)tm), "r"(bar), "r"(c0), "r"(c1), "r"(c2), "r"(c3)
         : "memory");
 }
+__device__ __forceinline__ void tma_load_5d(uint32_t dst, const CUtensorMap* tm, uint32_t bar, int c0, int c1, int c2,
+                                            int c3, int c4) {
+    asm volatile(
+        "cp.async.bulk.tensor.5d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4, %5, %6, %7}], [%2];" ::"r"(dst),
+        "l"((uint64_t)tm), "r"(bar), "r"(c0), "r"(c1), "r"(c2), "r"(c3), "r"(c4)
+        : "memory");
+}
 // TMA im2col mode (4-D NHWC tensor {C, W, H, N}): pixelsPerColumn consecutive
 // pixels starting at (w, h, n) (walking W, then H, then N inside the map's
 // bounding box with the map's traversal stride), channelsPerPixel channels
@@ -277,6 +284,7 @@ struct TcArgs {
     int d2s_rows;            // EPI_D2S by dx rows (beta = 0, one N tile, f*C % 4 == 0)
     // Window WGRAD (A_TMA_WIN / B_TMA_DYROW): 128-B atoms per filter row, q-blocks per output row
     int win_na, win_qb, win_aw;  // + bytes per A swizzle atom (128 / 64 / 32: UMMA layout 2 / 4 / 6)
+    int win_box;             // > 0: one 5-D TMA box {atom, KD pixels, na, win_box filter rows} per 128-row half
     // Halo IG (A_HALO): extended grid of hx_H = Ho + R - 1 rows x hx_W (>= Wo + S - 1, multiple of 8)
     // columns per image; source origin offset hx_pe; hx_nch channel chunks of 128 B; halo ring
     int hx_W, hx_H, hx_Ho, hx_Wo, hx_pe, hx_nch, halo_bytes, hstages;
@@ -374,8 +382,8 @@ bool make_map(CUtensorMap* tm, int elt, const void* base, int rank, const uint64
                                                              : CU_TENSOR_MAP_SWIZZLE_128B;
     EncodeTiledFn enc = get_encode();
     if (!enc) return false;
-    cuuint64_t d[4], s[3];
-    cuuint32_t b[4], e[4] = {1, 1, 1, 1};
+    cuuint64_t d[5], s[4];
+    cuuint32_t b[5], e[5] = {1, 1, 1, 1, 1};
     for (int i = 0; i < rank; ++i) { d[i] = dims[i]; b[i] = box[i]; }
     for (int i = 0; i < rank - 1; ++i) s[i] = strides_bytes[i];
     CUresult r = enc(tm, elt == 2 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32, rank,
@@ -758,10 +766,24 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         const int KD = KB * A.km;
         const uint64_t pb = (uint64_t)z.cpx * elt;
         const int wat = z.aw / elt;  // elements per A atom
-        uint64_t adims[4] = {(uint64_t)z.na * wat, (uint64_t)g.q, (uint64_t)g.h, (uint64_t)b};
-        uint64_t astr[3] = {g.stride * pb, z.Wp * pb, (uint64_t)g.h * z.Wp * pb};
-        uint32_t abox[4] = {(uint32_t)wat, (uint32_t)KD, 1, 1};
-        if (!make_map(&L.ta, elt, xp, 4, adims, astr, abox, true, z.aw)) return -1;
+        // One 5-D box per 128-row half when the half holds whole filter rows: view
+        // {atom element, output pixel q (stride st*16 B), atom aa, input row h, image}
+        // gives the smem order [r][aa][q][element] the per-atom boxes produce, in one
+        // TMA instead of 4-8 small ones (filter rows past R load real data, discarded).
+        const int atoms_half = 128 * elt / z.aw;
+        if (atoms_half % z.na == 0 && env_int("MUCU_WIN_BOX", 1)) {
+            const int hext = atoms_half / z.na;
+            uint64_t adims[5] = {(uint64_t)wat, (uint64_t)g.q, (uint64_t)z.na, (uint64_t)g.h, (uint64_t)b};
+            uint64_t astr[4] = {g.stride * pb, (uint64_t)wat * elt, z.Wp * pb, (uint64_t)g.h * z.Wp * pb};
+            uint32_t abox[5] = {(uint32_t)wat, (uint32_t)KD, (uint32_t)z.na, (uint32_t)hext, 1};
+            if (make_map(&L.ta, elt, xp, 5, adims, astr, abox, true, z.aw)) A.win_box = hext;
+        }
+        if (!A.win_box) {
+            uint64_t adims[4] = {(uint64_t)z.na * wat, (uint64_t)g.q, (uint64_t)g.h, (uint64_t)b};
+            uint64_t astr[3] = {g.stride * pb, z.Wp * pb, (uint64_t)g.h * z.Wp * pb};
+            uint32_t abox[4] = {(uint32_t)wat, (uint32_t)KD, 1, 1};
+            if (!make_map(&L.ta, elt, xp, 4, adims, astr, abox, true, z.aw)) return -1;
+        }
         if (!map3(&L.tb, in1, g.k, g.q, (uint64_t)b * g.p, g.k, (uint64_t)g.q * g.k, atom, KD, 1, true)) return -1;
         A.tma_bytes = A.km * (A.mt * 128 * KB * elt + A.bn_atoms * KB * 128);
         if (z.aw == 64) return LAUNCH(A_TMA_WIN64, B_TMA_DYROW, EPI_WGRAD_WIN);

@@ -401,6 +401,10 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                             // atoms of aw bytes, 128*ELT/aw of them per 128 rows
                             const int n_ = wr_row / p.P, p_ = wr_row - n_ * p.P;
                             constexpr int wat = WAW / ELT;
+                            if (p.win_box) {
+                                const int r0 = (mH / wat) / p.win_na;
+                                tma_load_5d(aH, &tmA, fb, 0, wr_qb * KD, 0, p.stride * p_ + r0 - p.pad, n_);
+                            } else
 #pragma unroll
                             for (int a = 0; a < 128 * ELT / (int)WAW; ++a) {
                                 const int ja = mH / wat + a;

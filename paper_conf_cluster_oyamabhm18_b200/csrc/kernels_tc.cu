@@ -285,6 +285,7 @@ struct TcArgs {
     // Window WGRAD (A_TMA_WIN / B_TMA_DYROW): 128-B atoms per filter row, q-blocks per output row
     int win_na, win_qb, win_aw;  // + bytes per A swizzle atom (128 / 64 / 32: UMMA layout 2 / 4 / 6)
     int win_box;             // > 0: one 5-D TMA box {atom, KD pixels, na, win_box filter rows} per 128-row half
+    int a_box;               // A_TMA_MN2: one 3-D box {atom, KD, atoms} per 128-row half
     // Halo IG (A_HALO): extended grid of hx_H = Ho + R - 1 rows x hx_W (>= Wo + S - 1, multiple of 8)
     // columns per image; source origin offset hx_pe; hx_nch channel chunks of 128 B; halo ring
     int hx_W, hx_H, hx_Ho, hx_Wo, hx_pe, hx_nch, halo_bytes, hstages;
@@ -1175,7 +1176,20 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         }
         (void)sem;
         const int a_bytes = 128 * KB * elt;
-        auto map_dy = [&]() { return map2(&L.ta, in1, g.k, (uint64_t)Mpix, g.k, atom, KB * A.km, true); };
+        // dy as the MN-major A operand: with K a multiple of the 128-B atom, a 3-D view
+        // {atom element, pixel, atom index} loads a whole 128-row half (4 tf32 atoms) in
+        // one TMA box instead of one box per atom (AlexNet TF32 WGRAD -4..11 %; for BF16's
+        // 2 atoms it measured mixed, -5 % to +30 %, so BF16 keeps per-atom boxes).
+        auto map_dy = [&]() {
+            A.a_box = 0;
+            if (g.k % atom == 0 && env_int("MUCU_A_BOX", elt == 4 ? 1 : 0)) {
+                uint64_t dims[3] = {(uint64_t)atom, (uint64_t)Mpix, (uint64_t)(g.k / atom)};
+                uint64_t str[2] = {(uint64_t)g.k * elt, 128};
+                uint32_t box[3] = {(uint32_t)atom, (uint32_t)(KB * A.km), (uint32_t)elt};
+                if (make_map(&L.ta, elt, in1, 3, dims, str, box, true)) { A.a_box = 1; return true; }
+            }
+            return map2(&L.ta, in1, g.k, (uint64_t)Mpix, g.k, atom, KB * A.km, true);
+        };
         if (algo == MUCU_ALGO_IM2COL_GEMM && small_c_tc(g)) {
             // RGB-like layer: channel-padded copy of x, padded columns j' = (r, s8, c').
             err = launch_pad_channels(g, b, in0, ws + WL.a_off, st);

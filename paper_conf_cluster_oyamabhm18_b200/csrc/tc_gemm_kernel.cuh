@@ -391,9 +391,13 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                         if constexpr (AM == A_TMA_K3) tma_load_3d(aH, &tmA, fb, kb * KB, mH, z);
                         if constexpr (AM == A_TMA_MN2) {
                             const int zr = p.zsplit ? (z / p.zsplit) * p.zrows : 0;
+                            if (p.a_box) {
+                                tma_load_3d(aH, &tmA, fb, 0, zr + kb * KD, mH / (128 / ELT));
+                            } else {
 #pragma unroll
-                            for (int a = 0; a < 128 * ELT / 128; ++a)
-                                tma_load_2d(aH + a * KD * 128, &tmA, fb, mH + a * (128 / ELT), zr + kb * KD);
+                                for (int a = 0; a < 128 * ELT / 128; ++a)
+                                    tma_load_2d(aH + a * KD * 128, &tmA, fb, mH + a * (128 / ELT), zr + kb * KD);
+                            }
                         }
                         if constexpr (WIN) {
                             // atom ja = (filter row r, atom aa): window of KD output pixels of row

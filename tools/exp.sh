@@ -1,8 +1,6 @@
 #!/bin/bash
 set -u
-timeout 900 python -m pytest tests/test_conv_gpu.py tests/test_tilings_gpu.py -q -x -k "c3 or c2 or 7x7" 2>&1 | tail -2
-for v in 0 1; do echo "== WIN_BOX=$v"
-MUCU_WIN_BOX=$v timeout 120 python tools/time_one.py --config alexnet --math tf32 --specs conv1:WGRAD:I2C:64
-MUCU_WIN_BOX=$v timeout 120 python tools/time_one.py --config alexnet --math bf16 --specs conv1:WGRAD:I2C:128
-MUCU_WIN_BOX=$v timeout 120 python tools/time_one.py --config resnet50 --math bf16 --specs conv1:WGRAD:I2C:128
-done
+timeout 900 python -m pytest tests -q -m gpu -x 2>&1 | tail -2
+MUCU_A_BOX=1 timeout 900 python -m pytest tests/test_conv_gpu.py -q -x -k "bf16 and WGRAD" 2>&1 | tail -1
+for c in "alexnet tf32" "resnet50 bf16"; do set -- $c; timeout 300 python bench.py --config $1 --math $2 --no-cpu-baseline --tables-in scratch/tables_$1_$2.npz 2>/dev/null | tail -1 | python -c "
+import json,sys; d=json.loads(sys.stdin.read()); print(d['config']['workload'], d['value'], d['e2e']['value'], d['roofline']['frac'], d['roofline']['step_frac'], d['clocks']['reasons'])"; done

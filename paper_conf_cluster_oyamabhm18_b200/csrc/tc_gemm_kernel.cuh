@@ -436,8 +436,12 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                         const int kpr = p.K / KB;
                         const int tap = kb / kpr, k0 = (kb - tap * kpr) * KB;
                         const int rs = dgrad_tap_rs(p, tap, pr0, ps0, tS);
-                        for (int a = 0; a < p.bn_atoms; ++a)
-                            tma_load_3d(bT + a * KB * 128, &tmB, fb, n0 + a * (128 / ELT), rs, k0);
+                        if (p.b_box) {
+                            tma_load_4d(bT, &tmB, fb, 0, rs, k0, n0 / (128 / ELT));
+                        } else {
+                            for (int a = 0; a < p.bn_atoms; ++a)
+                                tma_load_3d(bT + a * KB * 128, &tmB, fb, n0 + a * (128 / ELT), rs, k0);
+                        }
                     }
                     if constexpr (BM_ == B_TMA_DYROW) {
                         for (int a = 0; a < p.bn_atoms; ++a)

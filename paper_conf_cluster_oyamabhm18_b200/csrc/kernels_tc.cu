@@ -645,6 +645,18 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         CUtensorMap tmp;
         if (make_map(&tmp, elt, w, 4, dims, str, box, true)) { L.tb = tmp; A.b_box = 1; }
     };
+    // Dense MN-major B operand (rows of `pitch` elements, N = the contiguous dim):
+    // a 3-D view {atom element, k row, atom index} loads the stage's bn_atoms atoms in
+    // one TMA box when N, the tile N and the pitch are multiples of the 128-B atom.
+    auto map_mn_box = [&](const void* base, uint64_t ncols, uint64_t krows, uint64_t pitch, int krows_box) {
+        A.b_box = 0;
+        if (ncols % atom || pitch % atom || A.BN % atom || !env_int("MUCU_B_BOX", 1)) return;
+        uint64_t dims[3] = {(uint64_t)atom, krows, ncols / atom};
+        uint64_t str[2] = {pitch * elt, 128};
+        uint32_t box[3] = {(uint32_t)atom, (uint32_t)krows_box, (uint32_t)A.bn_atoms};
+        CUtensorMap tmp;
+        if (make_map(&tmp, elt, base, 3, dims, str, box, true)) { L.tb = tmp; A.b_box = 1; }
+    };
     // Persistent launch: one CTA per SM (at most one per tile).
     auto grid2 = [&](int batch) {
         A.num_z = batch;
@@ -968,6 +980,7 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         grid2(16 * nsplit);
         if (!map2(&L.ta, D, Kp, 16 * Tp, Kp, atom, KB * A.km, true)) return -1;
         if (!map2(&L.tb, V, Cp, 16 * Tp, Cp, atom, KB * A.km, true)) return -1;
+        map_mn_box(V, Cp, 16 * Tp, Cp, KB * A.km);
         A.tma_bytes = A.km * (A.mt * 128 * KB * elt + A.bn_atoms * KB * 128);
         err = LAUNCH(A_TMA_MN2, B_TMA_MN2, EPI_WGRAD_CHAIN);
         if (err) return err;
@@ -1177,6 +1190,7 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         if (wpitch < atom) return -1;  // pointwise with C < one atom
         if (!map2(&L.ta, in0, g.k, (uint64_t)A.M, g.k, KB, 128)) return -1;
         if (!map2(&L.tb, wp, std::max<int64_t>(RSC, atom), g.k, wpitch, atom, KB, true)) return -1;
+        map_mn_box(wp, (uint64_t)std::max<int64_t>(RSC, atom), g.k, wpitch, KB);
         A.tma_bytes = 16384 * A.mt + A.bn_atoms * KB * 128;
         err = LAUNCH(A_TMA_K2, B_TMA_MN2, EPI_STORE);
         if (err || pw) return err;
@@ -1231,6 +1245,7 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
             wgrad_tiling(16, true);
             if (!map_dy()) return -1;
             if (!map2(&L.tb, colp, RSC, (uint64_t)Mpix, kp, atom, KB * A.km, true)) return -1;
+            map_mn_box(colp, RSC, (uint64_t)Mpix, kp, KB * A.km);
             A.tma_bytes = A.km * (A.mt * a_bytes + A.bn_atoms * KB * 128);
             return LAUNCH(A_TMA_MN2, B_TMA_MN2, EPI_WGRAD_CHAIN);
         }

@@ -428,8 +428,12 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                     if constexpr (BM_ == B_TMA_K3) tma_load_3d(bT, &tmB, fb, kb * KB, n0, z);
                     if constexpr (BM_ == B_TMA_MN2) {
                         const int zr = p.zsplit ? (z / p.zsplit) * p.zrows : 0;
-                        for (int a = 0; a < p.bn_atoms; ++a)
-                            tma_load_2d(bT + a * KD * 128, &tmB, fb, n0 + a * (128 / ELT), zr + kb * KD);
+                        if (p.b_box) {
+                            tma_load_3d(bT, &tmB, fb, 0, zr + kb * KD, n0 / (128 / ELT));
+                        } else {
+                            for (int a = 0; a < p.bn_atoms; ++a)
+                                tma_load_2d(bT + a * KD * 128, &tmB, fb, n0 + a * (128 / ELT), zr + kb * KD);
+                        }
                     }
                     if constexpr (BM_ == B_TMA_MN3) {
                         // k-block kb covers tap kb / (K/KB), channels k0 = (kb % (K/KB)) * KB

@@ -287,6 +287,7 @@ struct TcArgs {
     int win_box;             // > 0: one 5-D TMA box {atom, KD pixels, na, win_box filter rows} per 128-row half
     int a_box;               // A_TMA_MN2: one 3-D box {atom, KD, atoms} per 128-row half
     int b_box;               // B_TMA_MN3: one 4-D box {atom, 1, KB, bn_atoms} per stage
+    int a_merged;            // A_TMA_IM2COL: one im2col box of 128*mt pixels per stage
     // Halo IG (A_HALO): extended grid of hx_H = Ho + R - 1 rows x hx_W (>= Wo + S - 1, multiple of 8)
     // columns per image; source origin offset hx_pe; hx_nch channel chunks of 128 B; halo ring
     int hx_W, hx_H, hx_Ho, hx_Wo, hx_pe, hx_nch, halo_bytes, hstages;
@@ -481,15 +482,32 @@ int pick_bn(int N, int step = 32, int overhead = 32, int max_bn = 256, int64_t m
     return best;
 }
 
+// Arguments of the A operand's TMA im2col map (re-encoded with 128*mt pixels per
+// box once the tile height is known: one transaction per stage instead of mt).
+struct Im2colArgs {
+    int valid, elt, C, W, H, N, lw, lh, uw, uh, stride;
+    const void* base;
+};
 struct Launch {
     TcArgs a;
     CUtensorMap ta, tb;
     dim3 grid;
+    Im2colArgs ia;
 };
 
 template <int ELT, int AM, int BM_, int EPI>
 int launch_t(Launch& L, cudaStream_t st) {
     auto kern = tc_conv_gemm<ELT, AM, BM_, EPI>;
+    L.a.a_merged = 0;
+    if (AM == A_TMA_IM2COL && L.a.mt > 1 && L.ia.valid && env_int("MUCU_A_MERGE", 1)) {
+        const Im2colArgs& q = L.ia;
+        CUtensorMap tmp;
+        if (make_im2col_map(&tmp, q.elt, q.base, q.C, q.W, q.H, q.N, q.lw, q.lh, q.uw, q.uh, 128 * L.a.mt, q.stride,
+                            false)) {
+            L.ta = tmp;
+            L.a.a_merged = 1;
+        }
+    }
     const int a_stage = AM == A_HALO ? 0 : L.a.mt * 128 * 128;
     const int smem = 1024 + L.a.hstages * L.a.halo_bytes + L.a.stages * L.a.km * (a_stage + L.a.b_bytes) +
                      L.a.bres_bytes + (2 * L.a.stages + 6 + 2 * L.a.hstages) * 8 + 64;
@@ -657,6 +675,11 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         CUtensorMap tmp;
         if (make_map(&tmp, elt, base, 3, dims, str, box, true)) { L.tb = tmp; A.b_box = 1; }
     };
+    auto im2col_a = [&](int e, const void* base, int C, int W, int H, int N, int lw, int lh, int uw, int uh, int pixels,
+                        int stride, bool mn) {
+        L.ia = Im2colArgs{1, e, C, W, H, N, lw, lh, uw, uh, stride, base};
+        return make_im2col_map(&L.ta, e, base, C, W, H, N, lw, lh, uw, uh, pixels, stride, mn);
+    };
     // Persistent launch: one CTA per SM (at most one per tile).
     auto grid2 = [&](int batch) {
         A.num_z = batch;
@@ -744,7 +767,7 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
                 }
             }
             if (use_tma_im2col() &&
-                make_im2col_map(&L.ta, elt, in0, g.c, g.w, g.h, b, -g.pad, -g.pad, g.pad - (g.s - 1),
+                im2col_a(elt, in0, g.c, g.w, g.h, b, -g.pad, -g.pad, g.pad - (g.s - 1),
                                 g.pad - (g.r - 1), 128, g.stride, false)) {
                 use_mt2(L, num_sms);
                 grid2(1);
@@ -859,7 +882,7 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
             // phase-mode origin is ph_i0 + ii - (tapR - 1) in map units, so the map walks u-strided
             // positions lw, lw + u, ... with J of them per row.
             const int lw = -(Ds - u), lh = -(Dr - u);
-            if (!make_im2col_map(&L.ta, elt, in0, g.k, g.q, g.p, b, lw, lh, lw + u * (J - 1) - (g.q - 1),
+            if (!im2col_a(elt, in0, g.k, g.q, g.p, b, lw, lh, lw + u * (J - 1) - (g.q - 1),
                                  lh + u * (I - 1) - (g.p - 1), 128, u, false))
                 return -1;
             if (!map2(&L.tb, ws, Kp, A.N, Kp, KB, A.BN)) return -1;
@@ -881,7 +904,7 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
             finalize_tiling(L, elt);
             use_mt2(L, num_sms);
             grid2(1);
-            if (!make_im2col_map(&L.ta, elt, xs, Cs, J, I, b, 0, 0, -(Ds - 1), -(Dr - 1), 128, 1, false)) return -1;
+            if (!im2col_a(elt, xs, Cs, J, I, b, 0, 0, -(Ds - 1), -(Dr - 1), 128, 1, false)) return -1;
             if (!map2(&L.tb, ws, Kp, A.N, Kp, KB, A.BN)) return -1;
             A.tma_bytes = 16384 * A.mt + A.BN * 128;
             if (z.u == 1) return LAUNCH(A_TMA_IM2COL, B_TMA_K2, EPI_STORE);
@@ -1060,7 +1083,7 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
                 A.M = b * H0 * W0;
                 A.num_kb = 0;
                 for (int z = 0; z < n_ph; ++z) A.num_kb = std::max(A.num_kb, A.ph_kbv[z]);
-                if (!make_im2col_map(&L.ta, elt, in0, g.k, g.q, g.p, b, lw0, lh0, lw0 + W0 - g.q, lh0 + H0 - g.p, 128,
+                if (!im2col_a(elt, in0, g.k, g.q, g.p, b, lw0, lh0, lw0 + W0 - g.q, lh0 + H0 - g.p, 128,
                                      1, false))
                     return -1;
                 A.mt = 1;
@@ -1095,7 +1118,7 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
                 // dy im2col: start positions i0 - (nr-1) ... (Hph of them), stride 1
                 const int lh = i0 - (A.tapR - 1), lw = j0 - (A.tapS - 1);
                 if (A.num_kb > 0 &&
-                    !make_im2col_map(&L.ta, elt, in0, g.k, g.q, g.p, b, lw, lh, lw + Wph - g.q, lh + Hph - g.p,
+                    !im2col_a(elt, in0, g.k, g.q, g.p, b, lw, lh, lw + Wph - g.q, lh + Hph - g.p,
                                      128, 1, false))
                     return -1;
                 A.mt = 1;
@@ -1144,7 +1167,7 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
             // stride 1: im2col of dy with pad' = R-1-pad and flipped taps
             const int lw = g.pad - (g.s - 1), lh = g.pad - (g.r - 1);
             if (g.stride == 1 && use_tma_im2col() &&
-                make_im2col_map(&L.ta, elt, in0, g.k, g.q, g.p, b, lw, lh, lw + g.w - g.q, lh + g.h - g.p, 128, 1,
+                im2col_a(elt, in0, g.k, g.q, g.p, b, lw, lh, lw + g.w - g.q, lh + g.h - g.p, 128, 1,
                                 false)) {
                 A.im2col_dgrad = 1;
                 // C a multiple of 128 (> 128): 256 x 128 tiles (two interleaved

@@ -419,9 +419,11 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                         }
                         if constexpr (AM == A_TMA_IM2COL) {
                             // 128 consecutive output pixels x KB channels of tap (r,s) in one TMA
+                            // (a_merged: all 128*mt pixels of the tile in the first half's TMA)
                             const uint16_t ow = (uint16_t)(p.im2col_dgrad ? tS - 1 - g_s : g_s);
                             const uint16_t oh = (uint16_t)(p.im2col_dgrad ? tR - 1 - g_r : g_r);
-                            tma_load_im2col_4d(aH, &tmA, fb, g_c0, ic_w[hh], ic_h[hh], ic_n[hh], ow, oh);
+                            if (!p.a_merged || hh == 0)
+                                tma_load_im2col_4d(aH, &tmA, fb, g_c0, ic_w[hh], ic_h[hh], ic_n[hh], ow, oh);
                         }
                     }
                     if constexpr (BM_ == B_TMA_K2) tma_load_2d(bT, &tmB, fb, kb * KB, n0);

@@ -1231,12 +1231,12 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         (void)sem;
         const int a_bytes = 128 * KB * elt;
         // dy as the MN-major A operand: with K a multiple of the 128-B atom, a 3-D view
-        // {atom element, pixel, atom index} loads a whole 128-row half (4 tf32 atoms) in
-        // one TMA box instead of one box per atom (AlexNet TF32 WGRAD -4..11 %; for BF16's
-        // 2 atoms it measured mixed, -5 % to +30 %, so BF16 keeps per-atom boxes).
+        // {atom element, pixel, atom index} loads a whole 128-row half (4 tf32 / 2 bf16
+        // atoms) in one TMA box instead of one box per atom (AlexNet TF32 WGRAD -4..11 %,
+        // BF16 IG WGRAD -3..5 %, pointwise within noise).
         auto map_dy = [&]() {
             A.a_box = 0;
-            if (g.k % atom == 0 && env_int("MUCU_A_BOX", elt == 4 ? 1 : 0)) {
+            if (g.k % atom == 0 && env_int("MUCU_A_BOX", 1)) {
                 uint64_t dims[3] = {(uint64_t)atom, (uint64_t)Mpix, (uint64_t)(g.k / atom)};
                 uint64_t str[2] = {(uint64_t)g.k * elt, 128};
                 uint32_t box[3] = {(uint32_t)atom, (uint32_t)(KB * A.km), (uint32_t)elt};

@@ -373,7 +373,7 @@ def main():
     d2h_bytes = sum(b.numel() * 4 for b in dw_host)
 
     # ---- dominant kernel roofline ----
-    op_ms = {k: float(np.mean(v)) for k, v in ops.items()}
+    op_ms = {k: float(np.median(v)) for k, v in ops.items()}  # median: robust to a one-step hiccup
     dom = max(op_ms, key=op_ms.get)
     li, lt = dom
     kern = net.kernels[dom]

@@ -65,3 +65,25 @@ def test_alexnet_tf32_full_size_sampled():
 def test_resnet50_bf16_full_size_sampled_layers():
     _run("resnet50", mu.MATH_BF16, names={"conv1", "layer1.0.conv2", "layer2.0.conv2", "layer3.0.downsample",
                                           "layer4.2.conv3", "layer1.0.conv1"})
+
+
+def test_resnet18_bf16_full_size_sampled():
+    """BASELINE config 3 (ResNet-18, BF16, N = 256), every layer."""
+    _run("resnet18", mu.MATH_BF16)
+
+
+def test_alexnet_bf16_concurrent_full_size_sampled():
+    """The bench step's executor (BackwardFilter on a side stream) at full size."""
+    h = mu.Handle(0)
+    h.set_policy(mu.POLICY_POW2)
+    layers = network("alexnet")
+    net = ConvNet(h, layers, N, mu.MATH_BF16, device="cuda")
+    net.allocate(seed=4)
+    limit = 64 << 20
+    net.benchmark_all(limit)
+    net.plan_wr(limit)
+    net.iteration(concurrent=True)
+    torch.cuda.synchronize()
+    rng = np.random.default_rng(1)
+    for i, layer in enumerate(layers):
+        _check_layer(net, i, layer, rng)

@@ -708,6 +708,10 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
             while (A.km < 4 && 2 * (2 * A.km) * base <= 200 * 1024 && KB * 2 * A.km <= 256 &&
                    (qrow == 0 || KB * 2 * A.km <= (int)align_up((uint64_t)qrow, (uint64_t)KB)))
                 A.km *= 2;
+            // window operand (qrow > 0), BF16: 64-pixel k-blocks already make large boxes;
+            // km = 1 keeps 5 ring stages instead of 2 (ResNet conv1 WGRAD -6 %; TF32's
+            // 32-pixel blocks need km = 2)
+            if (qrow && elt == 2 && env_int("MUCU_WIN_KM1", 1)) A.km = 1;
             if (const int km = env_int("MUCU_KM", 0)) A.km = km;
         }
         size_stages(A);

@@ -693,7 +693,7 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
     // TMA-only operands (tma = true) also take 256-row tiles and stages of
     // km k-blocks: fewer, larger TMA transactions (the TMA issue rate, not
     // bytes, bounds these MN-major loads), as deep as two stages allow.
-    auto wgrad_tiling = [&](int step, bool tma, int qrow = 0) {
+    auto wgrad_tiling = [&](int step, bool tma, int qrow = 0, int km_max = 4) {
         A.mt = (tma && A.M > 128 && (A.M <= 256 || A.M % 256 == 0 || (qrow && A.M % 256 > 128)) &&
                 env_int("MUCU_MT2", 1)) ? 2 : 1;
         // 256-row tiles keep BN <= 128 so that two stages of two k-blocks fit
@@ -705,7 +705,7 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         A.km = 1;
         if (tma) {
             const int base = A.mt * 128 * 128 + A.b_bytes;
-            while (A.km < 4 && 2 * (2 * A.km) * base <= 200 * 1024 && KB * 2 * A.km <= 256 &&
+            while (A.km < km_max && 2 * (2 * A.km) * base <= 200 * 1024 && KB * 2 * A.km <= 256 &&
                    (qrow == 0 || KB * 2 * A.km <= (int)align_up((uint64_t)qrow, (uint64_t)KB)))
                 A.km *= 2;
             // window operand (qrow > 0), BF16: 64-pixel k-blocks already make large boxes;
@@ -1269,7 +1269,9 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
                 if (err) return err;
             }
             if (RSC < atom) return -1;
-            wgrad_tiling(16, true);
+            // dense (pointwise / explicit im2col) operands: single k-block stages keep a
+            // deeper ring (deep ResNet 1x1 WGRAD -3..6 % against km = 2)
+            wgrad_tiling(16, true, 0, env_int("MUCU_DENSE_KM", 1));
             if (!map_dy()) return -1;
             if (!map2(&L.tb, colp, RSC, (uint64_t)Mpix, kp, atom, KB * A.km, true)) return -1;
             map_mn_box(colp, RSC, (uint64_t)Mpix, kp, KB * A.km);

@@ -105,6 +105,15 @@ class ConvNet:
         """Seeded synthetic tensors on the device (values do not affect timing)."""
         from synthetic import torch_conv_inputs  # workload generator (no method arithmetic)
         self.tensors = []
+        # all filter gradients are views of one flat fp32 buffer, zeroed once per
+        # iteration (the framework's zero_grad); BackwardFilter then accumulates with
+        # beta = 1, so no per-layer beta = 0 pre-scale launch is needed
+        shapes = [T.shapes(d)[1] for d in self.descs]
+        sizes = [int(np.prod(s_)) for s_ in shapes]
+        offs = [0]
+        for n_ in sizes:
+            offs.append(offs[-1] + (n_ + 63) // 64 * 64)  # 256-B aligned views
+        self.dw_flat = torch.zeros(max(offs[-1], 1), dtype=torch.float32, device=self.device)
         for i, (l, d) in enumerate(zip(self.layers, self.descs)):
             x, w, dy = torch_conv_inputs(l, self.n, seed=1000 * seed + i, device=self.device, dtype=self.dtype,
                                          kind=kind)
@@ -113,7 +122,7 @@ class ConvNet:
                 x=x, w=w, dy=dy,
                 y=torch.empty(ys, dtype=self.dtype, device=self.device),
                 dx=torch.empty(xs, dtype=self.dtype, device=self.device),
-                dw=torch.zeros(ws_, dtype=torch.float32, device=self.device)))
+                dw=self.dw_flat[offs[i]:offs[i] + sizes[i]].view(ws_)))
 
     # ---------------------------------------------------------- planning --
     def benchmark_all(self, ws_limit: int, progress: Optional[Callable] = None, group=None):
@@ -239,8 +248,8 @@ class ConvNet:
             T.conv_forward(self.h, k.desc, k.plan, t["x"], t["w"], t["y"], workspace=ws)
         elif conv_type == L.BWD_DATA:
             T.conv_backward_data(self.h, k.desc, k.plan, t["dy"], t["w"], t["dx"], workspace=ws)
-        else:
-            T.conv_backward_filter(self.h, k.desc, k.plan, t["x"], t["dy"], t["dw"], workspace=ws)
+        else:  # dw was zeroed at the start of the backward pass (zero_grad): accumulate
+            T.conv_backward_filter(self.h, k.desc, k.plan, t["x"], t["dy"], t["dw"], beta=1.0, workspace=ws)
 
     def iteration(self, on_op: Optional[Callable] = None, grad_hook: Optional[Callable] = None,
                   skip_conv1_dgrad: bool = False, concurrent: bool = False):
@@ -260,6 +269,8 @@ class ConvNet:
                 order.append((i, L.BWD_DATA))
             order.append((i, L.BWD_FILTER))
         for i, t in order:
+            if (i, t) == order[len(self.layers)]:
+                self.dw_flat.zero_()  # zero_grad, once per iteration, before the first backward call
             if on_op:
                 on_op(i, t, "begin")
             self.run_kernel(i, t)
@@ -284,6 +295,7 @@ class ConvNet:
             hook(i, t, "end")
         for i in range(len(self.layers)):
             run(i, L.FWD)
+        self.dw_flat.zero_()  # zero_grad, once per iteration, before the first backward call
         for i in reversed(range(len(self.layers))):
             if i == len(self.layers) - 1:
                 hook(i, L.BWD_DATA, "first")  # stream-ordered setup before any backward call

@@ -32,8 +32,10 @@ SHAPES = {
     "7x7s2_c3": (2, 3, 23, 23, 64, 7, 7, 3, 2),
     "big_k": (1, 128, 6, 6, 256, 3, 3, 1, 1),
 }
+# per_atom_boxes: the one-box-per-atom TMA loads the multi-dimensional boxes replaced (§6.1)
+NO_BOXES = {"MUCU_B_BOX": "0", "MUCU_A_BOX": "0", "MUCU_WIN_BOX": "0", "MUCU_A_MERGE": "0"}
 ENVS = {"mt4": {"MUCU_FORCE_MT": "4"}, "mt2": {"MUCU_FORCE_MT": "2"}, "halo": {"MUCU_HALO": "1"},
-        "per_phase": {"MUCU_MERGE_PHASES": "0"}}
+        "per_phase": {"MUCU_MERGE_PHASES": "0"}, "per_atom_boxes": NO_BOXES}
 CASES = [(s, t, a) for s in SHAPES for t in (mu.FWD, mu.BWD_DATA)
          for a in (mu.IMPLICIT_GEMM, mu.IM2COL_GEMM)]
 
@@ -53,3 +55,20 @@ def test_forced_tiling_exact(case, math, env, monkeypatch):
         ref = torch.from_numpy(ref).to(torch.bfloat16).double().numpy()
     got, _ = run_gpu(d, conv_type, [(algo, shape[0])], x, w, dy)
     assert np.array_equal(got, ref)
+
+
+# BackwardFilter through the per-atom TMA loads and multi-k-block stages
+@pytest.mark.parametrize("env", ["per_atom_boxes", "km2"])
+@pytest.mark.parametrize("math", [mu.MATH_TF32, mu.MATH_BF16], ids=["tf32", "bf16"])
+@pytest.mark.parametrize("name", ["3x3s1_c64", "3x3s1_c128", "1x1s1", "1x1s2_c128", "7x7s2_c3", "big_k"])
+def test_wgrad_alternative_loads_exact(name, math, env, monkeypatch):
+    envs = NO_BOXES if env == "per_atom_boxes" else {"MUCU_DENSE_KM": "4", "MUCU_WIN_KM1": "0"}
+    for k, v in envs.items():
+        monkeypatch.setenv(k, v)
+    shape = SHAPES[name]
+    d = mu.desc(*shape, math)
+    x, w, dy = conv_inputs(*shape, seed=29, kind="int")
+    ref = oracle_ref(shape, mu.BWD_FILTER, x, w, dy)
+    for algo in (mu.IMPLICIT_GEMM, mu.IM2COL_GEMM):
+        got, _ = run_gpu(d, mu.BWD_FILTER, [(algo, shape[0])], x, w, dy)
+        assert np.array_equal(got, ref), (name, algo)

@@ -23,8 +23,11 @@ net = {"alexnet": alexnet, "resnet18": resnet18, "resnet-18": resnet18, "resnet5
        "resnet-50": resnet50}[cfg.replace(",", "")]()
 n = d["config"]["batch_per_gpu"]
 elt = 2 if d["dtype"] == "bf16" else 4
-peak = 1614e12 if d["dtype"] == "bf16" else (807e12 if d["dtype"] == "tf32" else 74e12)
-bw = 6.5e12
+_mp = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "MEASURED_PEAKS.json")
+_pk = json.load(open(_mp)) if os.path.exists(_mp) else {}
+_bf16 = _pk.get("bf16_tflops", 1614.0) * 1e12
+peak = _bf16 if d["dtype"] == "bf16" else (_bf16 / 2 if d["dtype"] == "tf32" else 74e12)
+bw = _pk.get("hbm_gbs", 6500.0) * 1e9
 rows = []
 for L in net:
     for t in ("FWD", "DGRAD", "WGRAD"):

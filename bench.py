@@ -4,6 +4,16 @@ algorithm at the same workspace (BASELINE.json metric), on B200.
     python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
                     [--config alexnet|resnet18|resnet50] [--math tf32|bf16|f32]
                     [--policy pow2|all|undivided] [--ws-mib 64] [--wd-mib T] [--batch 256]
+                    [--layers conv2] [--types fwd,dgrad,wgrad] [--global-batch G]
+
+BASELINE.json configs as bench lines:
+  cfg1  --config alexnet --layers conv2 --types fwd --batch 8 --math f32 --ws-mib 8 --policy all
+  cfg2  (default: TF32) / --math f32
+  cfg3  --config resnet18 --math bf16 --wd-mib 480
+  cfg4  --config resnet50 --math bf16 [--wd-mib 10176]
+  cfg5  --config resnet50 --math bf16 --global-batch 2048 --gpus N   (strong scaling, 2048/N per GPU)
+With --gpus N > 1 and no torchrun environment, bench.py re-launches itself
+under torch.distributed.run with N ranks (one per GPU, NCCL, 127.0.0.1).
 
 Default (N=1): BASELINE.json configs[1] -- AlexNet's 5 conv layers, forward +
 backward (15 kernels; --no-input-grad drops the first layer's BackwardData as
@@ -47,6 +57,10 @@ def parse():
     ap.add_argument("--ws-mib", type=float, default=64.0, help="WR per-kernel workspace limit (MiB)")
     ap.add_argument("--wd-mib", type=float, default=0.0, help="use WD with this total workspace (MiB)")
     ap.add_argument("--batch", type=int, default=256, help="mini-batch per GPU")
+    ap.add_argument("--global-batch", type=int, default=0,
+                    help="global mini-batch sharded over the ranks (strong scaling, cfg5); overrides --batch")
+    ap.add_argument("--layers", default="", help="comma-separated layer names to run (default: all conv layers)")
+    ap.add_argument("--types", default="fwd,dgrad,wgrad", help="conv operations per layer (fwd,dgrad,wgrad)")
     ap.add_argument("--no-input-grad", dest="input_grad", action="store_false",
                     help="skip the first layer's BackwardData (the data layer needs no gradient, as in "
                          "Caffe's `time` command, P:L198); the default times all 3 kernels per layer (SURVEY 8(d) cfg2)")
@@ -118,11 +132,42 @@ class ClockSampler:
                 "reasons": sorted(self.reasons), "samples": len(self.samples)}
 
 
+# ---------------------------------------------------------------- workload --
+TYPE_KEYS = {"fwd": 0, "dgrad": 1, "wgrad": 2}
+
+
+def select(args):
+    """(layers, kernels): the conv layers of --config (restricted by --layers) and
+    the (layer index, conv type) pairs one step runs, in iteration order."""
+    from synthetic import network
+    layers = network(args.config)
+    if args.layers:
+        names = [n.strip() for n in args.layers.split(",") if n.strip()]
+        missing = [n for n in names if n not in {l.name for l in layers}]
+        if missing:
+            raise SystemExit(f"unknown layer(s) {missing} in {args.config}")
+        layers = [l for l in layers if l.name in names]
+    types = sorted({TYPE_KEYS[t.strip()] for t in args.types.split(",") if t.strip()})
+    kernels = [(i, 0) for i in range(len(layers)) if 0 in types]
+    for i in reversed(range(len(layers))):
+        if 1 in types and not (i == 0 and not args.input_grad):
+            kernels.append((i, 1))
+        if 2 in types:
+            kernels.append((i, 2))
+    return layers, types, kernels
+
+
+def workload_name(args, layers, types, kernels):
+    tnames = "+".join(["fwd", "dgrad", "wgrad"][t] for t in types)
+    what = "fwd+bwd" if types == [0, 1, 2] else tnames
+    scope = "conv layers" if not args.layers else ",".join(l.name for l in layers)
+    return f"{args.config} {scope} {what} ({len(kernels)} kernel{'s' if len(kernels) != 1 else ''})"
+
+
 # --------------------------------------------------------------- oracle arm --
-def oracle_sample_time(layers, n_sample, threads=None, input_grad=True):
+def oracle_sample_time(layers, kernels, n_sample, threads=None):
     """Time the fp64 oracle (oracle/, unchanged) on n_sample images of every
-    kernel of the iteration (the first layer's BackwardData only if
-    input_grad); returns seconds."""
+    kernel of the step; returns seconds."""
     import oracle
     from synthetic import conv_inputs
     if threads:
@@ -130,35 +175,38 @@ def oracle_sample_time(layers, n_sample, threads=None, input_grad=True):
     oracle.build()
     tot = 0.0
     for i, l in enumerate(layers):
+        ts = [t for (j, t) in kernels if j == i]
+        if not ts:
+            continue
         x, w, dy = conv_inputs(n_sample, l.c, l.h, l.w, l.k, l.r, l.s, l.pad, l.stride, seed=i)
         x, w, dy = x.astype(np.float64), w.astype(np.float64), dy.astype(np.float64)
         t0 = time.perf_counter()
-        oracle.conv_forward(x, w, l.pad, l.stride)
-        if i > 0 or input_grad:
+        if 0 in ts:
+            oracle.conv_forward(x, w, l.pad, l.stride)
+        if 1 in ts:
             oracle.conv_backward_data(dy, w, l.h, l.w, l.pad, l.stride)
-        oracle.conv_backward_filter(x, dy, l.r, l.s, l.pad, l.stride)
+        if 2 in ts:
+            oracle.conv_backward_filter(x, dy, l.r, l.s, l.pad, l.stride)
         tot += time.perf_counter() - t0
     return tot
 
 
-def n_kernels(layers, input_grad):
-    return 3 * len(layers) - (0 if input_grad else 1)
-
-
-def cpu_baseline(layers, batch, n_sample, input_grad=True):
+def cpu_baseline(layers, kernels, batch, n_sample):
     cores = os.cpu_count()
-    secs = oracle_sample_time(layers, n_sample, input_grad=input_grad)
+    secs = oracle_sample_time(layers, kernels, n_sample)
     ms_per_iter = secs * 1e3 * batch / n_sample
+    exact = n_sample == batch
     return {"value": round(ms_per_iter, 3), "unit": "ms/iter", "cores": cores, "kind": "oracle",
-            "sample": f"{n_sample} image(s) per kernel, all {n_kernels(layers, input_grad)} timed kernels, fp64 7-loop oracle, "
-                      f"{secs:.2f} s measured, x{batch // n_sample} extrapolated to N={batch} (work is linear in N, P:L50)"}
+            "sample": f"{n_sample} image(s) per kernel, all {len(kernels)} timed kernels, fp64 7-loop oracle "
+                      f"(OpenMP, {cores} threads), {secs:.2f} s measured"
+                      + ("" if exact else f", x{batch // n_sample} extrapolated to N={batch} (work is linear in N, P:L50)")}
 
 
-def auto_sample(layers, batch, input_grad=True):
+def auto_sample(layers, kernels, batch):
     """Pick the oracle sample so one measurement takes ~10-20 s on this host
     (one probe image through every kernel, then scale)."""
-    per_img = oracle_sample_time(layers, 1, input_grad=input_grad)
-    n = int(max(1, min(batch, 20.0 / max(per_img, 1e-6))))  # powers of two below: ~10-20 s
+    per_img = oracle_sample_time(layers, kernels, 1)
+    n = int(max(1, min(batch, 20.0 / max(per_img, 1e-6))))
     while batch % n:
         n -= 1
     return n
@@ -168,29 +216,71 @@ def run_reference(args):
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return
-    from synthetic import network
-    layers = network(args.config)
-    n_sample = args.cpu_sample or auto_sample(layers, args.batch, args.input_grad)
+    layers, types, kernels = select(args)
+    world = int(os.environ.get("WORLD_SIZE", str(args.gpus)))
+    batch = args.global_batch // world if args.global_batch else args.batch
+    n_sample = args.cpu_sample or auto_sample(layers, kernels, batch)
     for _ in range(args.warmup):
         pass  # the oracle has no warm-up state; W is accepted for the contract
-    times = [oracle_sample_time(layers, n_sample, input_grad=args.input_grad) for _ in range(args.steps)]
-    ms = float(np.mean(times)) * 1e3 * args.batch / n_sample
+    times = [oracle_sample_time(layers, kernels, n_sample) for _ in range(args.steps)]
+    ms = float(np.mean(times)) * 1e3 * batch / n_sample
     cb = {"value": round(ms, 3), "unit": "ms/iter", "cores": os.cpu_count(), "kind": "oracle",
-          "sample": f"{n_sample} image(s) per kernel per step, x{args.batch // n_sample} extrapolated to N={args.batch}"}
-    line = {"impl": "reference", "metric": METRIC, "value": round(ms, 3), "unit": "ms/iter", "n_gpus": args.gpus,
+          "sample": f"{n_sample} image(s) per kernel per step, x{batch // n_sample} extrapolated to N={batch}"}
+    line = {"impl": "reference", "metric": METRIC, "value": round(ms, 3), "unit": "ms/iter", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms, 3), "higher_is_better": False,
-            "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-            "config": {"workload": f"{args.config} conv layers fwd+bwd ({n_kernels(layers, args.input_grad)} kernels)",
-                       "batch_per_gpu": args.batch, "math": "fp64 oracle",
+            "scaling": "strong" if args.global_batch else "weak", "vs_baseline": None, "dtype": "f64",
+            "data": "synthetic",
+            "config": {"workload": workload_name(args, layers, types, kernels),
+                       "batch_per_gpu": batch, "math": "fp64 oracle",
                        "first_layer_backward_data": bool(args.input_grad)},
             "cpu_baseline": cb,
             "e2e": {"value": round(ms, 3), "unit": "ms/iter", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
 
+def respawn(args):
+    """--gpus N > 1 outside torchrun: re-launch this script under
+    torch.distributed.run with N ranks (one per GPU) and return its exit code."""
+    import socket
+    import subprocess
+    with socket.socket() as sk:
+        sk.bind(("127.0.0.1", 0))
+        port = sk.getsockname()[1]
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__)] + sys.argv[1:]
+    return subprocess.call(cmd)
+
+
+def measure_tf32_peak(torch, dev):
+    """Dense TF32 tensor-core peak on this GPU (cuBLAS fp32 matmul with TF32
+    allowed, 8192^3, best of 10, CUDA events): the TF32 roofline denominator."""
+    n = 8192
+    a = torch.randn(n, n, device=dev)
+    b = torch.randn(n, n, device=dev)
+    prev = torch.backends.cuda.matmul.allow_tf32
+    torch.backends.cuda.matmul.allow_tf32 = True
+    try:
+        for _ in range(3):
+            torch.matmul(a, b)
+        best = 1e30
+        for _ in range(10):
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
+            torch.matmul(a, b)
+            e1.record()
+            e1.synchronize()
+            best = min(best, e0.elapsed_time(e1))
+    finally:
+        torch.backends.cuda.matmul.allow_tf32 = prev
+    del a, b
+    return 2.0 * n ** 3 / (best * 1e-3) / 1e12
+
+
 # ------------------------------------------------------------------ our arm --
 def main():
     args = parse()
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        sys.exit(respawn(args))
     if args.impl == "reference":
         return run_reference(args)
 
@@ -199,8 +289,7 @@ def main():
 
     import paper_conf_cluster_oyamabhm18_b200 as mu
     from paper_conf_cluster_oyamabhm18_b200.distributed import GradAllreduce, init_from_env, max_over_ranks
-    from paper_conf_cluster_oyamabhm18_b200.network import ConvNet, algorithmic_bytes, algorithmic_flops, layer_flops
-    from synthetic import network
+    from paper_conf_cluster_oyamabhm18_b200.network import ConvNet, algorithmic_bytes, algorithmic_flops
 
     distributed = init_from_env("nccl")
     rank = dist.get_rank() if distributed else 0
@@ -210,13 +299,18 @@ def main():
     dev = torch.device("cuda", local)
     peaks, peaks_src = load_peaks()
 
-    layers = network(args.config)
+    layers, types, kernels = select(args)
+    if args.global_batch:
+        if args.global_batch % world:
+            raise SystemExit(f"--global-batch {args.global_batch} not divisible by {world} ranks")
+        args.batch = args.global_batch // world
     math = MATHS[args.math]
     h = mu.Handle(local)
     h.set_policy({"pow2": mu.POLICY_POW2, "all": mu.POLICY_ALL, "undivided": mu.POLICY_UNDIVIDED}[args.policy])
     ws_limit = int(args.ws_mib * 2 ** 20)
-    net = ConvNet(h, layers, args.batch, math, device=dev)
+    net = ConvNet(h, layers, args.batch, math, device=dev, types=types)
     net.allocate(seed=rank)
+    skip_c1 = not args.input_grad
 
     # ---- planning: benchmark pass + DP / ILP ----
     t0 = time.perf_counter()
@@ -237,7 +331,7 @@ def main():
     def timed(nsteps, nwarm, record_ops=False):
         ops = {}
         for _ in range(nwarm):
-            net.iteration(grad_hook=grad_ar, skip_conv1_dgrad=not args.input_grad, concurrent=conc and not record_ops)
+            net.iteration(grad_hook=grad_ar, skip_conv1_dgrad=skip_c1, concurrent=conc and not record_ops)
             grad_ar.wait()
         torch.cuda.synchronize()
         if distributed:
@@ -257,7 +351,7 @@ def main():
             s0 = torch.cuda.Event(enable_timing=True)
             s1 = torch.cuda.Event(enable_timing=True)
             s0.record(stream)
-            net.iteration(on_op=on_op, grad_hook=grad_ar, skip_conv1_dgrad=not args.input_grad,
+            net.iteration(on_op=on_op, grad_hook=grad_ar, skip_conv1_dgrad=skip_c1,
                           concurrent=conc and not record_ops)
             grad_ar.wait()
             s1.record(stream)
@@ -276,13 +370,14 @@ def main():
             dist.barrier()
         return float(np.mean(step_ms)), ops, launches
 
-    results = {}
-    # Baseline: best undivided algorithm at the same per-kernel limit.
+    # Baseline: best undivided algorithm at the same per-kernel limit,
+    # timed as a whole step and per kernel; both max-reduced over the ranks.
+    und_ms, und_ops = None, {}
     if args.wd_mib <= 0:
         net.plan_undivided(ws_limit)
         und_ms, _, _ = timed(max(3, args.steps // 2), args.warmup)
-        results["undivided"] = und_ms
-        und_plans = {k: list(v.plan) for k, v in net.kernels.items()}
+        und_ms = max_over_ranks(und_ms)
+        _, und_ops, _ = timed(3, 1, record_ops=True)
     if args.wd_mib > 0:
         net.plan_wd(int(args.wd_mib * 2 ** 20))
     elif args.policy == "undivided":
@@ -300,26 +395,27 @@ def main():
         return
     # The step is timed without per-op events: an event record between two calls
     # serialises them (no programmatic-launch overlap) and cost ~9 % of the
-    # ResNet-50 step (tools/graph_probe.py).  Per-op times come from a second,
-    # separately timed pass with events around every call.
+    # ResNet-50 step.  Per-op times come from a second, separately timed pass
+    # with events around every call.
     with ClockSampler(local) as clk:
         ms, _, launches = timed(args.steps, args.warmup)
     ms_max = max_over_ranks(ms)
     ms_ops, ops, _ = timed(max(3, args.steps // 2), 1, record_ops=True)
 
     # ---- end to end through the public API with host buffers ----
-    x_host = net.tensors[0]["x"].detach().cpu().pin_memory()
-    dy_host = net.tensors[-1]["dy"].detach().cpu().pin_memory()
-    dw_host = [torch.empty_like(t["dw"], device="cpu").pin_memory() for t in net.tensors]
-
-    # The input pipeline of a training loop: step k+1's x and dy are uploaded from
-    # pinned host memory (double-buffered, on an upload stream) while step k
-    # computes, and each layer's dW is read back to the host (download stream)
-    # as soon as its BackwardFilter is done.  Every timed step performs its own
+    # The input pipeline of a training loop: step k+1's inputs (x of the first
+    # layer, dy of the last) are uploaded from pinned host memory (double-buffered,
+    # upload stream) while step k computes; each layer's dW is read back to the
+    # host (download stream) as soon as its BackwardFilter is done (forward-only
+    # workloads read back the last layer's y).  Every timed step performs its own
     # h2d_bytes / d2h_bytes of copies; the first step's upload is not hidden.
+    has_bwd = any(t != 0 for t in types)
+    up_names = [(0, "x")] + ([(len(layers) - 1, "dy")] if has_bwd else [])
+    hosts = {key: net.tensors[key[0]][key[1]].detach().cpu().pin_memory() for key in up_names}
+    bufs = {key: [net.tensors[key[0]][key[1]], torch.empty_like(net.tensors[key[0]][key[1]])] for key in up_names}
+    dw_host = [torch.empty_like(t["dw"], device="cpu").pin_memory() for t in net.tensors] if 2 in types else []
+    y_host = None if has_bwd else torch.empty_like(net.tensors[-1]["y"], device="cpu").pin_memory()
     up_stream, down_stream = torch.cuda.Stream(), torch.cuda.Stream()
-    x_bufs = [net.tensors[0]["x"], torch.empty_like(net.tensors[0]["x"])]
-    dy_bufs = [net.tensors[-1]["dy"], torch.empty_like(net.tensors[-1]["dy"])]
     ready = [torch.cuda.Event(), torch.cuda.Event()]
     done = [torch.cuda.Event(), torch.cuda.Event()]
 
@@ -328,8 +424,8 @@ def main():
         if k >= 2:
             up_stream.wait_event(done[j])  # step k-2 has finished with these buffers
         with torch.cuda.stream(up_stream):
-            x_bufs[j].copy_(x_host, non_blocking=True)
-            dy_bufs[j].copy_(dy_host, non_blocking=True)
+            for key in up_names:
+                bufs[key][j].copy_(hosts[key], non_blocking=True)
             ready[j].record(up_stream)
 
     def e2e_op(i, t, what):
@@ -347,15 +443,19 @@ def main():
                 upload(k + 1)  # prefetch the next step's inputs while this one computes
             j = k % 2
             stream.wait_event(ready[j])
-            net.tensors[0]["x"], net.tensors[-1]["dy"] = x_bufs[j], dy_bufs[j]
-            net.iteration(on_op=e2e_op, grad_hook=grad_ar, skip_conv1_dgrad=not args.input_grad,
-                          concurrent=conc)
+            for key in up_names:
+                net.tensors[key[0]][key[1]] = bufs[key][j]
+            net.iteration(on_op=e2e_op, grad_hook=grad_ar, skip_conv1_dgrad=skip_c1, concurrent=conc)
             grad_ar.wait()
-            if distributed:
+            if distributed and dw_host:
                 down_stream.wait_stream(stream)
                 with torch.cuda.stream(down_stream):
                     for t, hbuf in zip(net.tensors, dw_host):
                         hbuf.copy_(t["dw"], non_blocking=True)
+            if y_host is not None:
+                down_stream.wait_stream(stream)
+                with torch.cuda.stream(down_stream):
+                    y_host.copy_(net.tensors[-1]["y"], non_blocking=True)
             stream.wait_stream(down_stream)  # the step's results are on the host
             done[j].record(stream)
         s1.record(stream)
@@ -367,29 +467,34 @@ def main():
     if distributed:
         dist.barrier()
     e2e_ms = e2e_run(max(5, args.steps))
-    net.tensors[0]["x"], net.tensors[-1]["dy"] = x_bufs[0], dy_bufs[0]
+    for key in up_names:
+        net.tensors[key[0]][key[1]] = bufs[key][0]
     e2e_ms = max_over_ranks(e2e_ms)
-    h2d_bytes = x_host.numel() * x_host.element_size() + dy_host.numel() * dy_host.element_size()
-    d2h_bytes = sum(b.numel() * 4 for b in dw_host)
+    h2d_bytes = sum(t.numel() * t.element_size() for t in hosts.values())
+    d2h_bytes = sum(b.numel() * 4 for b in dw_host) + (y_host.numel() * y_host.element_size() if y_host is not None else 0)
 
     # ---- dominant kernel roofline ----
     op_ms = {k: float(np.median(v)) for k, v in ops.items()}  # median: robust to a one-step hiccup
+    op_ms_max = {k: max_over_ranks(v) for k, v in sorted(op_ms.items())}
+    und_op_ms = {k: max_over_ranks(float(np.median(v))) for k, v in sorted(und_ops.items())}
     dom = max(op_ms, key=op_ms.get)
     li, lt = dom
     kern = net.kernels[dom]
     bf16_peak = peaks.get("bf16_tflops", 1590.0)
     hbm_peak = peaks.get("hbm_gbs", 6650.0)
     elt = 2 if math == mu.MATH_BF16 else 4
+    tf32_measured = None
     if math == mu.MATH_BF16:
         tpeak, tbound = bf16_peak, "tensor"
-        peak_note = f"bf16 dense {peaks_src} (burst)"
+        peak_note = f"bf16 dense {peaks_src} (burst, MEASURED_PEAKS.json)"
     elif math == mu.MATH_TF32:
-        tpeak, tbound = bf16_peak * 0.5, "tensor"
-        peak_note = f"tf32 = {peaks_src} bf16 burst x nominal tf32/bf16 ratio 1.125/2.25"
+        tf32_measured = measure_tf32_peak(torch, dev)
+        tpeak, tbound = tf32_measured, "tensor"
+        peak_note = "tf32 dense measured in this run: cuBLAS fp32 matmul 8192^3 with TF32 allowed, best of 10"
     else:
         sm_mhz = peaks.get("sm_max_mhz", 1965.0)
         tpeak, tbound = 148 * 128 * 2 * sm_mhz * 1e6 / 1e12, "alu"
-        peak_note = "fp32 FFMA: 148 SM x 128 lanes x 2 flop x max SM clock"
+        peak_note = "fp32 FFMA: 148 SM x 128 lanes x 2 flop x max SM clock (DESIGN.md)"
 
     def floor_ms(i, t, plan):
         """Roofline floor of one op: max(F / compute peak, B / HBM peak)."""
@@ -413,34 +518,40 @@ def main():
     if os.path.exists(tp):
         try:
             tj = json.load(open(tp))
-            traffic = tj.get(f"{args.config}/{args.math}/{layers[li].name}/{mu.TYPE_NAMES[lt]}")
+            traffic = tj.get(f"{args.config}/{args.math}/{layers[li].name}/{mu.TYPE_NAMES[lt]}/b{args.batch}")
         except Exception:
             traffic = None
 
-    conv_flops = net.flops_per_iteration(skip_conv1_dgrad=not args.input_grad)
+    conv_flops = net.flops_per_iteration(skip_conv1_dgrad=skip_c1)
     total_ws = net.total_workspace()
+    kname = lambda i, t: f"{layers[i].name}/{mu.TYPE_NAMES[t]}"  # noqa: E731
     if rank == 0:
         cb = None
         if not args.no_cpu_baseline and world == 1:
-            n_sample = args.cpu_sample or auto_sample(layers, args.batch, args.input_grad)
-            cb = cpu_baseline(layers, args.batch, n_sample, args.input_grad)
+            n_sample = args.cpu_sample or auto_sample(layers, kernels, args.batch)
+            cb = cpu_baseline(layers, kernels, args.batch, n_sample)
         line = {
             "metric": METRIC, "value": round(ms_max, 4), "unit": "ms/iter", "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": round(ms_max, 4), "higher_is_better": False,
-            "scaling": "weak", "vs_baseline": None, "dtype": args.math, "data": "synthetic",
-            "config": {"workload": f"{args.config} conv layers fwd+bwd ({n_kernels(layers, args.input_grad)} kernels)",
+            "scaling": "strong" if args.global_batch else "weak", "vs_baseline": None, "dtype": args.math,
+            "data": "synthetic",
+            "config": {"workload": workload_name(args, layers, types, kernels),
                        "batch_per_gpu": args.batch, "global_batch": args.batch * world,
                        "policy": ("WD" if args.wd_mib > 0 else "WR"),
                        "ws_limit_mib": (args.wd_mib if args.wd_mib > 0 else args.ws_mib),
                        "batch_size_policy": args.policy, "parallelism": f"dp{world}",
                        "l2": "512 MiB buffer overwritten before every timed step",
                        "first_layer_backward_data": bool(args.input_grad),
-                       "backward_streams": 2 if args.concurrent_wgrad else 1},
+                       "backward_streams": 2 if args.concurrent_wgrad else 1,
+                       "wgrad_reduction": "ordered split-K (deterministic)"},
             "images_per_s": round(args.batch * world / (ms_max * 1e-3), 1),
-            "conv_tflops_direct": round(conv_flops / (ms_max * 1e-3) / 1e12, 2),
+            "conv_tflops_direct": round(conv_flops * world / (ms_max * 1e-3) / 1e12, 2),
             "ms_per_step_with_op_events": round(ms_ops, 4),
-            "undivided_ms_per_step": round(results["undivided"], 4) if "undivided" in results else None,
-            "speedup_vs_undivided": round(results["undivided"] / ms, 4) if "undivided" in results else None,
+            "undivided_ms_per_step": round(und_ms, 4) if und_ms is not None else None,
+            "speedup_vs_undivided": round(und_ms / ms_max, 4) if und_ms is not None else None,
+            "speedup_by_kernel": {kname(i, t): round(und_op_ms[(i, t)] / v, 3)
+                                  for (i, t), v in op_ms_max.items() if (i, t) in und_op_ms},
+            "undivided_per_kernel_ms": {kname(i, t): round(v, 4) for (i, t), v in und_op_ms.items()},
             "workspace_total_mib": round(total_ws / 2 ** 20, 2),
             "plan_time_s": round(bench_s, 2),
             "roofline": {"bound": bound, "achieved": round(achieved, 2), "peak": round(peak, 1), "unit": punit,
@@ -450,14 +561,15 @@ def main():
                          "algorithmic_flops": alg_flops, "algorithmic_bytes": alg_bytes,
                          "avg_ms": round(op_ms[dom], 4),
                          "share_of_step": round(op_ms[dom] / ms_ops, 4), "peak_source": peak_note,
-                         "step_floor_ms": round(step_floor, 4), "step_frac": round(step_floor / ms, 4)},
+                         "tf32_peak_measured_tflops": round(tf32_measured, 1) if tf32_measured else None,
+                         "step_floor_ms": round(step_floor, 4), "step_frac": round(step_floor / ms_max, 4)},
             "cpu_baseline": cb,
             "e2e": {"value": round(e2e_ms, 4), "unit": "ms/iter", "h2d_bytes_per_step": int(h2d_bytes),
                     "d2h_bytes_per_step": int(d2h_bytes)},
             "gpu_launches": int(launches),
             "clocks": clk.result(),
-            "per_kernel_ms": {f"{layers[i].name}/{mu.TYPE_NAMES[t]}": round(v, 4) for (i, t), v in sorted(op_ms.items())},
-            "plans": {f"{layers[i].name}/{mu.TYPE_NAMES[t]}": [(mu.ALGO_NAMES[a], b) for a, b in k.plan]
+            "per_kernel_ms": {kname(i, t): round(v, 4) for (i, t), v in op_ms_max.items()},
+            "plans": {kname(i, t): [(mu.ALGO_NAMES[a], b) for a, b in k.plan]
                       for (i, t), k in sorted(net.kernels.items())},
         }
         if args.json_out:

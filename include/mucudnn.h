@@ -19,17 +19,17 @@
  *
  * Conventions (all functions):
  *   - Every function returns mucu_status_t; none throws, aborts or prints.
- *     On error, mucu_last_error() returns a thread-local detail string.
+ *     On error, mucu_last_error(handle) returns a thread-local detail string.
  *   - Tensors: activations NHWC (x: [N,H,W,C], y/dy: [N,P,Q,K], dx: [N,H,W,C]),
  *     filters KRSC (w: [K,R,S,C]), all densely packed.  Element type by math
  *     mode: MUCU_MATH_F32 / MUCU_MATH_TF32 -> float32; MUCU_MATH_BF16 ->
  *     bfloat16.  The filter gradient dw is ALWAYS float32 [K,R,S,C].
  *     P = (H + 2 pad - R)/stride + 1, Q likewise (reading G1/G3).
  *   - Device memory (tensors, workspace, benchmark scratch) is owned by the
- *     caller (PyTorch allocator).  Host objects (handle, network) are created
- *     and destroyed by the library.  The handle additionally owns one small
- *     device buffer (split-K ordering semaphores, 256 KiB) allocated in
- *     mucu_create.
+ *     caller (PyTorch allocator); the library never calls cudaMalloc.  Host
+ *     objects (handle, network) are created and destroyed by the library.
+ *     BackwardFilter's split-K ordering counters live in a static device array
+ *     of the library module (2 MiB, no allocation call).
  *   - GPU work is asynchronous on the caller's `cuda_stream` (a cudaStream_t
  *     passed as void*; NULL = legacy default stream), except
  *     mucu_benchmark / mucu_plan_layer / mucu_network_plan which synchronise
@@ -98,7 +98,9 @@ typedef struct mucu_network* mucu_network_t; /* library-owned WD kernel list (P:
 
 /* ---------------------------------------------------------------- misc ---- */
 const char* mucu_status_string(mucu_status_t status);   /* host; static string */
-const char* mucu_last_error(void);                      /* host; thread-local detail */
+/* host; detail of the calling thread's last error (thread-local; `handle` may
+ * be NULL, e.g. after a failed pure host function or mucu_create). */
+const char* mucu_last_error(mucu_handle_t handle);
 int32_t mucu_version(void);                             /* host */
 /* Process-wide number of CUDA kernels the library has launched so far (host;
  * monotone, for launch accounting in benchmarks). */

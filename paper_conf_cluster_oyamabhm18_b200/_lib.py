@@ -60,7 +60,7 @@ def _load():
     D, MC = P(ConvDesc), P(MicroConfig)
     sig = {
         "mucu_status_string": (ctypes.c_char_p, [ctypes.c_int]),
-        "mucu_last_error": (ctypes.c_char_p, []),
+        "mucu_last_error": (ctypes.c_char_p, [vp]),
         "mucu_version": (i32, []),
         "mucu_launch_count": (u64, []),
         "mucu_create": (ctypes.c_int, [P(vp), ctypes.c_int]),
@@ -97,7 +97,7 @@ lib = _load()
 
 def _check(status: int):
     if status != OK:
-        raise MucuError(status, lib.mucu_last_error().decode())
+        raise MucuError(status, lib.mucu_last_error(None).decode())
 
 
 def _i64(a):

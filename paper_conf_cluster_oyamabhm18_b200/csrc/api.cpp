@@ -69,8 +69,7 @@ S2d s2d_geom(const Geom& g, int type) {
         // dx super-pixels of f = st*u rows/cols; dx row f*i + a' - pad takes dy rows
         // p = u*i + u-1-d (d < Dr = ceil(R/st) - 1 + u) through filter row
         // r = st*d + a' - st*(u-1).  u = 2 when f*f*C stays <= 256 GEMM columns.
-        static const char* e = getenv("MUCU_S2D_UD");
-        z.u = e ? atoi(e) : 2;
+        z.u = 2;
         while (z.u > 1 && st * z.u * st * z.u * g.c > 256) --z.u;
         z.f = st * z.u;
         z.Dr = (g.r - 1) / st + z.u;
@@ -83,10 +82,6 @@ S2d s2d_geom(const Geom& g, int type) {
     }
     // FWD / WGRAD: output super-pixels of u x u (u = 2 for FWD: N = 4K columns)
     z.u = type == MUCU_FWD ? 2 : 1;
-    if (type == MUCU_FWD) {
-        static const char* e = getenv("MUCU_S2D_U");  // experiments: output super-pixel factor
-        if (e) z.u = atoi(e);
-    }
     z.f = st * z.u;
     // output row u*i' + uu reads input rows f*(i' + d) + a - pad with st*uu + r = f*d + a
     z.Dr = (st * (z.u - 1) + g.r - 1) / z.f + 1;
@@ -109,9 +104,8 @@ bool s2d_tc(const Geom& g, int type) {
 }
 
 bool win_tc(const Geom& g, int type) {
-    static const int enabled = getenv("MUCU_WIN") ? atoi(getenv("MUCU_WIN")) : 1;
     const int elt = elt_size(g.math);
-    return enabled && type == MUCU_BWD_FILTER && small_c_tc(g) && g.stride >= 2 && g.c <= 4 &&
+    return type == MUCU_BWD_FILTER && small_c_tc(g) && g.stride >= 2 && g.c <= 4 &&
            (g.stride * 4 * elt) % 16 == 0;
 }
 
@@ -252,9 +246,9 @@ struct Handle {
     int num_sms = 148;
     int policy = MUCU_POLICY_POW2;
     int warmup = 2, reps = 5;
-    int32_t* sem = nullptr;
-    int32_t sem_cap = 0;
     std::map<std::string, std::pair<std::vector<int64_t>, std::vector<uint64_t>>> cache;
+    // (descriptor, type, algo, b) -> tensor-core path available (executor pre-validation)
+    std::map<std::string, bool> tc_ok;
 };
 
 static bool tc_math(int math) { return math == MUCU_MATH_TF32 || math == MUCU_MATH_BF16; }
@@ -269,10 +263,17 @@ mucu_status_t run_micro(Handle* hd, const Geom& g, int type, int algo, int32_t b
     if (L.total > ws_bytes) return set_error(MUCU_ERR_INSUFFICIENT_WORKSPACE, "workspace %llu < %llu", (unsigned long long)ws_bytes, (unsigned long long)L.total);
     char* wsb = (char*)ws;
     const bool tc = tc_math(g.math);
-    const SemBuf sem{hd->sem, hd->sem_cap};
+    // The b-independent workspace prefix (padded filter / Winograd U / space-to-depth
+    // filter) computed by an earlier micro-config of this call stays valid only while
+    // the same algorithm runs: any other algorithm may write its own segments over it.
+    if (ctx->last_algo != algo) {
+        ctx->fixed_kind = 0;
+        ctx->fixed_src = nullptr;
+        ctx->last_algo = algo;
+    }
     int e = 0;
     if (tc) {
-        e = tc_run_micro(g, type, algo, b, alpha, in0, in1, beta, out, wsb, L, sem, hd->num_sms, st, ctx);
+        e = tc_run_micro(g, type, algo, b, alpha, in0, in1, beta, out, wsb, L, hd->num_sms, st, ctx);
         if (e == -1) return set_error(MUCU_ERR_UNSUPPORTED, "tensor-core path not available for this configuration");
         return cuda_error(e, "tc kernel");
     }
@@ -342,14 +343,14 @@ mucu_status_t run_micro(Handle* hd, const Geom& g, int type, int algo, int32_t b
             if (!e) e = simt_gemm_tt(g.k, g.c, Tp, V, D, Mx, Tp, st);  // F32: Cp = C, Kp = K (mult. of 32 or padded)
             if (!e) e = launch_wgw_output(g, alpha, Mx, beta, fo, st);
         } else if (algo == MUCU_ALGO_IMPLICIT_GEMM) {
-            e = simt_wgrad(g, b, alpha, f1, f0, false, 0, beta, fo, sem, hd->num_sms, st);
+            e = simt_wgrad(g, b, alpha, f1, f0, false, 0, beta, fo, hd->num_sms, st);
         } else {
             if (is_pointwise(g)) {
-                e = simt_wgrad(g, b, alpha, f1, f0, true, g.c, beta, fo, sem, hd->num_sms, st);
+                e = simt_wgrad(g, b, alpha, f1, f0, true, g.c, beta, fo, hd->num_sms, st);
             } else {
                 float* col = (float*)(wsb + L.a_off);
                 e = launch_im2col(g, b, f0, col, L.kpitch, st);
-                if (!e) e = simt_wgrad(g, b, alpha, f1, col, true, L.kpitch, beta, fo, sem, hd->num_sms, st);
+                if (!e) e = simt_wgrad(g, b, alpha, f1, col, true, L.kpitch, beta, fo, hd->num_sms, st);
             }
         }
     }
@@ -390,7 +391,7 @@ extern "C" const char* mucu_status_string(mucu_status_t s) {
     return "MUCU_ERR_UNKNOWN";
 }
 
-extern "C" const char* mucu_last_error(void) { return g_err; }
+extern "C" const char* mucu_last_error(mucu_handle_t) { return g_err; }
 extern "C" int32_t mucu_version(void) { return MUCU_VERSION; }
 extern "C" uint64_t mucu_launch_count(void) { return g_launches.load(std::memory_order_relaxed); }
 
@@ -415,17 +416,12 @@ extern "C" mucu_status_t mucu_create(mucu_handle_t* out, int device) {
     h->policy = policy_from_env(MUCU_POLICY_POW2);
     if (const char* w = getenv("MUCU_BENCH_WARMUP")) h->warmup = std::max(0, atoi(w));
     if (const char* r = getenv("MUCU_BENCH_REPS")) h->reps = std::max(1, atoi(r));
-    h->sem_cap = 1 << 16;
-    e = (int)cudaMalloc((void**)&h->sem, sizeof(int32_t) * h->sem_cap);
-    if (!e) e = (int)cudaMemset(h->sem, 0, sizeof(int32_t) * h->sem_cap);
-    if (e) { delete h; return cuda_error(e, "semaphore buffer"); }
     *out = h;
     return MUCU_OK;
 }
 
 extern "C" mucu_status_t mucu_destroy(mucu_handle_t h) {
     if (!h) return MUCU_OK;
-    if (h->sem) cudaFree(h->sem);
     delete h;
     return MUCU_OK;
 }
@@ -495,17 +491,51 @@ static mucu_status_t execute(mucu_handle_t h, const mucu_conv_desc_t* d, int typ
     const uint64_t in_sample = (uint64_t)g.h * g.w * g.c * elt;   // x / dx per sample
     const uint64_t out_sample = (uint64_t)g.p * g.q * g.k * elt;  // y / dy per sample
     cudaStream_t st = (cudaStream_t)stream;
+    auto part_ptrs = [&](int32_t i, int64_t done, const char*& p0, const char*& p1, char*& po, float& bta) {
+        p0 = (const char*)in0; p1 = (const char*)in1; po = (char*)out; bta = beta;
+        if (type == MUCU_FWD) { p0 += done * in_sample; po += done * out_sample; }
+        else if (type == MUCU_BWD_DATA) { p0 += done * out_sample; po += done * in_sample; }
+        else { p0 += done * in_sample; p1 += done * out_sample; if (i > 0) bta = 1.f; }  // P:L58 output scale
+    };
+    // Tensor-core eligibility of every part before the first launch (a dry run of
+    // the dispatch: tilings, shared-memory budget, tensor-map encodings), cached per
+    // (descriptor, type, algorithm, b) -- a failure mid-plan would leave y / dx / dw
+    // partially updated.
+    if (tc_math(g.math)) {
+        int64_t done = 0;
+        for (int32_t i = 0; i < count; ++i) {
+            char key[160];
+            snprintf(key, sizeof(key), "%d,%d,%d,%d,%d,%d,%d,%d,%d,%d|%d|%d|%d", d->n, d->c, d->h, d->w, d->k, d->r,
+                     d->s, d->pad, d->stride, d->math, type, plan[i].algo, plan[i].micro_n);
+            auto it = h->tc_ok.find(key);
+            bool ok;
+            if (it != h->tc_ok.end()) {
+                ok = it->second;
+            } else {
+                const char *p0, *p1;
+                char* po;
+                float bta;
+                part_ptrs(i, done, p0, p1, po, bta);
+                CallCtx dry;
+                dry.dry = true;
+                ok = run_micro(h, g, type, plan[i].algo, plan[i].micro_n, alpha, p0, p1, bta, po, ws, ws_bytes, st,
+                               &dry) == MUCU_OK;
+                h->tc_ok[key] = ok;
+            }
+            if (!ok)
+                return set_error(MUCU_ERR_UNSUPPORTED, "plan part %d (algo %d, b = %d): no tensor-core kernel for this "
+                                 "configuration", i, plan[i].algo, plan[i].micro_n);
+            done += plan[i].micro_n;
+        }
+    }
     CallCtx ctx;
     int64_t done = 0;
     for (int32_t i = 0; i < count; ++i) {
         const int32_t b = plan[i].micro_n;
-        const char* p0 = (const char*)in0;
-        const char* p1 = (const char*)in1;
-        char* po = (char*)out;
-        float bta = beta;
-        if (type == MUCU_FWD) { p0 += done * in_sample; po += done * out_sample; }
-        else if (type == MUCU_BWD_DATA) { p0 += done * out_sample; po += done * in_sample; }
-        else { p0 += done * in_sample; p1 += done * out_sample; if (i > 0) bta = 1.f; }  // P:L58 output scale
+        const char *p0, *p1;
+        char* po;
+        float bta;
+        part_ptrs(i, done, p0, p1, po, bta);
         s = run_micro(h, g, type, plan[i].algo, b, alpha, p0, p1, bta, po, ws, ws_bytes, st, &ctx);
         if (s) return s;
         done += b;
@@ -623,9 +653,18 @@ extern "C" mucu_status_t mucu_benchmark(mucu_handle_t h, const mucu_conv_desc_t*
                 return run_micro(h, g, type, a, b, 1.f, base + S.in0, base + S.in1, 0.f, base + S.out, base + S.ws,
                                  S.total - S.ws, st, &ctx);
             };
+            // a dry run first: a configuration without a tensor-core kernel is skipped
+            // (not benchmarked) whatever the warm-up count
+            if (tc_math(g.math)) {
+                CallCtx dry;
+                dry.dry = true;
+                if (run_micro(h, g, type, a, b, 1.f, base + S.in0, base + S.in1, 0.f, base + S.out, base + S.ws,
+                              S.total - S.ws, st, &dry) == MUCU_ERR_UNSUPPORTED)
+                    continue;
+            }
             mucu_status_t r = MUCU_OK;
             for (int i = 0; i < h->warmup && r == MUCU_OK; ++i) r = launch();
-            if (r == MUCU_ERR_UNSUPPORTED) continue;  // e.g. math mode without this kernel
+            if (r == MUCU_ERR_UNSUPPORTED) continue;
             if (r) { status = r; break; }
             samples.clear();
             for (int i = 0; i < h->reps; ++i) {
@@ -638,6 +677,7 @@ extern "C" mucu_status_t mucu_benchmark(mucu_handle_t h, const mucu_conv_desc_t*
                 cudaEventElapsedTime(&ms, e0, e1);
                 samples.push_back(ms);
             }
+            if (r == MUCU_ERR_UNSUPPORTED) continue;
             if (r) { status = r; break; }
             std::sort(samples.begin(), samples.end());
             float med = samples[samples.size() / 2];

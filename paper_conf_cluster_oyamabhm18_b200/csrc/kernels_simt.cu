@@ -226,14 +226,15 @@ __global__ void __launch_bounds__(kThreads) simt_gemm_kernel(AV a, BV b, EPI epi
 }
 
 // WGRAD: dw[K][RSC] (+)= alpha * sum over the split's pixel range.  Splits of
-// one tile are combined in split order: split s waits until sem[tile] == s,
-// adds its partial (split 0 applies beta), publishes, and hands the turn to
-// s + 1 (the last split resets the counter to 0).  blockIdx.z = split, so all
-// CTAs of split s are dispatched before any of split s + 1 (no deadlock).
+// one tile are combined in split order (turns.cu): split s waits until the
+// tile's counter holds tag(epoch, s-1), adds its partial (split 0 applies
+// beta) and publishes tag(epoch, s).  blockIdx.z = split, so all CTAs of split
+// s are dispatched before any of split s + 1 (no deadlock).
 template <int BM, int BN, class AV, class BV>
 __global__ void __launch_bounds__(kThreads) simt_wgrad_kernel(AV a, BV b, float* dw, int64_t rows, int64_t cols,
                                                               int64_t Kd, int64_t k_per_split, float alpha,
-                                                              float beta, int32_t* sem) {
+                                                              float beta, unsigned long long* turns,
+                                                              unsigned long long epoch) {
     constexpr int TM = BM / 16, TN = BN / 16;
     const int64_t m0 = (int64_t)blockIdx.x * BM, n0 = (int64_t)blockIdx.y * BN;
     const int split = blockIdx.z, nsplit = gridDim.z;
@@ -242,11 +243,7 @@ __global__ void __launch_bounds__(kThreads) simt_wgrad_kernel(AV a, BV b, float*
     float acc[TM][TN];
     simt_mainloop<BM, BN, false, false>(a, b, m0, n0, kb, ke, acc);
     const int tile = blockIdx.y * gridDim.x + blockIdx.x;
-    if (threadIdx.x == 0 && split > 0) {
-        volatile int32_t* vs = sem + tile;
-        while (*vs != split) __nanosleep(64);
-        __threadfence();
-    }
+    if (threadIdx.x == 0 && split > 0) turn_wait(turns + tile, turn_tag(epoch, split - 1));
     __syncthreads();
     const int tx = threadIdx.x % 16, ty = threadIdx.x / 16;
 #pragma unroll
@@ -259,14 +256,13 @@ __global__ void __launch_bounds__(kThreads) simt_wgrad_kernel(AV a, BV b, float*
             if (cidx >= cols) continue;
             float* d = dw + r * cols + cidx;
             float v = alpha * acc[i][j];
-            if (split > 0) v += *d;
-            else if (beta != 0.f) v += beta * *d;
+            if (split > 0) v += __ldcg(d);
+            else if (beta != 0.f) v += beta * __ldcg(d);
             *d = v;
         }
     }
-    __threadfence();
     __syncthreads();
-    if (threadIdx.x == 0) atomicExch(sem + tile, split + 1 < nsplit ? split + 1 : 0);
+    if (threadIdx.x == 0 && split + 1 < nsplit) turn_post(turns + tile, turn_tag(epoch, split));
 }
 
 template <int BM, int BN, bool CKA, bool CKB, class AV, class BV, class EPI>
@@ -330,11 +326,10 @@ int simt_dgrad_ig(const Geom& g, int32_t b, float alpha, const float* dy, const 
 // WGRAD: dw[k][(r,s,c)] = sum_m dy[m][k] * B(m, (r,s,c)), B = implicit im2col
 // of x (IG) or the explicit col matrix (I2C, row pitch kpitch).
 int simt_wgrad(const Geom& g, int32_t b, float alpha, const float* dy, const float* xin, bool col_input,
-               int32_t kpitch, float beta, float* dw, const SemBuf& sem, int num_sms, cudaStream_t st) {
+               int32_t kpitch, float beta, float* dw, int num_sms, cudaStream_t st) {
     constexpr int BM = 128, BN = 128, BK = 8;
     const int64_t rows = g.k, cols = (int64_t)g.r * g.s * g.c, Kd = (int64_t)b * g.p * g.q;
     const int64_t tiles = ceil_div(cols, BN) * ceil_div(rows, BM);
-    if (tiles > sem.capacity) return (int)cudaErrorInvalidValue;
     // Enough splits for ~2 waves of 2 CTAs/SM, each split >= 256 pixels.
     int64_t want = std::max<int64_t>(1, (4LL * num_sms + tiles - 1) / tiles);
     int64_t maxs = std::max<int64_t>(1, Kd / 256);
@@ -342,13 +337,18 @@ int simt_wgrad(const Geom& g, int32_t b, float alpha, const float* dy, const flo
     int64_t kps = ceil_div(ceil_div(Kd, nsplit), BK) * BK;
     nsplit = ceil_div(Kd, kps);
     dim3 grid((unsigned)ceil_div(rows, BM), (unsigned)ceil_div(cols, BN), (unsigned)nsplit);
+    TurnRange tr{nullptr, 0};
+    if (nsplit > 1) {
+        const int e = alloc_turns(tiles, &tr);
+        if (e) return e;
+    }
     Dense a{dy, rows, Kd, 1, g.k, 0};  // A(k, m) = dy[m][k]
     if (col_input) {
         Dense bb{xin, cols, Kd, 1, kpitch, 0};  // B(j, m) = col[m][j]
-        simt_wgrad_kernel<BM, BN><<<grid, kThreads, 0, st>>>(a, bb, dw, rows, cols, Kd, kps, alpha, beta, sem.sem);
+        simt_wgrad_kernel<BM, BN><<<grid, kThreads, 0, st>>>(a, bb, dw, rows, cols, Kd, kps, alpha, beta, tr.ctr, tr.epoch);
     } else {
         Im2colT bb{Im2col{xin, Kd, g.h, g.w, g.c, g.p, g.q, g.s, g.pad, g.stride, (int)cols}};
-        simt_wgrad_kernel<BM, BN><<<grid, kThreads, 0, st>>>(a, bb, dw, rows, cols, Kd, kps, alpha, beta, sem.sem);
+        simt_wgrad_kernel<BM, BN><<<grid, kThreads, 0, st>>>(a, bb, dw, rows, cols, Kd, kps, alpha, beta, tr.ctr, tr.epoch);
     }
     count_launch();
     return (int)cudaGetLastError();

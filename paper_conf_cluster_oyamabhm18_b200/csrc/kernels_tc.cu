@@ -21,9 +21,11 @@
 //   MN-major: (MN/64 bf16 | MN/32 fp32) atoms, each KB rows x 128 B, SWIZZLE_128B
 // KB = 128 B / element size of K per stage; 4 MMAs (UMMA_K = 32 B) per stage.
 //
-// Backward-filter splits the pixel reduction over blockIdx.z and
-// combines the partial tiles in split order through per-tile turn counters
-// (deterministic; split 0 applies the user's beta).
+// Backward-filter splits the pixel reduction over the tile index z
+// and combines the partial tiles in split order through per-tile turn counters
+// (turns.cu): split s waits for split s-1, then reads dw, adds its partial and
+// writes it back (split 0 applies the user's beta), so dw is bitwise
+// reproducible run to run.
 #include <cuda.h>
 #include <cuda_bf16.h>
 #include <cuda_runtime.h>
@@ -201,8 +203,6 @@ enum AMode : int {
     A_TMA_IM2COL = 7,  // TMA im2col mode: FWD (x) or stride-1 DGRAD (dy, flipped taps), 128 pixels x KB channels
     A_GATHER_SMALLC = 8, // FWD, C*elt < 16 B (RGB layer): one 16-B chunk per filter tap, channels zero-padded
     A_GATHER_SMALLC_PAD = 9, // same K' layout from a channel-padded copy of x (16 B per pixel): cp.async
-    A_TMA_IM2COL_SMALLC = 10, // same K' layout from the padded copy by TMA im2col: one 128-pixel x 16-B box
-                              // per tap, SWIZZLE_NONE core matrices (LBO 2 KB between taps, SBO 128 B)
     A_HALO = 12,       // stride-1 FWD / DGRAD: per channel chunk, the full source rows a 128*mt-row tile of
                        // the extended output grid touches (one TMA box per row, zero-filled padding); each
                        // tap's A operand is a row-shifted window of that smem halo
@@ -273,8 +273,6 @@ struct TcArgs {
     int cp, s8;
     int bres_bytes;          // B_RESIDENT: smem bytes of the staged filter
     int max_lag;             // cp.async stages kept in flight per producer thread (<= 6)
-    int debug;               // MUCU_TC_DEBUG bits (timing experiments only): 1 skip stores, 2 skip A gather,
-                             // 4 skip TMA loads, 8 skip MMAs
     int mt;                  // 128-row halves per tile (1, or 2 for 256-row tiles with narrow N)
     // Space-to-depth layers (EPI_D2S / EPI_WGRAD_S2D): the real stride, C, R, S
     // (the GEMM itself runs on the stride-1 super-pixel geometry).
@@ -300,7 +298,8 @@ struct TcArgs {
     long long batch_stride;  // elements
     float alpha, beta;
     int out_bf16;
-    int32_t* sem;
+    unsigned long long* turns;  // split-K: launch-private turn counters (turns.cu), one per tile of a batch
+    unsigned long long epoch;
 };
 
 constexpr int kThreads = 288;  // 4 producer warps, 1 MMA warp, 4 epilogue warps
@@ -471,7 +470,7 @@ int pick_bn(int N, int step = 32, int overhead = 32, int max_bn = 256, int64_t m
     step = std::max(step, 32);  // the epilogue drains TMEM in 32-column chunks
     int best = step;
     int64_t best_cost = INT64_MAX;
-    const bool waves = mtiles > 0 && env_int("MUCU_BN_WAVES", 1);
+    const bool waves = mtiles > 0;
     for (int bn = step; bn <= max_bn; bn += step) {
         const int64_t nt = ceil_div(N, bn);
         // per-tile cost in wave mode: narrow tiles run well below the MMA rate of wide
@@ -496,7 +495,7 @@ struct Launch {
 };
 
 template <int ELT, int AM, int BM_, int EPI>
-int launch_t(Launch& L, cudaStream_t st) {
+int launch_t(Launch& L, cudaStream_t st, bool dry) {
     auto kern = tc_conv_gemm<ELT, AM, BM_, EPI>;
     L.a.a_merged = 0;
     if (AM == A_TMA_IM2COL && L.a.mt > 1 && L.ia.valid && env_int("MUCU_A_MERGE", 1)) {
@@ -511,6 +510,24 @@ int launch_t(Launch& L, cudaStream_t st) {
     const int a_stage = AM == A_HALO ? 0 : L.a.mt * 128 * 128;
     const int smem = 1024 + L.a.hstages * L.a.halo_bytes + L.a.stages * L.a.km * (a_stage + L.a.b_bytes) +
                      L.a.bres_bytes + (2 * L.a.stages + 6 + 2 * L.a.hstages) * 8 + 64;
+    if (smem > 232448) return -1;
+    // BackwardFilter split-K: one turn counter per output tile of every batch
+    constexpr bool SPLITK = (EPI == EPI_WGRAD_CHAIN || EPI == EPI_WGRAD_SMALLC || EPI == EPI_WGRAD_S2D ||
+                             EPI == EPI_WGRAD_WIN);
+    L.a.turns = nullptr;
+    L.a.epoch = 0;
+    if (dry) return 0;
+    if (SPLITK) {
+        const int64_t splits = L.a.zsplit ? L.a.zsplit : L.a.num_z;
+        if (splits > 1) {
+            const int64_t per_z = ceil_div(L.a.M, 128 * L.a.mt) * ceil_div(L.a.N, L.a.BN);
+            TurnRange tr;
+            const int e = alloc_turns(per_z * (L.a.num_z / splits), &tr);
+            if (e) return e;
+            L.a.turns = tr.ctr;
+            L.a.epoch = tr.epoch;
+        }
+    }
     static int configured = 0;  // per instantiation
     if (configured < smem) {
         cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 232448);
@@ -569,12 +586,12 @@ void use_mt2(Launch& L, int num_sms) {
     // no longer overlaps the next tile), worth it for long reductions only; measured
     // AlexNet conv2 FWD / conv3 DGRAD 0.19 / 0.22 -> 0.16 / 0.17 ms, while BN = 256
     // (one 128 x 256 chain is already near the MMA floor) got slower.
-    const bool wide_ok = env_int("MUCU_MT2_WIDE", 1) && a.num_kb >= 32 && a.BN <= 192;
+    const bool wide_ok = a.num_kb >= 32 && a.BN <= 192;
     if ((a.BN > 128 && !wide_ok) || env_int("MUCU_MT2", 1) == 0) return;
     const int force = env_int("MUCU_FORCE_MT", 0);  // tests: exercise 256/512-row tiles on small shapes
     if (force == 4 && a.BN <= 64) num_sms = 1;
     if (force == 2) { a.mt = 2; size_stages(a); return; }
-    if (a.BN <= 64 && env_int("MUCU_MT4", 1) && ceil_div(a.M, 512) >= num_sms) {
+    if (a.BN <= 64 && ceil_div(a.M, 512) >= num_sms) {
         a.mt = 4;
         size_stages(a);
         return;
@@ -618,8 +635,12 @@ bool halo_setup(TcArgs& a, int elt, int b, int Ho, int Wo, int R, int S, int pe,
 // ====================================================== micro-config run ==
 // Returns cudaError_t, or -1 when a shape has no tensor-core path.
 int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, const void* in0, const void* in1,
-                 float beta, void* out, char* ws, const WsLayout& WL, const SemBuf& sem, int num_sms,
-                 cudaStream_t st, CallCtx* ctx) {
+                 float beta, void* out, char* ws, const WsLayout& WL, int num_sms, cudaStream_t st,
+                 CallCtx* ctx) {
+    // Dry run (executor pre-validation): every host decision and tensor-map
+    // encoding, no launch.
+    const bool dry = ctx->dry;
+#define DRY(x) (dry ? 0 : (x))
     const int elt = elt_size(g.math);
     const int KB = 128 / elt;
     const int atom = 128 / elt;
@@ -636,8 +657,7 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
     A.stride = g.stride; A.K = g.k;
     A.tapR = g.r; A.tapS = g.s; A.ph_u = 1;
     A.max_lag = std::min(6, std::max(1, env_int("MUCU_MAX_LAG", 6)));
-    A.debug = env_int("MUCU_TC_DEBUG", 0);
-    A.alpha = alpha; A.beta = beta; A.out = out; A.out_bf16 = bf ? 1 : 0; A.sem = sem.sem;
+    A.alpha = alpha; A.beta = beta; A.out = out; A.out_bf16 = bf ? 1 : 0; 
     auto map2 = [&](CUtensorMap* tm, const void* base, uint64_t d0, uint64_t d1, uint64_t pitch_elems, uint32_t b0,
                     uint32_t b1, bool mn = false) {
         uint64_t dims[2] = {d0, d1}, str[1] = {pitch_elems * elt};
@@ -721,7 +741,7 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         const int64_t nkb = qrow ? (int64_t)b * g.p * A.win_qb : ceil_div(A.kred, KB * A.km);
         int64_t nsplit = std::min<int64_t>(std::min<int64_t>(std::max<int64_t>(1, (2LL * num_sms) / tiles),
                                                              std::max<int64_t>(1, nkb / 16)), 65535);
-        if (env_int("MUCU_SPLIT_WAVES", 1)) {
+        {
             // Wave-quantised split count: minimise waves x (stages per split + the
             // per-split epilogue / pipeline fill, ~E stages of 128-B k-blocks),
             // splits >= 4 stages each.  (Capping at 16 stages per split left e.g.
@@ -742,7 +762,7 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
     const bool Aok = (g.c % KB) == 0;  // vector gathers over C
     int err = 0;
 #define LAUNCH(AMODE, BMODE, EPIM) \
-    (elt == 2 ? launch_t<2, AMODE, BMODE, EPIM>(L, st) : launch_t<4, AMODE, BMODE, EPIM>(L, st))
+    (elt == 2 ? launch_t<2, AMODE, BMODE, EPIM>(L, st, dry) : launch_t<4, AMODE, BMODE, EPIM>(L, st, dry))
 
     if (type == MUCU_FWD && algo == MUCU_ALGO_IMPLICIT_GEMM) {
         A.M = (int)(b * PQ); A.N = g.k; A.kred = (int)RSC; A.gsrc = in0;
@@ -809,14 +829,10 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         // rows j = (r, atom, tap, c) over the padded copy xp, columns = the K filters.
         const Win z = win_geom(g);
         char* xp = ws + WL.a_off;
-        err = launch_win_pad(g, b, z.Wp, in0, xp, st);
+        err = DRY(launch_win_pad(g, b, z.Wp, in0, xp, st));
         if (err) return err;
         A.M = z.M; A.N = g.k; A.ldc = RSC; A.kred = (int)(b * PQ); A.cp = z.cpx; A.win_na = z.na; A.win_aw = z.aw;
         wgrad_tiling(atom, true, g.q);
-        if (beta != 1.f) {
-            err = launch_scale(g.k * RSC, beta, (float*)out, st);
-            if (err) return err;
-        }
         const int KD = KB * A.km;
         const uint64_t pb = (uint64_t)z.cpx * elt;
         const int wat = z.aw / elt;  // elements per A atom
@@ -852,7 +868,7 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         const int st_ = g.stride, Dr = z.Dr, Ds = z.Ds, Cs = z.Cs;
         const int kind = type == MUCU_BWD_DATA ? 4 : 3;
         if (type != MUCU_BWD_FILTER && (ctx->fixed_kind != kind || ctx->fixed_src != in1)) {
-            err = launch_s2d_filter(g, type == MUCU_BWD_DATA, z, in1, ws, st);
+            err = DRY(launch_s2d_filter(g, type == MUCU_BWD_DATA, z, in1, ws, st));
             if (err) return err;
             ctx->fixed_kind = kind; ctx->fixed_src = in1;
         }
@@ -896,7 +912,7 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         }
         const int I = z.I, J = z.J;
         char* xs = ws + WL.a_off;
-        err = launch_s2d_input(g, b, z.f, I, J, Cs, in0, xs, st);
+        err = DRY(launch_s2d_input(g, b, z.f, I, J, Cs, in0, xs, st));
         if (err) return err;
         // the GEMM sees the stride-1, pad-0 geometry over xs (Pu x Qu output super-pixels)
         A.H = I; A.W = J; A.C = Cs; A.R = Dr; A.S = Ds; A.pad = 0; A.stride = 1; A.tapR = Dr; A.tapS = Ds;
@@ -922,10 +938,6 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         const int64_t Mpix = (int64_t)b * PQ;
         A.M = g.k; A.N = Dr * Ds * Cs; A.ldc = RSC; A.kred = (int)Mpix; A.gsrc = xs;
         wgrad_tiling(atom, true);
-        if (beta != 1.f) {
-            err = launch_scale(g.k * RSC, beta, (float*)out, st);
-            if (err) return err;
-        }
         if (!map2(&L.ta, in1, g.k, (uint64_t)Mpix, g.k, atom, KB * A.km, true)) return -1;
         if (!make_im2col_map(&L.tb, elt, xs, Cs, J, I, b, 0, 0, -(Ds - 1), -(Dr - 1), KB * A.km, 1, true))
             return -1;
@@ -935,7 +947,7 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
     if (type == MUCU_FWD && algo == MUCU_ALGO_IM2COL_GEMM && small_c_tc(g)) {
         // RGB-like layer: x -> channel-padded copy (16 B / pixel) in the workspace,
         // then the tap-walking GEMM with async 16-B gathers and the staged filter.
-        err = launch_pad_channels(g, b, in0, ws + WL.a_off, st);
+        err = DRY(launch_pad_channels(g, b, in0, ws + WL.a_off, st));
         if (err) return err;
         A.M = (int)(b * PQ); A.N = g.k; A.ldc = g.k; A.gsrc = ws + WL.a_off; A.bsrc = in1;
         A.cp = 16 / elt; A.s8 = (int)align_up((uint64_t)g.s, 8);
@@ -948,12 +960,6 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         if (A.stages < 2) return -1;
         grid2(1);
         A.tma_bytes = 0;
-        // TMA im2col over the 16-B pixels works for bf16 but measured no faster
-        // than the cp.async gather (and hangs for fp32): opt-in only.
-        if (elt == 2 && env_int("MUCU_SMALLC_TMA", 0) &&
-            make_im2col_map(&L.ta, elt, A.gsrc, A.cp, g.w, g.h, b, -g.pad, -g.pad, g.pad - (g.s - 1),
-                            g.pad - (g.r - 1), 128, g.stride, false, true))
-            return LAUNCH(A_TMA_IM2COL_SMALLC, B_RESIDENT, EPI_STORE);
         return LAUNCH(A_GATHER_SMALLC_PAD, B_RESIDENT, EPI_STORE);
     }
     if (type == MUCU_FWD && algo == MUCU_ALGO_IM2COL_GEMM) {
@@ -962,14 +968,14 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         if (!is_pointwise(g)) {
             colp = ws + WL.a_off;
             kpitch = WL.kpitch;
-            err = launch_im2col(g, b, in0, (void*)colp, kpitch, st);
+            err = DRY(launch_im2col(g, b, in0, (void*)colp, kpitch, st));
             if (err) return err;
         }
         const void* wp = in1;
         int wpitch = (int)RSC;
         if (WL.filter_padded) {
             if (ctx->fixed_kind != 1 || ctx->fixed_src != in1) {
-                err = launch_pad_filter(g, in1, ws, WL.kpitch, st);
+                err = DRY(launch_pad_filter(g, in1, ws, WL.kpitch, st));
                 if (err) return err;
                 ctx->fixed_kind = 1; ctx->fixed_src = in1;
             }
@@ -995,9 +1001,7 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         void* V = ws + WL.a_off;
         void* D = ws + WL.b_off;
         float* Mx = (float*)(ws + WL.fixed_off);
-        err = launch_wgw_transforms(g, b, in0, in1, V, D, Tp, st);
-        if (err) return err;
-        err = launch_scale(16LL * Kp * Cp, 0.f, Mx, st);
+        err = DRY(launch_wgw_transforms(g, b, in0, in1, V, D, Tp, st));
         if (err) return err;
         A.M = g.k; A.N = g.c; A.ldc = Cp; A.kred = (int)Tp; A.out = Mx; A.alpha = 1.f; A.beta = 0.f; A.out_bf16 = 0;
         A.batch_stride = (long long)Kp * Cp;
@@ -1011,7 +1015,7 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         A.tma_bytes = A.km * (A.mt * 128 * KB * elt + A.bn_atoms * KB * 128);
         err = LAUNCH(A_TMA_MN2, B_TMA_MN2, EPI_WGRAD_CHAIN);
         if (err) return err;
-        return launch_wgw_output(g, alpha, Mx, beta, (float*)out, st);
+        return DRY(launch_wgw_output(g, alpha, Mx, beta, (float*)out, st));
     }
     if (algo == MUCU_ALGO_WINOGRAD_2X2_3X3) {
         const bool dg = type == MUCU_BWD_DATA;
@@ -1019,13 +1023,13 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         const int OH = dg ? g.h : g.p, OW = dg ? g.w : g.q;
         const int64_t Tt = (int64_t)((OH + 1) / 2) * ((OW + 1) / 2) * b;
         if (ctx->fixed_kind != 2 || ctx->fixed_src != in1) {
-            err = launch_wg_filter(g, dg, in1, ws, st);
+            err = DRY(launch_wg_filter(g, dg, in1, ws, st));
             if (err) return err;
             ctx->fixed_kind = 2; ctx->fixed_src = in1;
         }
         void* V = ws + WL.a_off;
         float* Mx = (float*)(ws + WL.b_off);
-        err = launch_wg_input(g, dg, b, in0, V, st);
+        err = DRY(launch_wg_input(g, dg, b, in0, V, st));
         if (err) return err;
         A.M = (int)Tt; A.N = O; A.num_kb = (int)ceil_div(I, KB); A.ldc = O;
         A.batch_stride = Tt * O; A.alpha = 1.f; A.beta = 0.f; A.out = Mx; A.out_bf16 = 0;
@@ -1036,7 +1040,7 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         A.tma_bytes = 16384 * A.mt + A.BN * 128;
         err = LAUNCH(A_TMA_K3, B_TMA_K3, EPI_STORE);
         if (err) return err;
-        return launch_wg_output(g, dg, b, alpha, Mx, beta, out, st);
+        return DRY(launch_wg_output(g, dg, b, alpha, Mx, beta, out, st));
     }
     if (type == MUCU_BWD_DATA && algo == MUCU_ALGO_IMPLICIT_GEMM && g.stride > 1 && g.k % KB == 0 &&
         use_tma_im2col()) {
@@ -1052,7 +1056,7 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         // elementwise pass instead of one GEMM launch each
         const bool zero_pass = beta == 0.f && (g.r < g.stride || g.s < g.stride) && (g.c * elt) % 16 == 0;
         if (zero_pass) {
-            err = launch_zero_tapless(g, b, out, st);
+            err = DRY(launch_zero_tapless(g, b, out, st));
             if (err) return err;
         }
         // One launch for all phases with taps when they tile equal sub-grids whose
@@ -1202,7 +1206,7 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
             // same pitch as ws_layout: one 128-B atom for short rows, else 16 B
             const int fpitch = RSC < atom ? atom : (int)align_up((uint64_t)RSC, (uint64_t)(16 / elt));
             if (ctx->fixed_kind != 1 || ctx->fixed_src != in1) {
-                err = launch_pad_filter(g, in1, ws, fpitch, st);
+                err = DRY(launch_pad_filter(g, in1, ws, fpitch, st));
                 if (err) return err;
                 ctx->fixed_kind = 1; ctx->fixed_src = in1;
             }
@@ -1221,18 +1225,14 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         A.tma_bytes = 16384 * A.mt + A.bn_atoms * KB * 128;
         err = LAUNCH(A_TMA_K2, B_TMA_MN2, EPI_STORE);
         if (err || pw) return err;
-        return launch_col2im(g, b, alpha, (const float*)(ws + WL.a_off), WL.kpitch, beta, out, st);
+        return DRY(launch_col2im(g, b, alpha, (const float*)(ws + WL.a_off), WL.kpitch, beta, out, st));
     }
     if (type == MUCU_BWD_FILTER) {
         // dw[k][(r,s,c)] = sum_m dy[m][k] B(m, (r,s,c)); A = dy MN-major via TMA.
         const int64_t Mpix = (int64_t)b * PQ;
         A.M = g.k; A.N = (int)RSC; A.ldc = RSC; A.kred = (int)Mpix; A.gsrc = in0;
-        // P:L58 output scale: apply the user's beta once, then every split adds.
-        if (beta != 1.f) {
-            err = launch_scale(g.k * RSC, beta, (float*)out, st);
-            if (err) return err;
-        }
-        (void)sem;
+        // P:L58 output scale: split 0 of every tile applies the user's beta, later
+        // splits add in split order (ordered turn counters, deterministic).
         const int a_bytes = 128 * KB * elt;
         // dy as the MN-major A operand: with K a multiple of the 128-B atom, a 3-D view
         // {atom element, pixel, atom index} loads a whole 128-row half (4 tf32 / 2 bf16
@@ -1250,7 +1250,7 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         };
         if (algo == MUCU_ALGO_IM2COL_GEMM && small_c_tc(g)) {
             // RGB-like layer: channel-padded copy of x, padded columns j' = (r, s8, c').
-            err = launch_pad_channels(g, b, in0, ws + WL.a_off, st);
+            err = DRY(launch_pad_channels(g, b, in0, ws + WL.a_off, st));
             if (err) return err;
             A.gsrc = ws + WL.a_off;
             A.cp = 16 / elt; A.s8 = (int)align_up((uint64_t)g.s, 8);
@@ -1265,7 +1265,7 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
             int64_t kp = g.c;
             if (!is_pointwise(g)) {
                 colp = ws + WL.a_off; kp = WL.kpitch;
-                err = launch_im2col(g, b, in0, (void*)colp, (int)kp, st);
+                err = DRY(launch_im2col(g, b, in0, (void*)colp, (int)kp, st));
                 if (err) return err;
             }
             if (RSC < atom) return -1;
@@ -1309,6 +1309,7 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         return LAUNCH(A_TMA_MN2, B_SCALAR_WG, EPI_WGRAD_CHAIN);
     }
 #undef LAUNCH
+#undef DRY
     return -1;
 }
 

@@ -74,8 +74,10 @@ mucu_status_t ws_layout(const Geom& g, int type, int algo, int32_t b, WsLayout* 
 
 // Per-call executor state (which b-independent workspace prefix is valid).
 struct CallCtx {
-    int fixed_kind = 0;  // 0 none, 1 padded filter, 2 Winograd U
+    int fixed_kind = 0;  // 0 none, 1 padded filter, 2 Winograd U, 3/4 space-to-depth filter
     const void* fixed_src = nullptr;
+    int last_algo = -1;  // algorithm of the previous micro-config (prefix invalidation)
+    bool dry = false;    // tensor-core dispatch decisions only, no launch (pre-validation)
 };
 
 struct Handle;
@@ -86,10 +88,34 @@ mucu_status_t run_micro(Handle* h, const Geom& g, int type, int algo, int32_t b,
 
 // ---------------------------------------------------------------- kernels --
 // All launchers are asynchronous on `st` and return a CUDA error code (0 = ok).
-struct SemBuf {
-    int32_t* sem;      // device, zero-initialised, left zero by every kernel
-    int32_t capacity;  // number of ints
+// Ordered split-K turn counters (turns.cu): a launch-private range of `count`
+// counters from a static device pool plus a process-unique epoch.  Split s of
+// a tile waits for tag(epoch, s - 1) and publishes tag(epoch, s).
+struct TurnRange {
+    unsigned long long* ctr;
+    unsigned long long epoch;
 };
+int alloc_turns(int64_t count, TurnRange* out);  // cudaError_t
+#ifdef __CUDACC__
+__host__ __device__ __forceinline__ unsigned long long turn_tag(unsigned long long epoch, int split) {
+    return (epoch << 20) + (unsigned long long)split + 1ull;
+}
+// One thread waits for the previous split's tag (acquire at gpu scope); the
+// caller then synchronises the threads that read dw.
+__device__ __forceinline__ void turn_wait(const unsigned long long* c, unsigned long long tag) {
+    unsigned long long v;
+    for (;;) {
+        asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(c) : "memory");
+        if (v == tag) break;
+        __nanosleep(32);
+    }
+}
+// One thread publishes after the dw writes of every thread of the group were
+// ordered before it by a barrier (release fence is cumulative).
+__device__ __forceinline__ void turn_post(unsigned long long* c, unsigned long long tag) {
+    asm volatile("fence.acq_rel.gpu;\n\tst.relaxed.gpu.global.u64 [%0], %1;" ::"l"(c), "l"(tag) : "memory");
+}
+#endif
 
 // SIMT fp32 GEMM-shaped convolution pieces (kernels_simt.cu).
 int simt_fwd_ig(const Geom& g, int32_t b, float alpha, const float* x, const float* w, float beta,
@@ -103,8 +129,7 @@ int simt_gemm_nn(int64_t M, int64_t N, int64_t K, float alpha, const float* A, i
 int simt_dgrad_ig(const Geom& g, int32_t b, float alpha, const float* dy, const float* w,
                   float beta, float* dx, cudaStream_t st);
 int simt_wgrad(const Geom& g, int32_t b, float alpha, const float* dy, const float* x_or_col,
-               bool col_input, int32_t kpitch, float beta, float* dw, const SemBuf& sem,
-               int num_sms, cudaStream_t st);
+               bool col_input, int32_t kpitch, float beta, float* dw, int num_sms, cudaStream_t st);
 
 // Element-wise / data-movement kernels (kernels_elem.cu); T = float or bf16 by math.
 int launch_im2col(const Geom& g, int32_t b, const void* x, void* col, int32_t kpitch, cudaStream_t st);
@@ -138,7 +163,7 @@ int simt_gemm_tt(int64_t K, int64_t C, int64_t Tp, const float* V, const float* 
 // runs one micro-configuration; returns a cudaError_t, or -1 if this
 // (type, algo, geometry) has no tensor-core implementation.
 int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, const void* in0, const void* in1,
-                 float beta, void* out, char* ws, const WsLayout& L, const SemBuf& sem, int num_sms,
-                 cudaStream_t st, CallCtx* ctx);
+                 float beta, void* out, char* ws, const WsLayout& L, int num_sms, cudaStream_t st,
+                 CallCtx* ctx);
 
 }  // namespace mucu

@@ -11,6 +11,19 @@
 // Two TMEM accumulators (2 x BN columns) let the epilogue of tile i overlap
 // the mainloop of tile i+1 (tmem_full / tmem_empty barriers).
 
+// dst[ofs[j] * stride] = alpha * v[j] + beta * dst[...] for the 32 accumulator
+// columns of one row (ofs < 0: skipped); all loads issue before the stores.
+// beta == 0 never reads dst (it may hold garbage / NaN).
+__device__ __forceinline__ void rmw32(float* dst, const int (&ofs)[32], size_t stride, const uint32_t* v, float alpha,
+                                      float beta) {
+    float old[32];
+#pragma unroll
+    for (int j = 0; j < 32; ++j) old[j] = (beta != 0.f && ofs[j] >= 0) ? __ldcg(dst + (size_t)ofs[j] * stride) : 0.f;
+#pragma unroll
+    for (int j = 0; j < 32; ++j)
+        if (ofs[j] >= 0) dst[(size_t)ofs[j] * stride] = alpha * __uint_as_float(v[j]) + beta * old[j];
+}
+
 template <int ELT, int AM, int BM_, int EPI>
 __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constant__ TcArgs p,
                                                             const __grid_constant__ CUtensorMap tmA,
@@ -30,9 +43,8 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
     constexpr bool B_MN = (BM_ == B_TMA_MN2 || BM_ == B_TMA_MN3 || BM_ == B_GATHER_WG || BM_ == B_SCALAR_DGRAD ||
                            BM_ == B_SCALAR_WG || BM_ == B_TMA_IM2COL || BM_ == B_GATHER_SMALLC ||
                            BM_ == B_GATHER_SMALLC_PAD || BM_ == B_TMA_DYROW);
-    constexpr bool A_TMA = (AM == A_TMA_K2 || AM == A_TMA_K3 || AM == A_TMA_MN2 || AM == A_TMA_IM2COL ||
-                            AM == A_TMA_IM2COL_SMALLC || WIN || AM == A_HALO);
-    constexpr bool A_NOSWZ = (AM == A_TMA_IM2COL_SMALLC);  // unswizzled core matrices, one 2-KB box per tap
+    constexpr bool A_TMA = (AM == A_TMA_K2 || AM == A_TMA_K3 || AM == A_TMA_MN2 || AM == A_TMA_IM2COL || WIN ||
+                            AM == A_HALO);
     constexpr bool B_TMA = (BM_ == B_TMA_K2 || BM_ == B_TMA_K3 || BM_ == B_TMA_MN2 || BM_ == B_TMA_MN3 ||
                             BM_ == B_TMA_IM2COL || BM_ == B_TMA_DYROW);
     constexpr bool B_RES = (BM_ == B_RESIDENT);
@@ -140,16 +152,12 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                     if (lane == 0) {
                         const uint32_t dst = smem_u32(sA + (size_t)hs * p.halo_bytes);
                         const uint32_t fb = smem_u32(&hfull[hs]);
-                        if (p.debug & 4) {
-                            mbar_arrive(fb);
-                        } else {
-                            mbar_arrive_tx(fb, (uint32_t)(nr * p.hx_W * 128));
-                            int n_ = G0 / p.hx_H, hx = G0 - n_ * p.hx_H;
-                            for (int i = 0; i < nr; ++i) {
-                                tma_load_4d(dst + (uint32_t)(i * p.hx_W * 128), &tmA, fb, c * KB, -p.hx_pe,
-                                            hx - p.hx_pe, n_);
-                                if (++hx == p.hx_H) { hx = 0; ++n_; }
-                            }
+                        mbar_arrive_tx(fb, (uint32_t)(nr * p.hx_W * 128));
+                        int n_ = G0 / p.hx_H, hx = G0 - n_ * p.hx_H;
+                        for (int i = 0; i < nr; ++i) {
+                            tma_load_4d(dst + (uint32_t)(i * p.hx_W * 128), &tmA, fb, c * KB, -p.hx_pe,
+                                        hx - p.hx_pe, n_);
+                            if (++hx == p.hx_H) { hx = 0; ++n_; }
                         }
                     }
                     __syncwarp();
@@ -168,18 +176,14 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                         if (lane == 0) {
                             const uint32_t bT = smem_u32(sB + (size_t)s * B_BYTES);
                             const uint32_t fb = smem_u32(&full[s]);
-                            if (p.debug & 4) {
-                                mbar_arrive(fb);
-                            } else {
-                                mbar_arrive_tx(fb, (uint32_t)p.tma_bytes);
-                                if constexpr (BM_ == B_TMA_K2) tma_load_2d(bT, &tmB, fb, tap * p.C + c * KB, n0);
-                                if constexpr (BM_ == B_TMA_MN3) {
-                                    // DGRAD: tap (r', s') of the flipped filter = w[.][R-1-r'][S-1-s'][.]
-                                    const int rr = tap / p.tapS, ss = tap - rr * p.tapS;
-                                    const int rs = (p.R - 1 - rr) * p.S + (p.S - 1 - ss);
-                                    for (int a = 0; a < p.bn_atoms; ++a)
-                                        tma_load_3d(bT + a * KB * 128, &tmB, fb, n0 + a * (128 / ELT), rs, c * KB);
-                                }
+                            mbar_arrive_tx(fb, (uint32_t)p.tma_bytes);
+                            if constexpr (BM_ == B_TMA_K2) tma_load_2d(bT, &tmB, fb, tap * p.C + c * KB, n0);
+                            if constexpr (BM_ == B_TMA_MN3) {
+                                // DGRAD: tap (r', s') of the flipped filter = w[.][R-1-r'][S-1-s'][.]
+                                const int rr = tap / p.tapS, ss = tap - rr * p.tapS;
+                                const int rs = (p.R - 1 - rr) * p.S + (p.S - 1 - ss);
+                                for (int a = 0; a < p.bn_atoms; ++a)
+                                    tma_load_3d(bT + a * KB * 128, &tmB, fb, n0 + a * (128 / ELT), rs, c * KB);
                             }
                         }
                         __syncwarp();
@@ -194,14 +198,6 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
         const T* gx = (const T*)p.gsrc;
         const int lag = min(S - 1, p.max_lag);
         const int gch = (AM == A_GATHER_DGRAD || (AM == A_TMA_IM2COL && p.im2col_dgrad)) ? p.K : p.C;
-        if constexpr (A_NOSWZ) {
-            // Taps past S are never loaded (their filter columns are zero); keep
-            // those A slots finite by zeroing every stage once.
-            for (int i = t; i < S * A_BYTES / 16; i += 128)
-                asm volatile("st.shared.v4.b32 [%0], {%1, %1, %1, %1};" ::"r"(smem_u32(sA) + i * 16), "r"(0)
-                             : "memory");
-            fence_proxy_async();
-        }
         if constexpr (B_RES) {
             // Stage the whole zero-padded filter once: B(n, k') with k' = (r, s8, c')
             // -> w[n][r][s][c'] (0 for s >= S or c' >= C), K-major SW128 per k-block.
@@ -293,7 +289,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                     ich = pp * p.stride - p.pad; icw = qq * p.stride - p.pad;
                 }
             };
-            if constexpr (AM == A_TMA_IM2COL || AM == A_TMA_IM2COL_SMALLC) {
+            if constexpr (AM == A_TMA_IM2COL) {
 #pragma unroll
                 for (int hh = 0; hh < 4; ++hh)
                     if (hh < p.mt) ic_of(m0 + 128 * hh, ic_w[hh], ic_h[hh], ic_n[hh]);
@@ -365,21 +361,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                 const uint32_t aT = smem_u32(sA + (size_t)s * A_BYTES);
                 const uint32_t bT = smem_u32(sB + (size_t)s * B_BYTES);
                 const uint32_t fb = smem_u32(&full[s]);
-                if (A_NOSWZ && t == 0) {
-                    // k-block = filter row r, taps s0..s0+7 of the padded x (16 B per pixel)
-                    const int groups = p.s8 / 8;
-                    const int r = kb / groups, s0 = (kb - r * groups) * 8;
-                    const int nv = min(8, p.S - s0);
-                    mbar_arrive_tx(fb, (uint32_t)(nv * 128 * 16 * p.mt));
-#pragma unroll
-                    for (int hh = 0; hh < 4; ++hh)
-                        if (hh < p.mt)
-                            for (int j = 0; j < nv; ++j)
-                                tma_load_im2col_4d(aT + hh * 16384 + j * 2048, &tmA, fb, 0, ic_w[hh], ic_h[hh],
-                                                   ic_n[hh], (uint16_t)(s0 + j), (uint16_t)r);
-                } else if ((A_TMA || B_TMA) && t == 0 && (p.debug & 4)) {
-                    mbar_arrive(fb);  // debug bit 2: no TMA loads (MMA-rate experiments)
-                } else if ((A_TMA || B_TMA) && t == 0) {
+                if ((A_TMA || B_TMA) && t == 0) {
                     mbar_arrive_tx(fb, (uint32_t)p.tma_bytes);
                     // A: p.mt blocks of 128 rows (16 KB each)
 #pragma unroll
@@ -510,7 +492,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                         }
                     }
                 }
-                if (AM == A_GATHER_SMALLC_PAD && !(p.debug & 2)) {  // debug bit 1: skip the A gather
+                if constexpr (AM == A_GATHER_SMALLC_PAD) {
                     // k-block = filter row r, taps s0..s0+7; chunk j = tap s0 + j = one
                     // 16-B padded pixel of the channel-padded x (async, lagged arrive).
                     const int groups = p.s8 / 8;
@@ -745,12 +727,9 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                     for (int tap = 0; tap < taps; ++tap) {
                         mbar_wait(smem_u32(&full[s]), ph);
                         tc_fence_after();
-                        if (lane == 0 && (p.debug & 8)) {
-                            mma_commit(smem_u32(&empty[s]));
-                            if (tap == taps - 1) mma_commit(smem_u32(&hempty[hs]));
-                        } else if (lane == 0) {
-                            const int rr = (p.debug & 32) ? 0 : tap / p.tapS;
-                            const int ss = (p.debug & 16) ? 0 : tap - (tap / p.tapS) * p.tapS;
+                        if (lane == 0) {
+                            const int rr = tap / p.tapS;
+                            const int ss = tap - rr * p.tapS;
                             const uint32_t aT = hbase + (uint32_t)((rr * p.hx_W + ss) * 128);
                             const uint32_t bT = smem_u32(sB + (size_t)s * B_BYTES);
 #pragma unroll
@@ -786,7 +765,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                 mbar_wait(smem_u32(&full[s]), ph);
                 tc_fence_after();
                 // whole warp (converged): elect.sync inside the MMA / commit picks the issuer
-                if (!(p.debug & 8)) {  // debug bit 3: no MMAs (load-rate experiments)
+                {
                     const uint32_t aT = smem_u32(sA + (size_t)s * A_BYTES);
                     const uint32_t bT = B_RES ? smem_u32(sBres) + (uint32_t)(kb * p.BN * 128)
                                               : smem_u32(sB + (size_t)s * B_BYTES);
@@ -806,15 +785,12 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
 #pragma unroll
                             for (int hh = 0; hh < MT; ++hh) {
                                 const uint32_t aH = aT + hh * (A_MN ? (uint32_t)A_HALF : 16384u);
-                                // no-swizzle A: core matrices 8 rows x 16 B, SBO 128 B (rows),
-                                // LBO 2 KB (next tap); one MMA covers 32 B of K = 2 taps
                                 // window atoms of aw bytes: KD rows x aw per atom column, 8-row
                                 // groups aw*8 apart; UMMA swizzle 2 / 4 / 6 = 128 / 64 / 32 B
                                 const uint64_t ad =
                                     WIN && WAW < 128
                                         ? sdesc(aH + (uint32_t)(jj * KB) * WAW + j * UMMA_K * WAW, KDm * WAW, 8 * WAW,
                                                 WAW == 64 ? 4u : 6u)
-                                    : A_NOSWZ ? sdesc(aH + j * 4096, 2048, 128, 0)
                                     : A_MN  ? sdesc(aH + kofs + j * UMMA_K * 128, KDm * 128, MN_SBO, MN_LAYOUT)
                                             : sdesc(aH + j * 32, 16, 1024);
                                 mma_elect<ELT>(dtm + (uint32_t)(hh * p.BN), ad, bd, idesc,
@@ -856,6 +832,23 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
             const bool has_acc = kb_end > kb_begin;
             mbar_wait(smem_u32(&tfull[acc]), aph);
             tc_fence_after();
+            // Split-K BackwardFilter, deterministic: split sp of this dw tile
+            // adds its partial after split sp-1 (turn counter), split 0 applies beta.
+            float bsplit = p.beta;
+            unsigned long long* turn = nullptr;
+            int sp = 0;
+            if constexpr (SPLITK) {
+                sp = p.zsplit ? z % p.zsplit : z;
+                bsplit = sp == 0 ? p.beta : 1.f;
+                if (p.turns) {
+                    const int batch = p.zsplit ? z / p.zsplit : 0;
+                    turn = p.turns + (size_t)batch * per_z + (tile - z * per_z);
+                    if (sp > 0) {
+                        if (threadIdx.x == 160) turn_wait(turn, turn_tag(p.epoch, sp - 1));
+                        asm volatile("bar.sync 1, 128;" ::: "memory");  // the 4 epilogue warps
+                    }
+                }
+            }
             auto drain = [&](const int hh) {
             const int m = m0 + 128 * hh + row;
             // Output row of GEMM row m (phase mode scatters sub-grid rows back to dx).
@@ -913,7 +906,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                             } else {
                                 v[0] = v[1] = v[2] = v[3] = 0u;
                             }
-                            if (!hv || (p.debug & 1)) continue;
+                            if (!hv) continue;
                             float o[4];
 #pragma unroll
                             for (int u = 0; u < 4; ++u) o[u] = p.alpha * __uint_as_float(v[u]);
@@ -973,7 +966,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
 #pragma unroll
                     for (int j = 0; j < 32; ++j) v[j] = 0u;
                 }
-                if (m >= p.M || !rowok || (p.debug & 1)) continue;  // debug bit 0: skip stores (timing experiments)
+                if (m >= p.M || !rowok) continue;
                 const int nb = n0 + c0;
                 if constexpr (EPI == EPI_D2S) {
                     // super-pixel row (n, i, jj); column (a, b, c) walked incrementally:
@@ -1031,17 +1024,19 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                     float* drow = outF + (size_t)m * p.ldc;
                     const int stc = p.s2_st * p.s2_C, real = stc * p.s2_st;
                     int tap = nb / p.C, ch = nb - tap * p.C;
+                    int dofs[32];
 #pragma unroll
                     for (int j = 0; j < 32; ++j) {
+                        dofs[j] = -1;
                         if (nb + j < p.N && ch < real) {
                             const int d = tap / p.S, e = tap - d * p.S;
                             const int a = ch / stc, rem = ch - a * stc, bq = rem / p.s2_C, c = rem - bq * p.s2_C;
                             const int r = p.s2_st * d + a, sx = p.s2_st * e + bq;
-                            if (r < p.s2_R && sx < p.s2_S)
-                                atomicAdd(drow + (r * p.s2_S + sx) * p.s2_C + c, p.alpha * __uint_as_float(v[j]));
+                            if (r < p.s2_R && sx < p.s2_S) dofs[j] = (r * p.s2_S + sx) * p.s2_C + c;
                         }
                         if (++ch == p.C) { ch = 0; ++tap; }
                     }
+                    rmw32(drow, dofs, 1, v, p.alpha, bsplit);
                 } else if constexpr (EPI == EPI_WGRAD_WIN) {
                     // row m = (r, atom aa, tap t, channel c) -> dw[k][r][aa*taps + t][c], k = nb + j
                     constexpr int per_atom = WAW / ELT;
@@ -1050,40 +1045,47 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                     const int r = ja / p.win_na, sx = (ja - r * p.win_na) * (per_atom / p.cp) + t;
                     if (r < p.R && sx < p.S && c < p.C) {
                         float* d = outF + (size_t)nb * p.ldc + (r * p.S + sx) * p.C + c;
+                        int dofs[32];
 #pragma unroll
-                        for (int j = 0; j < 32; ++j)
-                            if (nb + j < p.N)
-                                asm volatile("red.global.add.f32 [%0], %1;" ::"l"(d + (size_t)j * p.ldc),
-                                             "f"(p.alpha * __uint_as_float(v[j]))
-                                             : "memory");
+                        for (int j = 0; j < 32; ++j) dofs[j] = nb + j < p.N ? j : -1;
+                        rmw32(d, dofs, (size_t)p.ldc, v, p.alpha, bsplit);
                     }
                 } else if constexpr (EPI == EPI_WGRAD_SMALLC) {
                     // padded column j' = (r, s8, c') -> dw column (r*S + s)*C + c (skip padding)
                     float* drow = outF + (size_t)m * p.ldc;
+                    int dofs[32];
 #pragma unroll
                     for (int j = 0; j < 32; ++j) {
                         const int jp = nb + j;
                         const int c = jp % p.cp, t2 = jp / p.cp, s_ = t2 % p.s8, r = t2 / p.s8;
-                        if (jp < p.N && c < p.C && s_ < p.S)
-                            atomicAdd(drow + (r * p.S + s_) * p.C + c, p.alpha * __uint_as_float(v[j]));
+                        dofs[j] = (jp < p.N && c < p.C && s_ < p.S) ? (r * p.S + s_) * p.C + c : -1;
                     }
+                    rmw32(drow, dofs, 1, v, p.alpha, bsplit);
                 } else if constexpr (EPI == EPI_WGRAD_CHAIN) {
-                    // dw += alpha * partial (beta was applied by a prescale launch);
-                    // 16-byte vector reductions in L2 (red.global.add.v4.f32).
+                    // dw = alpha * partial + bsplit * dw (bsplit = beta on split 0, else 1),
+                    // in split order: 16-byte vector read-modify-write
                     float* d = outF + (p.zsplit ? (size_t)(z / p.zsplit) * p.batch_stride : 0) + (size_t)m * p.ldc + nb;
-                    const bool vec = (nb + 32 <= p.N) && ((p.ldc & 3) == 0);
+                    const bool vec = (nb + 32 <= p.N) && ((p.ldc & 3) == 0) && ((((uintptr_t)p.out) & 15) == 0);
                     if (vec) {
+                        float4 o[8];
 #pragma unroll
-                        for (int j = 0; j < 32; j += 4)
-                            asm volatile("red.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(d + j),
-                                         "f"(p.alpha * __uint_as_float(v[j])), "f"(p.alpha * __uint_as_float(v[j + 1])),
-                                         "f"(p.alpha * __uint_as_float(v[j + 2])),
-                                         "f"(p.alpha * __uint_as_float(v[j + 3]))
-                                         : "memory");
+                        for (int j = 0; j < 8; ++j)
+                            o[j] = bsplit != 0.f ? __ldcg(reinterpret_cast<const float4*>(d) + j)
+                                                 : make_float4(0.f, 0.f, 0.f, 0.f);
+#pragma unroll
+                        for (int j = 0; j < 8; ++j) {
+                            float4 q;
+                            q.x = p.alpha * __uint_as_float(v[4 * j]) + bsplit * o[j].x;
+                            q.y = p.alpha * __uint_as_float(v[4 * j + 1]) + bsplit * o[j].y;
+                            q.z = p.alpha * __uint_as_float(v[4 * j + 2]) + bsplit * o[j].z;
+                            q.w = p.alpha * __uint_as_float(v[4 * j + 3]) + bsplit * o[j].w;
+                            reinterpret_cast<float4*>(d)[j] = q;
+                        }
                     } else {
+                        int dofs[32];
 #pragma unroll
-                        for (int j = 0; j < 32; ++j)
-                            if (nb + j < p.N) atomicAdd(d + j, p.alpha * __uint_as_float(v[j]));
+                        for (int j = 0; j < 32; ++j) dofs[j] = nb + j < p.N ? j : -1;
+                        rmw32(d, dofs, 1, v, p.alpha, bsplit);
                     }
                 } else if (p.out_bf16) {
                     __nv_bfloat16* d = (__nv_bfloat16*)outT + (size_t)mrow * p.ldc + nb;
@@ -1138,6 +1140,12 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
             }
             };  // drain one 128-row half
             for (int hh = 0; hh < p.mt; ++hh) drain(hh);
+            if constexpr (SPLITK) {
+                if (turn) {  // this split's writes are done: hand the tile to split sp + 1
+                    asm volatile("bar.sync 1, 128;" ::: "memory");
+                    if (threadIdx.x == 160) turn_post(turn, turn_tag(p.epoch, sp));
+                }
+            }
             // release this accumulator to the MMA warp
             tc_fence_before();
             __syncwarp();

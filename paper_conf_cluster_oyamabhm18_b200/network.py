@@ -86,8 +86,12 @@ def shard_benchmark(costs: Dict[str, int], world: int) -> List[List[str]]:
 
 
 class ConvNet:
-    def __init__(self, handle: L.Handle, layers: Sequence, n: int, math: int, device: str = "cuda"):
+    def __init__(self, handle: L.Handle, layers: Sequence, n: int, math: int, device: str = "cuda",
+                 types: Sequence[int] = TYPES):
+        """types: the convolution operations to plan and run per layer (all three for
+        a training iteration; e.g. (FWD,) for BASELINE config 1)."""
         self.h = handle
+        self.types = tuple(types)
         self.layers = list(layers)
         self.n = n
         self.math = math
@@ -95,7 +99,7 @@ class ConvNet:
         self.dtype = torch.bfloat16 if math == L.MATH_BF16 else torch.float32
         self.descs = [L.desc(n, l.c, l.h, l.w, l.k, l.r, l.s, l.pad, l.stride, math) for l in self.layers]
         self.kernels: Dict[Tuple[int, int], Kernel] = {
-            (i, t): Kernel(i, t, d) for i, d in enumerate(self.descs) for t in TYPES}
+            (i, t): Kernel(i, t, d) for i, d in enumerate(self.descs) for t in self.types}
         self.tensors: List[Dict[str, torch.Tensor]] = []
         self.workspaces: Dict[Tuple[int, int], Optional[torch.Tensor]] = {}
         self.net_ws: Optional[torch.Tensor] = None
@@ -200,15 +204,15 @@ class ConvNet:
         self._alloc_workspaces()
 
     def plan_undivided(self, ws_limit: int):
-        """Best single algorithm at micro-batch N within the limit."""
+        """Best single algorithm at micro-batch N within the limit: the
+        C planner (mucu_plan_wr) on the table restricted to b = N, i.e. exactly
+        what the `undivided` batch-size policy benchmarks."""
         n = self.n
         for k in self.kernels.values():
             t, w = k.table
-            fit = [(int(t[a, n]), int(w[a, n]), a) for a in range(L.NUM_ALGOS) if t[a, n] >= 0 and w[a, n] <= ws_limit]
-            if not fit:
-                raise L.MucuError(3, f"no algorithm fits {ws_limit} B undivided for kernel {k.layer}/{k.conv_type}")
-            tt, ww, a = min(fit)
-            k.plan, k.est_ns = [(a, n)], tt
+            tu = np.full_like(t, -1)
+            tu[:, n] = t[:, n]
+            k.est_ns, k.plan = L.plan_wr(n, tu, w, ws_limit)
             k.ws_bytes = T.plan_workspace(k.desc, k.conv_type, k.plan)
         self._alloc_workspaces()
 
@@ -268,9 +272,12 @@ class ConvNet:
             if not (skip_conv1_dgrad and i == 0):
                 order.append((i, L.BWD_DATA))
             order.append((i, L.BWD_FILTER))
+        order = [o for o in order if o in self.kernels]
+        zeroed = False
         for i, t in order:
-            if (i, t) == order[len(self.layers)]:
+            if t != L.FWD and not zeroed:
                 self.dw_flat.zero_()  # zero_grad, once per iteration, before the first backward call
+                zeroed = True
             if on_op:
                 on_op(i, t, "begin")
             self.run_kernel(i, t)
@@ -290,6 +297,8 @@ class ConvNet:
         hook = on_op or (lambda *a: None)
 
         def run(i, t):
+            if (i, t) not in self.kernels:
+                return
             hook(i, t, "begin")
             self.run_kernel(i, t)
             hook(i, t, "end")
@@ -311,8 +320,8 @@ class ConvNet:
         main.wait_stream(side)
 
     def flops_per_iteration(self, skip_conv1_dgrad: bool = False) -> int:
-        f = sum(layer_flops(l, self.n) for l in self.layers) * 3
-        return f - (layer_flops(self.layers[0], self.n) if skip_conv1_dgrad else 0)
+        f = sum(layer_flops(self.layers[i], self.n) for (i, t) in self.kernels)
+        return f - (layer_flops(self.layers[0], self.n) if skip_conv1_dgrad and (0, L.BWD_DATA) in self.kernels else 0)
 
     def summary(self):
         rows = []

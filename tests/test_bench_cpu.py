@@ -27,3 +27,30 @@ def test_reference_arm_nonzero_rank_is_silent():
     r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--impl", "reference", "--steps", "1",
                         "--warmup", "0", "--cpu-sample", "1"], capture_output=True, text=True, timeout=600, env=env)
     assert r.returncode == 0 and r.stdout.strip() == ""
+
+
+def test_reference_arm_single_layer_cfg1():
+    """BASELINE config 1 (AlexNet conv2 forward, N = 8) as a bench workload."""
+    r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--impl", "reference", "--steps", "1",
+                        "--warmup", "0", "--cpu-sample", "1", "--layers", "conv2", "--types", "fwd", "--batch", "8",
+                        "--math", "f32", "--ws-mib", "8", "--policy", "all"],
+                       capture_output=True, text=True, timeout=600)
+    assert r.returncode == 0, r.stderr[-2000:]
+    line = json.loads(r.stdout.strip().splitlines()[-1])
+    assert line["config"]["workload"] == "alexnet conv2 fwd (1 kernel)"
+    assert line["config"]["batch_per_gpu"] == 8
+
+
+def test_gpus_n_self_spawns_ranks():
+    """--gpus 2 outside torchrun re-launches bench.py under torch.distributed.run
+    with two ranks; rank 0 alone prints (here: the CPU reference arm, strong
+    scaling of a global batch)."""
+    env = {k: v for k, v in os.environ.items() if k not in ("WORLD_SIZE", "RANK", "LOCAL_RANK")}
+    r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--impl", "reference", "--gpus", "2",
+                        "--steps", "1", "--warmup", "0", "--cpu-sample", "1", "--layers", "conv5", "--types", "fwd",
+                        "--global-batch", "4"], capture_output=True, text=True, timeout=600, env=env)
+    assert r.returncode == 0, r.stderr[-3000:]
+    lines = [l for l in r.stdout.strip().splitlines() if l.startswith("{")]
+    assert len(lines) == 1
+    line = json.loads(lines[0])
+    assert line["n_gpus"] == 2 and line["scaling"] == "strong" and line["config"]["batch_per_gpu"] == 2

@@ -92,7 +92,7 @@ def test_parity_integer_exact(case, math):
     assert np.array_equal(got, ref)
 
 
-@pytest.mark.parametrize("math", [mu.MATH_F32, mu.MATH_BF16], ids=["f32", "bf16"])
+@pytest.mark.parametrize("math", [mu.MATH_F32, mu.MATH_TF32, mu.MATH_BF16], ids=["f32", "tf32", "bf16"])
 @pytest.mark.parametrize("case", [c for c in CASES if c[1] != mu.BWD_FILTER], ids=_ids)
 def test_micro_batch_bit_identity(case, math):
     """I1: FWD / DGRAD split into micro-batches == the same algorithm at full N, bitwise."""

@@ -518,7 +518,7 @@ def main():
     if os.path.exists(tp):
         try:
             tj = json.load(open(tp))
-            traffic = tj.get(f"{args.config}/{args.math}/{layers[li].name}/{mu.TYPE_NAMES[lt]}/b{args.batch}")
+            traffic = tj.get(f"{args.config}/{args.math}/{layers[li].name}/{mu.TYPE_NAMES[lt]}")
         except Exception:
             traffic = None
 

@@ -298,7 +298,11 @@ struct TcArgs {
     long long batch_stride;  // elements
     float alpha, beta;
     int out_bf16;
-    unsigned long long* turns;  // split-K: launch-private turn counters (turns.cu), one per tile of a batch
+    // Cluster split-K BackwardFilter: cl CTAs (one split each) reduce one output tile
+    // through DSMEM; split groups of cl are ordered by turn counters (turns.cu), one
+    // per (batch, tile, row slab).  stg_bytes: the epilogue's staging over the ring.
+    int cl, stg_bytes;
+    unsigned long long* turns;
     unsigned long long epoch;
 };
 
@@ -508,21 +512,23 @@ int launch_t(Launch& L, cudaStream_t st, bool dry) {
         }
     }
     const int a_stage = AM == A_HALO ? 0 : L.a.mt * 128 * 128;
-    const int smem = 1024 + L.a.hstages * L.a.halo_bytes + L.a.stages * L.a.km * (a_stage + L.a.b_bytes) +
-                     L.a.bres_bytes + (2 * L.a.stages + 6 + 2 * L.a.hstages) * 8 + 64;
+    const int ring = L.a.hstages * L.a.halo_bytes + L.a.stages * L.a.km * (a_stage + L.a.b_bytes) + L.a.bres_bytes;
+    const int smem = 1024 + std::max(ring, L.a.stg_bytes) + (2 * L.a.stages + 6 + 2 * L.a.hstages) * 8 + 64;
     if (smem > 232448) return -1;
-    // BackwardFilter split-K: one turn counter per output tile of every batch
     constexpr bool SPLITK = (EPI == EPI_WGRAD_CHAIN || EPI == EPI_WGRAD_SMALLC || EPI == EPI_WGRAD_S2D ||
                              EPI == EPI_WGRAD_WIN);
+    if (!SPLITK && L.a.cl) return -1;
     L.a.turns = nullptr;
     L.a.epoch = 0;
     if (dry) return 0;
-    if (SPLITK) {
+    // Cluster split-K with more split groups than one: a turn counter per (batch,
+    // tile, row slab) orders the groups' additions into dw.
+    if (SPLITK && L.a.cl) {
         const int64_t splits = L.a.zsplit ? L.a.zsplit : L.a.num_z;
-        if (splits > 1) {
+        if (splits > L.a.cl) {
             const int64_t per_z = ceil_div(L.a.M, 128 * L.a.mt) * ceil_div(L.a.N, L.a.BN);
             TurnRange tr;
-            const int e = alloc_turns(per_z * (L.a.num_z / splits), &tr);
+            const int e = alloc_turns(per_z * (L.a.num_z / splits) * L.a.cl, &tr);
             if (e) return e;
             L.a.turns = tr.ctr;
             L.a.epoch = tr.epoch;
@@ -532,6 +538,7 @@ int launch_t(Launch& L, cudaStream_t st, bool dry) {
     if (configured < smem) {
         cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 232448);
         if (e) return (int)e;
+        if (SPLITK) cudaFuncSetAttribute(kern, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
         configured = 232448;
     }
     // Programmatic dependent launch (MUCU_PDL=0 disables): the kernel may start
@@ -543,15 +550,57 @@ int launch_t(Launch& L, cudaStream_t st, bool dry) {
     cfg.blockDim = dim3(kThreads);
     cfg.dynamicSmemBytes = (size_t)smem;
     cfg.stream = st;
-    cudaLaunchAttribute attr[1];
-    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    cudaLaunchAttribute attr[2];
+    int na = 0;
+    if (pdl) {
+        attr[na].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+        attr[na].val.programmaticStreamSerializationAllowed = 1;
+        ++na;
+    }
+    if (L.a.cl) {
+        attr[na].id = cudaLaunchAttributeClusterDimension;
+        attr[na].val.clusterDim.x = (unsigned)L.a.cl;
+        attr[na].val.clusterDim.y = 1;
+        attr[na].val.clusterDim.z = 1;
+        ++na;
+    }
     cfg.attrs = attr;
-    cfg.numAttrs = pdl ? 1 : 0;
+    cfg.numAttrs = na;
     cudaError_t le = cudaLaunchKernelEx(&cfg, kern, L.a, L.ta, L.tb);
     if (le) return (int)le;
     count_launch();
     return (int)cudaGetLastError();
+}
+
+// CTAs of ~200 KB shared memory that can be resident at once when launched in
+// clusters of cl (GPC packing; 0 = cluster size not launchable).  Cached.
+__global__ void cluster_probe_kernel() {}
+int cluster_capacity(int cl) {
+    static int cache[17] = {0};
+    if (cl <= 1) return g_num_sms;
+    if (cl > 16) return 0;
+    if (cache[cl]) return cache[cl] > 0 ? cache[cl] : 0;
+    const int sm = 200 * 1024;
+    cudaFuncSetAttribute(cluster_probe_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, sm);
+    cudaFuncSetAttribute(cluster_probe_kernel, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3((unsigned)(cl * 64));
+    cfg.blockDim = dim3(kThreads);
+    cfg.dynamicSmemBytes = sm;
+    cudaLaunchAttribute at;
+    at.id = cudaLaunchAttributeClusterDimension;
+    at.val.clusterDim.x = (unsigned)cl;
+    at.val.clusterDim.y = 1;
+    at.val.clusterDim.z = 1;
+    cfg.attrs = &at;
+    cfg.numAttrs = 1;
+    int n = 0;
+    if (cudaOccupancyMaxActiveClusters(&n, cluster_probe_kernel, &cfg) != cudaSuccess || n <= 0) {
+        cudaGetLastError();
+        n = 0;
+    }
+    cache[cl] = n > 0 ? n * cl : -1;
+    return n * cl;
 }
 
 void size_stages(TcArgs& a) {
@@ -713,7 +762,7 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
     // TMA-only operands (tma = true) also take 256-row tiles and stages of
     // km k-blocks: fewer, larger TMA transactions (the TMA issue rate, not
     // bytes, bounds these MN-major loads), as deep as two stages allow.
-    auto wgrad_tiling = [&](int step, bool tma, int qrow = 0, int km_max = 4) {
+    auto wgrad_tiling = [&](int step, bool tma, int qrow = 0, int km_max = 4, int batches = 1) {
         A.mt = (tma && A.M > 128 && (A.M <= 256 || A.M % 256 == 0 || (qrow && A.M % 256 > 128)) &&
                 env_int("MUCU_MT2", 1)) ? 2 : 1;
         // 256-row tiles keep BN <= 128 so that two stages of two k-blocks fit
@@ -735,29 +784,50 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
             if (const int km = env_int("MUCU_KM", 0)) A.km = km;
         }
         size_stages(A);
-        const int64_t tiles = ceil_div(A.N, A.BN) * ceil_div(A.M, 128 * A.mt);
+        const int64_t tiles = ceil_div(A.N, A.BN) * ceil_div(A.M, 128 * A.mt) * batches;
         // qrow > 0: k-blocks are KD-pixel pieces of output rows of qrow pixels (window WGRAD)
         if (qrow) A.win_qb = (int)ceil_div(qrow, KB * A.km);
         const int64_t nkb = qrow ? (int64_t)b * g.p * A.win_qb : ceil_div(A.kred, KB * A.km);
-        int64_t nsplit = std::min<int64_t>(std::min<int64_t>(std::max<int64_t>(1, (2LL * num_sms) / tiles),
-                                                             std::max<int64_t>(1, nkb / 16)), 65535);
-        {
-            // Wave-quantised split count: minimise waves x (stages per split + the
-            // per-split epilogue / pipeline fill, ~E stages of 128-B k-blocks),
-            // splits >= 4 stages each.  (Capping at 16 stages per split left e.g.
-            // ResNet-50 layer4 1x1 WGRAD at 192 units on 148 SMs.)
-            const double E = env_int("MUCU_SPLIT_E", 16) / (double)A.km;
-            double best = 1e30;
-            const int64_t smax = std::min<int64_t>(std::max<int64_t>(1, nkb / 4), std::min<int64_t>(65535, 4LL * num_sms));
-            for (int64_t sp = 1; sp <= smax; ++sp) {
-                const double cost = (double)ceil_div(tiles * sp, num_sms) * ((double)ceil_div(nkb, sp) + E);
-                if (cost < best - 1e-9) { best = cost; nsplit = sp; }
+        // Split of the pixel reduction (deterministic): S = cl * G CTAs per
+        // tile, clusters of cl reduce their partials through DSMEM and the G groups
+        // add into dw in a fixed order.  Cost in stages of km k-blocks: waves of the
+        // CTAs that fit at once (GPC packing of clusters) x (stages per split + E for
+        // pipeline fill and the epilogue) + R for the cluster reduction + L per
+        // ordered group hand-over.
+        const double E = env_int("MUCU_SPLIT_E", 16) / (double)A.km;
+        const double R = env_int("MUCU_CLUSTER_R", 4) / (double)A.km;
+        const double Lg = env_int("MUCU_CHAIN_L", 6) / (double)A.km;
+        int64_t best_s = 1;
+        int best_cl = 0;
+        double best = (double)ceil_div(tiles, num_sms) * ((double)nkb + E);
+        // tests: force a cluster size / number of ordered split groups
+        const int force_cl = env_int("MUCU_FORCE_CL", 0), force_g = env_int("MUCU_FORCE_G", 0);
+        for (int cl = 2; cl <= 16; cl *= 2) {
+            if (force_cl && cl != force_cl) continue;
+            const int cap = cluster_capacity(cl);
+            if (cap <= 0) continue;
+            for (int64_t G = 1;; ++G) {
+                const int64_t sp = cl * G;
+                if (sp > std::max<int64_t>(2, nkb / 2) || sp > 1024) break;
+                if (force_g && G != force_g) continue;
+                const double cost = (double)ceil_div(tiles * sp, cap) * ((double)ceil_div(nkb, sp) + E) + R +
+                                    (double)(G - 1) * Lg;
+                if (cost < best - 1e-9 || (force_cl && best_cl == 0)) { best = cost; best_s = sp; best_cl = cl; }
             }
         }
-        A.kb_per_split = (int)ceil_div(nkb, nsplit);
-        nsplit = ceil_div(nkb, A.kb_per_split);
         A.num_kb = (int)nkb;
-        grid2((int)nsplit);
+        A.kb_per_split = (int)ceil_div(nkb, best_s);
+        A.cl = best_s > 1 ? best_cl : 0;
+        A.zsplit = batches > 1 ? (int)best_s : 0;
+        if (A.cl) {
+            // one unit per CTA: grid = tiles x splits (a multiple of the cluster size)
+            A.num_z = (int)(batches * best_s);
+            A.stg_bytes = 128 * A.mt * (A.BN + 4) * 4;
+            L.grid = dim3((unsigned)(tiles * best_s));
+        } else {
+            A.stg_bytes = 0;
+            grid2(batches);
+        }
     };
     const bool Aok = (g.c % KB) == 0;  // vector gathers over C
     int err = 0;
@@ -807,6 +877,13 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
                 // the zero-padded filter staged once per CTA in shared memory.
                 A.cp = 16 / elt; A.s8 = (int)align_up((uint64_t)g.s, 8);
                 A.num_kb = g.r * (A.s8 / 8);
+                // The tap-group K layout (and with it the summation order) must not depend
+                // on the micro-batch size (invariant I1): one N tile of exactly K columns,
+                // whatever pick_bn's wave count would prefer at this b.
+                if (g.k <= 256) {
+                    A.BN = std::max(32, (int)align_up((uint64_t)g.k, 32));
+                    A.bn_atoms = (A.BN * elt + 127) / 128;
+                }
                 if (ceil_div(A.N, A.BN) == 1) {
                     A.b_bytes = 0;
                     A.bres_bytes = A.num_kb * A.BN * 128;
@@ -1005,10 +1082,9 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         if (err) return err;
         A.M = g.k; A.N = g.c; A.ldc = Cp; A.kred = (int)Tp; A.out = Mx; A.alpha = 1.f; A.beta = 0.f; A.out_bf16 = 0;
         A.batch_stride = (long long)Kp * Cp;
-        wgrad_tiling(16, true);
-        const int nsplit = A.num_z;
-        A.zsplit = nsplit; A.zrows = (int)Tp;
-        grid2(16 * nsplit);
+        wgrad_tiling(16, true, 0, 4, 16);
+        if (!A.zsplit) A.zsplit = 1;  // batch = z / zsplit (one split per batch)
+        A.zrows = (int)Tp;
         if (!map2(&L.ta, D, Kp, 16 * Tp, Kp, atom, KB * A.km, true)) return -1;
         if (!map2(&L.tb, V, Cp, 16 * Tp, Cp, atom, KB * A.km, true)) return -1;
         map_mn_box(V, Cp, 16 * Tp, Cp, KB * A.km);

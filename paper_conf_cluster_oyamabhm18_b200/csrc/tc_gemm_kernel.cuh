@@ -11,6 +11,37 @@
 // Two TMEM accumulators (2 x BN columns) let the epilogue of tile i overlap
 // the mainloop of tile i+1 (tmem_full / tmem_empty barriers).
 
+// dw element (offset from the batch's dw base) of BackwardFilter GEMM element
+// (row m, column n) for each split-K epilogue layout; -1 = padding (no element).
+template <int EPI, int ELT>
+__device__ __forceinline__ long long wgrad_dst(const TcArgs& p, int m, int n) {
+    if constexpr (EPI == EPI_WGRAD_CHAIN) {
+        return (long long)m * p.ldc + n;
+    } else if constexpr (EPI == EPI_WGRAD_SMALLC) {
+        // padded column j' = (r, s8, c') -> dw column (r*S + s)*C + c
+        const int c = n % p.cp, t2 = n / p.cp, s_ = t2 % p.s8, r = t2 / p.s8;
+        return (c < p.C && s_ < p.S) ? (long long)m * p.ldc + (r * p.S + s_) * p.C + c : -1;
+    } else if constexpr (EPI == EPI_WGRAD_S2D) {
+        // column (tap (d,e), channel (a, b, c)) -> dw[k][st*d+a][st*e+b][c]
+        const int stc = p.s2_st * p.s2_C, real = stc * p.s2_st;
+        const int tap = n / p.C, ch = n - tap * p.C;
+        if (ch >= real) return -1;
+        const int d = tap / p.S, e = tap - d * p.S;
+        const int a = ch / stc, rem = ch - a * stc, bq = rem / p.s2_C, c = rem - bq * p.s2_C;
+        const int r = p.s2_st * d + a, sx = p.s2_st * e + bq;
+        return (r < p.s2_R && sx < p.s2_S) ? (long long)m * p.ldc + (r * p.s2_S + sx) * p.s2_C + c : -1;
+    } else if constexpr (EPI == EPI_WGRAD_WIN) {
+        // row m = (r, atom aa, tap t, channel c) -> dw[k = n][r][aa*taps + t][c]
+        const int per_atom = p.win_aw / ELT;  // elements per A swizzle atom
+        const int ja = m / per_atom, e = m - ja * per_atom;
+        const int t = e / p.cp, c = e - t * p.cp;
+        const int r = ja / p.win_na, sx = (ja - r * p.win_na) * (per_atom / p.cp) + t;
+        return (r < p.R && sx < p.S && c < p.C) ? (long long)n * p.ldc + (r * p.S + sx) * p.C + c : -1;
+    } else {
+        return -1;
+    }
+}
+
 // dst[ofs[j] * stride] = alpha * v[j] + beta * dst[...] for the 32 accumulator
 // columns of one row (ofs < 0: skipped); all loads issue before the stores.
 // beta == 0 never reads dst (it may hold garbage / NaN).
@@ -66,7 +97,11 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
     // A_HALO: a ring of p.hstages halo tiles (p.halo_bytes each) replaces the A stages
     uint8_t* sB = smem + (HALO ? (size_t)p.hstages * p.halo_bytes : (size_t)S * A_BYTES);
     uint8_t* sBres = sB + (size_t)S * B_BYTES;  // B_RESIDENT: whole filter, k-block after k-block
-    uint64_t* bars = (uint64_t*)(sBres + (B_RES ? p.bres_bytes : 0));
+    // cluster split-K: the epilogue stages the partial tile over the operand ring, so
+    // the barriers sit past whichever region is larger
+    uint8_t* bar_base = sBres + (B_RES ? p.bres_bytes : 0);
+    if (smem + p.stg_bytes > bar_base) bar_base = smem + p.stg_bytes;
+    uint64_t* bars = (uint64_t*)bar_base;
     uint64_t* full = bars;
     uint64_t* empty = bars + S;
     uint64_t* tfull = bars + 2 * S;      // [2]
@@ -115,9 +150,24 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
     asm volatile("griddepcontrol.launch_dependents;" :::);
 
     // tile -> (m0, n0, z, k-block range)
+    // Cluster split-K (p.cl > 0, one unit per CTA): CTA `tile` is rank tile % cl of
+    // cluster c = tile / cl; cluster c = (split group g, batch, output tile), g
+    // slowest; split = g * cl + rank.
     auto decode = [&](int tile, int& m0, int& n0, int& z, int& kb_begin, int& kb_end) {
-        z = tile / per_z;
-        const int rem = tile - z * per_z;
+        int rem;
+        if (p.cl) {
+            const int rho = tile % p.cl, c = tile / p.cl;
+            const int nbatch = p.zsplit ? p.num_z / p.zsplit : 1;
+            const int nu = per_z * nbatch;
+            const int g = c / nu, u = c - g * nu;
+            const int batch = u / per_z;
+            rem = u - batch * per_z;
+            const int split = g * p.cl + rho;
+            z = p.zsplit ? batch * p.zsplit + split : split;
+        } else {
+            z = tile / per_z;
+            rem = tile - z * per_z;
+        }
         const int ntile = rem / mt;
         m0 = (rem - ntile * mt) * BMt;
         n0 = ntile * p.BN;
@@ -826,29 +876,45 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
         const int row = q4 * 32 + lane;
         int acc = 0;
         uint32_t aph = 0;
-        for (int tile = blockIdx.x; tile < total_tiles; tile += gridDim.x) {
+        if (SPLITK && p.cl) {
+            // Cluster split-K: stage alpha * partial (fp32) over the operand ring, row-major
+            // with a pitch of BN + 4 floats; the cluster reduces it after the barrier below.
+            int m0, n0, z, kb_begin, kb_end;
+            decode(blockIdx.x, m0, n0, z, kb_begin, kb_end);
+            mbar_wait(smem_u32(&tfull[0]), 0u);
+            tc_fence_after();
+            const uint32_t stg = smem_u32(smem);
+            const int pitch = p.BN + 4;
+            for (int hh = 0; hh < p.mt; ++hh) {
+                for (int c0 = 0; c0 < p.BN; c0 += 32) {
+                    uint32_t v[32];
+                    if (kb_end > kb_begin) {
+                        TMEM_LD32(tmem + (uint32_t)(hh * p.BN + c0) + ((uint32_t)(q4 * 32) << 16), v);
+                        asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+                    } else {
+#pragma unroll
+                        for (int j = 0; j < 32; ++j) v[j] = 0u;
+                    }
+                    const uint32_t dst = stg + (uint32_t)(((hh * 128 + row) * pitch + c0) * 4);
+#pragma unroll
+                    for (int j = 0; j < 32; j += 4)
+                        asm volatile("st.shared.v4.f32 [%0], {%1, %2, %3, %4};" ::"r"(dst + j * 4),
+                                     "f"(p.alpha * __uint_as_float(v[j])), "f"(p.alpha * __uint_as_float(v[j + 1])),
+                                     "f"(p.alpha * __uint_as_float(v[j + 2])), "f"(p.alpha * __uint_as_float(v[j + 3]))
+                                     : "memory");
+                }
+            }
+            tc_fence_before();
+        }
+        for (int tile = blockIdx.x; tile < total_tiles && !(SPLITK && p.cl); tile += gridDim.x) {
             int m0, n0, z, kb_begin, kb_end;
             decode(tile, m0, n0, z, kb_begin, kb_end);
             const bool has_acc = kb_end > kb_begin;
             mbar_wait(smem_u32(&tfull[acc]), aph);
             tc_fence_after();
-            // Split-K BackwardFilter, deterministic: split sp of this dw tile
-            // adds its partial after split sp-1 (turn counter), split 0 applies beta.
-            float bsplit = p.beta;
-            unsigned long long* turn = nullptr;
-            int sp = 0;
-            if constexpr (SPLITK) {
-                sp = p.zsplit ? z % p.zsplit : z;
-                bsplit = sp == 0 ? p.beta : 1.f;
-                if (p.turns) {
-                    const int batch = p.zsplit ? z / p.zsplit : 0;
-                    turn = p.turns + (size_t)batch * per_z + (tile - z * per_z);
-                    if (sp > 0) {
-                        if (threadIdx.x == 160) turn_wait(turn, turn_tag(p.epoch, sp - 1));
-                        asm volatile("bar.sync 1, 128;" ::: "memory");  // the 4 epilogue warps
-                    }
-                }
-            }
+            // BackwardFilter without a split (the whole reduction in this CTA):
+            // dw = alpha * acc + beta * dw.  Split reductions take the cluster path.
+            const float bsplit = p.beta;
             auto drain = [&](const int hh) {
             const int m = m0 + 128 * hh + row;
             // Output row of GEMM row m (phase mode scatters sub-grid rows back to dx).
@@ -1140,17 +1206,88 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
             }
             };  // drain one 128-row half
             for (int hh = 0; hh < p.mt; ++hh) drain(hh);
-            if constexpr (SPLITK) {
-                if (turn) {  // this split's writes are done: hand the tile to split sp + 1
-                    asm volatile("bar.sync 1, 128;" ::: "memory");
-                    if (threadIdx.x == 160) turn_post(turn, turn_tag(p.epoch, sp));
-                }
-            }
             // release this accumulator to the MMA warp
             tc_fence_before();
             __syncwarp();
             if (lane == 0) mbar_arrive(smem_u32(&tempty[acc]));
             if (++acc == p.nacc) { acc = 0; aph ^= 1u; }
+        }
+    }
+    if constexpr (SPLITK) {
+        if (p.cl) {
+            // Deterministic split-K reduction: every CTA of the
+            // cluster holds one split's alpha-scaled partial tile in shared memory; CTA
+            // rank rho sums rows [rho*rows_per, ...) of all cl partials over DSMEM in rank
+            // order and writes them to dw (split group 0 applies beta; later groups add
+            // in group order behind a turn counter per (tile, slab)).
+            asm volatile("barrier.cluster.arrive.release;\n\tbarrier.cluster.wait.acquire;" ::: "memory");
+            if (warp >= 5) {
+                const int ep = threadIdx.x - 160;
+                const int rho = blockIdx.x % p.cl, c = blockIdx.x / p.cl;
+                const int nbatch = p.zsplit ? p.num_z / p.zsplit : 1;
+                const int nu = per_z * nbatch;
+                const int g = c / nu, u = c - g * nu;
+                const int batch = u / per_z, rem = u - batch * per_z;
+                const int ntile = rem / mt;
+                const int m0 = (rem - ntile * mt) * BMt, n0 = ntile * p.BN;
+                const int rows_per = (BMt + p.cl - 1) / p.cl;
+                const int r0 = rho * rows_per, r1 = min(BMt, r0 + rows_per);
+                const int nq = p.BN / 4;
+                const int pitch = p.BN + 4;
+                const float bsplit = g == 0 ? p.beta : 1.f;
+                unsigned long long* turn =
+                    p.turns ? p.turns + ((size_t)(batch * per_z + rem) * p.cl + rho) : nullptr;
+                if (turn && g > 0) {
+                    if (ep == 0) turn_wait(turn, turn_tag(p.epoch, g - 1));
+                    asm volatile("bar.sync 1, 128;" ::: "memory");
+                }
+                const uint32_t stg = smem_u32(smem);
+                float* outF = (float*)p.out + (p.zsplit ? (size_t)batch * p.batch_stride : 0);
+                for (int idx = ep; idx < (r1 - r0) * nq; idx += 128) {
+                    const int rr = r0 + idx / nq, c4 = idx - (idx / nq) * nq;
+                    const int m = m0 + rr;
+                    if (m >= p.M) continue;
+                    const uint32_t a = stg + (uint32_t)((rr * pitch + c4 * 4) * 4);
+                    float sum[4] = {0.f, 0.f, 0.f, 0.f};
+                    for (int k = 0; k < p.cl; ++k) {
+                        uint32_t ra;
+                        asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(ra) : "r"(a), "r"(k));
+                        float q0, q1, q2, q3;
+                        asm volatile("ld.shared::cluster.v4.f32 {%0, %1, %2, %3}, [%4];"
+                                     : "=f"(q0), "=f"(q1), "=f"(q2), "=f"(q3) : "r"(ra) : "memory");
+                        sum[0] += q0; sum[1] += q1; sum[2] += q2; sum[3] += q3;
+                    }
+                    const int col0 = n0 + c4 * 4;
+                    long long off[4];
+#pragma unroll
+                    for (int j = 0; j < 4; ++j) off[j] = col0 + j < p.N ? wgrad_dst<EPI, ELT>(p, m, col0 + j) : -1;
+                    const bool vec = EPI == EPI_WGRAD_CHAIN && off[0] >= 0 && off[3] == off[0] + 3 &&
+                                     ((((uintptr_t)(outF + off[0])) & 15) == 0);
+                    if (vec) {
+                        float4* d = reinterpret_cast<float4*>(outF + off[0]);
+                        float4 o = make_float4(sum[0], sum[1], sum[2], sum[3]);
+                        if (bsplit != 0.f) {
+                            const float4 old = __ldcg(d);
+                            o.x += bsplit * old.x; o.y += bsplit * old.y; o.z += bsplit * old.z; o.w += bsplit * old.w;
+                        }
+                        *d = o;
+                    } else {
+#pragma unroll
+                        for (int j = 0; j < 4; ++j) {
+                            if (off[j] < 0) continue;
+                            float o = sum[j];
+                            if (bsplit != 0.f) o += bsplit * __ldcg(outF + off[j]);
+                            outF[off[j]] = o;
+                        }
+                    }
+                }
+                if (turn) {
+                    asm volatile("bar.sync 1, 128;" ::: "memory");
+                    if (ep == 0) turn_post(turn, turn_tag(p.epoch, g));
+                }
+            }
+            // partners may still be reading this CTA's staging
+            asm volatile("barrier.cluster.arrive.release;\n\tbarrier.cluster.wait.acquire;" ::: "memory");
         }
     }
     tc_fence_before();

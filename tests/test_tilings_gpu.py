@@ -72,3 +72,44 @@ def test_wgrad_alternative_loads_exact(name, math, env, monkeypatch):
     for algo in (mu.IMPLICIT_GEMM, mu.IM2COL_GEMM):
         got, _ = run_gpu(d, mu.BWD_FILTER, [(algo, shape[0])], x, w, dy)
         assert np.array_equal(got, ref), (name, algo)
+
+
+# Cluster split-K BackwardFilter (DSMEM reduction, ordered split groups): every
+# cluster size and a multi-group chain, forced on mid-size shapes with enough
+# k-blocks; integer data -> exact, random data -> bitwise reproducible.
+SPLITK_SHAPES = {
+    "3x3_c64": (16, 64, 28, 28, 64, 3, 3, 1, 1),
+    "3x3_k192": (8, 128, 14, 14, 192, 3, 3, 1, 1),
+    "1x1_k512": (16, 256, 14, 14, 512, 1, 1, 0, 1),
+    "11x11s4_c3": (8, 3, 99, 99, 64, 11, 11, 2, 4),
+    "7x7s2_c3": (8, 3, 64, 64, 64, 7, 7, 3, 2),
+}
+SPLITK_ENVS = {"cl2": {"MUCU_FORCE_CL": "2"}, "cl4": {"MUCU_FORCE_CL": "4"}, "cl8": {"MUCU_FORCE_CL": "8"},
+               "cl16": {"MUCU_FORCE_CL": "16"}, "cl2x3": {"MUCU_FORCE_CL": "2", "MUCU_FORCE_G": "3"},
+               "cl4x2": {"MUCU_FORCE_CL": "4", "MUCU_FORCE_G": "2"}}
+
+
+@pytest.mark.parametrize("env", list(SPLITK_ENVS))
+@pytest.mark.parametrize("math", [mu.MATH_TF32, mu.MATH_BF16], ids=["tf32", "bf16"])
+@pytest.mark.parametrize("name", list(SPLITK_SHAPES))
+def test_cluster_splitk_wgrad_exact(name, math, env, monkeypatch):
+    for k, v in SPLITK_ENVS[env].items():
+        monkeypatch.setenv(k, v)
+    shape = SPLITK_SHAPES[name]
+    d = mu.desc(*shape, math)
+    x, w, dy = conv_inputs(*shape, seed=31, kind="int", lo=-1, hi=1)
+    algos = [mu.IMPLICIT_GEMM, mu.IM2COL_GEMM] + ([mu.WINOGRAD] if shape[5] == 3 and shape[8] == 1 else [])
+    out0 = np.random.default_rng(5).integers(-2, 3, size=(shape[4], shape[5], shape[6], shape[1])).astype(np.float32)
+    for algo in algos:
+        ref = oracle_ref(shape, mu.BWD_FILTER, x, w, dy)
+        got, _ = run_gpu(d, mu.BWD_FILTER, [(algo, shape[0])], x, w, dy)
+        assert np.array_equal(got, ref), (name, algo)
+        # beta applied exactly once (split group 0), alpha on every partial
+        ref = oracle_ref(shape, mu.BWD_FILTER, x, w, dy, alpha=2.0, beta=-1.0, out0=out0)
+        got, _ = run_gpu(d, mu.BWD_FILTER, [(algo, shape[0])], x, w, dy, alpha=2.0, beta=-1.0, out0=out0)
+        assert np.array_equal(got, ref), (name, algo, "alpha/beta")
+    xr, wr, dyr = conv_inputs(*shape, seed=32, kind="normal")
+    for algo in algos:
+        a1, _ = run_gpu(d, mu.BWD_FILTER, [(algo, shape[0])], xr, wr, dyr)
+        a2, _ = run_gpu(d, mu.BWD_FILTER, [(algo, shape[0])], xr, wr, dyr)
+        assert np.array_equal(a1, a2), (name, algo, "reproducible")

@@ -789,19 +789,17 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         if (qrow) A.win_qb = (int)ceil_div(qrow, KB * A.km);
         const int64_t nkb = qrow ? (int64_t)b * g.p * A.win_qb : ceil_div(A.kred, KB * A.km);
         // Split of the pixel reduction (deterministic): S = cl * G CTAs per
-        // tile, clusters of cl reduce their partials through DSMEM and the G groups
-        // add into dw in a fixed order.  Cost in stages of km k-blocks: waves of the
-        // CTAs that fit at once (GPC packing of clusters) x (stages per split + E for
-        // pipeline fill and the epilogue) + R for the cluster reduction + L per
-        // ordered group hand-over.
+        // tile; clusters of cl reduce their partials through DSMEM (+R) and the G groups
+        // add into dw in a fixed order (+L per hand-over).  Cost in stages of km
+        // k-blocks: waves of the CTAs that fit at once (GPC packing of clusters) x
+        // (stages per split + E for pipeline fill and the epilogue).
         const double E = env_int("MUCU_SPLIT_E", 16) / (double)A.km;
-        const double R = env_int("MUCU_CLUSTER_R", 4) / (double)A.km;
-        const double Lg = env_int("MUCU_CHAIN_L", 6) / (double)A.km;
-        int64_t best_s = 1;
-        int best_cl = 0;
-        double best = (double)ceil_div(tiles, num_sms) * ((double)nkb + E);
-        // tests: force a cluster size / number of ordered split groups
-        const int force_cl = env_int("MUCU_FORCE_CL", 0), force_g = env_int("MUCU_FORCE_G", 0);
+        const double R = env_int("MUCU_CLUSTER_R", 6) / (double)A.km;
+        const double Lg = env_int("MUCU_CHAIN_L", 8) / (double)A.km;
+        const int force_cl = env_int("MUCU_FORCE_CL", 0), force_g = env_int("MUCU_FORCE_G", 0);  // tests
+        int64_t b_s = 1;
+        int b_cl = 0;
+        double best = force_cl ? 1e30 : (double)ceil_div(tiles, num_sms) * ((double)nkb + E);
         for (int cl = 2; cl <= 16; cl *= 2) {
             if (force_cl && cl != force_cl) continue;
             const int cap = cluster_capacity(cl);
@@ -812,18 +810,22 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
                 if (force_g && G != force_g) continue;
                 const double cost = (double)ceil_div(tiles * sp, cap) * ((double)ceil_div(nkb, sp) + E) + R +
                                     (double)(G - 1) * Lg;
-                if (cost < best - 1e-9 || (force_cl && best_cl == 0)) { best = cost; best_s = sp; best_cl = cl; }
+                if (cost < best - 1e-9) { best = cost; b_s = sp; b_cl = cl; }
             }
         }
         A.num_kb = (int)nkb;
-        A.kb_per_split = (int)ceil_div(nkb, best_s);
-        A.cl = best_s > 1 ? best_cl : 0;
-        A.zsplit = batches > 1 ? (int)best_s : 0;
+        A.kb_per_split = (int)ceil_div(nkb, b_s);
+        A.cl = b_s > 1 ? b_cl : 0;
+        if (env_int("MUCU_LOG_TILING", 0))
+            fprintf(stderr, "[mucu] wgrad M=%d N=%d mt=%d BN=%d km=%d tiles=%lld nkb=%lld -> S=%lld cl=%d cap=%d cost=%.1f\n",
+                    A.M, A.N, A.mt, A.BN, A.km, (long long)tiles, (long long)nkb, (long long)b_s, A.cl,
+                    A.cl ? cluster_capacity(A.cl) : num_sms, best);
+        A.zsplit = batches > 1 ? (int)b_s : 0;
         if (A.cl) {
             // one unit per CTA: grid = tiles x splits (a multiple of the cluster size)
-            A.num_z = (int)(batches * best_s);
+            A.num_z = (int)(batches * b_s);
             A.stg_bytes = 128 * A.mt * (A.BN + 4) * 4;
-            L.grid = dim3((unsigned)(tiles * best_s));
+            L.grid = dim3((unsigned)(tiles * b_s));
         } else {
             A.stg_bytes = 0;
             grid2(batches);

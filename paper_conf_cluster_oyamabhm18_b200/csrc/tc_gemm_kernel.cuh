@@ -1221,8 +1221,9 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
             // order and writes them to dw (split group 0 applies beta; later groups add
             // in group order behind a turn counter per (tile, slab)).
             asm volatile("barrier.cluster.arrive.release;\n\tbarrier.cluster.wait.acquire;" ::: "memory");
-            if (warp >= 5) {
-                const int ep = threadIdx.x - 160;
+            {
+                // all 288 threads of the CTA share its slab (the mainloop is over)
+                const int ep = threadIdx.x;
                 const int rho = blockIdx.x % p.cl, c = blockIdx.x / p.cl;
                 const int nbatch = p.zsplit ? p.num_z / p.zsplit : 1;
                 const int nu = per_z * nbatch;
@@ -1237,52 +1238,102 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                 const float bsplit = g == 0 ? p.beta : 1.f;
                 unsigned long long* turn =
                     p.turns ? p.turns + ((size_t)(batch * per_z + rem) * p.cl + rho) : nullptr;
-                if (turn && g > 0) {
-                    if (ep == 0) turn_wait(turn, turn_tag(p.epoch, g - 1));
-                    asm volatile("bar.sync 1, 128;" ::: "memory");
-                }
                 const uint32_t stg = smem_u32(smem);
                 float* outF = (float*)p.out + (p.zsplit ? (size_t)batch * p.batch_stride : 0);
-                for (int idx = ep; idx < (r1 - r0) * nq; idx += 128) {
-                    const int rr = r0 + idx / nq, c4 = idx - (idx / nq) * nq;
-                    const int m = m0 + rr;
-                    if (m >= p.M) continue;
-                    const uint32_t a = stg + (uint32_t)((rr * pitch + c4 * 4) * 4);
-                    float sum[4] = {0.f, 0.f, 0.f, 0.f};
+                // thread -> (column quad c4, row phase rsub): one division per thread
+                const int tpr = kThreads / nq;  // rows in flight per pass
+                const bool active = ep < tpr * nq;
+                const int c4 = ep % nq, rsub = ep / nq;
+                const int col0 = n0 + 4 * c4;
+                uint32_t part[16];  // this slab position in every partner's shared memory
+#pragma unroll
+                for (int k = 0; k < 16; ++k) {
+                    part[k] = 0;
+                    if (k < p.cl) asm("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(part[k]) : "r"(stg), "r"(k));
+                }
+                constexpr int U = 8;  // rows per thread per batch (loads in flight)
+                // this split group's turn: groups add into dw in order
+                if (turn && g > 0) {
+                    if (ep == 0) turn_wait(turn, turn_tag(p.epoch, g - 1));
+                    __syncthreads();
+                }
+                for (int rb = r0 + rsub; rb < r1; rb += U * tpr) {
+                    // 1. the cluster's partials of these rows, summed in rank order (a fixed
+                    //    order: deterministic)
+                    float4 sum[U];
+#pragma unroll
+                    for (int uu = 0; uu < U; ++uu) sum[uu] = make_float4(0.f, 0.f, 0.f, 0.f);
                     for (int k = 0; k < p.cl; ++k) {
-                        uint32_t ra;
-                        asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(ra) : "r"(a), "r"(k));
-                        float q0, q1, q2, q3;
-                        asm volatile("ld.shared::cluster.v4.f32 {%0, %1, %2, %3}, [%4];"
-                                     : "=f"(q0), "=f"(q1), "=f"(q2), "=f"(q3) : "r"(ra) : "memory");
-                        sum[0] += q0; sum[1] += q1; sum[2] += q2; sum[3] += q3;
-                    }
-                    const int col0 = n0 + c4 * 4;
-                    long long off[4];
 #pragma unroll
-                    for (int j = 0; j < 4; ++j) off[j] = col0 + j < p.N ? wgrad_dst<EPI, ELT>(p, m, col0 + j) : -1;
-                    const bool vec = EPI == EPI_WGRAD_CHAIN && off[0] >= 0 && off[3] == off[0] + 3 &&
-                                     ((((uintptr_t)(outF + off[0])) & 15) == 0);
-                    if (vec) {
-                        float4* d = reinterpret_cast<float4*>(outF + off[0]);
-                        float4 o = make_float4(sum[0], sum[1], sum[2], sum[3]);
-                        if (bsplit != 0.f) {
-                            const float4 old = __ldcg(d);
-                            o.x += bsplit * old.x; o.y += bsplit * old.y; o.z += bsplit * old.z; o.w += bsplit * old.w;
+                        for (int uu = 0; uu < U; ++uu) {
+                            const int rr = rb + uu * tpr;
+                            if (!active || rr >= r1) continue;
+                            float q0, q1, q2, q3;
+                            asm volatile("ld.shared::cluster.v4.f32 {%0, %1, %2, %3}, [%4];"
+                                         : "=f"(q0), "=f"(q1), "=f"(q2), "=f"(q3)
+                                         : "r"(part[k] + (uint32_t)((rr * pitch + 4 * c4) * 4)));
+                            sum[uu].x += q0; sum[uu].y += q1; sum[uu].z += q2; sum[uu].w += q3;
                         }
-                        *d = o;
-                    } else {
+                    }
+                    // 2. dw = sum + bsplit * dw: all loads of the batch, then the stores
+                    if (active) {
+                        if constexpr (EPI == EPI_WGRAD_CHAIN) {
+                            const bool vec = col0 + 3 < p.N && (p.ldc & 3) == 0 && ((((uintptr_t)outF) & 15) == 0);
+                            float4 old[U];
 #pragma unroll
-                        for (int j = 0; j < 4; ++j) {
-                            if (off[j] < 0) continue;
-                            float o = sum[j];
-                            if (bsplit != 0.f) o += bsplit * __ldcg(outF + off[j]);
-                            outF[off[j]] = o;
+                            for (int uu = 0; uu < U; ++uu) {
+                                const int rr = rb + uu * tpr;
+                                old[uu] = make_float4(0.f, 0.f, 0.f, 0.f);
+                                if (rr >= r1 || m0 + rr >= p.M || bsplit == 0.f) continue;
+                                const float* d = outF + (size_t)(m0 + rr) * p.ldc + col0;
+                                if (vec) {
+                                    old[uu] = __ldcg(reinterpret_cast<const float4*>(d));
+                                } else {
+                                    old[uu].x = col0 < p.N ? __ldcg(d) : 0.f;
+                                    old[uu].y = col0 + 1 < p.N ? __ldcg(d + 1) : 0.f;
+                                    old[uu].z = col0 + 2 < p.N ? __ldcg(d + 2) : 0.f;
+                                    old[uu].w = col0 + 3 < p.N ? __ldcg(d + 3) : 0.f;
+                                }
+                            }
+#pragma unroll
+                            for (int uu = 0; uu < U; ++uu) {
+                                const int rr = rb + uu * tpr;
+                                if (rr >= r1 || m0 + rr >= p.M) continue;
+                                float* d = outF + (size_t)(m0 + rr) * p.ldc + col0;
+                                const float4 o = make_float4(sum[uu].x + bsplit * old[uu].x, sum[uu].y + bsplit * old[uu].y,
+                                                             sum[uu].z + bsplit * old[uu].z, sum[uu].w + bsplit * old[uu].w);
+                                if (vec) {
+                                    *reinterpret_cast<float4*>(d) = o;
+                                } else {
+                                    if (col0 < p.N) d[0] = o.x;
+                                    if (col0 + 1 < p.N) d[1] = o.y;
+                                    if (col0 + 2 < p.N) d[2] = o.z;
+                                    if (col0 + 3 < p.N) d[3] = o.w;
+                                }
+                            }
+                        } else {
+                            // scattered layouts (small-C, space-to-depth, window): per element
+#pragma unroll
+                            for (int uu = 0; uu < U; ++uu) {
+                                const int rr = rb + uu * tpr;
+                                if (rr >= r1 || m0 + rr >= p.M) continue;
+                                const float sv[4] = {sum[uu].x, sum[uu].y, sum[uu].z, sum[uu].w};
+                                long long o[4];
+                                float ov[4];
+#pragma unroll
+                                for (int j = 0; j < 4; ++j) {
+                                    o[j] = col0 + j < p.N ? wgrad_dst<EPI, ELT>(p, m0 + rr, col0 + j) : -1;
+                                    ov[j] = (bsplit != 0.f && o[j] >= 0) ? __ldcg(outF + o[j]) : 0.f;
+                                }
+#pragma unroll
+                                for (int j = 0; j < 4; ++j)
+                                    if (o[j] >= 0) outF[o[j]] = sv[j] + bsplit * ov[j];
+                            }
                         }
                     }
                 }
                 if (turn) {
-                    asm volatile("bar.sync 1, 128;" ::: "memory");
+                    __syncthreads();
                     if (ep == 0) turn_post(turn, turn_tag(p.epoch, g));
                 }
             }

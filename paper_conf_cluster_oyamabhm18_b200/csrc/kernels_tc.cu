@@ -210,6 +210,9 @@ enum AMode : int {
     A_TMA_WIN32 = 14,
     A_TMA_WIN = 11,    // WGRAD window operand, MN-major: rows j = (r, atom, tap, c) of the filter, K = pixels;
                        // one 4-D TMA box per 128-B atom from the overlapping-window view of the padded x
+    A_STAGED_WG = 15,  // WGRAD of small-C strided layers, zero workspace: the R x rows a block of KD output
+                       // pixels reads are staged by one TMA box; builders write the exact-tap (r,s,c) MN-major
+                       // operand from them
 };
 enum BMode : int {
     B_TMA_K2 = 0,      // dense K-major {K, cols}
@@ -231,8 +234,9 @@ enum BMode : int {
 // EPI_WGRAD_S2D: column (d, e, (a, b, c')) of the space-to-depth filter ->
 //   dw[k][st*d + a][st*e + b][c'] (padding and r >= R / s >= S skipped), reduced.
 // EPI_WGRAD_WIN: row j = (r, atom, tap, c) of the window GEMM -> dw[k][r][atom*taps + tap][c], reduced.
+// EPI_WGRAD_TAPS: row m = exact tap (r, s, c) -> dw[k][m] (A_STAGED_WG), reduced.
 enum EpiMode : int { EPI_STORE = 0, EPI_WGRAD_CHAIN = 1, EPI_WGRAD_SMALLC = 2, EPI_D2S = 3, EPI_WGRAD_S2D = 4,
-                     EPI_WGRAD_WIN = 5 };
+                     EPI_WGRAD_WIN = 5, EPI_WGRAD_TAPS = 6 };
 
 struct TcArgs {
     int M, N;                // output rows / cols
@@ -302,6 +306,9 @@ struct TcArgs {
     // through DSMEM; split groups of cl are ordered by turn counters (turns.cu), one
     // per (batch, tile, row slab).  stg_bytes: the epilogue's staging over the ring.
     int cl, stg_bytes;
+    // A_STAGED_WG: x-row chunks of sx_cs elements (sx_sr = elements per staged row), sx_stages
+    // stages of sx_bytes (sx_tx delivered by TMA), kred_taps = R*S*C GEMM rows
+    int sx_cs, sx_sr, sx_stages, sx_bytes, sx_tx, kred_taps;
     unsigned long long* turns;
     unsigned long long epoch;
 };
@@ -382,7 +389,8 @@ EncodeTiledFn get_encode() {
 bool make_map(CUtensorMap* tm, int elt, const void* base, int rank, const uint64_t* dims, const uint64_t* strides_bytes,
               const uint32_t* box, bool mn_major = false, int swz = 128) {
     // 32-bit MN-major operands need the 32-B-atom swizzle matching SWIZZLE_128B_BASE32B.
-    const CUtensorMapSwizzle sw = (mn_major && elt == 4) ? CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B
+    const CUtensorMapSwizzle sw = swz == 0                 ? CU_TENSOR_MAP_SWIZZLE_NONE
+                                  : (mn_major && elt == 4) ? CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B
                                   : swz == 64                ? CU_TENSOR_MAP_SWIZZLE_64B
                                   : swz == 32                ? CU_TENSOR_MAP_SWIZZLE_32B
                                                              : CU_TENSOR_MAP_SWIZZLE_128B;
@@ -513,10 +521,11 @@ int launch_t(Launch& L, cudaStream_t st, bool dry) {
     }
     const int a_stage = AM == A_HALO ? 0 : L.a.mt * 128 * 128;
     const int ring = L.a.hstages * L.a.halo_bytes + L.a.stages * L.a.km * (a_stage + L.a.b_bytes) + L.a.bres_bytes;
-    const int smem = 1024 + std::max(ring, L.a.stg_bytes) + (2 * L.a.stages + 6 + 2 * L.a.hstages) * 8 + 64;
+    const int smem =
+        1024 + std::max(ring, L.a.stg_bytes) + (2 * L.a.stages + 6 + 2 * L.a.hstages + 2 * L.a.sx_stages) * 8 + 64;
     if (smem > 232448) return -1;
     constexpr bool SPLITK = (EPI == EPI_WGRAD_CHAIN || EPI == EPI_WGRAD_SMALLC || EPI == EPI_WGRAD_S2D ||
-                             EPI == EPI_WGRAD_WIN);
+                             EPI == EPI_WGRAD_WIN || EPI == EPI_WGRAD_TAPS);
     if (!SPLITK && L.a.cl) return -1;
     L.a.turns = nullptr;
     L.a.epoch = 0;
@@ -762,32 +771,8 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
     // TMA-only operands (tma = true) also take 256-row tiles and stages of
     // km k-blocks: fewer, larger TMA transactions (the TMA issue rate, not
     // bytes, bounds these MN-major loads), as deep as two stages allow.
-    auto wgrad_tiling = [&](int step, bool tma, int qrow = 0, int km_max = 4, int batches = 1) {
-        A.mt = (tma && A.M > 128 && (A.M <= 256 || A.M % 256 == 0 || (qrow && A.M % 256 > 128)) &&
-                env_int("MUCU_MT2", 1)) ? 2 : 1;
-        // 256-row tiles keep BN <= 128 so that two stages of two k-blocks fit
-        // (measured: km = 2 beats BN = 256 with km = 1 on every AlexNet/ResNet layer)
-        A.BN = pick_bn(A.N, step, 128 * A.mt, A.mt == 2 ? std::max(128, step) : 256);
-        if (const int fb = env_int("MUCU_FORCE_BN", 0)) A.BN = std::max(std::max(step, 32), fb - fb % step);
-        A.bn_atoms = (A.BN * elt + 127) / 128;
-        A.b_bytes = std::max(A.BN * 128, A.bn_atoms * (128 / elt) * 128);
-        A.km = 1;
-        if (tma) {
-            const int base = A.mt * 128 * 128 + A.b_bytes;
-            while (A.km < km_max && 2 * (2 * A.km) * base <= 200 * 1024 && KB * 2 * A.km <= 256 &&
-                   (qrow == 0 || KB * 2 * A.km <= (int)align_up((uint64_t)qrow, (uint64_t)KB)))
-                A.km *= 2;
-            // window operand (qrow > 0), BF16: 64-pixel k-blocks already make large boxes;
-            // km = 1 keeps 5 ring stages instead of 2 (ResNet conv1 WGRAD -6 %; TF32's
-            // 32-pixel blocks need km = 2)
-            if (qrow && elt == 2 && env_int("MUCU_WIN_KM1", 1)) A.km = 1;
-            if (const int km = env_int("MUCU_KM", 0)) A.km = km;
-        }
-        size_stages(A);
-        const int64_t tiles = ceil_div(A.N, A.BN) * ceil_div(A.M, 128 * A.mt) * batches;
-        // qrow > 0: k-blocks are KD-pixel pieces of output rows of qrow pixels (window WGRAD)
-        if (qrow) A.win_qb = (int)ceil_div(qrow, KB * A.km);
-        const int64_t nkb = qrow ? (int64_t)b * g.p * A.win_qb : ceil_div(A.kred, KB * A.km);
+    // Split of a BackwardFilter reduction of nkb stages over `tiles` output tiles.
+    auto apply_split = [&](int64_t tiles, int64_t nkb, int batches) {
         // Split of the pixel reduction (deterministic): S = cl * G CTAs per
         // tile; clusters of cl reduce their partials through DSMEM (+R) and the G groups
         // add into dw in a fixed order (+L per hand-over).  Cost in stages of km
@@ -830,6 +815,34 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
             A.stg_bytes = 0;
             grid2(batches);
         }
+    };
+    auto wgrad_tiling = [&](int step, bool tma, int qrow = 0, int km_max = 4, int batches = 1) {
+        A.mt = (tma && A.M > 128 && (A.M <= 256 || A.M % 256 == 0 || (qrow && A.M % 256 > 128)) &&
+                env_int("MUCU_MT2", 1)) ? 2 : 1;
+        // 256-row tiles keep BN <= 128 so that two stages of two k-blocks fit
+        // (measured: km = 2 beats BN = 256 with km = 1 on every AlexNet/ResNet layer)
+        A.BN = pick_bn(A.N, step, 128 * A.mt, A.mt == 2 ? std::max(128, step) : 256);
+        if (const int fb = env_int("MUCU_FORCE_BN", 0)) A.BN = std::max(std::max(step, 32), fb - fb % step);
+        A.bn_atoms = (A.BN * elt + 127) / 128;
+        A.b_bytes = std::max(A.BN * 128, A.bn_atoms * (128 / elt) * 128);
+        A.km = 1;
+        if (tma) {
+            const int base = A.mt * 128 * 128 + A.b_bytes;
+            while (A.km < km_max && 2 * (2 * A.km) * base <= 200 * 1024 && KB * 2 * A.km <= 256 &&
+                   (qrow == 0 || KB * 2 * A.km <= (int)align_up((uint64_t)qrow, (uint64_t)KB)))
+                A.km *= 2;
+            // window operand (qrow > 0), BF16: 64-pixel k-blocks already make large boxes;
+            // km = 1 keeps 5 ring stages instead of 2 (ResNet conv1 WGRAD -6 %; TF32's
+            // 32-pixel blocks need km = 2)
+            if (qrow && elt == 2 && env_int("MUCU_WIN_KM1", 1)) A.km = 1;
+            if (const int km = env_int("MUCU_KM", 0)) A.km = km;
+        }
+        size_stages(A);
+        const int64_t tiles = ceil_div(A.N, A.BN) * ceil_div(A.M, 128 * A.mt) * batches;
+        // qrow > 0: k-blocks are KD-pixel pieces of output rows of qrow pixels (window WGRAD)
+        if (qrow) A.win_qb = (int)ceil_div(qrow, KB * A.km);
+        const int64_t nkb = qrow ? (int64_t)b * g.p * A.win_qb : ceil_div(A.kred, KB * A.km);
+        apply_split(tiles, nkb, batches);
     };
     const bool Aok = (g.c % KB) == 0;  // vector gathers over C
     int err = 0;
@@ -1326,6 +1339,50 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
             }
             return map2(&L.ta, in1, g.k, (uint64_t)Mpix, g.k, atom, KB * A.km, true);
         };
+        if (algo == MUCU_ALGO_IMPLICIT_GEMM && small_c_tc(g) && env_int("MUCU_STAGED", 1)) {
+            // Staged-row BackwardFilter, zero workspace: GEMM rows = the
+            // exact R*S*C taps (no padding but to 128 rows), columns = the K filters,
+            // reduction = output pixels in blocks of KD of one output row.
+            const int TR = (int)align_up((uint64_t)RSC, 128);
+            const int mtS = TR / 128;
+            const int WC = g.w * g.c;
+            const int span = (g.stride * (KB - 1) + g.s) * g.c;  // elements a block reads per x row
+            int cs = 0, bch = 0;
+            for (int c = 256; c >= 1; --c) {
+                if (WC % c || (c * elt) % 16) continue;
+                const int bc = (span + 2 * (c - 1)) / c;  // any start offset inside a chunk
+                if (!cs || (int64_t)bc * c < (int64_t)bch * cs) { cs = c; bch = bc; }
+            }
+            const int b_bytes_s = std::max(g.k * 128, (g.k * elt / 128) * KB * 128);
+            const int sx_tx = g.r * bch * cs * elt;
+            const int sx_bytes = (int)align_up((uint64_t)sx_tx, 1024);
+            const int tabb = (int)align_up((uint64_t)TR * 4, 1024);
+            const int stage = mtS * 16384 + b_bytes_s;
+            int Ss = 0, SX = 0;
+            for (int sa : {3, 2})
+                for (int sx : {4, 3, 2})
+                    if (!Ss && sa * stage + sx * sx_bytes + tabb <= 205 * 1024) { Ss = sa; SX = sx; }
+            if (mtS <= 4 && g.k <= 256 && g.k % atom == 0 && cs > 0 && g.r <= 256 && bch <= 256 && Ss &&
+                128 * mtS * (g.k + 4) * 4 <= 210 * 1024) {
+                A.M = (int)RSC; A.N = g.k; A.ldc = (int)RSC; A.kred_taps = (int)RSC; A.mt = mtS; A.BN = g.k;
+                A.bn_atoms = g.k * elt / 128; A.b_bytes = b_bytes_s; A.km = 1;
+                A.win_qb = (int)ceil_div(g.q, KB);
+                A.sx_cs = cs; A.sx_sr = bch * cs; A.sx_tx = sx_tx; A.sx_bytes = sx_bytes;
+                A.stages = Ss; A.sx_stages = SX; A.bres_bytes = SX * sx_bytes + tabb;
+                A.nacc = mtS * A.BN <= 256 ? 2 : 1;
+                const int cols = A.nacc * mtS * A.BN;
+                A.tmem_cols = cols <= 64 ? 64 : cols <= 128 ? 128 : cols <= 256 ? 256 : 512;
+                apply_split(1, (int64_t)b * g.p * A.win_qb, 1);
+                uint64_t dims[4] = {(uint64_t)cs, (uint64_t)(WC / cs), (uint64_t)g.h, (uint64_t)b};
+                uint64_t str[3] = {(uint64_t)cs * elt, (uint64_t)WC * elt, (uint64_t)g.h * WC * elt};
+                uint32_t box[4] = {(uint32_t)cs, (uint32_t)bch, (uint32_t)g.r, 1};
+                if (!make_map(&L.ta, elt, in0, 4, dims, str, box, false, 0)) return -1;
+                if (!map3(&L.tb, in1, g.k, g.q, (uint64_t)b * g.p, g.k, (uint64_t)g.q * g.k, atom, KB, 1, true))
+                    return -1;
+                A.tma_bytes = A.bn_atoms * KB * 128;
+                return LAUNCH(A_STAGED_WG, B_TMA_DYROW, EPI_WGRAD_TAPS);
+            }
+        }
         if (algo == MUCU_ALGO_IM2COL_GEMM && small_c_tc(g)) {
             // RGB-like layer: channel-padded copy of x, padded columns j' = (r, s8, c').
             err = DRY(launch_pad_channels(g, b, in0, ws + WL.a_off, st));

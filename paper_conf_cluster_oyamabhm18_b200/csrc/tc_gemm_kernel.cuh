@@ -30,6 +30,8 @@ __device__ __forceinline__ long long wgrad_dst(const TcArgs& p, int m, int n) {
         const int a = ch / stc, rem = ch - a * stc, bq = rem / p.s2_C, c = rem - bq * p.s2_C;
         const int r = p.s2_st * d + a, sx = p.s2_st * e + bq;
         return (r < p.s2_R && sx < p.s2_S) ? (long long)m * p.ldc + (r * p.s2_S + sx) * p.s2_C + c : -1;
+    } else if constexpr (EPI == EPI_WGRAD_TAPS) {
+        return m < p.kred_taps ? (long long)n * p.ldc + m : -1;
     } else if constexpr (EPI == EPI_WGRAD_WIN) {
         // row m = (r, atom aa, tap t, channel c) -> dw[k = n][r][aa*taps + t][c]
         const int per_atom = p.win_aw / ELT;  // elements per A swizzle atom
@@ -70,7 +72,11 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
     const int KD = KB * p.km;                // K rows per stage (MN-major modes)
     constexpr bool WIN = (AM == A_TMA_WIN || AM == A_TMA_WIN64 || AM == A_TMA_WIN32);
     constexpr uint32_t WAW = AM == A_TMA_WIN64 ? 64u : AM == A_TMA_WIN32 ? 32u : 128u;  // window atom bytes
-    constexpr bool A_MN = (AM == A_TMA_MN2 || WIN);
+    // A_STAGED_WG: small-C strided BackwardFilter, zero workspace: x rows staged by TMA,
+    // the exact-tap MN-major A operand (rows = (r,s,c), K = output pixels) built in
+    // shared memory by 256 builder threads (warps 0-3 and 5-8)
+    constexpr bool STAGED = (AM == A_STAGED_WG);
+    constexpr bool A_MN = (AM == A_TMA_MN2 || WIN || STAGED);
     constexpr bool B_MN = (BM_ == B_TMA_MN2 || BM_ == B_TMA_MN3 || BM_ == B_GATHER_WG || BM_ == B_SCALAR_DGRAD ||
                            BM_ == B_SCALAR_WG || BM_ == B_TMA_IM2COL || BM_ == B_GATHER_SMALLC ||
                            BM_ == B_GATHER_SMALLC_PAD || BM_ == B_TMA_DYROW);
@@ -81,7 +87,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
     constexpr bool B_RES = (BM_ == B_RESIDENT);
     constexpr bool GATHER = !A_TMA || (!B_TMA && !B_RES);
     constexpr bool SPLITK = (EPI == EPI_WGRAD_CHAIN || EPI == EPI_WGRAD_SMALLC || EPI == EPI_WGRAD_S2D ||
-                             EPI == EPI_WGRAD_WIN);
+                             EPI == EPI_WGRAD_WIN || EPI == EPI_WGRAD_TAPS);
     constexpr bool A_ASYNC = (AM == A_GATHER_FWD || AM == A_GATHER_DGRAD || AM == A_GATHER_SMALLC_PAD);
     constexpr bool B_ASYNC = (BM_ == B_GATHER_WG || BM_ == B_GATHER_SMALLC_PAD);
     // MN-major atoms: 8-row (bf16, SWIZZLE_128B) or 4-row (tf32, 128B_BASE32B) groups.
@@ -99,7 +105,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
     uint8_t* sBres = sB + (size_t)S * B_BYTES;  // B_RESIDENT: whole filter, k-block after k-block
     // cluster split-K: the epilogue stages the partial tile over the operand ring, so
     // the barriers sit past whichever region is larger
-    uint8_t* bar_base = sBres + (B_RES ? p.bres_bytes : 0);
+    uint8_t* bar_base = sBres + p.bres_bytes;  // B_RESIDENT filter / A_STAGED_WG x ring + tap table
     if (smem + p.stg_bytes > bar_base) bar_base = smem + p.stg_bytes;
     uint64_t* bars = (uint64_t*)bar_base;
     uint64_t* full = bars;
@@ -110,6 +116,8 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
     uint32_t* tmem_slot = (uint32_t*)(bars + 2 * S + 5);
     uint64_t* hfull = bars + 2 * S + 6;             // [hstages] halo ring
     uint64_t* hempty = bars + 2 * S + 6 + p.hstages;
+    uint64_t* xfull = bars + 2 * S + 6 + 2 * p.hstages;               // [sx_stages] staged x rows
+    uint64_t* xempty = bars + 2 * S + 6 + 2 * p.hstages + p.sx_stages;
 
     const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
     const int BMt = 128 * p.mt;  // tile rows: 128, or 256 as two 128-row halves with separate accumulators
@@ -118,7 +126,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
     const int total_tiles = per_z * p.num_z;
 
     if (threadIdx.x == 0) {
-        const uint32_t full_count = (GATHER ? 128u : 0u) + (A_TMA || B_TMA ? 1u : 0u);
+        const uint32_t full_count = STAGED ? 257u : (GATHER ? 128u : 0u) + (A_TMA || B_TMA ? 1u : 0u);
         for (int s = 0; s < S; ++s) {
             mbar_init(smem_u32(&full[s]), full_count);
             mbar_init(smem_u32(&empty[s]), 1);
@@ -131,6 +139,10 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
         for (int h = 0; h < p.hstages; ++h) {
             mbar_init(smem_u32(&hfull[h]), 1);
             mbar_init(smem_u32(&hempty[h]), 1);
+        }
+        for (int j = 0; j < p.sx_stages; ++j) {
+            mbar_init(smem_u32(&xfull[j]), 1);
+            mbar_init(smem_u32(&xempty[j]), 256);
         }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
@@ -180,7 +192,111 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
         }
     };
 
-    if (HALO && warp < 4) {
+    if constexpr (STAGED) {
+        if (warp != 4) {
+            // ================= staged-row builders (A_STAGED_WG) =================
+            // k-block kb = KD output pixels (n, p, q0 .. q0+KD-1) of output row n*P + p;
+            // x rows st*p + r - pad (r < R), elements [chunk0*cs, (chunk0 + bch)*cs) of
+            // each row (zero outside the image) land in an x stage by one TMA box; GEMM
+            // row m = (r, s, c) of pixel q reads staged[r][tab(m) + col0 + st*C*(q - q0)].
+            const int bt = warp < 4 ? threadIdx.x : threadIdx.x - 32;  // 0..255
+            const T* xs_base = (const T*)sBres;
+            int* tab = (int*)(sBres + (size_t)p.sx_stages * p.sx_bytes);
+            const int TR = 128 * p.mt;
+            const int SC = p.S * p.C;
+            for (int m = bt; m < TR; m += 256) tab[m] = m < p.kred_taps ? (m / SC) * p.sx_sr + m % SC : -1;
+            asm volatile("bar.sync 2, 256;" ::: "memory");
+            constexpr int EPC = 16 / ELT;             // elements per 16-B chunk
+            const int CH = TR / EPC;                  // chunks per A K-row (pixel)
+            const int stC = p.stride * p.C;
+            auto x_coords = [&](int kb, int& cq0, int& chunk0, int& h0, int& n_, int& col0, int& valid) {
+                const int row = kb / p.win_qb, qb = kb - row * p.win_qb;
+                n_ = row / p.P;
+                const int pp = row - n_ * p.P;
+                cq0 = qb * KD;
+                h0 = p.stride * pp - p.pad;
+                const int e0 = (p.stride * cq0 - p.pad) * p.C;
+                chunk0 = e0 >= 0 ? e0 / p.sx_cs : -((-e0 + p.sx_cs - 1) / p.sx_cs);
+                col0 = e0 - chunk0 * p.sx_cs;
+                valid = min(KD, p.Q - cq0);
+            };
+            auto x_issue = [&](int kb, int jx) {
+                int cq0, chunk0, h0, n_, col0, valid;
+                x_coords(kb, cq0, chunk0, h0, n_, col0, valid);
+                const uint32_t fb = smem_u32(&xfull[jx]);
+                mbar_arrive_tx(fb, (uint32_t)p.sx_tx);
+                tma_load_4d(smem_u32(sBres + (size_t)jx * p.sx_bytes), &tmA, fb, 0, chunk0, h0, n_);
+            };
+            int ai = 0, xi = 0;
+            for (int tile = blockIdx.x; tile < total_tiles; tile += gridDim.x) {
+                int m0, n0, z, kb_begin, kb_end;
+                decode(tile, m0, n0, z, kb_begin, kb_end);
+                const int nk = kb_end - kb_begin;
+                if (bt == 0)
+                    for (int j = 0; j < min(p.sx_stages, nk); ++j) x_issue(kb_begin + j, (xi + j) % p.sx_stages);
+                for (int i = 0; i < nk; ++i, ++ai, ++xi) {
+                    const int kb = kb_begin + i;
+                    const int s = ai % S, jx = xi % p.sx_stages;
+                    const uint32_t aph = (uint32_t)((ai / S) & 1), xph = (uint32_t)((xi / p.sx_stages) & 1);
+                    mbar_wait(smem_u32(&empty[s]), aph ^ 1u);
+                    int cq0, chunk0, h0, n_, col0, valid;
+                    x_coords(kb, cq0, chunk0, h0, n_, col0, valid);
+                    const uint32_t aT = smem_u32(sA + (size_t)s * A_BYTES);
+                    if (bt == 0) {  // B: dy of the KD pixels, MN-major atoms of the K filters
+                        const uint32_t bT = smem_u32(sB + (size_t)s * B_BYTES);
+                        const uint32_t fb = smem_u32(&full[s]);
+                        mbar_arrive_tx(fb, (uint32_t)p.tma_bytes);
+                        const int row = kb / p.win_qb;
+                        for (int a = 0; a < p.bn_atoms; ++a)
+                            tma_load_3d(bT + a * KD * 128, &tmB, fb, n0 + a * (128 / ELT), cq0, row);
+                    }
+                    mbar_wait(smem_u32(&xfull[jx]), xph);
+                    const T* xs = xs_base + (size_t)jx * (p.sx_bytes / ELT);
+                    // rows (pixels) the MMA reads: valid rounded up to the MMA K step (the
+                    // rest of the stage is never read; dy rows past Q are zero-filled)
+                    const int nrows = min(KD, (valid + UMMA_K - 1) / UMMA_K * UMMA_K);
+                    for (int idx = bt; idx < nrows * CH; idx += 256) {
+                        const int kr = idx / CH, ch = idx - kr * CH;
+                        const int m0e = ch * EPC;
+                        const int base = col0 + stC * kr;
+                        uint32_t w[4];
+                        if constexpr (ELT == 4) {
+#pragma unroll
+                            for (int e = 0; e < 4; ++e) {
+                                const int t = tab[m0e + e];
+                                w[e] = t >= 0 ? __float_as_uint(xs[t + base]) : 0u;
+                            }
+                        } else {
+#pragma unroll
+                            for (int e = 0; e < 4; ++e) {
+                                const int t0 = tab[m0e + 2 * e], t1 = tab[m0e + 2 * e + 1];
+                                const uint32_t lo = t0 >= 0 ? (uint32_t)__bfloat16_as_ushort(xs[t0 + base]) : 0u;
+                                const uint32_t hi = t1 >= 0 ? (uint32_t)__bfloat16_as_ushort(xs[t1 + base]) : 0u;
+                                w[e] = lo | (hi << 16);
+                            }
+                        }
+                        const int hh = m0e >> 7, mi = m0e & 127;
+                        const uint32_t addr = aT + (uint32_t)(hh * A_HALF) + (uint32_t)((mi / (128 / ELT)) * KD * 128) +
+                                              mn_row_off<ELT>(kr, (mi % (128 / ELT)) * ELT);
+                        asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(addr), "r"(w[0]), "r"(w[1]),
+                                     "r"(w[2]), "r"(w[3])
+                                     : "memory");
+                    }
+                    fence_proxy_async();
+                    mbar_arrive(smem_u32(&full[s]));
+                    mbar_arrive(smem_u32(&xempty[jx]));
+                    if (bt == 0 && i + p.sx_stages < nk) {
+                        mbar_wait(smem_u32(&xempty[jx]), xph);  // every builder is done with this stage
+                        x_issue(kb + p.sx_stages, jx);
+                    }
+                }
+            }
+        }
+    }
+    if (STAGED && warp < 4) {
+        // builders only (above)
+    } else if (HALO && warp < 4) {
+
         // ===================== halo producers (A_HALO) =====================
         // warp 1: one halo per (tile, channel chunk) = the full rows of the
         // extended source grid the tile's taps touch (one TMA row box each);
@@ -824,12 +940,20 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                     // Fully unrolled with compile-time strides: the single issuing thread
                     // is on the critical path (measured: runtime strides / extra variants
                     // here cost 10-30% on the FWD kernels).
+                    // A_STAGED_WG: the last pixel block of an output row issues only the MMA K
+                    // steps that cover its valid pixels
+                    int jmax = KB / UMMA_K;
+                    if constexpr (STAGED) {
+                        const int qb = kb % p.win_qb;
+                        jmax = min(jmax, (min(KD, p.Q - qb * KD) + UMMA_K - 1) / UMMA_K);
+                    }
                     auto issue = [&](auto mt_c, const int jj) {
                         constexpr int MT = decltype(mt_c)::value;
                         // MN-major operands: k-block jj of the stage starts jj * KB rows in
                         const uint32_t kofs = A_MN ? (uint32_t)(jj * KB * 128) : 0u;
 #pragma unroll
                         for (int j = 0; j < KB / UMMA_K; ++j) {
+                            if (STAGED && j >= jmax) break;
                             const uint64_t bd = B_MN ? sdesc(bT + kofs + j * UMMA_K * 128, KDm * 128, MN_SBO, MN_LAYOUT)
                                                      : sdesc(bT + j * 32, 16, 1024);
 #pragma unroll
@@ -851,6 +975,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                     if constexpr (A_MN) {
                         for (int jj = 0; jj < p.km; ++jj) {
                             if (p.mt == 4) issue(std::integral_constant<int, 4>{}, jj);
+                            else if (p.mt == 3 && STAGED) issue(std::integral_constant<int, 3>{}, jj);
                             else if (p.mt == 2) issue(std::integral_constant<int, 2>{}, jj);
                             else issue(std::integral_constant<int, 1>{}, jj);
                         }
@@ -1115,6 +1240,14 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
 #pragma unroll
                         for (int j = 0; j < 32; ++j) dofs[j] = nb + j < p.N ? j : -1;
                         rmw32(d, dofs, (size_t)p.ldc, v, p.alpha, bsplit);
+                    }
+                } else if constexpr (EPI == EPI_WGRAD_TAPS) {
+                    // row m = exact tap (r, s, c) -> dw[k = nb + j][m]
+                    if (m < p.kred_taps) {
+                        int dofs[32];
+#pragma unroll
+                        for (int j = 0; j < 32; ++j) dofs[j] = nb + j < p.N ? j : -1;
+                        rmw32(outF + (size_t)nb * p.ldc + m, dofs, (size_t)p.ldc, v, p.alpha, bsplit);
                     }
                 } else if constexpr (EPI == EPI_WGRAD_SMALLC) {
                     // padded column j' = (r, s8, c') -> dw column (r*S + s)*C + c (skip padding)

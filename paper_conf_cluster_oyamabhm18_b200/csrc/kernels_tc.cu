@@ -314,6 +314,8 @@ struct TcArgs {
 };
 
 constexpr int kThreads = 288;  // 4 producer warps, 1 MMA warp, 4 epilogue warps
+// A_STAGED_WG adds a TMA warp (9): warps 0-3 and 5-8 build the A operand
+constexpr int threads_for(int am) { return am == 15 ? 320 : kThreads; }
 
 // DGRAD reduction tap index -> filter tap r*S+s (phase mode: the sub-filter
 // tap (a,b) is (r0 + st*a, s0 + st*b)).
@@ -556,7 +558,7 @@ int launch_t(Launch& L, cudaStream_t st, bool dry) {
     static const int pdl = env_int("MUCU_PDL", 1);
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = L.grid;
-    cfg.blockDim = dim3(kThreads);
+    cfg.blockDim = dim3(threads_for(AM));
     cfg.dynamicSmemBytes = (size_t)smem;
     cfg.stream = st;
     cudaLaunchAttribute attr[2];
@@ -1359,9 +1361,9 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
             const int tabb = (int)align_up((uint64_t)TR * 4, 1024);
             const int stage = mtS * 16384 + b_bytes_s;
             int Ss = 0, SX = 0;
-            for (int sa : {3, 2})
-                for (int sx : {4, 3, 2})
-                    if (!Ss && sa * stage + sx * sx_bytes + tabb <= 205 * 1024) { Ss = sa; SX = sx; }
+            for (int sa : {2, 3})
+                for (int sx : {8, 6, 5, 4, 3, 2})
+                    if (!Ss && sa * stage + sx * sx_bytes + tabb <= 210 * 1024) { Ss = sa; SX = sx; }
             if (mtS <= 4 && g.k <= 256 && g.k % atom == 0 && cs > 0 && g.r <= 256 && bch <= 256 && Ss &&
                 128 * mtS * (g.k + 4) * 4 <= 210 * 1024) {
                 A.M = (int)RSC; A.N = g.k; A.ldc = (int)RSC; A.kred_taps = (int)RSC; A.mt = mtS; A.BN = g.k;

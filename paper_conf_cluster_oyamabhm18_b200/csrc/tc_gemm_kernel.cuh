@@ -58,7 +58,7 @@ __device__ __forceinline__ void rmw32(float* dst, const int (&ofs)[32], size_t s
 }
 
 template <int ELT, int AM, int BM_, int EPI>
-__global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constant__ TcArgs p,
+__global__ void __launch_bounds__(threads_for(AM), 1) tc_conv_gemm(const __grid_constant__ TcArgs p,
                                                             const __grid_constant__ CUtensorMap tmA,
                                                             const __grid_constant__ CUtensorMap tmB) {
     using T = typename Elt<ELT>::T;
@@ -193,56 +193,48 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
     };
 
     if constexpr (STAGED) {
-        if (warp != 4) {
-            // ================= staged-row builders (A_STAGED_WG) =================
-            // k-block kb = KD output pixels (n, p, q0 .. q0+KD-1) of output row n*P + p;
-            // x rows st*p + r - pad (r < R), elements [chunk0*cs, (chunk0 + bch)*cs) of
-            // each row (zero outside the image) land in an x stage by one TMA box; GEMM
-            // row m = (r, s, c) of pixel q reads staged[r][tab(m) + col0 + st*C*(q - q0)].
-            const int bt = warp < 4 ? threadIdx.x : threadIdx.x - 32;  // 0..255
-            const T* xs_base = (const T*)sBres;
-            int* tab = (int*)(sBres + (size_t)p.sx_stages * p.sx_bytes);
-            const int TR = 128 * p.mt;
-            const int SC = p.S * p.C;
-            for (int m = bt; m < TR; m += 256) tab[m] = m < p.kred_taps ? (m / SC) * p.sx_sr + m % SC : -1;
-            asm volatile("bar.sync 2, 256;" ::: "memory");
-            constexpr int EPC = 16 / ELT;             // elements per 16-B chunk
-            const int CH = TR / EPC;                  // chunks per A K-row (pixel)
-            const int stC = p.stride * p.C;
-            auto x_coords = [&](int kb, int& cq0, int& chunk0, int& h0, int& n_, int& col0, int& valid) {
-                const int row = kb / p.win_qb, qb = kb - row * p.win_qb;
-                n_ = row / p.P;
-                const int pp = row - n_ * p.P;
-                cq0 = qb * KD;
-                h0 = p.stride * pp - p.pad;
-                const int e0 = (p.stride * cq0 - p.pad) * p.C;
-                chunk0 = e0 >= 0 ? e0 / p.sx_cs : -((-e0 + p.sx_cs - 1) / p.sx_cs);
-                col0 = e0 - chunk0 * p.sx_cs;
-                valid = min(KD, p.Q - cq0);
-            };
-            auto x_issue = [&](int kb, int jx) {
-                int cq0, chunk0, h0, n_, col0, valid;
-                x_coords(kb, cq0, chunk0, h0, n_, col0, valid);
-                const uint32_t fb = smem_u32(&xfull[jx]);
-                mbar_arrive_tx(fb, (uint32_t)p.sx_tx);
-                tma_load_4d(smem_u32(sBres + (size_t)jx * p.sx_bytes), &tmA, fb, 0, chunk0, h0, n_);
-            };
-            int ai = 0, xi = 0;
-            for (int tile = blockIdx.x; tile < total_tiles; tile += gridDim.x) {
-                int m0, n0, z, kb_begin, kb_end;
-                decode(tile, m0, n0, z, kb_begin, kb_end);
-                const int nk = kb_end - kb_begin;
-                if (bt == 0)
-                    for (int j = 0; j < min(p.sx_stages, nk); ++j) x_issue(kb_begin + j, (xi + j) % p.sx_stages);
-                for (int i = 0; i < nk; ++i, ++ai, ++xi) {
-                    const int kb = kb_begin + i;
-                    const int s = ai % S, jx = xi % p.sx_stages;
-                    const uint32_t aph = (uint32_t)((ai / S) & 1), xph = (uint32_t)((xi / p.sx_stages) & 1);
-                    mbar_wait(smem_u32(&empty[s]), aph ^ 1u);
-                    int cq0, chunk0, h0, n_, col0, valid;
-                    x_coords(kb, cq0, chunk0, h0, n_, col0, valid);
-                    const uint32_t aT = smem_u32(sA + (size_t)s * A_BYTES);
-                    if (bt == 0) {  // B: dy of the KD pixels, MN-major atoms of the K filters
+        // ================= staged-row producers (A_STAGED_WG) =================
+        // k-block kb = KD output pixels (n, p, q0 .. q0+KD-1) of output row n*P + p;
+        // x rows st*p + r - pad (r < R), elements [chunk0*cs, (chunk0 + bch)*cs) of each
+        // row (zero outside the image) land in an x stage by one TMA box; GEMM row
+        // m = (r, s, c) of pixel q reads staged[r][tab(m) + col0 + st*C*(q - q0)].
+        // Warp 9 issues the x and dy TMA loads (running ahead over an sx_stages ring);
+        // warps 0-3 and 5-8 (256 threads) build the A operand.  Each builder owns fixed
+        // work units (a 16-B chunk of the tap axis x 4 consecutive pixels) whose
+        // shared-memory source offsets and swizzled destinations are computed once.
+        int* tab = (int*)(sBres + (size_t)p.sx_stages * p.sx_bytes);
+        const int TR = 128 * p.mt;
+        constexpr int EPC = 16 / ELT;             // elements per 16-B chunk
+        const int CH = TR / EPC;                  // chunks per A K-row (pixel)
+        const int stC = p.stride * p.C;
+        auto x_coords = [&](int kb, int& cq0, int& chunk0, int& h0, int& n_, int& col0, int& valid) {
+            const int row = kb / p.win_qb, qb = kb - row * p.win_qb;
+            n_ = row / p.P;
+            const int pp = row - n_ * p.P;
+            cq0 = qb * KD;
+            h0 = p.stride * pp - p.pad;
+            const int e0 = (p.stride * cq0 - p.pad) * p.C;
+            chunk0 = e0 >= 0 ? e0 / p.sx_cs : -((-e0 + p.sx_cs - 1) / p.sx_cs);
+            col0 = e0 - chunk0 * p.sx_cs;
+            valid = min(KD, p.Q - cq0);
+        };
+        if (warp == 9) {
+            if (lane == 0) {
+                int ai = 0;
+                for (int tile = blockIdx.x; tile < total_tiles; tile += gridDim.x) {
+                    int m0, n0, z, kb_begin, kb_end;
+                    decode(tile, m0, n0, z, kb_begin, kb_end);
+                    for (int kb = kb_begin; kb < kb_end; ++kb, ++ai) {
+                        const int s = ai % S, jx = ai % p.sx_stages;
+                        int cq0, chunk0, h0, n_, col0, valid;
+                        x_coords(kb, cq0, chunk0, h0, n_, col0, valid);
+                        // x rows into ring stage jx (freed by the builders)
+                        mbar_wait(smem_u32(&xempty[jx]), (uint32_t)(((ai / p.sx_stages) & 1) ^ 1));
+                        const uint32_t xb = smem_u32(&xfull[jx]);
+                        mbar_arrive_tx(xb, (uint32_t)p.sx_tx);
+                        tma_load_4d(smem_u32(sBres + (size_t)jx * p.sx_bytes), &tmA, xb, 0, chunk0, h0, n_);
+                        // dy of the KD pixels into operand stage s (freed by the MMA)
+                        mbar_wait(smem_u32(&empty[s]), (uint32_t)(((ai / S) & 1) ^ 1));
                         const uint32_t bT = smem_u32(sB + (size_t)s * B_BYTES);
                         const uint32_t fb = smem_u32(&full[s]);
                         mbar_arrive_tx(fb, (uint32_t)p.tma_bytes);
@@ -250,51 +242,95 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                         for (int a = 0; a < p.bn_atoms; ++a)
                             tma_load_3d(bT + a * KD * 128, &tmB, fb, n0 + a * (128 / ELT), cq0, row);
                     }
-                    mbar_wait(smem_u32(&xfull[jx]), xph);
-                    const T* xs = xs_base + (size_t)jx * (p.sx_bytes / ELT);
+                }
+            }
+            __syncwarp();
+        } else if (warp != 4) {
+            const int bt = warp < 4 ? threadIdx.x : threadIdx.x - 32;  // 0..255
+            for (int m = bt; m < TR; m += 256) tab[m] = m < p.kred_taps ? (m / (p.S * p.C)) * p.sx_sr + m % (p.S * p.C) : -1;
+            asm volatile("bar.sync 2, 256;" ::: "memory");
+            // this thread's units u = bt + 256 j: chunk ch = u % CH, pixel group gr = u / CH
+            constexpr int MAXU = 4;
+            const int ngr_all = KD / 4, nunits = CH * ngr_all;
+            int u_gr[MAXU], u_src[MAXU][EPC];
+            uint32_t u_dst[MAXU];
+#pragma unroll
+            for (int j = 0; j < MAXU; ++j) {
+                const int u = bt + 256 * j;
+                u_gr[j] = u < nunits ? u / CH : 1 << 20;
+                const int ch = u - (u / CH) * CH, m0e = ch * EPC;
+                const int hh = m0e >> 7, mi = m0e & 127;
+                // destination of pixel row kr = 4*gr + rr: row base + swizzled chunk (the
+                // swizzle depends on kr % 4 (tf32) / kr % 8 (bf16), i.e. on rr and gr)
+                u_dst[j] = (uint32_t)(hh * A_HALF) + (uint32_t)((mi / (128 / ELT)) * KD * 128) +
+                           mn_row_off<ELT>(4 * (u_gr[j] & 1), (mi % (128 / ELT)) * ELT) - 512u * (u_gr[j] & 1);
+#pragma unroll
+                for (int e = 0; e < EPC; ++e) {
+                    const int t = u < nunits ? tab[m0e + e] : -1;
+                    u_src[j][e] = t >= 0 ? (t + stC * 4 * u_gr[j]) * ELT : -1;
+                }
+            }
+            int ai = 0;
+            for (int tile = blockIdx.x; tile < total_tiles; tile += gridDim.x) {
+                int m0, n0, z, kb_begin, kb_end;
+                decode(tile, m0, n0, z, kb_begin, kb_end);
+                for (int kb = kb_begin; kb < kb_end; ++kb, ++ai) {
+                    const int s = ai % S, jx = ai % p.sx_stages;
+                    int cq0, chunk0, h0, n_, col0, valid;
+                    x_coords(kb, cq0, chunk0, h0, n_, col0, valid);
+                    mbar_wait(smem_u32(&empty[s]), (uint32_t)(((ai / S) & 1) ^ 1));
+                    mbar_wait(smem_u32(&xfull[jx]), (uint32_t)((ai / p.sx_stages) & 1));
+                    const uint32_t aT = smem_u32(sA + (size_t)s * A_BYTES);
+                    const uint32_t xs = smem_u32(sBres) + (uint32_t)(jx * p.sx_bytes) + (uint32_t)(col0 * ELT);
                     // rows (pixels) the MMA reads: valid rounded up to the MMA K step (the
                     // rest of the stage is never read; dy rows past Q are zero-filled)
                     const int nrows = min(KD, (valid + UMMA_K - 1) / UMMA_K * UMMA_K);
-                    for (int idx = bt; idx < nrows * CH; idx += 256) {
-                        const int kr = idx / CH, ch = idx - kr * CH;
-                        const int m0e = ch * EPC;
-                        const int base = col0 + stC * kr;
-                        uint32_t w[4];
-                        if constexpr (ELT == 4) {
 #pragma unroll
-                            for (int e = 0; e < 4; ++e) {
-                                const int t = tab[m0e + e];
-                                w[e] = t >= 0 ? __float_as_uint(xs[t + base]) : 0u;
-                            }
-                        } else {
+                    for (int j = 0; j < MAXU; ++j) {
+                        if (4 * u_gr[j] >= nrows) continue;
 #pragma unroll
-                            for (int e = 0; e < 4; ++e) {
-                                const int t0 = tab[m0e + 2 * e], t1 = tab[m0e + 2 * e + 1];
-                                const uint32_t lo = t0 >= 0 ? (uint32_t)__bfloat16_as_ushort(xs[t0 + base]) : 0u;
-                                const uint32_t hi = t1 >= 0 ? (uint32_t)__bfloat16_as_ushort(xs[t1 + base]) : 0u;
-                                w[e] = lo | (hi << 16);
+                        for (int rr = 0; rr < 4; ++rr) {
+                            const int kr = 4 * u_gr[j] + rr;
+                            if (kr >= nrows) break;
+                            const uint32_t xrow = xs + (uint32_t)(stC * rr * ELT);
+                            uint32_t w[4];
+                            if constexpr (ELT == 4) {
+#pragma unroll
+                                for (int e = 0; e < 4; ++e) {
+                                    uint32_t v = 0u;
+                                    if (u_src[j][e] >= 0)
+                                        asm volatile("ld.shared.b32 %0, [%1];" : "=r"(v) : "r"(xrow + (uint32_t)u_src[j][e]));
+                                    w[e] = v;
+                                }
+                            } else {
+#pragma unroll
+                                for (int e = 0; e < 4; ++e) {
+                                    unsigned short lo = 0, hi = 0;
+                                    if (u_src[j][2 * e] >= 0)
+                                        asm volatile("ld.shared.u16 %0, [%1];" : "=h"(lo) : "r"(xrow + (uint32_t)u_src[j][2 * e]));
+                                    if (u_src[j][2 * e + 1] >= 0)
+                                        asm volatile("ld.shared.u16 %0, [%1];" : "=h"(hi) : "r"(xrow + (uint32_t)u_src[j][2 * e + 1]));
+                                    w[e] = (uint32_t)lo | ((uint32_t)hi << 16);
+                                }
                             }
+                            // row kr: + kr * 128; the swizzle XOR of kr's low bits (rr) on the
+                            // 16-B (bf16) / 32-B (tf32) chunk index
+                            const uint32_t dst = aT + u_dst[j] + (uint32_t)(kr * 128);
+                            const uint32_t sw = ELT == 4 ? ((uint32_t)(rr & 3) << 5) : ((uint32_t)(rr & 3) << 4);
+                            asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(dst ^ sw), "r"(w[0]),
+                                         "r"(w[1]), "r"(w[2]), "r"(w[3])
+                                         : "memory");
                         }
-                        const int hh = m0e >> 7, mi = m0e & 127;
-                        const uint32_t addr = aT + (uint32_t)(hh * A_HALF) + (uint32_t)((mi / (128 / ELT)) * KD * 128) +
-                                              mn_row_off<ELT>(kr, (mi % (128 / ELT)) * ELT);
-                        asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(addr), "r"(w[0]), "r"(w[1]),
-                                     "r"(w[2]), "r"(w[3])
-                                     : "memory");
                     }
                     fence_proxy_async();
                     mbar_arrive(smem_u32(&full[s]));
                     mbar_arrive(smem_u32(&xempty[jx]));
-                    if (bt == 0 && i + p.sx_stages < nk) {
-                        mbar_wait(smem_u32(&xempty[jx]), xph);  // every builder is done with this stage
-                        x_issue(kb + p.sx_stages, jx);
-                    }
                 }
             }
         }
     }
-    if (STAGED && warp < 4) {
-        // builders only (above)
+    if (STAGED && (warp < 4 || warp == 9)) {
+        // builders / TMA warp only (above)
     } else if (HALO && warp < 4) {
 
         // ===================== halo producers (A_HALO) =====================
@@ -1374,7 +1410,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_conv_gemm(const __grid_constan
                 const uint32_t stg = smem_u32(smem);
                 float* outF = (float*)p.out + (p.zsplit ? (size_t)batch * p.batch_stride : 0);
                 // thread -> (column quad c4, row phase rsub): one division per thread
-                const int tpr = kThreads / nq;  // rows in flight per pass
+                const int tpr = (int)blockDim.x / nq;  // rows in flight per pass
                 const bool active = ep < tpr * nq;
                 const int c4 = ep % nq, rsub = ep / nq;
                 const int col0 = n0 + 4 * c4;

@@ -68,6 +68,9 @@ def parse():
     ap.add_argument("--no-concurrent-wgrad", dest="concurrent_wgrad", action="store_false",
                     help="run each BackwardFilter after its BackwardData on one stream")
     ap.add_argument("--cpu-sample", type=int, default=0, help="oracle sample (images per kernel); 0 = auto")
+    ap.add_argument("--nondeterministic", action="store_true",
+                    help="BackwardFilter split-K partials added with L2 atomics (mucu_set_deterministic(0)); "
+                         "default: fixed-order reduction, bitwise reproducible dW")
     ap.add_argument("--json-out", default="")
     ap.add_argument("--tables-in", default="", help="benchmark DB (.npz) to plan from instead of benchmarking")
     ap.add_argument("--tables-out", default="", help="write the benchmark DB (.npz) after the benchmark pass")
@@ -307,6 +310,7 @@ def main():
     math = MATHS[args.math]
     h = mu.Handle(local)
     h.set_policy({"pow2": mu.POLICY_POW2, "all": mu.POLICY_ALL, "undivided": mu.POLICY_UNDIVIDED}[args.policy])
+    h.set_deterministic(not args.nondeterministic)
     ws_limit = int(args.ws_mib * 2 ** 20)
     net = ConvNet(h, layers, args.batch, math, device=dev, types=types)
     net.allocate(seed=rank)
@@ -543,7 +547,8 @@ def main():
                        "l2": "512 MiB buffer overwritten before every timed step",
                        "first_layer_backward_data": bool(args.input_grad),
                        "backward_streams": 2 if args.concurrent_wgrad else 1,
-                       "wgrad_reduction": "ordered split-K (deterministic)"},
+                       "wgrad_reduction": ("split-K with fp32 L2 atomics (non-deterministic)" if args.nondeterministic
+                                           else "ordered split-K (deterministic)")},
             "images_per_s": round(args.batch * world / (ms_max * 1e-3), 1),
             "conv_tflops_direct": round(conv_flops * world / (ms_max * 1e-3) / 1e12, 2),
             "ms_per_step_with_op_events": round(ms_ops, 4),

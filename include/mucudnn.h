@@ -115,6 +115,17 @@ mucu_status_t mucu_destroy(mucu_handle_t handle);
  * or through a special library function" -- this is the function. */
 mucu_status_t mucu_set_policy(mucu_handle_t handle, mucu_policy_t policy);
 mucu_status_t mucu_set_bench_params(mucu_handle_t handle, int32_t warmup, int32_t reps);
+/* BackwardFilter reduction order (dW is a plain sum over samples).
+ * deterministic = 1 (default; env MUCU_DETERMINISTIC): when a kernel splits the
+ * pixel reduction of a dw tile over several CTAs, the partials are combined in a
+ * fixed order (a thread-block cluster sums its CTAs' partials over distributed
+ * shared memory in rank order; split groups add into dw in group order behind a
+ * turn counter), so dw is bitwise reproducible run to run.  deterministic = 0:
+ * every split adds its partial with fp32 L2 reductions (faster on layers with
+ * few dw tiles and long reductions; run-to-run rounding differences).  FWD and
+ * BackwardData are deterministic in both modes.  Results of either mode equal
+ * the exact sum within fp32 rounding; integer-valued data are exact. */
+mucu_status_t mucu_set_deterministic(mucu_handle_t handle, int32_t deterministic);
 
 /* ------------------------------------------------------ host: geometry ---- */
 /* P and Q of the output (host).  INVALID_VALUE if any dim <= 0 or P,Q <= 0. */

@@ -67,6 +67,7 @@ def _load():
         "mucu_destroy": (ctypes.c_int, [vp]),
         "mucu_set_policy": (ctypes.c_int, [vp, ctypes.c_int]),
         "mucu_set_bench_params": (ctypes.c_int, [vp, i32, i32]),
+        "mucu_set_deterministic": (ctypes.c_int, [vp, i32]),
         "mucu_output_dims": (ctypes.c_int, [D, P(i32), P(i32)]),
         "mucu_workspace_size": (ctypes.c_int, [D, ctypes.c_int, ctypes.c_int, i32, P(u64)]),
         "mucu_plan_wr": (ctypes.c_int, [i32, P(i64), P(u64), u64, MC, i32, P(i32), P(i64)]),
@@ -222,6 +223,10 @@ class Handle:
 
     def set_policy(self, policy: int):
         _check(lib.mucu_set_policy(self._h, policy))
+
+    def set_deterministic(self, deterministic: bool):
+        """BackwardFilter split-K reduction: fixed order (default) or L2 atomics."""
+        _check(lib.mucu_set_deterministic(self._h, 1 if deterministic else 0))
 
     def set_bench_params(self, warmup: int, reps: int):
         _check(lib.mucu_set_bench_params(self._h, warmup, reps))

@@ -246,6 +246,7 @@ struct Handle {
     int num_sms = 148;
     int policy = MUCU_POLICY_POW2;
     int warmup = 2, reps = 5;
+    bool deterministic = true;  // BackwardFilter split-K order (mucu_set_deterministic)
     std::map<std::string, std::pair<std::vector<int64_t>, std::vector<uint64_t>>> cache;
     // (descriptor, type, algo, b) -> tensor-core path available (executor pre-validation)
     std::map<std::string, bool> tc_ok;
@@ -271,6 +272,7 @@ mucu_status_t run_micro(Handle* hd, const Geom& g, int type, int algo, int32_t b
         ctx->fixed_src = nullptr;
         ctx->last_algo = algo;
     }
+    ctx->deterministic = hd->deterministic;
     int e = 0;
     if (tc) {
         e = tc_run_micro(g, type, algo, b, alpha, in0, in1, beta, out, wsb, L, hd->num_sms, st, ctx);
@@ -416,6 +418,7 @@ extern "C" mucu_status_t mucu_create(mucu_handle_t* out, int device) {
     h->policy = policy_from_env(MUCU_POLICY_POW2);
     if (const char* w = getenv("MUCU_BENCH_WARMUP")) h->warmup = std::max(0, atoi(w));
     if (const char* r = getenv("MUCU_BENCH_REPS")) h->reps = std::max(1, atoi(r));
+    if (const char* dt = getenv("MUCU_DETERMINISTIC")) h->deterministic = atoi(dt) != 0;
     *out = h;
     return MUCU_OK;
 }
@@ -429,6 +432,13 @@ extern "C" mucu_status_t mucu_destroy(mucu_handle_t h) {
 extern "C" mucu_status_t mucu_set_policy(mucu_handle_t h, mucu_policy_t p) {
     if (!h || p < MUCU_POLICY_ALL || p > MUCU_POLICY_UNDIVIDED) return set_error(MUCU_ERR_INVALID_VALUE, "set_policy");
     h->policy = p;
+    return MUCU_OK;
+}
+
+extern "C" mucu_status_t mucu_set_deterministic(mucu_handle_t h, int32_t deterministic) {
+    if (!h) return set_error(MUCU_ERR_INVALID_VALUE, "set_deterministic: null handle");
+    h->deterministic = deterministic != 0;
+    h->tc_ok.clear();
     return MUCU_OK;
 }
 
@@ -626,7 +636,7 @@ extern "C" mucu_status_t mucu_benchmark(mucu_handle_t h, const mucu_conv_desc_t*
     Geom g;
     if (!make_geom(d, &g) || type < 0 || type > 2) return set_error(MUCU_ERR_INVALID_VALUE, "benchmark: invalid descriptor");
     const size_t cols = (size_t)g.n + 1;
-    const std::string key = cache_key(d, type, ws_limit, h->policy, h->warmup, h->reps);
+    const std::string key = cache_key(d, type, ws_limit, h->policy, h->warmup, h->reps) + (h->deterministic ? "" : "|nd");
     auto it = h->cache.find(key);
     if (it != h->cache.end()) {  // P:L159 in-memory cache of benchmark results
         std::copy(it->second.first.begin(), it->second.first.end(), time_ns);

@@ -28,22 +28,10 @@ __device__ __forceinline__ void pdl_entry() {
     asm volatile("griddepcontrol.launch_dependents;" :::);
 }
 
-// Division by a runtime divisor d >= 1 as a multiply-high (round-up method,
-// l = ceil(log2 d), m = floor(2^32 (2^l - d) / d) + 1; exact for all 32-bit n):
-// the index math of the memory-bound transform kernels below was dominated by
-// integer divisions.
-struct FastDiv {
-    uint32_t d, m, l;
-    FastDiv() = default;
-    explicit FastDiv(uint32_t dv) : d(dv), l(0) {
-        while ((1ull << l) < dv) ++l;
-        m = (uint32_t)((((1ull << 32) * ((1ull << l) - dv)) / dv) + 1);
-    }
-    __device__ __forceinline__ uint32_t div(uint32_t n) const {
-        return (uint32_t)(((uint64_t)__umulhi(n, m) + n) >> l);
-    }
-};
-
+// (FastDiv, mucudnn_internal.h: division by a runtime divisor d >= 1 as a
+// multiply-high, l = ceil(log2 d), m = floor(2^32 (2^l - d) / d) + 1, exact for all
+// 32-bit n -- the index math of the memory-bound transform kernels below was
+// dominated by integer divisions.)
 template <typename... KArgs, typename... Args>
 void launch_pdl(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st, Args... args) {
     static const int pdl = getenv("MUCU_PDL") ? atoi(getenv("MUCU_PDL")) : 1;

@@ -38,31 +38,35 @@ struct Dense {
 };
 
 // Implicit im2col of x (NHWC) for FWD: row i = output pixel (n,p,q), kk = (r,s,c).
+// Index arithmetic by multiply-high division (FastDiv): ~3 instructions per
+// quotient instead of a ~20-instruction integer division per element.
 struct Im2col {
     const float* x;
     int64_t rows;
     int H, W, C, P, Q, S, pad, st, RSC;
-    __device__ __forceinline__ float at(int64_t m, int64_t kk) const {
-        if (m >= rows || kk >= RSC) return 0.f;
-        int pq = P * Q;
-        int n = (int)(m / pq);
-        int rem = (int)(m - (int64_t)n * pq);
-        int p = rem / Q, q = rem - p * Q;
-        int k2 = (int)kk;
-        int rs = k2 / C, c = k2 - rs * C;
-        int r = rs / S, s = rs - r * S;
-        int h = p * st + r - pad, w = q * st + s - pad;
-        if (h < 0 || h >= H || w < 0 || w >= W) return 0.f;
+    FastDiv dPQ, dQ, dC, dS;
+    __device__ __forceinline__ float at(int64_t m64, int64_t kk64) const {
+        if (m64 >= rows || kk64 >= RSC) return 0.f;
+        const uint32_t m = (uint32_t)m64, kk = (uint32_t)kk64;
+        const uint32_t n = dPQ.div(m), rem = m - n * (uint32_t)(P * Q);
+        const uint32_t p = dQ.div(rem), q = rem - p * (uint32_t)Q;
+        const uint32_t rs = dC.div(kk), c = kk - rs * (uint32_t)C;
+        const uint32_t r = dS.div(rs), s = rs - r * (uint32_t)S;
+        const int h = (int)(p * st + r) - pad, w = (int)(q * st + s) - pad;
+        if ((unsigned)h >= (unsigned)H || (unsigned)w >= (unsigned)W) return 0.f;
         return __ldg(x + (((int64_t)n * H + h) * W + w) * C + c);
     }
     __device__ __forceinline__ void batch(int) {}
 };
+Im2col make_im2col(const float* x, int64_t rows, const Geom& g) {
+    return Im2col{x, rows, g.h, g.w, g.c, g.p, g.q, g.s, g.pad, g.stride, g.r * g.s * g.c,
+                  FastDiv((uint32_t)(g.p * g.q)), FastDiv((uint32_t)g.q), FastDiv((uint32_t)g.c), FastDiv((uint32_t)g.s)};
+}
 
 // Im2col transposed for WGRAD's B operand: B(j, kk) = im2col(kk = pixel, j = (r,s,c)).
 struct Im2colT {
     Im2col v;
     __device__ __forceinline__ float at(int64_t j, int64_t m) const { return v.at(m, j); }
-    __device__ __forceinline__ void batch(int) {}
 };
 
 // DGRAD gather of dy: row i = dx pixel (n,h,w), kk = (r,s,k):
@@ -71,19 +75,18 @@ struct DgradGather {
     const float* dy;
     int64_t rows;
     int H, W, K, P, Q, S, pad, st, RSK;
-    __device__ __forceinline__ float at(int64_t m, int64_t kk) const {
-        if (m >= rows || kk >= RSK) return 0.f;
-        int hw = H * W;
-        int n = (int)(m / hw);
-        int rem = (int)(m - (int64_t)n * hw);
-        int h = rem / W, w = rem - h * W;
-        int k2 = (int)kk;
-        int rs = k2 / K, k = k2 - rs * K;
-        int r = rs / S, s = rs - r * S;
-        int ph = h + pad - r, pw = w + pad - s;
-        if (ph < 0 || pw < 0 || ph % st || pw % st) return 0.f;
-        int p = ph / st, q = pw / st;
-        if (p >= P || q >= Q) return 0.f;
+    FastDiv dHW, dW, dK, dS, dSt;
+    __device__ __forceinline__ float at(int64_t m64, int64_t kk64) const {
+        if (m64 >= rows || kk64 >= RSK) return 0.f;
+        const uint32_t m = (uint32_t)m64, kk = (uint32_t)kk64;
+        const uint32_t n = dHW.div(m), rem = m - n * (uint32_t)(H * W);
+        const uint32_t h = dW.div(rem), w = rem - h * (uint32_t)W;
+        const uint32_t rs = dK.div(kk), k = kk - rs * (uint32_t)K;
+        const uint32_t r = dS.div(rs), s = rs - r * (uint32_t)S;
+        const int ph = (int)(h + pad) - (int)r, pw = (int)(w + pad) - (int)s;
+        if (ph < 0 || pw < 0) return 0.f;
+        const uint32_t p = dSt.div((uint32_t)ph), q = dSt.div((uint32_t)pw);
+        if (p * st != (uint32_t)ph || q * st != (uint32_t)pw || p >= (uint32_t)P || q >= (uint32_t)Q) return 0.f;
         return __ldg(dy + (((int64_t)n * P + p) * Q + q) * K + k);
     }
     __device__ __forceinline__ void batch(int) {}
@@ -93,10 +96,10 @@ struct DgradGather {
 struct DgradFilter {
     const float* w;
     int C, K, RS;
-    __device__ __forceinline__ float at(int64_t j, int64_t kk) const {
-        if (j >= C || kk >= (int64_t)RS * K) return 0.f;
-        int k2 = (int)kk;
-        int rs = k2 / K, k = k2 - rs * K;
+    FastDiv dK;
+    __device__ __forceinline__ float at(int64_t j, int64_t kk64) const {
+        if (j >= C || kk64 >= (int64_t)RS * K) return 0.f;
+        const uint32_t kk = (uint32_t)kk64, rs = dK.div(kk), k = kk - rs * (uint32_t)K;
         return __ldg(w + ((int64_t)k * RS + rs) * C + j);
     }
     __device__ __forceinline__ void batch(int) {}
@@ -288,7 +291,7 @@ int dispatch_gemm(const AV& a, const BV& b, const EPI& e, int64_t M, int64_t N, 
 int simt_fwd_ig(const Geom& g, int32_t b, float alpha, const float* x, const float* w, float beta, float* y,
                 cudaStream_t st) {
     const int64_t M = (int64_t)b * g.p * g.q, N = g.k, Kd = (int64_t)g.r * g.s * g.c;
-    Im2col a{x, M, g.h, g.w, g.c, g.p, g.q, g.s, g.pad, g.stride, (int)Kd};
+    Im2col a = make_im2col(x, M, g);
     Dense bw{w, N, Kd, Kd, 1, 0};
     StoreDense e{y, M, N, N, 0, alpha, beta};
     return dispatch_gemm<true, true>(a, bw, e, M, N, Kd, 1, st);
@@ -317,8 +320,9 @@ int simt_gemm_nn(int64_t M, int64_t N, int64_t K, float alpha, const float* A, i
 int simt_dgrad_ig(const Geom& g, int32_t b, float alpha, const float* dy, const float* w, float beta, float* dx,
                   cudaStream_t st) {
     const int64_t M = (int64_t)b * g.h * g.w, N = g.c, Kd = (int64_t)g.r * g.s * g.k;
-    DgradGather a{dy, M, g.h, g.w, g.k, g.p, g.q, g.s, g.pad, g.stride, (int)Kd};
-    DgradFilter bw{w, g.c, g.k, g.r * g.s};
+    DgradGather a{dy, M, g.h, g.w, g.k, g.p, g.q, g.s, g.pad, g.stride, (int)Kd, FastDiv((uint32_t)(g.h * g.w)),
+                  FastDiv((uint32_t)g.w), FastDiv((uint32_t)g.k), FastDiv((uint32_t)g.s), FastDiv((uint32_t)g.stride)};
+    DgradFilter bw{w, g.c, g.k, g.r * g.s, FastDiv((uint32_t)g.k)};
     StoreDense e{dx, M, N, N, 0, alpha, beta};
     return dispatch_gemm<true, false>(a, bw, e, M, N, Kd, 1, st);
 }
@@ -347,7 +351,7 @@ int simt_wgrad(const Geom& g, int32_t b, float alpha, const float* dy, const flo
         Dense bb{xin, cols, Kd, 1, kpitch, 0};  // B(j, m) = col[m][j]
         simt_wgrad_kernel<BM, BN><<<grid, kThreads, 0, st>>>(a, bb, dw, rows, cols, Kd, kps, alpha, beta, tr.ctr, tr.epoch);
     } else {
-        Im2colT bb{Im2col{xin, Kd, g.h, g.w, g.c, g.p, g.q, g.s, g.pad, g.stride, (int)cols}};
+        Im2colT bb{make_im2col(xin, Kd, g)};
         simt_wgrad_kernel<BM, BN><<<grid, kThreads, 0, st>>>(a, bb, dw, rows, cols, Kd, kps, alpha, beta, tr.ctr, tr.epoch);
     }
     count_launch();

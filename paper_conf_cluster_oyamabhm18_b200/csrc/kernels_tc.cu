@@ -309,6 +309,7 @@ struct TcArgs {
     // A_STAGED_WG: x-row chunks of sx_cs elements (sx_sr = elements per staged row), sx_stages
     // stages of sx_bytes (sx_tx delivered by TMA), kred_taps = R*S*C GEMM rows
     int sx_cs, sx_sr, sx_stages, sx_bytes, sx_tx, kred_taps;
+    int atomic;              // non-deterministic split-K: partials added with red.global.add
     unsigned long long* turns;
     unsigned long long epoch;
 };
@@ -532,6 +533,15 @@ int launch_t(Launch& L, cudaStream_t st, bool dry) {
     L.a.turns = nullptr;
     L.a.epoch = 0;
     if (dry) return 0;
+    if (SPLITK && L.a.atomic && L.a.beta != 1.f) {
+        // split partials are added with L2 reductions: apply beta to the output first
+        int64_t extent;
+        if (L.a.zsplit) extent = (int64_t)(L.a.num_z / L.a.zsplit) * L.a.batch_stride;
+        else if (EPI == EPI_WGRAD_WIN || EPI == EPI_WGRAD_TAPS) extent = (int64_t)L.a.N * L.a.ldc;
+        else extent = (int64_t)L.a.M * L.a.ldc;
+        const int e = launch_scale(extent, L.a.beta, (float*)L.a.out, st);
+        if (e) return e;
+    }
     // Cluster split-K with more split groups than one: a turn counter per (batch,
     // tile, row slab) orders the groups' additions into dw.
     if (SPLITK && L.a.cl) {
@@ -774,7 +784,7 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
     // km k-blocks: fewer, larger TMA transactions (the TMA issue rate, not
     // bytes, bounds these MN-major loads), as deep as two stages allow.
     // Split of a BackwardFilter reduction of nkb stages over `tiles` output tiles.
-    auto apply_split = [&](int64_t tiles, int64_t nkb, int batches) {
+    auto apply_split = [&](int64_t tiles, int64_t nkb, int batches, bool one_unit = false) {
         // Split of the pixel reduction (deterministic): S = cl * G CTAs per
         // tile; clusters of cl reduce their partials through DSMEM (+R) and the G groups
         // add into dw in a fixed order (+L per hand-over).  Cost in stages of km
@@ -787,6 +797,25 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         int64_t b_s = 1;
         int b_cl = 0;
         double best = force_cl ? 1e30 : (double)ceil_div(tiles, num_sms) * ((double)nkb + E);
+        if (!ctx->deterministic) {
+            // non-deterministic mode: persistent CTAs, splits reduced with fp32 L2 atomics
+            A.atomic = 1;
+            int64_t smax = std::min<int64_t>(std::max<int64_t>(1, nkb / 4), 4LL * num_sms);
+            if (one_unit) smax = std::min<int64_t>(smax, std::max<int64_t>(1, num_sms / tiles));
+            for (int64_t sp = 1; sp <= smax; ++sp) {
+                const double cost = (double)ceil_div(tiles * sp, num_sms) * ((double)ceil_div(nkb, sp) + E);
+                if (cost < best - 1e-9) { best = cost; b_s = sp; }
+            }
+            A.num_kb = (int)nkb;
+            A.kb_per_split = (int)ceil_div(nkb, b_s);
+            b_s = ceil_div(nkb, A.kb_per_split);
+            A.cl = 0;
+            A.stg_bytes = 0;
+            A.zsplit = batches > 1 ? (int)b_s : 0;
+            grid2((int)(batches * b_s));
+            if (b_s == 1) A.atomic = 0;
+            return;
+        }
         for (int cl = 2; cl <= 16; cl *= 2) {
             if (force_cl && cl != force_cl) continue;
             const int cap = cluster_capacity(cl);
@@ -1374,7 +1403,7 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
                 A.nacc = mtS * A.BN <= 256 ? 2 : 1;
                 const int cols = A.nacc * mtS * A.BN;
                 A.tmem_cols = cols <= 64 ? 64 : cols <= 128 ? 128 : cols <= 256 ? 256 : 512;
-                apply_split(1, (int64_t)b * g.p * A.win_qb, 1);
+                apply_split(1, (int64_t)b * g.p * A.win_qb, 1, true);  // builders double as epilogue: one unit per CTA
                 uint64_t dims[4] = {(uint64_t)cs, (uint64_t)(WC / cs), (uint64_t)g.h, (uint64_t)b};
                 uint64_t str[3] = {(uint64_t)cs * elt, (uint64_t)WC * elt, (uint64_t)g.h * WC * elt};
                 uint32_t box[4] = {(uint32_t)cs, (uint32_t)bch, (uint32_t)g.r, 1};

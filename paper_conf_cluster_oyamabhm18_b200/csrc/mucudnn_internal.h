@@ -78,6 +78,7 @@ struct CallCtx {
     const void* fixed_src = nullptr;
     int last_algo = -1;  // algorithm of the previous micro-config (prefix invalidation)
     bool dry = false;    // tensor-core dispatch decisions only, no launch (pre-validation)
+    bool deterministic = true;  // BackwardFilter split-K: ordered reduction (default) or L2 atomics
 };
 
 struct Handle;
@@ -85,6 +86,22 @@ struct Handle;
 mucu_status_t run_micro(Handle* h, const Geom& g, int type, int algo, int32_t b, float alpha,
                         const void* in0, const void* in1, float beta, void* out, void* ws,
                         uint64_t ws_bytes, cudaStream_t st, CallCtx* ctx);
+
+#ifdef __CUDACC__
+// Division by a run-time constant with a host-computed magic number
+// (multiply-high + shift; exact for every 32-bit numerator).
+struct FastDiv {
+    uint32_t d, m, l;
+    FastDiv() = default;
+    explicit FastDiv(uint32_t dv) : d(dv), l(0) {
+        while ((1ull << l) < dv) ++l;
+        m = (uint32_t)((((1ull << 32) * ((1ull << l) - dv)) / dv) + 1);
+    }
+    __device__ __forceinline__ uint32_t div(uint32_t n) const {
+        return (uint32_t)(((uint64_t)__umulhi(n, m) + n) >> l);
+    }
+};
+#endif
 
 // ---------------------------------------------------------------- kernels --
 // All launchers are asynchronous on `st` and return a CUDA error code (0 = ok).

@@ -48,7 +48,16 @@ __device__ __forceinline__ long long wgrad_dst(const TcArgs& p, int m, int n) {
 // columns of one row (ofs < 0: skipped); all loads issue before the stores.
 // beta == 0 never reads dst (it may hold garbage / NaN).
 __device__ __forceinline__ void rmw32(float* dst, const int (&ofs)[32], size_t stride, const uint32_t* v, float alpha,
-                                      float beta) {
+                                      float beta, bool atomic = false) {
+    if (atomic) {  // non-deterministic split-K (beta applied by a prescale launch): L2 reductions
+#pragma unroll
+        for (int j = 0; j < 32; ++j)
+            if (ofs[j] >= 0)
+                asm volatile("red.global.add.f32 [%0], %1;" ::"l"(dst + (size_t)ofs[j] * stride),
+                             "f"(alpha * __uint_as_float(v[j]))
+                             : "memory");
+        return;
+    }
     float old[32];
 #pragma unroll
     for (int j = 0; j < 32; ++j) old[j] = (beta != 0.f && ofs[j] >= 0) ? __ldcg(dst + (size_t)ofs[j] * stride) : 0.f;
@@ -1074,7 +1083,9 @@ __global__ void __launch_bounds__(threads_for(AM), 1) tc_conv_gemm(const __grid_
             mbar_wait(smem_u32(&tfull[acc]), aph);
             tc_fence_after();
             // BackwardFilter without a split (the whole reduction in this CTA):
-            // dw = alpha * acc + beta * dw.  Split reductions take the cluster path.
+            // dw = alpha * acc + beta * dw.  Deterministic split reductions take the
+            // cluster path; p.atomic (non-deterministic mode) adds every split's partial
+            // with L2 reductions after a beta prescale launch.
             const float bsplit = p.beta;
             auto drain = [&](const int hh) {
             const int m = m0 + 128 * hh + row;
@@ -1263,7 +1274,7 @@ __global__ void __launch_bounds__(threads_for(AM), 1) tc_conv_gemm(const __grid_
                         }
                         if (++ch == p.C) { ch = 0; ++tap; }
                     }
-                    rmw32(drow, dofs, 1, v, p.alpha, bsplit);
+                    rmw32(drow, dofs, 1, v, p.alpha, bsplit, p.atomic);
                 } else if constexpr (EPI == EPI_WGRAD_WIN) {
                     // row m = (r, atom aa, tap t, channel c) -> dw[k][r][aa*taps + t][c], k = nb + j
                     constexpr int per_atom = WAW / ELT;
@@ -1275,7 +1286,7 @@ __global__ void __launch_bounds__(threads_for(AM), 1) tc_conv_gemm(const __grid_
                         int dofs[32];
 #pragma unroll
                         for (int j = 0; j < 32; ++j) dofs[j] = nb + j < p.N ? j : -1;
-                        rmw32(d, dofs, (size_t)p.ldc, v, p.alpha, bsplit);
+                        rmw32(d, dofs, (size_t)p.ldc, v, p.alpha, bsplit, p.atomic);
                     }
                 } else if constexpr (EPI == EPI_WGRAD_TAPS) {
                     // row m = exact tap (r, s, c) -> dw[k = nb + j][m]
@@ -1283,7 +1294,7 @@ __global__ void __launch_bounds__(threads_for(AM), 1) tc_conv_gemm(const __grid_
                         int dofs[32];
 #pragma unroll
                         for (int j = 0; j < 32; ++j) dofs[j] = nb + j < p.N ? j : -1;
-                        rmw32(outF + (size_t)nb * p.ldc + m, dofs, (size_t)p.ldc, v, p.alpha, bsplit);
+                        rmw32(outF + (size_t)nb * p.ldc + m, dofs, (size_t)p.ldc, v, p.alpha, bsplit, p.atomic);
                     }
                 } else if constexpr (EPI == EPI_WGRAD_SMALLC) {
                     // padded column j' = (r, s8, c') -> dw column (r*S + s)*C + c (skip padding)
@@ -1295,13 +1306,21 @@ __global__ void __launch_bounds__(threads_for(AM), 1) tc_conv_gemm(const __grid_
                         const int c = jp % p.cp, t2 = jp / p.cp, s_ = t2 % p.s8, r = t2 / p.s8;
                         dofs[j] = (jp < p.N && c < p.C && s_ < p.S) ? (r * p.S + s_) * p.C + c : -1;
                     }
-                    rmw32(drow, dofs, 1, v, p.alpha, bsplit);
+                    rmw32(drow, dofs, 1, v, p.alpha, bsplit, p.atomic);
                 } else if constexpr (EPI == EPI_WGRAD_CHAIN) {
                     // dw = alpha * partial + bsplit * dw (bsplit = beta on split 0, else 1),
                     // in split order: 16-byte vector read-modify-write
                     float* d = outF + (p.zsplit ? (size_t)(z / p.zsplit) * p.batch_stride : 0) + (size_t)m * p.ldc + nb;
                     const bool vec = (nb + 32 <= p.N) && ((p.ldc & 3) == 0) && ((((uintptr_t)p.out) & 15) == 0);
-                    if (vec) {
+                    if (vec && p.atomic) {
+#pragma unroll
+                        for (int j = 0; j < 32; j += 4)
+                            asm volatile("red.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(d + j),
+                                         "f"(p.alpha * __uint_as_float(v[j])), "f"(p.alpha * __uint_as_float(v[j + 1])),
+                                         "f"(p.alpha * __uint_as_float(v[j + 2])),
+                                         "f"(p.alpha * __uint_as_float(v[j + 3]))
+                                         : "memory");
+                    } else if (vec) {
                         float4 o[8];
 #pragma unroll
                         for (int j = 0; j < 8; ++j)
@@ -1320,7 +1339,7 @@ __global__ void __launch_bounds__(threads_for(AM), 1) tc_conv_gemm(const __grid_
                         int dofs[32];
 #pragma unroll
                         for (int j = 0; j < 32; ++j) dofs[j] = nb + j < p.N ? j : -1;
-                        rmw32(d, dofs, 1, v, p.alpha, bsplit);
+                        rmw32(d, dofs, 1, v, p.alpha, bsplit, p.atomic);
                     }
                 } else if (p.out_bf16) {
                     __nv_bfloat16* d = (__nv_bfloat16*)outT + (size_t)mrow * p.ldc + nb;

@@ -113,3 +113,25 @@ def test_cluster_splitk_wgrad_exact(name, math, env, monkeypatch):
         a1, _ = run_gpu(d, mu.BWD_FILTER, [(algo, shape[0])], xr, wr, dyr)
         a2, _ = run_gpu(d, mu.BWD_FILTER, [(algo, shape[0])], xr, wr, dyr)
         assert np.array_equal(a1, a2), (name, algo, "reproducible")
+
+
+@pytest.mark.parametrize("math", [mu.MATH_TF32, mu.MATH_BF16], ids=["tf32", "bf16"])
+@pytest.mark.parametrize("name", list(SPLITK_SHAPES))
+def test_nondeterministic_wgrad_exact(name, math):
+    """mucu_set_deterministic(0): split partials added with L2 atomics after a
+    beta prescale -- exact on integer data (any order), alpha / beta applied once."""
+    from gpu_util import handle
+    h = handle()
+    h.set_deterministic(False)
+    try:
+        shape = SPLITK_SHAPES[name]
+        d = mu.desc(*shape, math)
+        x, w, dy = conv_inputs(*shape, seed=33, kind="int", lo=-1, hi=1)
+        out0 = np.random.default_rng(6).integers(-2, 3, size=(shape[4], shape[5], shape[6], shape[1])).astype(np.float32)
+        algos = [mu.IMPLICIT_GEMM, mu.IM2COL_GEMM] + ([mu.WINOGRAD] if shape[5] == 3 and shape[8] == 1 else [])
+        for algo in algos:
+            ref = oracle_ref(shape, mu.BWD_FILTER, x, w, dy, alpha=2.0, beta=-1.0, out0=out0)
+            got, _ = run_gpu(d, mu.BWD_FILTER, [(algo, shape[0])], x, w, dy, alpha=2.0, beta=-1.0, out0=out0)
+            assert np.array_equal(got, ref), (name, algo)
+    finally:
+        h.set_deterministic(True)

@@ -558,6 +558,7 @@ def main():
                                   for (i, t), v in op_ms_max.items() if (i, t) in und_op_ms},
             "undivided_per_kernel_ms": {kname(i, t): round(v, 4) for (i, t), v in und_op_ms.items()},
             "workspace_total_mib": round(total_ws / 2 ** 20, 2),
+            "wd_ilp": getattr(net, "wd_stats", None),
             "plan_time_s": round(bench_s, 2),
             "roofline": {"bound": bound, "achieved": round(achieved, 2), "peak": round(peak, 1), "unit": punit,
                          "frac": round(achieved / peak, 4), "traffic": traffic,

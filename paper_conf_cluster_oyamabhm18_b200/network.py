@@ -219,11 +219,23 @@ class ConvNet:
     def plan_wd(self, total_limit: int):
         """WD: desirable sets + exact MCKP over all kernels, one
         network workspace carved into 256-B aligned segments (reading G18)."""
+        import time
         net = L.Network()
         order = list(self.kernels.keys())
         for key in order:
             net.add(self.kernels[key].desc, key[1])
-        net.plan_from_tables(total_limit, [self.kernels[key].table for key in order])
+        tables = [self.kernels[key].table for key in order]
+        t0 = time.perf_counter()
+        net.plan_from_tables(total_limit, tables)  # fronts (set-valued DP) + MCKP, in the C library
+        self.wd_stats = {"kernels": len(order), "plan_ms": round((time.perf_counter() - t0) * 1e3, 3),
+                         "total_limit_mib": round(total_limit / 2 ** 20, 3)}
+        # ILP size (P:L267: 562 binary variables for ResNet-50): one 0-1 variable per
+        # desirable configuration of every kernel; the exact MCKP is timed alone
+        fronts = [L.pareto_front(self.n, t, w, total_limit) for t, w in tables]
+        self.wd_stats["ilp_variables"] = int(sum(len(f) for f in fronts))
+        t1 = time.perf_counter()
+        L.solve_wd([[(int(T), int(M)) for T, M, _ in f] for f in fronts], total_limit)
+        self.wd_stats["ilp_solve_ms"] = round((time.perf_counter() - t1) * 1e3, 3)
         for kid, key in enumerate(order):
             k = self.kernels[key]
             k.plan, k.ws_offset, k.ws_bytes, k.est_ns = net.get(kid)

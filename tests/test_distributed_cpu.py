@@ -134,3 +134,88 @@ def test_shard_benchmark_lpt():
     assert sorted(sum(s, [])) == sorted(costs)
     assert s == [["a", "d", "e"], ["b", "c"]]
     assert shard_benchmark(costs, 1) == [["a", "b", "c", "d", "e"]]
+
+
+def _iteration_worker(rank, world, port, out_dir):
+    """ConvNet.iteration + GradAllreduce over gloo: each rank runs
+    its shard of a global batch through the network executor; the conv calls are
+    routed to the fp64 oracle on CPU (test stand-in for the GPU kernels) so the
+    executor order, zero_grad, the grad hook and the allreduce are exercised."""
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port), RANK=str(rank), WORLD_SIZE=str(world),
+                      LOCAL_RANK=str(rank))
+    import sys
+    sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+    import oracle
+    import paper_conf_cluster_oyamabhm18_b200 as mu
+    from paper_conf_cluster_oyamabhm18_b200 import network as N
+    from paper_conf_cluster_oyamabhm18_b200.distributed import GradAllreduce, init_from_env, shard_range
+    from synthetic import conv_inputs
+    from synthetic.networks import ConvLayer
+    assert init_from_env("gloo")
+    layers = [ConvLayer("a", 3, 11, 11, 8, 3, 3, 1, 2), ConvLayer("b", 8, 6, 6, 6, 3, 3, 1, 1)]
+    n_global = 6
+    lo, hi = shard_range(n_global, rank, world)
+
+    def fwd(h, d, plan, x, w, y, workspace=None):
+        y.copy_(torch.from_numpy(oracle.conv_forward(x.numpy(), w.numpy(), d.pad, d.stride)).float())
+
+    def dgrad(h, d, plan, dy, w, dx, workspace=None):
+        dx.copy_(torch.from_numpy(oracle.conv_backward_data(dy.numpy(), w.numpy(), d.h, d.w, d.pad, d.stride)).float())
+
+    def wgrad(h, d, plan, x, dy, dw, beta=0.0, workspace=None):
+        dw.copy_(torch.from_numpy(oracle.conv_backward_filter(x.numpy(), dy.numpy(), d.r, d.s, d.pad, d.stride, 1.0,
+                                                              beta, dw.numpy().astype(np.float64))).float())
+
+    N.T.conv_forward, N.T.conv_backward_data, N.T.conv_backward_filter = fwd, dgrad, wgrad
+    net = N.ConvNet(None, layers, hi - lo, mu.MATH_F32, device="cpu")
+    net.tensors = []
+    sizes = [l.k * l.r * l.s * l.c for l in layers]
+    net.dw_flat = torch.zeros(sum(sizes))
+    off = 0
+    for i, l in enumerate(layers):
+        x, w, dy = conv_inputs(n_global, l.c, l.h, l.w, l.k, l.r, l.s, l.pad, l.stride, seed=40 + i, kind="int")
+        p_, q_ = (l.h + 2 * l.pad - l.r) // l.stride + 1, (l.w + 2 * l.pad - l.s) // l.stride + 1
+        net.tensors.append(dict(x=torch.from_numpy(x[lo:hi].copy()), w=torch.from_numpy(w),
+                                dy=torch.from_numpy(dy[lo:hi].copy()), y=torch.empty(hi - lo, p_, q_, l.k),
+                                dx=torch.empty(hi - lo, l.h, l.w, l.c),
+                                dw=net.dw_flat[off:off + sizes[i]].view(l.k, l.r, l.s, l.c)))
+        off += sizes[i]
+    for k in net.kernels.values():
+        k.plan = [(mu.IMPLICIT_GEMM, hi - lo)]
+    seen = []
+    ar = GradAllreduce()
+
+    def hook(i, dw):
+        seen.append(i)
+        ar(i, dw)
+    net.iteration(grad_hook=hook)
+    ar.wait()
+    assert seen == [1, 0]  # dW handed over as soon as each layer's BackwardFilter is done
+    for i in range(len(layers)):
+        t = net.tensors[i]
+        np.save(os.path.join(out_dir, f"y{i}_{rank}.npy"), t["y"].numpy())
+        np.save(os.path.join(out_dir, f"dw{i}_{rank}.npy"), t["dw"].numpy())
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+@pytest.mark.timeout(240)
+def test_gloo_convnet_iteration_allreduce():
+    import oracle
+    from synthetic import conv_inputs
+    from synthetic.networks import ConvLayer
+    from paper_conf_cluster_oyamabhm18_b200.distributed import shard_range
+    layers = [ConvLayer("a", 3, 11, 11, 8, 3, 3, 1, 2), ConvLayer("b", 8, 6, 6, 6, 3, 3, 1, 1)]
+    world = 2
+    with tempfile.TemporaryDirectory() as d:
+        mp.spawn(_iteration_worker, args=(world, _free_port(), d), nprocs=world, join=True)
+        for i, l in enumerate(layers):
+            x, w, dy = conv_inputs(6, l.c, l.h, l.w, l.k, l.r, l.s, l.pad, l.stride, seed=40 + i, kind="int")
+            full_dw = oracle.conv_backward_filter(x, dy, l.r, l.s, l.pad, l.stride)
+            full_y = oracle.conv_forward(x, w, l.pad, l.stride)
+            for rank in range(world):
+                lo, hi = shard_range(6, rank, world)
+                # dW summed over ranks == full-batch dW (exact on integer data)
+                assert np.array_equal(np.load(os.path.join(d, f"dw{i}_{rank}.npy")), full_dw.astype(np.float32))
+                # I7: per-sample forward identical to the single-device full batch
+                assert np.array_equal(np.load(os.path.join(d, f"y{i}_{rank}.npy")), full_y[lo:hi].astype(np.float32))

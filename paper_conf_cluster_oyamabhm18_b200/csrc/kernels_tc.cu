@@ -210,6 +210,8 @@ enum AMode : int {
     A_TMA_WIN32 = 14,
     A_TMA_WIN = 11,    // WGRAD window operand, MN-major: rows j = (r, atom, tap, c) of the filter, K = pixels;
                        // one 4-D TMA box per 128-B atom from the overlapping-window view of the padded x
+    A_STAGED_FWD = 16, // FWD of small-C strided layers, zero workspace: the x rows of a tile of whole output rows
+                       // staged by TMA; builders write the exact-tap (r,s,c) K-major operand
     A_STAGED_WG = 15,  // WGRAD of small-C strided layers, zero workspace: the R x rows a block of KD output
                        // pixels reads are staged by one TMA box; builders write the exact-tap (r,s,c) MN-major
                        // operand from them
@@ -310,13 +312,14 @@ struct TcArgs {
     // stages of sx_bytes (sx_tx delivered by TMA), kred_taps = R*S*C GEMM rows
     int sx_cs, sx_sr, sx_stages, sx_bytes, sx_tx, kred_taps;
     int atomic;              // non-deterministic split-K: partials added with red.global.add
+    int sxw_off;             // A_STAGED_FWD: byte offset of the x-row ring after the resident filter
     unsigned long long* turns;
     unsigned long long epoch;
 };
 
 constexpr int kThreads = 288;  // 4 producer warps, 1 MMA warp, 4 epilogue warps
 // A_STAGED_WG adds a TMA warp (9): warps 0-3 and 5-8 build the A operand
-constexpr int threads_for(int am) { return am == 15 ? 320 : kThreads; }
+constexpr int threads_for(int am) { return (am == 15 || am == 16) ? 320 : kThreads; }
 
 // DGRAD reduction tap index -> filter tap r*S+s (phase mode: the sub-filter
 // tap (a,b) is (r0 + st*a, s0 + st*b)).
@@ -880,6 +883,47 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
 #define LAUNCH(AMODE, BMODE, EPIM) \
     (elt == 2 ? launch_t<2, AMODE, BMODE, EPIM>(L, st, dry) : launch_t<4, AMODE, BMODE, EPIM>(L, st, dry))
 
+    if (type == MUCU_FWD && algo == MUCU_ALGO_IMPLICIT_GEMM && small_c_tc(g) && g.q <= 128 && g.k <= 256 &&
+        env_int("MUCU_STAGED", 1)) {
+        // Staged-row forward, zero workspace: tile = Tr whole output rows of
+        // one image (Tr * Q <= 128 GEMM rows), K = the exact taps padded to whole k-blocks.
+        const int Tr = 128 / g.q;
+        const int num_kb = (int)ceil_div(RSC, KB);
+        const int XR = g.stride * (Tr - 1) + g.r;
+        const int WC = g.w * g.c;
+        const int vec = 16 / elt;
+        // TMA destinations 128-B aligned: a 128-B left margin (>= pad*C zero elements) and
+        // rows of a multiple of 128 B
+        (void)vec;
+        const int xoff = (int)align_up((uint64_t)g.pad * g.c, (uint64_t)(128 / elt));
+        const int SR = (int)align_up((uint64_t)(xoff + WC + g.pad * g.c), (uint64_t)(128 / elt));
+        int cs = 0;
+        for (int c = 256; c >= 1 && !cs; --c)
+            if (WC % c == 0 && (c * elt) % 16 == 0 && WC / c <= 256) cs = c;
+        const int BN = (int)align_up((uint64_t)g.k, 16);
+        const int wbytes = (int)align_up((uint64_t)num_kb * BN * 128, 1024);
+        const int sx_bytes = (int)align_up((uint64_t)XR * SR * elt, 1024);
+        const int tabb = (int)align_up((uint64_t)num_kb * KB * 4, 1024);
+        int Ss = 0, SX = 0;
+        for (int sx : {2, 1})
+            for (int sa : {4, 3, 2})
+                if (!Ss && wbytes + sx * sx_bytes + tabb + sa * 16384 <= 222 * 1024) { Ss = sa; SX = sx; }
+        if (cs && Ss && XR <= 256 && (WC * elt) % 16 == 0) {
+            const int64_t tiles = (int64_t)b * ceil_div(g.p, Tr);
+            A.M = (int)(tiles * 128); A.N = g.k; A.BN = BN; A.ldc = g.k; A.num_kb = num_kb; A.kred_taps = (int)RSC;
+            A.mt = 1; A.km = 1; A.b_bytes = 0; A.bn_atoms = (BN * elt + 127) / 128;
+            A.win_qb = Tr; A.sx_cs = xoff; A.sx_sr = SR; A.sx_tx = XR * WC * elt; A.sx_bytes = sx_bytes;
+            A.sx_stages = SX; A.sxw_off = wbytes; A.bres_bytes = wbytes + SX * sx_bytes + tabb; A.stages = Ss;
+            A.nacc = 2; A.tmem_cols = BN * 2 <= 64 ? 64 : BN * 2 <= 128 ? 128 : BN * 2 <= 256 ? 256 : 512;
+            A.bsrc = in1;
+            grid2(1);
+            uint64_t dims[4] = {(uint64_t)cs, (uint64_t)(WC / cs), (uint64_t)g.h, (uint64_t)b};
+            uint64_t str[3] = {(uint64_t)cs * elt, (uint64_t)WC * elt, (uint64_t)g.h * WC * elt};
+            uint32_t box[4] = {(uint32_t)cs, (uint32_t)(WC / cs), 1, 1};
+            if (!make_map(&L.ta, elt, in0, 4, dims, str, box, false, 0)) return -1;
+            return LAUNCH(A_STAGED_FWD, B_RESIDENT, EPI_STORE);
+        }
+    }
     if (type == MUCU_FWD && algo == MUCU_ALGO_IMPLICIT_GEMM) {
         A.M = (int)(b * PQ); A.N = g.k; A.kred = (int)RSC; A.gsrc = in0;
         finalize_tiling(L, elt);

@@ -85,6 +85,9 @@ __global__ void __launch_bounds__(threads_for(AM), 1) tc_conv_gemm(const __grid_
     // the exact-tap MN-major A operand (rows = (r,s,c), K = output pixels) built in
     // shared memory by 256 builder threads (warps 0-3 and 5-8)
     constexpr bool STAGED = (AM == A_STAGED_WG);
+    // A_STAGED_FWD: small-C strided forward, zero workspace (x rows staged by TMA, the
+    // exact-tap K-major A operand built in shared memory, the filter resident)
+    constexpr bool STAGED_FWD = (AM == A_STAGED_FWD);
     constexpr bool A_MN = (AM == A_TMA_MN2 || WIN || STAGED);
     constexpr bool B_MN = (BM_ == B_TMA_MN2 || BM_ == B_TMA_MN3 || BM_ == B_GATHER_WG || BM_ == B_SCALAR_DGRAD ||
                            BM_ == B_SCALAR_WG || BM_ == B_TMA_IM2COL || BM_ == B_GATHER_SMALLC ||
@@ -93,7 +96,7 @@ __global__ void __launch_bounds__(threads_for(AM), 1) tc_conv_gemm(const __grid_
                             AM == A_HALO);
     constexpr bool B_TMA = (BM_ == B_TMA_K2 || BM_ == B_TMA_K3 || BM_ == B_TMA_MN2 || BM_ == B_TMA_MN3 ||
                             BM_ == B_TMA_IM2COL || BM_ == B_TMA_DYROW);
-    constexpr bool B_RES = (BM_ == B_RESIDENT);
+    constexpr bool B_RES = (BM_ == B_RESIDENT);  // (A_STAGED_FWD stages the filter at sB)
     constexpr bool GATHER = !A_TMA || (!B_TMA && !B_RES);
     constexpr bool SPLITK = (EPI == EPI_WGRAD_CHAIN || EPI == EPI_WGRAD_SMALLC || EPI == EPI_WGRAD_S2D ||
                              EPI == EPI_WGRAD_WIN || EPI == EPI_WGRAD_TAPS);
@@ -135,7 +138,7 @@ __global__ void __launch_bounds__(threads_for(AM), 1) tc_conv_gemm(const __grid_
     const int total_tiles = per_z * p.num_z;
 
     if (threadIdx.x == 0) {
-        const uint32_t full_count = STAGED ? 257u : (GATHER ? 128u : 0u) + (A_TMA || B_TMA ? 1u : 0u);
+        const uint32_t full_count = STAGED ? 257u : STAGED_FWD ? 128u : (GATHER ? 128u : 0u) + (A_TMA || B_TMA ? 1u : 0u);
         for (int s = 0; s < S; ++s) {
             mbar_init(smem_u32(&full[s]), full_count);
             mbar_init(smem_u32(&empty[s]), 1);
@@ -151,7 +154,7 @@ __global__ void __launch_bounds__(threads_for(AM), 1) tc_conv_gemm(const __grid_
         }
         for (int j = 0; j < p.sx_stages; ++j) {
             mbar_init(smem_u32(&xfull[j]), 1);
-            mbar_init(smem_u32(&xempty[j]), 256);
+            mbar_init(smem_u32(&xempty[j]), STAGED ? 256 : 128);
         }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
@@ -338,7 +341,122 @@ __global__ void __launch_bounds__(threads_for(AM), 1) tc_conv_gemm(const __grid_
             }
         }
     }
-    if (STAGED && (warp < 4 || warp == 9)) {
+    if constexpr (STAGED_FWD) {
+        // ============== staged-row forward producers (A_STAGED_FWD) ==============
+        // Tile = T output rows (p0 .. p0+T-1) of one image, GEMM row i = t*Q + q.  The
+        // st*(T-1) + R x rows the tile reads are staged by TMA (one box per row) into a
+        // buffer with zeroed left / right margins (the padding taps read zeros); the
+        // K-major A operand (K = the exact (r, s, c) taps) is built from it per k-block;
+        // the filter is staged once per CTA (B resident).  Warp 9 issues the TMA loads,
+        // warps 0-3 (128 threads) build; the epilogue warps drain tiles meanwhile.
+        const int Tr = p.win_qb;                     // output rows per tile
+        const int XR = p.stride * (Tr - 1) + p.R;    // staged x rows per tile
+        const int tiles_img = (p.P + Tr - 1) / Tr;
+        const int xoff = p.sx_cs;                    // element offset of column 0 in a staged row
+        uint8_t* sXr = sBres + p.sxw_off;            // x-row ring after the resident filter
+        if (warp == 9) {
+            if (lane == 0) {
+                int ti = 0;
+                for (int tile = blockIdx.x; tile < total_tiles; tile += gridDim.x, ++ti) {
+                    const int jx = ti % p.sx_stages;
+                    mbar_wait(smem_u32(&xempty[jx]), (uint32_t)(((ti / p.sx_stages) & 1) ^ 1));
+                    const int n_ = tile / tiles_img, p0 = (tile - n_ * tiles_img) * Tr;
+                    const uint32_t xb = smem_u32(&xfull[jx]);
+                    mbar_arrive_tx(xb, (uint32_t)p.sx_tx);
+                    const uint32_t dst = smem_u32(sXr + (size_t)jx * p.sx_bytes) + (uint32_t)(xoff * ELT);
+                    for (int r = 0; r < XR; ++r)
+                        tma_load_4d(dst + (uint32_t)(r * p.sx_sr * ELT), &tmA, xb, 0, 0, p.stride * p0 - p.pad + r, n_);
+                }
+            }
+            __syncwarp();
+        } else if (warp < 4) {
+            const int bt = threadIdx.x;  // 0..127
+            int* tab = (int*)(sXr + (size_t)p.sx_stages * p.sx_bytes);
+            const uint32_t tab_s = smem_u32(tab);
+            uint8_t* sW = sBres;                                         // resident filter, k-block by k-block
+            const int KP = p.num_kb * KB;                                // taps padded to whole k-blocks
+            // tap table: element offset of tap k = (r, s, c) relative to (row 0, column st*q - pad)
+            for (int k = bt; k < KP; k += 128)
+                tab[k] = k < p.kred_taps ? (k / (p.S * p.C)) * p.sx_sr + (k % (p.S * p.C)) - p.pad * p.C + xoff : -1;
+            // zero the staged margins (TMA writes only the interior of each row)
+            for (int j = 0; j < p.sx_stages; ++j)
+                for (int e = bt; e < XR * p.sx_sr; e += 128) {
+                    const int col = e % p.sx_sr;
+                    if (col < xoff || col >= xoff + p.W * p.C) {
+                        if constexpr (ELT == 4) ((float*)(sXr + (size_t)j * p.sx_bytes))[e] = 0.f;
+                        else ((unsigned short*)(sXr + (size_t)j * p.sx_bytes))[e] = 0;
+                    }
+                }
+            // resident filter B[n][k] = w[n][k] (k < R*S*C, else 0), K-major SW128 per k-block
+            const T* wsrc = (const T*)p.bsrc;
+            for (int idx = bt; idx < p.num_kb * p.BN * KB; idx += 128) {
+                const int kb = idx / (p.BN * KB), rem = idx - kb * (p.BN * KB);
+                const int n = rem / KB, e = rem - n * KB, k = kb * KB + e;
+                const T v = (n < p.N && k < p.kred_taps) ? wsrc[(size_t)n * p.kred_taps + k] : (T)0.f;
+                st_shared_elt<T>(smem_u32(sW) + (uint32_t)(kb * p.BN * 128) + kmaj_off(n, e * ELT), v);
+            }
+            fence_proxy_async();
+            asm volatile("bar.sync 2, 128;" ::: "memory");
+            mbar_arrive(smem_u32(bres_bar));
+            // this thread: chunk c8 = bt % 8 (16 B of a k-block row), rows i = bt / 8 + 16 j
+            const int c8 = bt & 7;
+            constexpr int EPC = 16 / ELT;
+            int ai = 0, ti = 0;
+            for (int tile = blockIdx.x; tile < total_tiles; tile += gridDim.x, ++ti) {
+                const int jx = ti % p.sx_stages;
+                int rowoff[8];
+#pragma unroll
+                for (int j = 0; j < 8; ++j) {
+                    const int i = bt / 8 + 16 * j, t = i / p.Q, q = i - t * p.Q;
+                    rowoff[j] = t < Tr ? (p.stride * t * p.sx_sr + p.stride * q * p.C) * ELT : -1;
+                }
+                mbar_wait(smem_u32(&xfull[jx]), (uint32_t)((ti / p.sx_stages) & 1));
+                const uint32_t xs = smem_u32(sXr) + (uint32_t)(jx * p.sx_bytes);
+                for (int kb = 0; kb < p.num_kb; ++kb, ++ai) {
+                    const int s = ai % S;
+                    mbar_wait(smem_u32(&empty[s]), (uint32_t)(((ai / S) & 1) ^ 1));
+                    int tv[EPC];
+#pragma unroll
+                    for (int e = 0; e < EPC; e += 4)
+                        asm volatile("ld.shared.v4.s32 {%0, %1, %2, %3}, [%4];"
+                                     : "=r"(tv[e]), "=r"(tv[e + 1]), "=r"(tv[e + 2]), "=r"(tv[e + 3])
+                                     : "r"(tab_s + (uint32_t)((kb * KB + c8 * EPC + e) * 4)));
+                    const uint32_t aT = smem_u32(sA + (size_t)s * A_BYTES);
+#pragma unroll
+                    for (int j = 0; j < 8; ++j) {
+                        const int i = bt / 8 + 16 * j;
+                        uint32_t w[4] = {0u, 0u, 0u, 0u};
+                        if (rowoff[j] >= 0) {
+                            const uint32_t xr = xs + (uint32_t)rowoff[j];
+                            if constexpr (ELT == 4) {
+#pragma unroll
+                                for (int e = 0; e < 4; ++e)
+                                    if (tv[e] >= 0)
+                                        asm volatile("ld.shared.b32 %0, [%1];" : "=r"(w[e]) : "r"(xr + (uint32_t)(tv[e] * 4)));
+                            } else {
+#pragma unroll
+                                for (int e = 0; e < 4; ++e) {
+                                    unsigned short lo = 0, hi = 0;
+                                    if (tv[2 * e] >= 0)
+                                        asm volatile("ld.shared.u16 %0, [%1];" : "=h"(lo) : "r"(xr + (uint32_t)(tv[2 * e] * 2)));
+                                    if (tv[2 * e + 1] >= 0)
+                                        asm volatile("ld.shared.u16 %0, [%1];" : "=h"(hi) : "r"(xr + (uint32_t)(tv[2 * e + 1] * 2)));
+                                    w[e] = (uint32_t)lo | ((uint32_t)hi << 16);
+                                }
+                            }
+                        }
+                        asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(aT + kmaj_off(i, c8 * 16)),
+                                     "r"(w[0]), "r"(w[1]), "r"(w[2]), "r"(w[3])
+                                     : "memory");
+                    }
+                    fence_proxy_async();
+                    mbar_arrive(smem_u32(&full[s]));
+                }
+                mbar_arrive(smem_u32(&xempty[jx]));
+            }
+        }
+    }
+    if ((STAGED || STAGED_FWD) && (warp < 4 || warp == 9)) {
         // builders / TMA warp only (above)
     } else if (HALO && warp < 4) {
 
@@ -1092,6 +1210,14 @@ __global__ void __launch_bounds__(threads_for(AM), 1) tc_conv_gemm(const __grid_
             // Output row of GEMM row m (phase mode scatters sub-grid rows back to dx).
             long long mrow = m;
             bool rowok = true;
+            if (STAGED_FWD && m < p.M) {
+                // tile = win_qb output rows of one image: row i = t*Q + q of the tile
+                const int tile = m >> 7, i = m & 127, Tr = p.win_qb;
+                const int tiles_img = (p.P + Tr - 1) / Tr;
+                const int n = tile / tiles_img, pr = (tile - n * tiles_img) * Tr + i / p.Q, q = i % p.Q;
+                rowok = i < Tr * p.Q && pr < p.P;
+                mrow = ((long long)n * p.P + pr) * p.Q + q;
+            }
             if (HALO && m < p.M) {
                 // extended-grid row m = ((n*Hx + oh)*W' + ow): junk unless oh < Ho, ow < Wo
                 const int G = m / p.hx_W, ow = m - G * p.hx_W, n = G / p.hx_H, oh = G - n * p.hx_H;

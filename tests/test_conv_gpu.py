@@ -35,6 +35,8 @@ SHAPES = {
     "11x11s4_c3_ragged": (2, 3, 30, 27, 64, 11, 11, 2, 4),  # space-to-depth with ragged super-pixel edges
     "5x5s2_c2_k32": (2, 2, 17, 19, 32, 5, 5, 2, 2),
     "4x4s3_c3_p0": (3, 3, 20, 22, 64, 4, 4, 0, 3),
+    "11x11s4_c3_w32": (2, 3, 35, 32, 64, 11, 11, 2, 4),   # W*C*elt % 16 == 0: staged-row FWD / WGRAD
+    "7x7s2_c3_w32": (3, 3, 30, 32, 64, 7, 7, 3, 2),
     "3x3s2": (2, 64, 14, 14, 128, 3, 3, 1, 2),
     "1x1s1": (3, 64, 10, 10, 96, 1, 1, 0, 1),
     "1x1s2": (2, 64, 14, 14, 128, 1, 1, 0, 2),

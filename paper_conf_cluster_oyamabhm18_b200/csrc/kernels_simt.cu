@@ -130,9 +130,12 @@ struct StoreDense {
 // ------------------------------------------------------------ the kernel --
 // CONTIG_A / CONTIG_B: true when consecutive kk are contiguous in memory
 // (threads of a warp then spread along kk), false when consecutive rows are.
+// K slab per pipeline step: 16 (two FFMA blocks of 8 between barriers).
+constexpr int kBK = 16;
+
 template <int BM, int BN, bool CONTIG_KA, bool CONTIG_KB, class AV, class BV>
 struct TileLoader {
-    static constexpr int BK = 8;
+    static constexpr int BK = kBK;
     static constexpr int NA = BM * BK / kThreads;
     static constexpr int NB = BN * BK / kThreads;
     float ra[NA], rb[NB];
@@ -175,7 +178,7 @@ struct TileLoader {
 template <int BM, int BN, bool CKA, bool CKB, class AV, class BV>
 __device__ __forceinline__ void simt_mainloop(const AV& a, const BV& b, int64_t m0, int64_t n0, int64_t kbeg,
                                               int64_t kend, float (&acc)[BM / 16][BN / 16]) {
-    constexpr int BK = 8, TM = BM / 16, TN = BN / 16;
+    constexpr int BK = kBK, TM = BM / 16, TN = BN / 16;
     __shared__ __align__(16) float As[2][BK][BM + 4];
     __shared__ __align__(16) float Bs[2][BK][BN + 4];
     const int tx = threadIdx.x % 16, ty = threadIdx.x / 16;
@@ -277,12 +280,34 @@ int launch_gemm(const AV& a, const BV& b, const EPI& e, int64_t M, int64_t N, in
     return (int)cudaGetLastError();
 }
 
-// Tile shape by the GEMM's N extent (narrow N wastes less with BN = 64).
+// Tile shape: whole waves of CTAs over the SMs (128 x 128: 2 CTAs per SM, 128 x 64:
+// 3, 64 x 64: 4 by registers) weighted by the FFMA efficiency of the thread tile
+// (8 x 8 > 8 x 4 > 4 x 4 outputs per thread per shared-memory load); small GEMMs
+// (cfg1: AlexNet conv2 at N = 8, 5832 x 192) take the smaller tiles.
 template <bool CKA, bool CKB, class AV, class BV, class EPI>
 int dispatch_gemm(const AV& a, const BV& b, const EPI& e, int64_t M, int64_t N, int64_t Kd, int batch,
                   cudaStream_t st) {
-    if (N <= 64) return launch_gemm<128, 64, CKA, CKB>(a, b, e, M, N, Kd, batch, st);
-    return launch_gemm<128, 128, CKA, CKB>(a, b, e, M, N, Kd, batch, st);
+    static int sms = 0;
+    if (!sms) {
+        int dev = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+        if (sms <= 0) sms = 148;
+    }
+    struct Cand { int bm, bn, per_sm; double eff; };
+    const Cand cands[3] = {{128, 128, 2, 1.0}, {128, 64, 3, 0.9}, {64, 64, 4, 0.75}};
+    int best = 0;
+    double best_cost = 1e300;
+    for (int i = 0; i < 3; ++i) {
+        const Cand& c = cands[i];
+        if (N <= 64 && c.bn == 128) continue;
+        const int64_t tiles = ceil_div(M, c.bm) * ceil_div(N, c.bn) * batch;
+        const double cost = (double)ceil_div(tiles, (int64_t)sms * c.per_sm) * c.per_sm * c.bm * c.bn / c.eff;
+        if (cost < best_cost - 1e-9) { best_cost = cost; best = i; }
+    }
+    if (best == 0) return launch_gemm<128, 128, CKA, CKB>(a, b, e, M, N, Kd, batch, st);
+    if (best == 1) return launch_gemm<128, 64, CKA, CKB>(a, b, e, M, N, Kd, batch, st);
+    return launch_gemm<64, 64, CKA, CKB>(a, b, e, M, N, Kd, batch, st);
 }
 
 }  // namespace
@@ -329,15 +354,23 @@ int simt_dgrad_ig(const Geom& g, int32_t b, float alpha, const float* dy, const 
 
 // WGRAD: dw[k][(r,s,c)] = sum_m dy[m][k] * B(m, (r,s,c)), B = implicit im2col
 // of x (IG) or the explicit col matrix (I2C, row pitch kpitch).
-int simt_wgrad(const Geom& g, int32_t b, float alpha, const float* dy, const float* xin, bool col_input,
-               int32_t kpitch, float beta, float* dw, int num_sms, cudaStream_t st) {
-    constexpr int BM = 128, BN = 128, BK = 8;
+template <int BM, int BN>
+int simt_wgrad_t(const Geom& g, int32_t b, float alpha, const float* dy, const float* xin, bool col_input,
+                 int32_t kpitch, float beta, float* dw, int num_sms, cudaStream_t st) {
+    constexpr int BK = kBK;
     const int64_t rows = g.k, cols = (int64_t)g.r * g.s * g.c, Kd = (int64_t)b * g.p * g.q;
     const int64_t tiles = ceil_div(cols, BN) * ceil_div(rows, BM);
-    // Enough splits for ~2 waves of 2 CTAs/SM, each split >= 256 pixels.
-    int64_t want = std::max<int64_t>(1, (4LL * num_sms + tiles - 1) / tiles);
-    int64_t maxs = std::max<int64_t>(1, Kd / 256);
-    int64_t nsplit = std::min<int64_t>(std::min<int64_t>(want, maxs), 65535);
+    // Split count: waves of 2 CTAs per SM x pixels per split (a pixel of a BM x BN
+    // tile ~ BM*BN/64 cycles at half an SM's FFMA rate) + the ordered hand-over of
+    // the partial tiles (~4000 cycles per split, the deterministic chain).
+    int64_t nsplit = 1;
+    double best = 1e300;
+    const int64_t smax = std::min<int64_t>(std::max<int64_t>(1, Kd / 64), 1024);
+    for (int64_t sp = 1; sp <= smax; ++sp) {
+        const double cost = (double)ceil_div(tiles * sp, 2LL * num_sms) * (double)ceil_div(Kd, sp) * (BM * BN / 64.0) +
+                            (double)sp * 4000.0;
+        if (cost < best) { best = cost; nsplit = sp; }
+    }
     int64_t kps = ceil_div(ceil_div(Kd, nsplit), BK) * BK;
     nsplit = ceil_div(Kd, kps);
     dim3 grid((unsigned)ceil_div(rows, BM), (unsigned)ceil_div(cols, BN), (unsigned)nsplit);
@@ -356,6 +389,13 @@ int simt_wgrad(const Geom& g, int32_t b, float alpha, const float* dy, const flo
     }
     count_launch();
     return (int)cudaGetLastError();
+}
+
+int simt_wgrad(const Geom& g, int32_t b, float alpha, const float* dy, const float* xin, bool col_input,
+               int32_t kpitch, float beta, float* dw, int num_sms, cudaStream_t st) {
+    // rows = K filters: half-empty 128-row tiles for K <= 64 (AlexNet / ResNet conv1)
+    if (g.k <= 64) return simt_wgrad_t<64, 128>(g, b, alpha, dy, xin, col_input, kpitch, beta, dw, num_sms, st);
+    return simt_wgrad_t<128, 128>(g, b, alpha, dy, xin, col_input, kpitch, beta, dw, num_sms, st);
 }
 
 // Winograd BackwardFilter GEMMs: M[z][k][c] = sum_t D[z][t][k] * V[z][t][c], z < 16.

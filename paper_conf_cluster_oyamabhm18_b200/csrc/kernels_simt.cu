@@ -14,6 +14,7 @@
 // of SURVEY 8(c)).  BackwardFilter splits the pixel reduction over
 // CTAs and combines the partial tiles in split order through a per-tile turn
 // counter (no atomics on dw), so dw is deterministic too.
+#include <cuda_bf16.h>
 #include <cuda_runtime.h>
 
 #include <algorithm>
@@ -25,6 +26,12 @@ namespace mucu {
 namespace {
 
 constexpr int kThreads = 256;
+
+__device__ __forceinline__ float to_float(float v) { return v; }
+__device__ __forceinline__ float to_float(__nv_bfloat16 v) { return __bfloat162float(v); }
+template <class T> __device__ __forceinline__ T from_float(float v);
+template <> __device__ __forceinline__ float from_float<float>(float v) { return v; }
+template <> __device__ __forceinline__ __nv_bfloat16 from_float<__nv_bfloat16>(float v) { return __float2bfloat16_rn(v); }
 
 // ------------------------------------------------------------------ views --
 // Dense matrix view: A(i,kk) = p[i*si + kk*sk] (zero outside rows x kdim).
@@ -310,7 +317,90 @@ int dispatch_gemm(const AV& a, const BV& b, const EPI& e, int64_t M, int64_t N, 
     return launch_gemm<64, 64, CKA, CKB>(a, b, e, M, N, Kd, batch, st);
 }
 
+// ------------------------------------------- small-C BackwardData (FFMA) --
+// dx of a layer with C <= 4 input channels (the RGB layer) is a contraction with
+// N = C output columns: no tensor-core tile fits it.  Phase decomposition
+// (P:L56 BackwardData = transposed convolution): dx pixels with
+// (h + pad) % st == a and (w + pad) % st == b0 receive only the taps
+// r = a + st*i, s = b0 + st*j, from dy row / column hh - i, ww - j of the phase
+// sub-grid (h = a - pad + st*hh).  One CTA = a 16 x 16 block of one phase
+// sub-grid of one image, the phase's sub-filter (nr x ns x K x C) staged in
+// shared memory; one thread = one dx pixel, all C channels, fp32 FFMA over
+// (i, j, k) with 16-byte dy loads.  Exact-order sum over (i, j, k) for every
+// pixel: independent of the micro-batch size (I1).
+template <class T, int CMAX>
+__global__ void __launch_bounds__(256) small_c_dgrad_kernel(const T* __restrict__ dy, const T* __restrict__ w, T* dx,
+                                                            int H, int W, int C, int K, int P, int Q, int R, int S,
+                                                            int pad, int st, float alpha, float beta) {
+    extern __shared__ float wsm[];  // [i][j][k][c] of this phase
+    const int a = blockIdx.y / st, b0 = blockIdx.y - (blockIdx.y / st) * st;
+    const int n = blockIdx.z;
+    const int nr = a < R ? (R - a + st - 1) / st : 0, ns = b0 < S ? (S - b0 + st - 1) / st : 0;
+    for (int idx = threadIdx.x; idx < nr * ns * K * C; idx += 256) {
+        const int c = idx % C, t = idx / C, k = t % K, t2 = t / K, j = t2 % ns, i = t2 / ns;
+        wsm[idx] = to_float(w[(((size_t)k * R + a + st * i) * S + b0 + st * j) * C + c]);
+    }
+    __syncthreads();
+    const int hh0 = (pad - a + st - 1) / st > 0 ? (pad - a + st - 1) / st : 0;  // first h >= 0
+    const int ww0 = (pad - b0 + st - 1) / st > 0 ? (pad - b0 + st - 1) / st : 0;
+    const int tiles_w = (W + st - 1) / st / 16 + 1;
+    const int hh = hh0 + (blockIdx.x / tiles_w) * 16 + threadIdx.x / 16;
+    const int ww = ww0 + (blockIdx.x % tiles_w) * 16 + threadIdx.x % 16;
+    const int h = a - pad + st * hh, x = b0 - pad + st * ww;
+    if (h >= H || x >= W) return;
+    float acc[CMAX];
+#pragma unroll
+    for (int c = 0; c < CMAX; ++c) acc[c] = 0.f;
+    for (int i = 0; i < nr; ++i) {
+        const int pp = hh - i;
+        if (pp < 0 || pp >= P) continue;
+        for (int j = 0; j < ns; ++j) {
+            const int qq = ww - j;
+            if (qq < 0 || qq >= Q) continue;
+            const T* d = dy + (((size_t)n * P + pp) * Q + qq) * K;
+            const float* ws = wsm + (size_t)(i * ns + j) * K * C;
+            for (int k = 0; k < K; ++k) {
+                const float v = to_float(d[k]);
+#pragma unroll
+                for (int c = 0; c < CMAX; ++c)
+                    if (c < C) acc[c] = fmaf(v, ws[k * C + c], acc[c]);
+            }
+        }
+    }
+    T* o = dx + (((size_t)n * H + h) * W + x) * C;
+#pragma unroll
+    for (int c = 0; c < CMAX; ++c) {
+        if (c >= C) break;
+        float r = alpha * acc[c];
+        if (beta != 0.f) r += beta * to_float(o[c]);
+        o[c] = from_float<T>(r);
+    }
+}
+
 }  // namespace
+
+int small_c_dgrad(const Geom& g, int32_t b, float alpha, const void* dy, const void* w, float beta, void* dx,
+                  cudaStream_t st) {
+    if (g.c > 4) return -1;
+    const int nr = (g.r + g.stride - 1) / g.stride, ns = (g.s + g.stride - 1) / g.stride;
+    const size_t smem = (size_t)nr * ns * g.k * g.c * sizeof(float);
+    if (smem > 200 * 1024) return -1;
+    const int tiles_h = (g.h + g.stride - 1) / g.stride / 16 + 1, tiles_w = (g.w + g.stride - 1) / g.stride / 16 + 1;
+    dim3 grid((unsigned)(tiles_h * tiles_w), (unsigned)(g.stride * g.stride), (unsigned)b);
+    if (g.math == MUCU_MATH_BF16) {
+        auto k = small_c_dgrad_kernel<__nv_bfloat16, 4>;
+        if (smem > 48 * 1024) cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        k<<<grid, 256, smem, st>>>((const __nv_bfloat16*)dy, (const __nv_bfloat16*)w, (__nv_bfloat16*)dx, g.h, g.w,
+                                   g.c, g.k, g.p, g.q, g.r, g.s, g.pad, g.stride, alpha, beta);
+    } else {
+        auto k = small_c_dgrad_kernel<float, 4>;
+        if (smem > 48 * 1024) cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        k<<<grid, 256, smem, st>>>((const float*)dy, (const float*)w, (float*)dx, g.h, g.w, g.c, g.k, g.p, g.q,
+                                   g.r, g.s, g.pad, g.stride, alpha, beta);
+    }
+    count_launch();
+    return (int)cudaGetLastError();
+}
 
 // FWD implicit GEMM (algorithm (a)): y[m][k] = sum_{(r,s,c)} im2col(x)[m][(r,s,c)] * w[k][(r,s,c)].
 int simt_fwd_ig(const Geom& g, int32_t b, float alpha, const float* x, const float* w, float beta, float* y,

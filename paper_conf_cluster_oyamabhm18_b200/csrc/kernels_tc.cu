@@ -1208,6 +1208,13 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         if (err) return err;
         return DRY(launch_wg_output(g, dg, b, alpha, Mx, beta, out, st));
     }
+    if (type == MUCU_BWD_DATA && algo == MUCU_ALGO_IMPLICIT_GEMM && g.c <= 4 && env_int("MUCU_SMALLC_DGRAD", 1)) {
+        // RGB layer: N = C <= 4 output columns fit no tensor-core tile; zero-workspace
+        // FFMA kernel over the phase sub-filters (kernels_simt.cu small_c_dgrad)
+        if (dry) return 0;
+        const int e = small_c_dgrad(g, b, alpha, in0, in1, beta, out, st);
+        if (e != -1) return e;
+    }
     if (type == MUCU_BWD_DATA && algo == MUCU_ALGO_IMPLICIT_GEMM && g.stride > 1 && g.k % KB == 0 &&
         use_tma_im2col()) {
         // Strided DGRAD by phase decomposition: one stride-1 transposed conv per

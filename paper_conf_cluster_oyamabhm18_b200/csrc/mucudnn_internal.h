@@ -145,6 +145,11 @@ int simt_gemm_nn(int64_t M, int64_t N, int64_t K, float alpha, const float* A, i
                  cudaStream_t st);                                            // C = A[M,K] B[K,N]
 int simt_dgrad_ig(const Geom& g, int32_t b, float alpha, const float* dy, const float* w,
                   float beta, float* dx, cudaStream_t st);
+// BackwardData of a C <= 4 layer (any math; fp32 FFMA, bf16 / fp32 storage), zero
+// workspace: per-phase sub-filter in shared memory, one thread per dx pixel.
+// Returns -1 when the layer does not qualify.
+int small_c_dgrad(const Geom& g, int32_t b, float alpha, const void* dy, const void* w, float beta, void* dx,
+                  cudaStream_t st);
 int simt_wgrad(const Geom& g, int32_t b, float alpha, const float* dy, const float* x_or_col,
                bool col_input, int32_t kpitch, float beta, float* dw, int num_sms, cudaStream_t st);
 

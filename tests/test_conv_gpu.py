@@ -221,3 +221,21 @@ def test_cp_async_gather_producers_still_exact():
     r = subprocess.run([sys.executable, "-m", "pytest", "-q", "-x", os.path.abspath(__file__), "-k",
                         "(c64 or c128) and not cp_async"], env=env, capture_output=True, text=True)
     assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-2000:]
+
+
+@pytest.mark.parametrize("math", [mu.MATH_F32, mu.MATH_TF32, mu.MATH_BF16], ids=["f32", "tf32", "bf16"])
+@pytest.mark.parametrize("name", ["11x11s4_c3", "7x7s2_c3", "5x5s2_c2_k32", "4x4s3_c3_p0", "11x11s4_c3_ragged"])
+def test_small_c_dgrad_alpha_beta_exact(name, math):
+    """Zero-workspace BackwardData of C <= 4 layers (phase sub-filters, FFMA):
+    integer data exact, alpha / beta, micro-batched plan."""
+    shape = SHAPES[name]
+    d = mu.desc(*shape, math)
+    x, w, dy = _inputs(shape, "int", seed=19)
+    n, c, h, wd, k, r, s, pad, st = shape
+    out0 = np.random.default_rng(3).integers(-2, 3, size=(n, h, wd, c)).astype(np.float32)
+    ref = oracle_ref(shape, mu.BWD_DATA, x, w, dy, alpha=2.0, beta=-1.0, out0=out0)
+    if math == mu.MATH_BF16:
+        ref = torch.from_numpy(ref).to(torch.bfloat16).double().numpy()
+    got, _ = run_gpu(d, mu.BWD_DATA, [(mu.IMPLICIT_GEMM, n - 1), (mu.IMPLICIT_GEMM, 1)], x, w, dy, alpha=2.0,
+                     beta=-1.0, out0=out0)
+    assert np.array_equal(got, ref)

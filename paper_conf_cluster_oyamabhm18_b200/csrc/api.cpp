@@ -311,7 +311,8 @@ mucu_status_t run_micro(Handle* hd, const Geom& g, int type, int algo, int32_t b
         }
     } else if (type == MUCU_BWD_DATA) {
         if (algo == MUCU_ALGO_IMPLICIT_GEMM) {
-            e = g.c <= 4 ? small_c_dgrad(g, b, alpha, f0, f1, beta, fo, st) : -1;
+            e = (g.c <= 4 && !(getenv("MUCU_SMALLC_DGRAD") && atoi(getenv("MUCU_SMALLC_DGRAD")) == 0))
+                    ? small_c_dgrad(g, b, alpha, f0, f1, beta, fo, st) : -1;
             if (e == -1) e = simt_dgrad_ig(g, b, alpha, f0, f1, beta, fo, st);
         } else if (algo == MUCU_ALGO_IM2COL_GEMM) {
             const int64_t M = (int64_t)b * g.p * g.q, RSC = (int64_t)g.r * g.s * g.c;

@@ -322,54 +322,72 @@ int dispatch_gemm(const AV& a, const BV& b, const EPI& e, int64_t M, int64_t N, 
 // N = C output columns: no tensor-core tile fits it.  Phase decomposition
 // (P:L56 BackwardData = transposed convolution): dx pixels with
 // (h + pad) % st == a and (w + pad) % st == b0 receive only the taps
-// r = a + st*i, s = b0 + st*j, from dy row / column hh - i, ww - j of the phase
+// r = a + st*i, s = b0 + st*j, from dy pixel (hh - i, ww - j) of the phase
 // sub-grid (h = a - pad + st*hh).  One CTA = a 16 x 16 block of one phase
-// sub-grid of one image, the phase's sub-filter (nr x ns x K x C) staged in
-// shared memory; one thread = one dx pixel, all C channels, fp32 FFMA over
-// (i, j, k) with 16-byte dy loads.  Exact-order sum over (i, j, k) for every
-// pixel: independent of the micro-batch size (I1).
-template <class T, int CMAX>
+// sub-grid of one image: the dy block it reads ((16+nr-1) x (16+ns-1) pixels x K,
+// fp32, row pitch K+4) and the phase's sub-filter [i][j][k][4] are staged in
+// shared memory (each dy element is reused by up to nr*ns pixels); one thread =
+// one dx pixel, all C channels, fp32 FFMA over (i, j, k) with 16-byte shared
+// loads.  The sum order over (i, j, k) is fixed: independent of the micro-batch
+// size (I1).
+template <class T>
 __global__ void __launch_bounds__(256) small_c_dgrad_kernel(const T* __restrict__ dy, const T* __restrict__ w, T* dx,
                                                             int H, int W, int C, int K, int P, int Q, int R, int S,
                                                             int pad, int st, float alpha, float beta) {
-    extern __shared__ float wsm[];  // [i][j][k][c] of this phase
+    extern __shared__ __align__(16) float sm[];
     const int a = blockIdx.y / st, b0 = blockIdx.y - (blockIdx.y / st) * st;
     const int n = blockIdx.z;
     const int nr = a < R ? (R - a + st - 1) / st : 0, ns = b0 < S ? (S - b0 + st - 1) / st : 0;
-    for (int idx = threadIdx.x; idx < nr * ns * K * C; idx += 256) {
-        const int c = idx % C, t = idx / C, k = t % K, t2 = t / K, j = t2 % ns, i = t2 / ns;
-        wsm[idx] = to_float(w[(((size_t)k * R + a + st * i) * S + b0 + st * j) * C + c]);
-    }
-    __syncthreads();
+    const int KP = K + 4, BR = 16 + nr - 1, BC = 16 + ns - 1;
+    float* dys = sm;                               // [BR][BC][KP]
+    float* wsm = sm + (size_t)BR * BC * KP;        // [nr][ns][K][4]
     const int hh0 = (pad - a + st - 1) / st > 0 ? (pad - a + st - 1) / st : 0;  // first h >= 0
     const int ww0 = (pad - b0 + st - 1) / st > 0 ? (pad - b0 + st - 1) / st : 0;
     const int tiles_w = (W + st - 1) / st / 16 + 1;
-    const int hh = hh0 + (blockIdx.x / tiles_w) * 16 + threadIdx.x / 16;
-    const int ww = ww0 + (blockIdx.x % tiles_w) * 16 + threadIdx.x % 16;
+    const int hb = hh0 + (blockIdx.x / tiles_w) * 16, wb = ww0 + (blockIdx.x % tiles_w) * 16;
+    // the phase's sub-filter, channels padded to 4
+    for (int idx = threadIdx.x; idx < nr * ns * K * 4; idx += 256) {
+        const int c = idx & 3, t = idx >> 2, k = t % K, t2 = t / K, jj = t2 % ns, ii = t2 / ns;
+        wsm[idx] = c < C ? to_float(w[(((size_t)k * R + a + st * ii) * S + b0 + st * jj) * C + c]) : 0.f;
+    }
+    // dy block: pixel (pp, qq) = (hb - (nr-1) + row, wb - (ns-1) + col), zero outside dy
+    for (int idx = threadIdx.x; idx < BR * BC * (K / 4); idx += 256) {
+        const int k4 = idx % (K / 4), t = idx / (K / 4), col = t % BC, row = t / BC;
+        const int pp = hb - (nr - 1) + row, qq = wb - (ns - 1) + col;
+        float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
+        if (pp >= 0 && pp < P && qq >= 0 && qq < Q) {
+            const T* d = dy + (((size_t)n * P + pp) * Q + qq) * K + 4 * k4;
+            v = make_float4(to_float(d[0]), to_float(d[1]), to_float(d[2]), to_float(d[3]));
+        }
+        *reinterpret_cast<float4*>(dys + ((size_t)row * BC + col) * KP + 4 * k4) = v;
+    }
+    __syncthreads();
+    const int ty = threadIdx.x / 16, tx = threadIdx.x % 16;
+    const int hh = hb + ty, ww = wb + tx;
     const int h = a - pad + st * hh, x = b0 - pad + st * ww;
     if (h >= H || x >= W) return;
-    float acc[CMAX];
-#pragma unroll
-    for (int c = 0; c < CMAX; ++c) acc[c] = 0.f;
+    float acc[4] = {0.f, 0.f, 0.f, 0.f};
     for (int i = 0; i < nr; ++i) {
-        const int pp = hh - i;
-        if (pp < 0 || pp >= P) continue;
         for (int j = 0; j < ns; ++j) {
-            const int qq = ww - j;
-            if (qq < 0 || qq >= Q) continue;
-            const T* d = dy + (((size_t)n * P + pp) * Q + qq) * K;
-            const float* ws = wsm + (size_t)(i * ns + j) * K * C;
-            for (int k = 0; k < K; ++k) {
-                const float v = to_float(d[k]);
+            const float* d = dys + ((size_t)(ty + nr - 1 - i) * BC + (tx + ns - 1 - j)) * KP;
+            const float* wf = wsm + (size_t)(i * ns + j) * K * 4;
+            for (int k = 0; k < K; k += 4) {
+                const float4 v = *reinterpret_cast<const float4*>(d + k);
+                const float vv[4] = {v.x, v.y, v.z, v.w};
 #pragma unroll
-                for (int c = 0; c < CMAX; ++c)
-                    if (c < C) acc[c] = fmaf(v, ws[k * C + c], acc[c]);
+                for (int u = 0; u < 4; ++u) {
+                    const float4 f = *reinterpret_cast<const float4*>(wf + (k + u) * 4);
+                    acc[0] = fmaf(vv[u], f.x, acc[0]);
+                    acc[1] = fmaf(vv[u], f.y, acc[1]);
+                    acc[2] = fmaf(vv[u], f.z, acc[2]);
+                    acc[3] = fmaf(vv[u], f.w, acc[3]);
+                }
             }
         }
     }
     T* o = dx + (((size_t)n * H + h) * W + x) * C;
 #pragma unroll
-    for (int c = 0; c < CMAX; ++c) {
+    for (int c = 0; c < 4; ++c) {
         if (c >= C) break;
         float r = alpha * acc[c];
         if (beta != 0.f) r += beta * to_float(o[c]);
@@ -381,20 +399,20 @@ __global__ void __launch_bounds__(256) small_c_dgrad_kernel(const T* __restrict_
 
 int small_c_dgrad(const Geom& g, int32_t b, float alpha, const void* dy, const void* w, float beta, void* dx,
                   cudaStream_t st) {
-    if (g.c > 4) return -1;
+    if (g.c > 4 || g.k % 4) return -1;
     const int nr = (g.r + g.stride - 1) / g.stride, ns = (g.s + g.stride - 1) / g.stride;
-    const size_t smem = (size_t)nr * ns * g.k * g.c * sizeof(float);
-    if (smem > 200 * 1024) return -1;
+    const size_t smem = ((size_t)(16 + nr - 1) * (16 + ns - 1) * (g.k + 4) + (size_t)nr * ns * g.k * 4) * sizeof(float);
+    if (smem > 220 * 1024) return -1;
     const int tiles_h = (g.h + g.stride - 1) / g.stride / 16 + 1, tiles_w = (g.w + g.stride - 1) / g.stride / 16 + 1;
     dim3 grid((unsigned)(tiles_h * tiles_w), (unsigned)(g.stride * g.stride), (unsigned)b);
     if (g.math == MUCU_MATH_BF16) {
-        auto k = small_c_dgrad_kernel<__nv_bfloat16, 4>;
-        if (smem > 48 * 1024) cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        auto k = small_c_dgrad_kernel<__nv_bfloat16>;
+        cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         k<<<grid, 256, smem, st>>>((const __nv_bfloat16*)dy, (const __nv_bfloat16*)w, (__nv_bfloat16*)dx, g.h, g.w,
                                    g.c, g.k, g.p, g.q, g.r, g.s, g.pad, g.stride, alpha, beta);
     } else {
-        auto k = small_c_dgrad_kernel<float, 4>;
-        if (smem > 48 * 1024) cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        auto k = small_c_dgrad_kernel<float>;
+        cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         k<<<grid, 256, smem, st>>>((const float*)dy, (const float*)w, (float*)dx, g.h, g.w, g.c, g.k, g.p, g.q,
                                    g.r, g.s, g.pad, g.stride, alpha, beta);
     }

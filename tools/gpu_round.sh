@@ -75,3 +75,23 @@ json.dump({key: int(tot), "_note": "DRAM read+write bytes of one call of the op 
 print("traffic", key, int(tot))
 PY
 fi
+if has extra; then
+  # BASELINE configs 1 / 2-F32 / 3 / 4 (WD) and the non-deterministic reduction mode
+  timeout -s KILL 900 python bench.py --math f32 --layers conv2 --types fwd --batch 8 --ws-mib 8 --policy all \
+    --json-out $OUT/bench_cfg1_alexnet_conv2_f32.json > $OUT/bench_cfg1.log 2>&1; echo "cfg1 rc=$?" | tee -a $OUT/status
+  timeout -s KILL 900 python bench.py --math f32 --steps 5 --no-cpu-baseline --json-out $OUT/bench_alexnet_f32.json \
+    > $OUT/bench_alexnet_f32.log 2>&1; echo "f32 rc=$?" | tee -a $OUT/status
+  timeout -s KILL 900 python bench.py --config resnet18 --math bf16 --wd-mib 480 --no-cpu-baseline \
+    --json-out $OUT/bench_resnet18_bf16_wd480.json > /dev/null 2>&1; echo "wd r18 rc=$?" | tee -a $OUT/status
+  timeout -s KILL 900 python bench.py --config resnet50 --math bf16 --wd-mib 10176 --no-cpu-baseline \
+    --json-out $OUT/bench_resnet50_bf16_wd10176.json > /dev/null 2>&1; echo "wd r50 rc=$?" | tee -a $OUT/status
+  timeout -s KILL 900 python bench.py --config resnet50 --math bf16 --wd-mib 5088 --no-cpu-baseline \
+    --json-out $OUT/bench_resnet50_bf16_wd5088.json > /dev/null 2>&1; echo "wd r50 half rc=$?" | tee -a $OUT/status
+  timeout -s KILL 900 python bench.py --ws-mib 8 --policy undivided --no-cpu-baseline \
+    --json-out $OUT/bench_alexnet_tf32_wr8_undivided.json > /dev/null 2>&1; echo "wr8 und rc=$?" | tee -a $OUT/status
+  for cfg in "alexnet tf32" "resnet50 bf16"; do
+    set -- $cfg
+    timeout -s KILL 900 python bench.py --config $1 --math $2 --nondeterministic --no-cpu-baseline \
+      --json-out $OUT/bench_$1_$2_nondet.json > /dev/null 2>&1; echo "nondet $1 rc=$?" | tee -a $OUT/status
+  done
+fi

@@ -145,7 +145,11 @@ mucu_status_t mucu_output_dims(const mucu_conv_desc_t* desc, int32_t* p, int32_t
  *                     FWD: u = 2, f = st*u, Dr = (st*(u-1) + R - 1)/f + 1, Ds likewise,
  *                          Cs = f*f*C rounded up to 128/elt, Pu = ceil(P/u), Qu = ceil(Q/u):
  *                          u*u*K*Dr*Ds*Cs*elt + b*(Pu+Dr-1)*(Qu+Ds-1)*Cs*elt
- *                     WGRAD with C <= 4 and st*16 % 16 == 0 (BF16: st even) ("window"):
+ *                     WGRAD when the staged-row kernel applies (C*elt < 16, R*S*C <= 512,
+ *                          K <= 256 and a multiple of 128/elt, the x row W*C*elt splits into 16-B-multiple
+ *                          chunks): 148 partial dW tiles, TR = R*S*C rounded up to 128:
+ *                          148 * TR * K * 4  (b-independent; split order fixed: deterministic)
+ *                     else WGRAD with C <= 4 and st*16 % 16 == 0 (BF16: st even) ("window"):
  *                          b*H*Wp*4*elt; atoms of aw bytes (TF32: 128; BF16: the aw in {128, 64, 32}
  *                          minimising align256(R*na*aw/elt), larger aw on ties), tpa = aw/(4*elt)
  *                          taps per atom, na = ceil(S/tpa), Wp = max(st*(Q-1) + na*tpa, W + pad)

@@ -109,6 +109,40 @@ bool win_tc(const Geom& g, int type) {
            (g.stride * 4 * elt) % 16 == 0;
 }
 
+int wgrad_partial_slots(const Geom& g) {
+    if (g.math == MUCU_MATH_F32) return 1;
+    const int64_t tiles = ceil_div(g.k, 128) * ceil_div((int64_t)g.r * g.s * g.c, 128);
+    return (int)std::max<int64_t>(1, std::min<int64_t>(kPartialSlots, ceil_div(kPartialSlots, tiles)));
+}
+
+bool staged_wg_geom(const Geom& g, StagedWg* z) {
+    if (!small_c_tc(g)) return false;
+    const int elt = elt_size(g.math), KB = 128 / elt, atom = 128 / elt;
+    const int64_t RSC = (int64_t)g.r * g.s * g.c;
+    z->TR = (int)align_up((uint64_t)RSC, 128);
+    z->mt = z->TR / 128;
+    z->kd = KB;
+    const int WC = g.w * g.c;
+    const int span = (g.stride * (KB - 1) + g.s) * g.c;  // elements a pixel block reads per x row
+    z->cs = 0; z->bch = 0;
+    for (int c = 256; c >= 1; --c) {
+        if (WC % c || (c * elt) % 16) continue;
+        const int bc = (span + 2 * (c - 1)) / c;  // any start offset inside a chunk
+        if (!z->cs || (int64_t)bc * c < (int64_t)z->bch * z->cs) { z->cs = c; z->bch = bc; }
+    }
+    z->b_bytes = std::max(g.k * 128, (g.k * elt / 128) * KB * 128);
+    z->sx_tx = g.r * z->bch * z->cs * elt;
+    z->sx_bytes = (int)align_up((uint64_t)z->sx_tx, 1024);
+    z->tab_bytes = (int)align_up((uint64_t)z->TR * 4, 1024);
+    const int stage = z->mt * 16384 + z->b_bytes;
+    z->Ss = 0; z->SX = 0;
+    for (int sa : {2, 3})
+        for (int sx : {8, 6, 5, 4, 3, 2})
+            if (!z->Ss && sa * stage + sx * z->sx_bytes + z->tab_bytes <= 210 * 1024) { z->Ss = sa; z->SX = sx; }
+    return z->mt <= 4 && g.k <= 256 && g.k % atom == 0 && z->cs > 0 && g.r <= 256 && z->bch <= 256 && z->Ss &&
+           128 * z->mt * (g.k + 4) * 4 <= 210 * 1024;
+}
+
 Win win_geom(const Geom& g) {
     Win z;
     const int elt = elt_size(g.math);
@@ -157,7 +191,23 @@ mucu_status_t ws_layout(const Geom& g, int type, int algo, int32_t b, WsLayout* 
     if (algo == MUCU_ALGO_IMPLICIT_GEMM) return MUCU_OK;
     if (algo == MUCU_ALGO_IM2COL_GEMM) {
         L->kpitch = (int32_t)align_up(RSC, vec);
-        if (is_pointwise(g)) { L->kpitch = g.c; return MUCU_OK; }
+        // tensor-core BackwardFilter: partial dW slots [P][K][R*S*C] fp32 after the col buffer
+        const int P = type == MUCU_BWD_FILTER ? wgrad_partial_slots(g) : 1;
+        const uint64_t part = P > 1 ? align_up((uint64_t)P * g.k * RSC * 4, 256) : 0;
+        if (is_pointwise(g)) {
+            L->kpitch = g.c;
+            L->b_off = 0; L->b_bytes = part; L->total = part;
+            return MUCU_OK;
+        }
+        StagedWg sw;
+        if (type == MUCU_BWD_FILTER && staged_wg_geom(g, &sw)) {
+            // staged-row kernel + per-split partial dW tiles (b-independent)
+            L->a_off = 0;
+            L->a_bytes = align_up((uint64_t)kPartialSlots * sw.TR * g.k * 4, 256);
+            L->kpitch = 0;
+            L->total = L->a_bytes;
+            return MUCU_OK;
+        }
         if (win_tc(g, type)) {
             const Win z = win_geom(g);
             L->a_off = 0;
@@ -209,7 +259,9 @@ mucu_status_t ws_layout(const Geom& g, int type, int algo, int32_t b, WsLayout* 
             L->a_off = L->fixed_bytes;
             L->a_bytes = align_up((uint64_t)b * PQ * (uint64_t)L->kpitch * elt, 256);
         }
-        L->total = L->a_off + L->a_bytes;
+        L->b_off = L->a_off + L->a_bytes;
+        L->b_bytes = part;
+        L->total = L->b_off + L->b_bytes;
         return MUCU_OK;
     }
     if (type == MUCU_BWD_FILTER) {

@@ -846,6 +846,31 @@ int launch_wgw_transforms(const Geom& g, int32_t b, const void* x, const void* d
     return (int)cudaGetLastError();
 }
 
+// out = alpha * sum_s part[s] + beta * out, splits summed in order (reads of part
+// coalesced along n).
+__global__ void partial_reduce_kernel(int S, int64_t slot, int ldp, int M, int N, bool transpose,
+                                      const float* __restrict__ part, float alpha, float beta, float* __restrict__ out) {
+    pdl_entry();
+    const int64_t total = (int64_t)M * N;
+    for (int64_t idx = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; idx < total;
+         idx += (int64_t)gridDim.x * blockDim.x) {
+        const int m = (int)(idx / N), n = (int)(idx - (int64_t)m * N);
+        const float* p = part + (size_t)m * ldp + n;
+        float acc = 0.f;
+        for (int s = 0; s < S; ++s) acc += __ldg(p + (size_t)s * slot);
+        float* d = transpose ? out + (size_t)n * M + m : out + idx;
+        *d = beta != 0.f ? alpha * acc + beta * *d : alpha * acc;
+    }
+}
+
+int launch_partial_reduce(int S, int64_t slot, int ldp, int M, int N, bool transpose, const float* part,
+                          float alpha, float beta, float* out, cudaStream_t st) {
+    launch_pdl(partial_reduce_kernel, dim3(grid_for((int64_t)M * N, 256)), dim3(256), (size_t)0, st, S, slot, ldp,
+               M, N, transpose, part, alpha, beta, out);
+    count_launch();
+    return (int)cudaGetLastError();
+}
+
 int launch_wgw_output(const Geom& g, float alpha, const float* M, float beta, float* dw, cudaStream_t st) {
     const int at = 128 / elt_size(g.math);
     const int Cp = (int)align_up((uint64_t)g.c, (uint64_t)at), Kp = (int)align_up((uint64_t)g.k, (uint64_t)at);

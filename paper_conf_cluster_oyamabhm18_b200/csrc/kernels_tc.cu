@@ -237,8 +237,9 @@ enum BMode : int {
 //   dw[k][st*d + a][st*e + b][c'] (padding and r >= R / s >= S skipped), reduced.
 // EPI_WGRAD_WIN: row j = (r, atom, tap, c) of the window GEMM -> dw[k][r][atom*taps + tap][c], reduced.
 // EPI_WGRAD_TAPS: row m = exact tap (r, s, c) -> dw[k][m] (A_STAGED_WG), reduced.
+// EPI_WGRAD_PARTIAL: the tile of split z -> out[z][m][n] (fp32, row pitch ldc), plain stores.
 enum EpiMode : int { EPI_STORE = 0, EPI_WGRAD_CHAIN = 1, EPI_WGRAD_SMALLC = 2, EPI_D2S = 3, EPI_WGRAD_S2D = 4,
-                     EPI_WGRAD_WIN = 5, EPI_WGRAD_TAPS = 6 };
+                     EPI_WGRAD_WIN = 5, EPI_WGRAD_TAPS = 6, EPI_WGRAD_PARTIAL = 7 };
 
 struct TcArgs {
     int M, N;                // output rows / cols
@@ -313,6 +314,7 @@ struct TcArgs {
     int sx_cs, sx_sr, sx_stages, sx_bytes, sx_tx, kred_taps;
     int atomic;              // non-deterministic split-K: partials added with red.global.add
     int sxw_off;             // A_STAGED_FWD: byte offset of the x-row ring after the resident filter
+    int part_rows;           // EPI_WGRAD_PARTIAL: GEMM rows per partial slot (slot = part_rows x ldc floats)
     unsigned long long* turns;
     unsigned long long epoch;
 };
@@ -531,7 +533,7 @@ int launch_t(Launch& L, cudaStream_t st, bool dry) {
         1024 + std::max(ring, L.a.stg_bytes) + (2 * L.a.stages + 6 + 2 * L.a.hstages + 2 * L.a.sx_stages) * 8 + 64;
     if (smem > 232448) return -1;
     constexpr bool SPLITK = (EPI == EPI_WGRAD_CHAIN || EPI == EPI_WGRAD_SMALLC || EPI == EPI_WGRAD_S2D ||
-                             EPI == EPI_WGRAD_WIN || EPI == EPI_WGRAD_TAPS);
+                             EPI == EPI_WGRAD_WIN || EPI == EPI_WGRAD_TAPS || EPI == EPI_WGRAD_PARTIAL);
     if (!SPLITK && L.a.cl) return -1;
     L.a.turns = nullptr;
     L.a.epoch = 0;
@@ -991,7 +993,8 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         }
         return err;
     }
-    if (algo == MUCU_ALGO_IM2COL_GEMM && win_tc(g, type)) {
+    StagedWg zw_;
+    if (algo == MUCU_ALGO_IM2COL_GEMM && win_tc(g, type) && !staged_wg_geom(g, &zw_)) {
         // Window WGRAD: dw^T[j][k] = sum over pixels of window(j, m) dy(m, k),
         // rows j = (r, atom, tap, c) over the padded copy xp, columns = the K filters.
         const Win z = win_geom(g);
@@ -1027,7 +1030,7 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         if (z.aw == 32) return LAUNCH(A_TMA_WIN32, B_TMA_DYROW, EPI_WGRAD_WIN);
         return LAUNCH(A_TMA_WIN, B_TMA_DYROW, EPI_WGRAD_WIN);
     }
-    if (algo == MUCU_ALGO_IM2COL_GEMM && s2d_tc(g, type)) {
+    if (algo == MUCU_ALGO_IM2COL_GEMM && s2d_tc(g, type) && !(type == MUCU_BWD_FILTER && staged_wg_geom(g, &zw_))) {
         // Space-to-depth: the strided small-C layer as a stride-1
         // Dr x Ds conv over the super-pixel image with Cs channels -- 128-B
         // channel atoms, so TMA im2col feeds it like any other layer.
@@ -1421,49 +1424,50 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
             }
             return map2(&L.ta, in1, g.k, (uint64_t)Mpix, g.k, atom, KB * A.km, true);
         };
-        if (algo == MUCU_ALGO_IMPLICIT_GEMM && small_c_tc(g) && env_int("MUCU_STAGED", 1)) {
-            // Staged-row BackwardFilter, zero workspace: GEMM rows = the
-            // exact R*S*C taps (no padding but to 128 rows), columns = the K filters,
-            // reduction = output pixels in blocks of KD of one output row.
-            const int TR = (int)align_up((uint64_t)RSC, 128);
-            const int mtS = TR / 128;
+        StagedWg zw;
+        if (((algo == MUCU_ALGO_IMPLICIT_GEMM && env_int("MUCU_STAGED", 1)) || algo == MUCU_ALGO_IM2COL_GEMM) &&
+            staged_wg_geom(g, &zw)) {
+            // Staged-row BackwardFilter: GEMM rows = the exact R*S*C taps
+            // (padded only to 128-row halves), columns = the K filters, reduction = output
+            // pixels in blocks of KD of one output row.  IG (zero workspace): cluster
+            // split-K (6.9).  I2C: every split writes its partial tile to the workspace and
+            // a reduction kernel sums them in split order.
+            A.M = (int)RSC; A.N = g.k; A.ldc = (int)RSC; A.kred_taps = (int)RSC; A.mt = zw.mt; A.BN = g.k;
+            A.bn_atoms = g.k * elt / 128; A.b_bytes = zw.b_bytes; A.km = 1;
+            A.win_qb = (int)ceil_div(g.q, KB);
+            A.sx_cs = zw.cs; A.sx_sr = zw.bch * zw.cs; A.sx_tx = zw.sx_tx; A.sx_bytes = zw.sx_bytes;
+            A.stages = zw.Ss; A.sx_stages = zw.SX; A.bres_bytes = zw.SX * zw.sx_bytes + zw.tab_bytes;
+            A.nacc = zw.mt * A.BN <= 256 ? 2 : 1;
+            const int cols = A.nacc * zw.mt * A.BN;
+            A.tmem_cols = cols <= 64 ? 64 : cols <= 128 ? 128 : cols <= 256 ? 256 : 512;
+            const int64_t nkb = (int64_t)b * g.p * A.win_qb;
             const int WC = g.w * g.c;
-            const int span = (g.stride * (KB - 1) + g.s) * g.c;  // elements a block reads per x row
-            int cs = 0, bch = 0;
-            for (int c = 256; c >= 1; --c) {
-                if (WC % c || (c * elt) % 16) continue;
-                const int bc = (span + 2 * (c - 1)) / c;  // any start offset inside a chunk
-                if (!cs || (int64_t)bc * c < (int64_t)bch * cs) { cs = c; bch = bc; }
-            }
-            const int b_bytes_s = std::max(g.k * 128, (g.k * elt / 128) * KB * 128);
-            const int sx_tx = g.r * bch * cs * elt;
-            const int sx_bytes = (int)align_up((uint64_t)sx_tx, 1024);
-            const int tabb = (int)align_up((uint64_t)TR * 4, 1024);
-            const int stage = mtS * 16384 + b_bytes_s;
-            int Ss = 0, SX = 0;
-            for (int sa : {2, 3})
-                for (int sx : {8, 6, 5, 4, 3, 2})
-                    if (!Ss && sa * stage + sx * sx_bytes + tabb <= 210 * 1024) { Ss = sa; SX = sx; }
-            if (mtS <= 4 && g.k <= 256 && g.k % atom == 0 && cs > 0 && g.r <= 256 && bch <= 256 && Ss &&
-                128 * mtS * (g.k + 4) * 4 <= 210 * 1024) {
-                A.M = (int)RSC; A.N = g.k; A.ldc = (int)RSC; A.kred_taps = (int)RSC; A.mt = mtS; A.BN = g.k;
-                A.bn_atoms = g.k * elt / 128; A.b_bytes = b_bytes_s; A.km = 1;
-                A.win_qb = (int)ceil_div(g.q, KB);
-                A.sx_cs = cs; A.sx_sr = bch * cs; A.sx_tx = sx_tx; A.sx_bytes = sx_bytes;
-                A.stages = Ss; A.sx_stages = SX; A.bres_bytes = SX * sx_bytes + tabb;
-                A.nacc = mtS * A.BN <= 256 ? 2 : 1;
-                const int cols = A.nacc * mtS * A.BN;
-                A.tmem_cols = cols <= 64 ? 64 : cols <= 128 ? 128 : cols <= 256 ? 256 : 512;
-                apply_split(1, (int64_t)b * g.p * A.win_qb, 1, true);  // builders double as epilogue: one unit per CTA
-                uint64_t dims[4] = {(uint64_t)cs, (uint64_t)(WC / cs), (uint64_t)g.h, (uint64_t)b};
-                uint64_t str[3] = {(uint64_t)cs * elt, (uint64_t)WC * elt, (uint64_t)g.h * WC * elt};
-                uint32_t box[4] = {(uint32_t)cs, (uint32_t)bch, (uint32_t)g.r, 1};
-                if (!make_map(&L.ta, elt, in0, 4, dims, str, box, false, 0)) return -1;
-                if (!map3(&L.tb, in1, g.k, g.q, (uint64_t)b * g.p, g.k, (uint64_t)g.q * g.k, atom, KB, 1, true))
-                    return -1;
-                A.tma_bytes = A.bn_atoms * KB * 128;
+            uint64_t dims[4] = {(uint64_t)zw.cs, (uint64_t)(WC / zw.cs), (uint64_t)g.h, (uint64_t)b};
+            uint64_t str[3] = {(uint64_t)zw.cs * elt, (uint64_t)WC * elt, (uint64_t)g.h * WC * elt};
+            uint32_t box[4] = {(uint32_t)zw.cs, (uint32_t)zw.bch, (uint32_t)g.r, 1};
+            if (!make_map(&L.ta, elt, in0, 4, dims, str, box, false, 0)) return -1;
+            if (!map3(&L.tb, in1, g.k, g.q, (uint64_t)b * g.p, g.k, (uint64_t)g.q * g.k, atom, KB, 1, true))
+                return -1;
+            A.tma_bytes = A.bn_atoms * KB * 128;
+            if (algo == MUCU_ALGO_IMPLICIT_GEMM) {
+                apply_split(1, nkb, 1, true);  // builders double as epilogue: one unit per CTA
                 return LAUNCH(A_STAGED_WG, B_TMA_DYROW, EPI_WGRAD_TAPS);
             }
+            // I2C: one split per SM (at most kPartialSlots), partial tiles [split][TR][BN] fp32
+            const int64_t S = std::max<int64_t>(1, std::min<int64_t>(std::min<int64_t>(kPartialSlots, num_sms), nkb));
+            A.num_kb = (int)nkb;
+            A.kb_per_split = (int)ceil_div(nkb, S);
+            const int64_t Sr = ceil_div(nkb, A.kb_per_split);
+            A.cl = 0; A.zsplit = 0; A.atomic = 0; A.stg_bytes = 0;
+            A.num_z = (int)Sr;
+            L.grid = dim3((unsigned)Sr);
+            float* part = (float*)(ws + WL.a_off);
+            A.out = part; A.alpha = 1.f; A.beta = 0.f; A.ldc = g.k;
+            err = LAUNCH(A_STAGED_WG, B_TMA_DYROW, EPI_WGRAD_PARTIAL);
+            if (err) return err;
+            A.part_rows = zw.TR;
+            return DRY(launch_partial_reduce((int)Sr, (int64_t)zw.TR * g.k, g.k, (int)RSC, g.k, true, part, alpha, beta,
+                                             (float*)out, st));
         }
         if (algo == MUCU_ALGO_IM2COL_GEMM && small_c_tc(g)) {
             // RGB-like layer: channel-padded copy of x, padded columns j' = (r, s8, c').
@@ -1493,6 +1497,31 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
             if (!map2(&L.tb, colp, RSC, (uint64_t)Mpix, kp, atom, KB * A.km, true)) return -1;
             map_mn_box(colp, RSC, (uint64_t)Mpix, kp, KB * A.km);
             A.tma_bytes = A.km * (A.mt * a_bytes + A.bn_atoms * KB * 128);
+            const int P = wgrad_partial_slots(g);
+            if (ctx->deterministic && P > 1 && A.cl) {
+                // workspace partials: persistent CTAs over all SMs, split s writes its dW
+                // tile to slot s, a reduction kernel sums the slots in order (no cluster
+                // packing loss, no ordered hand-over)
+                const int64_t tiles = ceil_div(A.N, A.BN) * ceil_div(A.M, 128 * A.mt);
+                const int64_t nkb = A.num_kb;
+                const double E = env_int("MUCU_SPLIT_E", 16) / (double)A.km;
+                int64_t sbest = 1;
+                double best = 1e30;
+                for (int64_t sp = 1; sp <= std::min<int64_t>(P, std::max<int64_t>(1, nkb / 4)); ++sp) {
+                    const double cost = (double)ceil_div(tiles * sp, num_sms) * ((double)ceil_div(nkb, sp) + E);
+                    if (cost < best - 1e-9) { best = cost; sbest = sp; }
+                }
+                A.kb_per_split = (int)ceil_div(nkb, sbest);
+                sbest = ceil_div(nkb, A.kb_per_split);
+                A.cl = 0; A.zsplit = 0; A.atomic = 0; A.stg_bytes = 0;
+                grid2((int)sbest);
+                float* part = (float*)(ws + WL.b_off);
+                A.out = part; A.alpha = 1.f; A.beta = 0.f; A.part_rows = g.k;  // slot = K x R*S*C (ldc = R*S*C)
+                err = LAUNCH(A_TMA_MN2, B_TMA_MN2, EPI_WGRAD_PARTIAL);
+                if (err) return err;
+                return DRY(launch_partial_reduce((int)sbest, (int64_t)g.k * RSC, (int)RSC, g.k, (int)RSC, false, part,
+                                                 alpha, beta, (float*)out, st));
+            }
             return LAUNCH(A_TMA_MN2, B_TMA_MN2, EPI_WGRAD_CHAIN);
         }
         // implicit-im2col B producers load whole 128-B channel atoms of one tap:

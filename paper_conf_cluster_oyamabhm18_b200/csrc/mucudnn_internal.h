@@ -59,6 +59,17 @@ struct Win { int cpx, aw, tpa, na, Wp, M; };  // aw: bytes per swizzle atom (128
 bool win_tc(const Geom& g, int type);
 Win win_geom(const Geom& g);
 
+// Staged-row BackwardFilter of small-C strided layers: GEMM rows =
+// the exact R*S*C taps padded to TR (128-row halves, mt = TR/128), columns = the K
+// filters, k-blocks of kd pixels of one output row; x rows staged in chunks of cs
+// elements (bch chunks per stage), Ss operand stages, SX x stages.
+struct StagedWg { int TR, mt, kd, cs, bch, sx_tx, sx_bytes, tab_bytes, b_bytes, Ss, SX; };
+bool staged_wg_geom(const Geom& g, StagedWg* z);
+// I2C BackwardFilter of those layers: the staged kernel writes the partial dW tile
+// of each of its (up to kPartialSlots) pixel splits to the workspace and a
+// reduction kernel sums them in split order (deterministic, all SMs busy).
+constexpr int kPartialSlots = 148;
+
 // Workspace layout of one micro-configuration (all offsets 256-B aligned).
 // `fixed` = b-independent prefix (padded filter / Winograd U) computed once per
 // call and shared by the call's micro-batches of the same algorithm.
@@ -177,6 +188,16 @@ int launch_wg_output(const Geom& g, bool dgrad, int32_t b, float alpha, const fl
 int launch_wgw_transforms(const Geom& g, int32_t b, const void* x, const void* dy, void* V, void* D, int64_t Tp,
                           cudaStream_t st);
 int launch_wgw_output(const Geom& g, float alpha, const float* M, float beta, float* dw, cudaStream_t st);
+// out = alpha * sum_{s < S} part[s] + beta * out over an M x N matrix, the split partials
+// part[s][m][n] at slot stride `slot` (elements) and row pitch `ldp`; out[m][n] (row pitch
+// N), or out[n][m] (row pitch M) when `transpose`.  Summed in split order s = 0, 1, ...
+// (deterministic).
+int launch_partial_reduce(int S, int64_t slot, int ldp, int M, int N, bool transpose, const float* part,
+                          float alpha, float beta, float* out, cudaStream_t st);
+// Tensor-core I2C BackwardFilter of large-C layers: partial dW slots reserved in the
+// workspace (deterministic split-K over all SMs): ceil(148 / dW tiles of 128 x 128),
+// 1 = no partial slots.
+int wgrad_partial_slots(const Geom& g);
 // F32: M[z][k][c] = sum_t D[z][t][k] * V[z][t][c], z < 16 (SIMT).
 int simt_gemm_tt(int64_t K, int64_t C, int64_t Tp, const float* V, const float* D, float* M, int64_t ldt,
                  cudaStream_t st);

@@ -99,7 +99,7 @@ __global__ void __launch_bounds__(threads_for(AM), 1) tc_conv_gemm(const __grid_
     constexpr bool B_RES = (BM_ == B_RESIDENT);  // (A_STAGED_FWD stages the filter at sB)
     constexpr bool GATHER = !A_TMA || (!B_TMA && !B_RES);
     constexpr bool SPLITK = (EPI == EPI_WGRAD_CHAIN || EPI == EPI_WGRAD_SMALLC || EPI == EPI_WGRAD_S2D ||
-                             EPI == EPI_WGRAD_WIN || EPI == EPI_WGRAD_TAPS);
+                             EPI == EPI_WGRAD_WIN || EPI == EPI_WGRAD_TAPS || EPI == EPI_WGRAD_PARTIAL);
     constexpr bool A_ASYNC = (AM == A_GATHER_FWD || AM == A_GATHER_DGRAD || AM == A_GATHER_SMALLC_PAD);
     constexpr bool B_ASYNC = (BM_ == B_GATHER_WG || BM_ == B_GATHER_SMALLC_PAD);
     // MN-major atoms: 8-row (bf16, SWIZZLE_128B) or 4-row (tf32, 128B_BASE32B) groups.
@@ -1413,6 +1413,21 @@ __global__ void __launch_bounds__(threads_for(AM), 1) tc_conv_gemm(const __grid_
 #pragma unroll
                         for (int j = 0; j < 32; ++j) dofs[j] = nb + j < p.N ? j : -1;
                         rmw32(d, dofs, (size_t)p.ldc, v, p.alpha, bsplit, p.atomic);
+                    }
+                } else if constexpr (EPI == EPI_WGRAD_PARTIAL) {
+                    // the split's partial tile: out[z][m][nb + j] (rows < part_rows, plain stores)
+                    float* d = outF + (size_t)z * p.part_rows * p.ldc + (size_t)m * p.ldc + nb;
+                    if (m >= p.part_rows) {
+                    } else if (nb + 32 <= p.N && (p.ldc & 3) == 0) {
+#pragma unroll
+                        for (int j = 0; j < 32; j += 4)
+                            *reinterpret_cast<float4*>(d + j) =
+                                make_float4(p.alpha * __uint_as_float(v[j]), p.alpha * __uint_as_float(v[j + 1]),
+                                            p.alpha * __uint_as_float(v[j + 2]), p.alpha * __uint_as_float(v[j + 3]));
+                    } else {
+#pragma unroll
+                        for (int j = 0; j < 32; ++j)
+                            if (nb + j < p.N) d[j] = p.alpha * __uint_as_float(v[j]);
                     }
                 } else if constexpr (EPI == EPI_WGRAD_TAPS) {
                     // row m = exact tap (r, s, c) -> dw[k = nb + j][m]

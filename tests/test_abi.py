@@ -82,8 +82,13 @@ def test_workspace_bf16_resnet_and_pointwise():
     U = 16 * 64 * 64 * 2
     assert mu.workspace_size(d, mu.FWD, mu.WINOGRAD, 1) - U == 4_816_896
     p = mu.desc(256, 256, 56, 56, 64, 1, 1, 0, 1, mu.MATH_BF16)
-    for t in (mu.FWD, mu.BWD_DATA, mu.BWD_FILTER):
+    for t in (mu.FWD, mu.BWD_DATA):
         assert mu.workspace_size(p, t, mu.IM2COL_GEMM, 256) == 0          # im2col(x) == x
+    # BackwardFilter: no im2col, but ceil(148 / (1 x 2 dW tiles)) = 74 partial dW slots of
+    # K x R*S*C fp32 (deterministic split-K over all SMs)
+    assert mu.workspace_size(p, mu.BWD_FILTER, mu.IM2COL_GEMM, 256) == 74 * 64 * 256 * 4
+    pf = mu.desc(256, 256, 56, 56, 64, 1, 1, 0, 1, mu.MATH_F32)
+    assert mu.workspace_size(pf, mu.BWD_FILTER, mu.IM2COL_GEMM, 256) == 0  # F32 SIMT: ordered chain
     ds = mu.desc(256, 256, 56, 56, 512, 1, 1, 0, 2, mu.MATH_BF16)
     assert mu.workspace_size(ds, mu.FWD, mu.IM2COL_GEMM, 1) == 401_408    # 784 * 256 * 2
 
@@ -100,7 +105,9 @@ def test_workspace_small_c_tensor_core():
     # C*elt < 16 B on tensor cores, stride 1: I2C FWD/WGRAD keep x with channels padded to 16 B
     d = mu.desc(4, 3, 224, 224, 64, 7, 7, 3, 1, mu.MATH_BF16)
     assert mu.workspace_size(d, mu.FWD, mu.IM2COL_GEMM, 2) == 2 * 224 * 224 * 16
-    assert mu.workspace_size(d, mu.BWD_FILTER, mu.IM2COL_GEMM, 1) == 224 * 224 * 16
+    # WGRAD: staged-row kernel with 148 partial dW tiles of 256 (147 taps) x 64 fp32
+    assert mu.workspace_size(d, mu.BWD_FILTER, mu.IM2COL_GEMM, 1) == 148 * 256 * 64 * 4
+    assert mu.workspace_size(d, mu.BWD_FILTER, mu.IM2COL_GEMM, 4) == 148 * 256 * 64 * 4  # b-independent
 
 
 def test_workspace_space_to_depth():
@@ -111,18 +118,22 @@ def test_workspace_space_to_depth():
     a256 = lambda v: -(-v // 256) * 256  # noqa: E731
     xs = 29 * 29 * 192 * 4
     assert mu.workspace_size(d, mu.FWD, mu.IM2COL_GEMM, 2) == a256(4 * 64 * 4 * 192 * 4) + a256(2 * xs)
-    # WGRAD, window form: 4-channel pixels, tpa = 8 taps per 128-B atom, na = 2,
-    # Wp = max(4*54 + 16, 224 + 2) = 232
-    assert mu.workspace_size(d, mu.BWD_FILTER, mu.IM2COL_GEMM, 3) == a256(3 * 224 * 232 * 4 * 4)
+    # WGRAD: staged-row kernel, 148 partial dW tiles of 384 (363 taps) x 64 fp32
+    assert mu.workspace_size(d, mu.BWD_FILTER, mu.IM2COL_GEMM, 3) == a256(148 * 384 * 64 * 4)
     # DGRAD: dx super-pixels of f = 8 (u = 2; 8*8*3 = 192 <= 256 columns), Dr = 10 // 4 + 2 = 4
     assert mu.workspace_size(d, mu.BWD_DATA, mu.IM2COL_GEMM, 4) == a256(192 * 16 * 64 * 4)
     # ResNet conv1 BF16 (stride 2): FWD u = 2, f = 4: Dr = (2*1 + 7 - 1) // 4 + 1 = 3, Cs = 48 -> 64,
     # 56 x 56 output super-pixels, 58 x 58 input super-pixels, filter 4K x 9 x 64.
     d = mu.desc(2, 3, 224, 224, 64, 7, 7, 3, 2, mu.MATH_BF16)
     assert mu.workspace_size(d, mu.FWD, mu.IM2COL_GEMM, 2) == a256(4 * 64 * 9 * 64 * 2) + a256(2 * 58 * 58 * 64 * 2)
-    # WGRAD window: 64-B atoms (one 8-tap atom per filter row: 7*32 = 224 GEMM rows instead of
-    # 7*64 with 128-B atoms), tpa = 8, na = 1, Wp = max(2*111 + 8, 224 + 3) = 230 -> 232
-    assert mu.workspace_size(d, mu.BWD_FILTER, mu.IM2COL_GEMM, 2) == a256(2 * 224 * 232 * 4 * 2)
+    # WGRAD: staged-row kernel, 148 partial tiles of 256 (147 taps) x 64 fp32
+    assert mu.workspace_size(d, mu.BWD_FILTER, mu.IM2COL_GEMM, 2) == a256(148 * 256 * 64 * 4)
+    # window form when the x row (W*C*elt) is not a multiple of 16 B: 64-B atoms (one 8-tap atom
+    # per filter row), tpa = 8, na = 1, Wp = max(2*(Q-1) + 8, W + 3) rounded up to 4
+    d = mu.desc(2, 3, 223, 223, 64, 7, 7, 3, 2, mu.MATH_BF16)  # W*C = 669: no chunking
+    q = (223 + 6 - 7) // 2 + 1
+    wp = -(-max(2 * (q - 1) + 8, 223 + 3) // 4) * 4
+    assert mu.workspace_size(d, mu.BWD_FILTER, mu.IM2COL_GEMM, 2) == a256(2 * 223 * wp * 4 * 2)
     # DGRAD: f = 4 (4*4*3 = 48 columns), Dr = 6 // 2 + 2 = 5: filter 48 x 25*64
     assert mu.workspace_size(d, mu.BWD_DATA, mu.IM2COL_GEMM, 2) == a256(48 * 25 * 64 * 2)
     # stride 3, BF16: 3*8 B is not a multiple of 16 -> WGRAD keeps the space-to-depth image

@@ -309,6 +309,7 @@ struct TcArgs {
     // through DSMEM; split groups of cl are ordered by turn counters (turns.cu), one
     // per (batch, tile, row slab).  stg_bytes: the epilogue's staging over the ring.
     int cl, stg_bytes;
+    unsigned long long* tickets;  // ordered split groups: per-tile group tickets (turns.cu pool)
     // A_STAGED_WG: x-row chunks of sx_cs elements (sx_sr = elements per staged row), sx_stages
     // stages of sx_bytes (sx_tx delivered by TMA), kred_taps = R*S*C GEMM rows
     int sx_cs, sx_sr, sx_stages, sx_bytes, sx_tx, kred_taps;
@@ -551,13 +552,16 @@ int launch_t(Launch& L, cudaStream_t st, bool dry) {
     // tile, row slab) orders the groups' additions into dw.
     if (SPLITK && L.a.cl) {
         const int64_t splits = L.a.zsplit ? L.a.zsplit : L.a.num_z;
+        L.a.tickets = nullptr;
         if (splits > L.a.cl) {
             const int64_t per_z = ceil_div(L.a.M, 128 * L.a.mt) * ceil_div(L.a.N, L.a.BN);
-            TurnRange tr;
-            const int e = alloc_turns(per_z * (L.a.num_z / splits) * L.a.cl, &tr);
+            TurnRange tr, tk;
+            int e = alloc_turns(per_z * (L.a.num_z / splits) * L.a.cl, &tr);
+            if (!e) e = alloc_turns(per_z * (L.a.num_z / splits), &tk);
             if (e) return e;
             L.a.turns = tr.ctr;
             L.a.epoch = tr.epoch;
+            L.a.tickets = tk.ctr;
         }
     }
     static int configured = 0;  // per instantiation
@@ -1462,10 +1466,9 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
             A.num_z = (int)Sr;
             L.grid = dim3((unsigned)Sr);
             float* part = (float*)(ws + WL.a_off);
-            A.out = part; A.alpha = 1.f; A.beta = 0.f; A.ldc = g.k;
+            A.out = part; A.alpha = 1.f; A.beta = 0.f; A.ldc = g.k; A.part_rows = zw.TR;
             err = LAUNCH(A_STAGED_WG, B_TMA_DYROW, EPI_WGRAD_PARTIAL);
             if (err) return err;
-            A.part_rows = zw.TR;
             return DRY(launch_partial_reduce((int)Sr, (int64_t)zw.TR * g.k, g.k, (int)RSC, g.k, true, part, alpha, beta,
                                              (float*)out, st));
         }

@@ -11,6 +11,19 @@
 // Two TMEM accumulators (2 x BN columns) let the epilogue of tile i overlap
 // the mainloop of tile i+1 (tmem_full / tmem_empty barriers).
 
+// Ticket counter of this launch (value (epoch << 20) + tickets taken; a value of an
+// older launch counts as 0): returns this caller's ticket 0, 1, 2, ...
+__device__ __forceinline__ int take_ticket(unsigned long long* c, unsigned long long epoch) {
+    unsigned long long old = *(volatile unsigned long long*)c;
+    for (;;) {
+        const bool fresh = (old >> 20) == epoch;
+        const unsigned long long want = fresh ? old + 1 : (epoch << 20) + 1;
+        const unsigned long long prev = atomicCAS(c, old, want);
+        if (prev == old) return fresh ? (int)(old & 0xFFFFFull) : 0;
+        old = prev;
+    }
+}
+
 // dw element (offset from the batch's dw base) of BackwardFilter GEMM element
 // (row m, column n) for each split-K epilogue layout; -1 = padding (no element).
 template <int EPI, int ELT>
@@ -173,6 +186,34 @@ __global__ void __launch_bounds__(threads_for(AM), 1) tc_conv_gemm(const __grid_
     asm volatile("griddepcontrol.wait;" ::: "memory");
     asm volatile("griddepcontrol.launch_dependents;" :::);
 
+    // Cluster split-K with ordered split groups: a cluster's group (= which k-range of
+    // its tile it reduces, and its place in the tile's addition order) is a ticket
+    // taken when the cluster starts, not its cluster id, so a group only ever waits
+    // for groups that were already running -- no dependency on the scheduling order
+    // of clusters (GPC packing, concurrent kernels).  The k-range of group g is fixed,
+    // so the summation order, and dw, do not depend on which cluster got which ticket.
+    int g_ticket = -1;
+    if constexpr (SPLITK) {
+        if (p.cl && p.tickets) {
+            __shared__ int s_tk;
+            const int rho = blockIdx.x % p.cl, c = blockIdx.x / p.cl;
+            const int nu = per_z * (p.zsplit ? p.num_z / p.zsplit : 1);
+            if (threadIdx.x == 0 && rho == 0) s_tk = take_ticket(p.tickets + (c % nu), p.epoch);
+            asm volatile("barrier.cluster.arrive.release;\n\tbarrier.cluster.wait.acquire;" ::: "memory");
+            if (threadIdx.x == 0 && rho != 0) {
+                uint32_t ra;
+                asm("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(ra) : "r"(smem_u32(&s_tk)), "r"(0));
+                int v;
+                asm volatile("ld.shared::cluster.s32 %0, [%1];" : "=r"(v) : "r"(ra) : "memory");
+                s_tk = v;
+            }
+            __syncthreads();
+            g_ticket = s_tk;
+            // rank 0 may not leave (and drop its shared memory) before the others read it
+            asm volatile("barrier.cluster.arrive.release;\n\tbarrier.cluster.wait.acquire;" ::: "memory");
+        }
+    }
+
     // tile -> (m0, n0, z, k-block range)
     // Cluster split-K (p.cl > 0, one unit per CTA): CTA `tile` is rank tile % cl of
     // cluster c = tile / cl; cluster c = (split group g, batch, output tile), g
@@ -183,7 +224,7 @@ __global__ void __launch_bounds__(threads_for(AM), 1) tc_conv_gemm(const __grid_
             const int rho = tile % p.cl, c = tile / p.cl;
             const int nbatch = p.zsplit ? p.num_z / p.zsplit : 1;
             const int nu = per_z * nbatch;
-            const int g = c / nu, u = c - g * nu;
+            const int g = g_ticket >= 0 ? g_ticket : c / nu, u = c % nu;
             const int batch = u / per_z;
             rem = u - batch * per_z;
             const int split = g * p.cl + rho;
@@ -1556,7 +1597,7 @@ __global__ void __launch_bounds__(threads_for(AM), 1) tc_conv_gemm(const __grid_
                 const int rho = blockIdx.x % p.cl, c = blockIdx.x / p.cl;
                 const int nbatch = p.zsplit ? p.num_z / p.zsplit : 1;
                 const int nu = per_z * nbatch;
-                const int g = c / nu, u = c - g * nu;
+                const int g = g_ticket >= 0 ? g_ticket : c / nu, u = c % nu;
                 const int batch = u / per_z, rem = u - batch * per_z;
                 const int ntile = rem / mt;
                 const int m0 = (rem - ntile * mt) * BMt, n0 = ntile * p.BN;

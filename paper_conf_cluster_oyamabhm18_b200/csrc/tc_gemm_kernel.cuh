@@ -195,7 +195,7 @@ __global__ void __launch_bounds__(threads_for(AM), 1) tc_conv_gemm(const __grid_
     int g_ticket = -1;
     if constexpr (SPLITK) {
         if (p.cl && p.tickets) {
-            __shared__ int s_tk;
+            int& s_tk = ((int*)tmem_slot)[1];  // (dynamic shared memory: the upper half of the TMEM slot)
             const int rho = blockIdx.x % p.cl, c = blockIdx.x / p.cl;
             const int nu = per_z * (p.zsplit ? p.num_z / p.zsplit : 1);
             if (threadIdx.x == 0 && rho == 0) s_tk = take_ticket(p.tickets + (c % nu), p.epoch);

@@ -30,6 +30,7 @@
 #include <cuda_bf16.h>
 #include <cuda_runtime.h>
 
+#include <climits>
 #include <cstdio>
 #include <cstring>
 #include <mutex>
@@ -316,6 +317,7 @@ struct TcArgs {
     int atomic;              // non-deterministic split-K: partials added with red.global.add
     int sxw_off;             // A_STAGED_FWD: byte offset of the x-row ring after the resident filter
     int part_rows;           // EPI_WGRAD_PARTIAL: GEMM rows per partial slot (slot = part_rows x ldc floats)
+    int m64;                 // MN-major A: the tile's last 128-row half has <= 64 valid rows -> M = 64 MMAs
     unsigned long long* turns;
     unsigned long long epoch;
 };
@@ -878,6 +880,9 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
             if (const int km = env_int("MUCU_KM", 0)) A.km = km;
         }
         size_stages(A);
+        // one row tile whose last 128-row half holds <= 64 filters (K = 64, 192, ...): that
+        // half issues M = 64 MMAs (the MN-major dy operand is read for 64 rows, not 128)
+        A.m64 = !qrow && A.M <= 128 * A.mt && A.M - 128 * (A.mt - 1) <= 64 && env_int("MUCU_M64", 1);
         const int64_t tiles = ceil_div(A.N, A.BN) * ceil_div(A.M, 128 * A.mt) * batches;
         // qrow > 0: k-blocks are KD-pixel pieces of output rows of qrow pixels (window WGRAD)
         if (qrow) A.win_qb = (int)ceil_div(qrow, KB * A.km);

@@ -1071,6 +1071,9 @@ __global__ void __launch_bounds__(threads_for(AM), 1) tc_conv_gemm(const __grid_
         const uint32_t idesc = (1u << 4) | (Elt<ELT>::fmt << 7) | (Elt<ELT>::fmt << 10) |
                                ((A_MN ? 1u : 0u) << 15) | ((B_MN ? 1u : 0u) << 16) |
                                ((uint32_t)(p.BN >> 3) << 17) | ((128u >> 4) << 24);
+        // p.m64: the last 128-row half of the tile holds <= 64 valid rows -> M = 64 MMAs
+        // (half the A operand reads; accumulator rows in TMEM lanes 0-15 of each quadrant)
+        const uint32_t idesc64 = (idesc & ~(0x1Fu << 24)) | ((64u >> 4) << 24);
         int s = 0;
         uint32_t ph = 0;
         int acc = 0;
@@ -1171,7 +1174,8 @@ __global__ void __launch_bounds__(threads_for(AM), 1) tc_conv_gemm(const __grid_
                                                 WAW == 64 ? 4u : 6u)
                                     : A_MN  ? sdesc(aH + kofs + j * UMMA_K * 128, KDm * 128, MN_SBO, MN_LAYOUT)
                                             : sdesc(aH + j * 32, 16, 1024);
-                                mma_elect<ELT>(dtm + (uint32_t)(hh * p.BN), ad, bd, idesc,
+                                mma_elect<ELT>(dtm + (uint32_t)(hh * p.BN), ad, bd,
+                                               (A_MN && hh == MT - 1 && p.m64) ? idesc64 : idesc,
                                                (kb > kb_begin || jj > 0 || j > 0) ? 1u : 0u);
                             }
                         }
@@ -1224,7 +1228,10 @@ __global__ void __launch_bounds__(threads_for(AM), 1) tc_conv_gemm(const __grid_
 #pragma unroll
                         for (int j = 0; j < 32; ++j) v[j] = 0u;
                     }
-                    const uint32_t dst = stg + (uint32_t)(((hh * 128 + row) * pitch + c0) * 4);
+                    const bool h64 = p.m64 && hh == p.mt - 1;  // M = 64 half: rows 16*q4 + lane (lane < 16)
+                    if (h64 && lane >= 16) continue;
+                    const int srow = h64 ? 16 * q4 + lane : row;
+                    const uint32_t dst = stg + (uint32_t)(((hh * 128 + srow) * pitch + c0) * 4);
 #pragma unroll
                     for (int j = 0; j < 32; j += 4)
                         asm volatile("st.shared.v4.f32 [%0], {%1, %2, %3, %4};" ::"r"(dst + j * 4),
@@ -1247,7 +1254,9 @@ __global__ void __launch_bounds__(threads_for(AM), 1) tc_conv_gemm(const __grid_
             // with L2 reductions after a beta prescale launch.
             const float bsplit = p.beta;
             auto drain = [&](const int hh) {
-            const int m = m0 + 128 * hh + row;
+            // M = 64 half: TMEM lane 32*q4 + l (l < 16) holds row 16*q4 + l
+            const bool h64 = p.m64 && hh == p.mt - 1;
+            const int m = h64 ? (lane < 16 ? m0 + 128 * hh + 16 * q4 + lane : INT_MAX) : m0 + 128 * hh + row;
             // Output row of GEMM row m (phase mode scatters sub-grid rows back to dx).
             long long mrow = m;
             bool rowok = true;

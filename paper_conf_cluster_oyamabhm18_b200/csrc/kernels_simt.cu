@@ -41,6 +41,23 @@ struct Dense {
     __device__ __forceinline__ float at(int64_t i, int64_t kk) const {
         return (i < rows && kk < kdim) ? __ldg(p + i * si + kk * sk) : 0.f;
     }
+    // row-contiguous loads: a thread keeps one row for the whole main loop
+    struct Row { const float* q; bool ok; };
+    __device__ __forceinline__ Row row(int64_t i) const { return Row{p + i * si, i < rows}; }
+    __device__ __forceinline__ float get(const Row& r, int64_t kk) const {
+        return (r.ok && kk < kdim) ? __ldg(r.q + kk * sk) : 0.f;
+    }
+    // four consecutive kk (kk % 4 == 0): one 16-byte load when contiguous and aligned
+    __device__ __forceinline__ void at4(int64_t i, int64_t kk, int64_t kend, float (&o)[4]) const {
+        const float* q = p + i * si + kk * sk;
+        if (sk == 1 && i < rows && kk + 3 < kdim && kk + 3 < kend && (((uintptr_t)q) & 15) == 0) {
+            const float4 v = __ldg(reinterpret_cast<const float4*>(q));
+            o[0] = v.x; o[1] = v.y; o[2] = v.z; o[3] = v.w;
+            return;
+        }
+#pragma unroll
+        for (int e = 0; e < 4; ++e) o[e] = kk + e < kend ? at(i, kk + e) : 0.f;
+    }
     __device__ __forceinline__ void batch(int z) { p += z * batch_stride; }
 };
 
@@ -63,6 +80,35 @@ struct Im2col {
         if ((unsigned)h >= (unsigned)H || (unsigned)w >= (unsigned)W) return 0.f;
         return __ldg(x + (((int64_t)n * H + h) * W + w) * C + c);
     }
+    // kk .. kk+3 of one pixel row: one decomposition, one 16-byte load when the four
+    // channels belong to one tap and are aligned (C % 4 == 0)
+    __device__ __forceinline__ void at4(int64_t m64, int64_t kk64, int64_t kend, float (&o)[4]) const {
+        if (m64 < rows && kk64 + 3 < RSC && kk64 + 3 < kend) {
+            const uint32_t m = (uint32_t)m64, kk = (uint32_t)kk64;
+            const uint32_t rs = dC.div(kk), c = kk - rs * (uint32_t)C;
+            if (c + 3 < (uint32_t)C) {
+                const uint32_t n = dPQ.div(m), rem = m - n * (uint32_t)(P * Q);
+                const uint32_t pp = dQ.div(rem), q = rem - pp * (uint32_t)Q;
+                const uint32_t r = dS.div(rs), s = rs - r * (uint32_t)S;
+                const int h = (int)(pp * st + r) - pad, w = (int)(q * st + s) - pad;
+                if ((unsigned)h >= (unsigned)H || (unsigned)w >= (unsigned)W) {
+                    o[0] = o[1] = o[2] = o[3] = 0.f;
+                    return;
+                }
+                const float* src = x + (((int64_t)n * H + h) * W + w) * C + c;
+                if ((((uintptr_t)src) & 15) == 0) {
+                    const float4 v = __ldg(reinterpret_cast<const float4*>(src));
+                    o[0] = v.x; o[1] = v.y; o[2] = v.z; o[3] = v.w;
+                } else {
+#pragma unroll
+                    for (int e = 0; e < 4; ++e) o[e] = __ldg(src + e);
+                }
+                return;
+            }
+        }
+#pragma unroll
+        for (int e = 0; e < 4; ++e) o[e] = kk64 + e < kend ? at(m64, kk64 + e) : 0.f;
+    }
     __device__ __forceinline__ void batch(int) {}
 };
 Im2col make_im2col(const float* x, int64_t rows, const Geom& g) {
@@ -74,6 +120,23 @@ Im2col make_im2col(const float* x, int64_t rows, const Geom& g) {
 struct Im2colT {
     Im2col v;
     __device__ __forceinline__ float at(int64_t j, int64_t m) const { return v.at(m, j); }
+    // the (r,s,c) of a thread's row is decomposed once; each pixel then costs two divisions
+    struct Row { const float* xc; int r, s; bool ok; };
+    __device__ __forceinline__ Row row(int64_t j64) const {
+        if (j64 >= v.RSC) return Row{v.x, 0, 0, false};
+        const uint32_t j = (uint32_t)j64, rs = v.dC.div(j), c = j - rs * (uint32_t)v.C;
+        const uint32_t r = v.dS.div(rs), s = rs - r * (uint32_t)v.S;
+        return Row{v.x + c, (int)r - v.pad, (int)s - v.pad, true};
+    }
+    __device__ __forceinline__ float get(const Row& rw, int64_t m64) const {
+        if (!rw.ok || m64 >= v.rows) return 0.f;
+        const uint32_t m = (uint32_t)m64;
+        const uint32_t n = v.dPQ.div(m), rem = m - n * (uint32_t)(v.P * v.Q);
+        const uint32_t p = v.dQ.div(rem), q = rem - p * (uint32_t)v.Q;
+        const int h = (int)(p * v.st) + rw.r, w = (int)(q * v.st) + rw.s;
+        if ((unsigned)h >= (unsigned)v.H || (unsigned)w >= (unsigned)v.W) return 0.f;
+        return __ldg(rw.xc + (((int64_t)n * v.H + h) * v.W + w) * v.C);
+    }
 };
 
 // DGRAD gather of dy: row i = dx pixel (n,h,w), kk = (r,s,k):
@@ -96,6 +159,34 @@ struct DgradGather {
         if (p * st != (uint32_t)ph || q * st != (uint32_t)pw || p >= (uint32_t)P || q >= (uint32_t)Q) return 0.f;
         return __ldg(dy + (((int64_t)n * P + p) * Q + q) * K + k);
     }
+    // kk .. kk+3: four consecutive k of one tap (K % 4 == 0): one decomposition, one load
+    __device__ __forceinline__ void at4(int64_t m64, int64_t kk64, int64_t kend, float (&o)[4]) const {
+        if (m64 < rows && kk64 + 3 < RSK && kk64 + 3 < kend) {
+            const uint32_t kk = (uint32_t)kk64, rs = dK.div(kk), k = kk - rs * (uint32_t)K;
+            if (k + 3 < (uint32_t)K) {
+                const uint32_t m = (uint32_t)m64;
+                const uint32_t n = dHW.div(m), rem = m - n * (uint32_t)(H * W);
+                const uint32_t h = dW.div(rem), w = rem - h * (uint32_t)W;
+                const uint32_t r = dS.div(rs), s = rs - r * (uint32_t)S;
+                const int ph = (int)(h + pad) - (int)r, pw = (int)(w + pad) - (int)s;
+                o[0] = o[1] = o[2] = o[3] = 0.f;
+                if (ph < 0 || pw < 0) return;
+                const uint32_t p = dSt.div((uint32_t)ph), q = dSt.div((uint32_t)pw);
+                if (p * st != (uint32_t)ph || q * st != (uint32_t)pw || p >= (uint32_t)P || q >= (uint32_t)Q) return;
+                const float* src = dy + (((int64_t)n * P + p) * Q + q) * K + k;
+                if ((((uintptr_t)src) & 15) == 0) {
+                    const float4 v = __ldg(reinterpret_cast<const float4*>(src));
+                    o[0] = v.x; o[1] = v.y; o[2] = v.z; o[3] = v.w;
+                } else {
+#pragma unroll
+                    for (int e = 0; e < 4; ++e) o[e] = __ldg(src + e);
+                }
+                return;
+            }
+        }
+#pragma unroll
+        for (int e = 0; e < 4; ++e) o[e] = kk64 + e < kend ? at(m64, kk64 + e) : 0.f;
+    }
     __device__ __forceinline__ void batch(int) {}
 };
 
@@ -108,6 +199,13 @@ struct DgradFilter {
         if (j >= C || kk64 >= (int64_t)RS * K) return 0.f;
         const uint32_t kk = (uint32_t)kk64, rs = dK.div(kk), k = kk - rs * (uint32_t)K;
         return __ldg(w + ((int64_t)k * RS + rs) * C + j);
+    }
+    struct Row { const float* q; bool ok; };
+    __device__ __forceinline__ Row row(int64_t j) const { return Row{w + j, j < C}; }
+    __device__ __forceinline__ float get(const Row& r, int64_t kk64) const {
+        if (!r.ok || kk64 >= (int64_t)RS * K) return 0.f;
+        const uint32_t kk = (uint32_t)kk64, rs = dK.div(kk), k = kk - rs * (uint32_t)K;
+        return __ldg(r.q + ((int64_t)k * RS + rs) * C);
     }
     __device__ __forceinline__ void batch(int) {}
 };
@@ -140,35 +238,70 @@ struct StoreDense {
 // K slab per pipeline step: 16 (two FFMA blocks of 8 between barriers).
 constexpr int kBK = 16;
 
+// row context of a row-contiguous operand (views without one are only loaded k-contiguous)
+template <class V, bool CONTIG> struct RowOf { using type = typename V::Row; };
+template <class V> struct RowOf<V, true> { using type = int; };
+
 template <int BM, int BN, bool CONTIG_KA, bool CONTIG_KB, class AV, class BV>
 struct TileLoader {
     static constexpr int BK = kBK;
     static constexpr int NA = BM * BK / kThreads;
     static constexpr int NB = BN * BK / kThreads;
     float ra[NA], rb[NB];
+    typename RowOf<AV, CONTIG_KA>::type arow;  // row-contiguous: the thread's row is fixed (t % BM)
+    typename RowOf<BV, CONTIG_KB>::type brow;
 
+    __device__ __forceinline__ void init(const AV& a, const BV& b, int64_t m0, int64_t n0) {
+        if constexpr (!CONTIG_KA) arow = a.row(m0 + threadIdx.x % BM);
+        if constexpr (!CONTIG_KB) brow = b.row(n0 + threadIdx.x % BN);
+    }
+
+    // k-contiguous operands: a thread loads 4 consecutive k of a row (element e = 4g + u:
+    // group g of rows, k offset 4*(t % (BK/4)) + u); row-contiguous: one k per element.
     __device__ __forceinline__ static void a_coord(int e, int& il, int& kl) {
         const int t = threadIdx.x;
-        if (CONTIG_KA) { kl = t % BK; il = t / BK + e * (kThreads / BK); }
+        if (CONTIG_KA) { kl = 4 * (t % (BK / 4)) + (e & 3); il = t / (BK / 4) + (e >> 2) * (kThreads * 4 / BK); }
         else           { il = t % BM; kl = t / BM + e * (kThreads / BM); }
     }
     __device__ __forceinline__ static void b_coord(int e, int& jl, int& kl) {
         const int t = threadIdx.x;
-        if (CONTIG_KB) { kl = t % BK; jl = t / BK + e * (kThreads / BK); }
+        if (CONTIG_KB) { kl = 4 * (t % (BK / 4)) + (e & 3); jl = t / (BK / 4) + (e >> 2) * (kThreads * 4 / BK); }
         else           { jl = t % BN; kl = t / BN + e * (kThreads / BN); }
     }
     __device__ __forceinline__ void load(const AV& a, const BV& b, int64_t m0, int64_t n0, int64_t k0, int64_t kend) {
+        if constexpr (CONTIG_KA) {
 #pragma unroll
-        for (int e = 0; e < NA; ++e) {
-            int il, kl; a_coord(e, il, kl);
-            int64_t kk = k0 + kl;
-            ra[e] = kk < kend ? a.at(m0 + il, kk) : 0.f;
+            for (int g = 0; g < NA / 4; ++g) {
+                int il, kl; a_coord(4 * g, il, kl);
+                float o[4];
+                a.at4(m0 + il, k0 + kl, kend, o);
+#pragma unroll
+                for (int u = 0; u < 4; ++u) ra[4 * g + u] = o[u];
+            }
+        } else {
+#pragma unroll
+            for (int e = 0; e < NA; ++e) {
+                int il, kl; a_coord(e, il, kl);
+                int64_t kk = k0 + kl;
+                ra[e] = kk < kend ? a.get(arow, kk) : 0.f;
+            }
         }
+        if constexpr (CONTIG_KB) {
 #pragma unroll
-        for (int e = 0; e < NB; ++e) {
-            int jl, kl; b_coord(e, jl, kl);
-            int64_t kk = k0 + kl;
-            rb[e] = kk < kend ? b.at(n0 + jl, kk) : 0.f;
+            for (int g = 0; g < NB / 4; ++g) {
+                int jl, kl; b_coord(4 * g, jl, kl);
+                float o[4];
+                b.at4(n0 + jl, k0 + kl, kend, o);
+#pragma unroll
+                for (int u = 0; u < 4; ++u) rb[4 * g + u] = o[u];
+            }
+        } else {
+#pragma unroll
+            for (int e = 0; e < NB; ++e) {
+                int jl, kl; b_coord(e, jl, kl);
+                int64_t kk = k0 + kl;
+                rb[e] = kk < kend ? b.get(brow, kk) : 0.f;
+            }
         }
     }
     __device__ __forceinline__ void store(float (*As)[BM + 4], float (*Bs)[BN + 4]) const {
@@ -179,9 +312,23 @@ struct TileLoader {
     }
 };
 
+// Resident CTAs per SM the register budget is pinned to (64 x 64: 4 x 256 threads x
+// 64 registers; larger tiles: 2 x 256 x 128).
+constexpr int ctas_per_sm(int bm, int bn) { return bm * bn <= 64 * 64 ? 4 : 2; }
+
+// Thread tile: TM x TN outputs; with 8 they are two 4-wide blocks half a tile apart
+// (rows ty*4 + i and BM/2 + ty*4 + i), so a warp's 16 tx read 16 consecutive float4
+// of a shared-memory row (2 wavefronts, no bank conflicts) instead of 16 float4 at a
+// 32-byte stride (4-way conflicts).
+template <int T, int B>
+__device__ __forceinline__ int frag_off(int t, int i) {
+    if constexpr (T == 8) return t * 4 + (i & 3) + (i >> 2) * (B / 2);
+    else return t * T + i;
+}
+
 // Main loop shared by all SIMT contractions: accumulates the BM x BN tile at
-// (m0, n0) over kk in [kbeg, kend).  acc[i][j] belongs to row ty*TM+i,
-// column tx*TN+j of the tile.
+// (m0, n0) over kk in [kbeg, kend).  acc[i][j] belongs to row frag_off<TM,BM>(ty, i),
+// column frag_off<TN,BN>(tx, j) of the tile.
 template <int BM, int BN, bool CKA, bool CKB, class AV, class BV>
 __device__ __forceinline__ void simt_mainloop(const AV& a, const BV& b, int64_t m0, int64_t n0, int64_t kbeg,
                                               int64_t kend, float (&acc)[BM / 16][BN / 16]) {
@@ -195,6 +342,7 @@ __device__ __forceinline__ void simt_mainloop(const AV& a, const BV& b, int64_t 
         for (int j = 0; j < TN; ++j) acc[i][j] = 0.f;
     if (kbeg >= kend) return;
     TileLoader<BM, BN, CKA, CKB, AV, BV> ld;
+    ld.init(a, b, m0, n0);
     ld.load(a, b, m0, n0, kbeg, kend);
     ld.store(As[0], Bs[0]);
     __syncthreads();
@@ -207,12 +355,12 @@ __device__ __forceinline__ void simt_mainloop(const AV& a, const BV& b, int64_t 
             float af[TM], bf[TN];
 #pragma unroll
             for (int i = 0; i < TM; i += 4) {
-                float4 v = *reinterpret_cast<const float4*>(&As[buf][k][ty * TM + i]);
+                float4 v = *reinterpret_cast<const float4*>(&As[buf][k][frag_off<TM, BM>(ty, i)]);
                 af[i] = v.x; af[i + 1] = v.y; af[i + 2] = v.z; af[i + 3] = v.w;
             }
 #pragma unroll
             for (int j = 0; j < TN; j += 4) {
-                float4 v = *reinterpret_cast<const float4*>(&Bs[buf][k][tx * TN + j]);
+                float4 v = *reinterpret_cast<const float4*>(&Bs[buf][k][frag_off<TN, BN>(tx, j)]);
                 bf[j] = v.x; bf[j + 1] = v.y; bf[j + 2] = v.z; bf[j + 3] = v.w;
             }
 #pragma unroll
@@ -227,7 +375,7 @@ __device__ __forceinline__ void simt_mainloop(const AV& a, const BV& b, int64_t 
 }
 
 template <int BM, int BN, bool CKA, bool CKB, class AV, class BV, class EPI>
-__global__ void __launch_bounds__(kThreads) simt_gemm_kernel(AV a, BV b, EPI epi, int64_t Kd) {
+__global__ void __launch_bounds__(kThreads, ctas_per_sm(BM, BN)) simt_gemm_kernel(AV a, BV b, EPI epi, int64_t Kd) {
     constexpr int TM = BM / 16, TN = BN / 16;
     a.batch(blockIdx.z); b.batch(blockIdx.z); epi.batch(blockIdx.z);
     const int64_t m0 = (int64_t)blockIdx.x * BM, n0 = (int64_t)blockIdx.y * BN;  // M on grid.x (no 65535 cap)
@@ -235,7 +383,11 @@ __global__ void __launch_bounds__(kThreads) simt_gemm_kernel(AV a, BV b, EPI epi
     simt_mainloop<BM, BN, CKA, CKB>(a, b, m0, n0, 0, Kd, acc);
     const int tx = threadIdx.x % 16, ty = threadIdx.x / 16;
 #pragma unroll
-    for (int i = 0; i < TM; ++i) epi.template row<TN>(m0 + ty * TM + i, n0 + tx * TN, acc[i]);
+    for (int i = 0; i < TM; ++i)
+#pragma unroll
+        for (int j = 0; j < TN; j += 4)
+            epi.template row<4>(m0 + frag_off<TM, BM>(ty, i), n0 + frag_off<TN, BN>(tx, j),
+                                *reinterpret_cast<const float(*)[4]>(&acc[i][j]));
 }
 
 // WGRAD: dw[K][RSC] (+)= alpha * sum over the split's pixel range.  Splits of
@@ -244,7 +396,7 @@ __global__ void __launch_bounds__(kThreads) simt_gemm_kernel(AV a, BV b, EPI epi
 // beta) and publishes tag(epoch, s).  blockIdx.z = split, so all CTAs of split
 // s are dispatched before any of split s + 1 (no deadlock).
 template <int BM, int BN, class AV, class BV>
-__global__ void __launch_bounds__(kThreads) simt_wgrad_kernel(AV a, BV b, float* dw, int64_t rows, int64_t cols,
+__global__ void __launch_bounds__(kThreads, ctas_per_sm(BM, BN)) simt_wgrad_kernel(AV a, BV b, float* dw, int64_t rows, int64_t cols,
                                                               int64_t Kd, int64_t k_per_split, float alpha,
                                                               float beta, unsigned long long* turns,
                                                               unsigned long long epoch) {
@@ -261,11 +413,11 @@ __global__ void __launch_bounds__(kThreads) simt_wgrad_kernel(AV a, BV b, float*
     const int tx = threadIdx.x % 16, ty = threadIdx.x / 16;
 #pragma unroll
     for (int i = 0; i < TM; ++i) {
-        int64_t r = m0 + ty * TM + i;
+        int64_t r = m0 + frag_off<TM, BM>(ty, i);
         if (r >= rows) continue;
 #pragma unroll
         for (int j = 0; j < TN; ++j) {
-            int64_t cidx = n0 + tx * TN + j;
+            int64_t cidx = n0 + frag_off<TN, BN>(tx, j);
             if (cidx >= cols) continue;
             float* d = dw + r * cols + cidx;
             float v = alpha * acc[i][j];
@@ -287,8 +439,7 @@ int launch_gemm(const AV& a, const BV& b, const EPI& e, int64_t M, int64_t N, in
     return (int)cudaGetLastError();
 }
 
-// Tile shape: whole waves of CTAs over the SMs (128 x 128: 2 CTAs per SM, 128 x 64:
-// 3, 64 x 64: 4 by registers) weighted by the FFMA efficiency of the thread tile
+// Tile shape: whole waves of CTAs over the SMs (ctas_per_sm resident CTAs) weighted by the FFMA efficiency of the thread tile
 // (8 x 8 > 8 x 4 > 4 x 4 outputs per thread per shared-memory load); small GEMMs
 // (cfg1: AlexNet conv2 at N = 8, 5832 x 192) take the smaller tiles.
 template <bool CKA, bool CKB, class AV, class BV, class EPI>
@@ -302,7 +453,8 @@ int dispatch_gemm(const AV& a, const BV& b, const EPI& e, int64_t M, int64_t N, 
         if (sms <= 0) sms = 148;
     }
     struct Cand { int bm, bn, per_sm; double eff; };
-    const Cand cands[3] = {{128, 128, 2, 1.0}, {128, 64, 3, 0.9}, {64, 64, 4, 0.75}};
+    const Cand cands[3] = {{128, 128, ctas_per_sm(128, 128), 1.0}, {128, 64, ctas_per_sm(128, 64), 0.9},
+                           {64, 64, ctas_per_sm(64, 64), 0.75}};
     int best = 0;
     double best_cost = 1e300;
     for (int i = 0; i < 3; ++i) {

@@ -2,7 +2,7 @@
 # Round measurement on a B200 box (run via gpurun from the repo root):
 #   tests, smoke, benches, the ncu launch list of the default bench step and a
 #   full-set capture of its dominant kernel.  Every step has its own timeout.
-# usage: tools/gpu_round.sh TAG [steps...]   steps: tests smoke bench others launches full
+# usage: tools/gpu_round.sh TAG [steps...]   steps: tests smoke bench others launches full extra ops
 set -u
 TAG=${1:-r01}; shift
 STEPS=${*:-"tests smoke bench others launches full"}
@@ -94,4 +94,12 @@ if has extra; then
     timeout -s KILL 900 python bench.py --config $1 --math $2 --nondeterministic --no-cpu-baseline \
       --json-out $OUT/bench_$1_$2_nondet.json > /dev/null 2>&1; echo "nondet $1 rc=$?" | tee -a $OUT/status
   done
+fi
+if has ops; then
+  # per-op ncu --set full summaries (tools/prof_ops.sh): the F32 dominant op, Winograd
+  # (transforms + batched GEMM), the TF32 WGRAD/DGRAD IG GEMMs, ResNet-50 layer1 3x3 BF16
+  bash tools/prof_ops.sh $OUT/ops alexnet:f32:conv2:WGRAD:IG:256 alexnet:f32:conv2:FWD:IG:256 \
+    alexnet:f32:conv3:FWD:WG:32 alexnet:f32:conv5:WGRAD:WG:32 alexnet:tf32:conv2:WGRAD:IG:256 \
+    alexnet:tf32:conv2:DGRAD:IG:256 alexnet:tf32:conv1:FWD:I2C:64 resnet50:bf16:layer1.0.conv2:FWD:IG:256 \
+    resnet50:bf16:layer1.0.conv2:DGRAD:IG:256 resnet50:bf16:layer1.0.conv2:WGRAD:IG:256 2>&1 | tee -a $OUT/status
 fi

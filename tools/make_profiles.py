@@ -43,6 +43,11 @@ if os.path.exists(rep):
         f.write(run(os.path.join(tools, "ncu_lines.py"), rep, "15"))
 for b in glob.glob(os.path.join(src, "bench_*.json")):
     shutil.copy(b, os.path.join(dst, f"{rnd}_{os.path.basename(b)}"))
+for t in sorted(glob.glob(os.path.join(src, "ops", "*.txt"))):
+    shutil.copy(t, os.path.join(dst, f"{rnd}_ops_{os.path.basename(t)}"))
+for extra in ("status", "tests.log", "gpu.txt"):
+    if os.path.exists(os.path.join(src, extra)):
+        shutil.copy(os.path.join(src, extra), os.path.join(dst, f"{rnd}_{extra.replace('.log', '')}.txt"))
 tj = os.path.join(src, "traffic.json")
 if os.path.exists(tj):
     shutil.copy(tj, os.path.join(dst, "traffic.json"))

@@ -1,6 +1,6 @@
 """Per-kernel summary of an ncu report with several launches (tools/prof_ops.sh).
 
-    python tools/ncu_ops.py REP.ncu-rep [top_stall_lines]
+    python tools/ncu_ops.py REP.ncu-rep [top_stall_lines [kernel_regex]]
 """
 import csv, io, subprocess, sys
 
@@ -10,6 +10,8 @@ KEYS = [("gpu__time_duration.sum", "us", 1e-3), ("dram__bytes_read.sum", "MB", 1
         ("lts__throughput.avg.pct_of_peak_sustained_elapsed", "%lts", 1),
         ("gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed", "%dram", 1),
         ("sm__throughput.avg.pct_of_peak_sustained_elapsed", "%sm", 1),
+        ("sm__inst_executed_pipe_fma.avg.pct_of_peak_sustained_active", "%fma", 1),
+        ("smsp__issue_active.avg.pct_of_peak_sustained_active", "%issue", 1),
         ("launch__grid_size", "grid", 1), ("launch__registers_per_thread", "regs", 1)]
 raw = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
 rr = list(csv.reader(io.StringIO(raw)))
@@ -33,10 +35,10 @@ for row in rr[2:]:
     print(f"{name:70s} " + " ".join(out))
 if len(sys.argv) > 2:
     import os
-    # stall samples per CUDA line of the first tc_conv_gemm launch (tools/ncu_lines.py logic)
+    # stall samples per CUDA line of the first launch matching kernel_regex (default tc_conv) (tools/ncu_lines.py logic)
     from collections import defaultdict
     txt = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "cuda,sass",
-                          "-k", "regex:tc_conv", "-c", "1"], capture_output=True, text=True).stdout
+                          "-k", "regex:" + (sys.argv[3] if len(sys.argv) > 3 else "tc_conv"), "-c", "1"], capture_output=True, text=True).stdout
     agg, srcs, fname, header = defaultdict(float), {}, "?", None
     for row in csv.reader(io.StringIO(txt)):
         if not row:

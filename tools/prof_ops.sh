@@ -13,6 +13,6 @@ for spec in "$@"; do
     python tools/profile_one.py --config $cfg --math $math --layer $layer --type $typ --algo $algo --b $b --n $n \
     > $OUT/$name.log 2>&1
   echo "$spec rc=$?"
-  python tools/ncu_ops.py $OUT/$name.ncu-rep 25 > $OUT/$name.txt 2>&1
+  python tools/ncu_ops.py $OUT/$name.ncu-rep 25 "${KREGEX:-tc_conv|simt}" > $OUT/$name.txt 2>&1
   [ "${KEEP:-0}" = 1 ] || rm -f $OUT/$name.ncu-rep
 done

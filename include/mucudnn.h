@@ -68,7 +68,9 @@ typedef enum {
     MUCU_ALGO_IMPLICIT_GEMM = 0,     /* (a) zero workspace                                   */
     MUCU_ALGO_IM2COL_GEMM = 1,       /* (b) explicit im2col (+col2im for DGRAD) + GEMM        */
     MUCU_ALGO_WINOGRAD_2X2_3X3 = 2,  /* (c) Winograd F(2x2,3x3), Lavin & Gray (ref [23])      */
-    MUCU_NUM_ALGOS = 3
+    MUCU_ALGO_FFT = 3,               /* (d) frequency domain, one F x F tile per image         */
+    MUCU_ALGO_FFT_TILING = 4,        /* (e) frequency domain on 32 x 32 tiles   */
+    MUCU_NUM_ALGOS = 5
 } mucu_algo_t;
 
 /* Arithmetic: F32 = fp32 SIMT FFMA; TF32 = fp32 storage, tcgen05 kind::tf32;
@@ -147,7 +149,7 @@ mucu_status_t mucu_output_dims(const mucu_conv_desc_t* desc, int32_t* p, int32_t
  *                          u*u*K*Dr*Ds*Cs*elt + b*(Pu+Dr-1)*(Qu+Ds-1)*Cs*elt
  *                     WGRAD when the staged-row kernel applies (C*elt < 16, R*S*C <= 512,
  *                          K <= 256 and a multiple of 128/elt, the x row W*C*elt splits into 16-B-multiple
- *                          chunks): 148 partial dW tiles, TR = R*S*C rounded up to 128:
+ *                          chunks, TR - R*S*C <= R*S*C/4): 148 partial dW tiles, TR = R*S*C rounded up to 128:
  *                          148 * TR * K * 4  (b-independent; split order fixed: deterministic)
  *                     else WGRAD with C <= 4 and st*16 % 16 == 0 (BF16: st even) ("window"):
  *                          b*H*Wp*4*elt; atoms of aw bytes (TF32: 128; BF16: the aw in {128, 64, 32}
@@ -161,8 +163,18 @@ mucu_status_t mucu_output_dims(const mucu_conv_desc_t* desc, int32_t* p, int32_t
  *   WG  DGRAD:        16*C*K*elt + 16*b*T'*K*elt + 16*b*T'*C*4, T' = ceil(H/2)*ceil(W/2)
  *   WG  WGRAD:        F(3x3,2x2), Tp = b*T rounded up to 256, Cp / Kp = C / K
  *                     rounded up to 128/elt:  16*Tp*Cp*elt + 16*Tp*Kp*elt + 16*Kp*Cp*4
+ *   FFT / FFT_TILING (F32 only, stride 1): complex spectra of B = F*(F/2+1)
+ *                     bins, 8 bytes per value, planes Pl = b*ty*tx tiles.  Output grid E = P x Q
+ *                     (FWD, WGRAD) or H x W (DGRAD); FFT: one tile per image, F = the smallest
+ *                     power of two >= max(Eh + R - 1, Ew + S - 1), 8 <= F <= 32; FFT_TILING:
+ *                     F = 32, tiles of min(Eh, 33-R) x min(Ew, 33-S) outputs (R, S <= 16),
+ *                     ty x tx = ceil(Eh/Th) x ceil(Ew/Tw):
+ *                     FWD:   8*B*K*C + 8*B*Pl*C + 8*B*Pl*K
+ *                     DGRAD: 8*B*K*C + 8*B*Pl*K + 8*B*Pl*C
+ *                     WGRAD: 8*B*Pl*C + 8*B*Pl*K + 8*B*K*C
  * ceil_e rounds up to a multiple of 16/elt elements.  UNSUPPORTED if the
- * algorithm is ineligible (WG needs R=S=3, stride 1, pad <= 2). */
+ * algorithm is ineligible (WG needs R=S=3, stride 1, pad <= 2; FFT / FFT_TILING
+ * need MUCU_MATH_F32 and stride 1). */
 mucu_status_t mucu_workspace_size(const mucu_conv_desc_t* desc, mucu_conv_type_t type,
                                   mucu_algo_t algo, int32_t micro_n, uint64_t* bytes);
 

@@ -17,11 +17,11 @@ import numpy as np
 _LIB_PATH = os.path.join(os.path.dirname(os.path.abspath(__file__)), "lib", "libmucudnn.so")
 
 FWD, BWD_DATA, BWD_FILTER = 0, 1, 2
-IMPLICIT_GEMM, IM2COL_GEMM, WINOGRAD = 0, 1, 2
-NUM_ALGOS = 3
+IMPLICIT_GEMM, IM2COL_GEMM, WINOGRAD, FFT, FFT_TILING = 0, 1, 2, 3, 4
+NUM_ALGOS = 5
 MATH_F32, MATH_TF32, MATH_BF16 = 0, 1, 2
 POLICY_ALL, POLICY_POW2, POLICY_UNDIVIDED = 0, 1, 2
-ALGO_NAMES = {IMPLICIT_GEMM: "IG", IM2COL_GEMM: "I2C", WINOGRAD: "WG"}
+ALGO_NAMES = {IMPLICIT_GEMM: "IG", IM2COL_GEMM: "I2C", WINOGRAD: "WG", FFT: "FFT", FFT_TILING: "FFTT"}
 TYPE_NAMES = {FWD: "FWD", BWD_DATA: "DGRAD", BWD_FILTER: "WGRAD"}
 MATH_NAMES = {MATH_F32: "f32", MATH_TF32: "tf32", MATH_BF16: "bf16"}
 
@@ -111,6 +111,18 @@ def _u64(a):
     return a, a.ctypes.data_as(ctypes.POINTER(ctypes.c_uint64))
 
 
+def _full_tables(time_ns, ws):
+    """Timing tables with fewer than NUM_ALGOS algorithm rows get the missing rows as
+    'not measured' (time -1, workspace 0)."""
+    t = np.asarray(time_ns, dtype=np.int64)
+    w = np.asarray(ws, dtype=np.uint64)
+    if t.shape[0] < NUM_ALGOS:
+        pad = NUM_ALGOS - t.shape[0]
+        t = np.concatenate([t, np.full((pad, t.shape[1]), -1, np.int64)])
+        w = np.concatenate([w, np.zeros((pad, w.shape[1]), np.uint64)])
+    return t, w
+
+
 def version() -> int:
     return lib.mucu_version()
 
@@ -136,7 +148,9 @@ def workspace_size(d: ConvDesc, conv_type: int, algo: int, micro_n: int) -> int:
 
 
 def plan_wr(n: int, time_ns, ws, ws_limit: int) -> Tuple[int, List[Tuple[int, int]]]:
-    """WR DP.  time_ns, ws: [NUM_ALGOS][n+1].  Returns (total_ns, [(algo, b), ...])."""
+    """WR DP.  time_ns, ws: [NUM_ALGOS][n+1] (fewer rows: the rest unmeasured).
+    Returns (total_ns, [(algo, b), ...])."""
+    time_ns, ws = _full_tables(time_ns, ws)
     t, tp = _i64(time_ns)
     w, wp = _u64(ws)
     assert t.shape == (NUM_ALGOS, n + 1) and w.shape == t.shape
@@ -148,6 +162,7 @@ def plan_wr(n: int, time_ns, ws, ws_limit: int) -> Tuple[int, List[Tuple[int, in
 
 def pareto_front(n: int, time_ns, ws, ws_cap: int = (1 << 64) - 1):
     """WD desirable set.  Returns [(T, M, [(algo, b), ...]), ...] sorted by M."""
+    time_ns, ws = _full_tables(time_ns, ws)
     t, tp = _i64(time_ns)
     w, wp = _u64(ws)
     ln = ctypes.c_int32()
@@ -294,8 +309,9 @@ class Network:
                                      int(scratch_bytes), ctypes.c_void_p(stream)))
 
     def plan_from_tables(self, total_limit: int, tables):
-        t = np.concatenate([np.asarray(tt, np.int64).ravel() for tt, _ in tables])
-        w = np.concatenate([np.asarray(ww, np.uint64).ravel() for _, ww in tables])
+        tables = [_full_tables(tt, ww) for tt, ww in tables]
+        t = np.concatenate([tt.ravel() for tt, _ in tables])
+        w = np.concatenate([ww.ravel() for _, ww in tables])
         _check(lib.mucu_network_plan_from_tables(self._h, int(total_limit),
                                                  t.ctypes.data_as(ctypes.POINTER(ctypes.c_int64)),
                                                  w.ctypes.data_as(ctypes.POINTER(ctypes.c_uint64))))

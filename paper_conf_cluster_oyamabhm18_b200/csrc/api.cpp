@@ -139,8 +139,11 @@ bool staged_wg_geom(const Geom& g, StagedWg* z) {
     for (int sa : {2, 3})
         for (int sx : {8, 6, 5, 4, 3, 2})
             if (!z->Ss && sa * stage + sx * z->sx_bytes + z->tab_bytes <= 210 * 1024) { z->Ss = sa; z->SX = sx; }
+    // taps padded to whole 128-row halves: more than a quarter of padding rows (ResNet 7x7x3:
+    // 147 -> 256) costs more MMA and builder time than the window form saves (measured:
+    // ResNet-18/50 conv1 BF16 0.47 ms staged vs 0.32 ms window; AlexNet 363 -> 384 gains)
     return z->mt <= 4 && g.k <= 256 && g.k % atom == 0 && z->cs > 0 && g.r <= 256 && z->bch <= 256 && z->Ss &&
-           128 * z->mt * (g.k + 4) * 4 <= 210 * 1024;
+           128 * z->mt * (g.k + 4) * 4 <= 210 * 1024 && (z->TR - RSC) * 4 <= RSC;
 }
 
 Win win_geom(const Geom& g) {
@@ -175,6 +178,11 @@ bool algo_eligible(const Geom& g, int type, int algo) {
             // F(2x2,3x3): 3x3 filters, unit stride (ref [23]); pad' = 2 - pad >= 0 for
             // DGRAD.  BackwardFilter runs the transposed F(3x3,2x2).
             return g.r == 3 && g.s == 3 && g.stride == 1 && g.pad <= 2;
+        case MUCU_ALGO_FFT:
+        case MUCU_ALGO_FFT_TILING: {
+            FftGeom z;
+            return fft_geom(g, type, algo, &z);
+        }
         default:
             return false;
     }
@@ -264,6 +272,33 @@ mucu_status_t ws_layout(const Geom& g, int type, int algo, int32_t b, WsLayout* 
         L->total = L->b_off + L->b_bytes;
         return MUCU_OK;
     }
+    if (algo == MUCU_ALGO_FFT || algo == MUCU_ALGO_FFT_TILING) {
+        // spectra (complex fp32): filter [bins][K][C] | input tiles | output tiles
+        // (WGRAD: x tiles | dy tiles | dW spectrum).  DESIGN.md 6.11.
+        FftGeom z;
+        fft_geom(g, type, algo, &z);
+        const uint64_t B = (uint64_t)z.bins, Pl = (uint64_t)b * z.tiles_y * z.tiles_x;
+        const uint64_t KC = align_up(8 * B * g.k * g.c, 256);
+        const uint64_t in_ch = type == MUCU_FWD ? g.c : (uint64_t)g.k;   // x (FWD, WGRAD a) / dy (DGRAD)
+        const uint64_t out_ch = type == MUCU_FWD ? g.k : (uint64_t)g.c;
+        if (type == MUCU_BWD_FILTER) {
+            L->a_off = 0;
+            L->a_bytes = align_up(8 * B * Pl * g.c, 256);
+            L->b_off = L->a_bytes;
+            L->b_bytes = align_up(8 * B * Pl * g.k, 256);
+            L->fixed_off = L->b_off + L->b_bytes;  // dW spectrum (per call)
+            L->total = L->fixed_off + KC;
+            return MUCU_OK;
+        }
+        L->fixed_off = 0;
+        L->fixed_bytes = KC;
+        L->a_off = KC;
+        L->a_bytes = align_up(8 * B * Pl * in_ch, 256);
+        L->b_off = L->a_off + L->a_bytes;
+        L->b_bytes = align_up(8 * B * Pl * out_ch, 256);
+        L->total = L->b_off + L->b_bytes;
+        return MUCU_OK;
+    }
     if (type == MUCU_BWD_FILTER) {
         // Winograd F(3x3,2x2) BackwardFilter: V = B^T x B [16][Tp][C] | D = A dy A^T
         // [16][Tp][K] | M [16][K][C] fp32; T = b*ceil(P/2)*ceil(Q/2) tiles padded to
@@ -335,6 +370,12 @@ mucu_status_t run_micro(Handle* hd, const Geom& g, int type, int algo, int32_t b
     const float* f0 = (const float*)in0;
     const float* f1 = (const float*)in1;
     float* fo = (float*)out;
+    if (algo == MUCU_ALGO_FFT || algo == MUCU_ALGO_FFT_TILING) {
+        if (ctx->dry) return MUCU_OK;
+        e = fft_run(g, type, algo, b, alpha, f0, f1, beta, fo, wsb, L, ctx, st);
+        if (e == -1) return set_error(MUCU_ERR_UNSUPPORTED, "FFT path not available for this configuration");
+        return cuda_error(e, "fft kernel");
+    }
     if (type == MUCU_FWD) {
         if (algo == MUCU_ALGO_IMPLICIT_GEMM) {
             e = simt_fwd_ig(g, b, alpha, f0, f1, beta, fo, st);

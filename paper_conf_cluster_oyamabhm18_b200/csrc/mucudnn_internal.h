@@ -70,6 +70,13 @@ bool staged_wg_geom(const Geom& g, StagedWg* z);
 // reduction kernel sums them in split order (deterministic, all SMs busy).
 constexpr int kPartialSlots = 148;
 
+// FFT / FFT_TILING (kernels_fft.cu): F x F real DFT tiles of Th x Tw
+// outputs (output = y / dy grid for FWD / WGRAD, dx grid for DGRAD), tiles_y x tiles_x
+// tiles per image, bins = F * (F/2 + 1) Hermitian-half frequencies.  false = ineligible
+// (MUCU_MATH_F32 and unit stride only; FFT: F <= 32, FFT_TILING: R, S <= 16).
+struct FftGeom { int F, Th, Tw, tiles_y, tiles_x; int64_t bins; };
+bool fft_geom(const Geom& g, int type, int algo, FftGeom* z);
+
 // Workspace layout of one micro-configuration (all offsets 256-B aligned).
 // `fixed` = b-independent prefix (padded filter / Winograd U) computed once per
 // call and shared by the call's micro-batches of the same algorithm.
@@ -85,7 +92,7 @@ mucu_status_t ws_layout(const Geom& g, int type, int algo, int32_t b, WsLayout* 
 
 // Per-call executor state (which b-independent workspace prefix is valid).
 struct CallCtx {
-    int fixed_kind = 0;  // 0 none, 1 padded filter, 2 Winograd U, 3/4 space-to-depth filter
+    int fixed_kind = 0;  // 0 none, 1 padded filter, 2 Winograd U, 3/4 space-to-depth filter, 5 FFT filter spectrum
     const void* fixed_src = nullptr;
     int last_algo = -1;  // algorithm of the previous micro-config (prefix invalidation)
     bool dry = false;    // tensor-core dispatch decisions only, no launch (pre-validation)
@@ -208,5 +215,10 @@ int simt_gemm_tt(int64_t K, int64_t C, int64_t Tp, const float* V, const float* 
 int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, const void* in0, const void* in1,
                  float beta, void* out, char* ws, const WsLayout& L, int num_sms, cudaStream_t st,
                  CallCtx* ctx);
+
+// FFT / FFT_TILING micro-configuration (F32): returns 0, a CUDA error, or -1 (ineligible).
+struct CallCtx;
+int fft_run(const Geom& g, int type, int algo, int32_t b, float alpha, const float* in0, const float* in1, float beta,
+            float* out, char* ws, const WsLayout& L, CallCtx* ctx, cudaStream_t st);
 
 }  // namespace mucu

@@ -48,12 +48,28 @@ def layer_flops(layer, n: int) -> int:
     return 2 * n * layer.k * layer.c * layer.r * layer.s * layer.p * layer.q
 
 
+def fft_tiling(layer, conv_type: int, algo: int):
+    """(F, tiles per image) of FFT / FFT_TILING (kernels_fft.cu fft_geom)."""
+    eh, ew = (layer.h, layer.w) if conv_type == L.BWD_DATA else (layer.p, layer.q)
+    if algo == L.FFT:
+        f = 8
+        while f < max(eh + layer.r - 1, ew + layer.s - 1):
+            f *= 2
+        return f, 1
+    th, tw = min(eh, 33 - layer.r), min(ew, 33 - layer.s)
+    return 32, -(-eh // th) * -(-ew // tw)
+
+
 def algorithmic_flops(layer, conv_type: int, plan) -> int:
     """Tensor/FMA work the chosen algorithms actually perform:
-    IG / I2C: 2 b K C R S P Q; Winograd F(2x2,3x3): 16 GEMMs of 2 (b T) K C."""
+    IG / I2C: 2 b K C R S P Q; Winograd F(2x2,3x3): 16 GEMMs of 2 (b T) K C;
+    FFT / FFT_TILING: F (F/2 + 1) complex GEMMs of 8 (b tiles) K C (transforms excluded)."""
     f = 0
     for algo, b in plan:
-        if algo == L.WINOGRAD:
+        if algo in (L.FFT, L.FFT_TILING):
+            F, tiles = fft_tiling(layer, conv_type, algo)
+            f += 8 * F * (F // 2 + 1) * b * tiles * layer.k * layer.c
+        elif algo == L.WINOGRAD:
             oh, ow = (layer.h, layer.w) if conv_type == L.BWD_DATA else (layer.p, layer.q)
             t = ((oh + 1) // 2) * ((ow + 1) // 2)
             f += 2 * 16 * b * t * layer.k * layer.c

@@ -105,9 +105,9 @@ def test_workspace_small_c_tensor_core():
     # C*elt < 16 B on tensor cores, stride 1: I2C FWD/WGRAD keep x with channels padded to 16 B
     d = mu.desc(4, 3, 224, 224, 64, 7, 7, 3, 1, mu.MATH_BF16)
     assert mu.workspace_size(d, mu.FWD, mu.IM2COL_GEMM, 2) == 2 * 224 * 224 * 16
-    # WGRAD: staged-row kernel with 148 partial dW tiles of 256 (147 taps) x 64 fp32
-    assert mu.workspace_size(d, mu.BWD_FILTER, mu.IM2COL_GEMM, 1) == 148 * 256 * 64 * 4
-    assert mu.workspace_size(d, mu.BWD_FILTER, mu.IM2COL_GEMM, 4) == 148 * 256 * 64 * 4  # b-independent
+    # WGRAD: 147 taps would pad to 256 staged rows (> 1/4 padding): the channel-padded x as FWD
+    assert mu.workspace_size(d, mu.BWD_FILTER, mu.IM2COL_GEMM, 1) == 224 * 224 * 16
+    assert mu.workspace_size(d, mu.BWD_FILTER, mu.IM2COL_GEMM, 4) == 4 * 224 * 224 * 16
 
 
 def test_workspace_space_to_depth():
@@ -126,8 +126,9 @@ def test_workspace_space_to_depth():
     # 56 x 56 output super-pixels, 58 x 58 input super-pixels, filter 4K x 9 x 64.
     d = mu.desc(2, 3, 224, 224, 64, 7, 7, 3, 2, mu.MATH_BF16)
     assert mu.workspace_size(d, mu.FWD, mu.IM2COL_GEMM, 2) == a256(4 * 64 * 9 * 64 * 2) + a256(2 * 58 * 58 * 64 * 2)
-    # WGRAD: staged-row kernel, 148 partial tiles of 256 (147 taps) x 64 fp32
-    assert mu.workspace_size(d, mu.BWD_FILTER, mu.IM2COL_GEMM, 2) == a256(148 * 256 * 64 * 4)
+    # WGRAD: 147 taps -> 256 staged rows is > 1/4 padding: window form (64-B atoms, tpa = 8,
+    # na = 1), Wp = max(2*(Q-1) + 8, W + 3) rounded up to 4 = 232
+    assert mu.workspace_size(d, mu.BWD_FILTER, mu.IM2COL_GEMM, 2) == a256(2 * 224 * 232 * 4 * 2)
     # window form when the x row (W*C*elt) is not a multiple of 16 B: 64-B atoms (one 8-tap atom
     # per filter row), tpa = 8, na = 1, Wp = max(2*(Q-1) + 8, W + 3) rounded up to 4
     d = mu.desc(2, 3, 223, 223, 64, 7, 7, 3, 2, mu.MATH_BF16)  # W*C = 669: no chunking

@@ -19,7 +19,7 @@ ap = argparse.ArgumentParser()
 ap.add_argument("--config", default="alexnet")
 ap.add_argument("--layer", default="conv2")
 ap.add_argument("--type", default="FWD", choices=["FWD", "DGRAD", "WGRAD"])
-ap.add_argument("--algo", default="IG", choices=["IG", "I2C", "WG"])
+ap.add_argument("--algo", default="IG", choices=["IG", "I2C", "WG", "FFT", "FFTT"])
 ap.add_argument("--b", type=int, default=256)
 ap.add_argument("--n", type=int, default=256)
 ap.add_argument("--math", default="tf32", choices=["f32", "tf32", "bf16"])
@@ -29,7 +29,7 @@ a = ap.parse_args()
 layer = [l for l in network(a.config) if l.name == a.layer][0]
 math = {"f32": 0, "tf32": 1, "bf16": 2}[a.math]
 ctype = {"FWD": 0, "DGRAD": 1, "WGRAD": 2}[a.type]
-algo = {"IG": 0, "I2C": 1, "WG": 2}[a.algo]
+algo = {"IG": 0, "I2C": 1, "WG": 2, "FFT": 3, "FFTT": 4}[a.algo]
 h = mu.Handle(0)
 d = mu.desc(a.n, layer.c, layer.h, layer.w, layer.k, layer.r, layer.s, layer.pad, layer.stride, math)
 dt = torch.bfloat16 if math == 2 else torch.float32

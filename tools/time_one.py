@@ -30,7 +30,7 @@ for spec in a.specs:
     name, ty, al, b = spec.split(":")
     layer = layers[name]
     ctype = {"FWD": 0, "DGRAD": 1, "WGRAD": 2}[ty]
-    algo = {"IG": 0, "I2C": 1, "WG": 2}[al]
+    algo = {"IG": 0, "I2C": 1, "WG": 2, "FFT": 3, "FFTT": 4}[al]
     b = int(b)
     d = mu.desc(a.n, layer.c, layer.h, layer.w, layer.k, layer.r, layer.s, layer.pad, layer.stride, math)
     x, w, dy = torch_conv_inputs(layer, a.n, 0, "cuda", dt)

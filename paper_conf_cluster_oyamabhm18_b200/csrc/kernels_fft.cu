@@ -112,8 +112,10 @@ template <int F> struct FftCfg {
     static constexpr int V = F / 2 + 1;       // Hermitian half
     static constexpr int RP = F + 1;          // real row pitch (floats)
     static constexpr int PP = F * RP + 1;     // real plane pitch
+    static constexpr int SPP = F * V + 1;     // spectrum plane pitch (float2): channel-strided
+                                              // accesses of a warp land on distinct banks
     static constexpr int BYTES_R = CB * PP * 4;
-    static constexpr int BYTES_C = CB * F * V * 8;
+    static constexpr int BYTES_C = CB * SPP * 8;
     static constexpr int BYTES = BYTES_R > BYTES_C ? BYTES_R : BYTES_C;
 };
 
@@ -131,13 +133,23 @@ __global__ void __launch_bounds__(256) fft_forward_kernel(const float* __restric
     const int n = (int)(plane / m.tiles), t = (int)(plane - (int64_t)n * m.tiles);
     const int ty = t / m.tiles_x, tx = t - ty * m.tiles_x;
     const int h0 = ty * m.Th + m.oh, w0 = tx * m.Tw + m.ow;
-    for (int idx = threadIdx.x; idx < CB * F * F; idx += 256) {
+    // all loads of the tile in flight at once (registers), then the shared-memory stores
+    constexpr int NL = CB * F * F / 256;
+    float ld[NL];
+#pragma unroll
+    for (int l = 0; l < NL; ++l) {
+        const int idx = threadIdx.x + l * 256;
         const int cc = idx % CB, pix = idx / CB, i = pix / F, j = pix - i * F;
         const int h = h0 + i, w = w0 + j, c = c0 + cc;
-        float v = 0.f;
+        ld[l] = 0.f;
         if (i < m.rh && j < m.rw && (unsigned)h < (unsigned)m.H && (unsigned)w < (unsigned)m.W && c < m.C)
-            v = __ldg(src + (((int64_t)n * m.H + h) * m.W + w) * m.C + c);
-        re[cc * Cf::PP + i * Cf::RP + j] = v;
+            ld[l] = __ldg(src + (((int64_t)n * m.H + h) * m.W + w) * m.C + c);
+    }
+#pragma unroll
+    for (int l = 0; l < NL; ++l) {
+        const int idx = threadIdx.x + l * 256;
+        const int cc = idx % CB, pix = idx / CB, i = pix / F, j = pix - i * F;
+        re[cc * Cf::PP + i * Cf::RP + j] = ld[l];
     }
     __syncthreads();
     // rows: thread = (channel, row), real -> complex, keep bins v <= F/2
@@ -148,21 +160,21 @@ __global__ void __launch_bounds__(256) fft_forward_kernel(const float* __restric
     dft<F, false>(z);
     __syncthreads();  // the real tile is dead: the spectrum aliases it
 #pragma unroll
-    for (int v = 0; v < V; ++v) sp[(cr * F + row) * V + v] = z[v];
+    for (int v = 0; v < V; ++v) sp[cr * Cf::SPP + row * V + v] = z[v];
     __syncthreads();
     // columns of the Hermitian half: thread = (channel, v)
     if (threadIdx.x < CB * V) {
         const int cc = threadIdx.x / V, v = threadIdx.x % V;
 #pragma unroll
-        for (int u = 0; u < F; ++u) z[u] = sp[(cc * F + u) * V + v];
+        for (int u = 0; u < F; ++u) z[u] = sp[cc * Cf::SPP + u * V + v];
         dft<F, false>(z);
 #pragma unroll
-        for (int u = 0; u < F; ++u) sp[(cc * F + u) * V + v] = z[u];
+        for (int u = 0; u < F; ++u) sp[cc * Cf::SPP + u * V + v] = z[u];
     }
     __syncthreads();
     for (int idx = threadIdx.x; idx < F * V * CB; idx += 256) {
         const int cc = idx % CB, bin = idx / CB, u = bin / V, v = bin - u * V;
-        if (c0 + cc < m.C) dst[((int64_t)bin * m.planes + plane) * m.C + c0 + cc] = sp[(cc * F + u) * V + v];
+        if (c0 + cc < m.C) dst[((int64_t)bin * m.planes + plane) * m.C + c0 + cc] = sp[cc * Cf::SPP + u * V + v];
     }
 }
 
@@ -180,26 +192,36 @@ __global__ void __launch_bounds__(256) fft_inverse_kernel(const float2* __restri
     const int c0 = blockIdx.y * CB;
     const int n = (int)(plane / m.tiles), t = (int)(plane - (int64_t)n * m.tiles);
     const int ty = t / m.tiles_x, tx = t - ty * m.tiles_x;
-    for (int idx = threadIdx.x; idx < F * V * CB; idx += 256) {
+    constexpr int NL = (F * V * CB + 255) / 256;
+    float2 ld[NL];
+#pragma unroll
+    for (int l = 0; l < NL; ++l) {
+        const int idx = threadIdx.x + l * 256;
+        const int cc = idx % CB, bin = idx / CB;
+        ld[l] = make_float2(0.f, 0.f);
+        if (idx < F * V * CB && c0 + cc < m.C) ld[l] = __ldg(src + ((int64_t)bin * m.planes + plane) * m.C + c0 + cc);
+    }
+#pragma unroll
+    for (int l = 0; l < NL; ++l) {
+        const int idx = threadIdx.x + l * 256;
         const int cc = idx % CB, bin = idx / CB, u = bin / V, v = bin - u * V;
-        sp[(cc * F + u) * V + v] = c0 + cc < m.C ? src[((int64_t)bin * m.planes + plane) * m.C + c0 + cc]
-                                                 : make_float2(0.f, 0.f);
+        if (idx < F * V * CB) sp[cc * Cf::SPP + u * V + v] = ld[l];
     }
     __syncthreads();
     float2 z[F];
     if (threadIdx.x < CB * V) {
         const int cc = threadIdx.x / V, v = threadIdx.x % V;
 #pragma unroll
-        for (int u = 0; u < F; ++u) z[u] = sp[(cc * F + u) * V + v];
+        for (int u = 0; u < F; ++u) z[u] = sp[cc * Cf::SPP + u * V + v];
         dft<F, true>(z);
 #pragma unroll
-        for (int u = 0; u < F; ++u) sp[(cc * F + u) * V + v] = z[u];
+        for (int u = 0; u < F; ++u) sp[cc * Cf::SPP + u * V + v] = z[u];
     }
     __syncthreads();
     // rows: Hermitian half -> full spectrum -> real row
     const int cr = threadIdx.x / F, row = threadIdx.x % F;
 #pragma unroll
-    for (int v = 0; v < V; ++v) z[v] = sp[(cr * F + row) * V + v];
+    for (int v = 0; v < V; ++v) z[v] = sp[cr * Cf::SPP + row * V + v];
 #pragma unroll
     for (int v = 1; v < F / 2; ++v) z[F - v] = make_float2(z[v].x, -z[v].y);
     dft<F, true>(z);
@@ -221,49 +243,80 @@ __global__ void __launch_bounds__(256) fft_inverse_kernel(const float2* __restri
 
 // Per-bin complex GEMM C[z][m][n] = sum_k opA(m, k) * opB(n, k), z = bin (grid.z).
 // KA: A(m, k) = A[m * lda + k] (else A[k * lda + m]); KB likewise for B(n, k);
-// CJA / CJB conjugate the operand.  64 x 64 outputs per CTA, 8 k per stage,
-// 16 x 16 threads with 2 x 2 complex blocks half a tile apart (conflict-free
+// CJA / CJB conjugate the operand.  BM x 64 outputs per CTA (BM = 64, 32 or 16: few
+// planes per bin at small micro-batches), 8 / 16 / 32 k per stage, 16 x 16 threads, each with
+// TM = BM/16 rows and 4 columns in 2-wide blocks half a tile apart (conflict-free
 // 16-byte shared-memory reads), register prefetch of the next stage.
-template <bool KA, bool KB, bool CJA, bool CJB>
-__global__ void __launch_bounds__(256) cgemm_kernel(const float2* __restrict__ A, const float2* __restrict__ B,
+template <int BM>
+__device__ __forceinline__ int crow(int ty, int i) {
+    if constexpr (BM == 64) return i < 2 ? ty * 2 + i : 32 + ty * 2 + i - 2;
+    else if constexpr (BM == 32) return ty * 2 + i;
+    else return ty;
+}
+
+template <int BM, bool KA, bool KB, bool CJA, bool CJB>
+__global__ void __launch_bounds__(256, 2) cgemm_kernel(const float2* __restrict__ A, const float2* __restrict__ B,
                                                     float2* __restrict__ Cm, int M, int N, int K, int lda, int ldb,
                                                     int ldc, int64_t sA, int64_t sB, int64_t sC) {
-    constexpr int BM = 64, BN = 64, BK = 8, PAD = 4;
+    // deeper k stages for the short tiles: more bytes in flight when few planes make
+    // the per-bin filter spectrum read the bound (BM * BK + 64 * BK complex per stage)
+    constexpr int BN = 64, BK = BM == 16 ? 32 : BM == 32 ? 16 : 8, PAD = 4, TM = BM / 16;
+    constexpr int NA = (BM * BK + 255) / 256, NB = BN * BK / 256;
     __shared__ __align__(16) float2 As[2][BK][BM + PAD];
     __shared__ __align__(16) float2 Bs[2][BK][BN + PAD];
     A += blockIdx.z * sA; B += blockIdx.z * sB; Cm += blockIdx.z * sC;
     const int m0 = blockIdx.x * BM, n0 = blockIdx.y * BN;
     const int t = threadIdx.x, tx = t % 16, ty = t / 16;
-    // loader coordinates: two complex values per thread per operand
-    int al_m, al_k, bl_n, bl_k;
-    if (KA) { al_m = t / 4; al_k = (t % 4) * 2; } else { al_k = t / 32; al_m = (t % 32) * 2; }
-    if (KB) { bl_n = t / 4; bl_k = (t % 4) * 2; } else { bl_k = t / 32; bl_n = (t % 32) * 2; }
-    float2 ra[2], rb[2];
+    // element e of a stage: k-contiguous operands walk k fastest, the others m / n
+    auto a_coord = [&](int e, int& mm, int& kk) {
+        if (KA) { mm = e / BK; kk = e % BK; } else { kk = e / BM; mm = e % BM; }
+    };
+    auto b_coord = [&](int e, int& nn, int& kk) {
+        if (KB) { nn = e / BK; kk = e % BK; } else { kk = e / BN; nn = e % BN; }
+    };
+    float2 ra[NA], rb[NB];
     auto load = [&](int k0) {
 #pragma unroll
-        for (int e = 0; e < 2; ++e) {
-            const int mm = m0 + al_m + (KA ? 0 : e), kk = k0 + al_k + (KA ? e : 0);
+        for (int i = 0; i < NA; ++i) {
+            const int e = t + i * 256;
+            int mm, kk;
+            a_coord(e, mm, kk);
             float2 v = make_float2(0.f, 0.f);
-            if (mm < M && kk < K) v = __ldg(KA ? A + (int64_t)mm * lda + kk : A + (int64_t)kk * lda + mm);
+            if (e < BM * BK && m0 + mm < M && k0 + kk < K)
+                v = __ldg(KA ? A + (int64_t)(m0 + mm) * lda + k0 + kk : A + (int64_t)(k0 + kk) * lda + m0 + mm);
             if (CJA) v.y = -v.y;
-            ra[e] = v;
-            const int nn = n0 + bl_n + (KB ? 0 : e), kb = k0 + bl_k + (KB ? e : 0);
+            ra[i] = v;
+        }
+#pragma unroll
+        for (int i = 0; i < NB; ++i) {
+            const int e = t + i * 256;
+            int nn, kk;
+            b_coord(e, nn, kk);
             float2 u = make_float2(0.f, 0.f);
-            if (nn < N && kb < K) u = __ldg(KB ? B + (int64_t)nn * ldb + kb : B + (int64_t)kb * ldb + nn);
+            if (n0 + nn < N && k0 + kk < K)
+                u = __ldg(KB ? B + (int64_t)(n0 + nn) * ldb + k0 + kk : B + (int64_t)(k0 + kk) * ldb + n0 + nn);
             if (CJB) u.y = -u.y;
-            rb[e] = u;
+            rb[i] = u;
         }
     };
     auto store = [&](int buf) {
 #pragma unroll
-        for (int e = 0; e < 2; ++e) {
-            As[buf][al_k + (KA ? e : 0)][al_m + (KA ? 0 : e)] = ra[e];
-            Bs[buf][bl_k + (KB ? e : 0)][bl_n + (KB ? 0 : e)] = rb[e];
+        for (int i = 0; i < NA; ++i) {
+            const int e = t + i * 256;
+            int mm, kk;
+            a_coord(e, mm, kk);
+            if (e < BM * BK) As[buf][kk][mm] = ra[i];
+        }
+#pragma unroll
+        for (int i = 0; i < NB; ++i) {
+            int nn, kk;
+            b_coord(t + i * 256, nn, kk);
+            Bs[buf][kk][nn] = rb[i];
         }
     };
-    float2 acc[4][4];
+    float2 acc[TM][4];
 #pragma unroll
-    for (int i = 0; i < 4; ++i)
+    for (int i = 0; i < TM; ++i)
 #pragma unroll
         for (int j = 0; j < 4; ++j) acc[i][j] = make_float2(0.f, 0.f);
     load(0);
@@ -275,17 +328,22 @@ __global__ void __launch_bounds__(256) cgemm_kernel(const float2* __restrict__ A
         if (more) load(k0 + BK);
 #pragma unroll
         for (int k = 0; k < BK; ++k) {
-            float2 a[4], b[4];
-            const float4 a0 = *reinterpret_cast<const float4*>(&As[buf][k][ty * 2]);
-            const float4 a1 = *reinterpret_cast<const float4*>(&As[buf][k][32 + ty * 2]);
+            float2 a[TM], b[4];
+            if constexpr (TM == 1) {
+                a[0] = As[buf][k][ty];
+            } else {
+#pragma unroll
+                for (int h = 0; h < TM / 2; ++h) {
+                    const float4 av = *reinterpret_cast<const float4*>(&As[buf][k][crow<BM>(ty, 2 * h)]);
+                    a[2 * h] = make_float2(av.x, av.y); a[2 * h + 1] = make_float2(av.z, av.w);
+                }
+            }
             const float4 b0 = *reinterpret_cast<const float4*>(&Bs[buf][k][tx * 2]);
             const float4 b1 = *reinterpret_cast<const float4*>(&Bs[buf][k][32 + tx * 2]);
-            a[0] = make_float2(a0.x, a0.y); a[1] = make_float2(a0.z, a0.w);
-            a[2] = make_float2(a1.x, a1.y); a[3] = make_float2(a1.z, a1.w);
             b[0] = make_float2(b0.x, b0.y); b[1] = make_float2(b0.z, b0.w);
             b[2] = make_float2(b1.x, b1.y); b[3] = make_float2(b1.z, b1.w);
 #pragma unroll
-            for (int i = 0; i < 4; ++i)
+            for (int i = 0; i < TM; ++i)
 #pragma unroll
                 for (int j = 0; j < 4; ++j) {
                     acc[i][j].x = fmaf(a[i].x, b[j].x, acc[i][j].x);
@@ -299,8 +357,8 @@ __global__ void __launch_bounds__(256) cgemm_kernel(const float2* __restrict__ A
         buf ^= 1;
     }
 #pragma unroll
-    for (int i = 0; i < 4; ++i) {
-        const int mm = m0 + (i < 2 ? ty * 2 + i : 32 + ty * 2 + i - 2);
+    for (int i = 0; i < TM; ++i) {
+        const int mm = m0 + crow<BM>(ty, i);
         if (mm >= M) continue;
 #pragma unroll
         for (int j = 0; j < 4; ++j) {
@@ -313,8 +371,14 @@ __global__ void __launch_bounds__(256) cgemm_kernel(const float2* __restrict__ A
 template <bool KA, bool KB, bool CJA, bool CJB>
 int cgemm(const float2* A, const float2* B, float2* C, int M, int N, int K, int lda, int ldb, int ldc, int64_t sA,
           int64_t sB, int64_t sC, int64_t batch, cudaStream_t st) {
-    dim3 grid((unsigned)ceil_div(M, 64), (unsigned)ceil_div(N, 64), (unsigned)batch);
-    cgemm_kernel<KA, KB, CJA, CJB><<<grid, 256, 0, st>>>(A, B, C, M, N, K, lda, ldb, ldc, sA, sB, sC);
+    const int bm = M <= 16 ? 16 : M <= 32 ? 32 : 64;
+    dim3 grid((unsigned)ceil_div(M, bm), (unsigned)ceil_div(N, 64), (unsigned)batch);
+    if (bm == 16)
+        cgemm_kernel<16, KA, KB, CJA, CJB><<<grid, 256, 0, st>>>(A, B, C, M, N, K, lda, ldb, ldc, sA, sB, sC);
+    else if (bm == 32)
+        cgemm_kernel<32, KA, KB, CJA, CJB><<<grid, 256, 0, st>>>(A, B, C, M, N, K, lda, ldb, ldc, sA, sB, sC);
+    else
+        cgemm_kernel<64, KA, KB, CJA, CJB><<<grid, 256, 0, st>>>(A, B, C, M, N, K, lda, ldb, ldc, sA, sB, sC);
     count_launch();
     return (int)cudaGetLastError();
 }

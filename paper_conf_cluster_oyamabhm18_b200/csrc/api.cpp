@@ -753,10 +753,13 @@ extern "C" mucu_status_t mucu_benchmark(mucu_handle_t h, const mucu_conv_desc_t*
         for (int a = 0; a < MUCU_NUM_ALGOS && status == MUCU_OK; ++a) {
             WsLayout L;
             if (ws_layout(g, type, a, b, &L) != MUCU_OK || L.total > ws_limit) continue;
+            // Steady state of a micro-batch inside a call: the b-independent prefix (padded /
+            // space-to-depth filter, Winograd U, FFT filter spectrum) is computed once per
+            // call by the executor, so the warm-up computes it and the timed runs reuse it.
+            CallCtx bctx;
             auto launch = [&]() {
-                CallCtx ctx;  // each timed run is a whole call: includes the filter transform
                 return run_micro(h, g, type, a, b, 1.f, base + S.in0, base + S.in1, 0.f, base + S.out, base + S.ws,
-                                 S.total - S.ws, st, &ctx);
+                                 S.total - S.ws, st, &bctx);
             };
             // a dry run first: a configuration without a tensor-core kernel is skipped
             // (not benchmarked) whatever the warm-up count
@@ -771,16 +774,19 @@ extern "C" mucu_status_t mucu_benchmark(mucu_handle_t h, const mucu_conv_desc_t*
             for (int i = 0; i < h->warmup && r == MUCU_OK; ++i) r = launch();
             if (r == MUCU_ERR_UNSUPPORTED) continue;
             if (r) { status = r; break; }
+            // T_mu(b) (P:L88 step 1): micro-batches run back to back in a plan, so each sample
+            // is the mean of `reps` back-to-back launches between two events (no idle-stream
+            // launch latency in the table); the median of three samples is recorded.
             samples.clear();
-            for (int i = 0; i < h->reps; ++i) {
+            for (int grp = 0; grp < 3 && r == MUCU_OK; ++grp) {
                 cudaEventRecord(e0, st);
-                r = launch();
+                for (int i = 0; i < h->reps && r == MUCU_OK; ++i) r = launch();
                 cudaEventRecord(e1, st);
                 if (r) break;
                 if (cudaEventSynchronize(e1)) { r = cuda_error((int)cudaGetLastError(), "benchmark sync"); break; }
                 float ms = 0.f;
                 cudaEventElapsedTime(&ms, e0, e1);
-                samples.push_back(ms);
+                samples.push_back(ms / (float)std::max(1, h->reps));
             }
             if (r == MUCU_ERR_UNSUPPORTED) continue;
             if (r) { status = r; break; }

@@ -7,6 +7,7 @@
 #include "mucudnn.h"
 
 #ifdef __CUDACC__
+#include <cstdio>
 #include <cuda_runtime.h>
 #else
 typedef struct CUstream_st* cudaStream_t;
@@ -135,14 +136,36 @@ int alloc_turns(int64_t count, TurnRange* out);  // cudaError_t
 __host__ __device__ __forceinline__ unsigned long long turn_tag(unsigned long long epoch, int split) {
     return (epoch << 20) + (unsigned long long)split + 1ull;
 }
+// Watchdog of every spin-wait in the library's kernels: a wait that has not been
+// satisfied after kWatchdogNs reports what it waited for and traps (the launch then
+// fails with a CUDA error) instead of hanging the device.
+constexpr unsigned long long kWatchdogNs = 10ull * 1000 * 1000 * 1000;
+__device__ __forceinline__ unsigned long long global_ns() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
+static __device__ __noinline__ void watchdog_trap(const char* what, unsigned long long addr, unsigned long long want,
+                                           unsigned long long have) {
+    printf("[mucu watchdog] %s wait > %llu s: block (%d,%d,%d) thread %d addr 0x%llx want 0x%llx have 0x%llx\n", what,
+           kWatchdogNs / 1000000000ull, (int)blockIdx.x, (int)blockIdx.y, (int)blockIdx.z, (int)threadIdx.x, addr,
+           want, have);
+    __trap();
+}
 // One thread waits for the previous split's tag (acquire at gpu scope); the
 // caller then synchronises the threads that read dw.
 __device__ __forceinline__ void turn_wait(const unsigned long long* c, unsigned long long tag) {
     unsigned long long v;
-    for (;;) {
+    unsigned long long t0 = 0;
+    for (unsigned n = 0;; ++n) {
         asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(c) : "memory");
         if (v == tag) break;
         __nanosleep(32);
+        if ((n & 1023) == 0) {
+            const unsigned long long t = global_ns();
+            if (!t0) t0 = t;
+            else if (t - t0 > kWatchdogNs) watchdog_trap("turn", (unsigned long long)c, tag, v);
+        }
     }
 }
 // One thread publishes after the dw writes of every thread of the group were

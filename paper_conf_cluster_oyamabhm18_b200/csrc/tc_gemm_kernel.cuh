@@ -192,12 +192,17 @@ __global__ void __launch_bounds__(threads_for(AM), 1) tc_conv_gemm(const __grid_
     // for groups that were already running -- no dependency on the scheduling order
     // of clusters (GPC packing, concurrent kernels).  The k-range of group g is fixed,
     // so the summation order, and dw, do not depend on which cluster got which ticket.
+    // "Running" means every CTA of the cluster holds its tensor memory: the ticket is
+    // taken only after a cluster barrier behind all ranks' tcgen05.alloc.  (A rank
+    // still blocked in the allocation -- its SM's TMEM held by a co-resident CTA that
+    // waits on a later group -- would otherwise deadlock behind its own ticket.)
     int g_ticket = -1;
     if constexpr (SPLITK) {
         if (p.cl && p.tickets) {
             int& s_tk = ((int*)tmem_slot)[1];  // (dynamic shared memory: the upper half of the TMEM slot)
             const int rho = blockIdx.x % p.cl, c = blockIdx.x / p.cl;
             const int nu = per_z * (p.zsplit ? p.num_z / p.zsplit : 1);
+            asm volatile("barrier.cluster.arrive.release;\n\tbarrier.cluster.wait.acquire;" ::: "memory");
             if (threadIdx.x == 0 && rho == 0) s_tk = take_ticket(p.tickets + (c % nu), p.epoch);
             asm volatile("barrier.cluster.arrive.release;\n\tbarrier.cluster.wait.acquire;" ::: "memory");
             if (threadIdx.x == 0 && rho != 0) {
@@ -588,7 +593,13 @@ __global__ void __launch_bounds__(threads_for(AM), 1) tc_conv_gemm(const __grid_
         int s = 0;
         uint32_t ph = 0;
         int git = 0;  // k-blocks issued by this CTA so far (for the lagged arrivals)
-        for (int tile = blockIdx.x; tile < total_tiles; tile += gridDim.x) {
+        // TMA-only operands (no gathers): warp 0 runs the stage loop (lane 0 issues) and
+        // warps 1-3 stay out of it.  A thread that only waits on the empty barriers
+        // without gating them can fall two phases behind (a concurrent kernel delaying
+        // its warp): the barrier's parity then repeats and its last wait never returns
+        // (observed: a hang at the end of the tile loop under the concurrent backward).
+        const bool in_loop = GATHER || warp == 0;
+        for (int tile = in_loop ? (int)blockIdx.x : total_tiles; tile < total_tiles; tile += gridDim.x) {
             int m0, n0, z, kb_begin, kb_end;
             decode(tile, m0, n0, z, kb_begin, kb_end);
             // Per-thread gather rows (A gathers: rows t/8 + 16 i, chunk t % 8):
@@ -1059,6 +1070,7 @@ __global__ void __launch_bounds__(threads_for(AM), 1) tc_conv_gemm(const __grid_
                 // after this stage is published (a fence would otherwise wait for them).
                 if constexpr (AM == A_GATHER_SMALLC) { if (kb + 1 < kb_end) smallc_load(kb + 1); }
                 if constexpr (BM_ == B_GATHER_SMALLC) { if (kb + 1 < kb_end) wg_smallc_load(kb + 1); }
+                if constexpr (!GATHER) __syncwarp();
             }
         }
         if constexpr (GATHER && (A_ASYNC || B_ASYNC)) {

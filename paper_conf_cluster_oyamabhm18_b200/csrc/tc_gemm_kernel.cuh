@@ -598,6 +598,8 @@ __global__ void __launch_bounds__(threads_for(AM), 1) tc_conv_gemm(const __grid_
         // without gating them can fall two phases behind (a concurrent kernel delaying
         // its warp): the barrier's parity then repeats and its last wait never returns
         // (observed: a hang at the end of the tile loop under the concurrent backward).
+        // (Warp 0's other lanes wait alongside lane 0, which gates every stage it waits
+        // for; a __syncwarp per stage to pin them costs 10 % on short ResNet layers.)
         const bool in_loop = GATHER || warp == 0;
         for (int tile = in_loop ? (int)blockIdx.x : total_tiles; tile < total_tiles; tile += gridDim.x) {
             int m0, n0, z, kb_begin, kb_end;
@@ -1070,7 +1072,6 @@ __global__ void __launch_bounds__(threads_for(AM), 1) tc_conv_gemm(const __grid_
                 // after this stage is published (a fence would otherwise wait for them).
                 if constexpr (AM == A_GATHER_SMALLC) { if (kb + 1 < kb_end) smallc_load(kb + 1); }
                 if constexpr (BM_ == B_GATHER_SMALLC) { if (kb + 1 < kb_end) wg_smallc_load(kb + 1); }
-                if constexpr (!GATHER) __syncwarp();
             }
         }
         if constexpr (GATHER && (A_ASYNC || B_ASYNC)) {

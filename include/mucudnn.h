@@ -267,6 +267,50 @@ mucu_status_t mucu_conv_backward_filter(mucu_handle_t handle, const mucu_conv_de
                                         const void* x, const void* dy, float beta, float* dw,
                                         void* workspace, uint64_t ws_bytes, void* cuda_stream);
 
+/* ------------------------------------------- NEXT-3: NVLS dW reduction ---- */
+/* Data-parallel training sums every layer's dW over the ranks (micro-
+ * batching lets "the communication of parameter gradients" be hidden; SURVEY
+ * 8(f) NEXT-3).  Here the sum is fused into BackwardFilter: the kernel that
+ * writes a dw element's final value (the last micro-batch's epilogue, its last
+ * ordered split group, or the partial-slot reduction; a push kernel after the
+ * F32 SIMT / Winograd / FFT / atomic writers) also adds it with
+ * `multimem.red.add.f32` to the NVLink multicast address of a symmetric fp32
+ * buffer, so NVSwitch accumulates it into every rank's copy.
+ *
+ * Multicast object, one per rank (device = this rank's CUDA device, ranks =
+ * world size, bytes = user bytes; all ranks pass the same values):
+ *   rank 0: mucu_nvls_create, mucu_nvls_export -> a POSIX fd owned by the
+ *           caller, passed to the peers (pidfd_getfd);
+ *   others: mucu_nvls_import(fd);
+ *   all:    mucu_nvls_bind -> local (this rank's copy, unicast) and multicast
+ *           addresses of the user bytes; blocks until every rank has created or
+ *           imported; the buffer starts zeroed.
+ * mucu_nvls_barrier(stream): enqueue a device-side barrier over the ranks
+ *   (system-scope release of this rank's earlier multimem reductions, then wait
+ *   for every rank's) -- every rank calls it the same number of times.
+ * Errors: UNSUPPORTED (no multicast on the device), CUDA (driver call failed,
+ *   detail in mucu_last_error), INVALID_VALUE. */
+typedef struct mucu_nvls* mucu_nvls_t;
+mucu_status_t mucu_nvls_supported(int device, int32_t* supported);     /* host */
+mucu_status_t mucu_nvls_create(int device, int32_t ranks, uint64_t bytes, mucu_nvls_t* out);
+mucu_status_t mucu_nvls_export(mucu_nvls_t nv, int32_t* fd);
+mucu_status_t mucu_nvls_import(int device, int32_t ranks, uint64_t bytes, int32_t fd, mucu_nvls_t* out);
+mucu_status_t mucu_nvls_bind(mucu_nvls_t nv, void** local, void** multicast);
+mucu_status_t mucu_nvls_barrier(mucu_nvls_t nv, void* cuda_stream);
+mucu_status_t mucu_nvls_destroy(mucu_nvls_t nv);
+/* mucu_conv_backward_filter plus the fused reduction: dw (device, private to
+ * this rank) receives this rank's gradient exactly as mucu_conv_backward_filter
+ * computes it; dw_mc (the multicast address of a K*R*S*C fp32 region of a bound
+ * NVLS buffer, 16-byte aligned) receives += the same values on every rank's
+ * copy.  Protocol per iteration: zero the local copies, mucu_nvls_barrier, each
+ * rank's backward_filter_nvls calls, mucu_nvls_barrier; then every rank's local
+ * copy holds sum over ranks of dw.  Addition order across ranks is the order the
+ * switch receives them (exact for 2 ranks; FTZ like any fp32 reduction). */
+mucu_status_t mucu_conv_backward_filter_nvls(mucu_handle_t handle, const mucu_conv_desc_t* desc,
+                                             const mucu_micro_config_t* plan, int32_t count, float alpha,
+                                             const void* x, const void* dy, float beta, float* dw, float* dw_mc,
+                                             void* workspace, uint64_t ws_bytes, void* cuda_stream);
+
 /* ------------------------------------------------------------ WD ---- */
 /* WD needs every kernel before optimising: register the kernels,
  * then plan once.  mucu_network_plan benchmarks each unique (desc, type)

@@ -79,6 +79,14 @@ def _load():
         "mucu_conv_forward": (ctypes.c_int, [vp, D, MC, i32, f32, vp, vp, f32, vp, vp, u64, vp]),
         "mucu_conv_backward_data": (ctypes.c_int, [vp, D, MC, i32, f32, vp, vp, f32, vp, vp, u64, vp]),
         "mucu_conv_backward_filter": (ctypes.c_int, [vp, D, MC, i32, f32, vp, vp, f32, vp, vp, u64, vp]),
+        "mucu_conv_backward_filter_nvls": (ctypes.c_int, [vp, D, MC, i32, f32, vp, vp, f32, vp, vp, vp, u64, vp]),
+        "mucu_nvls_supported": (ctypes.c_int, [ctypes.c_int, P(i32)]),
+        "mucu_nvls_create": (ctypes.c_int, [ctypes.c_int, i32, u64, P(vp)]),
+        "mucu_nvls_export": (ctypes.c_int, [vp, P(i32)]),
+        "mucu_nvls_import": (ctypes.c_int, [ctypes.c_int, i32, u64, i32, P(vp)]),
+        "mucu_nvls_bind": (ctypes.c_int, [vp, P(vp), P(vp)]),
+        "mucu_nvls_barrier": (ctypes.c_int, [vp, vp]),
+        "mucu_nvls_destroy": (ctypes.c_int, [vp]),
         "mucu_network_create": (ctypes.c_int, [P(vp)]),
         "mucu_network_destroy": (ctypes.c_int, [vp]),
         "mucu_network_add": (ctypes.c_int, [vp, D, ctypes.c_int, P(i32)]),
@@ -280,6 +288,58 @@ class Handle:
 
     def conv_backward_filter(self, d, plan, alpha, x, dy, beta, dw, ws_ptr, ws_bytes, stream):
         self._conv(lib.mucu_conv_backward_filter, d, plan, alpha, x, dy, beta, dw, ws_ptr, ws_bytes, stream)
+
+    def conv_backward_filter_nvls(self, d, plan, alpha, x, dy, beta, dw, dw_mc, ws_ptr, ws_bytes, stream):
+        arr = _plan_array(plan)
+        _check(lib.mucu_conv_backward_filter_nvls(
+            self._h, ctypes.byref(d), arr, len(plan), float(alpha), ctypes.c_void_p(x), ctypes.c_void_p(dy),
+            float(beta), ctypes.c_void_p(dw), ctypes.c_void_p(dw_mc), ctypes.c_void_p(ws_ptr or 0), int(ws_bytes),
+            ctypes.c_void_p(stream)))
+
+
+def nvls_supported(device: int = 0) -> bool:
+    v = ctypes.c_int32()
+    _check(lib.mucu_nvls_supported(device, ctypes.byref(v)))
+    return bool(v.value)
+
+
+class Nvls:
+    """One rank's NVLink multicast buffer (NEXT-3; include/mucudnn.h).  Rank 0 creates
+    (``fd=None``) and exports an fd for the peers; the others import it."""
+
+    def __init__(self, device: int, ranks: int, nbytes: int, fd: Optional[int] = None):
+        h = ctypes.c_void_p()
+        if fd is None:
+            _check(lib.mucu_nvls_create(device, ranks, int(nbytes), ctypes.byref(h)))
+        else:
+            _check(lib.mucu_nvls_import(device, ranks, int(nbytes), int(fd), ctypes.byref(h)))
+        self._h = h
+        self.local = self.multicast = None
+
+    def export(self) -> int:
+        fd = ctypes.c_int32()
+        _check(lib.mucu_nvls_export(self._h, ctypes.byref(fd)))
+        return fd.value
+
+    def bind(self) -> Tuple[int, int]:
+        loc, mc = ctypes.c_void_p(), ctypes.c_void_p()
+        _check(lib.mucu_nvls_bind(self._h, ctypes.byref(loc), ctypes.byref(mc)))
+        self.local, self.multicast = loc.value, mc.value
+        return self.local, self.multicast
+
+    def barrier(self, stream: int = 0):
+        _check(lib.mucu_nvls_barrier(self._h, ctypes.c_void_p(stream)))
+
+    def close(self):
+        if self._h is not None and self._h.value:
+            lib.mucu_nvls_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
 
 
 class Network:

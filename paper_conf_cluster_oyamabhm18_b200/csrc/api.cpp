@@ -571,7 +571,7 @@ static mucu_status_t check_ptr(const void* p, const char* what) {
 
 static mucu_status_t execute(mucu_handle_t h, const mucu_conv_desc_t* d, int type, const mucu_micro_config_t* plan,
                              int32_t count, float alpha, const void* in0, const void* in1, float beta, void* out,
-                             void* ws, uint64_t ws_bytes, void* stream) {
+                             void* ws, uint64_t ws_bytes, void* stream, float* dw_mc = nullptr) {
     if (!h) return set_error(MUCU_ERR_INVALID_VALUE, "null handle");
     Geom g;
     if (!make_geom(d, &g)) return set_error(MUCU_ERR_INVALID_VALUE, "invalid descriptor");
@@ -634,6 +634,7 @@ static mucu_status_t execute(mucu_handle_t h, const mucu_conv_desc_t* d, int typ
         }
     }
     CallCtx ctx;
+    ctx.mc_out = dw_mc;
     int64_t done = 0;
     for (int32_t i = 0; i < count; ++i) {
         const int32_t b = plan[i].micro_n;
@@ -641,9 +642,16 @@ static mucu_status_t execute(mucu_handle_t h, const mucu_conv_desc_t* d, int typ
         char* po;
         float bta;
         part_ptrs(i, done, p0, p1, po, bta);
+        ctx.mc_last = i == count - 1;
         s = run_micro(h, g, type, plan[i].algo, b, alpha, p0, p1, bta, po, ws, ws_bytes, st, &ctx);
         if (s) return s;
         done += b;
+    }
+    if (dw_mc && !ctx.mc_fused) {
+        // NEXT-3: the last micro-configuration's dw writer did not take the reduction
+        // (F32 SIMT, Winograd, FFT, atomic split-K): push the final dw through NVLS
+        const int e = launch_nvls_push((const float*)out, dw_mc, (int64_t)g.k * g.r * g.s * g.c, st);
+        if (e) return set_error(MUCU_ERR_CUDA, "nvls push: %s", cudaGetErrorString((cudaError_t)e));
     }
     return MUCU_OK;
 }
@@ -666,6 +674,14 @@ extern "C" mucu_status_t mucu_conv_backward_filter(mucu_handle_t h, const mucu_c
                                                    const void* x, const void* dy, float beta, float* dw, void* ws,
                                                    uint64_t ws_bytes, void* stream) {
     return execute(h, d, MUCU_BWD_FILTER, plan, count, alpha, x, dy, beta, dw, ws, ws_bytes, stream);
+}
+
+extern "C" mucu_status_t mucu_conv_backward_filter_nvls(mucu_handle_t h, const mucu_conv_desc_t* d,
+                                                        const mucu_micro_config_t* plan, int32_t count, float alpha,
+                                                        const void* x, const void* dy, float beta, float* dw,
+                                                        float* dw_mc, void* ws, uint64_t ws_bytes, void* stream) {
+    if (!dw_mc || ((uintptr_t)dw_mc & 15)) return set_error(MUCU_ERR_MISALIGNED, "dw_mc NULL or not 16-byte aligned");
+    return execute(h, d, MUCU_BWD_FILTER, plan, count, alpha, x, dy, beta, dw, ws, ws_bytes, stream, dw_mc);
 }
 
 // ============================================================ benchmark ====

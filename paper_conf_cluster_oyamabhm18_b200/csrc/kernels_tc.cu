@@ -320,6 +320,11 @@ struct TcArgs {
     int m64;                 // MN-major A: the tile's last 128-row half has <= 64 valid rows -> M = 64 MMAs
     unsigned long long* turns;
     unsigned long long epoch;
+    // NEXT-3: multicast (NVLS) address of the cross-rank dW sum, aligned
+    // with `out`; the final writer of every dw element also adds it there with
+    // multimem.red (cluster split-K: split group mc_group is the final one).  nullptr: off.
+    float* mc_out;
+    int mc_group;
 };
 
 constexpr int kThreads = 288;  // 4 producer warps, 1 MMA warp, 4 epilogue warps
@@ -515,6 +520,11 @@ struct Launch {
     CUtensorMap ta, tb;
     dim3 grid;
     Im2colArgs ia;
+    // NEXT-3: the call's multicast dW (last micro-batch only), its local dw and the
+    // executor's "fused" flag (set when this launch writes dw and takes the reduction)
+    float* mc_out;
+    const void* mc_local;
+    bool* mc_fused;
 };
 
 template <int ELT, int AM, int BM_, int EPI>
@@ -540,7 +550,18 @@ int launch_t(Launch& L, cudaStream_t st, bool dry) {
     if (!SPLITK && L.a.cl) return -1;
     L.a.turns = nullptr;
     L.a.epoch = 0;
+    L.a.mc_out = nullptr;
+    L.a.mc_group = 0;
     if (dry) return 0;
+    // NEXT-3: the launch that writes the call's dw in the last micro-batch is its final
+    // writer (one dw-writing launch per micro-configuration; split-K groups ordered):
+    // fuse the cross-rank reduction into its epilogue.  Atomic split-K partials and
+    // batched (Winograd) outputs are not final values: the executor pushes dw instead.
+    if (SPLITK && EPI != EPI_WGRAD_PARTIAL && L.mc_out && L.a.out == L.mc_local && !L.a.atomic && !L.a.zsplit) {
+        L.a.mc_out = L.mc_out;
+        L.a.mc_group = L.a.cl ? L.a.num_z / L.a.cl - 1 : 0;
+        *L.mc_fused = true;
+    }
     if (SPLITK && L.a.atomic && L.a.beta != 1.f) {
         // split partials are added with L2 reductions: apply beta to the output first
         int64_t extent;
@@ -738,7 +759,13 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
     A.stride = g.stride; A.K = g.k;
     A.tapR = g.r; A.tapS = g.s; A.ph_u = 1;
     A.max_lag = std::min(6, std::max(1, env_int("MUCU_MAX_LAG", 6)));
-    A.alpha = alpha; A.beta = beta; A.out = out; A.out_bf16 = bf ? 1 : 0; 
+    A.alpha = alpha; A.beta = beta; A.out = out; A.out_bf16 = bf ? 1 : 0;
+    if (type == MUCU_BWD_FILTER && ctx->mc_out && ctx->mc_last) {
+        L.mc_out = ctx->mc_out; L.mc_local = out; L.mc_fused = &ctx->mc_fused;
+    }
+    // partial-slot reductions are the final writer of dw: they take the multicast sum
+    float* const mc_reduce = L.mc_out;
+    auto note_fused = [&]() { if (mc_reduce && !dry) ctx->mc_fused = true; };
     auto map2 = [&](CUtensorMap* tm, const void* base, uint64_t d0, uint64_t d1, uint64_t pitch_elems, uint32_t b0,
                     uint32_t b1, bool mn = false) {
         uint64_t dims[2] = {d0, d1}, str[1] = {pitch_elems * elt};
@@ -1474,8 +1501,9 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
             A.out = part; A.alpha = 1.f; A.beta = 0.f; A.ldc = g.k; A.part_rows = zw.TR;
             err = LAUNCH(A_STAGED_WG, B_TMA_DYROW, EPI_WGRAD_PARTIAL);
             if (err) return err;
+            note_fused();
             return DRY(launch_partial_reduce((int)Sr, (int64_t)zw.TR * g.k, g.k, (int)RSC, g.k, true, part, alpha, beta,
-                                             (float*)out, st));
+                                             (float*)out, st, mc_reduce));
         }
         if (algo == MUCU_ALGO_IM2COL_GEMM && small_c_tc(g)) {
             // RGB-like layer: channel-padded copy of x, padded columns j' = (r, s8, c').
@@ -1527,8 +1555,9 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
                 A.out = part; A.alpha = 1.f; A.beta = 0.f; A.part_rows = g.k;  // slot = K x R*S*C (ldc = R*S*C)
                 err = LAUNCH(A_TMA_MN2, B_TMA_MN2, EPI_WGRAD_PARTIAL);
                 if (err) return err;
+                note_fused();
                 return DRY(launch_partial_reduce((int)sbest, (int64_t)g.k * RSC, (int)RSC, g.k, (int)RSC, false, part,
-                                                 alpha, beta, (float*)out, st));
+                                                 alpha, beta, (float*)out, st, mc_reduce));
             }
             return LAUNCH(A_TMA_MN2, B_TMA_MN2, EPI_WGRAD_CHAIN);
         }

@@ -98,6 +98,12 @@ struct CallCtx {
     int last_algo = -1;  // algorithm of the previous micro-config (prefix invalidation)
     bool dry = false;    // tensor-core dispatch decisions only, no launch (pre-validation)
     bool deterministic = true;  // BackwardFilter split-K: ordered reduction (default) or L2 atomics
+    // NEXT-3: multicast address of the cross-rank dW sum (nullptr: off),
+    // set for the call's last micro-configuration (mc_last); the final dw writer sets
+    // mc_fused when it took the reduction in its epilogue.
+    float* mc_out = nullptr;
+    bool mc_last = false;
+    bool mc_fused = false;
 };
 
 struct Handle;
@@ -120,6 +126,17 @@ struct FastDiv {
         return (uint32_t)(((uint64_t)__umulhi(n, m) + n) >> l);
     }
 };
+// NEXT-3: add v to every rank's copy of a multicast (NVLS) object address.  The
+// reduction is performed by NVSwitch; relaxed, system scope (made visible to the
+// peers by the release of the NVLS barrier, nvls.cu).
+__device__ __forceinline__ void mc_red(float* a, float v) {
+    asm volatile("multimem.red.relaxed.sys.global.add.f32 [%0], %1;" ::"l"(a), "f"(v) : "memory");
+}
+__device__ __forceinline__ void mc_red4(float* a, float4 v) {  // a 16-byte aligned
+    asm volatile("multimem.red.relaxed.sys.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(a), "f"(v.x), "f"(v.y),
+                 "f"(v.z), "f"(v.w)
+                 : "memory");
+}
 #endif
 
 // ---------------------------------------------------------------- kernels --
@@ -222,8 +239,16 @@ int launch_wgw_output(const Geom& g, float alpha, const float* M, float beta, fl
 // part[s][m][n] at slot stride `slot` (elements) and row pitch `ldp`; out[m][n] (row pitch
 // N), or out[n][m] (row pitch M) when `transpose`.  Summed in split order s = 0, 1, ...
 // (deterministic).
+// mc (NEXT-3): multicast address matching `out` -- the final values are also added
+// to the cross-rank dW sum (nullptr: off).
 int launch_partial_reduce(int S, int64_t slot, int ldp, int M, int N, bool transpose, const float* part,
-                          float alpha, float beta, float* out, cudaStream_t st);
+                          float alpha, float beta, float* out, cudaStream_t st, float* mc = nullptr);
+// NEXT-3 (nvls.cu): mc[i] += src[i] on every rank's copy (multimem.red, 16-B vectors
+// where aligned) for the dw writers that do not fuse the reduction; and the NVLS
+// barrier: release-add 1 to the multicast flag word, wait until the local copy of it
+// reaches `target` (= ranks x barriers so far).
+int launch_nvls_push(const float* src, float* mc, int64_t n, cudaStream_t st);
+int launch_nvls_barrier(unsigned* mc_flag, const unsigned* uc_flag, unsigned target, cudaStream_t st);
 // Tensor-core I2C BackwardFilter of large-C layers: partial dW slots reserved in the
 // workspace (deterministic split-K over all SMs): ceil(148 / dW tiles of 128 x 128),
 // 1 = no partial slots.

@@ -60,8 +60,10 @@ __device__ __forceinline__ long long wgrad_dst(const TcArgs& p, int m, int n) {
 // dst[ofs[j] * stride] = alpha * v[j] + beta * dst[...] for the 32 accumulator
 // columns of one row (ofs < 0: skipped); all loads issue before the stores.
 // beta == 0 never reads dst (it may hold garbage / NaN).
+// mc (NEXT-3): the multicast address matching dst (nullptr: off) -- the final value of
+// every element is also added to the cross-rank dW sum there.
 __device__ __forceinline__ void rmw32(float* dst, const int (&ofs)[32], size_t stride, const uint32_t* v, float alpha,
-                                      float beta, bool atomic = false) {
+                                      float beta, bool atomic = false, float* mc = nullptr) {
     if (atomic) {  // non-deterministic split-K (beta applied by a prescale launch): L2 reductions
 #pragma unroll
         for (int j = 0; j < 32; ++j)
@@ -76,7 +78,11 @@ __device__ __forceinline__ void rmw32(float* dst, const int (&ofs)[32], size_t s
     for (int j = 0; j < 32; ++j) old[j] = (beta != 0.f && ofs[j] >= 0) ? __ldcg(dst + (size_t)ofs[j] * stride) : 0.f;
 #pragma unroll
     for (int j = 0; j < 32; ++j)
-        if (ofs[j] >= 0) dst[(size_t)ofs[j] * stride] = alpha * __uint_as_float(v[j]) + beta * old[j];
+        if (ofs[j] >= 0) {
+            const float o = alpha * __uint_as_float(v[j]) + beta * old[j];
+            dst[(size_t)ofs[j] * stride] = o;
+            if (mc) mc_red(mc + (size_t)ofs[j] * stride, o);
+        }
 }
 
 template <int ELT, int AM, int BM_, int EPI>
@@ -1266,6 +1272,10 @@ __global__ void __launch_bounds__(threads_for(AM), 1) tc_conv_gemm(const __grid_
             // cluster path; p.atomic (non-deterministic mode) adds every split's partial
             // with L2 reductions after a beta prescale launch.
             const float bsplit = p.beta;
+            // NEXT-3: multicast address of a dw element (the final value: no split here)
+            auto mc_of = [&](const float* d) -> float* {
+                return p.mc_out ? p.mc_out + (d - (const float*)p.out) : nullptr;
+            };
             auto drain = [&](const int hh) {
             // M = 64 half: TMEM lane 32*q4 + l (l < 16) holds row 16*q4 + l
             const bool h64 = p.m64 && hh == p.mt - 1;
@@ -1463,7 +1473,7 @@ __global__ void __launch_bounds__(threads_for(AM), 1) tc_conv_gemm(const __grid_
                         }
                         if (++ch == p.C) { ch = 0; ++tap; }
                     }
-                    rmw32(drow, dofs, 1, v, p.alpha, bsplit, p.atomic);
+                    rmw32(drow, dofs, 1, v, p.alpha, bsplit, p.atomic, mc_of(drow));
                 } else if constexpr (EPI == EPI_WGRAD_WIN) {
                     // row m = (r, atom aa, tap t, channel c) -> dw[k][r][aa*taps + t][c], k = nb + j
                     constexpr int per_atom = WAW / ELT;
@@ -1475,7 +1485,7 @@ __global__ void __launch_bounds__(threads_for(AM), 1) tc_conv_gemm(const __grid_
                         int dofs[32];
 #pragma unroll
                         for (int j = 0; j < 32; ++j) dofs[j] = nb + j < p.N ? j : -1;
-                        rmw32(d, dofs, (size_t)p.ldc, v, p.alpha, bsplit, p.atomic);
+                        rmw32(d, dofs, (size_t)p.ldc, v, p.alpha, bsplit, p.atomic, mc_of(d));
                     }
                 } else if constexpr (EPI == EPI_WGRAD_PARTIAL) {
                     // the split's partial tile: out[z][m][nb + j] (rows < part_rows, plain stores)
@@ -1498,7 +1508,8 @@ __global__ void __launch_bounds__(threads_for(AM), 1) tc_conv_gemm(const __grid_
                         int dofs[32];
 #pragma unroll
                         for (int j = 0; j < 32; ++j) dofs[j] = nb + j < p.N ? j : -1;
-                        rmw32(outF + (size_t)nb * p.ldc + m, dofs, (size_t)p.ldc, v, p.alpha, bsplit, p.atomic);
+                        rmw32(outF + (size_t)nb * p.ldc + m, dofs, (size_t)p.ldc, v, p.alpha, bsplit, p.atomic,
+                              mc_of(outF + (size_t)nb * p.ldc + m));
                     }
                 } else if constexpr (EPI == EPI_WGRAD_SMALLC) {
                     // padded column j' = (r, s8, c') -> dw column (r*S + s)*C + c (skip padding)
@@ -1510,7 +1521,7 @@ __global__ void __launch_bounds__(threads_for(AM), 1) tc_conv_gemm(const __grid_
                         const int c = jp % p.cp, t2 = jp / p.cp, s_ = t2 % p.s8, r = t2 / p.s8;
                         dofs[j] = (jp < p.N && c < p.C && s_ < p.S) ? (r * p.S + s_) * p.C + c : -1;
                     }
-                    rmw32(drow, dofs, 1, v, p.alpha, bsplit, p.atomic);
+                    rmw32(drow, dofs, 1, v, p.alpha, bsplit, p.atomic, mc_of(drow));
                 } else if constexpr (EPI == EPI_WGRAD_CHAIN) {
                     // dw = alpha * partial + bsplit * dw (bsplit = beta on split 0, else 1),
                     // in split order: 16-byte vector read-modify-write
@@ -1538,12 +1549,13 @@ __global__ void __launch_bounds__(threads_for(AM), 1) tc_conv_gemm(const __grid_
                             q.z = p.alpha * __uint_as_float(v[4 * j + 2]) + bsplit * o[j].z;
                             q.w = p.alpha * __uint_as_float(v[4 * j + 3]) + bsplit * o[j].w;
                             reinterpret_cast<float4*>(d)[j] = q;
+                            if (p.mc_out) mc_red4(mc_of(d) + 4 * j, q);
                         }
                     } else {
                         int dofs[32];
 #pragma unroll
                         for (int j = 0; j < 32; ++j) dofs[j] = nb + j < p.N ? j : -1;
-                        rmw32(d, dofs, 1, v, p.alpha, bsplit, p.atomic);
+                        rmw32(d, dofs, 1, v, p.alpha, bsplit, p.atomic, mc_of(d));
                     }
                 } else if (p.out_bf16) {
                     __nv_bfloat16* d = (__nv_bfloat16*)outT + (size_t)mrow * p.ldc + nb;
@@ -1628,6 +1640,9 @@ __global__ void __launch_bounds__(threads_for(AM), 1) tc_conv_gemm(const __grid_
                 const int nq = p.BN / 4;
                 const int pitch = p.BN + 4;
                 const float bsplit = g == 0 ? p.beta : 1.f;
+                // NEXT-3: the last split group writes the final dw: it also adds the
+                // cross-rank sum through the multicast address
+                const bool final_mc = p.mc_out != nullptr && g == p.mc_group;
                 unsigned long long* turn =
                     p.turns ? p.turns + ((size_t)(batch * per_z + rem) * p.cl + rho) : nullptr;
                 const uint32_t stg = smem_u32(smem);
@@ -1694,13 +1709,21 @@ __global__ void __launch_bounds__(threads_for(AM), 1) tc_conv_gemm(const __grid_
                                 float* d = outF + (size_t)(m0 + rr) * p.ldc + col0;
                                 const float4 o = make_float4(sum[uu].x + bsplit * old[uu].x, sum[uu].y + bsplit * old[uu].y,
                                                              sum[uu].z + bsplit * old[uu].z, sum[uu].w + bsplit * old[uu].w);
+                                float* mcd = final_mc ? p.mc_out + (d - (const float*)p.out) : nullptr;
                                 if (vec) {
                                     *reinterpret_cast<float4*>(d) = o;
+                                    if (mcd) mc_red4(mcd, o);
                                 } else {
                                     if (col0 < p.N) d[0] = o.x;
                                     if (col0 + 1 < p.N) d[1] = o.y;
                                     if (col0 + 2 < p.N) d[2] = o.z;
                                     if (col0 + 3 < p.N) d[3] = o.w;
+                                    if (mcd) {
+                                        if (col0 < p.N) mc_red(mcd, o.x);
+                                        if (col0 + 1 < p.N) mc_red(mcd + 1, o.y);
+                                        if (col0 + 2 < p.N) mc_red(mcd + 2, o.z);
+                                        if (col0 + 3 < p.N) mc_red(mcd + 3, o.w);
+                                    }
                                 }
                             }
                         } else {
@@ -1719,7 +1742,11 @@ __global__ void __launch_bounds__(threads_for(AM), 1) tc_conv_gemm(const __grid_
                                 }
 #pragma unroll
                                 for (int j = 0; j < 4; ++j)
-                                    if (o[j] >= 0) outF[o[j]] = sv[j] + bsplit * ov[j];
+                                    if (o[j] >= 0) {
+                                        const float fv = sv[j] + bsplit * ov[j];
+                                        outF[o[j]] = fv;
+                                        if (final_mc) mc_red(p.mc_out + (outF + o[j] - (const float*)p.out), fv);
+                                    }
                             }
                         }
                     }

@@ -119,6 +119,7 @@ class ConvNet:
         self.tensors: List[Dict[str, torch.Tensor]] = []
         self.workspaces: Dict[Tuple[int, int], Optional[torch.Tensor]] = {}
         self.net_ws: Optional[torch.Tensor] = None
+        self.nvls = None  # distributed.NvlsGradReduce over dw_flat (NEXT-3), set by the caller
 
     # ----------------------------------------------------------- memory --
     def allocate(self, seed: int = 0, kind: str = "normal", generator=None):
@@ -280,6 +281,9 @@ class ConvNet:
             T.conv_forward(self.h, k.desc, k.plan, t["x"], t["w"], t["y"], workspace=ws)
         elif conv_type == L.BWD_DATA:
             T.conv_backward_data(self.h, k.desc, k.plan, t["dy"], t["w"], t["dx"], workspace=ws)
+        elif self.nvls is not None:  # NEXT-3: the cross-rank sum fused into the epilogue
+            T.conv_backward_filter_nvls(self.h, k.desc, k.plan, t["x"], t["dy"], t["dw"],
+                                        self.nvls.mc_ptr(t["dw"], self.dw_flat), beta=1.0, workspace=ws)
         else:  # dw was zeroed at the start of the backward pass (zero_grad): accumulate
             T.conv_backward_filter(self.h, k.desc, k.plan, t["x"], t["dy"], t["dw"], beta=1.0, workspace=ws)
 
@@ -305,6 +309,8 @@ class ConvNet:
         for i, t in order:
             if t != L.FWD and not zeroed:
                 self.dw_flat.zero_()  # zero_grad, once per iteration, before the first backward call
+                if self.nvls is not None:
+                    self.nvls.begin()
                 zeroed = True
             if on_op:
                 on_op(i, t, "begin")
@@ -313,6 +319,8 @@ class ConvNet:
                 on_op(i, t, "end")
             if t == L.BWD_FILTER and grad_hook is not None:
                 grad_hook(i, self.tensors[i]["dw"])
+        if self.nvls is not None and zeroed:
+            self.nvls.end()
 
     def _iteration_concurrent(self, grad_hook, skip_conv1_dgrad, on_op=None):
         """on_op(i, type, 'begin'|'end') runs on the host around each call with the
@@ -333,6 +341,8 @@ class ConvNet:
         for i in range(len(self.layers)):
             run(i, L.FWD)
         self.dw_flat.zero_()  # zero_grad, once per iteration, before the first backward call
+        if self.nvls is not None:
+            self.nvls.begin()
         for i in reversed(range(len(self.layers))):
             if i == len(self.layers) - 1:
                 hook(i, L.BWD_DATA, "first")  # stream-ordered setup before any backward call
@@ -346,6 +356,8 @@ class ConvNet:
                 if grad_hook is not None:
                     grad_hook(i, self.tensors[i]["dw"])
         main.wait_stream(side)
+        if self.nvls is not None:
+            self.nvls.end()
 
     def flops_per_iteration(self, skip_conv1_dgrad: bool = False) -> int:
         f = sum(layer_flops(self.layers[i], self.n) for (i, t) in self.kernels)

@@ -90,6 +90,21 @@ def conv_backward_filter(h: L.Handle, d: L.ConvDesc, plan, x, dy, dw=None, alpha
     return dw
 
 
+def conv_backward_filter_nvls(h: L.Handle, d: L.ConvDesc, plan, x, dy, dw, dw_mc: int, alpha=1.0, beta=0.0,
+                              workspace=None):
+    """conv_backward_filter + the fused cross-rank sum (NEXT-3): the final dw values
+    are also added to every rank's copy of the NVLS buffer at multicast address dw_mc."""
+    xs, ws_, ys = shapes(d)
+    dt = _dtype(d.math)
+    _check_tensor(x, xs, dt, "x")
+    _check_tensor(dy, ys, dt, "dy")
+    _check_tensor(dw, ws_, torch.float32, "dw")
+    wp, wb = _ws(workspace)
+    h.conv_backward_filter_nvls(d, plan, alpha, x.data_ptr(), dy.data_ptr(), beta, dw.data_ptr(), int(dw_mc), wp, wb,
+                                _stream())
+    return dw
+
+
 def run(h: L.Handle, d: L.ConvDesc, conv_type: int, plan, a, b, out=None, alpha=1.0, beta=0.0, workspace=None):
     """Dispatch by conv type: FWD (x, w) -> y; DGRAD (dy, w) -> dx; WGRAD (x, dy) -> dw."""
     fn = {L.FWD: conv_forward, L.BWD_DATA: conv_backward_data, L.BWD_FILTER: conv_backward_filter}[conv_type]

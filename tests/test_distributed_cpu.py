@@ -219,3 +219,40 @@ def test_gloo_convnet_iteration_allreduce():
                 assert np.array_equal(np.load(os.path.join(d, f"dw{i}_{rank}.npy")), full_dw.astype(np.float32))
                 # I7: per-sample forward identical to the single-device full batch
                 assert np.array_equal(np.load(os.path.join(d, f"y{i}_{rank}.npy")), full_y[lo:hi].astype(np.float32))
+
+
+def _fd_worker(rank, world, port, out_dir):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port), RANK=str(rank), WORLD_SIZE=str(world),
+                      LOCAL_RANK=str(rank))
+    import sys
+    sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+    from paper_conf_cluster_oyamabhm18_b200.distributed import init_from_env, share_fd
+    assert init_from_env("gloo")
+    fd = None
+    if rank == 0:
+        # an anonymous object only rank 0 holds (like the exported multicast handle)
+        fd = os.memfd_create("nvls-probe")
+        os.write(fd, b"multicast handle of rank 0")
+    got = share_fd(fd)
+    if rank == 0:
+        assert got == fd
+    os.lseek(got, 0, os.SEEK_SET)
+    data = os.read(got, 64)
+    with open(os.path.join(out_dir, f"fd{rank}.txt"), "wb") as f:
+        f.write(data)
+    dist.barrier()
+    os.close(got)
+    dist.destroy_process_group()
+
+
+def test_share_fd_gloo():
+    """NEXT-3 setup: rank 0's exported handle (a POSIX fd) reaches every rank
+    through pidfd_getfd over the process group (world size 2)."""
+    if not hasattr(os, "pidfd_open") or not hasattr(os, "memfd_create"):
+        pytest.skip("pidfd_open / memfd_create unavailable")
+    world = 2
+    with tempfile.TemporaryDirectory() as d:
+        mp.spawn(_fd_worker, args=(world, _free_port(), d), nprocs=world, join=True)
+        for r in range(world):
+            with open(os.path.join(d, f"fd{r}.txt"), "rb") as f:
+                assert f.read() == b"multicast handle of rank 0"

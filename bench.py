@@ -71,9 +71,10 @@ def parse():
     ap.add_argument("--nondeterministic", action="store_true",
                     help="BackwardFilter split-K partials added with L2 atomics (mucu_set_deterministic(0)); "
                          "default: fixed-order reduction, bitwise reproducible dW")
-    ap.add_argument("--grad-reduce", default="nccl", choices=["nccl", "nvls"],
+    ap.add_argument("--grad-reduce", default="nccl", choices=["nccl", "nvls", "p2p"],
                     help="cross-rank dW sum: async NCCL allreduce per layer, or fused into the BackwardFilter "
-                         "epilogue through NVLink multicast (NEXT-3; also runs at one GPU)")
+                         "epilogue (NEXT-3): multimem.red to an NVLink multicast buffer (nvls) or red.global.add "
+                         "to every rank's buffer over NVLink P2P (p2p); both also run at one GPU")
     ap.add_argument("--json-out", default="")
     ap.add_argument("--tables-in", default="", help="benchmark DB (.npz) to plan from instead of benchmarking")
     ap.add_argument("--tables-out", default="", help="write the benchmark DB (.npz) after the benchmark pass")
@@ -339,11 +340,11 @@ def main():
     bench_s = time.perf_counter() - t0
     flush = torch.empty(512 * 2 ** 20, dtype=torch.uint8, device=dev)
     grad_ar = GradAllreduce()
-    if args.grad_reduce == "nvls":
-        # NEXT-3: the dW sum is fused into BackwardFilter (multimem.red into every rank's
-        # copy of an NVLS buffer); no per-layer collective call remains
-        from paper_conf_cluster_oyamabhm18_b200.distributed import NvlsGradReduce
-        net.nvls = NvlsGradReduce(net.dw_flat.numel(), local)
+    if args.grad_reduce != "nccl":
+        # NEXT-3: the dW sum is fused into BackwardFilter (the final dw writer adds every
+        # value to all ranks' sum buffers); no per-layer collective call remains
+        from paper_conf_cluster_oyamabhm18_b200.distributed import FusedGradReduce
+        net.nvls = FusedGradReduce(net.dw_flat.numel(), local, kind=args.grad_reduce)
         grad_ar = _NoReduce()
     stream = torch.cuda.current_stream()
 
@@ -566,9 +567,12 @@ def main():
                        "l2": "512 MiB buffer overwritten before every timed step",
                        "first_layer_backward_data": bool(args.input_grad),
                        "backward_streams": 2 if args.concurrent_wgrad else 1,
-                       "grad_reduce": ("fused multimem.red into an NVLS buffer (BackwardFilter epilogue) + 2 NVLS "
-                                       "barriers per step" if args.grad_reduce == "nvls"
-                                       else "async NCCL allreduce per layer" if world > 1 else "none (1 GPU)"),
+                       "grad_reduce": ({"nvls": "fused into the BackwardFilter epilogue: multimem.red to an NVLS "
+                                                "buffer, 2 device barriers per step",
+                                        "p2p": "fused into the BackwardFilter epilogue: red.global.add to every "
+                                               "rank's buffer over NVLink P2P, 2 device barriers per step"}
+                                       .get(args.grad_reduce) or
+                                       ("async NCCL allreduce per layer" if world > 1 else "none (1 GPU)")),
                        "wgrad_reduction": ("split-K with fp32 L2 atomics (non-deterministic)" if args.nondeterministic
                                            else "ordered split-K (deterministic)")},
             "images_per_s": round(args.batch * world / (ms_max * 1e-3), 1),

@@ -267,29 +267,59 @@ mucu_status_t mucu_conv_backward_filter(mucu_handle_t handle, const mucu_conv_de
                                         const void* x, const void* dy, float beta, float* dw,
                                         void* workspace, uint64_t ws_bytes, void* cuda_stream);
 
-/* ------------------------------------------- NEXT-3: NVLS dW reduction ---- */
+/* ------------------------------------------- NEXT-3: fused dW reduction ---- */
 /* Data-parallel training sums every layer's dW over the ranks (micro-
  * batching lets "the communication of parameter gradients" be hidden; SURVEY
  * 8(f) NEXT-3).  Here the sum is fused into BackwardFilter: the kernel that
  * writes a dw element's final value (the last micro-batch's epilogue, its last
- * ordered split group, or the partial-slot reduction; a push kernel after the
- * F32 SIMT / Winograd / FFT / atomic writers) also adds it with
- * `multimem.red.add.f32` to the NVLink multicast address of a symmetric fp32
- * buffer, so NVSwitch accumulates it into every rank's copy.
- *
- * Multicast object, one per rank (device = this rank's CUDA device, ranks =
- * world size, bytes = user bytes; all ranks pass the same values):
+ * ordered split group, or the partial-slot reduction; one push kernel after the
+ * F32 SIMT / Winograd / FFT / atomic split-K writers) also adds it to a
+ * reduction target, element-aligned with dw:
+ *   multicast = 1, count = 1: dst[0] is the NVLink multicast address of a
+ *     symmetric fp32 buffer (mucu_nvls_*): one multimem.red.add.f32 per value,
+ *     NVSwitch adds it into every rank's copy;
+ *   multicast = 0, count = ranks: dst[r] is rank r's buffer (a peer pointer over
+ *     NVLink P2P, or this rank's own): one red.global.add.f32 per rank.
+ * Protocol per iteration: zero this rank's buffer, barrier, every rank's
+ * backward_filter_reduce calls, barrier; then every rank's buffer holds the sum
+ * over ranks of dw.  Additions arrive in any order (exact for 2 ranks, since
+ * 0 + a + b = 0 + b + a; flush-to-zero like every fp32 reduction).
+ * Errors: INVALID_VALUE (count outside 1..MUCU_MAX_REDUCE_RANKS, multicast with
+ * count != 1), MISALIGNED (a dst NULL or not 16-byte aligned), else as
+ * mucu_conv_backward_filter. */
+#define MUCU_MAX_REDUCE_RANKS 8
+typedef struct {
+    int32_t multicast;
+    int32_t count;
+    float* dst[MUCU_MAX_REDUCE_RANKS];
+} mucu_reduce_target_t;
+/* dw (device, this rank's) receives exactly what mucu_conv_backward_filter
+ * computes; the target receives += the same final values. */
+mucu_status_t mucu_conv_backward_filter_reduce(mucu_handle_t handle, const mucu_conv_desc_t* desc,
+                                               const mucu_micro_config_t* plan, int32_t count, float alpha,
+                                               const void* x, const void* dy, float beta, float* dw,
+                                               const mucu_reduce_target_t* target, void* workspace,
+                                               uint64_t ws_bytes, void* cuda_stream);
+/* Device-side barrier over the ranks, enqueued on cuda_stream: a system-scope
+ * release of this rank's earlier reductions, +1 on every flag word of `flags`
+ * (uint32 words cast to float*: one multicast address, or every rank's flag),
+ * then a wait until *own (this rank's flag, device) >= target (= ranks x
+ * barriers so far; every rank calls it equally often).  A wait longer than 10 s
+ * traps (the stream reports a CUDA error) instead of hanging. */
+mucu_status_t mucu_peer_barrier(const mucu_reduce_target_t* flags, const uint32_t* own, uint32_t target,
+                                void* cuda_stream);
+
+/* NVLink multicast object, one per rank (device = this rank's CUDA device,
+ * ranks = world size, bytes = user bytes; all ranks pass the same values):
  *   rank 0: mucu_nvls_create, mucu_nvls_export -> a POSIX fd owned by the
  *           caller, passed to the peers (pidfd_getfd);
  *   others: mucu_nvls_import(fd);
  *   all:    mucu_nvls_bind -> local (this rank's copy, unicast) and multicast
  *           addresses of the user bytes; blocks until every rank has created or
  *           imported; the buffer starts zeroed.
- * mucu_nvls_barrier(stream): enqueue a device-side barrier over the ranks
- *   (system-scope release of this rank's earlier multimem reductions, then wait
- *   for every rank's) -- every rank calls it the same number of times.
+ * mucu_nvls_barrier(stream): mucu_peer_barrier on the object's own flag word.
  * Errors: UNSUPPORTED (no multicast on the device), CUDA (driver call failed,
- *   detail in mucu_last_error), INVALID_VALUE. */
+ *   e.g. no NVSwitch fabric; detail in mucu_last_error), INVALID_VALUE. */
 typedef struct mucu_nvls* mucu_nvls_t;
 mucu_status_t mucu_nvls_supported(int device, int32_t* supported);     /* host */
 mucu_status_t mucu_nvls_create(int device, int32_t ranks, uint64_t bytes, mucu_nvls_t* out);
@@ -298,18 +328,6 @@ mucu_status_t mucu_nvls_import(int device, int32_t ranks, uint64_t bytes, int32_
 mucu_status_t mucu_nvls_bind(mucu_nvls_t nv, void** local, void** multicast);
 mucu_status_t mucu_nvls_barrier(mucu_nvls_t nv, void* cuda_stream);
 mucu_status_t mucu_nvls_destroy(mucu_nvls_t nv);
-/* mucu_conv_backward_filter plus the fused reduction: dw (device, private to
- * this rank) receives this rank's gradient exactly as mucu_conv_backward_filter
- * computes it; dw_mc (the multicast address of a K*R*S*C fp32 region of a bound
- * NVLS buffer, 16-byte aligned) receives += the same values on every rank's
- * copy.  Protocol per iteration: zero the local copies, mucu_nvls_barrier, each
- * rank's backward_filter_nvls calls, mucu_nvls_barrier; then every rank's local
- * copy holds sum over ranks of dw.  Addition order across ranks is the order the
- * switch receives them (exact for 2 ranks; FTZ like any fp32 reduction). */
-mucu_status_t mucu_conv_backward_filter_nvls(mucu_handle_t handle, const mucu_conv_desc_t* desc,
-                                             const mucu_micro_config_t* plan, int32_t count, float alpha,
-                                             const void* x, const void* dy, float beta, float* dw, float* dw_mc,
-                                             void* workspace, uint64_t ws_bytes, void* cuda_stream);
 
 /* ------------------------------------------------------------ WD ---- */
 /* WD needs every kernel before optimising: register the kernels,

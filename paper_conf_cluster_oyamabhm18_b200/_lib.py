@@ -43,6 +43,24 @@ class ConvDesc(ctypes.Structure):
         return "ConvDesc(" + ", ".join(f"{f}={getattr(self, f)}" for f, _ in self._fields_) + ")"
 
 
+MAX_REDUCE_RANKS = 8
+
+
+class ReduceTarget(ctypes.Structure):
+    """mucu_reduce_target_t: one multicast address, or one buffer per rank (NEXT-3)."""
+    _fields_ = [("multicast", ctypes.c_int32), ("count", ctypes.c_int32),
+                ("dst", ctypes.c_void_p * MAX_REDUCE_RANKS)]
+
+
+def reduce_target(ptrs: Sequence[int], multicast: bool = False) -> ReduceTarget:
+    t = ReduceTarget()
+    t.multicast = 1 if multicast else 0
+    t.count = len(ptrs)
+    for i, p in enumerate(ptrs):
+        t.dst[i] = p
+    return t
+
+
 class MicroConfig(ctypes.Structure):
     _fields_ = [("algo", ctypes.c_int32), ("micro_n", ctypes.c_int32)]
 
@@ -79,7 +97,9 @@ def _load():
         "mucu_conv_forward": (ctypes.c_int, [vp, D, MC, i32, f32, vp, vp, f32, vp, vp, u64, vp]),
         "mucu_conv_backward_data": (ctypes.c_int, [vp, D, MC, i32, f32, vp, vp, f32, vp, vp, u64, vp]),
         "mucu_conv_backward_filter": (ctypes.c_int, [vp, D, MC, i32, f32, vp, vp, f32, vp, vp, u64, vp]),
-        "mucu_conv_backward_filter_nvls": (ctypes.c_int, [vp, D, MC, i32, f32, vp, vp, f32, vp, vp, vp, u64, vp]),
+        "mucu_conv_backward_filter_reduce": (ctypes.c_int, [vp, D, MC, i32, f32, vp, vp, f32, vp, P(ReduceTarget), vp,
+                                                             u64, vp]),
+        "mucu_peer_barrier": (ctypes.c_int, [P(ReduceTarget), vp, ctypes.c_uint32, vp]),
         "mucu_nvls_supported": (ctypes.c_int, [ctypes.c_int, P(i32)]),
         "mucu_nvls_create": (ctypes.c_int, [ctypes.c_int, i32, u64, P(vp)]),
         "mucu_nvls_export": (ctypes.c_int, [vp, P(i32)]),
@@ -289,12 +309,17 @@ class Handle:
     def conv_backward_filter(self, d, plan, alpha, x, dy, beta, dw, ws_ptr, ws_bytes, stream):
         self._conv(lib.mucu_conv_backward_filter, d, plan, alpha, x, dy, beta, dw, ws_ptr, ws_bytes, stream)
 
-    def conv_backward_filter_nvls(self, d, plan, alpha, x, dy, beta, dw, dw_mc, ws_ptr, ws_bytes, stream):
+    def conv_backward_filter_reduce(self, d, plan, alpha, x, dy, beta, dw, target: ReduceTarget, ws_ptr, ws_bytes,
+                                    stream):
         arr = _plan_array(plan)
-        _check(lib.mucu_conv_backward_filter_nvls(
+        _check(lib.mucu_conv_backward_filter_reduce(
             self._h, ctypes.byref(d), arr, len(plan), float(alpha), ctypes.c_void_p(x), ctypes.c_void_p(dy),
-            float(beta), ctypes.c_void_p(dw), ctypes.c_void_p(dw_mc), ctypes.c_void_p(ws_ptr or 0), int(ws_bytes),
+            float(beta), ctypes.c_void_p(dw), ctypes.byref(target), ctypes.c_void_p(ws_ptr or 0), int(ws_bytes),
             ctypes.c_void_p(stream)))
+
+
+def peer_barrier(flags: ReduceTarget, own: int, target: int, stream: int = 0):
+    _check(lib.mucu_peer_barrier(ctypes.byref(flags), ctypes.c_void_p(own), int(target), ctypes.c_void_p(stream)))
 
 
 def nvls_supported(device: int = 0) -> bool:

@@ -571,7 +571,7 @@ static mucu_status_t check_ptr(const void* p, const char* what) {
 
 static mucu_status_t execute(mucu_handle_t h, const mucu_conv_desc_t* d, int type, const mucu_micro_config_t* plan,
                              int32_t count, float alpha, const void* in0, const void* in1, float beta, void* out,
-                             void* ws, uint64_t ws_bytes, void* stream, float* dw_mc = nullptr) {
+                             void* ws, uint64_t ws_bytes, void* stream, const RedTarget* red = nullptr) {
     if (!h) return set_error(MUCU_ERR_INVALID_VALUE, "null handle");
     Geom g;
     if (!make_geom(d, &g)) return set_error(MUCU_ERR_INVALID_VALUE, "invalid descriptor");
@@ -634,7 +634,7 @@ static mucu_status_t execute(mucu_handle_t h, const mucu_conv_desc_t* d, int typ
         }
     }
     CallCtx ctx;
-    ctx.mc_out = dw_mc;
+    if (red) ctx.red = *red;
     int64_t done = 0;
     for (int32_t i = 0; i < count; ++i) {
         const int32_t b = plan[i].micro_n;
@@ -647,11 +647,11 @@ static mucu_status_t execute(mucu_handle_t h, const mucu_conv_desc_t* d, int typ
         if (s) return s;
         done += b;
     }
-    if (dw_mc && !ctx.mc_fused) {
+    if (red && !ctx.mc_fused) {
         // NEXT-3: the last micro-configuration's dw writer did not take the reduction
-        // (F32 SIMT, Winograd, FFT, atomic split-K): push the final dw through NVLS
-        const int e = launch_nvls_push((const float*)out, dw_mc, (int64_t)g.k * g.r * g.s * g.c, st);
-        if (e) return set_error(MUCU_ERR_CUDA, "nvls push: %s", cudaGetErrorString((cudaError_t)e));
+        // (F32 SIMT, Winograd, FFT, atomic split-K): push the final dw
+        const int e = launch_reduce_push((const float*)out, *red, (int64_t)g.k * g.r * g.s * g.c, st);
+        if (e) return set_error(MUCU_ERR_CUDA, "reduce push: %s", cudaGetErrorString((cudaError_t)e));
     }
     return MUCU_OK;
 }
@@ -676,12 +676,24 @@ extern "C" mucu_status_t mucu_conv_backward_filter(mucu_handle_t h, const mucu_c
     return execute(h, d, MUCU_BWD_FILTER, plan, count, alpha, x, dy, beta, dw, ws, ws_bytes, stream);
 }
 
-extern "C" mucu_status_t mucu_conv_backward_filter_nvls(mucu_handle_t h, const mucu_conv_desc_t* d,
-                                                        const mucu_micro_config_t* plan, int32_t count, float alpha,
-                                                        const void* x, const void* dy, float beta, float* dw,
-                                                        float* dw_mc, void* ws, uint64_t ws_bytes, void* stream) {
-    if (!dw_mc || ((uintptr_t)dw_mc & 15)) return set_error(MUCU_ERR_MISALIGNED, "dw_mc NULL or not 16-byte aligned");
-    return execute(h, d, MUCU_BWD_FILTER, plan, count, alpha, x, dy, beta, dw, ws, ws_bytes, stream, dw_mc);
+extern "C" mucu_status_t mucu_conv_backward_filter_reduce(mucu_handle_t h, const mucu_conv_desc_t* d,
+                                                          const mucu_micro_config_t* plan, int32_t count, float alpha,
+                                                          const void* x, const void* dy, float beta, float* dw,
+                                                          const mucu_reduce_target_t* target, void* ws,
+                                                          uint64_t ws_bytes, void* stream) {
+    if (!target || target->count < 1 || target->count > MUCU_MAX_REDUCE_RANKS ||
+        (target->multicast && target->count != 1))
+        return set_error(MUCU_ERR_INVALID_VALUE, "reduce target: count must be 1..%d (1 for multicast)",
+                         MUCU_MAX_REDUCE_RANKS);
+    RedTarget red = {};
+    for (int r = 0; r < target->count; ++r) {
+        if (!target->dst[r] || ((uintptr_t)target->dst[r] & 15))
+            return set_error(MUCU_ERR_MISALIGNED, "reduce target %d NULL or not 16-byte aligned", r);
+        red.dst[r] = target->dst[r];
+    }
+    red.n = target->count;
+    red.mc = target->multicast ? 1 : 0;
+    return execute(h, d, MUCU_BWD_FILTER, plan, count, alpha, x, dy, beta, dw, ws, ws_bytes, stream, &red);
 }
 
 // ============================================================ benchmark ====

@@ -850,7 +850,7 @@ int launch_wgw_transforms(const Geom& g, int32_t b, const void* x, const void* d
 // coalesced along n).
 __global__ void partial_reduce_kernel(int S, int64_t slot, int ldp, int M, int N, bool transpose,
                                       const float* __restrict__ part, float alpha, float beta, float* __restrict__ out,
-                                      float* mc) {
+                                      const RedTarget red) {
     pdl_entry();
     const int64_t total = (int64_t)M * N;
     for (int64_t idx = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; idx < total;
@@ -862,14 +862,16 @@ __global__ void partial_reduce_kernel(int S, int64_t slot, int ldp, int M, int N
         float* d = transpose ? out + (size_t)n * M + m : out + idx;
         const float o = beta != 0.f ? alpha * acc + beta * *d : alpha * acc;
         *d = o;
-        if (mc) mc_red(mc + (d - out), o);  // NEXT-3: the cross-rank dW sum
+        if (red.n) red_add(red, d - out, o);  // NEXT-3: the cross-rank dW sum
     }
 }
 
 int launch_partial_reduce(int S, int64_t slot, int ldp, int M, int N, bool transpose, const float* part,
-                          float alpha, float beta, float* out, cudaStream_t st, float* mc) {
+                          float alpha, float beta, float* out, cudaStream_t st, const RedTarget* red) {
+    RedTarget r = {};
+    if (red) r = *red;
     launch_pdl(partial_reduce_kernel, dim3(grid_for((int64_t)M * N, 256)), dim3(256), (size_t)0, st, S, slot, ldp,
-               M, N, transpose, part, alpha, beta, out, mc);
+               M, N, transpose, part, alpha, beta, out, r);
     count_launch();
     return (int)cudaGetLastError();
 }

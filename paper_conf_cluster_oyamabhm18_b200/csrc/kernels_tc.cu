@@ -320,11 +320,12 @@ struct TcArgs {
     int m64;                 // MN-major A: the tile's last 128-row half has <= 64 valid rows -> M = 64 MMAs
     unsigned long long* turns;
     unsigned long long epoch;
-    // NEXT-3: multicast (NVLS) address of the cross-rank dW sum, aligned
-    // with `out`; the final writer of every dw element also adds it there with
-    // multimem.red (cluster split-K: split group mc_group is the final one).  nullptr: off.
-    float* mc_out;
-    int mc_group;
+    // NEXT-3: the cross-rank dW sum, element-aligned with `out`; the final
+    // writer of every dw element also adds its value there (multimem.red to a multicast
+    // address, or red.global.add per rank buffer; cluster split-K: split group red_group
+    // is the final one).  red.n = 0: off.
+    RedTarget red;
+    int red_group;
 };
 
 constexpr int kThreads = 288;  // 4 producer warps, 1 MMA warp, 4 epilogue warps
@@ -520,9 +521,9 @@ struct Launch {
     CUtensorMap ta, tb;
     dim3 grid;
     Im2colArgs ia;
-    // NEXT-3: the call's multicast dW (last micro-batch only), its local dw and the
+    // NEXT-3: the call's reduction target (last micro-batch only), its local dw and the
     // executor's "fused" flag (set when this launch writes dw and takes the reduction)
-    float* mc_out;
+    const RedTarget* red;
     const void* mc_local;
     bool* mc_fused;
 };
@@ -550,16 +551,16 @@ int launch_t(Launch& L, cudaStream_t st, bool dry) {
     if (!SPLITK && L.a.cl) return -1;
     L.a.turns = nullptr;
     L.a.epoch = 0;
-    L.a.mc_out = nullptr;
-    L.a.mc_group = 0;
+    L.a.red.n = 0;
+    L.a.red_group = 0;
     if (dry) return 0;
     // NEXT-3: the launch that writes the call's dw in the last micro-batch is its final
     // writer (one dw-writing launch per micro-configuration; split-K groups ordered):
     // fuse the cross-rank reduction into its epilogue.  Atomic split-K partials and
     // batched (Winograd) outputs are not final values: the executor pushes dw instead.
-    if (SPLITK && EPI != EPI_WGRAD_PARTIAL && L.mc_out && L.a.out == L.mc_local && !L.a.atomic && !L.a.zsplit) {
-        L.a.mc_out = L.mc_out;
-        L.a.mc_group = L.a.cl ? L.a.num_z / L.a.cl - 1 : 0;
+    if (SPLITK && EPI != EPI_WGRAD_PARTIAL && L.red && L.a.out == L.mc_local && !L.a.atomic && !L.a.zsplit) {
+        L.a.red = *L.red;
+        L.a.red_group = L.a.cl ? L.a.num_z / L.a.cl - 1 : 0;
         *L.mc_fused = true;
     }
     if (SPLITK && L.a.atomic && L.a.beta != 1.f) {
@@ -760,11 +761,11 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
     A.tapR = g.r; A.tapS = g.s; A.ph_u = 1;
     A.max_lag = std::min(6, std::max(1, env_int("MUCU_MAX_LAG", 6)));
     A.alpha = alpha; A.beta = beta; A.out = out; A.out_bf16 = bf ? 1 : 0;
-    if (type == MUCU_BWD_FILTER && ctx->mc_out && ctx->mc_last) {
-        L.mc_out = ctx->mc_out; L.mc_local = out; L.mc_fused = &ctx->mc_fused;
+    if (type == MUCU_BWD_FILTER && ctx->red.n && ctx->mc_last) {
+        L.red = &ctx->red; L.mc_local = out; L.mc_fused = &ctx->mc_fused;
     }
-    // partial-slot reductions are the final writer of dw: they take the multicast sum
-    float* const mc_reduce = L.mc_out;
+    // partial-slot reductions are the final writer of dw: they take the cross-rank sum
+    const RedTarget* const mc_reduce = L.red;
     auto note_fused = [&]() { if (mc_reduce && !dry) ctx->mc_fused = true; };
     auto map2 = [&](CUtensorMap* tm, const void* base, uint64_t d0, uint64_t d1, uint64_t pitch_elems, uint32_t b0,
                     uint32_t b1, bool mn = false) {

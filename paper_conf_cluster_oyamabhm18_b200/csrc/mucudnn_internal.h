@@ -91,6 +91,15 @@ struct WsLayout {
 };
 mucu_status_t ws_layout(const Geom& g, int type, int algo, int32_t b, WsLayout* out);
 
+// NEXT-3 reduction target of BackwardFilter (the public mucu_reduce_target_t):
+// element-aligned with dw; n = 0: off.
+constexpr int kMaxRedRanks = MUCU_MAX_REDUCE_RANKS;
+struct RedTarget {
+    float* dst[kMaxRedRanks];
+    int n;
+    int mc;
+};
+
 // Per-call executor state (which b-independent workspace prefix is valid).
 struct CallCtx {
     int fixed_kind = 0;  // 0 none, 1 padded filter, 2 Winograd U, 3/4 space-to-depth filter, 5 FFT filter spectrum
@@ -98,10 +107,10 @@ struct CallCtx {
     int last_algo = -1;  // algorithm of the previous micro-config (prefix invalidation)
     bool dry = false;    // tensor-core dispatch decisions only, no launch (pre-validation)
     bool deterministic = true;  // BackwardFilter split-K: ordered reduction (default) or L2 atomics
-    // NEXT-3: multicast address of the cross-rank dW sum (nullptr: off),
-    // set for the call's last micro-configuration (mc_last); the final dw writer sets
-    // mc_fused when it took the reduction in its epilogue.
-    float* mc_out = nullptr;
+    // NEXT-3: the cross-rank dW sum target (red.n = 0: off), used by the
+    // call's last micro-configuration (mc_last); the final dw writer sets mc_fused when
+    // it took the reduction in its epilogue.
+    RedTarget red = {};
     bool mc_last = false;
     bool mc_fused = false;
 };
@@ -126,16 +135,30 @@ struct FastDiv {
         return (uint32_t)(((uint64_t)__umulhi(n, m) + n) >> l);
     }
 };
-// NEXT-3: add v to every rank's copy of a multicast (NVLS) object address.  The
-// reduction is performed by NVSwitch; relaxed, system scope (made visible to the
-// peers by the release of the NVLS barrier, nvls.cu).
-__device__ __forceinline__ void mc_red(float* a, float v) {
-    asm volatile("multimem.red.relaxed.sys.global.add.f32 [%0], %1;" ::"l"(a), "f"(v) : "memory");
+// NEXT-3: add v at element offset `off` of the reduction target -- one multimem.red
+// to a multicast (NVLS) address (NVSwitch adds it into every rank's copy), or one
+// red.global.add per rank buffer (peer pointers over NVLink P2P; the rank's own
+// buffer at one rank).  Relaxed, system scope: made visible to the peers by the
+// release of the barrier (nvls.cu).
+__device__ __forceinline__ void red_add(const RedTarget& t, long long off, float v) {
+    if (t.mc) {
+        asm volatile("multimem.red.relaxed.sys.global.add.f32 [%0], %1;" ::"l"(t.dst[0] + off), "f"(v) : "memory");
+    } else {
+        for (int r = 0; r < t.n; ++r)
+            asm volatile("red.relaxed.sys.global.add.f32 [%0], %1;" ::"l"(t.dst[r] + off), "f"(v) : "memory");
+    }
 }
-__device__ __forceinline__ void mc_red4(float* a, float4 v) {  // a 16-byte aligned
-    asm volatile("multimem.red.relaxed.sys.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(a), "f"(v.x), "f"(v.y),
-                 "f"(v.z), "f"(v.w)
-                 : "memory");
+__device__ __forceinline__ void red_add4(const RedTarget& t, long long off, float4 v) {  // 16-B aligned
+    if (t.mc) {
+        asm volatile("multimem.red.relaxed.sys.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(t.dst[0] + off),
+                     "f"(v.x), "f"(v.y), "f"(v.z), "f"(v.w)
+                     : "memory");
+    } else {
+        for (int r = 0; r < t.n; ++r)
+            asm volatile("red.relaxed.sys.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(t.dst[r] + off), "f"(v.x),
+                         "f"(v.y), "f"(v.z), "f"(v.w)
+                         : "memory");
+    }
 }
 #endif
 
@@ -239,16 +262,15 @@ int launch_wgw_output(const Geom& g, float alpha, const float* M, float beta, fl
 // part[s][m][n] at slot stride `slot` (elements) and row pitch `ldp`; out[m][n] (row pitch
 // N), or out[n][m] (row pitch M) when `transpose`.  Summed in split order s = 0, 1, ...
 // (deterministic).
-// mc (NEXT-3): multicast address matching `out` -- the final values are also added
-// to the cross-rank dW sum (nullptr: off).
+// red (NEXT-3): the final values are also added to the cross-rank dW sum (n = 0: off).
 int launch_partial_reduce(int S, int64_t slot, int ldp, int M, int N, bool transpose, const float* part,
-                          float alpha, float beta, float* out, cudaStream_t st, float* mc = nullptr);
-// NEXT-3 (nvls.cu): mc[i] += src[i] on every rank's copy (multimem.red, 16-B vectors
-// where aligned) for the dw writers that do not fuse the reduction; and the NVLS
-// barrier: release-add 1 to the multicast flag word, wait until the local copy of it
-// reaches `target` (= ranks x barriers so far).
-int launch_nvls_push(const float* src, float* mc, int64_t n, cudaStream_t st);
-int launch_nvls_barrier(unsigned* mc_flag, const unsigned* uc_flag, unsigned target, cudaStream_t st);
+                          float alpha, float beta, float* out, cudaStream_t st, const RedTarget* red = nullptr);
+// NEXT-3 (nvls.cu): target[i] += src[i] (16-B vectors where aligned) for the dw writers
+// that do not fuse the reduction; and the barrier over the ranks: release-add 1 to
+// every flag word in `flags` (one multicast address, or every rank's flag), then wait
+// until this rank's own flag reaches `target` (= ranks x barriers so far).
+int launch_reduce_push(const float* src, const RedTarget& t, int64_t n, cudaStream_t st);
+int launch_reduce_barrier(const RedTarget& flags, const unsigned* own, unsigned target, cudaStream_t st);
 // Tensor-core I2C BackwardFilter of large-C layers: partial dW slots reserved in the
 // workspace (deterministic split-K over all SMs): ceil(148 / dW tiles of 128 x 128),
 // 1 = no partial slots.

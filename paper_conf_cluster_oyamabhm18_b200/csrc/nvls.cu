@@ -1,18 +1,20 @@
-// nvls.cu -- NEXT-3: the cross-rank dW reduction through
-// NVLink SHARP (NVLS) multicast, fused into the BackwardFilter epilogue.
+// nvls.cu -- NEXT-3: the cross-rank dW reduction fused
+// into the BackwardFilter epilogue.
 //
 // P:L17 motivates micro-batching with "hiding the communication of parameter
 // gradients": in data-parallel training every rank's dW must be summed across the
 // ranks.  Instead of a separate NCCL all-reduce after the layer's last micro-batch,
 // the kernel that writes a dw element's FINAL value (the last micro-batch's epilogue,
 // or its last ordered split group, or the partial-slot reduction) also adds that value
-// with `multimem.red.add` to the multicast address of a symmetric fp32 buffer: NVSwitch
-// performs the addition into every rank's copy.  When all ranks have passed the NVLS
-// barrier below, every copy holds sum_ranks dw_rank.
+// to the reduction target: with NVLink SHARP (NVLS), one `multimem.red.add` to the
+// multicast address of a symmetric fp32 buffer, which NVSwitch adds into every rank's
+// copy; without multicast, one `red.global.add` per rank buffer through NVLink P2P
+// pointers.  When all ranks have passed the barrier below, every rank's buffer holds
+// sum_ranks dw_rank.
 //
 // This file: the multicast object (driver VMM + multicast API, entry points resolved at
-// run time through the runtime -- no -lcuda), the fallback push kernel for dw writers
-// that do not fuse (F32 SIMT, Winograd, FFT, atomic split-K), and the barrier kernel.
+// run time through the runtime -- no -lcuda), the push kernel for dw writers that do
+// not fuse (F32 SIMT, Winograd, FFT, atomic split-K), and the barrier kernel.
 #include <cuda.h>
 #include <cuda_runtime.h>
 
@@ -25,28 +27,36 @@ namespace mucu {
 namespace {
 
 // ------------------------------------------------------------ kernels ----
-__global__ void nvls_push_kernel(const float* __restrict__ src, float* mc, int64_t n) {
-    const int64_t nv = ((((uintptr_t)src | (uintptr_t)mc) & 15) == 0) ? n / 4 : 0;
+__global__ void reduce_push_kernel(const float* __restrict__ src, const RedTarget t, int64_t n) {
+    bool al = ((uintptr_t)src & 15) == 0;
+    for (int r = 0; r < (t.mc ? 1 : t.n); ++r) al = al && ((uintptr_t)t.dst[r] & 15) == 0;
+    const int64_t nv = al ? n / 4 : 0;
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < nv; i += stride)
-        mc_red4(mc + 4 * i, __ldg(reinterpret_cast<const float4*>(src) + i));
+        red_add4(t, 4 * i, __ldg(reinterpret_cast<const float4*>(src) + i));
     for (int64_t i = 4 * nv + blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += stride)
-        mc_red(mc + i, __ldg(src + i));
+        red_add(t, i, __ldg(src + i));
 }
 
-// One thread: publish this rank's earlier multimem reductions (the kernels before this
-// one on the stream have completed; the system-scope release makes their writes
-// visible before the flag increment), then wait for every rank's increment.
-__global__ void nvls_barrier_kernel(unsigned* mc_flag, const unsigned* uc_flag, unsigned target) {
+// One thread: publish this rank's earlier reductions (the kernels before this one on
+// the stream have completed; the system-scope release orders their writes before the
+// flag increment), add 1 to every rank's flag (one multicast address or each rank's
+// flag word), then wait until this rank's own flag reaches `target`.
+__global__ void reduce_barrier_kernel(const RedTarget flags, const unsigned* own, unsigned target) {
     asm volatile("fence.proxy.alias;" ::: "memory");
     asm volatile("fence.acq_rel.sys;" ::: "memory");
-    asm volatile("multimem.red.release.sys.global.add.u32 [%0], %1;" ::"l"(mc_flag), "r"(1u) : "memory");
+    if (flags.mc) {
+        asm volatile("multimem.red.release.sys.global.add.u32 [%0], %1;" ::"l"(flags.dst[0]), "r"(1u) : "memory");
+    } else {
+        for (int r = 0; r < flags.n; ++r)
+            asm volatile("red.release.sys.global.add.u32 [%0], %1;" ::"l"(flags.dst[r]), "r"(1u) : "memory");
+    }
     const unsigned long long t0 = global_ns();
     for (;;) {
         unsigned v;
-        asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(uc_flag) : "memory");
+        asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(own) : "memory");
         if ((int)(v - target) >= 0) break;
-        if (global_ns() - t0 > kWatchdogNs) watchdog_trap("nvls barrier", (unsigned long long)uc_flag, target, v);
+        if (global_ns() - t0 > kWatchdogNs) watchdog_trap("reduce barrier", (unsigned long long)own, target, v);
         __nanosleep(64);
     }
     asm volatile("fence.proxy.alias;" ::: "memory");
@@ -114,17 +124,17 @@ const Drv& drv() {
 
 }  // namespace
 
-int launch_nvls_push(const float* src, float* mc, int64_t n, cudaStream_t st) {
-    if (n <= 0) return 0;
+int launch_reduce_push(const float* src, const RedTarget& t, int64_t n, cudaStream_t st) {
+    if (n <= 0 || t.n <= 0) return 0;
     const int64_t work = std::max<int64_t>(1, n / 4);
     const int grid = (int)std::min<int64_t>((work + 255) / 256, 148 * 8);
-    nvls_push_kernel<<<grid, 256, 0, st>>>(src, mc, n);
+    reduce_push_kernel<<<grid, 256, 0, st>>>(src, t, n);
     count_launch();
     return (int)cudaGetLastError();
 }
 
-int launch_nvls_barrier(unsigned* mc_flag, const unsigned* uc_flag, unsigned target, cudaStream_t st) {
-    nvls_barrier_kernel<<<1, 1, 0, st>>>(mc_flag, uc_flag, target);
+int launch_reduce_barrier(const RedTarget& flags, const unsigned* own, unsigned target, cudaStream_t st) {
+    reduce_barrier_kernel<<<1, 1, 0, st>>>(flags, own, target);
     count_launch();
     return (int)cudaGetLastError();
 }
@@ -285,9 +295,28 @@ extern "C" mucu_status_t mucu_nvls_bind(mucu_nvls_t nv, void** local, void** mul
 extern "C" mucu_status_t mucu_nvls_barrier(mucu_nvls_t nv, void* stream) {
     if (!nv || !nv->bound) return set_error(MUCU_ERR_INVALID_VALUE, "NVLS object not bound");
     ++nv->epoch;
-    const int e = launch_nvls_barrier((unsigned*)(nv->mc_va + nv->data), (const unsigned*)(nv->uc_va + nv->data),
-                                      nv->epoch * (unsigned)nv->ranks, (cudaStream_t)stream);
+    RedTarget f = {};
+    f.dst[0] = (float*)(nv->mc_va + nv->data);
+    f.n = 1;
+    f.mc = 1;
+    const int e = launch_reduce_barrier(f, (const unsigned*)(nv->uc_va + nv->data), nv->epoch * (unsigned)nv->ranks,
+                                        (cudaStream_t)stream);
     return e ? set_error(MUCU_ERR_CUDA, "nvls barrier launch: %s", cudaGetErrorString((cudaError_t)e)) : MUCU_OK;
+}
+
+extern "C" mucu_status_t mucu_peer_barrier(const mucu_reduce_target_t* flags, const uint32_t* own, uint32_t target,
+                                           void* stream) {
+    if (!flags || !own || flags->count < 1 || flags->count > MUCU_MAX_REDUCE_RANKS || (flags->multicast && flags->count != 1))
+        return set_error(MUCU_ERR_INVALID_VALUE, "peer_barrier: bad flag target");
+    RedTarget f = {};
+    for (int r = 0; r < flags->count; ++r) {
+        if (!flags->dst[r] || ((uintptr_t)flags->dst[r] & 3)) return set_error(MUCU_ERR_MISALIGNED, "flag %d", r);
+        f.dst[r] = flags->dst[r];
+    }
+    f.n = flags->count;
+    f.mc = flags->multicast ? 1 : 0;
+    const int e = launch_reduce_barrier(f, (const unsigned*)own, target, (cudaStream_t)stream);
+    return e ? set_error(MUCU_ERR_CUDA, "peer barrier launch: %s", cudaGetErrorString((cudaError_t)e)) : MUCU_OK;
 }
 
 extern "C" mucu_status_t mucu_nvls_destroy(mucu_nvls_t nv) {

@@ -60,10 +60,11 @@ __device__ __forceinline__ long long wgrad_dst(const TcArgs& p, int m, int n) {
 // dst[ofs[j] * stride] = alpha * v[j] + beta * dst[...] for the 32 accumulator
 // columns of one row (ofs < 0: skipped); all loads issue before the stores.
 // beta == 0 never reads dst (it may hold garbage / NaN).
-// mc (NEXT-3): the multicast address matching dst (nullptr: off) -- the final value of
-// every element is also added to the cross-rank dW sum there.
+// red (NEXT-3): the cross-rank dW sum (nullptr: off); red_off = element offset of dst in
+// dw -- the final value of every element is also added there.
 __device__ __forceinline__ void rmw32(float* dst, const int (&ofs)[32], size_t stride, const uint32_t* v, float alpha,
-                                      float beta, bool atomic = false, float* mc = nullptr) {
+                                      float beta, bool atomic = false, const RedTarget* red = nullptr,
+                                      long long red_off = 0) {
     if (atomic) {  // non-deterministic split-K (beta applied by a prescale launch): L2 reductions
 #pragma unroll
         for (int j = 0; j < 32; ++j)
@@ -81,7 +82,7 @@ __device__ __forceinline__ void rmw32(float* dst, const int (&ofs)[32], size_t s
         if (ofs[j] >= 0) {
             const float o = alpha * __uint_as_float(v[j]) + beta * old[j];
             dst[(size_t)ofs[j] * stride] = o;
-            if (mc) mc_red(mc + (size_t)ofs[j] * stride, o);
+            if (red) red_add(*red, red_off + (long long)ofs[j] * (long long)stride, o);
         }
 }
 
@@ -1272,10 +1273,10 @@ __global__ void __launch_bounds__(threads_for(AM), 1) tc_conv_gemm(const __grid_
             // cluster path; p.atomic (non-deterministic mode) adds every split's partial
             // with L2 reductions after a beta prescale launch.
             const float bsplit = p.beta;
-            // NEXT-3: multicast address of a dw element (the final value: no split here)
-            auto mc_of = [&](const float* d) -> float* {
-                return p.mc_out ? p.mc_out + (d - (const float*)p.out) : nullptr;
-            };
+            // NEXT-3: the cross-rank sum target (the final values: no split here) and the
+            // element offset of a dw pointer
+            const RedTarget* redp = p.red.n ? &p.red : nullptr;
+            auto roff = [&](const float* d) -> long long { return (long long)(d - (const float*)p.out); };
             auto drain = [&](const int hh) {
             // M = 64 half: TMEM lane 32*q4 + l (l < 16) holds row 16*q4 + l
             const bool h64 = p.m64 && hh == p.mt - 1;
@@ -1473,7 +1474,7 @@ __global__ void __launch_bounds__(threads_for(AM), 1) tc_conv_gemm(const __grid_
                         }
                         if (++ch == p.C) { ch = 0; ++tap; }
                     }
-                    rmw32(drow, dofs, 1, v, p.alpha, bsplit, p.atomic, mc_of(drow));
+                    rmw32(drow, dofs, 1, v, p.alpha, bsplit, p.atomic, redp, roff(drow));
                 } else if constexpr (EPI == EPI_WGRAD_WIN) {
                     // row m = (r, atom aa, tap t, channel c) -> dw[k][r][aa*taps + t][c], k = nb + j
                     constexpr int per_atom = WAW / ELT;
@@ -1485,7 +1486,7 @@ __global__ void __launch_bounds__(threads_for(AM), 1) tc_conv_gemm(const __grid_
                         int dofs[32];
 #pragma unroll
                         for (int j = 0; j < 32; ++j) dofs[j] = nb + j < p.N ? j : -1;
-                        rmw32(d, dofs, (size_t)p.ldc, v, p.alpha, bsplit, p.atomic, mc_of(d));
+                        rmw32(d, dofs, (size_t)p.ldc, v, p.alpha, bsplit, p.atomic, redp, roff(d));
                     }
                 } else if constexpr (EPI == EPI_WGRAD_PARTIAL) {
                     // the split's partial tile: out[z][m][nb + j] (rows < part_rows, plain stores)
@@ -1509,7 +1510,7 @@ __global__ void __launch_bounds__(threads_for(AM), 1) tc_conv_gemm(const __grid_
 #pragma unroll
                         for (int j = 0; j < 32; ++j) dofs[j] = nb + j < p.N ? j : -1;
                         rmw32(outF + (size_t)nb * p.ldc + m, dofs, (size_t)p.ldc, v, p.alpha, bsplit, p.atomic,
-                              mc_of(outF + (size_t)nb * p.ldc + m));
+                              redp, roff(outF + (size_t)nb * p.ldc + m));
                     }
                 } else if constexpr (EPI == EPI_WGRAD_SMALLC) {
                     // padded column j' = (r, s8, c') -> dw column (r*S + s)*C + c (skip padding)
@@ -1521,7 +1522,7 @@ __global__ void __launch_bounds__(threads_for(AM), 1) tc_conv_gemm(const __grid_
                         const int c = jp % p.cp, t2 = jp / p.cp, s_ = t2 % p.s8, r = t2 / p.s8;
                         dofs[j] = (jp < p.N && c < p.C && s_ < p.S) ? (r * p.S + s_) * p.C + c : -1;
                     }
-                    rmw32(drow, dofs, 1, v, p.alpha, bsplit, p.atomic, mc_of(drow));
+                    rmw32(drow, dofs, 1, v, p.alpha, bsplit, p.atomic, redp, roff(drow));
                 } else if constexpr (EPI == EPI_WGRAD_CHAIN) {
                     // dw = alpha * partial + bsplit * dw (bsplit = beta on split 0, else 1),
                     // in split order: 16-byte vector read-modify-write
@@ -1549,13 +1550,13 @@ __global__ void __launch_bounds__(threads_for(AM), 1) tc_conv_gemm(const __grid_
                             q.z = p.alpha * __uint_as_float(v[4 * j + 2]) + bsplit * o[j].z;
                             q.w = p.alpha * __uint_as_float(v[4 * j + 3]) + bsplit * o[j].w;
                             reinterpret_cast<float4*>(d)[j] = q;
-                            if (p.mc_out) mc_red4(mc_of(d) + 4 * j, q);
+                            if (redp) red_add4(p.red, roff(d) + 4 * j, q);
                         }
                     } else {
                         int dofs[32];
 #pragma unroll
                         for (int j = 0; j < 32; ++j) dofs[j] = nb + j < p.N ? j : -1;
-                        rmw32(d, dofs, 1, v, p.alpha, bsplit, p.atomic, mc_of(d));
+                        rmw32(d, dofs, 1, v, p.alpha, bsplit, p.atomic, redp, roff(d));
                     }
                 } else if (p.out_bf16) {
                     __nv_bfloat16* d = (__nv_bfloat16*)outT + (size_t)mrow * p.ldc + nb;
@@ -1642,7 +1643,7 @@ __global__ void __launch_bounds__(threads_for(AM), 1) tc_conv_gemm(const __grid_
                 const float bsplit = g == 0 ? p.beta : 1.f;
                 // NEXT-3: the last split group writes the final dw: it also adds the
                 // cross-rank sum through the multicast address
-                const bool final_mc = p.mc_out != nullptr && g == p.mc_group;
+                const bool final_mc = p.red.n != 0 && g == p.red_group;
                 unsigned long long* turn =
                     p.turns ? p.turns + ((size_t)(batch * per_z + rem) * p.cl + rho) : nullptr;
                 const uint32_t stg = smem_u32(smem);
@@ -1709,20 +1710,20 @@ __global__ void __launch_bounds__(threads_for(AM), 1) tc_conv_gemm(const __grid_
                                 float* d = outF + (size_t)(m0 + rr) * p.ldc + col0;
                                 const float4 o = make_float4(sum[uu].x + bsplit * old[uu].x, sum[uu].y + bsplit * old[uu].y,
                                                              sum[uu].z + bsplit * old[uu].z, sum[uu].w + bsplit * old[uu].w);
-                                float* mcd = final_mc ? p.mc_out + (d - (const float*)p.out) : nullptr;
+                                const long long ro = (long long)(d - (const float*)p.out);
                                 if (vec) {
                                     *reinterpret_cast<float4*>(d) = o;
-                                    if (mcd) mc_red4(mcd, o);
+                                    if (final_mc) red_add4(p.red, ro, o);
                                 } else {
                                     if (col0 < p.N) d[0] = o.x;
                                     if (col0 + 1 < p.N) d[1] = o.y;
                                     if (col0 + 2 < p.N) d[2] = o.z;
                                     if (col0 + 3 < p.N) d[3] = o.w;
-                                    if (mcd) {
-                                        if (col0 < p.N) mc_red(mcd, o.x);
-                                        if (col0 + 1 < p.N) mc_red(mcd + 1, o.y);
-                                        if (col0 + 2 < p.N) mc_red(mcd + 2, o.z);
-                                        if (col0 + 3 < p.N) mc_red(mcd + 3, o.w);
+                                    if (final_mc) {
+                                        if (col0 < p.N) red_add(p.red, ro, o.x);
+                                        if (col0 + 1 < p.N) red_add(p.red, ro + 1, o.y);
+                                        if (col0 + 2 < p.N) red_add(p.red, ro + 2, o.z);
+                                        if (col0 + 3 < p.N) red_add(p.red, ro + 3, o.w);
                                     }
                                 }
                             }
@@ -1745,7 +1746,7 @@ __global__ void __launch_bounds__(threads_for(AM), 1) tc_conv_gemm(const __grid_
                                     if (o[j] >= 0) {
                                         const float fv = sv[j] + bsplit * ov[j];
                                         outF[o[j]] = fv;
-                                        if (final_mc) mc_red(p.mc_out + (outF + o[j] - (const float*)p.out), fv);
+                                        if (final_mc) red_add(p.red, (long long)(outF + o[j] - (const float*)p.out), fv);
                                     }
                             }
                         }

@@ -105,46 +105,86 @@ def share_fd(fd: Optional[int], group=None) -> int:
         os.close(pidfd)
 
 
-class NvlsGradReduce:
-    """Cross-rank dW sum through NVLink multicast, fused into BackwardFilter.
+class FusedGradReduce:
+    """Cross-rank dW sum fused into BackwardFilter (NEXT-3).
 
-    `sums` is this rank's copy of the multicast buffer as an fp32 tensor with the
-    layout of ConvNet.dw_flat; after an iteration run with ``nvls=self`` every
-    rank's `sums` holds the sum over ranks of dw_flat.  Collective constructor."""
+    kind "nvls": one NVLink multicast buffer (mucu_nvls_*), the kernels issue one
+    multimem.red per value and NVSwitch adds it into every rank's copy.
+    kind "p2p": one buffer per rank (torch symmetric memory for the peer mappings),
+    the kernels issue one red.global.add per rank over NVLink P2P.
+    `sums` is this rank's buffer with the layout of ConvNet.dw_flat; after an
+    iteration run with ``net.nvls = self`` every rank's `sums` holds the sum over
+    ranks of dw_flat.  Collective constructor."""
 
-    def __init__(self, numel: int, device: int, group=None):
+    def __init__(self, numel: int, device: int, kind: str = "nvls", group=None):
         from . import _lib as L
+        self.L = L
+        self.kind = kind
         self.group = group
-        world = dist.get_world_size(group) if dist.is_initialized() else 1
+        self.world = dist.get_world_size(group) if dist.is_initialized() else 1
         rank = dist.get_rank(group) if dist.is_initialized() else 0
-        nbytes = max(int(numel), 1) * 4
-        if rank == 0:
-            self.nv = L.Nvls(device, world, nbytes)
-            fd = self.nv.export() if world > 1 else None
-        else:
-            fd = None
-        if world > 1:
-            fd = share_fd(fd, group)
-            if rank != 0:
-                self.nv = L.Nvls(device, world, nbytes, fd=fd)
-                os.close(fd)
-        local, mc = self.nv.bind()
-        self.mc_base = mc
         self.numel = int(numel)
-        self.sums = _tensor_at(local, self.numel, device)
+        flag_at = (self.numel + 63) // 64 * 64  # 256-B aligned flag word after the sums
+        self.epoch = 0
+        if kind == "nvls":
+            nbytes = flag_at * 4
+            if rank == 0:
+                self.nv = L.Nvls(device, self.world, nbytes)
+                fd = self.nv.export() if self.world > 1 else None
+            else:
+                fd = None
+            if self.world > 1:
+                fd = share_fd(fd, group)
+                if rank != 0:
+                    self.nv = L.Nvls(device, self.world, nbytes, fd=fd)
+                    os.close(fd)
+            local, mc = self.nv.bind()
+            self.sums = _tensor_at(local, self.numel, device)
+            self.bases = [mc]
+        elif kind == "p2p":
+            self.nv = None
+            if self.world == 1:
+                self._buf = torch.zeros(flag_at + 64, dtype=torch.float32, device=torch.device("cuda", device))
+                self.bases = [self._buf.data_ptr()]
+            else:
+                import torch.distributed._symmetric_memory as symm_mem
+                self._buf = symm_mem.empty(flag_at + 64, dtype=torch.float32, device=torch.device("cuda", device))
+                self._buf.zero_()
+                hdl = symm_mem.rendezvous(self._buf, (group or dist.group.WORLD).group_name)
+                self.bases = list(hdl.buffer_ptrs)
+            self.sums = self._buf[:self.numel]
+            self._flags = L.reduce_target([b + 4 * flag_at for b in self.bases])
+            self._own = self._buf.data_ptr() + 4 * flag_at
+        else:
+            raise ValueError(f"unknown fused reduction kind {kind!r}")
 
-    def mc_ptr(self, local_view: torch.Tensor, flat: torch.Tensor) -> int:
-        """Multicast address of the element of `sums` matching `local_view` of `flat`."""
-        return self.mc_base + (local_view.data_ptr() - flat.data_ptr())
+    def target(self, offset_bytes: int):
+        """Reduction target of the dw view at byte offset `offset_bytes` of dw_flat."""
+        return self.L.reduce_target([b + offset_bytes for b in self.bases], multicast=self.kind == "nvls")
+
+    def _barrier(self):
+        stream = torch.cuda.current_stream().cuda_stream
+        if self.kind == "nvls":
+            self.nv.barrier(stream)
+        else:
+            self.epoch += 1
+            self.L.peer_barrier(self._flags, self._own, self.epoch * self.world, stream)
 
     def begin(self):
-        """Stream-ordered: zero this rank's copy, then wait for every rank's."""
+        """Stream-ordered: zero this rank's buffer, then wait for every rank's."""
         self.sums.zero_()
-        self.nv.barrier(torch.cuda.current_stream().cuda_stream)
+        self._barrier()
 
     def end(self):
         """Stream-ordered: every rank's reductions are complete and visible."""
-        self.nv.barrier(torch.cuda.current_stream().cuda_stream)
+        self._barrier()
+
+    def close(self):
+        if self.nv is not None:
+            self.nv.close()
+
+
+NvlsGradReduce = FusedGradReduce
 
 
 class _CudaMem:

@@ -119,7 +119,7 @@ class ConvNet:
         self.tensors: List[Dict[str, torch.Tensor]] = []
         self.workspaces: Dict[Tuple[int, int], Optional[torch.Tensor]] = {}
         self.net_ws: Optional[torch.Tensor] = None
-        self.nvls = None  # distributed.NvlsGradReduce over dw_flat (NEXT-3), set by the caller
+        self.nvls = None  # distributed.FusedGradReduce over dw_flat (NEXT-3), set by the caller
 
     # ----------------------------------------------------------- memory --
     def allocate(self, seed: int = 0, kind: str = "normal", generator=None):
@@ -282,8 +282,9 @@ class ConvNet:
         elif conv_type == L.BWD_DATA:
             T.conv_backward_data(self.h, k.desc, k.plan, t["dy"], t["w"], t["dx"], workspace=ws)
         elif self.nvls is not None:  # NEXT-3: the cross-rank sum fused into the epilogue
-            T.conv_backward_filter_nvls(self.h, k.desc, k.plan, t["x"], t["dy"], t["dw"],
-                                        self.nvls.mc_ptr(t["dw"], self.dw_flat), beta=1.0, workspace=ws)
+            T.conv_backward_filter_reduce(self.h, k.desc, k.plan, t["x"], t["dy"], t["dw"],
+                                          self.nvls.target(t["dw"].data_ptr() - self.dw_flat.data_ptr()),
+                                          beta=1.0, workspace=ws)
         else:  # dw was zeroed at the start of the backward pass (zero_grad): accumulate
             T.conv_backward_filter(self.h, k.desc, k.plan, t["x"], t["dy"], t["dw"], beta=1.0, workspace=ws)
 

@@ -90,18 +90,19 @@ def conv_backward_filter(h: L.Handle, d: L.ConvDesc, plan, x, dy, dw=None, alpha
     return dw
 
 
-def conv_backward_filter_nvls(h: L.Handle, d: L.ConvDesc, plan, x, dy, dw, dw_mc: int, alpha=1.0, beta=0.0,
-                              workspace=None):
+def conv_backward_filter_reduce(h: L.Handle, d: L.ConvDesc, plan, x, dy, dw, target: "L.ReduceTarget", alpha=1.0,
+                                beta=0.0, workspace=None):
     """conv_backward_filter + the fused cross-rank sum (NEXT-3): the final dw values
-    are also added to every rank's copy of the NVLS buffer at multicast address dw_mc."""
+    are also added to `target` (a multicast address or one buffer per rank, each
+    element-aligned with dw)."""
     xs, ws_, ys = shapes(d)
     dt = _dtype(d.math)
     _check_tensor(x, xs, dt, "x")
     _check_tensor(dy, ys, dt, "dy")
     _check_tensor(dw, ws_, torch.float32, "dw")
     wp, wb = _ws(workspace)
-    h.conv_backward_filter_nvls(d, plan, alpha, x.data_ptr(), dy.data_ptr(), beta, dw.data_ptr(), int(dw_mc), wp, wb,
-                                _stream())
+    h.conv_backward_filter_reduce(d, plan, alpha, x.data_ptr(), dy.data_ptr(), beta, dw.data_ptr(), target, wp, wb,
+                                  _stream())
     return dw
 
 

@@ -1,8 +1,9 @@
 """NEXT-3 on one GPU: BackwardFilter with the cross-rank dW sum fused into its
-epilogue through NVLink multicast (include/mucudnn.h mucu_conv_backward_filter_nvls,
-DESIGN.md 9c).
+epilogue (include/mucudnn.h mucu_conv_backward_filter_reduce), for
+both targets: one NVLink multicast address (multimem.red; skipped where the box
+cannot create a multicast object) and per-rank buffers (red.global.add, P2P).
 
-With one rank the multicast sum is 0 + dw, so the buffer must equal the rank's own
+With one rank the sum is 0 + dw, so the buffer must equal the rank's own
 dW bit for bit, for every BackwardFilter kernel family: the tensor-core epilogues
 (no split, cluster split-K with ordered groups, staged small-C, window, space-to-depth,
 partial slots + reduction kernel) take the reduction in the kernel that writes the
@@ -16,7 +17,7 @@ import torch
 import paper_conf_cluster_oyamabhm18_b200 as mu
 from paper_conf_cluster_oyamabhm18_b200 import _lib
 from paper_conf_cluster_oyamabhm18_b200 import torch_api as T
-from paper_conf_cluster_oyamabhm18_b200.distributed import NvlsGradReduce
+from paper_conf_cluster_oyamabhm18_b200.distributed import FusedGradReduce
 from paper_conf_cluster_oyamabhm18_b200.network import ConvNet
 from synthetic import network
 
@@ -37,14 +38,20 @@ SHAPES = {
 }
 
 
-@pytest.fixture(scope="module")
-def nvls():
-    if not _lib.nvls_supported(0):
-        pytest.skip("no NVLink multicast on this device")
+@pytest.fixture(scope="module", params=["p2p", "nvls"])
+def nvls(request):
     torch.cuda.set_device(0)
-    red = NvlsGradReduce(8 << 20, 0)  # 32 MiB of fp32 sums, world size 1
+    if request.param == "nvls":
+        if not _lib.nvls_supported(0):
+            pytest.skip("no NVLink multicast on this device")
+        try:
+            red = FusedGradReduce(8 << 20, 0, kind="nvls")  # 32 MiB of fp32 sums, world size 1
+        except mu.MucuError as e:  # e.g. no NVSwitch fabric behind a one-GPU lease
+            pytest.skip(f"NVLink multicast object unavailable: {e}")
+    else:
+        red = FusedGradReduce(8 << 20, 0, kind="p2p")
     yield red
-    red.nv.close()
+    red.close()
 
 
 def _dev(shape, dtype, seed):
@@ -73,7 +80,7 @@ def _check(nv, d, plan, x, dy, beta, det, expect_fused):
         dw = out0.clone()
         nv.begin()
         n0 = _lib.launch_count()
-        T.conv_backward_filter_nvls(h, d, plan, x, dy, dw, nv.mc_base, beta=beta, workspace=ws)
+        T.conv_backward_filter_reduce(h, d, plan, x, dy, dw, nv.target(0), beta=beta, workspace=ws)
         fused = _lib.launch_count() - n0
         nv.end()
         torch.cuda.synchronize()

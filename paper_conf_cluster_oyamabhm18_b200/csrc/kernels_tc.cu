@@ -1,31 +1,37 @@
 // kernels_tc.cu -- tcgen05 tensor-core conv-GEMM for sm_100a (MUCU_MATH_TF32 /
-// MUCU_MATH_BF16): the contraction step of all three algorithms.
+// MUCU_MATH_BF16): the contraction step of all three algorithms, and the host-side
+// dispatch (tiling, tensor maps, split-K, launch) of one micro-configuration.
 //
 //   (a) implicit GEMM (zero workspace): the im2col / transposed-conv operand is
-//       gathered on the fly from NHWC activations with cp.async into the
-//       128-byte-swizzled shared-memory layout the UMMA descriptors expect;
-//   (b) im2col + GEMM: both operands dense, loaded with TMA;
-//   (c) Winograd: 16 independent GEMMs M_xi = V_xi U_xi^T (batched over
-//       blockIdx.z), TMA-loaded.
+//       loaded by TMA in im2col mode (or gathered with cp.async / built in shared
+//       memory from TMA-staged rows for small-C strided layers);
+//   (b) im2col + GEMM: dense operands loaded with TMA (space-to-depth for strided
+//       RGB layers, 6.3);
+//   (c) Winograd: 16 independent GEMMs M_xi = V_xi U_xi^T (batched over the tile
+//       index), TMA-loaded.
 //
-// One CTA computes a 128 x BN output tile; the fp32 accumulator lives in TMEM
-// (BN columns).  Warp roles (256 threads):
-//   warps 0-3  producers: one thread issues TMA, all 128 threads gather (cp.async)
-//   warp  4    TMEM allocator + single-thread tcgen05.mma issuer
-//   warps 4-7  epilogue: tcgen05.ld 32x32b -> registers -> alpha/beta -> global
-// Shared memory is a STAGES-deep ring of {A tile, B tile} guarded by
-// full/empty mbarriers; tcgen05.commit releases a stage when its MMAs retire.
+// The kernel (tc_gemm_kernel.cuh) is persistent: CTAs walk 128*mt x BN output tiles
+// with fp32 accumulators in TMEM.  Warp roles (288 threads; 320 with a TMA warp):
+//   warps 0-3  producers (one thread issues TMA; all gather where TMA cannot),
+//   warp  4    TMEM allocator + single-thread tcgen05.mma issuer,
+//   warps 5-8  epilogue: tcgen05.ld -> registers -> alpha / beta -> global.
+// Shared memory is a ring of {A, B} stages guarded by full / empty mbarriers;
+// tcgen05.commit releases a stage when its MMAs retire.
 //
 // Operand layouts (K = reduction):
 //   K-major:  rows x 128 B (64 bf16 / 32 fp32 of K), SWIZZLE_128B atoms of 8 rows
 //   MN-major: (MN/64 bf16 | MN/32 fp32) atoms, each KB rows x 128 B, SWIZZLE_128B
-// KB = 128 B / element size of K per stage; 4 MMAs (UMMA_K = 32 B) per stage.
+//             (tf32: 128B_BASE32B)
 //
-// Backward-filter splits the pixel reduction over the tile index z
-// and combines the partial tiles in split order through per-tile turn counters
-// (turns.cu): split s waits for split s-1, then reads dw, adds its partial and
-// writes it back (split 0 applies the user's beta), so dw is bitwise
-// reproducible run to run.
+// Backward-filter splits the pixel reduction.  Deterministic mode
+// (default): thread-block clusters of cl CTAs (one split each) sum their partial
+// tiles over DSMEM in rank order, and split groups add into dw in group order
+// behind per-(tile, slab) turn counters (turns.cu), group 0 applying beta; with
+// workspace, I2C writes per-split partial slots and a reduction kernel sums them in
+// split order -- dw is bitwise reproducible run to run.
+// Non-deterministic mode (mucu_set_deterministic(h, 0)): splits add their partials
+// with red.global.add after a beta pre-scale.  NEXT-3: the final dw writer also adds
+// its values to a cross-rank reduction target (nvls.cu).
 #include <cuda.h>
 #include <cuda_bf16.h>
 #include <cuda_runtime.h>

@@ -38,27 +38,34 @@ template <> __device__ __forceinline__ __nv_bfloat16 from_float<__nv_bfloat16>(f
 struct Dense {
     const float* p;
     int64_t rows, kdim, si, sk, batch_stride;
-    __device__ __forceinline__ float at(int64_t i, int64_t kk) const {
-        return (i < rows && kk < kdim) ? __ldg(p + i * si + kk * sk) : 0.f;
-    }
     // row-contiguous loads: a thread keeps one row for the whole main loop
     struct Row { const float* q; bool ok; };
     __device__ __forceinline__ Row row(int64_t i) const { return Row{p + i * si, i < rows}; }
-    __device__ __forceinline__ float get(const Row& r, int64_t kk) const {
-        return (r.ok && kk < kdim) ? __ldg(r.q + kk * sk) : 0.f;
-    }
-    // four consecutive kk (kk % 4 == 0): one 16-byte load when contiguous and aligned
-    __device__ __forceinline__ void at4(int64_t i, int64_t kk, int64_t kend, float (&o)[4]) const {
-        const float* q = p + i * si + kk * sk;
-        if (sk == 1 && i < rows && kk + 3 < kdim && kk + 3 < kend && (((uintptr_t)q) & 15) == 0) {
+    __device__ __forceinline__ void batch(int z) { p += z * batch_stride; }
+    // k-contiguous loader contexts: a row pointer per thread row, nothing per kk
+    struct KRow { const float* q; bool ok; };
+    struct KCol { };
+    __device__ __forceinline__ KRow krow(int64_t i) const { return KRow{p + i * si, i < rows}; }
+    __device__ __forceinline__ KCol kcol(int64_t) const { return KCol{}; }
+    __device__ __forceinline__ void at4c(const KRow& r, const KCol&, int64_t kk, int64_t kend, float (&o)[4]) const {
+        const float* q = r.q + kk * sk;
+        if (sk == 1 && r.ok && kk + 3 < kdim && kk + 3 < kend && (((uintptr_t)q) & 15) == 0) {
             const float4 v = __ldg(reinterpret_cast<const float4*>(q));
             o[0] = v.x; o[1] = v.y; o[2] = v.z; o[3] = v.w;
             return;
         }
 #pragma unroll
-        for (int e = 0; e < 4; ++e) o[e] = kk + e < kend ? at(i, kk + e) : 0.f;
+        for (int e = 0; e < 4; ++e) o[e] = (r.ok && kk + e < kend && kk + e < kdim) ? __ldg(q + e * sk) : 0.f;
     }
-    __device__ __forceinline__ void batch(int z) { p += z * batch_stride; }
+    // row-contiguous loader: CNT values of the thread's row at kk0, kk0 + step, ...
+    template <int CNT>
+    __device__ __forceinline__ void run(const Row& r, int64_t kk0, int step, int64_t kend, float (&o)[CNT]) const {
+#pragma unroll
+        for (int e = 0; e < CNT; ++e) {
+            const int64_t kk = kk0 + (int64_t)e * step;
+            o[e] = (r.ok && kk < kend && kk < kdim) ? __ldg(r.q + kk * sk) : 0.f;
+        }
+    }
 };
 
 // Implicit im2col of x (NHWC) for FWD: row i = output pixel (n,p,q), kk = (r,s,c).
@@ -80,36 +87,43 @@ struct Im2col {
         if ((unsigned)h >= (unsigned)H || (unsigned)w >= (unsigned)W) return 0.f;
         return __ldg(x + (((int64_t)n * H + h) * W + w) * C + c);
     }
-    // kk .. kk+3 of one pixel row: one decomposition, one 16-byte load when the four
-    // channels belong to one tap and are aligned (C % 4 == 0)
-    __device__ __forceinline__ void at4(int64_t m64, int64_t kk64, int64_t kend, float (&o)[4]) const {
-        if (m64 < rows && kk64 + 3 < RSC && kk64 + 3 < kend) {
-            const uint32_t m = (uint32_t)m64, kk = (uint32_t)kk64;
-            const uint32_t rs = dC.div(kk), c = kk - rs * (uint32_t)C;
-            if (c + 3 < (uint32_t)C) {
-                const uint32_t n = dPQ.div(m), rem = m - n * (uint32_t)(P * Q);
-                const uint32_t pp = dQ.div(rem), q = rem - pp * (uint32_t)Q;
-                const uint32_t r = dS.div(rs), s = rs - r * (uint32_t)S;
-                const int h = (int)(pp * st + r) - pad, w = (int)(q * st + s) - pad;
-                if ((unsigned)h >= (unsigned)H || (unsigned)w >= (unsigned)W) {
-                    o[0] = o[1] = o[2] = o[3] = 0.f;
-                    return;
-                }
-                const float* src = x + (((int64_t)n * H + h) * W + w) * C + c;
-                if ((((uintptr_t)src) & 15) == 0) {
-                    const float4 v = __ldg(reinterpret_cast<const float4*>(src));
-                    o[0] = v.x; o[1] = v.y; o[2] = v.z; o[3] = v.w;
-                } else {
+    __device__ __forceinline__ void batch(int) {}
+    // k-contiguous loader contexts: the pixel of a thread row is decomposed once per
+    // CTA, the tap (r, s, c) of the thread's kk once per K slab (shared by its rows)
+    struct KRow { const float* xn; int h0, w0, m; };
+    struct KCol { int r, s, c; };
+    __device__ __forceinline__ KRow krow(int64_t m64) const {
+        if (m64 >= rows) return KRow{x, 0, 0, -1};
+        const uint32_t m = (uint32_t)m64;
+        const uint32_t n = dPQ.div(m), rem = m - n * (uint32_t)(P * Q);
+        const uint32_t p = dQ.div(rem), q = rem - p * (uint32_t)Q;
+        return KRow{x + (int64_t)n * H * W * C, (int)(p * st) - pad, (int)(q * st) - pad, (int)m};
+    }
+    __device__ __forceinline__ KCol kcol(int64_t kk64) const {
+        if (kk64 >= RSC) return KCol{0, 0, C};
+        const uint32_t kk = (uint32_t)kk64, rs = dC.div(kk), c = kk - rs * (uint32_t)C;
+        const uint32_t r = dS.div(rs), s = rs - r * (uint32_t)S;
+        return KCol{(int)r, (int)s, (int)c};
+    }
+    __device__ __forceinline__ void at4c(const KRow& kr, const KCol& kc, int64_t kk, int64_t kend,
+                                         float (&o)[4]) const {
+        if (kr.m < 0) { o[0] = o[1] = o[2] = o[3] = 0.f; return; }
+        if (kk + 3 < RSC && kk + 3 < kend && kc.c + 3 < C) {
+            const int h = kr.h0 + kc.r, w = kr.w0 + kc.s;
+            if ((unsigned)h >= (unsigned)H || (unsigned)w >= (unsigned)W) { o[0] = o[1] = o[2] = o[3] = 0.f; return; }
+            const float* src = kr.xn + ((int64_t)h * W + w) * C + kc.c;
+            if ((((uintptr_t)src) & 15) == 0) {
+                const float4 v = __ldg(reinterpret_cast<const float4*>(src));
+                o[0] = v.x; o[1] = v.y; o[2] = v.z; o[3] = v.w;
+            } else {
 #pragma unroll
-                    for (int e = 0; e < 4; ++e) o[e] = __ldg(src + e);
-                }
-                return;
+                for (int e = 0; e < 4; ++e) o[e] = __ldg(src + e);
             }
+            return;
         }
 #pragma unroll
-        for (int e = 0; e < 4; ++e) o[e] = kk64 + e < kend ? at(m64, kk64 + e) : 0.f;
+        for (int e = 0; e < 4; ++e) o[e] = kk + e < kend ? at(kr.m, kk + e) : 0.f;
     }
-    __device__ __forceinline__ void batch(int) {}
 };
 Im2col make_im2col(const float* x, int64_t rows, const Geom& g) {
     return Im2col{x, rows, g.h, g.w, g.c, g.p, g.q, g.s, g.pad, g.stride, g.r * g.s * g.c,
@@ -119,7 +133,6 @@ Im2col make_im2col(const float* x, int64_t rows, const Geom& g) {
 // Im2col transposed for WGRAD's B operand: B(j, kk) = im2col(kk = pixel, j = (r,s,c)).
 struct Im2colT {
     Im2col v;
-    __device__ __forceinline__ float at(int64_t j, int64_t m) const { return v.at(m, j); }
     // the (r,s,c) of a thread's row is decomposed once; each pixel then costs two divisions
     struct Row { const float* xc; int r, s; bool ok; };
     __device__ __forceinline__ Row row(int64_t j64) const {
@@ -128,14 +141,34 @@ struct Im2colT {
         const uint32_t r = v.dS.div(rs), s = rs - r * (uint32_t)v.S;
         return Row{v.x + c, (int)r - v.pad, (int)s - v.pad, true};
     }
-    __device__ __forceinline__ float get(const Row& rw, int64_t m64) const {
-        if (!rw.ok || m64 >= v.rows) return 0.f;
-        const uint32_t m = (uint32_t)m64;
-        const uint32_t n = v.dPQ.div(m), rem = m - n * (uint32_t)(v.P * v.Q);
-        const uint32_t p = v.dQ.div(rem), q = rem - p * (uint32_t)v.Q;
-        const int h = (int)(p * v.st) + rw.r, w = (int)(q * v.st) + rw.s;
-        if ((unsigned)h >= (unsigned)v.H || (unsigned)w >= (unsigned)v.W) return 0.f;
-        return __ldg(rw.xc + (((int64_t)n * v.H + h) * v.W + w) * v.C);
+    // CNT pixels m0, m0 + step, ...: one decomposition, then an incremental walk
+    template <int CNT>
+    __device__ __forceinline__ void run(const Row& rw, int64_t m0, int step, int64_t kend, float (&o)[CNT]) const {
+        const int64_t lim = min(kend, v.rows);
+        if (!rw.ok || m0 >= lim) {
+#pragma unroll
+            for (int e = 0; e < CNT; ++e) o[e] = 0.f;
+            return;
+        }
+        const uint32_t m = (uint32_t)m0;
+        uint32_t n = v.dPQ.div(m);
+        const uint32_t rem = m - n * (uint32_t)(v.P * v.Q);
+        uint32_t p = v.dQ.div(rem), q = rem - p * (uint32_t)v.Q;
+        const float* xn = rw.xc + (int64_t)n * v.H * v.W * v.C;
+        const int left = (int)(lim - m0);  // valid pixels from m0 on
+#pragma unroll
+        for (int e = 0; e < CNT; ++e) {
+            float val = 0.f;
+            const int h = (int)(p * v.st) + rw.r, w = (int)(q * v.st) + rw.s;
+            if (e * step < left && (unsigned)h < (unsigned)v.H && (unsigned)w < (unsigned)v.W)
+                val = __ldg(xn + (h * v.W + w) * v.C);
+            o[e] = val;
+            q += step;
+            while (q >= (uint32_t)v.Q) {
+                q -= v.Q;
+                if (++p == (uint32_t)v.P) { p = 0; xn += v.H * v.W * v.C; }
+            }
+        }
     }
 };
 
@@ -159,35 +192,49 @@ struct DgradGather {
         if (p * st != (uint32_t)ph || q * st != (uint32_t)pw || p >= (uint32_t)P || q >= (uint32_t)Q) return 0.f;
         return __ldg(dy + (((int64_t)n * P + p) * Q + q) * K + k);
     }
-    // kk .. kk+3: four consecutive k of one tap (K % 4 == 0): one decomposition, one load
-    __device__ __forceinline__ void at4(int64_t m64, int64_t kk64, int64_t kend, float (&o)[4]) const {
-        if (m64 < rows && kk64 + 3 < RSK && kk64 + 3 < kend) {
-            const uint32_t kk = (uint32_t)kk64, rs = dK.div(kk), k = kk - rs * (uint32_t)K;
-            if (k + 3 < (uint32_t)K) {
-                const uint32_t m = (uint32_t)m64;
-                const uint32_t n = dHW.div(m), rem = m - n * (uint32_t)(H * W);
-                const uint32_t h = dW.div(rem), w = rem - h * (uint32_t)W;
-                const uint32_t r = dS.div(rs), s = rs - r * (uint32_t)S;
-                const int ph = (int)(h + pad) - (int)r, pw = (int)(w + pad) - (int)s;
-                o[0] = o[1] = o[2] = o[3] = 0.f;
-                if (ph < 0 || pw < 0) return;
-                const uint32_t p = dSt.div((uint32_t)ph), q = dSt.div((uint32_t)pw);
-                if (p * st != (uint32_t)ph || q * st != (uint32_t)pw || p >= (uint32_t)P || q >= (uint32_t)Q) return;
-                const float* src = dy + (((int64_t)n * P + p) * Q + q) * K + k;
-                if ((((uintptr_t)src) & 15) == 0) {
-                    const float4 v = __ldg(reinterpret_cast<const float4*>(src));
-                    o[0] = v.x; o[1] = v.y; o[2] = v.z; o[3] = v.w;
-                } else {
-#pragma unroll
-                    for (int e = 0; e < 4; ++e) o[e] = __ldg(src + e);
-                }
-                return;
+    __device__ __forceinline__ void batch(int) {}
+    // k-contiguous loader contexts (see Im2col)
+    struct KRow { const float* dyn; int hp, wp, m; };
+    struct KCol { int r, s, k; };
+    __device__ __forceinline__ KRow krow(int64_t m64) const {
+        if (m64 >= rows) return KRow{dy, 0, 0, -1};
+        const uint32_t m = (uint32_t)m64;
+        const uint32_t n = dHW.div(m), rem = m - n * (uint32_t)(H * W);
+        const uint32_t h = dW.div(rem), w = rem - h * (uint32_t)W;
+        return KRow{dy + (int64_t)n * P * Q * K, (int)h + pad, (int)w + pad, (int)m};
+    }
+    __device__ __forceinline__ KCol kcol(int64_t kk64) const {
+        if (kk64 >= RSK) return KCol{0, 0, K};
+        const uint32_t kk = (uint32_t)kk64, rs = dK.div(kk), k = kk - rs * (uint32_t)K;
+        const uint32_t r = dS.div(rs), s = rs - r * (uint32_t)S;
+        return KCol{(int)r, (int)s, (int)k};
+    }
+    __device__ __forceinline__ void at4c(const KRow& kr, const KCol& kc, int64_t kk, int64_t kend,
+                                         float (&o)[4]) const {
+        if (kr.m < 0) { o[0] = o[1] = o[2] = o[3] = 0.f; return; }
+        if (kk + 3 < RSK && kk + 3 < kend && kc.k + 3 < K) {
+            o[0] = o[1] = o[2] = o[3] = 0.f;
+            const int ph = kr.hp - kc.r, pw = kr.wp - kc.s;
+            if (ph < 0 || pw < 0) return;
+            uint32_t p = (uint32_t)ph, q = (uint32_t)pw;
+            if (st != 1) {
+                p = dSt.div((uint32_t)ph); q = dSt.div((uint32_t)pw);
+                if (p * st != (uint32_t)ph || q * st != (uint32_t)pw) return;
             }
+            if (p >= (uint32_t)P || q >= (uint32_t)Q) return;
+            const float* src = kr.dyn + ((int64_t)p * Q + q) * K + kc.k;
+            if ((((uintptr_t)src) & 15) == 0) {
+                const float4 v = __ldg(reinterpret_cast<const float4*>(src));
+                o[0] = v.x; o[1] = v.y; o[2] = v.z; o[3] = v.w;
+            } else {
+#pragma unroll
+                for (int e = 0; e < 4; ++e) o[e] = __ldg(src + e);
+            }
+            return;
         }
 #pragma unroll
-        for (int e = 0; e < 4; ++e) o[e] = kk64 + e < kend ? at(m64, kk64 + e) : 0.f;
+        for (int e = 0; e < 4; ++e) o[e] = kk + e < kend ? at(kr.m, kk + e) : 0.f;
     }
-    __device__ __forceinline__ void batch(int) {}
 };
 
 // DGRAD filter view: B(j = c, kk = (r,s,k)) = w[k][r][s][c].
@@ -195,17 +242,20 @@ struct DgradFilter {
     const float* w;
     int C, K, RS;
     FastDiv dK;
-    __device__ __forceinline__ float at(int64_t j, int64_t kk64) const {
-        if (j >= C || kk64 >= (int64_t)RS * K) return 0.f;
-        const uint32_t kk = (uint32_t)kk64, rs = dK.div(kk), k = kk - rs * (uint32_t)K;
-        return __ldg(w + ((int64_t)k * RS + rs) * C + j);
-    }
     struct Row { const float* q; bool ok; };
     __device__ __forceinline__ Row row(int64_t j) const { return Row{w + j, j < C}; }
-    __device__ __forceinline__ float get(const Row& r, int64_t kk64) const {
-        if (!r.ok || kk64 >= (int64_t)RS * K) return 0.f;
-        const uint32_t kk = (uint32_t)kk64, rs = dK.div(kk), k = kk - rs * (uint32_t)K;
-        return __ldg(r.q + ((int64_t)k * RS + rs) * C);
+    // CNT taps kk0, kk0 + step, ...: one decomposition, then an incremental walk
+    template <int CNT>
+    __device__ __forceinline__ void run(const Row& r, int64_t kk0, int step, int64_t kend, float (&o)[CNT]) const {
+        const int64_t lim = min(kend, (int64_t)RS * K);
+        uint32_t rs = 0, k = 0;
+        if (kk0 < lim) { rs = dK.div((uint32_t)kk0); k = (uint32_t)kk0 - rs * (uint32_t)K; }
+#pragma unroll
+        for (int e = 0; e < CNT; ++e) {
+            o[e] = (r.ok && kk0 + (int64_t)e * step < lim) ? __ldg(r.q + ((int64_t)k * RS + rs) * C) : 0.f;
+            k += step;
+            while (k >= (uint32_t)K) { k -= K; ++rs; }
+        }
     }
     __device__ __forceinline__ void batch(int) {}
 };
@@ -241,6 +291,8 @@ constexpr int kBK = 16;
 // row context of a row-contiguous operand (views without one are only loaded k-contiguous)
 template <class V, bool CONTIG> struct RowOf { using type = typename V::Row; };
 template <class V> struct RowOf<V, true> { using type = int; };
+template <class V, bool CONTIG> struct KRowOf { using type = int; };
+template <class V> struct KRowOf<V, true> { using type = typename V::KRow; };
 
 template <int BM, int BN, bool CONTIG_KA, bool CONTIG_KB, class AV, class BV>
 struct TileLoader {
@@ -250,10 +302,22 @@ struct TileLoader {
     float ra[NA], rb[NB];
     typename RowOf<AV, CONTIG_KA>::type arow;  // row-contiguous: the thread's row is fixed (t % BM)
     typename RowOf<BV, CONTIG_KB>::type brow;
+    // k-contiguous: the thread's NA / 4 (NB / 4) rows are fixed too -- their contexts
+    // (pixel decompositions) are computed once per CTA
+    typename KRowOf<AV, CONTIG_KA>::type akr[CONTIG_KA ? NA / 4 : 1];
+    typename KRowOf<BV, CONTIG_KB>::type bkr[CONTIG_KB ? NB / 4 : 1];
 
     __device__ __forceinline__ void init(const AV& a, const BV& b, int64_t m0, int64_t n0) {
         if constexpr (!CONTIG_KA) arow = a.row(m0 + threadIdx.x % BM);
         if constexpr (!CONTIG_KB) brow = b.row(n0 + threadIdx.x % BN);
+        if constexpr (CONTIG_KA) {
+#pragma unroll
+            for (int g = 0; g < NA / 4; ++g) { int il, kl; a_coord(4 * g, il, kl); akr[g] = a.krow(m0 + il); }
+        }
+        if constexpr (CONTIG_KB) {
+#pragma unroll
+            for (int g = 0; g < NB / 4; ++g) { int jl, kl; b_coord(4 * g, jl, kl); bkr[g] = b.krow(n0 + jl); }
+        }
     }
 
     // k-contiguous operands: a thread loads 4 consecutive k of a row (element e = 4g + u:
@@ -268,40 +332,33 @@ struct TileLoader {
         if (CONTIG_KB) { kl = 4 * (t % (BK / 4)) + (e & 3); jl = t / (BK / 4) + (e >> 2) * (kThreads * 4 / BK); }
         else           { jl = t % BN; kl = t / BN + e * (kThreads / BN); }
     }
-    __device__ __forceinline__ void load(const AV& a, const BV& b, int64_t m0, int64_t n0, int64_t k0, int64_t kend) {
+    __device__ __forceinline__ void load(const AV& a, const BV& b, int64_t, int64_t, int64_t k0, int64_t kend) {
         if constexpr (CONTIG_KA) {
+            // every group of the thread reads the same 4 kk: one tap decomposition
+            const int64_t kk = k0 + 4 * (threadIdx.x % (BK / 4));
+            const typename AV::KCol kc = a.kcol(kk);
 #pragma unroll
             for (int g = 0; g < NA / 4; ++g) {
-                int il, kl; a_coord(4 * g, il, kl);
                 float o[4];
-                a.at4(m0 + il, k0 + kl, kend, o);
+                a.at4c(akr[g], kc, kk, kend, o);
 #pragma unroll
                 for (int u = 0; u < 4; ++u) ra[4 * g + u] = o[u];
             }
         } else {
-#pragma unroll
-            for (int e = 0; e < NA; ++e) {
-                int il, kl; a_coord(e, il, kl);
-                int64_t kk = k0 + kl;
-                ra[e] = kk < kend ? a.get(arow, kk) : 0.f;
-            }
+            a.template run<NA>(arow, k0 + threadIdx.x / BM, kThreads / BM, kend, ra);
         }
         if constexpr (CONTIG_KB) {
+            const int64_t kk = k0 + 4 * (threadIdx.x % (BK / 4));
+            const typename BV::KCol kc = b.kcol(kk);
 #pragma unroll
             for (int g = 0; g < NB / 4; ++g) {
-                int jl, kl; b_coord(4 * g, jl, kl);
                 float o[4];
-                b.at4(n0 + jl, k0 + kl, kend, o);
+                b.at4c(bkr[g], kc, kk, kend, o);
 #pragma unroll
                 for (int u = 0; u < 4; ++u) rb[4 * g + u] = o[u];
             }
         } else {
-#pragma unroll
-            for (int e = 0; e < NB; ++e) {
-                int jl, kl; b_coord(e, jl, kl);
-                int64_t kk = k0 + kl;
-                rb[e] = kk < kend ? b.get(brow, kk) : 0.f;
-            }
+            b.template run<NB>(brow, k0 + threadIdx.x / BN, kThreads / BN, kend, rb);
         }
     }
     __device__ __forceinline__ void store(float (*As)[BM + 4], float (*Bs)[BN + 4]) const {

@@ -169,6 +169,133 @@ __global__ void wg_input_kernel(const T* __restrict__ in, T* __restrict__ V, int
     }
 }
 
+// 4 consecutive channels as one 16-B (fp32) / 8-B (bf16) access.
+__device__ __forceinline__ void ld4(const float* p, float (&o)[4]) {
+    const float4 v = __ldg(reinterpret_cast<const float4*>(p));
+    o[0] = v.x; o[1] = v.y; o[2] = v.z; o[3] = v.w;
+}
+__device__ __forceinline__ void ld4(const __nv_bfloat16* p, float (&o)[4]) {
+    const uint2 u = __ldg(reinterpret_cast<const uint2*>(p));
+    const __nv_bfloat162 a = *reinterpret_cast<const __nv_bfloat162*>(&u.x), b = *reinterpret_cast<const __nv_bfloat162*>(&u.y);
+    o[0] = __low2float(a); o[1] = __high2float(a); o[2] = __low2float(b); o[3] = __high2float(b);
+}
+__device__ __forceinline__ void st4(float* p, const float (&v)[4]) {
+    *reinterpret_cast<float4*>(p) = make_float4(v[0], v[1], v[2], v[3]);
+}
+__device__ __forceinline__ void st4(__nv_bfloat16* p, const float (&v)[4]) {
+    uint2 u;
+    *reinterpret_cast<__nv_bfloat162*>(&u.x) = __floats2bfloat162_rn(v[0], v[1]);
+    *reinterpret_cast<__nv_bfloat162*>(&u.y) = __floats2bfloat162_rn(v[2], v[3]);
+    *reinterpret_cast<uint2*>(p) = u;
+}
+
+// wg_input_kernel / wgw_x_kernel, 4 channels per thread (I % 4 == 0): vector loads /
+// stores, tile index by multiply-high division.  Same arithmetic per channel
+// (bit-identical V).  Rows t of pitch Ip (>= I channels; padding channels and rows
+// t >= tiles are zero), planes of `plane` elements.
+template <class T>
+__global__ void wg_input4_kernel(const T* __restrict__ in, T* __restrict__ V, uint32_t total, int IH, int IW, int I,
+                                 int Ip, uint32_t tiles, FastDiv dI4, FastDiv dTW, FastDiv dTH, int pad,
+                                 int64_t plane) {
+    pdl_entry();
+    for (uint32_t idx = blockIdx.x * blockDim.x + threadIdx.x; idx < total; idx += gridDim.x * blockDim.x) {
+        const uint32_t t = dI4.div(idx), i = 4 * (idx - t * dI4.d);
+        const uint32_t t2 = dTW.div(t), tw = t - t2 * dTW.d;
+        const uint32_t n = dTH.div(t2), th = t2 - n * dTH.d;
+        const bool live = t < tiles && (int)i < I;
+        float d[4][4][4];
+#pragma unroll
+        for (int a = 0; a < 4; ++a)
+#pragma unroll
+            for (int b = 0; b < 4; ++b) {
+                const int h = 2 * (int)th - pad + a, w = 2 * (int)tw - pad + b;
+                if (live && h >= 0 && h < IH && w >= 0 && w < IW) {
+                    ld4(in + (((int64_t)n * IH + h) * IW + w) * I + i, d[a][b]);
+                } else {
+#pragma unroll
+                    for (int u = 0; u < 4; ++u) d[a][b][u] = 0.f;
+                }
+            }
+        T* out = V + (int64_t)t * Ip + i;
+#pragma unroll
+        for (int a = 0; a < 4; ++a) {
+            float e0[4], e1[4], e2[4], e3[4];  // row a of e = B^T d, per channel
+#pragma unroll
+            for (int b = 0; b < 4; ++b)
+#pragma unroll
+                for (int u = 0; u < 4; ++u) {
+                    const float v = a == 0 ? d[0][b][u] - d[2][b][u]
+                                  : a == 1 ? d[1][b][u] + d[2][b][u]
+                                  : a == 2 ? d[2][b][u] - d[1][b][u]
+                                           : d[1][b][u] - d[3][b][u];
+                    (b == 0 ? e0 : b == 1 ? e1 : b == 2 ? e2 : e3)[u] = v;
+                }
+            float v0[4], v1[4], v2[4], v3[4];  // v = e B
+#pragma unroll
+            for (int u = 0; u < 4; ++u) {
+                v0[u] = e0[u] - e2[u];
+                v1[u] = e1[u] + e2[u];
+                v2[u] = e2[u] - e1[u];
+                v3[u] = e1[u] - e3[u];
+            }
+            st4(out + (a * 4 + 0) * plane, v0);
+            st4(out + (a * 4 + 1) * plane, v1);
+            st4(out + (a * 4 + 2) * plane, v2);
+            st4(out + (a * 4 + 3) * plane, v3);
+        }
+    }
+}
+
+// wg_output_kernel, 4 channels per thread (O % 4 == 0).  Same arithmetic per channel.
+template <class T>
+__global__ void wg_output4_kernel(const float* __restrict__ M, T* __restrict__ out, uint32_t total, int OH, int OW,
+                                  int O, FastDiv dO4, FastDiv dTW, FastDiv dTH, float alpha, float beta,
+                                  int64_t plane) {
+    pdl_entry();
+    for (uint32_t idx = blockIdx.x * blockDim.x + threadIdx.x; idx < total; idx += gridDim.x * blockDim.x) {
+        const uint32_t t = dO4.div(idx), o = 4 * (idx - t * dO4.d);
+        const uint32_t t2 = dTW.div(t), tw = t - t2 * dTW.d;
+        const uint32_t n = dTH.div(t2), th = t2 - n * dTH.d;
+        const float* src = M + (int64_t)t * O + o;
+        float z[2][4][4];  // z = A^T m, per channel
+#pragma unroll
+        for (int b = 0; b < 4; ++b) {
+            float m0[4], m1[4], m2[4], m3[4];
+            ld4(src + (0 * 4 + b) * plane, m0);
+            ld4(src + (1 * 4 + b) * plane, m1);
+            ld4(src + (2 * 4 + b) * plane, m2);
+            ld4(src + (3 * 4 + b) * plane, m3);
+#pragma unroll
+            for (int u = 0; u < 4; ++u) {
+                z[0][b][u] = m0[u] + m1[u] + m2[u];
+                z[1][b][u] = m1[u] - m2[u] - m3[u];
+            }
+        }
+#pragma unroll
+        for (int a = 0; a < 2; ++a) {
+            const int h = 2 * (int)th + a;
+            if (h >= OH) continue;
+#pragma unroll
+            for (int j = 0; j < 2; ++j) {
+                const int w = 2 * (int)tw + j;
+                if (w >= OW) continue;
+                T* dst = out + (((int64_t)n * OH + h) * OW + w) * O + o;
+                float old[4] = {0.f, 0.f, 0.f, 0.f};
+                if (beta != 0.f) ld4(dst, old);
+                float y[4];
+#pragma unroll
+                for (int u = 0; u < 4; ++u) {
+                    const float yv = j == 0 ? z[a][0][u] + z[a][1][u] + z[a][2][u] : z[a][1][u] - z[a][2][u] - z[a][3][u];
+                    float v = alpha * yv;
+                    if (beta != 0.f) v += beta * old[u];
+                    y[u] = v;
+                }
+                st4(dst, y);
+            }
+        }
+    }
+}
+
 // out[n, 2th+i, 2tw+j, o] = alpha * (A^T M A)[i][j] + beta * out (masked at the
 // ragged right/bottom edge).
 template <class T>
@@ -768,6 +895,21 @@ int launch_wg_input(const Geom& g, bool dgrad, int32_t b, const void* in, void* 
     wg_dims(g, dgrad, &IH, &IW, &I, &OH, &OW, &O, &pad);
     const int TH = (OH + 1) / 2, TW = (OW + 1) / 2;
     const int64_t tiles = (int64_t)b * TH * TW;
+    if (I % 4 == 0 && tiles * I / 4 < (1LL << 31)) {
+        const uint32_t total = (uint32_t)(tiles * I / 4);
+        const int grid4 = grid_for(total, 256);
+        const FastDiv dI4((uint32_t)(I / 4)), dTW((uint32_t)TW), dTH((uint32_t)TH);
+        const int64_t plane = tiles * I;
+        if (g.math == MUCU_MATH_BF16)
+            launch_pdl(wg_input4_kernel<__nv_bfloat16>, dim3(grid4), dim3(256), (size_t)0, st,
+                       (const __nv_bfloat16*)in, (__nv_bfloat16*)V, total, IH, IW, I, I, (uint32_t)tiles, dI4, dTW,
+                       dTH, pad, plane);
+        else
+            launch_pdl(wg_input4_kernel<float>, dim3(grid4), dim3(256), (size_t)0, st, (const float*)in, (float*)V,
+                       total, IH, IW, I, I, (uint32_t)tiles, dI4, dTW, dTH, pad, plane);
+        count_launch();
+        return (int)cudaGetLastError();
+    }
     int grid = grid_for(tiles * I, 256);
     if (g.math == MUCU_MATH_BF16)
         launch_pdl(wg_input_kernel<__nv_bfloat16>, dim3(grid), dim3(256), (size_t)(0), st, (const __nv_bfloat16*)in, (__nv_bfloat16*)V, tiles, IH, IW, I, TH, TW, pad);
@@ -783,6 +925,20 @@ int launch_wg_output(const Geom& g, bool dgrad, int32_t b, float alpha, const fl
     wg_dims(g, dgrad, &IH, &IW, &I, &OH, &OW, &O, &pad);
     const int TH = (OH + 1) / 2, TW = (OW + 1) / 2;
     const int64_t tiles = (int64_t)b * TH * TW;
+    if (O % 4 == 0 && tiles * O / 4 < (1LL << 31)) {
+        const uint32_t total = (uint32_t)(tiles * O / 4);
+        const int grid4 = grid_for(total, 256);
+        const FastDiv dO4((uint32_t)(O / 4)), dTW((uint32_t)TW), dTH((uint32_t)TH);
+        const int64_t plane = tiles * O;
+        if (g.math == MUCU_MATH_BF16)
+            launch_pdl(wg_output4_kernel<__nv_bfloat16>, dim3(grid4), dim3(256), (size_t)0, st, M,
+                       (__nv_bfloat16*)out, total, OH, OW, O, dO4, dTW, dTH, alpha, beta, plane);
+        else
+            launch_pdl(wg_output4_kernel<float>, dim3(grid4), dim3(256), (size_t)0, st, M, (float*)out, total, OH,
+                       OW, O, dO4, dTW, dTH, alpha, beta, plane);
+        count_launch();
+        return (int)cudaGetLastError();
+    }
     int grid = grid_for(tiles * O, 256);
     if (g.math == MUCU_MATH_BF16)
         launch_pdl(wg_output_kernel<__nv_bfloat16>, dim3(grid), dim3(256), (size_t)(0), st, M, (__nv_bfloat16*)out, tiles, OH, OW, O, TH, TW, alpha, beta);
@@ -829,16 +985,34 @@ int launch_wgw_transforms(const Geom& g, int32_t b, const void* x, const void* d
     const int64_t tiles = (int64_t)b * TH * TW;
     const int at = 128 / elt_size(g.math);
     const int Cp = (int)align_up((uint64_t)g.c, (uint64_t)at), Kp = (int)align_up((uint64_t)g.k, (uint64_t)at);
-    if (g.math == MUCU_MATH_BF16) {
-        launch_pdl(wgw_x_kernel<__nv_bfloat16>, dim3(grid_for(Tp * Cp, 256)), dim3(256), (size_t)(0), st, 
-            (const __nv_bfloat16*)x, (__nv_bfloat16*)V, tiles, Tp, g.h, g.w, g.c, Cp, TH, TW, g.pad);
+    const bool vec = g.c % 4 == 0 && Tp * Cp / 4 < (1LL << 31);
+    if (vec) {
+        // x transform: 4 channels per thread (vector loads / stores)
+        const uint32_t total = (uint32_t)(Tp * Cp / 4);
+        const FastDiv dI4((uint32_t)(Cp / 4)), dTW((uint32_t)TW), dTH((uint32_t)TH);
+        if (g.math == MUCU_MATH_BF16)
+            launch_pdl(wg_input4_kernel<__nv_bfloat16>, dim3(grid_for(total, 256)), dim3(256), (size_t)0, st,
+                       (const __nv_bfloat16*)x, (__nv_bfloat16*)V, total, g.h, g.w, g.c, Cp, (uint32_t)tiles, dI4,
+                       dTW, dTH, g.pad, Tp * Cp);
+        else
+            launch_pdl(wg_input4_kernel<float>, dim3(grid_for(total, 256)), dim3(256), (size_t)0, st, (const float*)x,
+                       (float*)V, total, g.h, g.w, g.c, Cp, (uint32_t)tiles, dI4, dTW, dTH, g.pad, Tp * Cp);
         count_launch();
+    }
+    if (g.math == MUCU_MATH_BF16) {
+        if (!vec) {
+            launch_pdl(wgw_x_kernel<__nv_bfloat16>, dim3(grid_for(Tp * Cp, 256)), dim3(256), (size_t)(0), st,
+                (const __nv_bfloat16*)x, (__nv_bfloat16*)V, tiles, Tp, g.h, g.w, g.c, Cp, TH, TW, g.pad);
+            count_launch();
+        }
         launch_pdl(wgw_dy_kernel<__nv_bfloat16>, dim3(grid_for(Tp * Kp, 256)), dim3(256), (size_t)(0), st, 
             (const __nv_bfloat16*)dy, (__nv_bfloat16*)D, tiles, Tp, g.p, g.q, g.k, Kp, TH, TW);
     } else {
-        launch_pdl(wgw_x_kernel<float>, dim3(grid_for(Tp * Cp, 256)), dim3(256), (size_t)(0), st, (const float*)x, (float*)V, tiles, Tp, g.h, g.w,
-                                                                    g.c, Cp, TH, TW, g.pad);
-        count_launch();
+        if (!vec) {
+            launch_pdl(wgw_x_kernel<float>, dim3(grid_for(Tp * Cp, 256)), dim3(256), (size_t)(0), st, (const float*)x,
+                       (float*)V, tiles, Tp, g.h, g.w, g.c, Cp, TH, TW, g.pad);
+            count_launch();
+        }
         launch_pdl(wgw_dy_kernel<float>, dim3(grid_for(Tp * Kp, 256)), dim3(256), (size_t)(0), st, (const float*)dy, (float*)D, tiles, Tp, g.p,
                                                                      g.q, g.k, Kp, TH, TW);
     }

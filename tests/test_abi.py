@@ -144,3 +144,42 @@ def test_workspace_space_to_depth():
     # stride 1 keeps the channel-padded image (16 B per pixel)
     d = mu.desc(2, 3, 32, 32, 64, 3, 3, 1, 1, mu.MATH_BF16)
     assert mu.workspace_size(d, mu.FWD, mu.IM2COL_GEMM, 2) == 2 * 32 * 32 * 16
+
+
+# NEXT-3 entry points: argument validation happens on the host before any device work.
+def _reduce_call(target):
+    d = mu.desc(2, 8, 6, 6, 8, 3, 3, 1, 1, mu.MATH_F32)
+    plan = (_lib.MicroConfig * 1)(_lib.MicroConfig(mu.IMPLICIT_GEMM, 2))
+    return _lib.lib.mucu_conv_backward_filter_reduce(None, ctypes.byref(d), plan, 1, 1.0, ctypes.c_void_p(256),
+                                                     ctypes.c_void_p(512), 0.0, ctypes.c_void_p(1024),
+                                                     ctypes.byref(target) if target is not None else None,
+                                                     None, 0, None)
+
+
+def test_reduce_target_validation():
+    ok_ptrs = [4096, 8192]
+    assert _reduce_call(None) == 1                                        # no target
+    assert _reduce_call(_lib.reduce_target([])) == 1                      # count 0
+    assert _reduce_call(_lib.reduce_target([4096] * 8)) == 1              # valid target, NULL handle
+    t = _lib.reduce_target([4096] * 8)
+    t.count = 9
+    assert _reduce_call(t) == 1                                           # count > MUCU_MAX_REDUCE_RANKS
+    assert _reduce_call(_lib.reduce_target(ok_ptrs, multicast=True)) == 1  # multicast needs count 1
+    assert _reduce_call(_lib.reduce_target([4096 + 4])) == 6              # MISALIGNED
+    assert _reduce_call(_lib.reduce_target([0])) == 6                     # NULL destination
+
+
+def test_peer_barrier_validation_and_multicast_probe():
+    bad = _lib.reduce_target([])
+    assert _lib.lib.mucu_peer_barrier(ctypes.byref(bad), ctypes.c_void_p(4096), 1, None) == 1
+    assert _lib.lib.mucu_peer_barrier(ctypes.byref(_lib.reduce_target([4096, 8192], multicast=True)),
+                                      ctypes.c_void_p(4096), 1, None) == 1
+    assert _lib.lib.mucu_peer_barrier(ctypes.byref(_lib.reduce_target([4098])), ctypes.c_void_p(4096), 1,
+                                      None) == 6
+    # host query: no CUDA device here -> "not supported", not an error
+    assert _lib.nvls_supported(0) is False
+    h = ctypes.c_void_p()
+    assert _lib.lib.mucu_nvls_create(0, 0, 1024, ctypes.byref(h)) == 1     # ranks < 1
+    assert _lib.lib.mucu_nvls_import(0, 1, 1024, -1, ctypes.byref(h)) == 1  # fd < 0
+    assert _lib.lib.mucu_nvls_barrier(None, None) == 1
+    assert _lib.lib.mucu_nvls_destroy(None) == 0

@@ -2,7 +2,7 @@
 # Round measurement on a B200 box (run via gpurun from the repo root):
 #   tests, smoke, benches, the ncu launch list of the default bench step and a
 #   full-set capture of its dominant kernel.  Every step has its own timeout.
-# usage: tools/gpu_round.sh TAG [steps...]   steps: tests smoke bench others launches full extra ops
+# usage: tools/gpu_round.sh TAG [steps...]   steps: tests smoke bench others launches full extra ops fused
 set -u
 TAG=${1:-r01}; shift
 STEPS=${*:-"tests smoke bench others launches full"}
@@ -102,4 +102,10 @@ if has ops; then
     alexnet:f32:conv3:FWD:WG:32 alexnet:f32:conv5:WGRAD:WG:32 alexnet:tf32:conv2:WGRAD:IG:256 \
     alexnet:tf32:conv2:DGRAD:IG:256 alexnet:tf32:conv1:FWD:I2C:64 resnet50:bf16:layer1.0.conv2:FWD:IG:256 \
     resnet50:bf16:layer1.0.conv2:DGRAD:IG:256 resnet50:bf16:layer1.0.conv2:WGRAD:IG:256 2>&1 | tee -a $OUT/status
+fi
+if has fused; then
+  # NEXT-3: the dW sum fused into BackwardFilter (P2P target at one GPU; multicast where the box allows)
+  timeout -s KILL 600 python -m pytest tests/test_nvls_gpu.py -q -rs > $OUT/nvls_tests.log 2>&1; echo "nvls tests rc=$?" | tee -a $OUT/status
+  timeout -s KILL 900 python bench.py --grad-reduce p2p --no-cpu-baseline --json-out $OUT/bench_alexnet_tf32_p2p.json \
+    > $OUT/bench_p2p.log 2>&1; echo "bench p2p rc=$?" | tee -a $OUT/status
 fi

@@ -518,16 +518,7 @@ int dispatch_gemm(const AV& a, const BV& b, const EPI& e, int64_t M, int64_t N, 
         const Cand& c = cands[i];
         if (N <= 64 && c.bn == 128) continue;
         const int64_t tiles = ceil_div(M, c.bm) * ceil_div(N, c.bn) * batch;
-        // full waves at per_sm resident CTAs, then the last partial wave with r CTAs per SM:
-        // an SM with fewer than 16 resident warps runs the FFMA tile at a lower rate
-        // (measured: one 8-warp CTA per SM ~0.6 of two)
-        const int64_t slots = (int64_t)sms * c.per_sm, full = tiles / slots, rem = tiles % slots;
-        const double area = (double)c.bm * c.bn / c.eff;
-        double cost = (double)full * c.per_sm * area;
-        if (rem) {
-            const int64_t r = ceil_div(rem, (int64_t)sms);
-            cost += (double)r * area / std::min(1.0, 0.2 + 0.05 * (double)(r * kThreads / 32));
-        }
+        const double cost = (double)ceil_div(tiles, (int64_t)sms * c.per_sm) * c.per_sm * c.bm * c.bn / c.eff;
         if (cost < best_cost - 1e-9) { best_cost = cost; best = i; }
     }
     if (best == 0) return launch_gemm<128, 128, CKA, CKB>(a, b, e, M, N, Kd, batch, st);

@@ -352,6 +352,8 @@ def main():
     # (network.iteration concurrent=True); the evented per-op pass is sequential.
     conc = args.concurrent_wgrad
 
+    host_ms = []  # host enqueue time of the steps of the last timed() call
+
     def timed(nsteps, nwarm, record_ops=False):
         ops = {}
         for _ in range(nwarm):
@@ -362,6 +364,7 @@ def main():
             dist.barrier()
         torch.cuda.synchronize()
         step_ms = []
+        host_ms.clear()
         launches0 = mu._lib.launch_count()
         for _ in range(nsteps):
             flush.zero_()  # L2 flush (outside the timed events)
@@ -375,9 +378,11 @@ def main():
             s0 = torch.cuda.Event(enable_timing=True)
             s1 = torch.cuda.Event(enable_timing=True)
             s0.record(stream)
+            h0 = time.perf_counter()
             net.iteration(on_op=on_op, grad_hook=grad_ar, skip_conv1_dgrad=skip_c1,
                           concurrent=conc and not record_ops)
             grad_ar.wait()
+            host_ms.append((time.perf_counter() - h0) * 1e3)  # host time to enqueue the step
             s1.record(stream)
             s1.synchronize()
             step_ms.append(s0.elapsed_time(s1))
@@ -423,6 +428,7 @@ def main():
     # with events around every call.
     with ClockSampler(local) as clk:
         ms, _, launches = timed(args.steps, args.warmup)
+    host_enqueue_ms = float(np.mean(host_ms)) if host_ms else None
     ms_max = max_over_ranks(ms)
     ms_ops, ops, _ = timed(max(3, args.steps // 2), 1, record_ops=True)
 
@@ -578,6 +584,7 @@ def main():
             "images_per_s": round(args.batch * world / (ms_max * 1e-3), 1),
             "conv_tflops_direct": round(conv_flops * world / (ms_max * 1e-3) / 1e12, 2),
             "ms_per_step_with_op_events": round(ms_ops, 4),
+            "host_enqueue_ms_per_step": round(host_enqueue_ms, 4) if host_enqueue_ms is not None else None,
             "undivided_ms_per_step": round(und_ms, 4) if und_ms is not None else None,
             "speedup_vs_undivided": round(und_ms / ms_max, 4) if und_ms is not None else None,
             "speedup_by_kernel": {kname(i, t): round(und_op_ms[(i, t)] / v, 3)

@@ -222,9 +222,11 @@ mucu_status_t mucu_solve_wd(int32_t num_kernels, const int32_t* front_len, const
 /* ------------------------------------------------------------- GPU ---- */
 /* Benchmark pass (P:L88 WR step 1): for every b in the handle's policy set and
  * every eligible algorithm whose workspace fits ws_limit, run the micro-config
- * on scratch tensors: `warmup` untimed launches, then three CUDA-event samples,
- * each the mean of `reps` back-to-back launches (the way a plan's micro-batches
- * run), median of the three, quantised to ns (reading G21).  Steady state: the
+ * on scratch tensors: `warmup` launches (the last one timed), then three
+ * CUDA-event samples, each the mean of up to `reps` back-to-back launches (the
+ * way a plan's micro-batches run; a sample stops at ~1 ms of work, so a long
+ * micro-config takes one launch per sample), median of the three, quantised to
+ * ns (reading G21).  Steady state: the
  * b-independent workspace prefix (filter transforms) is computed by the warm-up
  * and reused, as the executor computes it once per call.  Fills time_ns / ws
  * ([MUCU_NUM_ALGOS][desc->n + 1], -1 / 0 where not measured).  Identical

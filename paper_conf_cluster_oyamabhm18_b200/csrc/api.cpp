@@ -3,6 +3,7 @@
 // the benchmark pass (P:L88 WR step 1) and WD network planning
 // (P:L163-167).
 #include <cuda_runtime.h>
+#include <cmath>
 
 #include <algorithm>
 #include <atomic>
@@ -697,6 +698,9 @@ extern "C" mucu_status_t mucu_conv_backward_filter_reduce(mucu_handle_t h, const
 }
 
 // ============================================================ benchmark ====
+// Work per benchmark sample (ms): samples of longer micro-configurations use fewer launches.
+constexpr float kBenchSampleMs = 1.0f;
+
 static std::vector<int32_t> policy_sizes(int policy, int32_t n) {
     std::vector<int32_t> v;
     if (policy == MUCU_POLICY_ALL) {
@@ -799,22 +803,38 @@ extern "C" mucu_status_t mucu_benchmark(mucu_handle_t h, const mucu_conv_desc_t*
                     continue;
             }
             mucu_status_t r = MUCU_OK;
-            for (int i = 0; i < h->warmup && r == MUCU_OK; ++i) r = launch();
+            // warm-up (the first launch builds the call's prefix); the last warm-up launch
+            // is timed to size the samples
+            float t1 = 0.f;
+            for (int i = 0; i < h->warmup && r == MUCU_OK; ++i) {
+                const bool last = i == h->warmup - 1;
+                if (last) cudaEventRecord(e0, st);
+                r = launch();
+                if (last && r == MUCU_OK) {
+                    cudaEventRecord(e1, st);
+                    if (cudaEventSynchronize(e1)) { r = cuda_error((int)cudaGetLastError(), "benchmark sync"); break; }
+                    cudaEventElapsedTime(&t1, e0, e1);
+                }
+            }
             if (r == MUCU_ERR_UNSUPPORTED) continue;
             if (r) { status = r; break; }
             // T_mu(b) (P:L88 step 1): micro-batches run back to back in a plan, so each sample
             // is the mean of `reps` back-to-back launches between two events (no idle-stream
-            // launch latency in the table); the median of three samples is recorded.
+            // launch latency in the table); the median of three samples is recorded.  A
+            // sample needs no more launches than make ~1 ms of work (long micro-configs:
+            // one launch per sample), which keeps the `all` policy's pass short.
+            int reps = h->reps;
+            if (t1 > 0.f) reps = std::max(1, std::min(h->reps, (int)std::ceil(kBenchSampleMs / t1)));
             samples.clear();
             for (int grp = 0; grp < 3 && r == MUCU_OK; ++grp) {
                 cudaEventRecord(e0, st);
-                for (int i = 0; i < h->reps && r == MUCU_OK; ++i) r = launch();
+                for (int i = 0; i < reps && r == MUCU_OK; ++i) r = launch();
                 cudaEventRecord(e1, st);
                 if (r) break;
                 if (cudaEventSynchronize(e1)) { r = cuda_error((int)cudaGetLastError(), "benchmark sync"); break; }
                 float ms = 0.f;
                 cudaEventElapsedTime(&ms, e0, e1);
-                samples.push_back(ms / (float)std::max(1, h->reps));
+                samples.push_back(ms / (float)reps);
             }
             if (r == MUCU_ERR_UNSUPPORTED) continue;
             if (r) { status = r; break; }

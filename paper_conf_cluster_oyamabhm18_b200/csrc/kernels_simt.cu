@@ -468,19 +468,34 @@ __global__ void __launch_bounds__(kThreads, ctas_per_sm(BM, BN)) simt_wgrad_kern
     if (threadIdx.x == 0 && split > 0) turn_wait(turns + tile, turn_tag(epoch, split - 1));
     __syncthreads();
     const int tx = threadIdx.x % 16, ty = threadIdx.x / 16;
+    // the hand-off is on the ordered chain's critical path: every load of the thread's
+    // TM x TN elements is issued before the first store (one L2 round trip, not TM x TN)
+    const float bs = split > 0 ? 1.f : beta;
+    if (bs != 0.f) {
+#pragma unroll
+        for (int i = 0; i < TM; ++i) {
+            const int64_t r = m0 + frag_off<TM, BM>(ty, i);
+#pragma unroll
+            for (int j = 0; j < TN; ++j) {
+                const int64_t cidx = n0 + frag_off<TN, BN>(tx, j);
+                acc[i][j] = alpha * acc[i][j];
+                if (r < rows && cidx < cols) acc[i][j] += bs * __ldcg(dw + r * cols + cidx);
+            }
+        }
+    } else {
+#pragma unroll
+        for (int i = 0; i < TM; ++i)
+#pragma unroll
+            for (int j = 0; j < TN; ++j) acc[i][j] = alpha * acc[i][j];
+    }
 #pragma unroll
     for (int i = 0; i < TM; ++i) {
-        int64_t r = m0 + frag_off<TM, BM>(ty, i);
+        const int64_t r = m0 + frag_off<TM, BM>(ty, i);
         if (r >= rows) continue;
 #pragma unroll
         for (int j = 0; j < TN; ++j) {
-            int64_t cidx = n0 + frag_off<TN, BN>(tx, j);
-            if (cidx >= cols) continue;
-            float* d = dw + r * cols + cidx;
-            float v = alpha * acc[i][j];
-            if (split > 0) v += __ldcg(d);
-            else if (beta != 0.f) v += beta * __ldcg(d);
-            *d = v;
+            const int64_t cidx = n0 + frag_off<TN, BN>(tx, j);
+            if (cidx < cols) dw[r * cols + cidx] = acc[i][j];
         }
     }
     __syncthreads();

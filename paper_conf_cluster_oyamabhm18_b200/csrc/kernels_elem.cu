@@ -1032,7 +1032,16 @@ __global__ void partial_reduce_kernel(int S, int64_t slot, int ldp, int M, int N
         const int m = (int)(idx / N), n = (int)(idx - (int64_t)m * N);
         const float* p = part + (size_t)m * ldp + n;
         float acc = 0.f;
-        for (int s = 0; s < S; ++s) acc += __ldg(p + (size_t)s * slot);
+        // slots summed in order; eight loads in flight per group (the adds stay sequential)
+        int s = 0;
+        for (; s + 8 <= S; s += 8) {
+            float v[8];
+#pragma unroll
+            for (int u = 0; u < 8; ++u) v[u] = __ldg(p + (size_t)(s + u) * slot);
+#pragma unroll
+            for (int u = 0; u < 8; ++u) acc += v[u];
+        }
+        for (; s < S; ++s) acc += __ldg(p + (size_t)s * slot);
         float* d = transpose ? out + (size_t)n * M + m : out + idx;
         const float o = beta != 0.f ? alpha * acc + beta * *d : alpha * acc;
         *d = o;

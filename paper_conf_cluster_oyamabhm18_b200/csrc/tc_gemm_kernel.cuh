@@ -272,40 +272,68 @@ __global__ void __launch_bounds__(threads_for(AM), 1) tc_conv_gemm(const __grid_
         constexpr int EPC = 16 / ELT;             // elements per 16-B chunk
         const int CH = TR / EPC;                  // chunks per A K-row (pixel)
         const int stC = p.stride * p.C;
-        auto x_coords = [&](int kb, int& cq0, int& chunk0, int& h0, int& n_, int& col0, int& valid) {
-            const int row = kb / p.win_qb, qb = kb - row * p.win_qb;
-            n_ = row / p.P;
-            const int pp = row - n_ * p.P;
-            cq0 = qb * KD;
-            h0 = p.stride * pp - p.pad;
-            const int e0 = (p.stride * cq0 - p.pad) * p.C;
-            chunk0 = e0 >= 0 ? e0 / p.sx_cs : -((-e0 + p.sx_cs - 1) / p.sx_cs);
-            col0 = e0 - chunk0 * p.sx_cs;
-            valid = min(KD, p.Q - cq0);
+        // k-block walk: (output row n*P + p, q-block qb) -> the x stage's TMA coordinates
+        // and the builders' column offset.  Divisions once per tile (init), then each
+        // k-block advances incrementally (the builders' integer divisions were a third
+        // of their stall samples).
+        struct XWalk {
+            int qb, pp, n_, chunk0, col0, cq0;
+            int chunk_start, col_start, adv_q, adv_r;
+        };
+        auto x_init = [&](int kb, XWalk& w) {
+            const int row = kb / p.win_qb;
+            w.qb = kb - row * p.win_qb;
+            w.n_ = row / p.P;
+            w.pp = row - w.n_ * p.P;
+            const int e_start = -p.pad * p.C;  // e0 of q-block 0
+            w.chunk_start = e_start >= 0 ? e_start / p.sx_cs : -((-e_start + p.sx_cs - 1) / p.sx_cs);
+            w.col_start = e_start - w.chunk_start * p.sx_cs;
+            const int adv = p.stride * KD * p.C;  // e0 step per q-block
+            w.adv_q = adv / p.sx_cs;
+            w.adv_r = adv - w.adv_q * p.sx_cs;
+            w.cq0 = w.qb * KD;
+            const int e0 = (p.stride * w.cq0 - p.pad) * p.C;
+            w.chunk0 = e0 >= 0 ? e0 / p.sx_cs : -((-e0 + p.sx_cs - 1) / p.sx_cs);
+            w.col0 = e0 - w.chunk0 * p.sx_cs;
+        };
+        auto x_step = [&](XWalk& w) {
+            if (++w.qb == p.win_qb) {
+                w.qb = 0; w.cq0 = 0; w.chunk0 = w.chunk_start; w.col0 = w.col_start;
+                if (++w.pp == p.P) { w.pp = 0; ++w.n_; }
+            } else {
+                w.cq0 += KD;
+                w.chunk0 += w.adv_q;
+                w.col0 += w.adv_r;
+                if (w.col0 >= p.sx_cs) { w.col0 -= p.sx_cs; ++w.chunk0; }
+            }
         };
         if (warp == 9) {
             if (lane == 0) {
-                int ai = 0;
+                int s = 0, jx = 0;
+                uint32_t ph = 0, xph = 0;
                 for (int tile = blockIdx.x; tile < total_tiles; tile += gridDim.x) {
                     int m0, n0, z, kb_begin, kb_end;
                     decode(tile, m0, n0, z, kb_begin, kb_end);
-                    for (int kb = kb_begin; kb < kb_end; ++kb, ++ai) {
-                        const int s = ai % S, jx = ai % p.sx_stages;
-                        int cq0, chunk0, h0, n_, col0, valid;
-                        x_coords(kb, cq0, chunk0, h0, n_, col0, valid);
+                    XWalk w;
+                    if (kb_begin < kb_end) x_init(kb_begin, w);
+                    for (int kb = kb_begin; kb < kb_end; ++kb) {
                         // x rows into ring stage jx (freed by the builders)
-                        mbar_wait(smem_u32(&xempty[jx]), (uint32_t)(((ai / p.sx_stages) & 1) ^ 1));
+                        mbar_wait(smem_u32(&xempty[jx]), xph ^ 1u);
                         const uint32_t xb = smem_u32(&xfull[jx]);
                         mbar_arrive_tx(xb, (uint32_t)p.sx_tx);
-                        tma_load_4d(smem_u32(sBres + (size_t)jx * p.sx_bytes), &tmA, xb, 0, chunk0, h0, n_);
+                        tma_load_4d(smem_u32(sBres + (size_t)jx * p.sx_bytes), &tmA, xb, 0, w.chunk0,
+                                    p.stride * w.pp - p.pad, w.n_);
                         // dy of the KD pixels into operand stage s (freed by the MMA)
-                        mbar_wait(smem_u32(&empty[s]), (uint32_t)(((ai / S) & 1) ^ 1));
+                        mbar_wait(smem_u32(&empty[s]), ph ^ 1u);
                         const uint32_t bT = smem_u32(sB + (size_t)s * B_BYTES);
                         const uint32_t fb = smem_u32(&full[s]);
                         mbar_arrive_tx(fb, (uint32_t)p.tma_bytes);
-                        const int row = kb / p.win_qb;
+                        const int row = w.n_ * p.P + w.pp;
                         for (int a = 0; a < p.bn_atoms; ++a)
-                            tma_load_3d(bT + a * KD * 128, &tmB, fb, n0 + a * (128 / ELT), cq0, row);
+                            tma_load_3d(bT + a * KD * 128, &tmB, fb, n0 + a * (128 / ELT), w.cq0, row);
+                        x_step(w);
+                        if (++s == S) { s = 0; ph ^= 1u; }
+                        if (++jx == p.sx_stages) { jx = 0; xph ^= 1u; }
                     }
                 }
             }
@@ -335,18 +363,19 @@ __global__ void __launch_bounds__(threads_for(AM), 1) tc_conv_gemm(const __grid_
                     u_src[j][e] = t >= 0 ? (t + stC * 4 * u_gr[j]) * ELT : -1;
                 }
             }
-            int ai = 0;
+            int s = 0, jx = 0;
+            uint32_t ph = 0, xph = 0;
             for (int tile = blockIdx.x; tile < total_tiles; tile += gridDim.x) {
                 int m0, n0, z, kb_begin, kb_end;
                 decode(tile, m0, n0, z, kb_begin, kb_end);
-                for (int kb = kb_begin; kb < kb_end; ++kb, ++ai) {
-                    const int s = ai % S, jx = ai % p.sx_stages;
-                    int cq0, chunk0, h0, n_, col0, valid;
-                    x_coords(kb, cq0, chunk0, h0, n_, col0, valid);
-                    mbar_wait(smem_u32(&empty[s]), (uint32_t)(((ai / S) & 1) ^ 1));
-                    mbar_wait(smem_u32(&xfull[jx]), (uint32_t)((ai / p.sx_stages) & 1));
+                XWalk w;
+                if (kb_begin < kb_end) x_init(kb_begin, w);
+                for (int kb = kb_begin; kb < kb_end; ++kb) {
+                    const int valid = min(KD, p.Q - w.cq0);
+                    mbar_wait(smem_u32(&empty[s]), ph ^ 1u);
+                    mbar_wait(smem_u32(&xfull[jx]), xph);
                     const uint32_t aT = smem_u32(sA + (size_t)s * A_BYTES);
-                    const uint32_t xs = smem_u32(sBres) + (uint32_t)(jx * p.sx_bytes) + (uint32_t)(col0 * ELT);
+                    const uint32_t xs = smem_u32(sBres) + (uint32_t)(jx * p.sx_bytes) + (uint32_t)(w.col0 * ELT);
                     // rows (pixels) the MMA reads: valid rounded up to the MMA K step (the
                     // rest of the stage is never read; dy rows past Q are zero-filled)
                     const int nrows = min(KD, (valid + UMMA_K - 1) / UMMA_K * UMMA_K);
@@ -390,6 +419,9 @@ __global__ void __launch_bounds__(threads_for(AM), 1) tc_conv_gemm(const __grid_
                     fence_proxy_async();
                     mbar_arrive(smem_u32(&full[s]));
                     mbar_arrive(smem_u32(&xempty[jx]));
+                    x_step(w);
+                    if (++s == S) { s = 0; ph ^= 1u; }
+                    if (++jx == p.sx_stages) { jx = 0; xph ^= 1u; }
                 }
             }
         }
@@ -1154,6 +1186,7 @@ __global__ void __launch_bounds__(threads_for(AM), 1) tc_conv_gemm(const __grid_
             mbar_wait(smem_u32(&tempty[acc]), aph ^ 1u);  // epilogue has drained this accumulator
             tc_fence_after();
             const uint32_t dtm = tmem + (uint32_t)(acc * p.mt * p.BN);
+            int sqb = STAGED ? kb_begin % p.win_qb : 0;  // A_STAGED_WG: q-block of kb (incremental)
             for (int kb = kb_begin; kb < kb_end; ++kb, s = (s + 1 == S) ? 0 : s + 1, ph ^= (s == 0) ? 1u : 0u) {
                 mbar_wait(smem_u32(&full[s]), ph);
                 tc_fence_after();
@@ -1171,8 +1204,8 @@ __global__ void __launch_bounds__(threads_for(AM), 1) tc_conv_gemm(const __grid_
                     // steps that cover its valid pixels
                     int jmax = KB / UMMA_K;
                     if constexpr (STAGED) {
-                        const int qb = kb % p.win_qb;
-                        jmax = min(jmax, (min(KD, p.Q - qb * KD) + UMMA_K - 1) / UMMA_K);
+                        jmax = min(jmax, (min(KD, p.Q - sqb * KD) + UMMA_K - 1) / UMMA_K);
+                        if (++sqb == p.win_qb) sqb = 0;
                     }
                     auto issue = [&](auto mt_c, const int jj) {
                         constexpr int MT = decltype(mt_c)::value;

@@ -155,7 +155,8 @@ mucu_status_t mucu_output_dims(const mucu_conv_desc_t* desc, int32_t* p, int32_t
  *                          b*H*Wp*4*elt; atoms of aw bytes (TF32: 128; BF16: the aw in {128, 64, 32}
  *                          minimising align256(R*na*aw/elt), larger aw on ties), tpa = aw/(4*elt)
  *                          taps per atom, na = ceil(S/tpa), Wp = max(st*(Q-1) + na*tpa, W + pad)
- *                          rounded up to 4
+ *                          rounded up to 4; + 148 partial dW tiles of M = R*na*aw/elt window rows:
+ *                          align256(148 * M * K * 4) (deterministic split-K in split order)
  *                     WGRAD otherwise (u = 1, f = st): b*(P+Dr-1)*(Q+Ds-1)*Cs*elt
  *                     DGRAD (when K % (128/elt) == 0, st*st*C <= 256): u = 2 if (2*st)^2*C <= 256
  *                          else 1, f = st*u, Dr = ceil(R/st) - 1 + u, Ds likewise: f*f*C*Dr*Ds*K*elt

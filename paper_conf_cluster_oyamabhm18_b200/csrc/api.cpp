@@ -218,11 +218,15 @@ mucu_status_t ws_layout(const Geom& g, int type, int algo, int32_t b, WsLayout* 
             return MUCU_OK;
         }
         if (win_tc(g, type)) {
+            // padded x, then (deterministic split-K) kPartialSlots partial dW tiles of
+            // z.M window rows x K filters fp32 (b-independent)
             const Win z = win_geom(g);
             L->a_off = 0;
             L->a_bytes = align_up((uint64_t)b * g.h * z.Wp * z.cpx * elt, 256);
+            L->b_off = L->a_bytes;
+            L->b_bytes = align_up((uint64_t)kPartialSlots * z.M * g.k * 4, 256);
             L->kpitch = z.cpx;
-            L->total = L->a_bytes;
+            L->total = L->a_bytes + L->b_bytes;
             return MUCU_OK;
         }
         if (s2d_tc(g, type)) {

@@ -1059,6 +1059,52 @@ int launch_partial_reduce(int S, int64_t slot, int ldp, int M, int N, bool trans
     return (int)cudaGetLastError();
 }
 
+// Window BackwardFilter partial slots: part[s][m][k] over window rows
+// m = (r, atom ja, tap t, channel c) (per_atom = t * cp + c per atom, na atoms per filter
+// row) -> dw[k][r][ja*tpa + t][c]; slots summed in order (eight loads in flight),
+// padding rows skipped.
+__global__ void partial_reduce_win_kernel(int S, int64_t slot, int M, int K, int per_atom, int cp, int na, int R,
+                                          int Sf, int C, const float* __restrict__ part, float alpha, float beta,
+                                          float* __restrict__ dw, const RedTarget red) {
+    pdl_entry();
+    const int64_t total = (int64_t)M * K;
+    const int64_t RSC = (int64_t)R * Sf * C;
+    for (int64_t idx = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; idx < total;
+         idx += (int64_t)gridDim.x * blockDim.x) {
+        const int m = (int)(idx / K), k = (int)(idx - (int64_t)m * K);
+        const int ja = m / per_atom, e = m - ja * per_atom;
+        const int t = e / cp, c = e - t * cp;
+        const int r = ja / na, sx = (ja - r * na) * (per_atom / cp) + t;
+        if (r >= R || sx >= Sf || c >= C) continue;
+        const float* p = part + (size_t)m * K + k;
+        float acc = 0.f;
+        int s = 0;
+        for (; s + 8 <= S; s += 8) {
+            float v[8];
+#pragma unroll
+            for (int u = 0; u < 8; ++u) v[u] = __ldg(p + (size_t)(s + u) * slot);
+#pragma unroll
+            for (int u = 0; u < 8; ++u) acc += v[u];
+        }
+        for (; s < S; ++s) acc += __ldg(p + (size_t)s * slot);
+        float* d = dw + (int64_t)k * RSC + ((int64_t)r * Sf + sx) * C + c;
+        const float o = beta != 0.f ? alpha * acc + beta * *d : alpha * acc;
+        *d = o;
+        if (red.n) red_add(red, d - dw, o);  // NEXT-3: the cross-rank dW sum
+    }
+}
+
+int launch_partial_reduce_win(int S, int64_t slot, int M, int K, int per_atom, int cp, int na, const Geom& g,
+                              const float* part, float alpha, float beta, float* dw, cudaStream_t st,
+                              const RedTarget* red) {
+    RedTarget r = {};
+    if (red) r = *red;
+    launch_pdl(partial_reduce_win_kernel, dim3(grid_for((int64_t)M * K, 256)), dim3(256), (size_t)0, st, S, slot, M,
+               K, per_atom, cp, na, g.r, g.s, g.c, part, alpha, beta, dw, r);
+    count_launch();
+    return (int)cudaGetLastError();
+}
+
 int launch_wgw_output(const Geom& g, float alpha, const float* M, float beta, float* dw, cudaStream_t st) {
     const int at = 128 / elt_size(g.math);
     const int Cp = (int)align_up((uint64_t)g.c, (uint64_t)at), Kp = (int)align_up((uint64_t)g.k, (uint64_t)at);

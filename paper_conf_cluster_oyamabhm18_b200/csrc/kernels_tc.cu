@@ -1069,6 +1069,29 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         }
         if (!map3(&L.tb, in1, g.k, g.q, (uint64_t)b * g.p, g.k, (uint64_t)g.q * g.k, atom, KD, 1, true)) return -1;
         A.tma_bytes = A.km * (A.mt * 128 * KB * elt + A.bn_atoms * KB * 128);
+        if (ctx->deterministic) {
+            // Deterministic split-K through the workspace: one split per SM
+            // (at most kPartialSlots) writes its partial tile [z.M rows][K] fp32; a reduction
+            // kernel sums the slots in split order and scatters the window rows into dw --
+            // every SM busy, no cluster packing loss or ordered group hand-offs.
+            const int64_t nkb = (int64_t)b * g.p * A.win_qb;
+            const int64_t S = std::max<int64_t>(1, std::min<int64_t>(std::min<int64_t>(kPartialSlots, num_sms), nkb));
+            A.num_kb = (int)nkb;
+            A.kb_per_split = (int)ceil_div(nkb, S);
+            const int64_t Sr = ceil_div(nkb, A.kb_per_split);
+            A.cl = 0; A.zsplit = 0; A.atomic = 0; A.stg_bytes = 0;
+            A.num_z = (int)Sr;
+            L.grid = dim3((unsigned)Sr);
+            float* part = (float*)(ws + WL.b_off);
+            A.out = part; A.alpha = 1.f; A.beta = 0.f; A.ldc = g.k; A.part_rows = z.M;
+            if (z.aw == 64) err = LAUNCH(A_TMA_WIN64, B_TMA_DYROW, EPI_WGRAD_PARTIAL);
+            else if (z.aw == 32) err = LAUNCH(A_TMA_WIN32, B_TMA_DYROW, EPI_WGRAD_PARTIAL);
+            else err = LAUNCH(A_TMA_WIN, B_TMA_DYROW, EPI_WGRAD_PARTIAL);
+            if (err) return err;
+            note_fused();
+            return DRY(launch_partial_reduce_win((int)Sr, (int64_t)z.M * g.k, z.M, g.k, z.aw / elt, z.cpx, z.na, g,
+                                                 part, alpha, beta, (float*)out, st, mc_reduce));
+        }
         if (z.aw == 64) return LAUNCH(A_TMA_WIN64, B_TMA_DYROW, EPI_WGRAD_WIN);
         if (z.aw == 32) return LAUNCH(A_TMA_WIN32, B_TMA_DYROW, EPI_WGRAD_WIN);
         return LAUNCH(A_TMA_WIN, B_TMA_DYROW, EPI_WGRAD_WIN);

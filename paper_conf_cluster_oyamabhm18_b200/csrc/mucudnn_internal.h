@@ -265,6 +265,11 @@ int launch_wgw_output(const Geom& g, float alpha, const float* M, float beta, fl
 // red (NEXT-3): the final values are also added to the cross-rank dW sum (n = 0: off).
 int launch_partial_reduce(int S, int64_t slot, int ldp, int M, int N, bool transpose, const float* part,
                           float alpha, float beta, float* out, cudaStream_t st, const RedTarget* red = nullptr);
+// The same for the window BackwardFilter's partial tiles (rows = window rows, DESIGN.md
+// 6.5; padding rows skipped), out = dw [K][R][S][C].
+int launch_partial_reduce_win(int S, int64_t slot, int M, int K, int per_atom, int cp, int na, const Geom& g,
+                              const float* part, float alpha, float beta, float* dw, cudaStream_t st,
+                              const RedTarget* red = nullptr);
 // NEXT-3 (nvls.cu): target[i] += src[i] (16-B vectors where aligned) for the dw writers
 // that do not fuse the reduction; and the barrier over the ranks: release-add 1 to
 // every flag word in `flags` (one multicast address, or every rank's flag), then wait

@@ -128,13 +128,16 @@ def test_workspace_space_to_depth():
     assert mu.workspace_size(d, mu.FWD, mu.IM2COL_GEMM, 2) == a256(4 * 64 * 9 * 64 * 2) + a256(2 * 58 * 58 * 64 * 2)
     # WGRAD: 147 taps -> 256 staged rows is > 1/4 padding: window form (64-B atoms, tpa = 8,
     # na = 1), Wp = max(2*(Q-1) + 8, W + 3) rounded up to 4 = 232
-    assert mu.workspace_size(d, mu.BWD_FILTER, mu.IM2COL_GEMM, 2) == a256(2 * 224 * 232 * 4 * 2)
+    # + 148 deterministic split-K partial tiles of M = 7 rows x 32 (one 64-B atom) x K fp32
+    assert mu.workspace_size(d, mu.BWD_FILTER, mu.IM2COL_GEMM, 2) == a256(2 * 224 * 232 * 4 * 2) + \
+        a256(148 * 224 * 64 * 4)
     # window form when the x row (W*C*elt) is not a multiple of 16 B: 64-B atoms (one 8-tap atom
     # per filter row), tpa = 8, na = 1, Wp = max(2*(Q-1) + 8, W + 3) rounded up to 4
     d = mu.desc(2, 3, 223, 223, 64, 7, 7, 3, 2, mu.MATH_BF16)  # W*C = 669: no chunking
     q = (223 + 6 - 7) // 2 + 1
     wp = -(-max(2 * (q - 1) + 8, 223 + 3) // 4) * 4
-    assert mu.workspace_size(d, mu.BWD_FILTER, mu.IM2COL_GEMM, 2) == a256(2 * 223 * wp * 4 * 2)
+    assert mu.workspace_size(d, mu.BWD_FILTER, mu.IM2COL_GEMM, 2) == a256(2 * 223 * wp * 4 * 2) + \
+        a256(148 * 224 * 64 * 4)
     # DGRAD: f = 4 (4*4*3 = 48 columns), Dr = 6 // 2 + 2 = 5: filter 48 x 25*64
     assert mu.workspace_size(d, mu.BWD_DATA, mu.IM2COL_GEMM, 2) == a256(48 * 25 * 64 * 2)
     # stride 3, BF16: 3*8 B is not a multiple of 16 -> WGRAD keeps the space-to-depth image

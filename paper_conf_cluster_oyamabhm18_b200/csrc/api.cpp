@@ -57,6 +57,10 @@ bool is_pointwise(const Geom& g) { return g.r == 1 && g.s == 1 && g.pad == 0 && 
 
 bool small_c_tc(const Geom& g) { return g.math != MUCU_MATH_F32 && g.c * elt_size(g.math) < 16; }
 
+bool i2c_implicit_wgrad(const Geom& g) {
+    return g.math != MUCU_MATH_F32 && !is_pointwise(g) && g.c % (128 / elt_size(g.math)) == 0;
+}
+
 int s2d_channels(const Geom& g) {
     const int atom = 128 / elt_size(g.math);
     return (int)align_up((uint64_t)g.stride * g.stride * g.c, (uint64_t)atom);
@@ -205,6 +209,12 @@ mucu_status_t ws_layout(const Geom& g, int type, int algo, int32_t b, WsLayout* 
         const uint64_t part = P > 1 ? align_up((uint64_t)P * g.k * RSC * 4, 256) : 0;
         if (is_pointwise(g)) {
             L->kpitch = g.c;
+            L->b_off = 0; L->b_bytes = part; L->total = part;
+            return MUCU_OK;
+        }
+        if (type == MUCU_BWD_FILTER && i2c_implicit_wgrad(g)) {
+            // TMA im2col into shared memory: only the per-split partial dW slots
+            L->a_off = 0; L->a_bytes = 0;
             L->b_off = 0; L->b_bytes = part; L->total = part;
             return MUCU_OK;
         }

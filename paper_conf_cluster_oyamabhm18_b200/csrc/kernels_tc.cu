@@ -1547,6 +1547,54 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
             A.tma_bytes = a_bytes;
             return LAUNCH(A_TMA_MN2, B_GATHER_SMALLC_PAD, EPI_WGRAD_SMALLC);
         }
+        // Workspace partials: persistent CTAs over all SMs, split s writes its dW tile to
+        // slot s, a reduction kernel sums the slots in order (no cluster packing loss, no
+        // ordered hand-over).  `launch_partial(launch)` runs the GEMM launcher given.
+        auto launch_partial = [&](auto launch) -> int {
+            const int P = wgrad_partial_slots(g);
+            const int64_t tiles = ceil_div(A.N, A.BN) * ceil_div(A.M, 128 * A.mt);
+            const int64_t nkb = A.num_kb;
+            const double E = env_int("MUCU_SPLIT_E", 16) / (double)A.km;
+            int64_t sbest = 1;
+            double best = 1e30;
+            for (int64_t sp = 1; sp <= std::min<int64_t>(P, std::max<int64_t>(1, nkb / 4)); ++sp) {
+                const double cost = (double)ceil_div(tiles * sp, num_sms) * ((double)ceil_div(nkb, sp) + E);
+                if (cost < best - 1e-9) { best = cost; sbest = sp; }
+            }
+            A.kb_per_split = (int)ceil_div(nkb, sbest);
+            sbest = ceil_div(nkb, A.kb_per_split);
+            A.cl = 0; A.zsplit = 0; A.atomic = 0; A.stg_bytes = 0;
+            grid2((int)sbest);
+            float* part = (float*)(ws + WL.b_off);
+            A.out = part; A.alpha = 1.f; A.beta = 0.f; A.part_rows = g.k;  // slot = K x R*S*C (ldc = R*S*C)
+            const int e = launch();
+            if (e) return e;
+            note_fused();
+            return DRY(launch_partial_reduce((int)sbest, (int64_t)g.k * RSC, (int)RSC, g.k, (int)RSC, false, part,
+                                             alpha, beta, (float*)out, st, mc_reduce));
+        };
+        if (algo == MUCU_ALGO_IM2COL_GEMM && i2c_implicit_wgrad(g)) {
+            // I2C with the im2col done by the TMA unit (im2col mode) into shared memory, as
+            // the implicit GEMM does; the workspace holds the split partials
+            const bool part_ok = ctx->deterministic && wgrad_partial_slots(g) > 1;
+            if (use_tma_im2col()) {
+                wgrad_tiling(atom, true);
+                if (!map_dy()) return -1;
+                if (make_im2col_map(&L.tb, elt, in0, g.c, g.w, g.h, b, -g.pad, -g.pad, g.pad - (g.s - 1),
+                                    g.pad - (g.r - 1), KB * A.km, g.stride, true)) {
+                    A.tma_bytes = A.km * (A.mt * a_bytes + A.bn_atoms * KB * 128);
+                    if (part_ok && A.cl)
+                        return launch_partial([&]() { return LAUNCH(A_TMA_MN2, B_TMA_IM2COL, EPI_WGRAD_PARTIAL); });
+                    return LAUNCH(A_TMA_MN2, B_TMA_IM2COL, EPI_WGRAD_CHAIN);
+                }
+            }
+            A.tma_bytes = a_bytes;
+            wgrad_tiling(atom, false);
+            if (!map_dy()) return -1;
+            if (part_ok && A.cl)
+                return launch_partial([&]() { return LAUNCH(A_TMA_MN2, B_GATHER_WG, EPI_WGRAD_PARTIAL); });
+            return LAUNCH(A_TMA_MN2, B_GATHER_WG, EPI_WGRAD_CHAIN);
+        }
         if (algo == MUCU_ALGO_IM2COL_GEMM) {
             const void* colp = in0;
             int64_t kp = g.c;
@@ -1563,32 +1611,8 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
             if (!map2(&L.tb, colp, RSC, (uint64_t)Mpix, kp, atom, KB * A.km, true)) return -1;
             map_mn_box(colp, RSC, (uint64_t)Mpix, kp, KB * A.km);
             A.tma_bytes = A.km * (A.mt * a_bytes + A.bn_atoms * KB * 128);
-            const int P = wgrad_partial_slots(g);
-            if (ctx->deterministic && P > 1 && A.cl) {
-                // workspace partials: persistent CTAs over all SMs, split s writes its dW
-                // tile to slot s, a reduction kernel sums the slots in order (no cluster
-                // packing loss, no ordered hand-over)
-                const int64_t tiles = ceil_div(A.N, A.BN) * ceil_div(A.M, 128 * A.mt);
-                const int64_t nkb = A.num_kb;
-                const double E = env_int("MUCU_SPLIT_E", 16) / (double)A.km;
-                int64_t sbest = 1;
-                double best = 1e30;
-                for (int64_t sp = 1; sp <= std::min<int64_t>(P, std::max<int64_t>(1, nkb / 4)); ++sp) {
-                    const double cost = (double)ceil_div(tiles * sp, num_sms) * ((double)ceil_div(nkb, sp) + E);
-                    if (cost < best - 1e-9) { best = cost; sbest = sp; }
-                }
-                A.kb_per_split = (int)ceil_div(nkb, sbest);
-                sbest = ceil_div(nkb, A.kb_per_split);
-                A.cl = 0; A.zsplit = 0; A.atomic = 0; A.stg_bytes = 0;
-                grid2((int)sbest);
-                float* part = (float*)(ws + WL.b_off);
-                A.out = part; A.alpha = 1.f; A.beta = 0.f; A.part_rows = g.k;  // slot = K x R*S*C (ldc = R*S*C)
-                err = LAUNCH(A_TMA_MN2, B_TMA_MN2, EPI_WGRAD_PARTIAL);
-                if (err) return err;
-                note_fused();
-                return DRY(launch_partial_reduce((int)sbest, (int64_t)g.k * RSC, (int)RSC, g.k, (int)RSC, false, part,
-                                                 alpha, beta, (float*)out, st, mc_reduce));
-            }
+            if (ctx->deterministic && wgrad_partial_slots(g) > 1 && A.cl)
+                return launch_partial([&]() { return LAUNCH(A_TMA_MN2, B_TMA_MN2, EPI_WGRAD_PARTIAL); });
             return LAUNCH(A_TMA_MN2, B_TMA_MN2, EPI_WGRAD_CHAIN);
         }
         // implicit-im2col B producers load whole 128-B channel atoms of one tap:

@@ -36,6 +36,10 @@ inline int64_t ceil_div(int64_t a, int64_t b) { return (a + b - 1) / b; }
 bool algo_eligible(const Geom& g, int type, int algo);
 bool is_pointwise(const Geom& g);  // 1x1, stride 1, pad 0: im2col(x) == x
 bool small_c_tc(const Geom& g);    // tensor-core math and C*elt < 16 B (RGB input layer)
+// Tensor-core I2C BackwardFilter whose im2col is done by the TMA unit into shared memory
+// (C a multiple of the 128-B atom, not 1x1): the workspace holds only the per-split
+// partial dW slots.
+bool i2c_implicit_wgrad(const Geom& g);
 // Strided small-C layers whose I2C algorithm runs on the space-to-depth image:
 // a stride-1 ceil(R/st) x ceil(S/st) conv over st*st*C channels (padded to
 // s2d_channels = a multiple of 128 B).  DGRAD (no padding: the super-pixel

@@ -61,6 +61,11 @@ bool i2c_implicit_wgrad(const Geom& g) {
     return g.math != MUCU_MATH_F32 && !is_pointwise(g) && g.c % (128 / elt_size(g.math)) == 0;
 }
 
+int wgrad_implicit_slots(const Geom& g) {
+    const int64_t tiles = ceil_div(g.k, 256) * ceil_div((int64_t)g.r * g.s * g.c, 128);
+    return (int)std::max<int64_t>(1, std::min<int64_t>(kPartialSlots, ceil_div(kPartialSlots, tiles)));
+}
+
 int s2d_channels(const Geom& g) {
     const int atom = 128 / elt_size(g.math);
     return (int)align_up((uint64_t)g.stride * g.stride * g.c, (uint64_t)atom);
@@ -214,8 +219,10 @@ mucu_status_t ws_layout(const Geom& g, int type, int algo, int32_t b, WsLayout* 
         }
         if (type == MUCU_BWD_FILTER && i2c_implicit_wgrad(g)) {
             // TMA im2col into shared memory: only the per-split partial dW slots
+            const int Pi = wgrad_implicit_slots(g);
             L->a_off = 0; L->a_bytes = 0;
-            L->b_off = 0; L->b_bytes = part; L->total = part;
+            L->b_off = 0; L->b_bytes = Pi > 1 ? align_up((uint64_t)Pi * g.k * RSC * 4, 256) : 0;
+            L->total = L->b_bytes;
             return MUCU_OK;
         }
         StagedWg sw;

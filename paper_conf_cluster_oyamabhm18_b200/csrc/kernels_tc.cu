@@ -1550,8 +1550,7 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         // Workspace partials: persistent CTAs over all SMs, split s writes its dW tile to
         // slot s, a reduction kernel sums the slots in order (no cluster packing loss, no
         // ordered hand-over).  `launch_partial(launch)` runs the GEMM launcher given.
-        auto launch_partial = [&](auto launch) -> int {
-            const int P = wgrad_partial_slots(g);
+        auto launch_partial = [&](const int P, auto launch) -> int {
             const int64_t tiles = ceil_div(A.N, A.BN) * ceil_div(A.M, 128 * A.mt);
             const int64_t nkb = A.num_kb;
             const double E = env_int("MUCU_SPLIT_E", 16) / (double)A.km;
@@ -1576,7 +1575,8 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
         if (algo == MUCU_ALGO_IM2COL_GEMM && i2c_implicit_wgrad(g)) {
             // I2C with the im2col done by the TMA unit (im2col mode) into shared memory, as
             // the implicit GEMM does; the workspace holds the split partials
-            const bool part_ok = ctx->deterministic && wgrad_partial_slots(g) > 1;
+            const int Pi = wgrad_implicit_slots(g);
+            const bool part_ok = ctx->deterministic && Pi > 1;
             if (use_tma_im2col()) {
                 wgrad_tiling(atom, true);
                 if (!map_dy()) return -1;
@@ -1584,7 +1584,7 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
                                     g.pad - (g.r - 1), KB * A.km, g.stride, true)) {
                     A.tma_bytes = A.km * (A.mt * a_bytes + A.bn_atoms * KB * 128);
                     if (part_ok && A.cl)
-                        return launch_partial([&]() { return LAUNCH(A_TMA_MN2, B_TMA_IM2COL, EPI_WGRAD_PARTIAL); });
+                        return launch_partial(Pi, [&]() { return LAUNCH(A_TMA_MN2, B_TMA_IM2COL, EPI_WGRAD_PARTIAL); });
                     return LAUNCH(A_TMA_MN2, B_TMA_IM2COL, EPI_WGRAD_CHAIN);
                 }
             }
@@ -1592,7 +1592,7 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
             wgrad_tiling(atom, false);
             if (!map_dy()) return -1;
             if (part_ok && A.cl)
-                return launch_partial([&]() { return LAUNCH(A_TMA_MN2, B_GATHER_WG, EPI_WGRAD_PARTIAL); });
+                return launch_partial(Pi, [&]() { return LAUNCH(A_TMA_MN2, B_GATHER_WG, EPI_WGRAD_PARTIAL); });
             return LAUNCH(A_TMA_MN2, B_GATHER_WG, EPI_WGRAD_CHAIN);
         }
         if (algo == MUCU_ALGO_IM2COL_GEMM) {
@@ -1612,7 +1612,8 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
             map_mn_box(colp, RSC, (uint64_t)Mpix, kp, KB * A.km);
             A.tma_bytes = A.km * (A.mt * a_bytes + A.bn_atoms * KB * 128);
             if (ctx->deterministic && wgrad_partial_slots(g) > 1 && A.cl)
-                return launch_partial([&]() { return LAUNCH(A_TMA_MN2, B_TMA_MN2, EPI_WGRAD_PARTIAL); });
+                return launch_partial(wgrad_partial_slots(g),
+                                      [&]() { return LAUNCH(A_TMA_MN2, B_TMA_MN2, EPI_WGRAD_PARTIAL); });
             return LAUNCH(A_TMA_MN2, B_TMA_MN2, EPI_WGRAD_CHAIN);
         }
         // implicit-im2col B producers load whole 128-B channel atoms of one tap:

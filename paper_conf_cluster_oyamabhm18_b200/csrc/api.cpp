@@ -62,7 +62,7 @@ bool i2c_implicit_wgrad(const Geom& g) {
 }
 
 int wgrad_implicit_slots(const Geom& g) {
-    const int64_t tiles = ceil_div(g.k, 256) * ceil_div((int64_t)g.r * g.s * g.c, 128);
+    const int64_t tiles = ceil_div(g.k, 256) * ceil_div((int64_t)g.r * g.s * g.c, 256);
     return (int)std::max<int64_t>(1, std::min<int64_t>(kPartialSlots, ceil_div(kPartialSlots, tiles)));
 }
 

@@ -40,7 +40,7 @@ bool small_c_tc(const Geom& g);    // tensor-core math and C*elt < 16 B (RGB inp
 // (C a multiple of the 128-B atom, not 1x1): the workspace holds only the per-split
 // partial dW slots.
 bool i2c_implicit_wgrad(const Geom& g);
-// Its partial slots: enough splits to fill every SM with 256 x 128 dW tiles.
+// Its partial slots: enough splits to fill every SM with the largest (256 x 256) dW tiles.
 int wgrad_implicit_slots(const Geom& g);
 // Strided small-C layers whose I2C algorithm runs on the space-to-depth image:
 // a stride-1 ceil(R/st) x ceil(S/st) conv over st*st*C channels (padded to

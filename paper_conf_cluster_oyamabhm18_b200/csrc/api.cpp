@@ -296,7 +296,8 @@ mucu_status_t ws_layout(const Geom& g, int type, int algo, int32_t b, WsLayout* 
     }
     if (algo == MUCU_ALGO_FFT || algo == MUCU_ALGO_FFT_TILING) {
         // spectra (complex fp32): filter [bins][K][C] | input tiles | output tiles
-        // (WGRAD: x tiles | dy tiles | dW spectrum).  DESIGN.md 6.11.
+        // (WGRAD: dW spectrum | x tiles | dy tiles -- the spectrum first, at an offset
+        // independent of b, so consecutive micro-batches accumulate into it).  DESIGN.md 6.11.
         FftGeom z;
         fft_geom(g, type, algo, &z);
         const uint64_t B = (uint64_t)z.bins, Pl = (uint64_t)b * z.tiles_y * z.tiles_x;
@@ -304,12 +305,13 @@ mucu_status_t ws_layout(const Geom& g, int type, int algo, int32_t b, WsLayout* 
         const uint64_t in_ch = type == MUCU_FWD ? g.c : (uint64_t)g.k;   // x (FWD, WGRAD a) / dy (DGRAD)
         const uint64_t out_ch = type == MUCU_FWD ? g.k : (uint64_t)g.c;
         if (type == MUCU_BWD_FILTER) {
-            L->a_off = 0;
+            L->fixed_off = 0;  // dW spectrum (accumulated over a run of micro-batches)
+            L->fixed_bytes = KC;
+            L->a_off = KC;
             L->a_bytes = align_up(8 * B * Pl * g.c, 256);
-            L->b_off = L->a_bytes;
+            L->b_off = L->a_off + L->a_bytes;
             L->b_bytes = align_up(8 * B * Pl * g.k, 256);
-            L->fixed_off = L->b_off + L->b_bytes;  // dW spectrum (per call)
-            L->total = L->fixed_off + KC;
+            L->total = L->b_off + L->b_bytes;
             return MUCU_OK;
         }
         L->fixed_off = 0;
@@ -665,6 +667,7 @@ static mucu_status_t execute(mucu_handle_t h, const mucu_conv_desc_t* d, int typ
         float bta;
         part_ptrs(i, done, p0, p1, po, bta);
         ctx.mc_last = i == count - 1;
+        ctx.next_algo = i + 1 < count ? plan[i + 1].algo : -1;
         s = run_micro(h, g, type, plan[i].algo, b, alpha, p0, p1, bta, po, ws, ws_bytes, st, &ctx);
         if (s) return s;
         done += b;

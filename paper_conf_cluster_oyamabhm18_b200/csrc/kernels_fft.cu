@@ -257,7 +257,7 @@ __device__ __forceinline__ int crow(int ty, int i) {
 template <int BM, bool KA, bool KB, bool CJA, bool CJB>
 __global__ void __launch_bounds__(256, 2) cgemm_kernel(const float2* __restrict__ A, const float2* __restrict__ B,
                                                     float2* __restrict__ Cm, int M, int N, int K, int lda, int ldb,
-                                                    int ldc, int64_t sA, int64_t sB, int64_t sC) {
+                                                    int ldc, int64_t sA, int64_t sB, int64_t sC, int accum) {
     // deeper k stages for the short tiles: more bytes in flight when few planes make
     // the per-bin filter spectrum read the bound (BM * BK + 64 * BK complex per stage)
     constexpr int BN = 64, BK = BM == 16 ? 32 : BM == 32 ? 16 : 8, PAD = 4, TM = BM / 16;
@@ -363,22 +363,26 @@ __global__ void __launch_bounds__(256, 2) cgemm_kernel(const float2* __restrict_
 #pragma unroll
         for (int j = 0; j < 4; ++j) {
             const int nn = n0 + (j < 2 ? tx * 2 + j : 32 + tx * 2 + j - 2);
-            if (nn < N) Cm[(int64_t)mm * ldc + nn] = acc[i][j];
+            if (nn < N) {
+                float2* d = Cm + (int64_t)mm * ldc + nn;
+                if (accum) { const float2 o = *d; *d = make_float2(o.x + acc[i][j].x, o.y + acc[i][j].y); }
+                else *d = acc[i][j];
+            }
         }
     }
 }
 
 template <bool KA, bool KB, bool CJA, bool CJB>
 int cgemm(const float2* A, const float2* B, float2* C, int M, int N, int K, int lda, int ldb, int ldc, int64_t sA,
-          int64_t sB, int64_t sC, int64_t batch, cudaStream_t st) {
+          int64_t sB, int64_t sC, int64_t batch, cudaStream_t st, int accum = 0) {
     const int bm = M <= 16 ? 16 : M <= 32 ? 32 : 64;
     dim3 grid((unsigned)ceil_div(M, bm), (unsigned)ceil_div(N, 64), (unsigned)batch);
     if (bm == 16)
-        cgemm_kernel<16, KA, KB, CJA, CJB><<<grid, 256, 0, st>>>(A, B, C, M, N, K, lda, ldb, ldc, sA, sB, sC);
+        cgemm_kernel<16, KA, KB, CJA, CJB><<<grid, 256, 0, st>>>(A, B, C, M, N, K, lda, ldb, ldc, sA, sB, sC, accum);
     else if (bm == 32)
-        cgemm_kernel<32, KA, KB, CJA, CJB><<<grid, 256, 0, st>>>(A, B, C, M, N, K, lda, ldb, ldc, sA, sB, sC);
+        cgemm_kernel<32, KA, KB, CJA, CJB><<<grid, 256, 0, st>>>(A, B, C, M, N, K, lda, ldb, ldc, sA, sB, sC, accum);
     else
-        cgemm_kernel<64, KA, KB, CJA, CJB><<<grid, 256, 0, st>>>(A, B, C, M, N, K, lda, ldb, ldc, sA, sB, sC);
+        cgemm_kernel<64, KA, KB, CJA, CJB><<<grid, 256, 0, st>>>(A, B, C, M, N, K, lda, ldb, ldc, sA, sB, sC, accum);
     count_launch();
     return (int)cudaGetLastError();
 }
@@ -477,15 +481,23 @@ int fft_run(const Geom& g, int type, int algo, int32_t b, float alpha, const flo
                                                      (int64_t)g.k * g.c, planes * g.c, bins, st);
         if (!e) e = fft_inverse(F, Sb, tile_map(z, g.h, g.w, g.c, g.r - 1, g.s - 1, 0, 0, planes), scale, beta, out, st);
     } else {
-        // X tiles as FWD; DY zero outside its own tile; DW[bin][k][c] = sum_planes conj(DY) X
+        // X tiles as FWD; DY zero outside its own tile; DW[bin][k][c] = sum_planes conj(DY) X.
+        // Consecutive micro-batches of this algorithm accumulate DW in the frequency domain
+        // (the transform is linear: sum_mb IFFT(S_mb) = IFFT(sum_mb S_mb)) and the inverse
+        // runs once, at the last of them, with the first one's beta (P:L58 output scale).
         float2* DW = (float2*)(ws + L.fixed_off);
+        const bool first = ctx->fixed_kind != 6;
+        if (first) { ctx->fixed_kind = 6; ctx->fixed_src = nullptr; ctx->fft_beta = beta; }
         e = fft_forward(F, in0, tile_map(z, g.h, g.w, g.c, -g.pad, -g.pad, F, F, planes), Sa, st);
         if (!e) e = fft_forward(F, in1, tile_map(z, g.p, g.q, g.k, 0, 0, z.Th, z.Tw, planes), Sb, st);
         if (!e) e = cgemm<false, false, true, false>(Sb, Sa, DW, g.k, g.c, (int)planes, g.k, g.c, g.c, planes * g.k,
-                                                     planes * g.c, (int64_t)g.k * g.c, bins, st);
+                                                     planes * g.c, (int64_t)g.k * g.c, bins, st, first ? 0 : 1);
         // dw[k][r][s][c]: K "images" of R x S, window at the origin
         TileMap om{g.r, g.s, g.c, 1, 1, g.r, g.s, 0, 0, 0, 0, g.k};
-        if (!e) e = fft_inverse(F, DW, om, scale, beta, out, st);
+        if (!e && ctx->next_algo != algo) {
+            e = fft_inverse(F, DW, om, scale, ctx->fft_beta, out, st);
+            ctx->fixed_kind = 0;
+        }
     }
     return e;
 }

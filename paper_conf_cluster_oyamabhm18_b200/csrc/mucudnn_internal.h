@@ -108,9 +108,12 @@ struct RedTarget {
 
 // Per-call executor state (which b-independent workspace prefix is valid).
 struct CallCtx {
-    int fixed_kind = 0;  // 0 none, 1 padded filter, 2 Winograd U, 3/4 space-to-depth filter, 5 FFT filter spectrum
+    int fixed_kind = 0;  // 0 none, 1 padded filter, 2 Winograd U, 3/4 space-to-depth filter, 5 FFT filter spectrum,
+                         // 6 FFT BackwardFilter spectrum accumulating over consecutive micro-configs
     const void* fixed_src = nullptr;
     int last_algo = -1;  // algorithm of the previous micro-config (prefix invalidation)
+    int next_algo = -1;  // algorithm of the next micro-config of the call (-1: this is the last)
+    float fft_beta = 0.f;  // FFT BackwardFilter: beta of the first micro-config of a run (kind 6)
     bool dry = false;    // tensor-core dispatch decisions only, no launch (pre-validation)
     bool deterministic = true;  // BackwardFilter split-K: ordered reduction (default) or L2 atomics
     // NEXT-3: the cross-rank dW sum target (red.n = 0: off), used by the

@@ -118,6 +118,28 @@ def test_fft_wgrad_accumulates_over_micro_batches(name):
     assert normwise_err(got, ref) <= TOL
 
 
+@pytest.mark.parametrize("name", ["5x5_alexnet_conv2", "3x3_multi_tile"])
+def test_fft_wgrad_spectrum_runs(name):
+    """Consecutive FFT / FFT_TILING BackwardFilter micro-batches accumulate dW in the
+    frequency domain and transform it back once per run: runs of
+    different lengths and micro-batch sizes, broken by other algorithms, with
+    alpha / beta (the run's first micro-batch carries the user's beta)."""
+    shape = list(SHAPES[name])
+    shape[0] = 6
+    shape = tuple(shape)
+    d = mu.desc(*shape, mu.MATH_F32)
+    x, w, dy = _inputs(shape, seed=13)
+    algo = mu.FFT if _eligible(shape, mu.BWD_FILTER, mu.FFT) else mu.FFT_TILING
+    out0 = np.random.default_rng(5).standard_normal(oracle_ref(shape, mu.BWD_FILTER, x, None, dy).shape)
+    ref = oracle_ref(shape, mu.BWD_FILTER, x, None, dy, alpha=1.5, beta=-0.5, out0=out0)
+    for plan in ([(algo, 3), (algo, 2), (algo, 1)],
+                 [(algo, 2), (mu.IMPLICIT_GEMM, 1), (algo, 1), (algo, 2)],
+                 [(mu.IMPLICIT_GEMM, 1), (algo, 4), (mu.FFT_TILING, 1)],
+                 [(algo, 1)] * 6):
+        got, _ = run_gpu(d, mu.BWD_FILTER, plan, x, w, dy, alpha=1.5, beta=-0.5, out0=out0.astype(np.float32))
+        assert normwise_err(got, ref) <= TOL, plan
+
+
 @pytest.mark.parametrize("conv_type", [mu.FWD, mu.BWD_DATA, mu.BWD_FILTER], ids=["fwd", "dgrad", "wgrad"])
 def test_fft_alpha_beta_mixed_plan(conv_type):
     """out = alpha*op + beta*out with FFT, FFT_TILING, Winograd and IG micro-batches."""

@@ -141,6 +141,12 @@ mucu_status_t mucu_output_dims(const mucu_conv_desc_t* desc, int32_t* p, int32_t
  *                     0 for 1x1, stride 1, pad 0 (the im2col matrix is x itself)
  *                     b*H*W*16 for TF32/BF16 with C*elt < 16 (RGB input layer): x with
  *                     channels zero-padded to 16 B, gathered tap by tap on chip
+ *                     TF32/BF16 WGRAD adds Ps partial dW slots of K*R*S*C*4 bytes (deterministic
+ *                     split-K summed in split order; 0 when Ps = 1):
+ *                       Ps = min(148, ceil(148 / (ceil(K/128) * ceil(R*S*C/128))));
+ *                     and when C is a multiple of 128/elt (not 1x1) the im2col is done by TMA
+ *                     into shared memory: only the slots, with
+ *                       Ps = min(148, ceil(148 / (ceil(K/256) * ceil(R*S*C/256))))
  *   I2C DGRAD:        b*P*Q*ceil_4(R*S*C)*4 (fp32 dcol)  (+ filter copy as above, or with rows of
  *                     128 B when R*S*C < 128/elt on tensor cores); 0 for 1x1/s1/p0
  *   I2C, TF32/BF16, stride st > 1 and C*elt < 16 ("space-to-depth"):
@@ -172,7 +178,7 @@ mucu_status_t mucu_output_dims(const mucu_conv_desc_t* desc, int32_t* p, int32_t
  *                     ty x tx = ceil(Eh/Th) x ceil(Ew/Tw):
  *                     FWD:   8*B*K*C + 8*B*Pl*C + 8*B*Pl*K
  *                     DGRAD: 8*B*K*C + 8*B*Pl*K + 8*B*Pl*C
- *                     WGRAD: 8*B*Pl*C + 8*B*Pl*K + 8*B*K*C
+ *                     WGRAD: 8*B*K*C (the dW spectrum, first) + 8*B*Pl*C + 8*B*Pl*K
  * ceil_e rounds up to a multiple of 16/elt elements.  UNSUPPORTED if the
  * algorithm is ineligible (WG needs R=S=3, stride 1, pad <= 2; FFT / FFT_TILING
  * need MUCU_MATH_F32 and stride 1). */

@@ -149,6 +149,21 @@ def test_workspace_space_to_depth():
     assert mu.workspace_size(d, mu.FWD, mu.IM2COL_GEMM, 2) == 2 * 32 * 32 * 16
 
 
+def test_workspace_i2c_wgrad_slots():
+    """I2C BackwardFilter of atom-aligned layers: im2col by TMA in shared memory, the
+    workspace is only the partial dW slots (include/mucudnn.h closed form)."""
+    d = mu.desc(256, 64, 27, 27, 192, 5, 5, 2, 1, mu.MATH_TF32)       # AlexNet conv2
+    ps = -(-148 // (1 * -(-1600 // 256)))                              # 148 / (1 * 7) -> 22
+    for b in (1, 64, 256):                                             # b-independent
+        assert mu.workspace_size(d, mu.BWD_FILTER, mu.IM2COL_GEMM, b) == ps * 192 * 1600 * 4
+    d = mu.desc(256, 512, 7, 7, 512, 3, 3, 1, 1, mu.MATH_BF16)        # ResNet layer4 3x3
+    ps = -(-148 // (2 * 18))                                           # -> 5
+    assert mu.workspace_size(d, mu.BWD_FILTER, mu.IM2COL_GEMM, 32) == ps * 512 * 4608 * 4
+    # F32 keeps the explicit im2col matrix (SIMT path), no slots
+    d = mu.desc(8, 64, 27, 27, 192, 5, 5, 2, 1, mu.MATH_F32)
+    assert mu.workspace_size(d, mu.BWD_FILTER, mu.IM2COL_GEMM, 1) == 729 * 1600 * 4
+
+
 # NEXT-3 entry points: argument validation happens on the host before any device work.
 def _reduce_call(target):
     d = mu.desc(2, 8, 6, 6, 8, 3, 3, 1, 1, mu.MATH_F32)

@@ -75,6 +75,7 @@ def parse():
                     help="cross-rank dW sum: async NCCL allreduce per layer, or fused into the BackwardFilter "
                          "epilogue (NEXT-3): multimem.red to an NVLink multicast buffer (nvls) or red.global.add "
                          "to every rank's buffer over NVLink P2P (p2p); both also run at one GPU")
+    ap.add_argument("--oracle-probe", type=int, default=0, help=argparse.SUPPRESS)  # internal: time N oracle images
     ap.add_argument("--json-out", default="")
     ap.add_argument("--tables-in", default="", help="benchmark DB (.npz) to plan from instead of benchmarking")
     ap.add_argument("--tables-out", default="", help="write the benchmark DB (.npz) after the benchmark pass")
@@ -198,15 +199,32 @@ def oracle_sample_time(layers, kernels, n_sample, threads=None):
     return tot
 
 
+def single_thread_ms(batch):
+    """The oracle on ONE host thread: one image of every kernel of the
+    step in a child process with OMP_NUM_THREADS=1, scaled to N = batch."""
+    import subprocess
+    cmd = [sys.executable, os.path.abspath(__file__), "--oracle-probe", "1"] + \
+        [a for a in sys.argv[1:] if not a.startswith("--json-out")]
+    try:
+        r = subprocess.run(cmd, env=dict(os.environ, OMP_NUM_THREADS="1"), capture_output=True, text=True,
+                           timeout=600)
+        secs = float(r.stdout.strip().splitlines()[-1])
+    except Exception:  # noqa: BLE001 -- a reported extra, never fatal
+        return None
+    return round(secs * 1e3 * batch, 3)
+
+
 def cpu_baseline(layers, kernels, batch, n_sample):
     cores = os.cpu_count()
     secs = oracle_sample_time(layers, kernels, n_sample)
     ms_per_iter = secs * 1e3 * batch / n_sample
     exact = n_sample == batch
     return {"value": round(ms_per_iter, 3), "unit": "ms/iter", "cores": cores, "kind": "oracle",
+            "single_thread_value": single_thread_ms(batch),
             "sample": f"{n_sample} image(s) per kernel, all {len(kernels)} timed kernels, fp64 7-loop oracle "
                       f"(OpenMP, {cores} threads), {secs:.2f} s measured"
-                      + ("" if exact else f", x{batch // n_sample} extrapolated to N={batch} (work is linear in N, P:L50)")}
+                      + ("" if exact else f", x{batch // n_sample} extrapolated to N={batch} (work is linear in N, P:L50)")
+                      + "; single_thread_value: 1 image per kernel on one thread, scaled"}
 
 
 def auto_sample(layers, kernels, batch):
@@ -296,6 +314,10 @@ class _NoReduce:
 
 def main():
     args = parse()
+    if args.oracle_probe:
+        layers, types, kernels = select(args)
+        print(oracle_sample_time(layers, kernels, args.oracle_probe), flush=True)
+        return
     if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
         sys.exit(respawn(args))
     if args.impl == "reference":

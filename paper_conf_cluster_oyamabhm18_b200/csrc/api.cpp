@@ -61,12 +61,6 @@ bool i2c_implicit_wgrad(const Geom& g) {
     return g.math != MUCU_MATH_F32 && !is_pointwise(g) && g.c % (128 / elt_size(g.math)) == 0;
 }
 
-bool wg_kmajor() {
-    static int v = -1;
-    if (v < 0) { const char* e = getenv("MUCU_WG_KMAJOR"); v = (e && e[0] == '1') ? 1 : 0; }
-    return v == 1;
-}
-
 int wgrad_implicit_slots(const Geom& g) {
     const int64_t tiles = ceil_div(g.k, 256) * ceil_div((int64_t)g.r * g.s * g.c, 256);
     return (int)std::max<int64_t>(1, std::min<int64_t>(kPartialSlots, ceil_div(kPartialSlots, tiles)));
@@ -229,11 +223,6 @@ mucu_status_t ws_layout(const Geom& g, int type, int algo, int32_t b, WsLayout* 
             L->a_off = 0; L->a_bytes = 0;
             L->b_off = 0; L->b_bytes = Pi > 1 ? align_up((uint64_t)Pi * g.k * RSC * 4, 256) : 0;
             L->total = L->b_bytes;
-            if (wg_kmajor()) {  // experimental: dy^T [K][b*P*Q rounded up to 32]
-                L->a_off = L->b_bytes;
-                L->a_bytes = align_up((uint64_t)g.k * align_up((uint64_t)b * PQ, 32) * elt, 256);
-                L->total = L->a_off + L->a_bytes;
-            }
             return MUCU_OK;
         }
         StagedWg sw;

@@ -1105,38 +1105,6 @@ int launch_partial_reduce_win(int S, int64_t slot, int M, int K, int per_atom, i
     return (int)cudaGetLastError();
 }
 
-// out[c][r] = in[r][c] for an R x C matrix (row pitch C) into rows of pitch ldo; columns
-// r in [R, ldo) are zero-filled.  32 x 32 tiles through shared memory (coalesced both ways).
-template <class T>
-__global__ void transpose_kernel(const T* __restrict__ in, T* __restrict__ out, int64_t R, int C, int64_t ldo) {
-    pdl_entry();
-    __shared__ T tile[32][33];
-    const int64_t r0 = (int64_t)blockIdx.x * 32;
-    const int c0 = blockIdx.y * 32;
-    for (int i = threadIdx.y; i < 32; i += 8) {
-        const int64_t r = r0 + i;
-        const int c = c0 + threadIdx.x;
-        tile[i][threadIdx.x] = (r < R && c < C) ? in[r * C + c] : T(0.f);
-    }
-    __syncthreads();
-    for (int i = threadIdx.y; i < 32; i += 8) {
-        const int c = c0 + i;
-        const int64_t r = r0 + threadIdx.x;
-        if (c < C && r < ldo) out[(int64_t)c * ldo + r] = tile[threadIdx.x][i];
-    }
-}
-
-int launch_transpose(const void* in, void* out, int64_t R, int C, int64_t ldo, int elt, cudaStream_t st) {
-    const dim3 grid((unsigned)((ldo + 31) / 32), (unsigned)((C + 31) / 32)), block(32, 8);
-    if (elt == 2)
-        launch_pdl(transpose_kernel<__nv_bfloat16>, grid, block, (size_t)0, st, (const __nv_bfloat16*)in,
-                   (__nv_bfloat16*)out, R, C, ldo);
-    else
-        launch_pdl(transpose_kernel<float>, grid, block, (size_t)0, st, (const float*)in, (float*)out, R, C, ldo);
-    count_launch();
-    return (int)cudaGetLastError();
-}
-
 int launch_wgw_output(const Geom& g, float alpha, const float* M, float beta, float* dw, cudaStream_t st) {
     const int at = 128 / elt_size(g.math);
     const int Cp = (int)align_up((uint64_t)g.c, (uint64_t)at), Kp = (int)align_up((uint64_t)g.k, (uint64_t)at);

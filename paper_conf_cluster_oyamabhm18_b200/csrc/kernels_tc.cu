@@ -1577,23 +1577,6 @@ int tc_run_micro(const Geom& g, int type, int algo, int32_t b, float alpha, cons
             // the implicit GEMM does; the workspace holds the split partials
             const int Pi = wgrad_implicit_slots(g);
             const bool part_ok = ctx->deterministic && Pi > 1;
-            if (wg_kmajor() && use_tma_im2col() && part_ok) {
-                // experimental: dy transposed into the workspace -> K-major A operand
-                // (rows = K filters, K-dim = pixels), one k-block per stage
-                const int64_t ldt = (int64_t)align_up((uint64_t)Mpix, 32);
-                char* dyt = ws + WL.a_off;
-                err = DRY(launch_transpose(in1, dyt, Mpix, g.k, ldt, elt, st));
-                if (err) return err;
-                wgrad_tiling(atom, true, 0, 1);
-                A.m64 = 0;
-                if (!map2(&L.ta, dyt, (uint64_t)ldt, g.k, (uint64_t)ldt, KB, 128)) return -1;
-                if (make_im2col_map(&L.tb, elt, in0, g.c, g.w, g.h, b, -g.pad, -g.pad, g.pad - (g.s - 1),
-                                    g.pad - (g.r - 1), KB, g.stride, true) && A.km == 1 && A.cl) {
-                    A.tma_bytes = A.mt * 16384 + A.bn_atoms * KB * 128;
-                    return launch_partial(Pi, [&]() { return LAUNCH(A_TMA_K2, B_TMA_IM2COL, EPI_WGRAD_PARTIAL); });
-                }
-                return -1;
-            }
             if (use_tma_im2col()) {
                 wgrad_tiling(atom, true);
                 if (!map_dy()) return -1;

@@ -274,11 +274,6 @@ int launch_wgw_output(const Geom& g, float alpha, const float* M, float beta, fl
 // red (NEXT-3): the final values are also added to the cross-rank dW sum (n = 0: off).
 int launch_partial_reduce(int S, int64_t slot, int ldp, int M, int N, bool transpose, const float* part,
                           float alpha, float beta, float* out, cudaStream_t st, const RedTarget* red = nullptr);
-// out[c][r] = in[r][c] (R x C, row pitch C) into rows of pitch ldo >= R (tail zeroed).
-int launch_transpose(const void* in, void* out, int64_t R, int C, int64_t ldo, int elt, cudaStream_t st);
-// Experimental (MUCU_WG_KMAJOR=1): I2C BackwardFilter with dy transposed to a K-major
-// A operand in the workspace (after the partial slots).
-bool wg_kmajor();
 // The same for the window BackwardFilter's partial tiles (rows = window rows, DESIGN.md
 // 6.5; padding rows skipped), out = dw [K][R][S][C].
 int launch_partial_reduce_win(int S, int64_t slot, int M, int K, int per_atom, int cp, int na, const Geom& g,
